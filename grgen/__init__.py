@@ -1,0 +1,156 @@
+"""Seeded synthetic graph inputs shared by the CUDA path and the oracle.
+
+This module holds none of the GAS method's arithmetic: it only
+produces canonical COO edge lists from counter-based random draws, shaped like
+the paper's benchmark graphs (Table 1) as SURVEY.md §8(d)
+specifies for BASELINE.json configs 1-5.
+"""
+from __future__ import annotations
+
+import ctypes
+import os
+import subprocess
+
+import numpy as np
+
+_HERE = os.path.dirname(os.path.abspath(__file__))
+_SO = os.path.join(_HERE, "libgrgen.so")
+_SRC = os.path.join(_HERE, "grgen.c")
+_lib = None
+
+THREADS = max(1, min(32, os.cpu_count() or 1))
+
+
+def build(force: bool = False) -> str:
+    """Compile libgrgen.so (plain C, OpenMP) if missing or stale."""
+    if force or not os.path.exists(_SO) or os.path.getmtime(_SO) < max(
+        os.path.getmtime(_SRC), os.path.getmtime(os.path.join(_HERE, "grgen.h"))
+    ):
+        tmp = _SO + f".tmp{os.getpid()}"
+        subprocess.check_call(
+            ["gcc", "-O3", "-fopenmp", "-fPIC", "-shared", "-o", tmp, _SRC, "-lm"], cwd=_HERE
+        )
+        os.replace(tmp, _SO)
+    return _SO
+
+
+def lib():
+    global _lib
+    if _lib is None:
+        build()
+        L = ctypes.CDLL(_SO)
+        u32p = ctypes.POINTER(ctypes.c_uint32)
+        L.grgen_hash.restype = ctypes.c_uint64
+        L.grgen_hash.argtypes = [ctypes.c_uint64] * 3
+        L.grgen_rmat.restype = ctypes.c_int
+        L.grgen_rmat.argtypes = [ctypes.c_uint32, ctypes.c_uint64, ctypes.c_double, ctypes.c_double,
+                                 ctypes.c_double, ctypes.c_uint64, u32p, u32p, ctypes.c_int]
+        L.grgen_weights.restype = ctypes.c_int
+        L.grgen_weights.argtypes = [ctypes.c_uint64, ctypes.c_uint32, ctypes.c_uint32, ctypes.c_uint64,
+                                    u32p, ctypes.c_int]
+        L.grgen_grid.restype = ctypes.c_int64
+        L.grgen_grid.argtypes = [ctypes.c_uint32, ctypes.c_uint32, ctypes.c_double, ctypes.c_uint32,
+                                 ctypes.c_uint64, u32p, u32p, u32p, ctypes.c_uint64]
+        L.grgen_web.restype = ctypes.c_int64
+        L.grgen_web.argtypes = [ctypes.c_uint64, ctypes.c_double, ctypes.c_double, ctypes.c_uint32,
+                                ctypes.c_double, ctypes.c_double, ctypes.c_uint32, ctypes.c_double,
+                                ctypes.c_uint64, u32p, u32p, ctypes.c_uint64, ctypes.c_int]
+        _lib = L
+    return _lib
+
+
+def _p(a: np.ndarray):
+    return a.ctypes.data_as(ctypes.POINTER(ctypes.c_uint32))
+
+
+class Graph(dict):
+    """dict with keys n, src, dst, [w], name — attribute access for convenience."""
+
+    __getattr__ = dict.__getitem__
+
+    @property
+    def m(self) -> int:
+        return int(self["src"].shape[0])
+
+
+def rmat(scale: int, edgefactor: int = 16, seed: int = 1, a: float = 0.57, b: float = 0.19,
+         c: float = 0.19, m: int | None = None) -> Graph:
+    """R-MAT (Graph500 kron parameters), no noise, no permutation (vertex 0 is the hub)."""
+    m = int(edgefactor) << scale if m is None else int(m)
+    src = np.empty(m, np.uint32)
+    dst = np.empty(m, np.uint32)
+    rc = lib().grgen_rmat(scale, m, a, b, c, seed, _p(src), _p(dst), THREADS)
+    if rc != 0:
+        raise ValueError(f"grgen_rmat rc={rc}")
+    return Graph(n=1 << scale, src=src, dst=dst, name=f"rmat{scale}_ef{edgefactor}_s{seed}")
+
+
+def weights(m: int, lo: int = 1, hi: int = 64, seed: int = 1) -> np.ndarray:
+    w = np.empty(m, np.uint32)
+    rc = lib().grgen_weights(m, lo, hi, seed, _p(w), THREADS)
+    if rc != 0:
+        raise ValueError(f"grgen_weights rc={rc}")
+    return w
+
+
+def grid_road(W: int, H: int, p: float = 0.58, wmax: int = 64, seed: int = 3) -> Graph:
+    """Road-like lattice: p-kept lattice edges + seeded connectivity repair, symmetric weights."""
+    L = lib()
+    m = L.grgen_grid(W, H, p, wmax, seed, None, None, None, 0)
+    if m < 0:
+        raise ValueError(f"grgen_grid rc={m}")
+    src = np.empty(m, np.uint32)
+    dst = np.empty(m, np.uint32)
+    w = np.empty(m, np.uint32)
+    m2 = L.grgen_grid(W, H, p, wmax, seed, _p(src), _p(dst), _p(w), m)
+    if m2 != m:
+        raise ValueError(f"grgen_grid rc={m2}")
+    return Graph(n=W * H, src=src, dst=dst, w=w, name=f"grid{W}x{H}_s{seed}")
+
+
+WEB_DEFAULTS = dict(xmin=2.8, zexp=2.5, dmax=1 << 20, p_local=0.75, geo_p=1.0 / 64,
+                    local_cap=4096, rank_exp=0.8)
+
+
+def web(n: int, seed: int = 4, **kw) -> Graph:
+    """Web-like power law (uk-2002 shape), symmetrized, self-loops dropped."""
+    prm = dict(WEB_DEFAULTS)
+    prm.update(kw)
+    args = (n, prm["xmin"], prm["zexp"], prm["dmax"], prm["p_local"], prm["geo_p"],
+            prm["local_cap"], prm["rank_exp"], seed)
+    L = lib()
+    m = L.grgen_web(*args, None, None, 0, THREADS)
+    if m < 0:
+        raise ValueError(f"grgen_web rc={m}")
+    src = np.empty(m, np.uint32)
+    dst = np.empty(m, np.uint32)
+    m2 = L.grgen_web(*args, _p(src), _p(dst), m, THREADS)
+    if m2 != m:
+        raise ValueError(f"grgen_web rc={m2}")
+    return Graph(n=n, src=src, dst=dst, name=f"web{n}_s{seed}")
+
+
+# --------------------------------------------------------------------------
+# BASELINE.json configs; `reduced` gives the parity-test
+# sizes with the same shape.
+# --------------------------------------------------------------------------
+def config(i: int, reduced: bool = False) -> tuple[Graph, dict]:
+    """Return (graph, run) for BASELINE.json configs[i-1]."""
+    if i == 1:
+        g = rmat(12 if reduced else 16, edgefactor=38, seed=1)
+        return g, dict(algo="bfs", source=0)
+    if i == 2:
+        g = rmat(16 if reduced else 22, edgefactor=16, seed=2)
+        return g, dict(algo="pagerank", max_iters=30, damping=0.85)
+    if i == 3:
+        W = 300 if reduced else 4894
+        g = grid_road(W, W, p=0.58, wmax=64, seed=3)
+        return g, dict(algo="sssp", source=0)
+    if i == 4:
+        g = web(200_000 if reduced else 18_520_486, seed=4)
+        return g, dict(algo="cc")
+    if i == 5:
+        # cfg5 shape (R-MAT ef16); scale chosen by the caller's memory budget
+        g = rmat(18 if reduced else 31, edgefactor=16, seed=5)
+        return g, dict(algo="pagerank", max_iters=30, damping=0.85)
+    raise ValueError(i)

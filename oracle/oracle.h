@@ -1,0 +1,37 @@
+/* oracle.h — TEST INFRASTRUCTURE ONLY. A plain, slow, single-threaded CPU GAS
+ * engine written from the paper (§2.1, §4.4, §5.2
+ * L270, §5.3, Fig. 6). Only tests/, __graft_entry__.smoke()
+ * and bench.py's cpu_baseline / --impl reference legs may load it. It shares
+ * no code or headers with the CUDA path (paper_conf_sc_senguptasas15_b200/). */
+#ifndef GR_ORACLE_H
+#define GR_ORACLE_H
+#include <stdint.h>
+#ifdef __cplusplus
+extern "C" {
+#endif
+
+enum { OR_BFS = 0, OR_SSSP = 1, OR_PAGERANK = 2, OR_CC = 3 };
+#define OR_INF 0xFFFFFFFFu
+
+typedef struct or_graph or_graph;
+
+/* Build the oracle's own CSC (in-edges sorted by (dst, src, w)) and CSR
+ * (out-edges sorted by (src, dst, w)) from a COO list. w may be NULL.
+ * Returns NULL on bad input (id >= n) or allocation failure. */
+or_graph *or_graph_build(uint64_t n, uint64_t m, const uint32_t *src, const uint32_t *dst,
+                         const uint32_t *w);
+void or_graph_free(or_graph *g);
+
+/* Run one program to termination (or max_iters supersteps; 0 = unlimited).
+ * values_out: uint32_t[n] for BFS/SSSP/CC, double[n] for PAGERANK.
+ * trace_out (nullable): rows of 4 uint64 per superstep t:
+ *   |A_t|, |C_t|, sum_{v in A_t} indeg(v) (0 when gather is eliminated),
+ *   sum_{u in C_t} outdeg(u) (0 when FrontierActivate is eliminated).
+ * Returns the number of supersteps executed, or <0 on error. */
+int64_t or_run(or_graph *g, int algo, uint32_t source, uint32_t max_iters, double damping,
+               void *values_out, uint64_t *trace_out, uint64_t trace_cap, uint64_t *rows_out);
+
+#ifdef __cplusplus
+}
+#endif
+#endif

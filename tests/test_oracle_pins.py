@@ -1,0 +1,417 @@
+"""Pins for the oracle (SURVEY.md §8(c) "Pins").
+
+Each check compares the oracle with something other than itself: textbook
+algorithms from scipy / networkx, closed forms, a dense linear solve, and a
+pure-Python set-based brute force of the BSP frontier semantics on tiny
+graphs. A plausible mistake in the oracle (dropped term, wrong sign or index,
+transposed operand, off-by-one iteration, non-BSP update) fails at least one.
+"""
+from __future__ import annotations
+
+import collections
+import heapq
+import os
+
+import networkx as nx
+import numpy as np
+import pytest
+import scipy.sparse as sp
+import scipy.sparse.csgraph as csg
+
+import oracle
+from oracle import INF
+
+GOLDEN = os.path.join(os.path.dirname(__file__), "golden")
+
+
+# ----------------------------------------------------------------- helpers
+def rand_graph(rng, n, m, sym=False, wmax=None):
+    src = rng.integers(0, n, m).astype(np.uint32)
+    dst = rng.integers(0, n, m).astype(np.uint32)
+    w = rng.integers(1, wmax + 1, m).astype(np.uint32) if wmax else None
+    if sym:
+        src, dst = np.concatenate([src, dst]), np.concatenate([dst, src])
+        if w is not None:
+            w = np.concatenate([w, w])
+    return src, dst, w
+
+
+def queue_bfs(n, src, dst, s):
+    adj = collections.defaultdict(list)
+    for a, b in zip(src.tolist(), dst.tolist()):
+        adj[a].append(b)
+    d = [INF] * n
+    d[s] = 0
+    q = collections.deque([s])
+    while q:
+        u = q.popleft()
+        for x in adj[u]:
+            if d[x] == INF:
+                d[x] = d[u] + 1
+                q.append(x)
+    return np.array(d, np.uint32)
+
+
+def heap_dijkstra(n, src, dst, w, s):
+    adj = collections.defaultdict(list)
+    for a, b, c in zip(src.tolist(), dst.tolist(), w.tolist()):
+        adj[a].append((b, c))
+    d = [INF] * n
+    d[s] = 0
+    h = [(0, s)]
+    while h:
+        du, u = heapq.heappop(h)
+        if du > d[u]:
+            continue
+        for x, c in adj[u]:
+            if du + c < d[x]:
+                d[x] = du + c
+                heapq.heappush(h, (d[x], x))
+    return np.array(d, np.uint32)
+
+
+def union_find_min_label(n, src, dst):
+    p = list(range(n))
+
+    def f(x):
+        while p[x] != x:
+            p[x] = p[p[x]]
+            x = p[x]
+        return x
+
+    for a, b in zip(src.tolist(), dst.tolist()):
+        ra, rb = f(a), f(b)
+        if ra != rb:
+            p[max(ra, rb)] = min(ra, rb)
+    mn = {}
+    for v in range(n):
+        r = f(v)
+        mn[r] = min(mn.get(r, v), v)
+    return np.array([mn[f(v)] for v in range(n)], np.uint32)
+
+
+def dense_pagerank_fixed_point(n, src, dst, d=0.85):
+    """R* = (1-d)/n (I - d M^T)^-1 1 with M[u,v] = mult(u->v)/outdeg(u); dangling dropped."""
+    M = np.zeros((n, n))
+    for a, b in zip(src.tolist(), dst.tolist()):
+        M[a, b] += 1.0
+    out = M.sum(1)
+    nz = out > 0
+    M[nz] /= out[nz, None]
+    return np.linalg.solve(np.eye(n) - d * M.T, np.full(n, (1 - d) / n))
+
+
+def brute_trace(n, src, dst, w, algo, source=0, max_iters=0, d=0.85):
+    """Pure-Python set-based BSP GAS."""
+    ins = collections.defaultdict(list)
+    outs = collections.defaultdict(list)
+    for i, (a, b) in enumerate(zip(src.tolist(), dst.tolist())):
+        c = int(w[i]) if w is not None else 1
+        ins[b].append((a, c))
+        outs[a].append(b)
+    if algo == "pagerank":
+        val = {v: 1.0 / n for v in range(n)}
+        A = set(range(n))
+    elif algo == "cc":
+        val = {v: v for v in range(n)}
+        A = set(range(n))
+    else:
+        val = {v: INF for v in range(n)}
+        if algo == "bfs":
+            A = {source}
+        else:
+            val[source] = 0
+            A = set(outs[source])
+    rows, t = [], 0
+    while A and (max_iters == 0 or t < max_iters):
+        new = {}
+        gathered = 0
+        for v in A:
+            if algo == "bfs":
+                new[v] = t if val[v] == INF else val[v]
+                continue
+            gathered += len(ins[v])
+            if algo == "pagerank":
+                acc = sum(val[u] / len(outs[u]) for u, _ in ins[v])
+                new[v] = (1 - d) / n + d * acc
+            elif algo == "cc":
+                acc = min([val[u] for u, _ in ins[v]], default=INF)
+                new[v] = min(acc, val[v])
+            else:
+                acc = min([min(val[u] + c, INF) if val[u] != INF else INF for u, c in ins[v]],
+                          default=INF)
+                new[v] = min(acc, val[v])
+        C = set(A) if algo == "pagerank" else {v for v in A if new[v] != val[v]}
+        val.update(new)
+        if algo == "pagerank":
+            rows.append((len(A), len(C), gathered, 0))
+            A = set(range(n))
+        else:
+            rows.append((len(A), len(C), gathered, sum(len(outs[u]) for u in C)))
+            A = {x for u in C for x in outs[u]}
+        t += 1
+    return val, np.array(rows, np.uint64).reshape(-1, 4), t
+
+
+# ------------------------------------------------------------------- BFS
+@pytest.mark.parametrize("seed", range(12))
+def test_bfs_vs_queue_bfs_and_scipy(seed):
+    rng = np.random.default_rng(seed)
+    n = int(rng.integers(2, 80))
+    src, dst, _ = rand_graph(rng, n, int(rng.integers(0, 4 * n)))
+    s = int(rng.integers(0, n))
+    vals, tr, it = oracle.run(n, src, dst, "bfs", source=s)
+    np.testing.assert_array_equal(vals, queue_bfs(n, src, dst, s))
+    A = sp.csr_matrix((np.ones(len(src)), (src, dst)), shape=(n, n))
+    ref = csg.shortest_path(A, directed=True, unweighted=True, indices=s)
+    ref = np.where(np.isinf(ref), INF, ref).astype(np.uint32)
+    np.testing.assert_array_equal(vals, ref)
+
+
+def test_bfs_lattice_closed_form():
+    W, H = 13, 9
+    e = []
+    for r in range(H):
+        for c in range(W):
+            v = r * W + c
+            if c + 1 < W:
+                e += [(v, v + 1), (v + 1, v)]
+            if r + 1 < H:
+                e += [(v, v + W), (v + W, v)]
+    src, dst = np.array(e, np.uint32).T
+    vals, _, _ = oracle.run(W * H, src, dst, "bfs", source=0)
+    rr, cc = np.divmod(np.arange(W * H), W)
+    np.testing.assert_array_equal(vals, (rr + cc).astype(np.uint32))
+
+
+def test_bfs_directed_cycle_trace_closed_form():
+    n = 17
+    src = np.arange(n, dtype=np.uint32)
+    dst = ((src + 1) % n).astype(np.uint32)
+    vals, tr, it = oracle.run(n, src, dst, "bfs", source=0)
+    np.testing.assert_array_equal(vals, np.arange(n, dtype=np.uint32))
+    # t < n: one vertex active and changed, one out-edge activated; t = n: vertex 0 re-activated, unchanged
+    exp = [(1, 1, 0, 1)] * n + [(1, 0, 0, 0)]
+    np.testing.assert_array_equal(tr, np.array(exp, np.uint64))
+    assert it == n + 1
+
+
+def test_bfs_vs_networkx_rmat():
+    import grgen
+
+    g = grgen.rmat(10, 8, seed=11)
+    vals, _, _ = oracle.run(g.n, g.src, g.dst, "bfs", source=0)
+    G = nx.DiGraph()
+    G.add_nodes_from(range(g.n))
+    G.add_edges_from(zip(g.src.tolist(), g.dst.tolist()))
+    ref = np.full(g.n, INF, np.uint32)
+    for v, dd in nx.single_source_shortest_path_length(G, 0).items():
+        ref[v] = dd
+    np.testing.assert_array_equal(vals, ref)
+
+
+# ------------------------------------------------------------------ SSSP
+@pytest.mark.parametrize("seed", range(12))
+def test_sssp_vs_dijkstra_and_scipy(seed):
+    rng = np.random.default_rng(100 + seed)
+    n = int(rng.integers(2, 70))
+    src, dst, w = rand_graph(rng, n, int(rng.integers(0, 4 * n)), wmax=64)
+    s = int(rng.integers(0, n))
+    vals, _, _ = oracle.run(n, src, dst, "sssp", w=w, source=s)
+    np.testing.assert_array_equal(vals, heap_dijkstra(n, src, dst, w, s))
+    # scipy sums duplicate entries: reduce multi-edges to their minimum weight first
+    best = {}
+    for a, b, c in zip(src.tolist(), dst.tolist(), w.tolist()):
+        if a != b:
+            best[(a, b)] = min(best.get((a, b), c), c)
+    if best:
+        (ij, cw) = zip(*best.items())
+        ii, jj = zip(*ij)
+        A = sp.csr_matrix((np.array(cw, float), (ii, jj)), shape=(n, n))
+    else:
+        A = sp.csr_matrix((n, n))
+    ref = csg.dijkstra(A, directed=True, indices=s)
+    ref = np.where(np.isinf(ref), INF, ref).astype(np.uint32)
+    np.testing.assert_array_equal(vals, ref)
+
+
+def test_sssp_unit_weights_equals_bfs():
+    # "BFS is essentially SSSP with equal edge weights"
+    import grgen
+
+    g = grgen.rmat(11, 8, seed=5)
+    w = np.ones(g.m, np.uint32)
+    b, _, _ = oracle.run(g.n, g.src, g.dst, "bfs", source=3)
+    s, _, _ = oracle.run(g.n, g.src, g.dst, "sssp", w=w, source=3)
+    np.testing.assert_array_equal(b, s)
+
+
+def test_sssp_path_prefix_sums_and_lattice_manhattan():
+    rng = np.random.default_rng(7)
+    n = 40
+    w = rng.integers(1, 65, n - 1).astype(np.uint32)
+    src = np.arange(n - 1, dtype=np.uint32)
+    dst = src + 1
+    vals, tr, it = oracle.run(n, src, dst, "sssp", w=w, source=0)
+    np.testing.assert_array_equal(vals, np.concatenate([[0], np.cumsum(w)]).astype(np.uint32))
+    # path: exactly one vertex active and changed per superstep; A_0 = {1}
+    assert it == n - 1
+    np.testing.assert_array_equal(tr[:, :2], np.ones((n - 1, 2), np.uint64))
+    import grgen
+
+    g = grgen.grid_road(9, 7, p=1.0, wmax=1, seed=1)  # full lattice, unit weights
+    vals, _, _ = oracle.run(g.n, g.src, g.dst, "sssp", w=g.w, source=0)
+    rr, cc = np.divmod(np.arange(g.n), 9)
+    np.testing.assert_array_equal(vals, (rr + cc).astype(np.uint32))
+
+
+# -------------------------------------------------------------------- CC
+@pytest.mark.parametrize("seed", range(12))
+def test_cc_vs_union_find_and_scipy(seed):
+    rng = np.random.default_rng(200 + seed)
+    n = int(rng.integers(1, 90))
+    src, dst, _ = rand_graph(rng, n, int(rng.integers(0, 2 * n)), sym=True)
+    vals, _, _ = oracle.run(n, src, dst, "cc")
+    np.testing.assert_array_equal(vals, union_find_min_label(n, src, dst))
+    A = sp.csr_matrix((np.ones(len(src)), (src, dst)), shape=(n, n))
+    k, lab = csg.connected_components(A, directed=False)
+    assert len(np.unique(vals)) == k
+    for c in range(k):
+        members = np.nonzero(lab == c)[0]
+        assert np.all(vals[members] == members.min())
+
+
+def test_cc_disjoint_cycles_and_cliques():
+    edges, expect, base = [], [], 0
+    for kind, size in [("cycle", 5), ("clique", 4), ("cycle", 9), ("clique", 1), ("clique", 6)]:
+        vs = list(range(base, base + size))
+        if kind == "cycle" and size > 1:
+            for i in range(size):
+                a, b = vs[i], vs[(i + 1) % size]
+                edges += [(a, b), (b, a)]
+        else:
+            for a in vs:
+                for b in vs:
+                    if a != b:
+                        edges.append((a, b))
+        expect += [base] * size
+        base += size
+    # relabel by a permutation so the min id is not always the first vertex
+    perm = np.random.default_rng(3).permutation(base).astype(np.uint32)
+    src, dst = (perm[np.array(edges, np.int64).T] if edges else np.zeros((2, 0), np.uint32))
+    vals, _, _ = oracle.run(base, src, dst, "cc")
+    exp = np.empty(base, np.uint32)
+    blocks = np.array(expect)
+    for b in np.unique(blocks):
+        members = perm[blocks == b]
+        exp[members] = members.min()
+    np.testing.assert_array_equal(vals, exp)
+
+
+# -------------------------------------------------------------------- PR
+def test_pr_directed_cycle_uniform():
+    n = 23
+    src = np.arange(n, dtype=np.uint32)
+    dst = ((src + 1) % n).astype(np.uint32)
+    for iters in (1, 2, 30):
+        vals, tr, it = oracle.run(n, src, dst, "pagerank", max_iters=iters)
+        assert it == iters
+        np.testing.assert_allclose(vals, 1.0 / n, rtol=0, atol=1e-15)
+    np.testing.assert_array_equal(tr, np.tile(np.array([n, n, n, 0], np.uint64), (30, 1)))
+
+
+def test_pr_symmetric_star_closed_form():
+    k, d = 3, 0.85
+    n = k + 1
+    src = np.array([0] * k + list(range(1, n)), np.uint32)
+    dst = np.array(list(range(1, n)) + [0] * k, np.uint32)
+    vals, _, _ = oracle.run(n, src, dst, "pagerank", max_iters=200)
+    leaf = (1 + d / k) / (n * (1 + d))
+    hub = (1 - d) / n + d * k * leaf
+    np.testing.assert_allclose(vals[1:], leaf, atol=1e-13)
+    np.testing.assert_allclose(vals[0], hub, atol=1e-13)
+    np.testing.assert_allclose([leaf, hub], [0.1734234234, 0.4797297297], atol=1e-10)
+
+
+def test_pr_golden_example_dense_solve():
+    # tests/golden/pr_example.txt: edges {0->1,0->2,1->2,2->0,2->3}, vertex 3 dangling
+    path = os.path.join(GOLDEN, "pr_example.txt")
+    rows = [ln.split() for ln in open(path) if ln.strip() and not ln.startswith("#")]
+    edges = [(int(r[1]), int(r[2])) for r in rows if r[0] == "e"]
+    golden = np.array([float(r[2]) for r in rows if r[0] == "r"])
+    src, dst = np.array(edges, np.uint32).T
+    vals, _, _ = oracle.run(4, src, dst, "pagerank", max_iters=200)
+    np.testing.assert_allclose(vals, golden, atol=1e-8)
+    np.testing.assert_allclose(vals, dense_pagerank_fixed_point(4, src, dst), atol=1e-12)
+    v30, _, _ = oracle.run(4, src, dst, "pagerank", max_iters=30)
+    np.testing.assert_allclose(v30, golden, atol=2e-6)
+
+
+@pytest.mark.parametrize("seed", range(10))
+def test_pr_fixed_point_dense_solve(seed):
+    rng = np.random.default_rng(300 + seed)
+    n = int(rng.integers(4, 9))
+    src, dst, _ = rand_graph(rng, n, int(rng.integers(n, 4 * n)))
+    vals, _, _ = oracle.run(n, src, dst, "pagerank", max_iters=200)
+    np.testing.assert_allclose(vals, dense_pagerank_fixed_point(n, src, dst), atol=1e-12)
+
+
+@pytest.mark.parametrize("seed", range(6))
+def test_pr_30_iterations_matrix_power(seed):
+    rng = np.random.default_rng(400 + seed)
+    n = int(rng.integers(4, 30))
+    src, dst, _ = rand_graph(rng, n, 3 * n)
+    M = np.zeros((n, n))
+    np.add.at(M, (src, dst), 1.0)
+    out = M.sum(1)
+    M[out > 0] /= out[out > 0, None]
+    R = np.full(n, 1.0 / n)
+    for _ in range(30):
+        R = 0.15 / n + 0.85 * (M.T @ R)
+    vals, _, _ = oracle.run(n, src, dst, "pagerank", max_iters=30)
+    np.testing.assert_allclose(vals, R, atol=1e-15, rtol=1e-12)
+
+
+@pytest.mark.parametrize("seed", range(5))
+def test_pr_networkx_no_dangling(seed):
+    rng = np.random.default_rng(500 + seed)
+    n = 25
+    src, dst, _ = rand_graph(rng, n, 4 * n)
+    # give every vertex an out-edge (no dangling) — networkx then agrees exactly
+    src = np.concatenate([src, np.arange(n, dtype=np.uint32)])
+    dst = np.concatenate([dst, rng.integers(0, n, n).astype(np.uint32)])
+    vals, _, _ = oracle.run(n, src, dst, "pagerank", max_iters=200)
+    G = nx.MultiDiGraph()
+    G.add_nodes_from(range(n))
+    G.add_edges_from(zip(src.tolist(), dst.tolist()))
+    ref = nx.pagerank(G, alpha=0.85, tol=1e-15, max_iter=1000)
+    np.testing.assert_allclose(vals, [ref[v] for v in range(n)], atol=1e-12)
+    # invariant: no dangling vertex => sum_v R_t = 1 at every t
+    for iters in (1, 2, 7, 30):
+        v, _, _ = oracle.run(n, src, dst, "pagerank", max_iters=iters)
+        assert abs(v.sum() - 1.0) < 1e-12
+
+
+# -------------------------------------------------- frontier-trace pins
+@pytest.mark.parametrize("algo", ["bfs", "sssp", "cc", "pagerank"])
+@pytest.mark.parametrize("seed", range(8))
+def test_trace_vs_bruteforce(algo, seed):
+    rng = np.random.default_rng(600 + seed)
+    n = int(rng.integers(2, 40))
+    src, dst, w = rand_graph(rng, n, int(rng.integers(0, 3 * n)), sym=(algo == "cc"), wmax=64)
+    s = int(rng.integers(0, n))
+    mi = 7 if algo == "pagerank" else 0
+    vals, tr, it = oracle.run(n, src, dst, algo, w=w if algo == "sssp" else None, source=s,
+                              max_iters=mi)
+    bv, btr, bit = brute_trace(n, src, dst, w if algo == "sssp" else None, algo, s, mi)
+    assert it == bit
+    np.testing.assert_array_equal(tr, btr)
+    if algo == "pagerank":
+        np.testing.assert_allclose(vals, [bv[v] for v in range(n)], atol=1e-15, rtol=1e-13)
+    else:
+        np.testing.assert_array_equal(vals, np.array([bv[v] for v in range(n)], np.uint32))
+
+
+def test_oracle_rejects_bad_input():
+    with pytest.raises(ValueError):
+        oracle.OracleGraph(4, np.array([0, 5], np.uint32), np.array([1, 2], np.uint32))
