@@ -1,0 +1,290 @@
+#!/usr/bin/env python
+"""bench.py — GraphReduce-on-B200 benchmark (driver contract).
+
+Default workload (BASELINE.json configs[1]): PageRank, 30 iterations, d = 0.85,
+fp32, on a synthetic R-MAT scale-22 edgefactor-16 graph (4,194,304 vertices,
+67,108,864 edges), resident in HBM. One step = one gr_run (30 BSP supersteps).
+Metric: GTEPS = 30 * m / (seconds per run).
+
+  python bench.py [--gpus N] [--steps K] [--warmup W] [--impl reference] [--config 1..4]
+"""
+from __future__ import annotations
+
+import argparse
+import json
+import os
+import subprocess
+import sys
+import threading
+import time
+
+ROOT = os.path.dirname(os.path.abspath(__file__))
+sys.path.insert(0, ROOT)
+
+import numpy as np  # noqa: E402
+
+CONFIG_NAMES = {
+    1: "cfg1: BFS from 0, R-MAT s16 ef38 (kron_g500-logn16 shape), 1 GPU resident",
+    2: "cfg2: PageRank x30 d=0.85 fp32, R-MAT s22 ef16 (4,194,304 V / 67,108,864 E), resident",
+    3: "cfg3: SSSP from 0, road-like grid 4894x4894 weights 1-64, resident",
+    4: "cfg4: CC, web-like power law n=18,520,486 (uk-2002 shape), symmetrized, resident",
+}
+
+
+def peaks():
+    p = os.path.join(ROOT, "MEASURED_PEAKS.json")
+    if os.path.exists(p):
+        d = json.load(open(p))
+        return float(d["hbm_gbs"]), "measured (MEASURED_PEAKS.json hbm_gbs)"
+    return 6650.0, "fallback (B200_PROFILING.md 6.65 TB/s)"
+
+
+class ClockSampler:
+    """nvidia-smi clocks + throttle reasons sampled DURING the timed region."""
+
+    Q = ("index,clocks.sm,clocks.max.sm,power.draw,clocks_event_reasons.active,"
+         "clocks_event_reasons.hw_slowdown,clocks_event_reasons.hw_thermal_slowdown,"
+         "clocks_event_reasons.sw_thermal_slowdown,clocks_event_reasons.sw_power_cap")
+
+    def __init__(self, device=0):
+        self.device = device
+        self.proc = None
+        self.lines = []
+
+    def start(self):
+        try:
+            self.proc = subprocess.Popen(
+                ["nvidia-smi", "-i", str(self.device), f"--query-gpu={self.Q}", "--format=csv,noheader,nounits",
+                 "-lms", "100"], stdout=subprocess.PIPE, stderr=subprocess.DEVNULL, text=True)
+            self.t = threading.Thread(target=self._read, daemon=True)
+            self.t.start()
+        except Exception:
+            self.proc = None
+
+    def _read(self):
+        for ln in self.proc.stdout:
+            self.lines.append(ln.strip())
+
+    def stop(self):
+        if not self.proc:
+            return {"sm_mhz": None, "sm_max_mhz": None, "reasons": ["nvidia-smi unavailable"]}
+        self.proc.terminate()
+        try:
+            self.proc.wait(timeout=5)
+        except Exception:
+            self.proc.kill()
+        sm, mx, reasons = [], None, set()
+        names = ["hw_slowdown", "hw_thermal_slowdown", "sw_thermal_slowdown", "sw_power_cap"]
+        for ln in self.lines:
+            f = [x.strip() for x in ln.split(",")]
+            if len(f) < 9:
+                continue
+            try:
+                sm.append(float(f[1]))
+                mx = float(f[2])
+            except ValueError:
+                continue
+            for nm, v in zip(names, f[5:9]):
+                if v.lower().startswith("active"):
+                    reasons.add(nm)
+        return {"sm_mhz": float(np.median(sm)) if sm else None, "sm_max_mhz": mx, "reasons": sorted(reasons),
+                "samples": len(sm)}
+
+
+def make_graph(cfg: int):
+    import grgen
+
+    g, run = grgen.config(cfg)
+    w = g.get("w")
+    if run["algo"] == "sssp" and w is None:
+        w = grgen.weights(g.m, 1, 64, seed=cfg)
+    return g, w, run
+
+
+def metric_edges(cfg_run, stats, m):
+    """GTEPS numerator (DESIGN.md §7 / SURVEY reading R15)."""
+    a = cfg_run["algo"]
+    if a == "pagerank":
+        return cfg_run.get("max_iters", 30) * m
+    if a == "cc":
+        return m
+    return stats["edges_scattered"] + stats["edges_gathered"]  # BFS/SSSP: edges traversed
+
+
+def cpu_oracle_sample(g, w, run, budget_s=20.0):
+    """Time the oracle as it stands on a bounded sample of the workload."""
+    import oracle
+
+    og = oracle.OracleGraph(g.n, g.src, g.dst, w)
+    try:
+        if run["algo"] == "pagerank":
+            iters = 2
+            t = time.perf_counter()
+            og.run("pagerank", max_iters=iters)
+            dt = time.perf_counter() - t
+            return dict(value=iters * g.m / dt / 1e9, unit="GTEPS", cores=1, kind="oracle",
+                        sample=f"PageRank {iters} of 30 supersteps on the full graph (m={g.m}); "
+                               f"oracle CSC build not timed; {dt:.2f} s")
+        t = time.perf_counter()
+        vals, tr, it = og.run(run["algo"], source=run.get("source", 0))
+        dt = time.perf_counter() - t
+        edges = int(tr[:, 2].sum() + tr[:, 3].sum()) if run["algo"] != "cc" else g.m
+        return dict(value=edges / dt / 1e9, unit="GTEPS", cores=1, kind="oracle",
+                    sample=f"full {run['algo']} run ({it} supersteps); {dt:.2f} s")
+    finally:
+        og.close()
+
+
+def load_traffic(kernel):
+    p = os.path.join(ROOT, "profiles", "traffic.json")
+    if os.path.exists(p):
+        d = json.load(open(p))
+        return d.get(kernel)
+    return None
+
+
+def main():
+    ap = argparse.ArgumentParser()
+    ap.add_argument("--gpus", type=int, default=1)
+    ap.add_argument("--steps", type=int, default=5)
+    ap.add_argument("--warmup", type=int, default=3)
+    ap.add_argument("--impl", default="ours", choices=["ours", "reference"])
+    ap.add_argument("--config", type=int, default=2)
+    ap.add_argument("--e2e-steps", type=int, default=2)
+    ap.add_argument("--no-cpu", action="store_true")
+    args = ap.parse_args()
+
+    rank = int(os.environ.get("RANK", "0"))
+    world = int(os.environ.get("WORLD_SIZE", "1"))
+    local_rank = int(os.environ.get("LOCAL_RANK", "0"))
+
+    if args.impl == "reference":
+        if rank != 0:
+            return 0
+        g, w, run = make_graph(args.config)
+        per_step = []
+        for i in range(args.warmup + args.steps):
+            cb = cpu_oracle_sample(g, w, run)
+            if i >= args.warmup:
+                per_step.append(cb["value"])
+        val = float(np.median(per_step))
+        cb["value"] = val
+        line = {"impl": "reference", "metric": "GTEPS", "value": val, "unit": "GTEPS", "n_gpus": args.gpus,
+                "steps": args.steps, "warmup": args.warmup, "higher_is_better": True, "scaling": "strong",
+                "vs_baseline": None, "dtype": "f64", "data": "synthetic",
+                "config": {"workload": CONFIG_NAMES[args.config], "impl": "single-threaded CPU oracle"},
+                "cpu_baseline": cb, "e2e": {"value": val, "unit": "GTEPS", "h2d_bytes_per_step": 0,
+                                            "d2h_bytes_per_step": 0}}
+        print(json.dumps(line), flush=True)
+        return 0
+
+    import torch
+
+    if world > 1:
+        import torch.distributed as dist
+
+        dist.init_process_group("nccl" if torch.cuda.is_available() else "gloo")
+    torch.cuda.set_device(local_rank)
+    import paper_conf_sc_senguptasas15_b200 as gr
+
+    g, w, run = make_graph(args.config)
+    algo = run["algo"]
+    kw = dict(source=run.get("source", 0), max_iters=run.get("max_iters", 0), damping=run.get("damping", 0.85))
+    G = gr.GraphReduce(g.n, g.src, g.dst, w, device=local_rank, mode="resident")
+    info = G.info()
+    stream = torch.cuda.current_stream()
+    sp = stream.cuda_stream
+    for _ in range(max(3, args.warmup)):
+        G.run(algo, stream=sp, **kw)
+    if world > 1:
+        torch.distributed.barrier()
+    torch.cuda.synchronize()
+    clocks = ClockSampler(local_rank)
+    clocks.start()
+    e0, e1 = torch.cuda.Event(enable_timing=True), torch.cuda.Event(enable_timing=True)
+    kms, launches, stats = 0.0, 0, None
+    e0.record(stream)
+    for _ in range(args.steps):
+        stats = G.run(algo, stream=sp, profile=True, **kw)
+        kms += stats["kernel_ms"][0] if algo != "bfs" else stats["kernel_ms"][1]
+        launches += stats["kernel_launches"]
+    e1.record(stream)
+    torch.cuda.synchronize()
+    ck = clocks.stop()
+    ms = e0.elapsed_time(e1)
+    if world > 1:
+        t = torch.tensor([ms], device="cuda")
+        torch.distributed.all_reduce(t, op=torch.distributed.ReduceOp.MAX)
+        ms = float(t.item())
+        torch.distributed.barrier()
+    ms_step = ms / args.steps
+    edges = metric_edges(run, stats, g.m)
+    value = edges * world / (ms_step * 1e-3) / 1e9
+
+    # roofline of the dominant kernel (algorithmic bytes per launch / CUDA-event duration)
+    peak, peak_src = peaks()
+    n, m = g.n, g.m
+    if algo == "pagerank":
+        launches_per_step = run.get("max_iters", 30)
+        bytes_per_launch = 4 * m + 16 * n
+        kname = "k_pr_gather_apply"
+    else:
+        launches_per_step = max(1, stats["iterations"])
+        bytes_per_launch = stats["bytes_hbm_model"] / launches_per_step
+        kname = "k_gather_apply" if algo != "bfs" else "k_bfs_expand"
+    avg_launch_s = (kms / args.steps) * 1e-3 / launches_per_step
+    achieved = bytes_per_launch / avg_launch_s / 1e9
+    roof = {"bound": "hbm", "kernel": kname, "achieved": round(achieved, 1), "peak": peak, "unit": "GB/s",
+            "frac": round(achieved / peak, 4), "peak_source": peak_src,
+            "bytes_per_launch": int(bytes_per_launch), "avg_launch_us": round(avg_launch_s * 1e6, 2),
+            "kernel_share_of_step": round(kms / ms, 4) if ms > 0 else None,
+            "traffic": load_traffic(kname)}
+    run_roof = {"bytes_hbm_model_per_step": stats["bytes_hbm_model"],
+                "frac_of_step": round(stats["bytes_hbm_model"] / (ms_step * 1e-3) / 1e9 / peak, 4)}
+
+    # end to end through the public C ABI with host buffers (load + run + fetch)
+    e2e_vals, h2d = [], 0
+    src_p = torch.from_numpy(g.src).pin_memory().numpy()
+    dst_p = torch.from_numpy(g.dst).pin_memory().numpy()
+    w_p = torch.from_numpy(w).pin_memory().numpy() if w is not None else None
+    out = torch.empty(n, dtype=torch.float32 if algo == "pagerank" else torch.int32).pin_memory().numpy()
+    for i in range(args.e2e_steps):
+        t0 = time.perf_counter()
+        H = gr.gr_graph_load(n, src_p, dst_p, w_p, device=local_rank, mode="resident")
+        gr.gr_run(H, algo, **kw)
+        gr.gr_fetch_vertex_values(H, out)
+        dt = time.perf_counter() - t0
+        inf = gr.gr_graph_info_get(H)
+        gr.gr_graph_free(H)
+        e2e_vals.append(edges * world / dt / 1e9)
+    h2d = int(8 * m + (m if w is not None else 0))  # CSC + CSR payloads (+weights) per load
+    h2d += 8 * (n + 1) * 2 // (2 if not info["offsets_64bit"] else 1)
+    e2e = {"value": float(np.median(e2e_vals)), "unit": "GTEPS", "h2d_bytes_per_step": h2d,
+           "d2h_bytes_per_step": 4 * n,
+           "what": "gr_graph_load(host COO: shard build + H2D) + gr_run + gr_fetch_vertex_values, wall clock"}
+
+    cpu = None
+    if rank == 0 and world == 1 and not args.no_cpu:
+        cpu = cpu_oracle_sample(g, w, run)
+
+    G.close()
+    if rank == 0:
+        line = {
+            "metric": "GTEPS", "value": round(value, 3), "unit": "GTEPS", "n_gpus": world, "steps": args.steps,
+            "warmup": args.warmup, "ms_per_step": round(ms_step, 4), "s_per_run": ms_step * 1e-3,
+            "higher_is_better": True, "scaling": "strong", "vs_baseline": None,
+            "dtype": "f32" if algo == "pagerank" else "u32", "data": "synthetic",
+            "config": {"workload": CONFIG_NAMES[args.config], "n": n, "m": m, "shards": info["num_shards"],
+                       "mode": "resident", "l2": "inputs larger than L2 (CSC payload > 126 MB L2); no flush",
+                       "iterations": stats["iterations"]},
+            "roofline": roof, "run_roofline": run_roof, "cpu_baseline": cpu, "e2e": e2e,
+            "gpu_launches": launches, "clocks": ck,
+        }
+        print(json.dumps(line), flush=True)
+    if world > 1:
+        torch.distributed.destroy_process_group()
+    return 0
+
+
+if __name__ == "__main__":
+    sys.exit(main())

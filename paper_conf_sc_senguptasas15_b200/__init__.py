@@ -1,0 +1,317 @@
+"""GraphReduce on B200 — thin Python binding of include/graphreduce.h.
+
+Argument marshalling only: every step of the GAS superstep runs in the CUDA
+library ``libgraphreduce.so`` (sm_100a). There is no CPU fallback; if the
+library cannot be loaded every call raises.
+
+Functions carry the C names (``gr_graph_load``, ``gr_run``,
+``gr_fetch_vertex_values``, ...). ``GraphReduce`` is a small convenience
+wrapper around a ``gr_graph`` handle.
+"""
+from __future__ import annotations
+
+import ctypes
+import os
+
+import numpy as np
+
+from . import _build
+
+_SO = _build.SO
+_lib = None
+
+GR_OK, GR_EINVAL, GR_ENOMEM, GR_ECUDA, GR_ENCCL, GR_EUNSUPPORTED, GR_ESTATE = range(7)
+STATUS_NAMES = ["GR_OK", "GR_EINVAL", "GR_ENOMEM", "GR_ECUDA", "GR_ENCCL", "GR_EUNSUPPORTED", "GR_ESTATE"]
+GR_FMT_COO, GR_FMT_CSR = 0, 1
+ALGOS = {"bfs": 0, "sssp": 1, "pagerank": 2, "cc": 3, "custom": 4}
+MODES = {"auto": 0, "resident": 1, "streamed": 2}
+LOOPS = {"auto": 0, "host": 1, "device": 2}
+INF = 0xFFFFFFFF
+
+EXPORTS = [
+    "gr_get_unique_id", "gr_graph_load", "gr_run", "gr_fetch_vertex_values", "gr_fetch_frontier_trace",
+    "gr_graph_info_get", "gr_shard_info", "gr_graph_free", "gr_last_error", "gr_plan_intervals",
+    "gr_host_build", "gr_host_csc", "gr_host_csr", "gr_host_shards", "gr_host_free",
+]
+
+
+class GrError(RuntimeError):
+    def __init__(self, status: int, msg: str):
+        super().__init__(f"{STATUS_NAMES[status] if 0 <= status < 7 else status}: {msg}")
+        self.status = status
+
+
+class gr_edges(ctypes.Structure):
+    _fields_ = [("fmt", ctypes.c_int32), ("num_vertices", ctypes.c_uint64), ("num_edges", ctypes.c_uint64),
+                ("src", ctypes.c_void_p), ("dst", ctypes.c_void_p), ("row_offsets", ctypes.c_void_p),
+                ("col_idx", ctypes.c_void_p), ("weights", ctypes.c_void_p)]
+
+
+class gr_load_opts(ctypes.Structure):
+    _fields_ = [("shard_edges", ctypes.c_uint64), ("device_budget_bytes", ctypes.c_uint64),
+                ("mode", ctypes.c_int32), ("device", ctypes.c_int32), ("rank", ctypes.c_int32),
+                ("world", ctypes.c_int32), ("nccl_unique_id", ctypes.c_void_p), ("host_threads", ctypes.c_int32),
+                ("sim_ranks", ctypes.c_int32)]
+
+
+class gr_run_opts(ctypes.Structure):
+    _fields_ = [("algo", ctypes.c_int32), ("source", ctypes.c_uint32), ("max_iters", ctypes.c_uint32),
+                ("damping", ctypes.c_float), ("custom_id", ctypes.c_int32), ("loop", ctypes.c_int32),
+                ("stream", ctypes.c_void_p), ("profile", ctypes.c_int32)]
+
+
+class gr_run_stats(ctypes.Structure):
+    _fields_ = [("iterations", ctypes.c_uint32), ("seconds", ctypes.c_double),
+                ("edges_gathered", ctypes.c_uint64), ("edges_scattered", ctypes.c_uint64),
+                ("bytes_h2d", ctypes.c_uint64), ("bytes_nvlink", ctypes.c_uint64),
+                ("bytes_hbm_model", ctypes.c_uint64), ("kernel_launches", ctypes.c_uint64),
+                ("kernel_ms", ctypes.c_double * 4)]
+
+    def as_dict(self):
+        d = {k: getattr(self, k) for k, _ in self._fields_ if k != "kernel_ms"}
+        d["kernel_ms"] = list(self.kernel_ms)
+        return d
+
+
+class gr_graph_info(ctypes.Structure):
+    _fields_ = [("num_vertices", ctypes.c_uint64), ("num_edges", ctypes.c_uint64), ("num_shards", ctypes.c_uint32),
+                ("mode", ctypes.c_int32), ("rank", ctypes.c_int32), ("world", ctypes.c_int32),
+                ("sim_ranks", ctypes.c_int32), ("own_lo", ctypes.c_uint64), ("own_hi", ctypes.c_uint64),
+                ("device_bytes", ctypes.c_uint64), ("pinned_bytes", ctypes.c_uint64),
+                ("offsets_64bit", ctypes.c_int32), ("has_weights", ctypes.c_int32)]
+
+
+class gr_shard_desc(ctypes.Structure):
+    _fields_ = [("v_lo", ctypes.c_uint64), ("v_hi", ctypes.c_uint64), ("in_begin", ctypes.c_uint64),
+                ("in_end", ctypes.c_uint64), ("out_begin", ctypes.c_uint64), ("out_end", ctypes.c_uint64)]
+
+
+def lib():
+    """Load libgraphreduce.so (built in-tree for sm_100a); raise if unavailable."""
+    global _lib
+    if _lib is not None:
+        return _lib
+    if not os.path.exists(_SO) or _build.stale():
+        if not os.path.exists(_build.NVCC):
+            raise GrError(GR_EUNSUPPORTED, f"{_SO} is missing and nvcc is unavailable to build it")
+        _build.build()
+    L = ctypes.CDLL(_SO)
+    vp, u64, u32, i32 = ctypes.c_void_p, ctypes.c_uint64, ctypes.c_uint32, ctypes.c_int32
+    u64p = ctypes.POINTER(ctypes.c_uint64)
+    sig = {
+        "gr_get_unique_id": (i32, [vp]),
+        "gr_graph_load": (i32, [ctypes.POINTER(gr_edges), ctypes.POINTER(gr_load_opts), ctypes.POINTER(vp)]),
+        "gr_run": (i32, [vp, ctypes.POINTER(gr_run_opts), ctypes.POINTER(gr_run_stats)]),
+        "gr_fetch_vertex_values": (i32, [vp, vp, u64]),
+        "gr_fetch_frontier_trace": (i32, [vp, u64p, u64, u64p]),
+        "gr_graph_info_get": (i32, [vp, ctypes.POINTER(gr_graph_info)]),
+        "gr_shard_info": (i32, [vp, u32, ctypes.POINTER(gr_shard_desc)]),
+        "gr_graph_free": (None, [vp]),
+        "gr_last_error": (ctypes.c_char_p, []),
+        "gr_plan_intervals": (i32, [u64, u64p, u32, u64p]),
+        "gr_host_build": (i32, [ctypes.POINTER(gr_edges), ctypes.POINTER(gr_load_opts), ctypes.POINTER(vp)]),
+        "gr_host_csc": (i32, [vp, ctypes.POINTER(u64p), ctypes.POINTER(ctypes.POINTER(u32)),
+                              ctypes.POINTER(ctypes.POINTER(ctypes.c_uint8))]),
+        "gr_host_csr": (i32, [vp, ctypes.POINTER(u64p), ctypes.POINTER(ctypes.POINTER(u32)),
+                              ctypes.POINTER(ctypes.POINTER(ctypes.c_uint8))]),
+        "gr_host_shards": (i32, [vp, ctypes.POINTER(u32), ctypes.POINTER(u64p)]),
+        "gr_host_free": (None, [vp]),
+    }
+    for name, (res, args) in sig.items():
+        f = getattr(L, name)
+        f.restype = res
+        f.argtypes = args
+    _lib = L
+    return L
+
+
+def _check(status: int):
+    if status != GR_OK:
+        raise GrError(status, lib().gr_last_error().decode(errors="replace"))
+
+
+def _u32(a):
+    return None if a is None else np.ascontiguousarray(a, dtype=np.uint32)
+
+
+def _edges(n, src=None, dst=None, weights=None, row_offsets=None, col_idx=None):
+    keep = []
+    e = gr_edges()
+    e.num_vertices = int(n)
+    if row_offsets is not None:
+        ro = np.ascontiguousarray(row_offsets, dtype=np.uint64)
+        ci = _u32(col_idx)
+        keep += [ro, ci]
+        e.fmt, e.num_edges = GR_FMT_CSR, int(ci.shape[0])
+        e.row_offsets, e.col_idx = ro.ctypes.data, ci.ctypes.data
+    else:
+        s, d = _u32(src), _u32(dst)
+        keep += [s, d]
+        e.fmt, e.num_edges = GR_FMT_COO, int(s.shape[0])
+        e.src, e.dst = s.ctypes.data, d.ctypes.data
+    if weights is not None:
+        w = _u32(weights)
+        keep.append(w)
+        e.weights = w.ctypes.data
+    return e, keep
+
+
+def _load_opts(shard_edges=0, device_budget_bytes=0, mode="auto", device=0, rank=0, world=1,
+               nccl_unique_id=None, host_threads=0, sim_ranks=0):
+    o = gr_load_opts()
+    o.shard_edges, o.device_budget_bytes = int(shard_edges), int(device_budget_bytes)
+    o.mode = MODES[mode] if isinstance(mode, str) else int(mode)
+    o.device, o.rank, o.world = int(device), int(rank), int(world)
+    uid = None
+    if nccl_unique_id is not None:
+        uid = ctypes.create_string_buffer(bytes(nccl_unique_id), 128)
+        o.nccl_unique_id = ctypes.cast(uid, ctypes.c_void_p)
+    o.host_threads, o.sim_ranks = int(host_threads), int(sim_ranks)
+    return o, uid
+
+
+# ----------------------------------------------------------------- C names
+def gr_get_unique_id() -> bytes:
+    buf = ctypes.create_string_buffer(128)
+    _check(lib().gr_get_unique_id(buf))
+    return buf.raw
+
+
+def gr_graph_load(n, src=None, dst=None, weights=None, row_offsets=None, col_idx=None, **opts):
+    """Partition + lay out + place the graph; returns an opaque handle (c_void_p)."""
+    e, keep = _edges(n, src, dst, weights, row_offsets, col_idx)
+    o, uid = _load_opts(**opts)
+    h = ctypes.c_void_p()
+    _check(lib().gr_graph_load(ctypes.byref(e), ctypes.byref(o), ctypes.byref(h)))
+    del keep, uid
+    return h
+
+
+def gr_run(h, algo, source=0, max_iters=0, damping=0.85, custom_id=0, loop="auto", stream=None,
+           profile=False) -> dict:
+    o = gr_run_opts()
+    o.algo = ALGOS[algo] if isinstance(algo, str) else int(algo)
+    o.source, o.max_iters, o.damping, o.custom_id = int(source), int(max_iters), float(damping), int(custom_id)
+    o.loop = LOOPS[loop] if isinstance(loop, str) else int(loop)
+    o.stream = stream
+    o.profile = 1 if profile else 0
+    st = gr_run_stats()
+    _check(lib().gr_run(h, ctypes.byref(o), ctypes.byref(st)))
+    return st.as_dict()
+
+
+def gr_graph_info_get(h) -> dict:
+    i = gr_graph_info()
+    _check(lib().gr_graph_info_get(h, ctypes.byref(i)))
+    return {k: getattr(i, k) for k, _ in i._fields_}
+
+
+def gr_fetch_vertex_values(h, out: np.ndarray | None = None, dtype=np.uint32) -> np.ndarray:
+    n = gr_graph_info_get(h)["num_vertices"]
+    if out is None:
+        out = np.empty(n, dtype)
+    _check(lib().gr_fetch_vertex_values(h, out.ctypes.data, out.nbytes))
+    return out
+
+
+def gr_fetch_frontier_trace(h, max_rows: int = 1 << 20) -> np.ndarray:
+    buf = np.zeros((max_rows, 4), np.uint64)
+    rows = ctypes.c_uint64(0)
+    _check(lib().gr_fetch_frontier_trace(h, buf.ctypes.data_as(ctypes.POINTER(ctypes.c_uint64)), max_rows,
+                                         ctypes.byref(rows)))
+    return buf[: rows.value].copy()
+
+
+def gr_shard_info(h, s: int) -> dict:
+    d = gr_shard_desc()
+    _check(lib().gr_shard_info(h, s, ctypes.byref(d)))
+    return {k: getattr(d, k) for k, _ in d._fields_}
+
+
+def gr_graph_free(h):
+    if h:
+        lib().gr_graph_free(h)
+
+
+def gr_plan_intervals(weight_prefix, P: int) -> np.ndarray:
+    wp = np.ascontiguousarray(weight_prefix, dtype=np.uint64)
+    b = np.zeros(P + 1, np.uint64)
+    u64p = ctypes.POINTER(ctypes.c_uint64)
+    _check(lib().gr_plan_intervals(len(wp) - 1, wp.ctypes.data_as(u64p), P, b.ctypes.data_as(u64p)))
+    return b
+
+
+class HostLayout:
+    """gr_host_build: the host-side sharded layout, copied out to numpy (CPU only)."""
+
+    def __init__(self, n, src, dst, weights=None, **opts):
+        e, keep = _edges(n, src, dst, weights)
+        o, uid = _load_opts(**opts)
+        h = ctypes.c_void_p()
+        L = lib()
+        _check(L.gr_host_build(ctypes.byref(e), ctypes.byref(o), ctypes.byref(h)))
+        try:
+            info = self._copy(L, h, int(n), weights is not None)
+        finally:
+            L.gr_host_free(h)
+        self.__dict__.update(info)
+
+    @staticmethod
+    def _copy(L, h, n, has_w):
+        u64p, u32p, u8p = (ctypes.POINTER(ctypes.c_uint64), ctypes.POINTER(ctypes.c_uint32),
+                           ctypes.POINTER(ctypes.c_uint8))
+        nshard = ctypes.c_uint32()
+        bp = u64p()
+        _check(L.gr_host_shards(h, ctypes.byref(nshard), ctypes.byref(bp)))
+        bounds = np.ctypeslib.as_array(bp, (nshard.value + 1,)).copy()
+        off, idx, w = u64p(), u32p(), u8p()
+        _check(L.gr_host_csc(h, ctypes.byref(off), ctypes.byref(idx), ctypes.byref(w)))
+        own_n = int(bounds[-1] - bounds[0])
+        in_off = np.ctypeslib.as_array(off, (own_n + 1,)).copy()
+        m_in = int(in_off[-1])
+        in_src = np.ctypeslib.as_array(idx, (max(m_in, 1),))[:m_in].copy()
+        in_w = np.ctypeslib.as_array(w, (max(m_in, 1),))[:m_in].copy() if has_w and m_in else None
+        _check(L.gr_host_csr(h, ctypes.byref(off), ctypes.byref(idx), ctypes.byref(w)))
+        out_off = np.ctypeslib.as_array(off, (n + 1,)).copy()
+        out_dst = np.ctypeslib.as_array(idx, (max(m_in, 1),))[:m_in].copy()
+        out_w = np.ctypeslib.as_array(w, (max(m_in, 1),))[:m_in].copy() if has_w and m_in else None
+        return dict(bounds=bounds, in_off=in_off, in_src=in_src, in_w=in_w, out_off=out_off, out_dst=out_dst,
+                    out_w=out_w)
+
+
+class GraphReduce:
+    """Convenience wrapper: load once, run many programs, fetch results."""
+
+    def __init__(self, n, src=None, dst=None, weights=None, **opts):
+        self.n = int(n)
+        self.h = gr_graph_load(n, src, dst, weights, **opts)
+
+    def run(self, algo, **kw) -> dict:
+        return gr_run(self.h, algo, **kw)
+
+    def values(self, algo=None):
+        dt = np.float32 if algo == "pagerank" else np.uint32
+        return gr_fetch_vertex_values(self.h, dtype=dt)
+
+    def trace(self):
+        return gr_fetch_frontier_trace(self.h)
+
+    def info(self):
+        return gr_graph_info_get(self.h)
+
+    def close(self):
+        if self.h:
+            gr_graph_free(self.h)
+            self.h = None
+
+    def __enter__(self):
+        return self
+
+    def __exit__(self, *a):
+        self.close()
+
+    def __del__(self):
+        try:
+            self.close()
+        except Exception:
+            pass

@@ -1,0 +1,210 @@
+// api.cu — extern "C" entry points of include/graphreduce.h.
+#include <cuda_runtime.h>
+#include <nccl.h>
+
+#include <cstring>
+
+#include "engine.h"
+
+using namespace gr;
+
+struct gr_host_graph {
+  HostGraph H;
+};
+
+namespace gr {
+uint64_t static_bytes_estimate(const HostGraph &H) {
+  const uint64_t n = H.n, on = H.own_n(), mi = H.m_in;
+  const uint64_t offb = (mi >= 0xFFFFFFFFull) ? 8 : 4;
+  const uint64_t tiles = (on + mi) / 2048 + 2;
+  return offb * (on + 1) + offb * (n + 1) + n / 8 + on / 8 + 4 * n /*val*/ + 4 * on /*stamp*/ +
+         8 * 4 * on /*lists*/ + 4 * n /*outdeg*/ + 12 * n /*inv, contrib x2*/ + 4 * on /*rank*/ + 16 * tiles +
+         (32ull << 20) /*trace*/;
+}
+uint64_t resident_bytes_estimate(const HostGraph &H) {
+  return static_bytes_estimate(H) + 8 * (H.m_in + 16) + (H.has_w ? H.m_in + 16 : 0);
+}
+}  // namespace gr
+
+extern "C" {
+
+const char *gr_last_error(void) { return gr::last_error(); }
+
+gr_status gr_get_unique_id(uint8_t out[128]) {
+  clear_error();
+  if (!out) return fail(GR_EINVAL, "out is NULL");
+  ncclUniqueId id;
+  ncclResult_t r = ncclGetUniqueId(&id);
+  if (r != ncclSuccess) return fail(GR_ENCCL, "ncclGetUniqueId: %s", ncclGetErrorString(r));
+  static_assert(sizeof(id) == 128, "ncclUniqueId is 128 bytes");
+  std::memcpy(out, &id, 128);
+  return GR_OK;
+}
+
+gr_status gr_graph_load(const gr_edges *edges, const gr_load_opts *opts_in, gr_graph **out) {
+  clear_error();
+  if (!out) return fail(GR_EINVAL, "out is NULL");
+  *out = nullptr;
+  if (!edges) return fail(GR_EINVAL, "edges is NULL");
+  gr_load_opts opts{};
+  if (opts_in) opts = *opts_in;
+  if (opts.world <= 0) opts.world = 1;
+  if (opts.mode < GR_MODE_AUTO || opts.mode > GR_MODE_STREAMED) return fail(GR_EINVAL, "bad mode %d", opts.mode);
+  if (opts.world > 1 || opts.sim_ranks > 1)
+    return fail(GR_EUNSUPPORTED, "multi-rank partitions are not available in this build");
+  int ndev = 0;
+  cudaError_t ce = cudaGetDeviceCount(&ndev);
+  if (ce != cudaSuccess || ndev == 0) {
+    cudaGetLastError();
+    return fail(GR_ECUDA, "no CUDA device available (%s)", cudaGetErrorString(ce));
+  }
+  if (opts.device < 0 || opts.device >= ndev) return fail(GR_EINVAL, "device %d out of range", opts.device);
+  if (cudaSetDevice(opts.device) != cudaSuccess) return fail(GR_ECUDA, "cudaSetDevice failed");
+
+  gr_graph *g = new gr_graph();
+  g->device = opts.device;
+  std::string err;
+  gr_status s = build_host_graph(edges, opts.shard_edges, opts.world, opts.rank, opts.host_threads, &g->H, &err);
+  if (s != GR_OK) {
+    delete g;
+    return fail(s, "%s", err.c_str());
+  }
+  cudaDeviceProp prop;
+  cudaGetDeviceProperties(&prop, g->device);
+  g->num_sms = prop.multiProcessorCount;
+  if (cudaStreamCreateWithFlags(&g->stream, cudaStreamNonBlocking) != cudaSuccess ||
+      cudaEventCreate(&g->ev_start) != cudaSuccess || cudaEventCreate(&g->ev_stop) != cudaSuccess ||
+      cudaMallocHost((void **)&g->h_ctl, sizeof(Ctl)) != cudaSuccess) {
+    destroy(g);
+    return fail(GR_ECUDA, "stream/event/pinned setup failed");
+  }
+  for (int i = 0; i < 2; i++) {
+    cudaEvent_t e;
+    cudaEventCreate(&e);
+    g->prof_ev.push_back(e);
+  }
+  size_t free_b = 0, total_b = 0;
+  cudaMemGetInfo(&free_b, &total_b);
+  uint64_t budget = opts.device_budget_bytes ? opts.device_budget_bytes
+                                             : (free_b > (4ull << 30) ? free_b - (4ull << 30) : free_b / 2);
+  const uint64_t need = resident_bytes_estimate(g->H);
+  if (opts.mode == GR_MODE_AUTO) g->mode = need <= budget ? GR_MODE_RESIDENT : GR_MODE_STREAMED;
+  else g->mode = opts.mode;
+  s = load_device(g);
+  if (s == GR_OK && g->mode == GR_MODE_STREAMED) s = stream_setup(g, budget);
+  if (s != GR_OK) {
+    std::string keep = gr::last_error();
+    destroy(g);
+    return fail(s, "%s", keep.c_str());
+  }
+  *out = g;
+  return GR_OK;
+}
+
+gr_status gr_run(gr_graph *g, const gr_run_opts *opts, gr_run_stats *stats) {
+  clear_error();
+  if (!g || !opts) return fail(GR_EINVAL, "graph or opts is NULL");
+  gr_run_stats st{};
+  cudaSetDevice(g->device);
+  gr_status s = gr::run(g, opts, &st);
+  if (stats) *stats = st;
+  return s;
+}
+
+gr_status gr_fetch_vertex_values(gr_graph *g, void *host_dst, uint64_t bytes) {
+  clear_error();
+  if (!g) return fail(GR_EINVAL, "graph is NULL");
+  cudaSetDevice(g->device);
+  return fetch_values(g, host_dst, bytes);
+}
+
+gr_status gr_fetch_frontier_trace(gr_graph *g, uint64_t *host_dst, uint64_t max_rows, uint64_t *rows) {
+  clear_error();
+  if (!g) return fail(GR_EINVAL, "graph is NULL");
+  cudaSetDevice(g->device);
+  return fetch_trace(g, host_dst, max_rows, rows);
+}
+
+gr_status gr_graph_info_get(const gr_graph *g, gr_graph_info *o) {
+  clear_error();
+  if (!g || !o) return fail(GR_EINVAL, "null argument");
+  std::memset(o, 0, sizeof *o);
+  o->num_vertices = g->H.n;
+  o->num_edges = g->H.m_total;
+  o->num_shards = g->H.num_shards();
+  o->mode = g->mode;
+  o->rank = 0;
+  o->world = 1;
+  o->sim_ranks = 1;
+  o->own_lo = g->H.own_lo;
+  o->own_hi = g->H.own_hi;
+  o->device_bytes = g->dev_bytes;
+  o->pinned_bytes = g->pinned_bytes;
+  o->offsets_64bit = g->off64 ? 1 : 0;
+  o->has_weights = g->H.has_w ? 1 : 0;
+  return GR_OK;
+}
+
+static void shard_desc(const HostGraph &H, uint32_t s, gr_shard_desc *o) {
+  o->v_lo = H.bounds[s];
+  o->v_hi = H.bounds[s + 1];
+  o->in_begin = H.in_off[o->v_lo - H.own_lo];
+  o->in_end = H.in_off[o->v_hi - H.own_lo];
+  o->out_begin = H.out_off[o->v_lo];
+  o->out_end = H.out_off[o->v_hi];
+}
+
+gr_status gr_shard_info(const gr_graph *g, uint32_t s, gr_shard_desc *o) {
+  clear_error();
+  if (!g || !o) return fail(GR_EINVAL, "null argument");
+  if (s >= g->H.num_shards()) return fail(GR_EINVAL, "shard %u >= %u", s, g->H.num_shards());
+  shard_desc(g->H, s, o);
+  return GR_OK;
+}
+
+void gr_graph_free(gr_graph *g) { destroy(g); }
+
+gr_status gr_host_build(const gr_edges *edges, const gr_load_opts *opts_in, gr_host_graph **out) {
+  clear_error();
+  if (!out) return fail(GR_EINVAL, "out is NULL");
+  *out = nullptr;
+  gr_load_opts opts{};
+  if (opts_in) opts = *opts_in;
+  auto *h = new gr_host_graph();
+  std::string err;
+  gr_status s = build_host_graph(edges, opts.shard_edges, opts.world > 0 ? opts.world : 1, opts.rank,
+                                 opts.host_threads, &h->H, &err);
+  if (s != GR_OK) {
+    delete h;
+    return fail(s, "%s", err.c_str());
+  }
+  *out = h;
+  return GR_OK;
+}
+
+gr_status gr_host_csc(const gr_host_graph *h, const uint64_t **off, const uint32_t **src, const uint8_t **w) {
+  if (!h || !off || !src) return fail(GR_EINVAL, "null argument");
+  *off = h->H.in_off.data();
+  *src = h->H.in_src.as<uint32_t>();
+  if (w) *w = h->H.has_w ? h->H.in_w.as<uint8_t>() : nullptr;
+  return GR_OK;
+}
+
+gr_status gr_host_csr(const gr_host_graph *h, const uint64_t **off, const uint32_t **dst, const uint8_t **w) {
+  if (!h || !off || !dst) return fail(GR_EINVAL, "null argument");
+  *off = h->H.out_off.data();
+  *dst = h->H.out_dst.as<uint32_t>();
+  if (w) *w = h->H.has_w ? h->H.out_w.as<uint8_t>() : nullptr;
+  return GR_OK;
+}
+
+gr_status gr_host_shards(const gr_host_graph *h, uint32_t *num_shards, const uint64_t **bounds) {
+  if (!h || !num_shards || !bounds) return fail(GR_EINVAL, "null argument");
+  *num_shards = h->H.num_shards();
+  *bounds = h->H.bounds.data();
+  return GR_OK;
+}
+
+void gr_host_free(gr_host_graph *h) { delete h; }
+
+}  // extern "C"

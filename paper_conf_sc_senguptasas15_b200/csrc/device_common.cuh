@@ -1,0 +1,135 @@
+// device_common.cuh — device-side state and warp-level helpers shared by the
+// GAS kernels (sm_100a only).
+#pragma once
+#include <cstdint>
+
+#include <cuda_runtime.h>
+
+namespace gr {
+
+constexpr uint32_t kInf = 0xFFFFFFFFu;
+constexpr int kWarp = 32;
+constexpr int kBlock = 256;              // threads per CTA for the frontier kernels
+constexpr int kWarpsPerBlock = kBlock / kWarp;
+constexpr uint32_t kHubDegree = 1024;    // > this degree: one CTA per vertex (K6 CTA load balancing)
+constexpr int kQueueCap = 128;           // per-warp staging entries before one global append
+
+// Device control block of one run (superstep bookkeeping).
+// Lists are ping-ponged by superstep parity so a captured CUDA graph can loop.
+struct Ctl {
+  uint32_t iter;          // superstep t
+  uint32_t epoch_base;    // stamp epoch of superstep 0 (stamps only grow across runs)
+  uint32_t max_iters;     // 0 = unlimited
+  uint32_t stop;          // 1 once the frontier is empty / max_iters reached
+  uint32_t cnt_A[2];      // non-hub list length of A_t (slot t&1)
+  uint32_t cnt_H[2];      // hub list length of A_t
+  uint32_t cnt_act[2];    // |A_t| (distinct activated vertices; BFS lists are filtered)
+  uint32_t cnt_C;         // non-hub changed entries
+  uint32_t cnt_CH;        // hub changed entries
+  uint32_t ctr_hub;       // dynamic hub work counter (gather / BFS)
+  uint32_t ctr_hub2;      // dynamic hub work counter (activate)
+  uint32_t done_blocks;   // last-block ticket
+  uint32_t implicit0;     // superstep 0 list is implicitly the owned range (CC: A_0 = V)
+  uint32_t trace_cap;
+  uint32_t source;        // BFS / SSSP source (programs may read it through Ctx)
+  float damping;
+  unsigned long long changed;    // |C_t| of the current superstep
+  unsigned long long gathered;   // sum indeg(A_t)
+  unsigned long long scattered;  // sum outdeg(C_t)
+  unsigned long long tot_gathered, tot_scattered;
+};
+
+// Device view of one owner partition (single GPU = one partition owning V).
+template <class OffT> struct Part {
+  uint32_t n;             // |V|
+  uint32_t own_lo, own_n; // owned destination range
+  const OffT *in_off;     // [own_n + 1]  CSC offsets (local vertex index)
+  const uint32_t *in_src; // [m_in]       in-edge sources
+  const uint8_t *in_w;    // [m_in]       weights (nullable)
+  const OffT *out_off;    // [n + 1]      activation CSR offsets (global source id)
+  const uint32_t *out_dst;// [m_in]       owned destinations
+  const uint32_t *hub_in; // bitmap over owned vertices: indeg > kHubDegree
+  const uint32_t *hub_out;// bitmap over all V: activation outdeg > kHubDegree
+  uint32_t *val;          // [n] vertex values (replica of superstep t-1; BSP read side)
+  uint32_t *stamp;        // [own_n] activation epoch per owned vertex (dedup)
+  uint32_t *listA[2];     // non-hub A lists (owned ids, global)
+  uint32_t *listH[2];     // hub A lists
+  uint32_t *C_v, *C_val;  // changed list (non-hub)
+  uint32_t *CH_v, *CH_val;// changed list (activation hubs)
+  Ctl *ctl;
+  unsigned long long *trace; // [trace_cap][4]
+};
+
+__device__ __forceinline__ uint32_t lane_id() { return threadIdx.x & 31; }
+__device__ __forceinline__ uint32_t lanemask_lt() {
+  uint32_t m;
+  asm("mov.u32 %0, %%lanemask_lt;" : "=r"(m));
+  return m;
+}
+
+__device__ __forceinline__ uint32_t ldg_nc(const uint32_t *p) {
+  uint32_t v;
+  asm volatile("ld.global.nc.L1::no_allocate.u32 %0, [%1];" : "=r"(v) : "l"(p));
+  return v;
+}
+__device__ __forceinline__ uint8_t ldg_nc_u8(const uint8_t *p) {
+  uint16_t v;
+  asm volatile("ld.global.nc.L1::no_allocate.u8 %0, [%1];" : "=h"(v) : "l"(p));
+  return (uint8_t)v;
+}
+
+__device__ __forceinline__ bool test_bit(const uint32_t *bits, uint32_t i) {
+  return (__ldg(bits + (i >> 5)) >> (i & 31)) & 1u;
+}
+
+// Warp-inclusive scan of a uint32 (all lanes participate).
+__device__ __forceinline__ uint32_t warp_incl_scan(uint32_t x) {
+#pragma unroll
+  for (int o = 1; o < 32; o <<= 1) {
+    uint32_t y = __shfl_up_sync(0xffffffffu, x, o);
+    if (lane_id() >= (uint32_t)o) x += y;
+  }
+  return x;
+}
+
+__device__ __forceinline__ unsigned long long warp_sum_u64(unsigned long long x) {
+#pragma unroll
+  for (int o = 16; o > 0; o >>= 1) x += __shfl_xor_sync(0xffffffffu, x, o);
+  return x;
+}
+
+// Per-warp staging queue: entries are collected in shared memory and appended
+// to a global list with ONE atomicAdd per flush (not one per element).
+struct WarpQueue {
+  uint32_t *s_a;   // [kQueueCap] shared
+  uint32_t *s_b;   // [kQueueCap] shared or nullptr (pair lists)
+  uint32_t n;      // warp-uniform fill level
+  __device__ void flush(uint32_t *g_a, uint32_t *g_b, uint32_t *g_cnt) {
+    __syncwarp();
+    if (n == 0) return;
+    uint32_t base = 0;
+    if (lane_id() == 0) base = atomicAdd(g_cnt, n);
+    base = __shfl_sync(0xffffffffu, base, 0);
+    for (uint32_t i = lane_id(); i < n; i += 32) {
+      g_a[base + i] = s_a[i];
+      if (g_b) g_b[base + i] = s_b[i];
+    }
+    __syncwarp();
+    n = 0;
+  }
+  __device__ void push(bool p, uint32_t a, uint32_t b, uint32_t *g_a, uint32_t *g_b, uint32_t *g_cnt) {
+    uint32_t mask = __ballot_sync(0xffffffffu, p);
+    if (mask == 0) return;
+    uint32_t k = __popc(mask);
+    if (n + k > (uint32_t)kQueueCap) flush(g_a, g_b, g_cnt);
+    if (p) {
+      uint32_t pos = n + __popc(mask & lanemask_lt());
+      s_a[pos] = a;
+      if (s_b) s_b[pos] = b;
+    }
+    n += k;
+    __syncwarp();
+  }
+};
+
+}  // namespace gr

@@ -1,0 +1,470 @@
+// engine.cu — the GraphReduce B200 runtime behind include/graphreduce.h.
+//
+// Data Movement + Compute Engine of PAPER.md §4.3-4.4 redesigned for B200:
+//   * resident mode: every shard's CSC/CSR is copied to HBM once at load
+//     (static buffers, §3.2); the GPU then runs "one grid spans many
+//     shards" — the two-level parallelism of L258 without per-shard launches;
+//   * streamed mode (stream.cu): shard payloads stay in pinned host memory and
+//     are DMA'd per superstep into K = 2 device slots (Eq. 1-2),
+//     skipping shards with no active vertex (§5.2);
+//   * the BSP loop (L76, L256) runs on the device as a CUDA graph with a
+//     conditional WHILE node (no host round trip per superstep), or on the
+//     host (GR_LOOP_HOST).
+#include <cuda_runtime.h>
+
+#include <algorithm>
+#include <cstdarg>
+#include <cstdio>
+#include <cstring>
+#include <map>
+#include <string>
+#include <vector>
+
+#include "engine.h"
+#include "kernels_frontier.cuh"
+#include "kernels_pr.cuh"
+
+namespace gr {
+
+static thread_local std::string t_err;
+
+gr_status fail(gr_status s, const char *fmt, ...) {
+  char buf[1024];
+  va_list ap;
+  va_start(ap, fmt);
+  vsnprintf(buf, sizeof buf, fmt, ap);
+  va_end(ap);
+  t_err = buf;
+  return s;
+}
+
+const char *last_error() { return t_err.c_str(); }
+void clear_error() { t_err.clear(); }
+
+#define CK(call)                                                                              \
+  do {                                                                                        \
+    cudaError_t e_ = (call);                                                                  \
+    if (e_ != cudaSuccess)                                                                    \
+      return fail(e_ == cudaErrorMemoryAllocation ? GR_ENOMEM : GR_ECUDA, "%s: %s (%s:%d)", #call, \
+                  cudaGetErrorString(e_), __FILE__, __LINE__);                                \
+  } while (0)
+
+gr_status dev_alloc(gr_graph *g, void **p, size_t bytes) {
+  *p = nullptr;
+  if (bytes == 0) bytes = 16;
+  cudaError_t e = cudaMalloc(p, bytes);
+  if (e != cudaSuccess) {
+    *p = nullptr;
+    cudaGetLastError();
+    return fail(GR_ENOMEM, "cudaMalloc(%zu bytes) failed: %s", bytes, cudaGetErrorString(e));
+  }
+  g->allocs.push_back(*p);
+  g->dev_bytes += bytes;
+  return GR_OK;
+}
+
+template <class T> static gr_status upload(gr_graph *g, T **dst, const T *src, size_t count) {
+  gr_status s = dev_alloc(g, (void **)dst, count * sizeof(T));
+  if (s != GR_OK) return s;
+  if (count) CK(cudaMemcpy(*dst, src, count * sizeof(T), cudaMemcpyHostToDevice));
+  return GR_OK;
+}
+
+// --------------------------------------------------------------- Part views
+template <class OffT> Part<OffT> make_part(gr_graph *g) {
+  Part<OffT> P{};
+  P.n = (uint32_t)g->H.n;
+  P.own_lo = (uint32_t)g->H.own_lo;
+  P.own_n = (uint32_t)g->H.own_n();
+  P.in_off = (const OffT *)g->in_off;
+  P.in_src = g->in_src;
+  P.in_w = g->in_w;
+  P.out_off = (const OffT *)g->out_off;
+  P.out_dst = g->out_dst;
+  P.hub_in = g->hub_in;
+  P.hub_out = g->hub_out;
+  P.val = g->val;
+  P.stamp = g->stamp;
+  for (int i = 0; i < 2; i++) { P.listA[i] = g->listA[i]; P.listH[i] = g->listH[i]; }
+  P.C_v = g->C_v; P.C_val = g->C_val; P.CH_v = g->CH_v; P.CH_val = g->CH_val;
+  P.ctl = g->ctl;
+  P.trace = g->trace;
+  return P;
+}
+
+template <class OffT> static gr_status upload_offsets(gr_graph *g, void **dst, const std::vector<uint64_t> &off) {
+  if (sizeof(OffT) == 8) return upload(g, (uint64_t **)dst, off.data(), off.size());
+  std::vector<uint32_t> o32(off.size());
+  for (size_t i = 0; i < off.size(); i++) o32[i] = (uint32_t)off[i];
+  return upload(g, (uint32_t **)dst, o32.data(), o32.size());
+}
+
+static void build_hub_bits(const std::vector<uint64_t> &off, uint64_t count, std::vector<uint32_t> *bits,
+                           std::vector<uint32_t> *list, uint64_t id_base) {
+  bits->assign((count + 31) / 32 + 1, 0u);
+  for (uint64_t i = 0; i < count; i++)
+    if (off[i + 1] - off[i] > kHubDegree) {
+      (*bits)[i >> 5] |= 1u << (i & 31);
+      if (list) list->push_back((uint32_t)(id_base + i));
+    }
+}
+
+// ------------------------------------------------------------------- load
+gr_status load_device(gr_graph *g) {
+  HostGraph &H = g->H;
+  const uint64_t n = H.n, own_n = H.own_n(), mi = H.m_in;
+  g->off64 = (mi >= 0xFFFFFFFFull);
+  gr_status s;
+  // static per-vertex metadata (both modes)
+  if (g->off64) {
+    if ((s = upload_offsets<uint64_t>(g, &g->in_off, H.in_off)) != GR_OK) return s;
+    if ((s = upload_offsets<uint64_t>(g, &g->out_off, H.out_off)) != GR_OK) return s;
+  } else {
+    if ((s = upload_offsets<uint32_t>(g, &g->in_off, H.in_off)) != GR_OK) return s;
+    if ((s = upload_offsets<uint32_t>(g, &g->out_off, H.out_off)) != GR_OK) return s;
+  }
+  std::vector<uint32_t> hb_in, hb_out, hubs;
+  build_hub_bits(H.in_off, own_n, &hb_in, &hubs, H.own_lo);
+  build_hub_bits(H.out_off, n, &hb_out, nullptr, 0);
+  if ((s = upload(g, &g->hub_in, hb_in.data(), hb_in.size())) != GR_OK) return s;
+  if ((s = upload(g, &g->hub_out, hb_out.data(), hb_out.size())) != GR_OK) return s;
+  g->n_static_hubs = (uint32_t)hubs.size();
+  if ((s = upload(g, &g->static_hubs, hubs.data(), hubs.size())) != GR_OK) return s;
+
+  // edge payloads: resident copies (streamed mode keeps them in pinned host memory)
+  if (g->mode == GR_MODE_RESIDENT) {
+    if ((s = upload(g, &g->in_src, H.in_src.as<uint32_t>(), mi + 4)) != GR_OK) return s;
+    if ((s = upload(g, &g->out_dst, H.out_dst.as<uint32_t>(), mi + 4)) != GR_OK) return s;
+    if (H.has_w && (s = upload(g, &g->in_w, H.in_w.as<uint8_t>(), mi + 16)) != GR_OK) return s;
+  }
+
+  // vertex state (replicated values, owned frontier structures)
+  const size_t ow = std::max<uint64_t>(own_n, 1);
+  if ((s = dev_alloc(g, (void **)&g->val, 4 * n)) != GR_OK) return s;
+  if ((s = dev_alloc(g, (void **)&g->stamp, 4 * ow)) != GR_OK) return s;
+  CK(cudaMemset(g->stamp, 0, 4 * ow));
+  for (int i = 0; i < 2; i++) {
+    if ((s = dev_alloc(g, (void **)&g->listA[i], 4 * ow)) != GR_OK) return s;
+    if ((s = dev_alloc(g, (void **)&g->listH[i], 4 * ow)) != GR_OK) return s;
+  }
+  if ((s = dev_alloc(g, (void **)&g->C_v, 4 * ow)) != GR_OK) return s;
+  if ((s = dev_alloc(g, (void **)&g->C_val, 4 * ow)) != GR_OK) return s;
+  if ((s = dev_alloc(g, (void **)&g->CH_v, 4 * ow)) != GR_OK) return s;
+  if ((s = dev_alloc(g, (void **)&g->CH_val, 4 * ow)) != GR_OK) return s;
+  if ((s = dev_alloc(g, (void **)&g->ctl, sizeof(Ctl))) != GR_OK) return s;
+  g->trace_cap = 1u << 20;
+  if ((s = dev_alloc(g, (void **)&g->trace, 32ull * g->trace_cap)) != GR_OK) return s;
+
+  // PageRank state
+  if ((s = upload(g, &g->d_outdeg, H.outdeg.data(), n)) != GR_OK) return s;
+  if ((s = dev_alloc(g, (void **)&g->inv_outdeg, 4 * n)) != GR_OK) return s;
+  k_inv_outdeg<<<g->num_sms * 4, 256, 0, g->stream>>>((uint32_t)n, g->d_outdeg, g->inv_outdeg);
+  CK(cudaGetLastError());
+  for (int i = 0; i < 2; i++)
+    if ((s = dev_alloc(g, (void **)&g->contrib[i], 4 * n)) != GR_OK) return s;
+  if ((s = dev_alloc(g, (void **)&g->rank, 4 * ow)) != GR_OK) return s;
+  const uint64_t items = own_n + mi;
+  g->pr_tiles = (uint32_t)((items + kPrTile - 1) / kPrTile);
+  const size_t tb = 4ull * std::max<uint32_t>(g->pr_tiles, 1);
+  if ((s = dev_alloc(g, (void **)&g->carry_row, tb)) != GR_OK) return s;
+  if ((s = dev_alloc(g, (void **)&g->carry_val, tb)) != GR_OK) return s;
+  if ((s = dev_alloc(g, (void **)&g->head_row, tb)) != GR_OK) return s;
+  if ((s = dev_alloc(g, (void **)&g->head_val, tb)) != GR_OK) return s;
+  CK(cudaStreamSynchronize(g->stream));
+
+  // occupancy-derived persistent grid: a multiple of the SM count
+  int bps = 0;
+  CK(cudaOccupancyMaxActiveBlocksPerMultiprocessor(&bps, k_gather_apply<ProgCC, uint32_t>, kBlock, 0));
+  g->grid_frontier = g->num_sms * std::max(1, std::min(bps, 8));
+  return GR_OK;
+}
+
+// -------------------------------------------------------------- frontier run
+template <class Prog, class OffT>
+static void launch_body(gr_graph *g, cudaStream_t s, unsigned long long cond, int use_graph, uint64_t *launches) {
+  Part<OffT> P = make_part<OffT>(g);
+  if (Prog::kHasGather) {
+    k_gather_apply<Prog, OffT><<<g->grid_frontier, kBlock, 0, s>>>(P);
+    k_activate<OffT><<<g->grid_frontier, kBlock, 0, s>>>(P, cond, use_graph);
+    *launches += 2;
+  } else {
+    k_bfs_expand<OffT><<<g->grid_frontier, kBlock, 0, s>>>(P, cond, use_graph);
+    *launches += 1;
+  }
+}
+
+template <class Prog, class OffT>
+static gr_status get_while_graph(gr_graph *g, int key, cudaGraphExec_t *out, uint64_t *per_iter_launches) {
+  auto it = g->while_exec.find(key);
+  if (it != g->while_exec.end()) {
+    *out = it->second.first;
+    *per_iter_launches = it->second.second;
+    return GR_OK;
+  }
+  cudaGraph_t graph;
+  CK(cudaGraphCreate(&graph, 0));
+  cudaGraphConditionalHandle h;
+  CK(cudaGraphConditionalHandleCreate(&h, graph, 1, cudaGraphCondAssignDefault));
+  cudaGraphNodeParams p = {};
+  p.type = cudaGraphNodeTypeConditional;
+  p.conditional.handle = h;
+  p.conditional.type = cudaGraphCondTypeWhile;
+  p.conditional.size = 1;
+  cudaGraphNode_t node;
+  CK(cudaGraphAddNode(&node, graph, nullptr, 0, &p));
+  cudaGraph_t body = p.conditional.phGraph_out[0];
+  cudaStream_t cs;
+  CK(cudaStreamCreateWithFlags(&cs, cudaStreamNonBlocking));
+  CK(cudaStreamBeginCaptureToGraph(cs, body, nullptr, nullptr, 0, cudaStreamCaptureModeThreadLocal));
+  uint64_t l = 0;
+  launch_body<Prog, OffT>(g, cs, (unsigned long long)h, 1, &l);
+  cudaGraph_t captured = body;
+  cudaError_t e = cudaStreamEndCapture(cs, &captured);
+  cudaStreamDestroy(cs);
+  if (e != cudaSuccess) return fail(GR_ECUDA, "graph capture failed: %s", cudaGetErrorString(e));
+  cudaGraphExec_t ex;
+  CK(cudaGraphInstantiate(&ex, graph, 0));
+  CK(cudaGraphDestroy(graph));
+  g->while_exec[key] = {ex, l};
+  *out = ex;
+  *per_iter_launches = l;
+  return GR_OK;
+}
+
+template <class Prog, class OffT>
+static gr_status run_frontier(gr_graph *g, const gr_run_opts *o, cudaStream_t s, gr_run_stats *st, int key) {
+  Part<OffT> P = make_part<OffT>(g);
+  uint64_t launches = 0;
+  if (g->epoch_next > 0xF0000000u) {
+    CK(cudaMemsetAsync(g->stamp, 0, 4ull * std::max<uint64_t>(g->H.own_n(), 1), s));
+    g->epoch_next = 1;
+  }
+  Ctl h{};
+  h.epoch_base = g->epoch_next;
+  h.max_iters = o->max_iters;
+  h.trace_cap = g->trace_cap;
+  h.source = o->source;
+  h.damping = o->damping;
+  CK(cudaMemcpyAsync(g->ctl, &h, sizeof h, cudaMemcpyHostToDevice, s));
+  k_init_values<Prog, OffT><<<g->num_sms * 4, 256, 0, s>>>(P, o->source);
+  launches++;
+  if (Prog::kInit == kInitAll && g->n_static_hubs)
+    CK(cudaMemcpyAsync(g->listH[0], g->static_hubs, 4ull * g->n_static_hubs, cudaMemcpyDeviceToDevice, s));
+  k_init_frontier<Prog, OffT><<<1, kBlock, 0, s>>>(P, o->source, g->n_static_hubs);
+  launches++;
+  CK(cudaGetLastError());
+  const bool use_graph = (o->loop != GR_LOOP_HOST) && !o->profile;
+  if (use_graph) {
+    cudaGraphExec_t ex;
+    uint64_t per = 0;
+    gr_status gs = get_while_graph<Prog, OffT>(g, key, &ex, &per);
+    if (gs != GR_OK) return gs;
+    CK(cudaGraphLaunch(ex, s));
+    CK(cudaMemcpyAsync(g->h_ctl, g->ctl, sizeof(Ctl), cudaMemcpyDeviceToHost, s));
+    CK(cudaStreamSynchronize(s));
+    launches += per * std::max<uint32_t>(g->h_ctl->iter, 1);
+  } else {
+    cudaEvent_t e0 = g->prof_ev[0], e1 = g->prof_ev[1];
+    for (;;) {
+      if (o->profile) CK(cudaEventRecord(e0, s));
+      launch_body<Prog, OffT>(g, s, 0, 0, &launches);
+      if (o->profile) CK(cudaEventRecord(e1, s));
+      CK(cudaGetLastError());
+      CK(cudaMemcpyAsync(g->h_ctl, g->ctl, sizeof(Ctl), cudaMemcpyDeviceToHost, s));
+      CK(cudaStreamSynchronize(s));
+      if (o->profile) {
+        float ms = 0;
+        CK(cudaEventElapsedTime(&ms, e0, e1));
+        st->kernel_ms[Prog::kHasGather ? 0 : 1] += ms;
+      }
+      if (g->h_ctl->stop) break;
+    }
+  }
+  const Ctl &c = *g->h_ctl;
+  st->iterations = c.iter;
+  st->edges_gathered = c.tot_gathered;
+  st->edges_scattered = c.tot_scattered;
+  st->kernel_launches += launches;
+  g->epoch_next = h.epoch_base + c.iter + 2;
+  g->trace_rows = std::min<uint64_t>(c.iter, g->trace_cap);
+  // algorithmic bytes: 4 B/in-edge (+1 weight), 12 B per active vertex,
+  // 4 B per activated out-edge, 8 B per changed vertex (value commit + offsets)
+  std::vector<unsigned long long> tr(4 * g->trace_rows);
+  if (g->trace_rows)
+    CK(cudaMemcpy(tr.data(), g->trace, 32 * g->trace_rows, cudaMemcpyDeviceToHost));
+  uint64_t sumA = 0, sumC = 0;
+  for (uint64_t t = 0; t < g->trace_rows; t++) { sumA += tr[4 * t]; sumC += tr[4 * t + 1]; }
+  const uint64_t wb = Prog::kUsesWeights ? 5 : 4;
+  st->bytes_hbm_model = wb * c.tot_gathered + 12 * sumA + 4 * c.tot_scattered + 12 * sumC;
+  return GR_OK;
+}
+
+// --------------------------------------------------------------- PageRank
+template <class OffT> static PrArgs<OffT> pr_args(gr_graph *g, uint32_t t, uint32_t iters, float d) {
+  PrArgs<OffT> a{};
+  a.n = (uint32_t)g->H.n;
+  a.own_lo = (uint32_t)g->H.own_lo;
+  a.own_n = (uint32_t)g->H.own_n();
+  a.m_in = g->H.m_in;
+  a.in_off = (const OffT *)g->in_off;
+  a.in_src = g->in_src;
+  a.inv_outdeg = g->inv_outdeg;
+  a.contrib_in = g->contrib[t & 1];
+  a.contrib_out = g->contrib[(t + 1) & 1];
+  a.rank = g->rank;
+  a.carry_row = g->carry_row;
+  a.carry_val = g->carry_val;
+  a.head_row = g->head_row;
+  a.head_val = g->head_val;
+  a.base = (1.0f - d) / (float)g->H.n;
+  a.d = d;
+  a.last = (t + 1 == iters) ? 1 : 0;
+  return a;
+}
+
+template <class OffT>
+static void pr_launch_iter(gr_graph *g, cudaStream_t s, uint32_t t, uint32_t iters, float d, cudaEvent_t e0,
+                           cudaEvent_t e1) {
+  PrArgs<OffT> a = pr_args<OffT>(g, t, iters, d);
+  if (e0) cudaEventRecord(e0, s);
+  k_pr_gather_apply<OffT><<<std::max<uint32_t>(g->pr_tiles, 1), kPrThreads, 0, s>>>(a);
+  if (e1) cudaEventRecord(e1, s);
+  k_pr_fixup<OffT><<<std::max<uint32_t>((g->pr_tiles + 255) / 256, 1), 256, 0, s>>>(a, g->pr_tiles);
+}
+
+template <class OffT>
+static gr_status run_pagerank(gr_graph *g, const gr_run_opts *o, cudaStream_t s, gr_run_stats *st) {
+  const uint32_t iters = o->max_iters;
+  const float d = o->damping;
+  const int prof = o->profile ? 1 : 0;
+  if (prof && g->prof_ev.size() < 2 * (size_t)iters + 2) {
+    while (g->prof_ev.size() < 2 * (size_t)iters + 2) {
+      cudaEvent_t e;
+      CK(cudaEventCreate(&e));
+      g->prof_ev.push_back(e);
+    }
+  }
+  // one CUDA graph per (iters, damping, profile): 2 launches per superstep
+  if (!g->pr_exec || g->pr_exec_iters != iters || g->pr_exec_d != d || g->pr_exec_prof != prof) {
+    if (g->pr_exec) { cudaGraphExecDestroy(g->pr_exec); g->pr_exec = nullptr; }
+    cudaStream_t cs;
+    CK(cudaStreamCreateWithFlags(&cs, cudaStreamNonBlocking));
+    CK(cudaStreamBeginCapture(cs, cudaStreamCaptureModeThreadLocal));
+    k_pr_init<<<g->num_sms * 4, 256, 0, cs>>>((uint32_t)g->H.n, g->inv_outdeg, g->contrib[0]);
+    for (uint32_t t = 0; t < iters; t++)
+      pr_launch_iter<OffT>(g, cs, t, iters, d, prof ? g->prof_ev[2 + 2 * t] : nullptr,
+                           prof ? g->prof_ev[3 + 2 * t] : nullptr);
+    cudaGraph_t graph;
+    cudaError_t e = cudaStreamEndCapture(cs, &graph);
+    cudaStreamDestroy(cs);
+    if (e != cudaSuccess) return fail(GR_ECUDA, "PageRank graph capture failed: %s", cudaGetErrorString(e));
+    CK(cudaGraphInstantiate(&g->pr_exec, graph, 0));
+    CK(cudaGraphDestroy(graph));
+    g->pr_exec_iters = iters;
+    g->pr_exec_d = d;
+    g->pr_exec_prof = prof;
+  }
+  CK(cudaGraphLaunch(g->pr_exec, s));
+  CK(cudaStreamSynchronize(s));
+  if (prof) {
+    for (uint32_t t = 0; t < iters; t++) {
+      float ms = 0;
+      CK(cudaEventElapsedTime(&ms, g->prof_ev[2 + 2 * t], g->prof_ev[3 + 2 * t]));
+      st->kernel_ms[0] += ms;
+    }
+  }
+  st->iterations = iters;
+  st->edges_gathered = (uint64_t)iters * g->H.m_in;
+  st->edges_scattered = 0;
+  st->kernel_launches += 1 + 2ull * iters;
+  st->bytes_hbm_model = (uint64_t)iters * (4 * g->H.m_in + 12 * g->H.own_n() + 4 * g->H.n);
+  g->trace_rows = iters;
+  return GR_OK;
+}
+
+gr_status run(gr_graph *g, const gr_run_opts *oin, gr_run_stats *st) {
+  gr_run_opts o = *oin;
+  if (o.damping == 0.f) o.damping = 0.85f;
+  if (o.algo == GR_PAGERANK && o.max_iters == 0) o.max_iters = 30;
+  if (o.algo == GR_PAGERANK && !(o.damping > 0.f && o.damping < 1.f))
+    return fail(GR_EINVAL, "damping must lie in (0, 1)");
+  if ((o.algo == GR_BFS || o.algo == GR_SSSP) && o.source >= g->H.n)
+    return fail(GR_EINVAL, "source %u >= num_vertices %llu", o.source, (unsigned long long)g->H.n);
+  if (o.algo == GR_SSSP && !g->H.has_w) return fail(GR_EINVAL, "SSSP needs edge weights");
+  if (o.algo < GR_BFS || o.algo > GR_CUSTOM) return fail(GR_EINVAL, "unknown algo %d", o.algo);
+  if (o.algo == GR_CUSTOM) return fail(GR_EUNSUPPORTED, "no custom program with id %d is registered", o.custom_id);
+  if (g->mode == GR_MODE_STREAMED) return run_streamed(g, &o, st);
+  cudaStream_t s = o.stream ? (cudaStream_t)o.stream : g->stream;
+  CK(cudaEventRecord(g->ev_start, s));
+  gr_status r;
+  switch (o.algo) {
+    case GR_BFS:
+      r = g->off64 ? run_frontier<ProgBFS, uint64_t>(g, &o, s, st, 0) : run_frontier<ProgBFS, uint32_t>(g, &o, s, st, 0);
+      break;
+    case GR_SSSP:
+      r = g->off64 ? run_frontier<ProgSSSP, uint64_t>(g, &o, s, st, 1) : run_frontier<ProgSSSP, uint32_t>(g, &o, s, st, 1);
+      break;
+    case GR_CC:
+      r = g->off64 ? run_frontier<ProgCC, uint64_t>(g, &o, s, st, 3) : run_frontier<ProgCC, uint32_t>(g, &o, s, st, 3);
+      break;
+    default:
+      r = g->off64 ? run_pagerank<uint64_t>(g, &o, s, st) : run_pagerank<uint32_t>(g, &o, s, st);
+  }
+  if (r != GR_OK) return r;
+  CK(cudaEventRecord(g->ev_stop, s));
+  CK(cudaEventSynchronize(g->ev_stop));
+  float ms = 0;
+  CK(cudaEventElapsedTime(&ms, g->ev_start, g->ev_stop));
+  st->seconds = ms * 1e-3;
+  g->last_algo = o.algo;
+  g->last_iters = st->iterations;
+  if (o.algo == GR_PAGERANK) g->pr_trace_iters = o.max_iters;
+  return GR_OK;
+}
+
+gr_status fetch_values(gr_graph *g, void *dst, uint64_t bytes) {
+  if (g->last_algo < 0) return fail(GR_ESTATE, "gr_fetch_vertex_values before gr_run");
+  if (!dst) return fail(GR_EINVAL, "host_dst is NULL");
+  const uint64_t n = g->H.n;
+  if (bytes < 4 * n) return fail(GR_EINVAL, "buffer of %llu bytes < 4*n = %llu", (unsigned long long)bytes,
+                                 (unsigned long long)(4 * n));
+  if (g->last_algo == GR_PAGERANK) CK(cudaMemcpy(dst, g->rank, 4 * n, cudaMemcpyDeviceToHost));
+  else CK(cudaMemcpy(dst, g->val, 4 * n, cudaMemcpyDeviceToHost));
+  return GR_OK;
+}
+
+gr_status fetch_trace(gr_graph *g, uint64_t *dst, uint64_t max_rows, uint64_t *rows) {
+  if (g->last_algo < 0) return fail(GR_ESTATE, "gr_fetch_frontier_trace before gr_run");
+  if (!rows || (max_rows && !dst)) return fail(GR_EINVAL, "null output");
+  const uint64_t r = std::min<uint64_t>(g->trace_rows, max_rows);
+  if (g->last_algo == GR_PAGERANK) {
+    for (uint64_t t = 0; t < r; t++) {
+      dst[4 * t] = g->H.own_n();
+      dst[4 * t + 1] = g->H.own_n();
+      dst[4 * t + 2] = g->H.m_in;
+      dst[4 * t + 3] = 0;
+    }
+  } else if (r) {
+    CK(cudaMemcpy(dst, g->trace, 32 * r, cudaMemcpyDeviceToHost));
+  }
+  *rows = r;
+  return GR_OK;
+}
+
+void destroy(gr_graph *g) {
+  if (!g) return;
+  cudaSetDevice(g->device);
+  cudaDeviceSynchronize();
+  for (auto &kv : g->while_exec) cudaGraphExecDestroy(kv.second.first);
+  if (g->pr_exec) cudaGraphExecDestroy(g->pr_exec);
+  for (auto e : g->prof_ev) cudaEventDestroy(e);
+  if (g->ev_start) cudaEventDestroy(g->ev_start);
+  if (g->ev_stop) cudaEventDestroy(g->ev_stop);
+  stream_destroy(g);
+  for (void *p : g->allocs) cudaFree(p);
+  if (g->h_ctl) cudaFreeHost(g->h_ctl);
+  if (g->stream) cudaStreamDestroy(g->stream);
+  delete g;
+}
+
+}  // namespace gr

@@ -1,0 +1,82 @@
+// engine.h — internal state of a loaded graph (the opaque gr_graph).
+#pragma once
+#include <cuda_runtime.h>
+
+#include <map>
+#include <string>
+#include <utility>
+#include <vector>
+
+#include "device_common.cuh"
+#include "graphreduce.h"
+#include "host_graph.h"
+
+struct gr_graph {
+  int device = 0;
+  int num_sms = 148;
+  cudaStream_t stream = nullptr;
+  gr::HostGraph H;               // host layout (pinned payloads in streamed mode)
+  int mode = GR_MODE_RESIDENT;
+  bool off64 = false;
+  uint64_t dev_bytes = 0, pinned_bytes = 0;
+  std::vector<void *> allocs;
+
+  // topology (device)
+  void *in_off = nullptr, *out_off = nullptr;     // OffT arrays
+  uint32_t *in_src = nullptr, *out_dst = nullptr; // resident payloads
+  uint8_t *in_w = nullptr;
+  uint32_t *hub_in = nullptr, *hub_out = nullptr, *static_hubs = nullptr;
+  uint32_t n_static_hubs = 0;
+
+  // frontier-program state
+  uint32_t *val = nullptr, *stamp = nullptr;
+  uint32_t *listA[2] = {nullptr, nullptr}, *listH[2] = {nullptr, nullptr};
+  uint32_t *C_v = nullptr, *C_val = nullptr, *CH_v = nullptr, *CH_val = nullptr;
+  gr::Ctl *ctl = nullptr;
+  gr::Ctl *h_ctl = nullptr;      // pinned mirror
+  unsigned long long *trace = nullptr;
+  uint32_t trace_cap = 0;
+  int grid_frontier = 0;
+
+  // PageRank state
+  uint32_t *d_outdeg = nullptr;
+  float *inv_outdeg = nullptr, *contrib[2] = {nullptr, nullptr}, *rank = nullptr;
+  uint32_t *carry_row = nullptr, *head_row = nullptr;
+  float *carry_val = nullptr, *head_val = nullptr;
+  uint32_t pr_tiles = 0;
+  cudaGraphExec_t pr_exec = nullptr;
+  uint32_t pr_exec_iters = 0;
+  float pr_exec_d = 0.f;
+  int pr_exec_prof = -1;
+  uint32_t pr_trace_iters = 0;
+
+  // run bookkeeping
+  int last_algo = -1;
+  uint32_t last_iters = 0;
+  uint32_t epoch_next = 1;
+  uint64_t trace_rows = 0;
+  std::map<int, std::pair<cudaGraphExec_t, uint64_t>> while_exec;
+  cudaEvent_t ev_start = nullptr, ev_stop = nullptr;
+  std::vector<cudaEvent_t> prof_ev;
+
+  // streamed mode (stream.cu)
+  void *streamer = nullptr;
+};
+
+namespace gr {
+gr_status fail(gr_status s, const char *fmt, ...);
+const char *last_error();
+void clear_error();
+gr_status dev_alloc(gr_graph *g, void **p, size_t bytes);
+gr_status load_device(gr_graph *g);
+gr_status run(gr_graph *g, const gr_run_opts *o, gr_run_stats *st);
+gr_status fetch_values(gr_graph *g, void *dst, uint64_t bytes);
+gr_status fetch_trace(gr_graph *g, uint64_t *dst, uint64_t max_rows, uint64_t *rows);
+void destroy(gr_graph *g);
+// streamed mode
+gr_status stream_setup(gr_graph *g, uint64_t budget);
+gr_status run_streamed(gr_graph *g, const gr_run_opts *o, gr_run_stats *st);
+void stream_destroy(gr_graph *g);
+uint64_t resident_bytes_estimate(const HostGraph &H);
+uint64_t static_bytes_estimate(const HostGraph &H);
+}  // namespace gr

@@ -1,0 +1,532 @@
+// kernels_frontier.cuh — frontier-driven GAS superstep kernels (SSSP, CC, BFS,
+// custom programs). SURVEY.md §8(a) rows a2, a4, a5, a6, a7.
+//
+// One superstep t (§4.4, BSP):
+//   k_gather_apply  : for v in A_t: acc = (+) gatherMap(val[u], w) over in-edges
+//                     (L250-251), then apply (L252) against val[v]; changed
+//                     vertices go to the changed list C_t WITH their new value.
+//                     val[] is not written here, so every gather reads the
+//                     values of superstep t-1 (BSP, reading R5).
+//   k_activate      : commit val[u] = new for u in C_t, then FrontierActivate
+//                     (L254, L270): atomically stamp every out-neighbour x with
+//                     the epoch of t+1; the first stamper appends x to A_{t+1}.
+//                     The last CTA to finish closes the superstep (trace row,
+//                     counters, termination, CUDA-graph loop condition).
+//   k_bfs_expand    : BFS phase fusion (L276): apply (depth = t) + activate in
+//                     one pass over A_t; gather eliminated (L274).
+// Load balancing (CTA load balancing from the active list, L270, L352): a warp
+// takes 32 list entries; lanes with degree > 32 are processed warp-
+// cooperatively one at a time, lanes with degree <= 32 are packed 32 edges per
+// round (owner found by a shuffle binary search); vertices with degree >
+// kHubDegree live in a separate hub list processed one CTA per vertex.
+#pragma once
+#include "device_common.cuh"
+#include "gr/program.cuh"
+
+namespace gr {
+
+// ----------------------------------------------------------------- helpers
+template <class Prog>
+__device__ __forceinline__ typename Prog::GatherT warp_reduce_prog(typename Prog::GatherT x) {
+#pragma unroll
+  for (int o = 16; o > 0; o >>= 1) x = Prog::gatherReduce(x, __shfl_xor_sync(0xffffffffu, x, o));
+  return x;
+}
+
+template <class Prog, class OffT>
+__device__ __forceinline__ typename Prog::GatherT map_edge(const Part<OffT> &P, uint64_t e, uint32_t dval,
+                                                           const Ctx &cx) {
+  uint32_t u = ldg_nc(P.in_src + e);
+  uint32_t w = Prog::kUsesWeights ? (uint32_t)ldg_nc_u8(P.in_w + e) : 0u;
+  return Prog::gatherMap(dval, P.val[u], w, cx);
+}
+
+// Gather for up to 32 vertices held one per lane (valid, beg, deg, dval).
+// Returns the gatherReduce result of the lane's own vertex.
+template <class Prog, class OffT>
+__device__ typename Prog::GatherT gather_warp(const Part<OffT> &P, bool valid, uint64_t beg, uint32_t deg,
+                                              uint32_t dval, uint32_t *sred, const Ctx &cx) {
+  using G = typename Prog::GatherT;
+  const uint32_t lane = lane_id();
+  G acc = Prog::identity();
+  // warp-cooperative: one vertex of degree in (32, kHubDegree] at a time
+  uint32_t big = __ballot_sync(0xffffffffu, valid && deg > 32);
+  while (big) {
+    const int L = __ffs(big) - 1;
+    big &= big - 1;
+    const uint64_t b = __shfl_sync(0xffffffffu, beg, L);
+    const uint32_t d = __shfl_sync(0xffffffffu, deg, L);
+    const uint32_t dv = __shfl_sync(0xffffffffu, dval, L);
+    G r = Prog::identity();
+    uint32_t k = lane;
+    for (; k + 96 < d; k += 128) {  // 4 independent loads in flight per lane
+      G a0 = map_edge<Prog>(P, b + k, dv, cx), a1 = map_edge<Prog>(P, b + k + 32, dv, cx);
+      G a2 = map_edge<Prog>(P, b + k + 64, dv, cx), a3 = map_edge<Prog>(P, b + k + 96, dv, cx);
+      r = Prog::gatherReduce(r, Prog::gatherReduce(Prog::gatherReduce(a0, a1), Prog::gatherReduce(a2, a3)));
+    }
+    for (; k < d; k += 32) r = Prog::gatherReduce(r, map_edge<Prog>(P, b + k, dv, cx));
+    r = warp_reduce_prog<Prog>(r);
+    if ((int)lane == L) acc = r;
+  }
+  // fine-grained: pack the edges of all lanes with degree <= 32, 32 per round
+  const uint32_t sd = (valid && deg <= 32) ? deg : 0u;
+  const uint32_t incl = warp_incl_scan(sd);
+  const uint32_t excl = incl - sd;
+  const uint32_t total = __shfl_sync(0xffffffffu, incl, 31);
+  if (total == 0) return acc;
+  sred[lane] = Prog::identity();
+  __syncwarp();
+  for (uint32_t r0 = 0; r0 < total; r0 += 32) {
+    const uint32_t k = r0 + lane;
+    int o = 0;
+#pragma unroll
+    for (int step = 16; step > 0; step >>= 1) {
+      const uint32_t e = __shfl_sync(0xffffffffu, excl, o + step);
+      if (e <= k) o += step;
+    }
+    const uint64_t ob = __shfl_sync(0xffffffffu, beg, o);
+    const uint32_t oe = __shfl_sync(0xffffffffu, excl, o);
+    const uint32_t odv = __shfl_sync(0xffffffffu, dval, o);
+    G x = (k < total) ? map_edge<Prog>(P, ob + (k - oe), odv, cx) : Prog::identity();
+    // segmented inclusive scan keyed by owner lane (owners are non-decreasing)
+    const int prev_o = __shfl_up_sync(0xffffffffu, o, 1);
+    uint32_t f = (lane == 0 || prev_o != o) ? 1u : 0u;
+#pragma unroll
+    for (int d = 1; d < 32; d <<= 1) {
+      const G y = __shfl_up_sync(0xffffffffu, x, d);
+      const uint32_t g = __shfl_up_sync(0xffffffffu, f, d);
+      if (lane >= (uint32_t)d) {
+        if (!f) x = Prog::gatherReduce(y, x);
+        f |= g;
+      }
+    }
+    const int next_o = __shfl_down_sync(0xffffffffu, o, 1);
+    if (lane == 31 || next_o != o) sred[o] = Prog::gatherReduce(sred[o], x);
+    __syncwarp();
+  }
+  if (sd > 0) acc = sred[lane];
+  __syncwarp();
+  return acc;
+}
+
+// Block-wide gather of one hub vertex.
+template <class Prog, class OffT>
+__device__ typename Prog::GatherT gather_block(const Part<OffT> &P, uint64_t beg, uint32_t deg, uint32_t dval,
+                                               typename Prog::GatherT *sblk, const Ctx &cx) {
+  using G = typename Prog::GatherT;
+  G r = Prog::identity();
+  uint32_t k = threadIdx.x;
+  for (; k + 3 * kBlock < deg; k += 4 * kBlock) {
+    G a0 = map_edge<Prog>(P, beg + k, dval, cx), a1 = map_edge<Prog>(P, beg + k + kBlock, dval, cx);
+    G a2 = map_edge<Prog>(P, beg + k + 2 * kBlock, dval, cx), a3 = map_edge<Prog>(P, beg + k + 3 * kBlock, dval, cx);
+    r = Prog::gatherReduce(r, Prog::gatherReduce(Prog::gatherReduce(a0, a1), Prog::gatherReduce(a2, a3)));
+  }
+  for (; k < deg; k += kBlock) r = Prog::gatherReduce(r, map_edge<Prog>(P, beg + k, dval, cx));
+  r = warp_reduce_prog<Prog>(r);
+  if (lane_id() == 0) sblk[threadIdx.x / 32] = r;
+  __syncthreads();
+  G t = Prog::identity();
+  if (threadIdx.x == 0)
+    for (int i = 0; i < kWarpsPerBlock; i++) t = Prog::gatherReduce(t, sblk[i]);
+  __syncthreads();
+  return t;  // valid in thread 0
+}
+
+// FrontierActivate of out-edge targets x (one per lane, `act` marks real ones):
+// stamp with `epoch`; the first stamper appends x (BFS: only if still unvisited).
+template <bool kBfsFilter, class OffT>
+__device__ __forceinline__ uint32_t activate_lanes(const Part<OffT> &P, bool act, uint32_t x, uint32_t epoch,
+                                                   const uint32_t *hub_bits, WarpQueue &qA, WarpQueue &qH,
+                                                   uint32_t slot) {
+  bool newly = false;
+  if (act) {
+    const uint32_t lx = x - P.own_lo;
+    newly = atomicExch(P.stamp + lx, epoch) != epoch;
+  }
+  bool keep = newly;
+  if (kBfsFilter && keep) keep = (*(volatile uint32_t *)(P.val + x) == kInf);
+  const bool hub = keep && test_bit(hub_bits, kBfsFilter ? x : x - P.own_lo);
+  qA.push(keep && !hub, x, 0, P.listA[slot], nullptr, &P.ctl->cnt_A[slot]);
+  qH.push(hub, x, 0, P.listH[slot], nullptr, &P.ctl->cnt_H[slot]);
+  return __popc(__ballot_sync(0xffffffffu, newly));
+}
+
+// Expand the out-edges of up to 32 source vertices (one per lane).
+template <bool kBfsFilter, class OffT>
+__device__ uint32_t expand_warp(const Part<OffT> &P, bool valid, uint64_t beg, uint32_t deg, uint32_t epoch,
+                                const uint32_t *hub_bits, WarpQueue &qA, WarpQueue &qH, uint32_t slot) {
+  const uint32_t lane = lane_id();
+  uint32_t nact = 0;
+  uint32_t big = __ballot_sync(0xffffffffu, valid && deg > 32);
+  while (big) {
+    const int L = __ffs(big) - 1;
+    big &= big - 1;
+    const uint64_t b = __shfl_sync(0xffffffffu, beg, L);
+    const uint32_t d = __shfl_sync(0xffffffffu, deg, L);
+    for (uint32_t r0 = 0; r0 < d; r0 += 32) {
+      const uint32_t k = r0 + lane;
+      const bool act = k < d;
+      const uint32_t x = act ? ldg_nc(P.out_dst + b + k) : 0u;
+      nact += activate_lanes<kBfsFilter>(P, act, x, epoch, hub_bits, qA, qH, slot);
+    }
+  }
+  const uint32_t sd = (valid && deg <= 32) ? deg : 0u;
+  const uint32_t incl = warp_incl_scan(sd);
+  const uint32_t excl = incl - sd;
+  const uint32_t total = __shfl_sync(0xffffffffu, incl, 31);
+  for (uint32_t r0 = 0; r0 < total; r0 += 32) {
+    const uint32_t k = r0 + lane;
+    int o = 0;
+#pragma unroll
+    for (int step = 16; step > 0; step >>= 1) {
+      const uint32_t e = __shfl_sync(0xffffffffu, excl, o + step);
+      if (e <= k) o += step;
+    }
+    const uint64_t ob = __shfl_sync(0xffffffffu, beg, o);
+    const uint32_t oe = __shfl_sync(0xffffffffu, excl, o);
+    const bool act = k < total;
+    const uint32_t x = act ? ldg_nc(P.out_dst + ob + (k - oe)) : 0u;
+    nact += activate_lanes<kBfsFilter>(P, act, x, epoch, hub_bits, qA, qH, slot);
+  }
+  return nact;  // warp-uniform
+}
+
+// Block-wide expansion of one hub source (all warps, uniform rounds).
+template <bool kBfsFilter, class OffT>
+__device__ uint32_t expand_block(const Part<OffT> &P, uint64_t beg, uint32_t deg, uint32_t epoch,
+                                 const uint32_t *hub_bits, WarpQueue &qA, WarpQueue &qH, uint32_t slot) {
+  uint32_t nact = 0;
+  for (uint32_t r0 = 0; r0 < deg; r0 += kBlock) {
+    const uint32_t k = r0 + threadIdx.x;
+    const bool act = k < deg;
+    const uint32_t x = act ? ldg_nc(P.out_dst + beg + k) : 0u;
+    nact += activate_lanes<kBfsFilter>(P, act, x, epoch, hub_bits, qA, qH, slot);
+  }
+  return nact;  // per-warp count
+}
+
+// Last CTA of the superstep's final kernel closes superstep t.
+template <class OffT>
+__device__ void finish_superstep(const Part<OffT> &P, unsigned long long cond_handle, int use_graph) {
+  __shared__ bool s_last;
+  __syncthreads();
+  if (threadIdx.x == 0) {
+    __threadfence();
+    const uint32_t tk = atomicAdd(&P.ctl->done_blocks, 1u);
+    s_last = (tk == gridDim.x - 1);
+  }
+  __syncthreads();
+  if (!s_last || threadIdx.x != 0) return;
+  __threadfence();
+  volatile Ctl *c = P.ctl;
+  const uint32_t t = c->iter, slot = t & 1u, ns = slot ^ 1u;
+  if (t < c->trace_cap) {
+    volatile unsigned long long *row = P.trace + 4ull * t;
+    row[0] = c->cnt_act[slot];
+    row[1] = c->changed;
+    row[2] = c->gathered;
+    row[3] = c->scattered;
+  }
+  c->tot_gathered = c->tot_gathered + c->gathered;
+  c->tot_scattered = c->tot_scattered + c->scattered;
+  c->changed = 0;
+  c->gathered = 0;
+  c->scattered = 0;
+  c->cnt_C = 0;
+  c->cnt_CH = 0;
+  c->ctr_hub = 0;
+  c->ctr_hub2 = 0;
+  c->cnt_A[slot] = 0;
+  c->cnt_H[slot] = 0;
+  c->cnt_act[slot] = 0;
+  c->done_blocks = 0;
+  c->iter = t + 1;
+  const bool stop = (c->cnt_act[ns] == 0) || (c->max_iters != 0 && t + 1 >= c->max_iters);
+  c->stop = stop ? 1u : 0u;
+  __threadfence();
+  if (use_graph) cudaGraphSetConditional((cudaGraphConditionalHandle)cond_handle, stop ? 0u : 1u);
+}
+
+// ------------------------------------------------------------- kernels
+template <class Prog, class OffT>
+__global__ void __launch_bounds__(kBlock) k_gather_apply(const __grid_constant__ Part<OffT> P) {
+  using G = typename Prog::GatherT;
+  Ctl *ctl = P.ctl;
+  if (*(volatile uint32_t *)&ctl->stop) return;
+  const uint32_t t = *(volatile uint32_t *)&ctl->iter;
+  const uint32_t slot = t & 1u;
+  const Ctx cx{t, P.n, ctl->source, ctl->damping};
+  const bool implicit = ctl->implicit0 && t == 0;
+  const uint32_t nA = implicit ? P.own_n : *(volatile uint32_t *)&ctl->cnt_A[slot];
+  const uint32_t nH = *(volatile uint32_t *)&ctl->cnt_H[slot];
+  const uint32_t *LA = P.listA[slot];
+  const uint32_t *LH = P.listH[slot];
+
+  __shared__ uint32_t sq[kWarpsPerBlock][4][kQueueCap];
+  __shared__ uint32_t sred[kWarpsPerBlock][32];
+  __shared__ G sblk[kWarpsPerBlock];
+  __shared__ uint32_t s_h;
+  const uint32_t warp = threadIdx.x / 32, lane = lane_id();
+  WarpQueue qC{sq[warp][0], sq[warp][1], 0}, qCH{sq[warp][2], sq[warp][3], 0};
+  unsigned long long my_g = 0, my_c = 0;
+
+  // Phase 1: non-hub active vertices, 32 per warp, static grid stride
+  const uint32_t gw = blockIdx.x * kWarpsPerBlock + warp, nw = gridDim.x * kWarpsPerBlock;
+  for (uint32_t base = gw * 32u; base < nA; base += nw * 32u) {
+    const uint32_t idx = base + lane;
+    bool valid = idx < nA;
+    uint32_t v = 0;
+    if (valid) v = implicit ? P.own_lo + idx : LA[idx];
+    const uint32_t lv = v - P.own_lo;
+    if (valid && implicit && test_bit(P.hub_in, lv)) valid = false;  // served by the hub list
+    uint64_t beg = 0;
+    uint32_t deg = 0, cur = 0;
+    if (valid) {
+      beg = (uint64_t)P.in_off[lv];
+      deg = (uint32_t)((uint64_t)P.in_off[lv + 1] - beg);
+      cur = P.val[v];
+    }
+    const G acc = gather_warp<Prog>(P, valid, beg, deg, cur, sred[warp], cx);
+    bool changed = false;
+    uint32_t nv = cur;
+    if (valid) {
+      changed = Prog::apply(&nv, acc, cx);
+      my_g += deg;
+    }
+    const bool hubo = changed && test_bit(P.hub_out, v);
+    qC.push(changed && !hubo, v, nv, P.C_v, P.C_val, &ctl->cnt_C);
+    qCH.push(hubo, v, nv, P.CH_v, P.CH_val, &ctl->cnt_CH);
+    my_c += changed ? 1 : 0;
+  }
+  qC.flush(P.C_v, P.C_val, &ctl->cnt_C);
+  qCH.flush(P.CH_v, P.CH_val, &ctl->cnt_CH);
+
+  // Phase 2: hub vertices, one CTA each (dynamic)
+  for (;;) {
+    __syncthreads();
+    if (threadIdx.x == 0) s_h = atomicAdd(&ctl->ctr_hub, 1u);
+    __syncthreads();
+    const uint32_t h = s_h;
+    if (h >= nH) break;
+    const uint32_t v = LH[h], lv = v - P.own_lo;
+    const uint64_t beg = (uint64_t)P.in_off[lv];
+    const uint32_t deg = (uint32_t)((uint64_t)P.in_off[lv + 1] - beg);
+    const uint32_t cur = P.val[v];
+    const G acc = gather_block<Prog>(P, beg, deg, cur, sblk, cx);
+    if (threadIdx.x == 0) {
+      uint32_t nv = cur;
+      const bool changed = Prog::apply(&nv, acc, cx);
+      my_g += deg;
+      if (changed) {
+        my_c += 1;
+        if (test_bit(P.hub_out, v)) {
+          const uint32_t pos = atomicAdd(&ctl->cnt_CH, 1u);
+          P.CH_v[pos] = v; P.CH_val[pos] = nv;
+        } else {
+          const uint32_t pos = atomicAdd(&ctl->cnt_C, 1u);
+          P.C_v[pos] = v; P.C_val[pos] = nv;
+        }
+      }
+    }
+  }
+  my_g = warp_sum_u64(my_g);
+  my_c = warp_sum_u64(my_c);
+  if (lane == 0) {
+    if (my_g) atomicAdd(&ctl->gathered, my_g);
+    if (my_c) atomicAdd(&ctl->changed, my_c);
+  }
+}
+
+template <class OffT>
+__global__ void __launch_bounds__(kBlock) k_activate(const __grid_constant__ Part<OffT> P, unsigned long long cond, int use_graph) {
+  Ctl *ctl = P.ctl;
+  if (*(volatile uint32_t *)&ctl->stop) {
+    if (use_graph && blockIdx.x == 0 && threadIdx.x == 0)
+      cudaGraphSetConditional((cudaGraphConditionalHandle)cond, 0u);
+    return;
+  }
+  const uint32_t t = *(volatile uint32_t *)&ctl->iter;
+  const uint32_t ns = (t + 1) & 1u;
+  const uint32_t epoch = ctl->epoch_base + t + 1;
+  const uint32_t nC = *(volatile uint32_t *)&ctl->cnt_C;
+  const uint32_t nCH = *(volatile uint32_t *)&ctl->cnt_CH;
+
+  __shared__ uint32_t sq[kWarpsPerBlock][2][kQueueCap];
+  __shared__ uint32_t s_h;
+  const uint32_t warp = threadIdx.x / 32, lane = lane_id();
+  WarpQueue qA{sq[warp][0], nullptr, 0}, qH{sq[warp][1], nullptr, 0};
+  unsigned long long my_s = 0, my_act = 0;
+
+  const uint32_t gw = blockIdx.x * kWarpsPerBlock + warp, nw = gridDim.x * kWarpsPerBlock;
+  for (uint32_t base = gw * 32u; base < nC; base += nw * 32u) {
+    const uint32_t idx = base + lane;
+    const bool valid = idx < nC;
+    uint64_t beg = 0;
+    uint32_t deg = 0;
+    if (valid) {
+      const uint32_t u = P.C_v[idx];
+      P.val[u] = P.C_val[idx];  // BSP commit of superstep t
+      beg = (uint64_t)P.out_off[u];
+      deg = (uint32_t)((uint64_t)P.out_off[u + 1] - beg);
+      my_s += deg;
+    }
+    my_act += expand_warp<false>(P, valid, beg, deg, epoch, P.hub_in, qA, qH, ns);
+  }
+  qA.flush(P.listA[ns], nullptr, &ctl->cnt_A[ns]);
+  qH.flush(P.listH[ns], nullptr, &ctl->cnt_H[ns]);
+  for (;;) {
+    __syncthreads();
+    if (threadIdx.x == 0) s_h = atomicAdd(&ctl->ctr_hub2, 1u);
+    __syncthreads();
+    const uint32_t h = s_h;
+    if (h >= nCH) break;
+    const uint32_t u = P.CH_v[h];
+    if (threadIdx.x == 0) P.val[u] = P.CH_val[h];
+    const uint64_t beg = (uint64_t)P.out_off[u];
+    const uint32_t deg = (uint32_t)((uint64_t)P.out_off[u + 1] - beg);
+    if (threadIdx.x == 0) my_s += deg;
+    const uint32_t a = expand_block<false>(P, beg, deg, epoch, P.hub_in, qA, qH, ns);
+    if (lane == 0) my_act += a;
+  }
+  qA.flush(P.listA[ns], nullptr, &ctl->cnt_A[ns]);
+  qH.flush(P.listH[ns], nullptr, &ctl->cnt_H[ns]);
+  my_s = warp_sum_u64(my_s);
+  if (lane == 0) {
+    if (my_s) atomicAdd(&ctl->scattered, my_s);
+    if (my_act) atomicAdd(&ctl->cnt_act[ns], (uint32_t)my_act);
+  }
+  finish_superstep(P, cond, use_graph);
+}
+
+// BFS: apply (depth = t, L276) fused with FrontierActivate; no gather (L274).
+template <class OffT>
+__global__ void __launch_bounds__(kBlock) k_bfs_expand(const __grid_constant__ Part<OffT> P, unsigned long long cond, int use_graph) {
+  Ctl *ctl = P.ctl;
+  if (*(volatile uint32_t *)&ctl->stop) {
+    if (use_graph && blockIdx.x == 0 && threadIdx.x == 0)
+      cudaGraphSetConditional((cudaGraphConditionalHandle)cond, 0u);
+    return;
+  }
+  const uint32_t t = *(volatile uint32_t *)&ctl->iter;
+  const uint32_t slot = t & 1u, ns = slot ^ 1u;
+  const uint32_t epoch = ctl->epoch_base + t + 1;
+  const uint32_t nA = *(volatile uint32_t *)&ctl->cnt_A[slot];
+  const uint32_t nH = *(volatile uint32_t *)&ctl->cnt_H[slot];
+  const uint32_t *LA = P.listA[slot];
+  const uint32_t *LH = P.listH[slot];
+
+  __shared__ uint32_t sq[kWarpsPerBlock][2][kQueueCap];
+  __shared__ uint32_t s_h;
+  __shared__ bool s_changed;
+  const uint32_t warp = threadIdx.x / 32, lane = lane_id();
+  WarpQueue qA{sq[warp][0], nullptr, 0}, qH{sq[warp][1], nullptr, 0};
+  unsigned long long my_s = 0, my_c = 0, my_act = 0;
+
+  const uint32_t gw = blockIdx.x * kWarpsPerBlock + warp, nw = gridDim.x * kWarpsPerBlock;
+  for (uint32_t base = gw * 32u; base < nA; base += nw * 32u) {
+    const uint32_t idx = base + lane;
+    bool changed = false;
+    uint64_t beg = 0;
+    uint32_t deg = 0;
+    if (idx < nA) {
+      const uint32_t v = LA[idx];
+      if (P.val[v] == kInf) {  // apply: depth = iteration number
+        P.val[v] = t;
+        changed = true;
+        beg = (uint64_t)P.out_off[v];
+        deg = (uint32_t)((uint64_t)P.out_off[v + 1] - beg);
+        my_s += deg;
+        my_c += 1;
+      }
+    }
+    my_act += expand_warp<true>(P, changed, beg, deg, epoch, P.hub_out, qA, qH, ns);
+  }
+  qA.flush(P.listA[ns], nullptr, &ctl->cnt_A[ns]);
+  qH.flush(P.listH[ns], nullptr, &ctl->cnt_H[ns]);
+  for (;;) {
+    __syncthreads();
+    if (threadIdx.x == 0) s_h = atomicAdd(&ctl->ctr_hub, 1u);
+    __syncthreads();
+    const uint32_t h = s_h;
+    if (h >= nH) break;
+    const uint32_t v = LH[h];
+    if (threadIdx.x == 0) {
+      s_changed = (P.val[v] == kInf);
+      if (s_changed) { P.val[v] = t; my_c += 1; }
+    }
+    __syncthreads();
+    if (!s_changed) continue;
+    const uint64_t beg = (uint64_t)P.out_off[v];
+    const uint32_t deg = (uint32_t)((uint64_t)P.out_off[v + 1] - beg);
+    if (threadIdx.x == 0) my_s += deg;
+    const uint32_t a = expand_block<true>(P, beg, deg, epoch, P.hub_out, qA, qH, ns);
+    if (lane == 0) my_act += a;
+  }
+  qA.flush(P.listA[ns], nullptr, &ctl->cnt_A[ns]);
+  qH.flush(P.listH[ns], nullptr, &ctl->cnt_H[ns]);
+  my_s = warp_sum_u64(my_s);
+  my_c = warp_sum_u64(my_c);
+  if (lane == 0) {
+    if (my_s) atomicAdd(&ctl->scattered, my_s);
+    if (my_c) atomicAdd(&ctl->changed, my_c);
+    if (my_act) atomicAdd(&ctl->cnt_act[ns], (uint32_t)my_act);
+  }
+  finish_superstep(P, cond, use_graph);
+}
+
+// ----------------------------------------------------------- initialisation
+template <class Prog, class OffT>
+__global__ void k_init_values(const __grid_constant__ Part<OffT> P, uint32_t source) {
+  const Ctx cx{0, P.n, source, 0.f};
+  for (uint64_t v = blockIdx.x * (uint64_t)blockDim.x + threadIdx.x; v < P.n; v += (uint64_t)gridDim.x * blockDim.x)
+    P.val[v] = Prog::initValue((uint32_t)v, cx);
+}
+
+// Stage 1 (L62): the starting frontier A_0. One CTA.
+template <class Prog, class OffT>
+__global__ void __launch_bounds__(kBlock) k_init_frontier(const __grid_constant__ Part<OffT> P, uint32_t source, uint32_t n_static_hubs) {
+  Ctl *ctl = P.ctl;
+  const uint32_t epoch0 = ctl->epoch_base;
+  const bool owned = source >= P.own_lo && source < P.own_lo + P.own_n;
+  if (Prog::kInit == kInitAll) {
+    if (threadIdx.x == 0) {
+      ctl->implicit0 = 1;
+      ctl->cnt_A[0] = P.own_n;
+      ctl->cnt_H[0] = n_static_hubs;  // listH[0] pre-filled with the static in-hub list
+      ctl->cnt_act[0] = P.own_n;
+      ctl->stop = (P.own_n == 0);
+    }
+    return;
+  }
+  if (Prog::kInit == kInitSource) {
+    if (threadIdx.x == 0) {
+      if (owned) {
+        P.stamp[source - P.own_lo] = epoch0;
+        const bool hub = test_bit(Prog::kHasGather ? P.hub_in : P.hub_out,
+                                  Prog::kHasGather ? source - P.own_lo : source);
+        if (hub) { P.listH[0][0] = source; ctl->cnt_H[0] = 1; }
+        else { P.listA[0][0] = source; ctl->cnt_A[0] = 1; }
+        ctl->cnt_act[0] = 1;
+      }
+      ctl->stop = owned ? 0u : 1u;
+    }
+    return;
+  }
+  // kInitSourceChanged: the source is "changed" at initialisation; A_0 = out-neighbours.
+  __shared__ uint32_t sq[kWarpsPerBlock][2][kQueueCap];
+  const uint32_t warp = threadIdx.x / 32;
+  WarpQueue qA{sq[warp][0], nullptr, 0}, qH{sq[warp][1], nullptr, 0};
+  const uint64_t beg = (uint64_t)P.out_off[source];
+  const uint32_t deg = (uint32_t)((uint64_t)P.out_off[source + 1] - beg);
+  const uint32_t a = expand_block<false>(P, beg, deg, epoch0, P.hub_in, qA, qH, 0);
+  qA.flush(P.listA[0], nullptr, &ctl->cnt_A[0]);
+  qH.flush(P.listH[0], nullptr, &ctl->cnt_H[0]);
+  if (lane_id() == 0 && a) atomicAdd(&ctl->cnt_act[0], a);
+  __syncthreads();
+  if (threadIdx.x == 0) {
+    __threadfence();
+    ctl->stop = (*(volatile uint32_t *)&ctl->cnt_act[0] == 0) ? 1u : 0u;
+  }
+}
+
+}  // namespace gr

@@ -1,0 +1,203 @@
+// kernels_pr.cuh — PageRank superstep (reading R1): all vertices
+// active, FrontierActivate eliminated (phase elimination, §5.3).
+//
+//   gather  (L250-251): acc[v] = sum_{(u->v)} contrib[u],  contrib[u] = R_t(u)/outdeg(u)
+//   apply   (L252):     R_{t+1}(v) = (1-d)/n + d*acc[v];  contrib'[v] = R_{t+1}(v)/outdeg(v)
+//
+// Load balancing (CTA load balancing, L260; merge-path over the CSC offsets,
+// K6 in SURVEY §2.3): the merged sequence of row-ends (one per destination) and
+// in-edges is cut into tiles of exactly kPrTile items, so hubs and empty rows
+// cost the same per item. Each tile stages its offsets and the gathered source
+// contributions in shared memory (the random gathers are issued together for
+// memory-level parallelism), each thread walks kPrIpt consecutive items, and a
+// segmented scan over the threads joins rows split between threads. Rows that
+// start in an earlier tile are finished by k_pr_fixup in a fixed order, so the
+// fp32 sum order is deterministic run to run.
+#pragma once
+#include "device_common.cuh"
+
+namespace gr {
+
+constexpr int kPrThreads = 256;
+constexpr int kPrIpt = 8;
+constexpr int kPrTile = kPrThreads * kPrIpt;
+constexpr uint32_t kNoRow = 0xFFFFFFFFu;
+
+template <class OffT> struct PrArgs {
+  uint32_t n, own_lo, own_n;
+  uint64_t m_in;
+  const OffT *in_off;        // [own_n + 1]
+  const uint32_t *in_src;    // [m_in]
+  const float *inv_outdeg;   // [n]
+  const float *contrib_in;   // [n]   contributions of superstep t-1 (read side)
+  float *contrib_out;        // [n]   owned slice written
+  float *rank;               // [own_n] written on the last iteration
+  uint32_t *carry_row;       // [num_tiles]
+  float *carry_val;
+  uint32_t *head_row;
+  float *head_val;
+  float base, d;             // (1-d)/n, d
+  int last;                  // 1: write rank instead of contrib_out
+};
+
+template <class OffT>
+__device__ __forceinline__ void pr_apply_row(const PrArgs<OffT> &a, uint32_t lrow, float acc) {
+  const float R = a.base + a.d * acc;
+  const uint32_t v = a.own_lo + lrow;
+  if (a.last) a.rank[lrow] = R;
+  else a.contrib_out[v] = R * __ldg(a.inv_outdeg + v);
+}
+
+// Merge-path search over (row ends, edge indices) for diagonal `diag`.
+template <class OffT>
+__device__ __forceinline__ uint32_t merge_path_rows(const OffT *in_off, uint32_t rows, uint64_t nnz, uint64_t diag) {
+  uint64_t lo = diag > nnz ? diag - nnz : 0;
+  uint64_t hi = diag < rows ? diag : rows;
+  while (lo < hi) {
+    const uint64_t p = (lo + hi) >> 1;
+    if ((uint64_t)in_off[p + 1] <= diag - p - 1) lo = p + 1;
+    else hi = p;
+  }
+  return (uint32_t)lo;
+}
+
+template <class OffT>
+__global__ void __launch_bounds__(kPrThreads, 4) k_pr_gather_apply(const __grid_constant__ PrArgs<OffT> a) {
+  __shared__ uint32_t s_end[kPrTile + 1];   // row ends, local to the tile's first edge
+  __shared__ float s_val[kPrTile];          // contrib[src] of the tile's edges
+  __shared__ float s_tot[kPrTile];          // per-row partial totals
+  __shared__ uint32_t s_crow[kPrThreads];
+  __shared__ float s_cval[kPrThreads];
+  __shared__ uint32_t s_wkey_first[kPrThreads / 32], s_wkey_last[kPrThreads / 32];
+  __shared__ float s_wval_last[kPrThreads / 32];
+  __shared__ uint64_t s_i0, s_i1, s_j0, s_j1, s_rowstart0;
+
+  const uint32_t tid = threadIdx.x, lane = tid & 31, warp = tid >> 5;
+  const uint64_t total = (uint64_t)a.own_n + a.m_in;
+  const uint64_t d0 = (uint64_t)blockIdx.x * kPrTile;
+  const uint64_t d1 = d0 + kPrTile < total ? d0 + kPrTile : total;
+  if (tid < 2) {
+    const uint64_t diag = tid == 0 ? d0 : d1;
+    const uint32_t i = merge_path_rows(a.in_off, a.own_n, a.m_in, diag);
+    if (tid == 0) { s_i0 = i; s_j0 = diag - i; s_rowstart0 = (uint64_t)a.in_off[i]; }
+    else { s_i1 = i; s_j1 = diag - i; }
+  }
+  __syncthreads();
+  const uint64_t i0 = s_i0, j0 = s_j0;
+  const uint32_t ni = (uint32_t)(s_i1 - i0), nj = (uint32_t)(s_j1 - j0);
+
+  // stage row ends (local) and gathered contributions
+  for (uint32_t k = tid; k <= ni; k += kPrThreads) {
+    const uint64_t r = i0 + k;
+    uint64_t e = r < a.own_n ? (uint64_t)a.in_off[r + 1] - j0 : (uint64_t)nj;
+    s_end[k] = (uint32_t)(e < nj ? e : nj);
+  }
+  {
+    uint32_t src[kPrIpt];
+#pragma unroll
+    for (int q = 0; q < kPrIpt; q++) {
+      const uint32_t k = tid + q * kPrThreads;
+      src[q] = k < nj ? ldg_nc(a.in_src + j0 + k) : 0u;
+    }
+    float v[kPrIpt];
+#pragma unroll
+    for (int q = 0; q < kPrIpt; q++) {
+      const uint32_t k = tid + q * kPrThreads;
+      v[q] = k < nj ? __ldg(a.contrib_in + src[q]) : 0.f;
+    }
+#pragma unroll
+    for (int q = 0; q < kPrIpt; q++) {
+      const uint32_t k = tid + q * kPrThreads;
+      if (k < nj) s_val[k] = v[q];
+    }
+  }
+  __syncthreads();
+
+  // per-thread merge walk over kPrIpt items
+  const uint32_t tile_items = ni + nj;
+  const uint32_t dt = min(tid * kPrIpt, tile_items);
+  uint32_t lo = dt > nj ? dt - nj : 0, hi = dt < ni ? dt : ni;
+  while (lo < hi) {
+    const uint32_t p = (lo + hi) >> 1;
+    if (s_end[p] <= dt - p - 1) lo = p + 1;
+    else hi = p;
+  }
+  uint32_t i = lo, j = dt - lo;
+  float run = 0.f;
+  const uint32_t dend = min(dt + kPrIpt, tile_items);
+#pragma unroll
+  for (int q = 0; q < kPrIpt; q++) {
+    if (dt + q < dend) {
+      if (j < s_end[i]) { run += s_val[j]; ++j; }
+      else { s_tot[i] = run; run = 0.f; ++i; }
+    }
+  }
+  s_crow[tid] = i;
+
+  // segmented inclusive scan of the thread carries (keys non-decreasing)
+  float x = run;
+#pragma unroll
+  for (int o = 1; o < 32; o <<= 1) {
+    const float y = __shfl_up_sync(0xffffffffu, x, o);
+    const uint32_t ky = __shfl_up_sync(0xffffffffu, i, o);
+    if (lane >= (uint32_t)o && ky == i) x += y;
+  }
+  if (lane == 0) s_wkey_first[warp] = i;
+  if (lane == 31) { s_wkey_last[warp] = i; s_wval_last[warp] = x; }
+  __syncthreads();
+  if (i == s_wkey_first[warp]) {
+    for (int w = (int)warp - 1; w >= 0; w--) {
+      if (s_wkey_last[w] != i) break;
+      x += s_wval_last[w];
+      if (s_wkey_first[w] != i) break;
+    }
+  }
+  s_cval[tid] = x;
+  __syncthreads();
+  // the last thread of each carry run adds it to the row finished by the next thread
+  const bool run_end = (tid == kPrThreads - 1) || (s_crow[tid + 1] != i);
+  if (run_end && i < ni) s_tot[i] += x;
+  __syncthreads();
+
+  // apply the rows whose end lies in this tile (coalesced over destinations)
+  const bool head = (ni > 0) && (s_rowstart0 < j0);  // row i0 began in an earlier tile
+  for (uint32_t k = tid; k < ni; k += kPrThreads) {
+    if (k == 0 && head) continue;
+    pr_apply_row(a, (uint32_t)(i0 + k), s_tot[k]);
+  }
+  if (tid == 0) {
+    a.head_row[blockIdx.x] = head ? (uint32_t)i0 : kNoRow;
+    a.head_val[blockIdx.x] = head ? s_tot[0] : 0.f;
+    const uint64_t i1 = s_i1;
+    a.carry_row[blockIdx.x] = i1 < a.own_n ? (uint32_t)i1 : kNoRow;
+    a.carry_val[blockIdx.x] = s_cval[kPrThreads - 1];
+  }
+}
+
+// Rows spanning tiles: head partial + the carries of the preceding tiles, in order.
+template <class OffT>
+__global__ void k_pr_fixup(const __grid_constant__ PrArgs<OffT> a, uint32_t num_tiles) {
+  for (uint32_t c = blockIdx.x * blockDim.x + threadIdx.x; c < num_tiles; c += gridDim.x * blockDim.x) {
+    const uint32_t row = a.head_row[c];
+    if (row == kNoRow) continue;
+    float acc = a.head_val[c];
+    for (int64_t p = (int64_t)c - 1; p >= 0 && a.carry_row[p] == row; p--) acc += a.carry_val[p];
+    pr_apply_row(a, row, acc);
+  }
+}
+
+// contrib_0[u] = R_0(u) / outdeg(u) with R_0 = 1/n (reading R3); dangling -> 0 (R2).
+__global__ void k_pr_init(uint32_t n, const float *inv_outdeg, float *contrib) {
+  const float r0 = 1.0f / (float)n;
+  for (uint64_t v = blockIdx.x * (uint64_t)blockDim.x + threadIdx.x; v < n; v += (uint64_t)gridDim.x * blockDim.x)
+    contrib[v] = r0 * inv_outdeg[v];
+}
+
+__global__ void k_inv_outdeg(uint32_t n, const uint32_t *outdeg, float *inv) {
+  for (uint64_t v = blockIdx.x * (uint64_t)blockDim.x + threadIdx.x; v < n; v += (uint64_t)gridDim.x * blockDim.x) {
+    const uint32_t d = outdeg[v];
+    inv[v] = d ? 1.0f / (float)d : 0.f;
+  }
+}
+
+}  // namespace gr

@@ -1,0 +1,165 @@
+"""GPU parity: the CUDA path through the C ABI vs the oracle.
+
+BFS / SSSP / CC bit-exact, frontier traces identical; PageRank within
+max|dR| <= 1e-6 and L1 <= 1e-5 of the fp64 oracle (BASELINE.json north_star),
+plus the internal gates of SURVEY §8(c): relative error <= 1e-4 where
+R >= 1/n and |sum R - sum R_oracle| <= 1e-5.
+"""
+import numpy as np
+import pytest
+
+import grgen
+import oracle
+import paper_conf_sc_senguptasas15_b200 as gr
+
+pytestmark = pytest.mark.gpu
+
+PR_MAX, PR_L1 = 1e-6, 1e-5
+
+
+def check_pr(got, ref, n):
+    got = got.astype(np.float64)
+    err = np.abs(got - ref)
+    assert err.max() <= PR_MAX, err.max()
+    assert err.sum() <= PR_L1, err.sum()
+    big = ref >= 1.0 / n
+    if big.any():
+        assert (err[big] / ref[big]).max() <= 1e-4
+    assert abs(got.sum() - ref.sum()) <= 1e-5
+
+
+def compare(n, src, dst, w, algo, source=0, max_iters=0, loops=("device", "host"), **load):
+    og = oracle.OracleGraph(n, src, dst, w)
+    ref, rtr, rit = og.run(algo, source=source, max_iters=max_iters)
+    og.close()
+    with gr.GraphReduce(n, src, dst, w, **load) as G:
+        for loop in loops:
+            st = G.run(algo, source=source, max_iters=max_iters, loop=loop)
+            got = G.values(algo)
+            tr = G.trace()
+            assert st["iterations"] == rit, (loop, st["iterations"], rit)
+            if algo == "pagerank":
+                check_pr(got, ref, n)
+            else:
+                np.testing.assert_array_equal(got, ref)
+                np.testing.assert_array_equal(tr, rtr)
+                assert st["edges_gathered"] == int(rtr[:, 2].sum())
+                assert st["edges_scattered"] == int(rtr[:, 3].sum())
+    return st
+
+
+def rand_graph(seed, n, m, sym=False, wmax=64):
+    rng = np.random.default_rng(seed)
+    src = rng.integers(0, n, m).astype(np.uint32)
+    dst = rng.integers(0, n, m).astype(np.uint32)
+    w = rng.integers(1, wmax + 1, m).astype(np.uint32)
+    if sym:
+        src, dst, w = np.concatenate([src, dst]), np.concatenate([dst, src]), np.concatenate([w, w])
+    return src, dst, w
+
+
+@pytest.mark.parametrize("algo", ["bfs", "sssp", "cc", "pagerank"])
+@pytest.mark.parametrize("seed,n,m", [(1, 1, 0), (2, 7, 20), (3, 200, 900), (4, 5000, 3000), (5, 3001, 40000)])
+def test_random_graphs(algo, seed, n, m):
+    src, dst, w = rand_graph(seed, n, m, sym=(algo == "cc"))
+    compare(n, src, dst, w, algo, source=seed % n)
+
+
+def hub_graph(k=5000, extra=3000, seed=9):
+    """Star hubs above the CTA-per-vertex threshold plus random edges (both directions)."""
+    rng = np.random.default_rng(seed)
+    n = k + 10
+    s = [np.zeros(k, np.uint32), np.arange(1, k + 1, dtype=np.uint32)]
+    d = [np.arange(1, k + 1, dtype=np.uint32), np.zeros(k, np.uint32)]
+    s.append(np.full(2000, 3, np.uint32))
+    d.append(rng.integers(0, n, 2000).astype(np.uint32))
+    s.append(rng.integers(0, n, extra).astype(np.uint32))
+    d.append(rng.integers(0, n, extra).astype(np.uint32))
+    src, dst = np.concatenate(s), np.concatenate(d)
+    src, dst = np.concatenate([src, dst]), np.concatenate([dst, src])
+    w = rng.integers(1, 65, len(src)).astype(np.uint32)
+    return n, src, dst, w
+
+
+@pytest.mark.parametrize("algo", ["bfs", "sssp", "cc", "pagerank"])
+def test_hubs(algo):
+    n, src, dst, w = hub_graph()
+    for s in (0, 5, n - 1):
+        compare(n, src, dst, w, algo, source=s)
+
+
+@pytest.mark.parametrize("cfg", [1, 2, 3, 4])
+def test_reduced_configs(cfg):
+    g, run = grgen.config(cfg, reduced=True)
+    w = g.get("w")
+    if run["algo"] == "sssp" and w is None:
+        w = grgen.weights(g.m, 1, 64, seed=cfg)
+    compare(g.n, g.src, g.dst, w, run["algo"], source=run.get("source", 0), max_iters=run.get("max_iters", 0))
+
+
+def test_sssp_unit_weights_equals_bfs_and_rmat_weights():
+    g = grgen.rmat(14, 16, seed=7)
+    w = np.ones(g.m, np.uint32)
+    with gr.GraphReduce(g.n, g.src, g.dst, w) as G:
+        G.run("bfs", source=0)
+        b = G.values()
+        G.run("sssp", source=0)
+        s = G.values()
+    np.testing.assert_array_equal(b, s)
+    w = grgen.weights(g.m, 1, 64, seed=11)
+    compare(g.n, g.src, g.dst, w, "sssp", source=0)
+
+
+def test_repeated_runs_and_epochs():
+    g = grgen.rmat(13, 8, seed=3)
+    w = grgen.weights(g.m, 1, 64, seed=1)
+    og = oracle.OracleGraph(g.n, g.src, g.dst, w)
+    with gr.GraphReduce(g.n, g.src, g.dst, w) as G:
+        for algo, s in [("bfs", 0), ("bfs", 17), ("sssp", 5), ("cc", 0), ("bfs", 0), ("pagerank", 0), ("sssp", 0)]:
+            G.run(algo, source=s)
+            ref, rtr, _ = og.run(algo, source=s)
+            if algo == "pagerank":
+                check_pr(G.values(algo), ref, g.n)
+            else:
+                np.testing.assert_array_equal(G.values(), ref)
+                np.testing.assert_array_equal(G.trace(), rtr)
+    og.close()
+
+
+def test_pr_iteration_counts_and_closed_form_cycle():
+    n = 1000
+    src = np.arange(n, dtype=np.uint32)
+    dst = ((src + 1) % n).astype(np.uint32)
+    with gr.GraphReduce(n, src, dst) as G:
+        for it in (1, 2, 30, 50):
+            st = G.run("pagerank", max_iters=it)
+            assert st["iterations"] == it
+            np.testing.assert_allclose(G.values("pagerank"), 1.0 / n, rtol=1e-6)
+
+
+def test_max_iters_truncates_frontier_programs():
+    g = grgen.grid_road(60, 60, seed=3)
+    compare(g.n, g.src, g.dst, g.w, "sssp", source=0, max_iters=7)
+    compare(g.n, g.src, g.dst, g.w, "bfs", source=0, max_iters=3)
+
+
+def test_errors_through_abi():
+    src = np.array([0, 1, 2], np.uint32)
+    dst = np.array([1, 2, 0], np.uint32)
+    with gr.GraphReduce(3, src, dst) as G:
+        with pytest.raises(gr.GrError) as ei:
+            G.run("sssp", source=0)  # no weights
+        assert ei.value.status == gr.GR_EINVAL
+        with pytest.raises(gr.GrError) as ei:
+            gr.gr_fetch_vertex_values(G.h)
+        assert ei.value.status == gr.GR_ESTATE
+        with pytest.raises(gr.GrError):
+            G.run("bfs", source=3)
+        with pytest.raises(gr.GrError):
+            G.run("pagerank", damping=1.5)
+        G.run("bfs", source=0)
+        with pytest.raises(gr.GrError):
+            gr.gr_fetch_vertex_values(G.h, np.empty(2, np.uint32))
+        with pytest.raises(gr.GrError) as ei:
+            G.run("custom", custom_id=77)
+        assert ei.value.status == gr.GR_EUNSUPPORTED
