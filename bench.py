@@ -187,11 +187,14 @@ def main():
     torch.cuda.set_device(local_rank)
     import paper_conf_sc_senguptasas15_b200 as gr
 
+    t0 = time.perf_counter()
     g, w, run = make_graph(args.config)
+    print(f"[bench] generated {g.name}: n={g.n} m={g.m} in {time.perf_counter() - t0:.1f}s", file=sys.stderr)
     algo = run["algo"]
     kw = dict(source=run.get("source", 0), max_iters=run.get("max_iters", 0), damping=run.get("damping", 0.85))
     G = gr.GraphReduce(g.n, g.src, g.dst, w, device=local_rank, mode="resident")
     info = G.info()
+    print(f"[bench] loaded in {time.perf_counter() - t0:.1f}s total: {info}", file=sys.stderr)
     stream = torch.cuda.current_stream()
     sp = stream.cuda_stream
     for _ in range(max(3, args.warmup)):
@@ -259,7 +262,7 @@ def main():
         e2e_vals.append(edges * world / dt / 1e9)
     h2d = int(8 * m + (m if w is not None else 0))  # CSC + CSR payloads (+weights) per load
     h2d += 8 * (n + 1) * 2 // (2 if not info["offsets_64bit"] else 1)
-    e2e = {"value": float(np.median(e2e_vals)), "unit": "GTEPS", "h2d_bytes_per_step": h2d,
+    e2e = {"value": float(np.median(e2e_vals)) if e2e_vals else None, "unit": "GTEPS", "h2d_bytes_per_step": h2d,
            "d2h_bytes_per_step": 4 * n,
            "what": "gr_graph_load(host COO: shard build + H2D) + gr_run + gr_fetch_vertex_values, wall clock"}
 

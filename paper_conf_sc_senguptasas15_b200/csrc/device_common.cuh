@@ -11,7 +11,8 @@ constexpr uint32_t kInf = 0xFFFFFFFFu;
 constexpr int kWarp = 32;
 constexpr int kBlock = 256;              // threads per CTA for the frontier kernels
 constexpr int kWarpsPerBlock = kBlock / kWarp;
-constexpr uint32_t kHubDegree = 1024;    // > this degree: one CTA per vertex (K6 CTA load balancing)
+constexpr uint32_t kHubDegree = 1024;    // > this degree: hub, split into chunks (K6 CTA load balancing)
+constexpr uint32_t kChunk = 4096;        // edges per hub chunk (one CTA each)
 constexpr int kQueueCap = 128;           // per-warp staging entries before one global append
 
 // Device control block of one run (superstep bookkeeping).
@@ -26,6 +27,8 @@ struct Ctl {
   uint32_t cnt_act[2];    // |A_t| (distinct activated vertices; BFS lists are filtered)
   uint32_t cnt_C;         // non-hub changed entries
   uint32_t cnt_CH;        // hub changed entries
+  uint32_t cnt_K[2];      // chunk-list length of the A_t hubs
+  uint32_t cnt_KC;        // chunk-list length of the changed hubs
   uint32_t ctr_hub;       // dynamic hub work counter (gather / BFS)
   uint32_t ctr_hub2;      // dynamic hub work counter (activate)
   uint32_t done_blocks;   // last-block ticket
@@ -37,7 +40,26 @@ struct Ctl {
   unsigned long long gathered;   // sum indeg(A_t)
   unsigned long long scattered;  // sum outdeg(C_t)
   unsigned long long tot_gathered, tot_scattered;
+  unsigned long long prof;               // 1: kernels stamp %globaltimer
+  unsigned long long kstart[2], kend[2]; // per-kernel span of the current superstep (ns)
+  unsigned long long kns[2];             // accumulated kernel ns: [0] gather+apply, [1] activate / BFS expand
 };
+
+__device__ __forceinline__ unsigned long long gtimer() {
+  unsigned long long t;
+  asm volatile("mov.u64 %0, %%globaltimer;" : "=l"(t));
+  return t;
+}
+// device-side kernel timing inside CUDA-graph loops (first block start .. last block end)
+__device__ __forceinline__ void prof_begin(Ctl *c, int k) {
+  if (c->prof && threadIdx.x == 0) atomicMin(&c->kstart[k], gtimer());
+}
+__device__ __forceinline__ void prof_end(Ctl *c, int k) {
+  if (c->prof) {
+    __syncthreads();
+    if (threadIdx.x == 0) atomicMax(&c->kend[k], gtimer());
+  }
+}
 
 // Device view of one owner partition (single GPU = one partition owning V).
 template <class OffT> struct Part {
@@ -56,6 +78,9 @@ template <class OffT> struct Part {
   uint32_t *listH[2];     // hub A lists
   uint32_t *C_v, *C_val;  // changed list (non-hub)
   uint32_t *CH_v, *CH_val;// changed list (activation hubs)
+  uint32_t *chkA_h[2], *chkA_c[2]; // A_t hub chunks: (position in listH, chunk index)
+  uint32_t *chkC_h, *chkC_c;       // changed-hub chunks: (position in CH list, chunk index)
+  uint32_t *hub_acc, *hub_done;    // per A-hub position: chunk-combined gather result, chunks done
   Ctl *ctl;
   unsigned long long *trace; // [trace_cap][4]
 };

@@ -70,28 +70,6 @@ template <class T> static gr_status upload(gr_graph *g, T **dst, const T *src, s
   return GR_OK;
 }
 
-// --------------------------------------------------------------- Part views
-template <class OffT> Part<OffT> make_part(gr_graph *g) {
-  Part<OffT> P{};
-  P.n = (uint32_t)g->H.n;
-  P.own_lo = (uint32_t)g->H.own_lo;
-  P.own_n = (uint32_t)g->H.own_n();
-  P.in_off = (const OffT *)g->in_off;
-  P.in_src = g->in_src;
-  P.in_w = g->in_w;
-  P.out_off = (const OffT *)g->out_off;
-  P.out_dst = g->out_dst;
-  P.hub_in = g->hub_in;
-  P.hub_out = g->hub_out;
-  P.val = g->val;
-  P.stamp = g->stamp;
-  for (int i = 0; i < 2; i++) { P.listA[i] = g->listA[i]; P.listH[i] = g->listH[i]; }
-  P.C_v = g->C_v; P.C_val = g->C_val; P.CH_v = g->CH_v; P.CH_val = g->CH_val;
-  P.ctl = g->ctl;
-  P.trace = g->trace;
-  return P;
-}
-
 template <class OffT> static gr_status upload_offsets(gr_graph *g, void **dst, const std::vector<uint64_t> &off) {
   if (sizeof(OffT) == 8) return upload(g, (uint64_t **)dst, off.data(), off.size());
   std::vector<uint32_t> o32(off.size());
@@ -130,6 +108,36 @@ gr_status load_device(gr_graph *g) {
   if ((s = upload(g, &g->hub_out, hb_out.data(), hb_out.size())) != GR_OK) return s;
   g->n_static_hubs = (uint32_t)hubs.size();
   if ((s = upload(g, &g->static_hubs, hubs.data(), hubs.size())) != GR_OK) return s;
+  // hub chunk capacities: every hub appears at most once per list
+  uint64_t hubs_in = 0, chunks_in = 0, hubs_out = 0, chunks_out = 0;
+  std::vector<uint32_t> sch_h, sch_c;
+  for (uint64_t i = 0; i < own_n; i++) {
+    const uint64_t d = H.in_off[i + 1] - H.in_off[i];
+    if (d > kHubDegree) {
+      const uint64_t nch = (d + kChunk - 1) / kChunk;
+      for (uint64_t c = 0; c < nch; c++) { sch_h.push_back((uint32_t)hubs_in); sch_c.push_back((uint32_t)c); }
+      hubs_in++;
+      chunks_in += nch;
+    }
+  }
+  for (uint64_t u = 0; u < n; u++) {
+    const uint64_t d = H.out_off[u + 1] - H.out_off[u];
+    if (d > kHubDegree) { hubs_out++; chunks_out += (d + kChunk - 1) / kChunk; }
+  }
+  g->n_static_chunks = (uint32_t)sch_h.size();
+  if ((s = upload(g, &g->static_chk_h, sch_h.data(), sch_h.size())) != GR_OK) return s;
+  if ((s = upload(g, &g->static_chk_c, sch_c.data(), sch_c.size())) != GR_OK) return s;
+  const uint64_t chk_cap = std::max<uint64_t>(std::max(chunks_in, chunks_out), 1);
+  for (int i = 0; i < 2; i++) {
+    if ((s = dev_alloc(g, (void **)&g->chkA_h[i], 4 * chk_cap)) != GR_OK) return s;
+    if ((s = dev_alloc(g, (void **)&g->chkA_c[i], 4 * chk_cap)) != GR_OK) return s;
+  }
+  if ((s = dev_alloc(g, (void **)&g->chkC_h, 4 * std::max<uint64_t>(chunks_out, 1))) != GR_OK) return s;
+  if ((s = dev_alloc(g, (void **)&g->chkC_c, 4 * std::max<uint64_t>(chunks_out, 1))) != GR_OK) return s;
+  g->hub_cap = (uint32_t)std::max<uint64_t>(std::max(hubs_in, hubs_out), 1);
+  if ((s = dev_alloc(g, (void **)&g->hub_acc, 4ull * g->hub_cap)) != GR_OK) return s;
+  if ((s = dev_alloc(g, (void **)&g->hub_done, 4ull * g->hub_cap)) != GR_OK) return s;
+  CK(cudaMemset(g->hub_done, 0, 4ull * g->hub_cap));
 
   // edge payloads: resident copies (streamed mode keeps them in pinned host memory)
   if (g->mode == GR_MODE_RESIDENT) {
@@ -170,6 +178,16 @@ gr_status load_device(gr_graph *g) {
   if ((s = dev_alloc(g, (void **)&g->carry_val, tb)) != GR_OK) return s;
   if ((s = dev_alloc(g, (void **)&g->head_row, tb)) != GR_OK) return s;
   if ((s = dev_alloc(g, (void **)&g->head_val, tb)) != GR_OK) return s;
+  if (g->mode == GR_MODE_RESIDENT) {
+    if ((s = dev_alloc(g, (void **)&g->tile_row, 4ull * (g->pr_tiles + 1))) != GR_OK) return s;
+    if (g->off64)
+      k_pr_tiles<uint64_t><<<(g->pr_tiles + 256) / 256, 256, 0, g->stream>>>(
+          (const uint64_t *)g->in_off, 0, (uint32_t)own_n, mi, g->pr_tiles, g->tile_row);
+    else
+      k_pr_tiles<uint32_t><<<(g->pr_tiles + 256) / 256, 256, 0, g->stream>>>(
+          (const uint32_t *)g->in_off, 0, (uint32_t)own_n, mi, g->pr_tiles, g->tile_row);
+    CK(cudaGetLastError());
+  }
   CK(cudaStreamSynchronize(g->stream));
 
   // occupancy-derived persistent grid: a multiple of the SM count
@@ -245,15 +263,23 @@ static gr_status run_frontier(gr_graph *g, const gr_run_opts *o, cudaStream_t s,
   h.trace_cap = g->trace_cap;
   h.source = o->source;
   h.damping = o->damping;
+  h.prof = o->profile ? 1 : 0;
+  h.kstart[0] = h.kstart[1] = ~0ull;
   CK(cudaMemcpyAsync(g->ctl, &h, sizeof h, cudaMemcpyHostToDevice, s));
   k_init_values<Prog, OffT><<<g->num_sms * 4, 256, 0, s>>>(P, o->source);
-  launches++;
-  if (Prog::kInit == kInitAll && g->n_static_hubs)
+  k_fill_u32<<<std::min<uint32_t>((g->hub_cap + 255) / 256, 1024), 256, 0, s>>>(g->hub_acc, Prog::identity_host(),
+                                                                                 g->hub_cap);
+  CK(cudaMemsetAsync(g->hub_done, 0, 4ull * g->hub_cap, s));
+  launches += 2;
+  if (Prog::kInit == kInitAll && g->n_static_hubs) {
     CK(cudaMemcpyAsync(g->listH[0], g->static_hubs, 4ull * g->n_static_hubs, cudaMemcpyDeviceToDevice, s));
-  k_init_frontier<Prog, OffT><<<1, kBlock, 0, s>>>(P, o->source, g->n_static_hubs);
+    CK(cudaMemcpyAsync(g->chkA_h[0], g->static_chk_h, 4ull * g->n_static_chunks, cudaMemcpyDeviceToDevice, s));
+    CK(cudaMemcpyAsync(g->chkA_c[0], g->static_chk_c, 4ull * g->n_static_chunks, cudaMemcpyDeviceToDevice, s));
+  }
+  k_init_frontier<Prog, OffT><<<1, kBlock, 0, s>>>(P, o->source, g->n_static_hubs, g->n_static_chunks);
   launches++;
   CK(cudaGetLastError());
-  const bool use_graph = (o->loop != GR_LOOP_HOST) && !o->profile;
+  const bool use_graph = (o->loop != GR_LOOP_HOST);
   if (use_graph) {
     cudaGraphExec_t ex;
     uint64_t per = 0;
@@ -264,23 +290,19 @@ static gr_status run_frontier(gr_graph *g, const gr_run_opts *o, cudaStream_t s,
     CK(cudaStreamSynchronize(s));
     launches += per * std::max<uint32_t>(g->h_ctl->iter, 1);
   } else {
-    cudaEvent_t e0 = g->prof_ev[0], e1 = g->prof_ev[1];
     for (;;) {
-      if (o->profile) CK(cudaEventRecord(e0, s));
       launch_body<Prog, OffT>(g, s, 0, 0, &launches);
-      if (o->profile) CK(cudaEventRecord(e1, s));
       CK(cudaGetLastError());
       CK(cudaMemcpyAsync(g->h_ctl, g->ctl, sizeof(Ctl), cudaMemcpyDeviceToHost, s));
       CK(cudaStreamSynchronize(s));
-      if (o->profile) {
-        float ms = 0;
-        CK(cudaEventElapsedTime(&ms, e0, e1));
-        st->kernel_ms[Prog::kHasGather ? 0 : 1] += ms;
-      }
       if (g->h_ctl->stop) break;
     }
   }
   const Ctl &c = *g->h_ctl;
+  if (o->profile) {
+    st->kernel_ms[0] += c.kns[0] * 1e-6;
+    st->kernel_ms[1] += c.kns[1] * 1e-6;
+  }
   st->iterations = c.iter;
   st->edges_gathered = c.tot_gathered;
   st->edges_scattered = c.tot_scattered;
@@ -316,6 +338,7 @@ template <class OffT> static PrArgs<OffT> pr_args(gr_graph *g, uint32_t t, uint3
   a.carry_val = g->carry_val;
   a.head_row = g->head_row;
   a.head_val = g->head_val;
+  a.tile_row = g->tile_row;
   a.base = (1.0f - d) / (float)g->H.n;
   a.d = d;
   a.last = (t + 1 == iters) ? 1 : 0;
@@ -344,34 +367,40 @@ static gr_status run_pagerank(gr_graph *g, const gr_run_opts *o, cudaStream_t s,
       g->prof_ev.push_back(e);
     }
   }
-  // one CUDA graph per (iters, damping, profile): 2 launches per superstep
-  if (!g->pr_exec || g->pr_exec_iters != iters || g->pr_exec_d != d || g->pr_exec_prof != prof) {
-    if (g->pr_exec) { cudaGraphExecDestroy(g->pr_exec); g->pr_exec = nullptr; }
-    cudaStream_t cs;
-    CK(cudaStreamCreateWithFlags(&cs, cudaStreamNonBlocking));
-    CK(cudaStreamBeginCapture(cs, cudaStreamCaptureModeThreadLocal));
-    k_pr_init<<<g->num_sms * 4, 256, 0, cs>>>((uint32_t)g->H.n, g->inv_outdeg, g->contrib[0]);
-    for (uint32_t t = 0; t < iters; t++)
-      pr_launch_iter<OffT>(g, cs, t, iters, d, prof ? g->prof_ev[2 + 2 * t] : nullptr,
-                           prof ? g->prof_ev[3 + 2 * t] : nullptr);
-    cudaGraph_t graph;
-    cudaError_t e = cudaStreamEndCapture(cs, &graph);
-    cudaStreamDestroy(cs);
-    if (e != cudaSuccess) return fail(GR_ECUDA, "PageRank graph capture failed: %s", cudaGetErrorString(e));
-    CK(cudaGraphInstantiate(&g->pr_exec, graph, 0));
-    CK(cudaGraphDestroy(graph));
-    g->pr_exec_iters = iters;
-    g->pr_exec_d = d;
-    g->pr_exec_prof = prof;
-  }
-  CK(cudaGraphLaunch(g->pr_exec, s));
-  CK(cudaStreamSynchronize(s));
   if (prof) {
+    // direct launches with a CUDA event pair around every gather launch (events
+    // recorded inside a captured graph cannot be timed); the host enqueues all
+    // 2*iters launches without waiting, so the device runs them back to back
+    k_pr_init<<<g->num_sms * 4, 256, 0, s>>>((uint32_t)g->H.n, g->inv_outdeg, g->contrib[0]);
+    for (uint32_t t = 0; t < iters; t++)
+      pr_launch_iter<OffT>(g, s, t, iters, d, g->prof_ev[2 + 2 * t], g->prof_ev[3 + 2 * t]);
+    CK(cudaGetLastError());
+    CK(cudaStreamSynchronize(s));
     for (uint32_t t = 0; t < iters; t++) {
       float ms = 0;
       CK(cudaEventElapsedTime(&ms, g->prof_ev[2 + 2 * t], g->prof_ev[3 + 2 * t]));
       st->kernel_ms[0] += ms;
     }
+  } else {
+    // one CUDA graph per (iters, damping): 2 launches per superstep
+    if (!g->pr_exec || g->pr_exec_iters != iters || g->pr_exec_d != d) {
+      if (g->pr_exec) { cudaGraphExecDestroy(g->pr_exec); g->pr_exec = nullptr; }
+      cudaStream_t cs;
+      CK(cudaStreamCreateWithFlags(&cs, cudaStreamNonBlocking));
+      CK(cudaStreamBeginCapture(cs, cudaStreamCaptureModeThreadLocal));
+      k_pr_init<<<g->num_sms * 4, 256, 0, cs>>>((uint32_t)g->H.n, g->inv_outdeg, g->contrib[0]);
+      for (uint32_t t = 0; t < iters; t++) pr_launch_iter<OffT>(g, cs, t, iters, d, nullptr, nullptr);
+      cudaGraph_t graph;
+      cudaError_t e = cudaStreamEndCapture(cs, &graph);
+      cudaStreamDestroy(cs);
+      if (e != cudaSuccess) return fail(GR_ECUDA, "PageRank graph capture failed: %s", cudaGetErrorString(e));
+      CK(cudaGraphInstantiate(&g->pr_exec, graph, 0));
+      CK(cudaGraphDestroy(graph));
+      g->pr_exec_iters = iters;
+      g->pr_exec_d = d;
+    }
+    CK(cudaGraphLaunch(g->pr_exec, s));
+    CK(cudaStreamSynchronize(s));
   }
   st->iterations = iters;
   st->edges_gathered = (uint64_t)iters * g->H.m_in;

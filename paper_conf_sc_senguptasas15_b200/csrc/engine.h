@@ -27,6 +27,12 @@ struct gr_graph {
   uint8_t *in_w = nullptr;
   uint32_t *hub_in = nullptr, *hub_out = nullptr, *static_hubs = nullptr;
   uint32_t n_static_hubs = 0;
+  // hub chunk lists (kChunk edges per CTA work item)
+  uint32_t *chkA_h[2] = {nullptr, nullptr}, *chkA_c[2] = {nullptr, nullptr};
+  uint32_t *chkC_h = nullptr, *chkC_c = nullptr;
+  uint32_t *hub_acc = nullptr, *hub_done = nullptr;
+  uint32_t *static_chk_h = nullptr, *static_chk_c = nullptr;
+  uint32_t n_static_chunks = 0, hub_cap = 0;
 
   // frontier-program state
   uint32_t *val = nullptr, *stamp = nullptr;
@@ -44,6 +50,7 @@ struct gr_graph {
   uint32_t *carry_row = nullptr, *head_row = nullptr;
   float *carry_val = nullptr, *head_val = nullptr;
   uint32_t pr_tiles = 0;
+  uint32_t *tile_row = nullptr;  // merge-path tile starts (resident: [pr_tiles+1]; streamed: per shard)
   cudaGraphExec_t pr_exec = nullptr;
   uint32_t pr_exec_iters = 0;
   float pr_exec_d = 0.f;
@@ -64,6 +71,31 @@ struct gr_graph {
 };
 
 namespace gr {
+// --------------------------------------------------------------- Part views
+template <class OffT> inline Part<OffT> make_part(gr_graph *g) {
+  Part<OffT> P{};
+  P.n = (uint32_t)g->H.n;
+  P.own_lo = (uint32_t)g->H.own_lo;
+  P.own_n = (uint32_t)g->H.own_n();
+  P.in_off = (const OffT *)g->in_off;
+  P.in_src = g->in_src;
+  P.in_w = g->in_w;
+  P.out_off = (const OffT *)g->out_off;
+  P.out_dst = g->out_dst;
+  P.hub_in = g->hub_in;
+  P.hub_out = g->hub_out;
+  P.val = g->val;
+  P.stamp = g->stamp;
+  for (int i = 0; i < 2; i++) { P.listA[i] = g->listA[i]; P.listH[i] = g->listH[i]; }
+  P.C_v = g->C_v; P.C_val = g->C_val; P.CH_v = g->CH_v; P.CH_val = g->CH_val;
+  for (int i = 0; i < 2; i++) { P.chkA_h[i] = g->chkA_h[i]; P.chkA_c[i] = g->chkA_c[i]; }
+  P.chkC_h = g->chkC_h; P.chkC_c = g->chkC_c;
+  P.hub_acc = g->hub_acc; P.hub_done = g->hub_done;
+  P.ctl = g->ctl;
+  P.trace = g->trace;
+  return P;
+}
+
 gr_status fail(gr_status s, const char *fmt, ...);
 const char *last_error();
 void clear_error();

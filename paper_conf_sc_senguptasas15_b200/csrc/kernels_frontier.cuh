@@ -132,11 +132,49 @@ __device__ typename Prog::GatherT gather_block(const Part<OffT> &P, uint64_t beg
   return t;  // valid in thread 0
 }
 
+__device__ __forceinline__ uint32_t chunk_len(uint64_t deg, uint32_t ci) {
+  const uint64_t rest = deg - (uint64_t)ci * kChunk;
+  return (uint32_t)(rest < kChunk ? rest : kChunk);
+}
+
+// Append a hub to the A list of `slot` together with its edge chunks
+// (by out-degree for BFS, whose A-phase is the expansion; else by in-degree).
+template <bool kByOut, class OffT>
+__device__ void append_hub_A(const Part<OffT> &P, uint32_t x, uint32_t slot) {
+  Ctl *c = P.ctl;
+  const uint32_t pos = atomicAdd(&c->cnt_H[slot], 1u);
+  P.listH[slot][pos] = x;
+  const uint64_t deg = kByOut ? (uint64_t)P.out_off[x + 1] - (uint64_t)P.out_off[x]
+                              : (uint64_t)P.in_off[x - P.own_lo + 1] - (uint64_t)P.in_off[x - P.own_lo];
+  const uint32_t nch = (uint32_t)((deg + kChunk - 1) / kChunk);
+  const uint32_t kb = atomicAdd(&c->cnt_K[slot], nch);
+  for (uint32_t i = 0; i < nch; i++) {
+    P.chkA_h[slot][kb + i] = pos;
+    P.chkA_c[slot][kb + i] = i;
+  }
+}
+
+// Append a changed hub (by activation out-degree) with its out-edge chunks.
+template <class OffT>
+__device__ void append_hub_C(const Part<OffT> &P, uint32_t v, uint32_t nv) {
+  Ctl *c = P.ctl;
+  const uint32_t pos = atomicAdd(&c->cnt_CH, 1u);
+  P.CH_v[pos] = v;
+  P.CH_val[pos] = nv;
+  const uint64_t deg = (uint64_t)P.out_off[v + 1] - (uint64_t)P.out_off[v];
+  const uint32_t nch = (uint32_t)((deg + kChunk - 1) / kChunk);
+  const uint32_t kb = atomicAdd(&c->cnt_KC, nch);
+  for (uint32_t i = 0; i < nch; i++) {
+    P.chkC_h[kb + i] = pos;
+    P.chkC_c[kb + i] = i;
+  }
+}
+
 // FrontierActivate of out-edge targets x (one per lane, `act` marks real ones):
 // stamp with `epoch`; the first stamper appends x (BFS: only if still unvisited).
 template <bool kBfsFilter, class OffT>
 __device__ __forceinline__ uint32_t activate_lanes(const Part<OffT> &P, bool act, uint32_t x, uint32_t epoch,
-                                                   const uint32_t *hub_bits, WarpQueue &qA, WarpQueue &qH,
+                                                   const uint32_t *hub_bits, WarpQueue &qA,
                                                    uint32_t slot) {
   bool newly = false;
   if (act) {
@@ -147,14 +185,14 @@ __device__ __forceinline__ uint32_t activate_lanes(const Part<OffT> &P, bool act
   if (kBfsFilter && keep) keep = (*(volatile uint32_t *)(P.val + x) == kInf);
   const bool hub = keep && test_bit(hub_bits, kBfsFilter ? x : x - P.own_lo);
   qA.push(keep && !hub, x, 0, P.listA[slot], nullptr, &P.ctl->cnt_A[slot]);
-  qH.push(hub, x, 0, P.listH[slot], nullptr, &P.ctl->cnt_H[slot]);
+  if (hub) append_hub_A<kBfsFilter>(P, x, slot);
   return __popc(__ballot_sync(0xffffffffu, newly));
 }
 
 // Expand the out-edges of up to 32 source vertices (one per lane).
 template <bool kBfsFilter, class OffT>
 __device__ uint32_t expand_warp(const Part<OffT> &P, bool valid, uint64_t beg, uint32_t deg, uint32_t epoch,
-                                const uint32_t *hub_bits, WarpQueue &qA, WarpQueue &qH, uint32_t slot) {
+                                const uint32_t *hub_bits, WarpQueue &qA, uint32_t slot) {
   const uint32_t lane = lane_id();
   uint32_t nact = 0;
   uint32_t big = __ballot_sync(0xffffffffu, valid && deg > 32);
@@ -167,7 +205,7 @@ __device__ uint32_t expand_warp(const Part<OffT> &P, bool valid, uint64_t beg, u
       const uint32_t k = r0 + lane;
       const bool act = k < d;
       const uint32_t x = act ? ldg_nc(P.out_dst + b + k) : 0u;
-      nact += activate_lanes<kBfsFilter>(P, act, x, epoch, hub_bits, qA, qH, slot);
+      nact += activate_lanes<kBfsFilter>(P, act, x, epoch, hub_bits, qA, slot);
     }
   }
   const uint32_t sd = (valid && deg <= 32) ? deg : 0u;
@@ -186,7 +224,7 @@ __device__ uint32_t expand_warp(const Part<OffT> &P, bool valid, uint64_t beg, u
     const uint32_t oe = __shfl_sync(0xffffffffu, excl, o);
     const bool act = k < total;
     const uint32_t x = act ? ldg_nc(P.out_dst + ob + (k - oe)) : 0u;
-    nact += activate_lanes<kBfsFilter>(P, act, x, epoch, hub_bits, qA, qH, slot);
+    nact += activate_lanes<kBfsFilter>(P, act, x, epoch, hub_bits, qA, slot);
   }
   return nact;  // warp-uniform
 }
@@ -194,13 +232,13 @@ __device__ uint32_t expand_warp(const Part<OffT> &P, bool valid, uint64_t beg, u
 // Block-wide expansion of one hub source (all warps, uniform rounds).
 template <bool kBfsFilter, class OffT>
 __device__ uint32_t expand_block(const Part<OffT> &P, uint64_t beg, uint32_t deg, uint32_t epoch,
-                                 const uint32_t *hub_bits, WarpQueue &qA, WarpQueue &qH, uint32_t slot) {
+                                 const uint32_t *hub_bits, WarpQueue &qA, uint32_t slot) {
   uint32_t nact = 0;
   for (uint32_t r0 = 0; r0 < deg; r0 += kBlock) {
     const uint32_t k = r0 + threadIdx.x;
     const bool act = k < deg;
     const uint32_t x = act ? ldg_nc(P.out_dst + beg + k) : 0u;
-    nact += activate_lanes<kBfsFilter>(P, act, x, epoch, hub_bits, qA, qH, slot);
+    nact += activate_lanes<kBfsFilter>(P, act, x, epoch, hub_bits, qA, slot);
   }
   return nact;  // per-warp count
 }
@@ -227,6 +265,13 @@ __device__ void finish_superstep(const Part<OffT> &P, unsigned long long cond_ha
     row[2] = c->gathered;
     row[3] = c->scattered;
   }
+  if (c->prof) {
+    for (int k = 0; k < 2; k++) {
+      if (c->kend[k] > c->kstart[k]) c->kns[k] = c->kns[k] + (c->kend[k] - c->kstart[k]);
+      c->kstart[k] = ~0ull;
+      c->kend[k] = 0;
+    }
+  }
   c->tot_gathered = c->tot_gathered + c->gathered;
   c->tot_scattered = c->tot_scattered + c->scattered;
   c->changed = 0;
@@ -234,6 +279,8 @@ __device__ void finish_superstep(const Part<OffT> &P, unsigned long long cond_ha
   c->scattered = 0;
   c->cnt_C = 0;
   c->cnt_CH = 0;
+  c->cnt_KC = 0;
+  c->cnt_K[slot] = 0;
   c->ctr_hub = 0;
   c->ctr_hub2 = 0;
   c->cnt_A[slot] = 0;
@@ -258,16 +305,17 @@ __global__ void __launch_bounds__(kBlock) k_gather_apply(const __grid_constant__
   const Ctx cx{t, P.n, ctl->source, ctl->damping};
   const bool implicit = ctl->implicit0 && t == 0;
   const uint32_t nA = implicit ? P.own_n : *(volatile uint32_t *)&ctl->cnt_A[slot];
-  const uint32_t nH = *(volatile uint32_t *)&ctl->cnt_H[slot];
+  const uint32_t nK = *(volatile uint32_t *)&ctl->cnt_K[slot];
   const uint32_t *LA = P.listA[slot];
   const uint32_t *LH = P.listH[slot];
+  prof_begin(ctl, 0);
 
-  __shared__ uint32_t sq[kWarpsPerBlock][4][kQueueCap];
+  __shared__ uint32_t sq[kWarpsPerBlock][2][kQueueCap];
   __shared__ uint32_t sred[kWarpsPerBlock][32];
   __shared__ G sblk[kWarpsPerBlock];
   __shared__ uint32_t s_h;
   const uint32_t warp = threadIdx.x / 32, lane = lane_id();
-  WarpQueue qC{sq[warp][0], sq[warp][1], 0}, qCH{sq[warp][2], sq[warp][3], 0};
+  WarpQueue qC{sq[warp][0], sq[warp][1], 0};
   unsigned long long my_g = 0, my_c = 0;
 
   // Phase 1: non-hub active vertices, 32 per warp, static grid stride
@@ -278,7 +326,7 @@ __global__ void __launch_bounds__(kBlock) k_gather_apply(const __grid_constant__
     uint32_t v = 0;
     if (valid) v = implicit ? P.own_lo + idx : LA[idx];
     const uint32_t lv = v - P.own_lo;
-    if (valid && implicit && test_bit(P.hub_in, lv)) valid = false;  // served by the hub list
+    if (valid && implicit && test_bit(P.hub_in, lv)) valid = false;  // served by the hub chunks
     uint64_t beg = 0;
     uint32_t deg = 0, cur = 0;
     if (valid) {
@@ -294,37 +342,53 @@ __global__ void __launch_bounds__(kBlock) k_gather_apply(const __grid_constant__
       my_g += deg;
     }
     const bool hubo = changed && test_bit(P.hub_out, v);
+    if (hubo) append_hub_C(P, v, nv);
     qC.push(changed && !hubo, v, nv, P.C_v, P.C_val, &ctl->cnt_C);
-    qCH.push(hubo, v, nv, P.CH_v, P.CH_val, &ctl->cnt_CH);
     my_c += changed ? 1 : 0;
   }
   qC.flush(P.C_v, P.C_val, &ctl->cnt_C);
-  qCH.flush(P.CH_v, P.CH_val, &ctl->cnt_CH);
 
-  // Phase 2: hub vertices, one CTA each (dynamic)
-  for (;;) {
+  // Phase 2: hub chunks (kChunk in-edges each), dynamic over CTAs. Chunk results
+  // combine with Prog::atomicGather (exact for min); the last chunk applies.
+  for (; nK;) {
     __syncthreads();
     if (threadIdx.x == 0) s_h = atomicAdd(&ctl->ctr_hub, 1u);
     __syncthreads();
-    const uint32_t h = s_h;
-    if (h >= nH) break;
-    const uint32_t v = LH[h], lv = v - P.own_lo;
+    const uint32_t i = s_h;
+    if (i >= nK) break;
+    const uint32_t hp = P.chkA_h[slot][i], ci = P.chkA_c[slot][i];
+    const uint32_t v = LH[hp], lv = v - P.own_lo;
     const uint64_t beg = (uint64_t)P.in_off[lv];
-    const uint32_t deg = (uint32_t)((uint64_t)P.in_off[lv + 1] - beg);
+    const uint64_t deg = (uint64_t)P.in_off[lv + 1] - beg;
+    const uint64_t b = beg + (uint64_t)ci * kChunk;
+    const uint32_t len = chunk_len(deg, ci);
     const uint32_t cur = P.val[v];
-    const G acc = gather_block<Prog>(P, beg, deg, cur, sblk, cx);
+    const G r = gather_block<Prog>(P, b, len, cur, sblk, cx);
     if (threadIdx.x == 0) {
-      uint32_t nv = cur;
-      const bool changed = Prog::apply(&nv, acc, cx);
-      my_g += deg;
-      if (changed) {
-        my_c += 1;
-        if (test_bit(P.hub_out, v)) {
-          const uint32_t pos = atomicAdd(&ctl->cnt_CH, 1u);
-          P.CH_v[pos] = v; P.CH_val[pos] = nv;
-        } else {
-          const uint32_t pos = atomicAdd(&ctl->cnt_C, 1u);
-          P.C_v[pos] = v; P.C_val[pos] = nv;
+      const uint32_t nch = (uint32_t)((deg + kChunk - 1) / kChunk);
+      if (ci == 0) my_g += deg;
+      bool fin = (nch == 1);
+      G acc = r;
+      if (!fin) {
+        Prog::atomicGather(P.hub_acc + hp, r);
+        __threadfence();
+        fin = (atomicAdd(P.hub_done + hp, 1u) == nch - 1);
+        if (fin) {
+          __threadfence();
+          acc = atomicExch(P.hub_acc + hp, Prog::identity());
+          P.hub_done[hp] = 0;
+        }
+      }
+      if (fin) {
+        uint32_t nv = cur;
+        if (Prog::apply(&nv, acc, cx)) {
+          my_c += 1;
+          if (test_bit(P.hub_out, v)) append_hub_C(P, v, nv);
+          else {
+            const uint32_t pos = atomicAdd(&ctl->cnt_C, 1u);
+            P.C_v[pos] = v;
+            P.C_val[pos] = nv;
+          }
         }
       }
     }
@@ -335,10 +399,12 @@ __global__ void __launch_bounds__(kBlock) k_gather_apply(const __grid_constant__
     if (my_g) atomicAdd(&ctl->gathered, my_g);
     if (my_c) atomicAdd(&ctl->changed, my_c);
   }
+  prof_end(ctl, 0);
 }
 
 template <class OffT>
-__global__ void __launch_bounds__(kBlock) k_activate(const __grid_constant__ Part<OffT> P, unsigned long long cond, int use_graph) {
+__global__ void __launch_bounds__(kBlock) k_activate(const __grid_constant__ Part<OffT> P, unsigned long long cond,
+                                                     int use_graph) {
   Ctl *ctl = P.ctl;
   if (*(volatile uint32_t *)&ctl->stop) {
     if (use_graph && blockIdx.x == 0 && threadIdx.x == 0)
@@ -349,12 +415,13 @@ __global__ void __launch_bounds__(kBlock) k_activate(const __grid_constant__ Par
   const uint32_t ns = (t + 1) & 1u;
   const uint32_t epoch = ctl->epoch_base + t + 1;
   const uint32_t nC = *(volatile uint32_t *)&ctl->cnt_C;
-  const uint32_t nCH = *(volatile uint32_t *)&ctl->cnt_CH;
+  const uint32_t nKC = *(volatile uint32_t *)&ctl->cnt_KC;
+  prof_begin(ctl, 1);
 
-  __shared__ uint32_t sq[kWarpsPerBlock][2][kQueueCap];
+  __shared__ uint32_t sq[kWarpsPerBlock][kQueueCap];
   __shared__ uint32_t s_h;
   const uint32_t warp = threadIdx.x / 32, lane = lane_id();
-  WarpQueue qA{sq[warp][0], nullptr, 0}, qH{sq[warp][1], nullptr, 0};
+  WarpQueue qA{sq[warp], nullptr, 0};
   unsigned long long my_s = 0, my_act = 0;
 
   const uint32_t gw = blockIdx.x * kWarpsPerBlock + warp, nw = gridDim.x * kWarpsPerBlock;
@@ -370,37 +437,41 @@ __global__ void __launch_bounds__(kBlock) k_activate(const __grid_constant__ Par
       deg = (uint32_t)((uint64_t)P.out_off[u + 1] - beg);
       my_s += deg;
     }
-    my_act += expand_warp<false>(P, valid, beg, deg, epoch, P.hub_in, qA, qH, ns);
+    my_act += expand_warp<false>(P, valid, beg, deg, epoch, P.hub_in, qA, ns);
   }
-  qA.flush(P.listA[ns], nullptr, &ctl->cnt_A[ns]);
-  qH.flush(P.listH[ns], nullptr, &ctl->cnt_H[ns]);
-  for (;;) {
+  // changed hubs: out-edge chunks, dynamic over CTAs
+  for (; nKC;) {
     __syncthreads();
     if (threadIdx.x == 0) s_h = atomicAdd(&ctl->ctr_hub2, 1u);
     __syncthreads();
-    const uint32_t h = s_h;
-    if (h >= nCH) break;
-    const uint32_t u = P.CH_v[h];
-    if (threadIdx.x == 0) P.val[u] = P.CH_val[h];
+    const uint32_t i = s_h;
+    if (i >= nKC) break;
+    const uint32_t hp = P.chkC_h[i], ci = P.chkC_c[i];
+    const uint32_t u = P.CH_v[hp];
     const uint64_t beg = (uint64_t)P.out_off[u];
-    const uint32_t deg = (uint32_t)((uint64_t)P.out_off[u + 1] - beg);
-    if (threadIdx.x == 0) my_s += deg;
-    const uint32_t a = expand_block<false>(P, beg, deg, epoch, P.hub_in, qA, qH, ns);
+    const uint64_t deg = (uint64_t)P.out_off[u + 1] - beg;
+    if (threadIdx.x == 0 && ci == 0) {
+      P.val[u] = P.CH_val[hp];
+      my_s += deg;
+    }
+    const uint32_t len = chunk_len(deg, ci);
+    const uint32_t a = expand_block<false>(P, beg + (uint64_t)ci * kChunk, len, epoch, P.hub_in, qA, ns);
     if (lane == 0) my_act += a;
   }
   qA.flush(P.listA[ns], nullptr, &ctl->cnt_A[ns]);
-  qH.flush(P.listH[ns], nullptr, &ctl->cnt_H[ns]);
   my_s = warp_sum_u64(my_s);
   if (lane == 0) {
     if (my_s) atomicAdd(&ctl->scattered, my_s);
     if (my_act) atomicAdd(&ctl->cnt_act[ns], (uint32_t)my_act);
   }
+  prof_end(ctl, 1);
   finish_superstep(P, cond, use_graph);
 }
 
 // BFS: apply (depth = t, L276) fused with FrontierActivate; no gather (L274).
 template <class OffT>
-__global__ void __launch_bounds__(kBlock) k_bfs_expand(const __grid_constant__ Part<OffT> P, unsigned long long cond, int use_graph) {
+__global__ void __launch_bounds__(kBlock) k_bfs_expand(const __grid_constant__ Part<OffT> P, unsigned long long cond,
+                                                       int use_graph) {
   Ctl *ctl = P.ctl;
   if (*(volatile uint32_t *)&ctl->stop) {
     if (use_graph && blockIdx.x == 0 && threadIdx.x == 0)
@@ -411,15 +482,16 @@ __global__ void __launch_bounds__(kBlock) k_bfs_expand(const __grid_constant__ P
   const uint32_t slot = t & 1u, ns = slot ^ 1u;
   const uint32_t epoch = ctl->epoch_base + t + 1;
   const uint32_t nA = *(volatile uint32_t *)&ctl->cnt_A[slot];
-  const uint32_t nH = *(volatile uint32_t *)&ctl->cnt_H[slot];
+  const uint32_t nK = *(volatile uint32_t *)&ctl->cnt_K[slot];
   const uint32_t *LA = P.listA[slot];
   const uint32_t *LH = P.listH[slot];
+  prof_begin(ctl, 1);
 
-  __shared__ uint32_t sq[kWarpsPerBlock][2][kQueueCap];
+  __shared__ uint32_t sq[kWarpsPerBlock][kQueueCap];
   __shared__ uint32_t s_h;
   __shared__ bool s_changed;
   const uint32_t warp = threadIdx.x / 32, lane = lane_id();
-  WarpQueue qA{sq[warp][0], nullptr, 0}, qH{sq[warp][1], nullptr, 0};
+  WarpQueue qA{sq[warp], nullptr, 0};
   unsigned long long my_s = 0, my_c = 0, my_act = 0;
 
   const uint32_t gw = blockIdx.x * kWarpsPerBlock + warp, nw = gridDim.x * kWarpsPerBlock;
@@ -439,31 +511,36 @@ __global__ void __launch_bounds__(kBlock) k_bfs_expand(const __grid_constant__ P
         my_c += 1;
       }
     }
-    my_act += expand_warp<true>(P, changed, beg, deg, epoch, P.hub_out, qA, qH, ns);
+    my_act += expand_warp<true>(P, changed, beg, deg, epoch, P.hub_out, qA, ns);
   }
-  qA.flush(P.listA[ns], nullptr, &ctl->cnt_A[ns]);
-  qH.flush(P.listH[ns], nullptr, &ctl->cnt_H[ns]);
-  for (;;) {
+  // hub members of A_t (by out-degree): chunk 0 applies; every chunk expands if
+  // the hub's depth is unset or was set in this superstep
+  for (; nK;) {
     __syncthreads();
     if (threadIdx.x == 0) s_h = atomicAdd(&ctl->ctr_hub, 1u);
     __syncthreads();
-    const uint32_t h = s_h;
-    if (h >= nH) break;
-    const uint32_t v = LH[h];
+    const uint32_t i = s_h;
+    if (i >= nK) break;
+    const uint32_t hp = P.chkA_h[slot][i], ci = P.chkA_c[slot][i];
+    const uint32_t v = LH[hp];
+    const uint64_t beg = (uint64_t)P.out_off[v];
+    const uint64_t deg = (uint64_t)P.out_off[v + 1] - beg;
     if (threadIdx.x == 0) {
-      s_changed = (P.val[v] == kInf);
-      if (s_changed) { P.val[v] = t; my_c += 1; }
+      if (ci == 0 && P.val[v] == kInf) {
+        P.val[v] = t;
+        my_c += 1;
+        my_s += deg;
+      }
+      const uint32_t d = *(volatile uint32_t *)(P.val + v);
+      s_changed = (d == kInf || d == t);
     }
     __syncthreads();
     if (!s_changed) continue;
-    const uint64_t beg = (uint64_t)P.out_off[v];
-    const uint32_t deg = (uint32_t)((uint64_t)P.out_off[v + 1] - beg);
-    if (threadIdx.x == 0) my_s += deg;
-    const uint32_t a = expand_block<true>(P, beg, deg, epoch, P.hub_out, qA, qH, ns);
+    const uint32_t len = chunk_len(deg, ci);
+    const uint32_t a = expand_block<true>(P, beg + (uint64_t)ci * kChunk, len, epoch, P.hub_out, qA, ns);
     if (lane == 0) my_act += a;
   }
   qA.flush(P.listA[ns], nullptr, &ctl->cnt_A[ns]);
-  qH.flush(P.listH[ns], nullptr, &ctl->cnt_H[ns]);
   my_s = warp_sum_u64(my_s);
   my_c = warp_sum_u64(my_c);
   if (lane == 0) {
@@ -471,6 +548,7 @@ __global__ void __launch_bounds__(kBlock) k_bfs_expand(const __grid_constant__ P
     if (my_c) atomicAdd(&ctl->changed, my_c);
     if (my_act) atomicAdd(&ctl->cnt_act[ns], (uint32_t)my_act);
   }
+  prof_end(ctl, 1);
   finish_superstep(P, cond, use_graph);
 }
 
@@ -482,9 +560,16 @@ __global__ void k_init_values(const __grid_constant__ Part<OffT> P, uint32_t sou
     P.val[v] = Prog::initValue((uint32_t)v, cx);
 }
 
-// Stage 1 (L62): the starting frontier A_0. One CTA.
+static __global__ void k_fill_u32(uint32_t *p, uint32_t value, uint64_t count) {
+  for (uint64_t i = blockIdx.x * (uint64_t)blockDim.x + threadIdx.x; i < count; i += (uint64_t)gridDim.x * blockDim.x)
+    p[i] = value;
+}
+
+// Stage 1 (L62): the starting frontier A_0. One CTA. kInitAll expects listH[0]
+// and the chunk list of slot 0 pre-filled with the static in-hub list.
 template <class Prog, class OffT>
-__global__ void __launch_bounds__(kBlock) k_init_frontier(const __grid_constant__ Part<OffT> P, uint32_t source, uint32_t n_static_hubs) {
+__global__ void __launch_bounds__(kBlock) k_init_frontier(const __grid_constant__ Part<OffT> P, uint32_t source,
+                                                          uint32_t n_static_hubs, uint32_t n_static_chunks) {
   Ctl *ctl = P.ctl;
   const uint32_t epoch0 = ctl->epoch_base;
   const bool owned = source >= P.own_lo && source < P.own_lo + P.own_n;
@@ -492,7 +577,8 @@ __global__ void __launch_bounds__(kBlock) k_init_frontier(const __grid_constant_
     if (threadIdx.x == 0) {
       ctl->implicit0 = 1;
       ctl->cnt_A[0] = P.own_n;
-      ctl->cnt_H[0] = n_static_hubs;  // listH[0] pre-filled with the static in-hub list
+      ctl->cnt_H[0] = n_static_hubs;
+      ctl->cnt_K[0] = n_static_chunks;
       ctl->cnt_act[0] = P.own_n;
       ctl->stop = (P.own_n == 0);
     }
@@ -504,7 +590,7 @@ __global__ void __launch_bounds__(kBlock) k_init_frontier(const __grid_constant_
         P.stamp[source - P.own_lo] = epoch0;
         const bool hub = test_bit(Prog::kHasGather ? P.hub_in : P.hub_out,
                                   Prog::kHasGather ? source - P.own_lo : source);
-        if (hub) { P.listH[0][0] = source; ctl->cnt_H[0] = 1; }
+        if (hub) append_hub_A<!Prog::kHasGather>(P, source, 0);
         else { P.listA[0][0] = source; ctl->cnt_A[0] = 1; }
         ctl->cnt_act[0] = 1;
       }
@@ -513,14 +599,13 @@ __global__ void __launch_bounds__(kBlock) k_init_frontier(const __grid_constant_
     return;
   }
   // kInitSourceChanged: the source is "changed" at initialisation; A_0 = out-neighbours.
-  __shared__ uint32_t sq[kWarpsPerBlock][2][kQueueCap];
+  __shared__ uint32_t sq[kWarpsPerBlock][kQueueCap];
   const uint32_t warp = threadIdx.x / 32;
-  WarpQueue qA{sq[warp][0], nullptr, 0}, qH{sq[warp][1], nullptr, 0};
+  WarpQueue qA{sq[warp], nullptr, 0};
   const uint64_t beg = (uint64_t)P.out_off[source];
   const uint32_t deg = (uint32_t)((uint64_t)P.out_off[source + 1] - beg);
-  const uint32_t a = expand_block<false>(P, beg, deg, epoch0, P.hub_in, qA, qH, 0);
+  const uint32_t a = expand_block<false>(P, beg, deg, epoch0, P.hub_in, qA, 0);
   qA.flush(P.listA[0], nullptr, &ctl->cnt_A[0]);
-  qH.flush(P.listH[0], nullptr, &ctl->cnt_H[0]);
   if (lane_id() == 0 && a) atomicAdd(&ctl->cnt_act[0], a);
   __syncthreads();
   if (threadIdx.x == 0) {

@@ -22,11 +22,18 @@ constexpr int kPrThreads = 256;
 constexpr int kPrIpt = 8;
 constexpr int kPrTile = kPrThreads * kPrIpt;
 constexpr uint32_t kNoRow = 0xFFFFFFFFu;
+constexpr int kPrPad = kPrTile / kPrIpt;  // one pad word per kPrIpt items
+
+// Shared-memory index with one pad word per 8 items: thread t walks items
+// [8t, 8t+8), so unpadded reads of lanes t and t+4 would hit the same bank
+// (8-way conflicts); with the pad, lane t reads bank (9t + q) mod 32 (distinct).
+__device__ __forceinline__ uint32_t pr_pad(uint32_t i) { return i + (i >> 3); }
 
 template <class OffT> struct PrArgs {
-  uint32_t n, own_lo, own_n;
-  uint64_t m_in;
-  const OffT *in_off;        // [own_n + 1]
+  uint32_t n, own_lo, own_n; // own_lo/own_n: first global row and row count of this launch
+  uint64_t m_in;             // edges of this launch
+  uint64_t e_base;           // global edge index of in_src[0] (streamed shard slot; 0 resident)
+  const OffT *in_off;        // [own_n + 1] global edge offsets of this launch's rows
   const uint32_t *in_src;    // [m_in]
   const float *inv_outdeg;   // [n]
   const float *contrib_in;   // [n]   contributions of superstep t-1 (read side)
@@ -36,6 +43,7 @@ template <class OffT> struct PrArgs {
   float *carry_val;
   uint32_t *head_row;
   float *head_val;
+  const uint32_t *tile_row;  // [num_tiles + 1] merge-path row coordinate of each tile start (precomputed)
   float base, d;             // (1-d)/n, d
   int last;                  // 1: write rank instead of contrib_out
 };
@@ -50,22 +58,23 @@ __device__ __forceinline__ void pr_apply_row(const PrArgs<OffT> &a, uint32_t lro
 
 // Merge-path search over (row ends, edge indices) for diagonal `diag`.
 template <class OffT>
-__device__ __forceinline__ uint32_t merge_path_rows(const OffT *in_off, uint32_t rows, uint64_t nnz, uint64_t diag) {
+__device__ __forceinline__ uint32_t merge_path_rows(const OffT *in_off, uint64_t e_base, uint32_t rows, uint64_t nnz,
+                                                    uint64_t diag) {
   uint64_t lo = diag > nnz ? diag - nnz : 0;
   uint64_t hi = diag < rows ? diag : rows;
   while (lo < hi) {
     const uint64_t p = (lo + hi) >> 1;
-    if ((uint64_t)in_off[p + 1] <= diag - p - 1) lo = p + 1;
+    if ((uint64_t)in_off[p + 1] - e_base <= diag - p - 1) lo = p + 1;
     else hi = p;
   }
   return (uint32_t)lo;
 }
 
 template <class OffT>
-__global__ void __launch_bounds__(kPrThreads, 4) k_pr_gather_apply(const __grid_constant__ PrArgs<OffT> a) {
-  __shared__ uint32_t s_end[kPrTile + 1];   // row ends, local to the tile's first edge
-  __shared__ float s_val[kPrTile];          // contrib[src] of the tile's edges
-  __shared__ float s_tot[kPrTile];          // per-row partial totals
+__global__ void __launch_bounds__(kPrThreads, 6) k_pr_gather_apply(const __grid_constant__ PrArgs<OffT> a) {
+  __shared__ uint32_t s_end[kPrTile + 1 + kPrPad];  // row ends, local to the tile's first edge (padded)
+  __shared__ float s_val[kPrTile + kPrPad];         // contrib[src] of the tile's edges (padded)
+  __shared__ float s_tot[kPrTile + kPrPad];         // per-row partial totals (padded)
   __shared__ uint32_t s_crow[kPrThreads];
   __shared__ float s_cval[kPrThreads];
   __shared__ uint32_t s_wkey_first[kPrThreads / 32], s_wkey_last[kPrThreads / 32];
@@ -78,8 +87,8 @@ __global__ void __launch_bounds__(kPrThreads, 4) k_pr_gather_apply(const __grid_
   const uint64_t d1 = d0 + kPrTile < total ? d0 + kPrTile : total;
   if (tid < 2) {
     const uint64_t diag = tid == 0 ? d0 : d1;
-    const uint32_t i = merge_path_rows(a.in_off, a.own_n, a.m_in, diag);
-    if (tid == 0) { s_i0 = i; s_j0 = diag - i; s_rowstart0 = (uint64_t)a.in_off[i]; }
+    const uint32_t i = __ldg(a.tile_row + blockIdx.x + tid);  // == merge_path_rows(diag), precomputed
+    if (tid == 0) { s_i0 = i; s_j0 = diag - i; s_rowstart0 = (uint64_t)a.in_off[i] - a.e_base; }
     else { s_i1 = i; s_j1 = diag - i; }
   }
   __syncthreads();
@@ -89,8 +98,8 @@ __global__ void __launch_bounds__(kPrThreads, 4) k_pr_gather_apply(const __grid_
   // stage row ends (local) and gathered contributions
   for (uint32_t k = tid; k <= ni; k += kPrThreads) {
     const uint64_t r = i0 + k;
-    uint64_t e = r < a.own_n ? (uint64_t)a.in_off[r + 1] - j0 : (uint64_t)nj;
-    s_end[k] = (uint32_t)(e < nj ? e : nj);
+    uint64_t e = r < a.own_n ? (uint64_t)a.in_off[r + 1] - a.e_base - j0 : (uint64_t)nj;
+    s_end[pr_pad(k)] = (uint32_t)(e < nj ? e : nj);
   }
   {
     uint32_t src[kPrIpt];
@@ -108,7 +117,7 @@ __global__ void __launch_bounds__(kPrThreads, 4) k_pr_gather_apply(const __grid_
 #pragma unroll
     for (int q = 0; q < kPrIpt; q++) {
       const uint32_t k = tid + q * kPrThreads;
-      if (k < nj) s_val[k] = v[q];
+      if (k < nj) s_val[pr_pad(k)] = v[q];
     }
   }
   __syncthreads();
@@ -119,7 +128,7 @@ __global__ void __launch_bounds__(kPrThreads, 4) k_pr_gather_apply(const __grid_
   uint32_t lo = dt > nj ? dt - nj : 0, hi = dt < ni ? dt : ni;
   while (lo < hi) {
     const uint32_t p = (lo + hi) >> 1;
-    if (s_end[p] <= dt - p - 1) lo = p + 1;
+    if (s_end[pr_pad(p)] <= dt - p - 1) lo = p + 1;
     else hi = p;
   }
   uint32_t i = lo, j = dt - lo;
@@ -128,8 +137,8 @@ __global__ void __launch_bounds__(kPrThreads, 4) k_pr_gather_apply(const __grid_
 #pragma unroll
   for (int q = 0; q < kPrIpt; q++) {
     if (dt + q < dend) {
-      if (j < s_end[i]) { run += s_val[j]; ++j; }
-      else { s_tot[i] = run; run = 0.f; ++i; }
+      if (j < s_end[pr_pad(i)]) { run += s_val[pr_pad(j)]; ++j; }
+      else { s_tot[pr_pad(i)] = run; run = 0.f; ++i; }
     }
   }
   s_crow[tid] = i;
@@ -156,18 +165,18 @@ __global__ void __launch_bounds__(kPrThreads, 4) k_pr_gather_apply(const __grid_
   __syncthreads();
   // the last thread of each carry run adds it to the row finished by the next thread
   const bool run_end = (tid == kPrThreads - 1) || (s_crow[tid + 1] != i);
-  if (run_end && i < ni) s_tot[i] += x;
+  if (run_end && i < ni) s_tot[pr_pad(i)] += x;
   __syncthreads();
 
   // apply the rows whose end lies in this tile (coalesced over destinations)
   const bool head = (ni > 0) && (s_rowstart0 < j0);  // row i0 began in an earlier tile
   for (uint32_t k = tid; k < ni; k += kPrThreads) {
     if (k == 0 && head) continue;
-    pr_apply_row(a, (uint32_t)(i0 + k), s_tot[k]);
+    pr_apply_row(a, (uint32_t)(i0 + k), s_tot[pr_pad(k)]);
   }
   if (tid == 0) {
     a.head_row[blockIdx.x] = head ? (uint32_t)i0 : kNoRow;
-    a.head_val[blockIdx.x] = head ? s_tot[0] : 0.f;
+    a.head_val[blockIdx.x] = head ? s_tot[pr_pad(0)] : 0.f;
     const uint64_t i1 = s_i1;
     a.carry_row[blockIdx.x] = i1 < a.own_n ? (uint32_t)i1 : kNoRow;
     a.carry_val[blockIdx.x] = s_cval[kPrThreads - 1];
@@ -186,14 +195,27 @@ __global__ void k_pr_fixup(const __grid_constant__ PrArgs<OffT> a, uint32_t num_
   }
 }
 
+// Merge-path coordinates of every tile start (once per graph / shard): tile_row[c]
+// = rows consumed before diagonal c * kPrTile (the last entry is the end).
+template <class OffT>
+__global__ void k_pr_tiles(const OffT *in_off, uint64_t e_base, uint32_t rows, uint64_t nnz, uint32_t num_tiles,
+                           uint32_t *tile_row) {
+  const uint64_t total = (uint64_t)rows + nnz;
+  for (uint32_t c = blockIdx.x * blockDim.x + threadIdx.x; c <= num_tiles; c += gridDim.x * blockDim.x) {
+    uint64_t diag = (uint64_t)c * kPrTile;
+    if (diag > total) diag = total;
+    tile_row[c] = merge_path_rows(in_off, e_base, rows, nnz, diag);
+  }
+}
+
 // contrib_0[u] = R_0(u) / outdeg(u) with R_0 = 1/n (reading R3); dangling -> 0 (R2).
-__global__ void k_pr_init(uint32_t n, const float *inv_outdeg, float *contrib) {
+static __global__ void k_pr_init(uint32_t n, const float *inv_outdeg, float *contrib) {
   const float r0 = 1.0f / (float)n;
   for (uint64_t v = blockIdx.x * (uint64_t)blockDim.x + threadIdx.x; v < n; v += (uint64_t)gridDim.x * blockDim.x)
     contrib[v] = r0 * inv_outdeg[v];
 }
 
-__global__ void k_inv_outdeg(uint32_t n, const uint32_t *outdeg, float *inv) {
+static __global__ void k_inv_outdeg(uint32_t n, const uint32_t *outdeg, float *inv) {
   for (uint64_t v = blockIdx.x * (uint64_t)blockDim.x + threadIdx.x; v < n; v += (uint64_t)gridDim.x * blockDim.x) {
     const uint32_t d = outdeg[v];
     inv[v] = d ? 1.0f / (float)d : 0.f;

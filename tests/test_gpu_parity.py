@@ -163,3 +163,53 @@ def test_errors_through_abi():
         with pytest.raises(gr.GrError) as ei:
             G.run("custom", custom_id=77)
         assert ei.value.status == gr.GR_EUNSUPPORTED
+
+
+# ---------------------------------------------------------------- streamed mode
+@pytest.mark.parametrize("algo", ["bfs", "sssp", "cc", "pagerank"])
+@pytest.mark.parametrize("shard_edges", [3000, 40000])
+def test_streamed_equals_oracle(algo, shard_edges):
+    g = grgen.rmat(13, 16, seed=4)
+    src, dst = g.src, g.dst
+    if algo == "cc":
+        src, dst = np.concatenate([g.src, g.dst]), np.concatenate([g.dst, g.src])
+    w = grgen.weights(len(src), 1, 64, seed=5)
+    st = compare(g.n, src, dst, w, algo, source=1, loops=("host",), mode="streamed", shard_edges=shard_edges)
+    assert st["bytes_h2d"] > 0
+
+
+@pytest.mark.parametrize("algo", ["bfs", "sssp", "cc", "pagerank"])
+def test_streamed_hub_larger_than_shard(algo):
+    n, src, dst, w = hub_graph()
+    compare(n, src, dst, w, algo, source=0, loops=("host",), mode="streamed", shard_edges=2000)
+
+
+@pytest.mark.parametrize("cfg", [1, 3, 4])
+def test_streamed_reduced_configs(cfg):
+    g, run = grgen.config(cfg, reduced=True)
+    w = g.get("w")
+    compare(g.n, g.src, g.dst, w, run["algo"], source=run.get("source", 0), loops=("host",), mode="streamed",
+            shard_edges=max(1000, g.m // 16))
+
+
+def test_streamed_frontier_skips_inactive_shards():
+    # two disjoint directed paths: BFS from the first never copies a shard of the second
+    k = 20000
+    a = np.arange(k - 1, dtype=np.uint32)
+    src = np.concatenate([a, a + k])
+    dst = np.concatenate([a + 1, a + 1 + k])
+    with gr.GraphReduce(2 * k, src, dst, mode="streamed", shard_edges=4000) as G:
+        info = G.info()
+        assert info["mode"] == 2 and info["num_shards"] > 4
+        shards = [gr.gr_shard_info(G.h, s) for s in range(info["num_shards"])]
+        first = [s for s in shards if s["v_lo"] < k]
+        max_first = max(4 * (s["out_end"] - s["out_begin"]) for s in first)
+        st = G.run("bfs", source=0)
+        assert st["iterations"] == k
+        # one changed vertex per superstep => at most one shard's out-edges copied per superstep
+        assert st["bytes_h2d"] <= st["iterations"] * max_first
+        # and in total never more than the first path's shards once per superstep they were active
+        whole = 4 * (len(src))
+        assert st["bytes_h2d"] < st["iterations"] * whole / 4
+        d = G.values()
+        assert d[k - 1] == k - 1 and d[k] == gr.INF
