@@ -152,6 +152,8 @@ def main():
     ap.add_argument("--config", type=int, default=2)
     ap.add_argument("--e2e-steps", type=int, default=2)
     ap.add_argument("--no-cpu", action="store_true")
+    ap.add_argument("--loop", default="auto", choices=["auto", "host", "device"],
+                    help="superstep loop for frontier programs (host: profilable by ncu)")
     args = ap.parse_args()
 
     rank = int(os.environ.get("RANK", "0"))
@@ -191,7 +193,8 @@ def main():
     g, w, run = make_graph(args.config)
     print(f"[bench] generated {g.name}: n={g.n} m={g.m} in {time.perf_counter() - t0:.1f}s", file=sys.stderr)
     algo = run["algo"]
-    kw = dict(source=run.get("source", 0), max_iters=run.get("max_iters", 0), damping=run.get("damping", 0.85))
+    kw = dict(source=run.get("source", 0), max_iters=run.get("max_iters", 0), damping=run.get("damping", 0.85),
+              loop=args.loop)
     G = gr.GraphReduce(g.n, g.src, g.dst, w, device=local_rank, mode="resident")
     info = G.info()
     print(f"[bench] loaded in {time.perf_counter() - t0:.1f}s total: {info}", file=sys.stderr)

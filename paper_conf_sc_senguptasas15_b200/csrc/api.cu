@@ -50,8 +50,13 @@ gr_status gr_graph_load(const gr_edges *edges, const gr_load_opts *opts_in, gr_g
   if (opts_in) opts = *opts_in;
   if (opts.world <= 0) opts.world = 1;
   if (opts.mode < GR_MODE_AUTO || opts.mode > GR_MODE_STREAMED) return fail(GR_EINVAL, "bad mode %d", opts.mode);
-  if (opts.world > 1 || opts.sim_ranks > 1)
-    return fail(GR_EUNSUPPORTED, "multi-rank partitions are not available in this build");
+  const bool sim = opts.sim_ranks > 1;
+  if (sim) opts.world = opts.sim_ranks;
+  if (opts.rank < 0 || opts.rank >= opts.world) return fail(GR_EINVAL, "rank %d outside [0, %d)", opts.rank, opts.world);
+  if (opts.world > 1 && opts.mode == GR_MODE_STREAMED)
+    return fail(GR_EUNSUPPORTED, "streamed mode is single-rank (partition over GPUs to fit HBM instead)");
+  if (opts.world > 1 && !opts.nccl_unique_id)
+    return fail(GR_EINVAL, "world > 1 needs nccl_unique_id (simulated ranks: any 128-byte group key)");
   int ndev = 0;
   cudaError_t ce = cudaGetDeviceCount(&ndev);
   if (ce != cudaSuccess || ndev == 0) {
@@ -88,10 +93,17 @@ gr_status gr_graph_load(const gr_edges *edges, const gr_load_opts *opts_in, gr_g
   uint64_t budget = opts.device_budget_bytes ? opts.device_budget_bytes
                                              : (free_b > (4ull << 30) ? free_b - (4ull << 30) : free_b / 2);
   const uint64_t need = resident_bytes_estimate(g->H);
-  if (opts.mode == GR_MODE_AUTO) g->mode = need <= budget ? GR_MODE_RESIDENT : GR_MODE_STREAMED;
+  if (opts.mode == GR_MODE_AUTO) g->mode = (need <= budget || opts.world > 1) ? GR_MODE_RESIDENT : GR_MODE_STREAMED;
   else g->mode = opts.mode;
+  g->sim = sim;
   s = load_device(g);
   if (s == GR_OK && g->mode == GR_MODE_STREAMED) s = stream_setup(g, budget);
+  if (s == GR_OK && opts.world > 1) {
+    std::string cerr;
+    s = comm_create(opts.world, opts.rank, sim, opts.nccl_unique_id, g->device, &g->comm, &cerr);
+    if (s != GR_OK) fail(s, "%s", cerr.c_str());
+    if (s == GR_OK) s = part_setup(g);
+  }
   if (s != GR_OK) {
     std::string keep = gr::last_error();
     destroy(g);
@@ -133,9 +145,9 @@ gr_status gr_graph_info_get(const gr_graph *g, gr_graph_info *o) {
   o->num_edges = g->H.m_total;
   o->num_shards = g->H.num_shards();
   o->mode = g->mode;
-  o->rank = 0;
-  o->world = 1;
-  o->sim_ranks = 1;
+  o->rank = g->comm ? g->comm->rank : 0;
+  o->world = g->comm ? g->comm->world : 1;
+  o->sim_ranks = g->sim ? o->world : 1;
   o->own_lo = g->H.own_lo;
   o->own_hi = g->H.own_hi;
   o->device_bytes = g->dev_bytes;

@@ -1,0 +1,167 @@
+// comm.cu — NCCL and simulated (in-process) partition exchange. See comm.h.
+#include "comm.h"
+
+#include <nccl.h>
+
+#include <condition_variable>
+#include <cstring>
+#include <map>
+#include <memory>
+#include <mutex>
+
+namespace gr {
+
+// ------------------------------------------------------------------- NCCL
+struct NcclComm : Comm {
+  ncclComm_t comm = nullptr;
+  uint64_t *d_small = nullptr;  // world * 8 u64 scratch
+  uint64_t *h_small = nullptr;
+  ~NcclComm() override {
+    if (comm) ncclCommDestroy(comm);
+    if (d_small) cudaFree(d_small);
+    if (h_small) cudaFreeHost(h_small);
+  }
+  gr_status allgatherv(const void *send, void *recv, const std::vector<uint64_t> &counts,
+                       const std::vector<uint64_t> &displs, cudaStream_t s) override {
+    ncclResult_t r = ncclGroupStart();
+    for (int q = 0; q < world && r == ncclSuccess; q++) {
+      if (!counts[q]) continue;
+      char *dst = static_cast<char *>(recv) + displs[q];
+      r = ncclBroadcast(q == rank ? send : dst, dst, counts[q], ncclChar, q, comm, s);
+      if (q != rank) bytes_in += counts[q];
+    }
+    ncclResult_t r2 = ncclGroupEnd();
+    if (r != ncclSuccess || r2 != ncclSuccess) return GR_ENCCL;
+    return GR_OK;
+  }
+  gr_status allgather_small(const uint64_t *mine, int k, uint64_t *out, cudaStream_t s) override {
+    if (k > 8) return GR_EINVAL;
+    if (cudaMemcpyAsync(d_small + (size_t)rank * 8, mine, 8 * k, cudaMemcpyHostToDevice, s) != cudaSuccess)
+      return GR_ECUDA;
+    if (ncclAllGather(d_small + (size_t)rank * 8, d_small, 8, ncclUint64, comm, s) != ncclSuccess) return GR_ENCCL;
+    if (cudaMemcpyAsync(h_small, d_small, 64ull * world, cudaMemcpyDeviceToHost, s) != cudaSuccess ||
+        cudaStreamSynchronize(s) != cudaSuccess)
+      return GR_ECUDA;
+    for (int q = 0; q < world; q++)
+      for (int i = 0; i < k; i++) out[q * k + i] = h_small[q * 8 + i];
+    return GR_OK;
+  }
+};
+
+// -------------------------------------------------------------- simulated
+struct SimGroup {
+  int world = 0;
+  std::mutex mu;
+  std::condition_variable cv;
+  int arrived = 0;
+  uint64_t gen = 0;
+  std::vector<const void *> ptrs;
+  std::vector<uint64_t> small;  // world * 8
+  int members = 0;
+
+  void barrier() {
+    std::unique_lock<std::mutex> lk(mu);
+    const uint64_t g = gen;
+    if (++arrived == world) {
+      arrived = 0;
+      gen++;
+      cv.notify_all();
+    } else {
+      cv.wait(lk, [&] { return gen != g; });
+    }
+  }
+};
+
+static std::mutex g_sim_mu;
+static std::map<std::string, std::shared_ptr<SimGroup>> g_sim_groups;
+
+struct SimComm : Comm {
+  std::shared_ptr<SimGroup> grp;
+  std::string key;
+  ~SimComm() override {
+    std::lock_guard<std::mutex> lk(g_sim_mu);
+    if (--grp->members == 0) g_sim_groups.erase(key);
+  }
+  gr_status allgatherv(const void *send, void *recv, const std::vector<uint64_t> &counts,
+                       const std::vector<uint64_t> &displs, cudaStream_t s) override {
+    if (cudaStreamSynchronize(s) != cudaSuccess) return GR_ECUDA;  // own data ready
+    grp->ptrs[rank] = send;
+    grp->barrier();
+    for (int q = 0; q < world; q++) {
+      char *dst = static_cast<char *>(recv) + displs[q];
+      if (!counts[q] || grp->ptrs[q] == dst) continue;
+      if (cudaMemcpyAsync(dst, grp->ptrs[q], counts[q], cudaMemcpyDeviceToDevice, s) != cudaSuccess)
+        return GR_ECUDA;
+      if (q != rank) bytes_in += counts[q];
+    }
+    if (cudaStreamSynchronize(s) != cudaSuccess) return GR_ECUDA;
+    grp->barrier();  // peers may reuse their send buffers only after everyone copied
+    return GR_OK;
+  }
+  gr_status allgather_small(const uint64_t *mine, int k, uint64_t *out, cudaStream_t s) override {
+    if (k > 8) return GR_EINVAL;
+    if (cudaStreamSynchronize(s) != cudaSuccess) return GR_ECUDA;
+    for (int i = 0; i < k; i++) grp->small[rank * 8 + i] = mine[i];
+    grp->barrier();
+    for (int q = 0; q < world; q++)
+      for (int i = 0; i < k; i++) out[q * k + i] = grp->small[q * 8 + i];
+    grp->barrier();
+    return GR_OK;
+  }
+};
+
+gr_status comm_create(int world, int rank, bool sim, const void *id128, int device, Comm **out, std::string *err) {
+  *out = nullptr;
+  if (world <= 1) return GR_OK;
+  if (!id128) {
+    *err = "world > 1 needs nccl_unique_id (128 bytes; any 128 bytes name a simulated group)";
+    return GR_EINVAL;
+  }
+  if (sim) {
+    auto *c = new SimComm();
+    c->rank = rank;
+    c->world = world;
+    c->key.assign(static_cast<const char *>(id128), 128);
+    {
+      std::lock_guard<std::mutex> lk(g_sim_mu);
+      auto &g = g_sim_groups[c->key];
+      if (!g) {
+        g = std::make_shared<SimGroup>();
+        g->world = world;
+        g->ptrs.assign(world, nullptr);
+        g->small.assign(8ull * world, 0);
+      }
+      if (g->world != world) {
+        delete c;
+        *err = "simulated group world mismatch";
+        return GR_EINVAL;
+      }
+      g->members++;
+      c->grp = g;
+    }
+    *out = c;
+    return GR_OK;
+  }
+  auto *c = new NcclComm();
+  c->rank = rank;
+  c->world = world;
+  ncclUniqueId id;
+  std::memcpy(&id, id128, sizeof id);
+  cudaSetDevice(device);
+  ncclResult_t r = ncclCommInitRank(&c->comm, world, id, rank);
+  if (r != ncclSuccess) {
+    *err = std::string("ncclCommInitRank: ") + ncclGetErrorString(r);
+    c->comm = nullptr;
+    delete c;
+    return GR_ENCCL;
+  }
+  if (cudaMalloc(&c->d_small, 64ull * world) != cudaSuccess || cudaMallocHost(&c->h_small, 64ull * world) != cudaSuccess) {
+    delete c;
+    *err = "comm scratch allocation failed";
+    return GR_ENOMEM;
+  }
+  *out = c;
+  return GR_OK;
+}
+
+}  // namespace gr

@@ -1,0 +1,39 @@
+// comm.h — the per-superstep exchange between owner partitions.
+//
+// Multi-GPU is the paper's future-work item (1) (§8). Destination
+// intervals shard naturally: each rank owns a contiguous destination range, so
+// one exchange per superstep suffices — an allgather of the changed vertices
+// (frontier programs) or of the owned contribution slices (PageRank).
+//   NcclComm : one process per GPU, NCCL over NVLink/NVSwitch (allgatherv as a
+//              grouped ncclBroadcast from every root).
+//   SimComm  : G "ranks" as host threads sharing ONE device (tests on a 1-GPU
+//              box): the same protocol with device-to-device copies.
+#pragma once
+#include <cuda_runtime.h>
+
+#include <cstdint>
+#include <string>
+#include <vector>
+
+#include "graphreduce.h"
+
+namespace gr {
+
+struct Comm {
+  int rank = 0, world = 1;
+  uint64_t bytes_in = 0;  // bytes received from peers (NVLink for NCCL)
+  virtual ~Comm() = default;
+  // allgatherv of device bytes: rank r's `counts[r]` bytes land at recv + displs[r]
+  // on every rank. `send` may alias recv + displs[rank]. Stream-ordered on s.
+  virtual gr_status allgatherv(const void *send, void *recv, const std::vector<uint64_t> &counts,
+                               const std::vector<uint64_t> &displs, cudaStream_t s) = 0;
+  // allgather of k host uint64 per rank (synchronous w.r.t. s): out[r*k + i]
+  virtual gr_status allgather_small(const uint64_t *mine, int k, uint64_t *out, cudaStream_t s) = 0;
+};
+
+// Create the communicator for a loaded partition. world <= 1 returns nullptr.
+// sim: in-process simulated group keyed by the 128-byte id.
+gr_status comm_create(int world, int rank, bool sim, const void *id128, int device, Comm **out,
+                      std::string *err);
+
+}  // namespace gr

@@ -31,7 +31,7 @@ struct Ctl {
   uint32_t cnt_KC;        // chunk-list length of the changed hubs
   uint32_t ctr_hub;       // dynamic hub work counter (gather / BFS)
   uint32_t ctr_hub2;      // dynamic hub work counter (activate)
-  uint32_t done_blocks;   // last-block ticket
+  uint32_t done_blocks;   // (unused; see tick1/tick2)
   uint32_t implicit0;     // superstep 0 list is implicitly the owned range (CC: A_0 = V)
   uint32_t trace_cap;
   uint32_t source;        // BFS / SSSP source (programs may read it through Ctx)
@@ -40,10 +40,31 @@ struct Ctl {
   unsigned long long gathered;   // sum indeg(A_t)
   unsigned long long scattered;  // sum outdeg(C_t)
   unsigned long long tot_gathered, tot_scattered;
+  // per-superstep counters spread over kSlots addresses (CTA b adds to slot b % kSlots)
+  unsigned long long part_g[64], part_c[64], part_s[64], part_a[64];
+  uint32_t tick1[64];     // two-level last-CTA ticket: groups of 32 CTAs
+  uint32_t tick2;
+  uint32_t ext_loop;      // partitioned runs: the host decides termination (global counts)
+  uint32_t no_hub_c;      // partitioned runs: changed hubs are classified after the exchange
   unsigned long long prof;               // 1: kernels stamp %globaltimer
   unsigned long long kstart[2], kend[2]; // per-kernel span of the current superstep (ns)
   unsigned long long kns[2];             // accumulated kernel ns: [0] gather+apply, [1] activate / BFS expand
 };
+
+constexpr int kSlots = 64;
+
+// Block-wide sum of a per-thread u64 (all threads call; result valid in thread 0).
+__device__ __forceinline__ unsigned long long block_sum_u64(unsigned long long x, unsigned long long *s8) {
+#pragma unroll
+  for (int o = 16; o > 0; o >>= 1) x += __shfl_xor_sync(0xffffffffu, x, o);
+  __syncthreads();
+  if ((threadIdx.x & 31) == 0) s8[threadIdx.x >> 5] = x;
+  __syncthreads();
+  unsigned long long t = 0;
+  if (threadIdx.x == 0)
+    for (int i = 0; i < (int)(blockDim.x >> 5); i++) t += s8[i];
+  return t;
+}
 
 __device__ __forceinline__ unsigned long long gtimer() {
   unsigned long long t;
@@ -103,6 +124,20 @@ __device__ __forceinline__ uint8_t ldg_nc_u8(const uint8_t *p) {
   return (uint8_t)v;
 }
 
+// L2-coherent read (bypasses L1, so stamps written by other SMs are seen)
+__device__ __forceinline__ uint32_t ld_cg(const uint32_t *p) {
+  uint32_t v;
+  asm volatile("ld.global.cg.u32 %0, [%1];" : "=r"(v) : "l"(p));
+  return v;
+}
+
+// First-stamper test: a plain L2 read filters the (many) edges that reach an
+// already-stamped vertex, so only the first few pay the serialized atomic on a
+// popular target's address.
+__device__ __forceinline__ bool stamp_first(uint32_t *stamp, uint32_t epoch) {
+  return ld_cg(stamp) != epoch && atomicExch(stamp, epoch) != epoch;
+}
+
 __device__ __forceinline__ bool test_bit(const uint32_t *bits, uint32_t i) {
   return (__ldg(bits + (i >> 5)) >> (i & 31)) & 1u;
 }
@@ -136,6 +171,26 @@ struct WarpQueue {
     if (lane_id() == 0) base = atomicAdd(g_cnt, n);
     base = __shfl_sync(0xffffffffu, base, 0);
     for (uint32_t i = lane_id(); i < n; i += 32) {
+      g_a[base + i] = s_a[i];
+      if (g_b) g_b[base + i] = s_b[i];
+    }
+    __syncwarp();
+    n = 0;
+  }
+  // Final flush of every warp of the CTA with ONE global atomic (all threads call).
+  __device__ void block_flush(uint32_t *g_a, uint32_t *g_b, uint32_t *g_cnt, uint32_t *s_off) {
+    const uint32_t w = threadIdx.x >> 5, nw = blockDim.x >> 5;
+    __syncthreads();
+    if ((threadIdx.x & 31) == 0) s_off[w] = n;
+    __syncthreads();
+    if (threadIdx.x == 0) {
+      uint32_t tot = 0;
+      for (uint32_t i = 0; i < nw; i++) { const uint32_t c = s_off[i]; s_off[i] = tot; tot += c; }
+      s_off[nw] = tot ? atomicAdd(g_cnt, tot) : 0u;
+    }
+    __syncthreads();
+    const uint32_t base = s_off[nw] + s_off[w];
+    for (uint32_t i = threadIdx.x & 31; i < n; i += 32) {
       g_a[base + i] = s_a[i];
       if (g_b) g_b[base + i] = s_b[i];
     }

@@ -426,6 +426,18 @@ gr_status run(gr_graph *g, const gr_run_opts *oin, gr_run_stats *st) {
   cudaStream_t s = o.stream ? (cudaStream_t)o.stream : g->stream;
   CK(cudaEventRecord(g->ev_start, s));
   gr_status r;
+  if (g->comm) {
+    r = run_part(g, &o, s, st);
+    if (r != GR_OK) return r;
+    CK(cudaEventRecord(g->ev_stop, s));
+    CK(cudaEventSynchronize(g->ev_stop));
+    float ms = 0;
+    CK(cudaEventElapsedTime(&ms, g->ev_start, g->ev_stop));
+    st->seconds = ms * 1e-3;
+    g->last_algo = o.algo;
+    g->last_iters = st->iterations;
+    return GR_OK;
+  }
   switch (o.algo) {
     case GR_BFS:
       r = g->off64 ? run_frontier<ProgBFS, uint64_t>(g, &o, s, st, 0) : run_frontier<ProgBFS, uint32_t>(g, &o, s, st, 0);
@@ -457,6 +469,7 @@ gr_status fetch_values(gr_graph *g, void *dst, uint64_t bytes) {
   const uint64_t n = g->H.n;
   if (bytes < 4 * n) return fail(GR_EINVAL, "buffer of %llu bytes < 4*n = %llu", (unsigned long long)bytes,
                                  (unsigned long long)(4 * n));
+  if (g->comm) return part_fetch_values(g, dst, bytes);
   if (g->last_algo == GR_PAGERANK) CK(cudaMemcpy(dst, g->rank, 4 * n, cudaMemcpyDeviceToHost));
   else CK(cudaMemcpy(dst, g->val, 4 * n, cudaMemcpyDeviceToHost));
   return GR_OK;
@@ -465,6 +478,7 @@ gr_status fetch_values(gr_graph *g, void *dst, uint64_t bytes) {
 gr_status fetch_trace(gr_graph *g, uint64_t *dst, uint64_t max_rows, uint64_t *rows) {
   if (g->last_algo < 0) return fail(GR_ESTATE, "gr_fetch_frontier_trace before gr_run");
   if (!rows || (max_rows && !dst)) return fail(GR_EINVAL, "null output");
+  if (g->comm) return part_fetch_trace(g, dst, max_rows, rows);
   const uint64_t r = std::min<uint64_t>(g->trace_rows, max_rows);
   if (g->last_algo == GR_PAGERANK) {
     for (uint64_t t = 0; t < r; t++) {
@@ -490,6 +504,8 @@ void destroy(gr_graph *g) {
   if (g->ev_start) cudaEventDestroy(g->ev_start);
   if (g->ev_stop) cudaEventDestroy(g->ev_stop);
   stream_destroy(g);
+  delete g->comm;
+  g->comm = nullptr;
   for (void *p : g->allocs) cudaFree(p);
   if (g->h_ctl) cudaFreeHost(g->h_ctl);
   if (g->stream) cudaStreamDestroy(g->stream);

@@ -7,6 +7,7 @@
 #include <utility>
 #include <vector>
 
+#include "comm.h"
 #include "device_common.cuh"
 #include "graphreduce.h"
 #include "host_graph.h"
@@ -68,6 +69,12 @@ struct gr_graph {
 
   // streamed mode (stream.cu)
   void *streamer = nullptr;
+
+  // partitioned (multi-GPU / simulated ranks) mode (engine_part.cu)
+  gr::Comm *comm = nullptr;
+  bool sim = false;
+  uint32_t *X_v = nullptr, *X_val = nullptr;  // exchanged changed set
+  float *rank_all = nullptr;                  // PageRank fetch assembly
 };
 
 namespace gr {
@@ -111,4 +118,9 @@ gr_status run_streamed(gr_graph *g, const gr_run_opts *o, gr_run_stats *st);
 void stream_destroy(gr_graph *g);
 uint64_t resident_bytes_estimate(const HostGraph &H);
 uint64_t static_bytes_estimate(const HostGraph &H);
+// partitioned mode
+gr_status part_setup(gr_graph *g);
+gr_status run_part(gr_graph *g, const gr_run_opts *o, cudaStream_t s, gr_run_stats *st);
+gr_status part_fetch_values(gr_graph *g, void *dst, uint64_t bytes);
+gr_status part_fetch_trace(gr_graph *g, uint64_t *dst, uint64_t max_rows, uint64_t *rows);
 }  // namespace gr

@@ -1,0 +1,269 @@
+// engine_part.cu — partitioned (multi-GPU) superstep drivers. SURVEY §8(e).
+//
+// Rank g owns destinations [own_lo, own_hi) (gr_plan_intervals over in+out
+// degree, identical on every rank), their CSC, and an activation CSR holding
+// the same edges grouped by source — so FrontierActivate targets only owned
+// vertices and no frontier OR-reduction is needed. Vertex values are
+// replicated. One exchange per superstep:
+//   frontier programs: allgatherv of the changed set (vertex, new value), then
+//     every rank commits all of it to its replica and activates its owned
+//     out-neighbours;
+//   PageRank: allgatherv of the owned contribution slices.
+// The loop is host-driven (termination needs the GLOBAL |A_{t+1}|).
+#include <cuda_runtime.h>
+
+#include <algorithm>
+#include <vector>
+
+#include "comm.h"
+#include "engine.h"
+#include "kernels_frontier.cuh"
+#include "kernels_pr.cuh"
+
+namespace gr {
+
+#define PCK(call)                                                                              \
+  do {                                                                                         \
+    cudaError_t e_ = (call);                                                                   \
+    if (e_ != cudaSuccess)                                                                     \
+      return fail(e_ == cudaErrorMemoryAllocation ? GR_ENOMEM : GR_ECUDA, "%s: %s (%s:%d)", #call, \
+                  cudaGetErrorString(e_), __FILE__, __LINE__);                                 \
+  } while (0)
+#define XCK(call)                                                      \
+  do {                                                                 \
+    gr_status s_ = (call);                                             \
+    if (s_ != GR_OK) return fail(s_, "exchange failed: %s", #call);    \
+  } while (0)
+
+gr_status part_setup(gr_graph *g) {
+  gr_status s;
+  const uint64_t n = g->H.n;
+  if ((s = dev_alloc(g, (void **)&g->X_v, 4 * n)) != GR_OK) return s;
+  if ((s = dev_alloc(g, (void **)&g->X_val, 4 * n)) != GR_OK) return s;
+  if ((s = dev_alloc(g, (void **)&g->rank_all, 4 * n)) != GR_OK) return s;
+  return GR_OK;
+}
+
+static void owner_bytes(const gr_graph *g, uint64_t elem, std::vector<uint64_t> *cnt, std::vector<uint64_t> *dsp) {
+  const auto &o = g->H.owners;
+  const int W = (int)o.size() - 1;
+  cnt->resize(W);
+  dsp->resize(W);
+  for (int q = 0; q < W; q++) {
+    (*cnt)[q] = (o[q + 1] - o[q]) * elem;
+    (*dsp)[q] = o[q] * elem;
+  }
+}
+
+// sum one u64 over ranks
+static gr_status global_sum(Comm *c, uint64_t mine, uint64_t *out, cudaStream_t s) {
+  std::vector<uint64_t> all(c->world);
+  gr_status st = c->allgather_small(&mine, 1, all.data(), s);
+  uint64_t t = 0;
+  for (uint64_t v : all) t += v;
+  *out = t;
+  return st;
+}
+
+template <class Prog, class OffT>
+gr_status run_frontier_part(gr_graph *g, const gr_run_opts *o, cudaStream_t s, gr_run_stats *st) {
+  Comm *C = g->comm;
+  Part<OffT> P = make_part<OffT>(g);
+  uint64_t launches = 0;
+  if (g->epoch_next > 0xF0000000u) {
+    PCK(cudaMemsetAsync(g->stamp, 0, 4ull * std::max<uint64_t>(g->H.own_n(), 1), s));
+    g->epoch_next = 1;
+  }
+  Ctl h{};
+  h.epoch_base = g->epoch_next;
+  h.max_iters = o->max_iters;
+  h.trace_cap = g->trace_cap;
+  h.source = o->source;
+  h.damping = o->damping;
+  h.ext_loop = 1;
+  h.no_hub_c = 1;
+  h.kstart[0] = h.kstart[1] = ~0ull;
+  PCK(cudaMemcpyAsync(g->ctl, &h, sizeof h, cudaMemcpyHostToDevice, s));
+  k_init_values<Prog, OffT><<<g->num_sms * 4, 256, 0, s>>>(P, o->source);
+  k_fill_u32<<<std::min<uint32_t>((g->hub_cap + 255) / 256, 1024), 256, 0, s>>>(g->hub_acc, Prog::identity_host(),
+                                                                                 g->hub_cap);
+  PCK(cudaMemsetAsync(g->hub_done, 0, 4ull * g->hub_cap, s));
+  if (Prog::kInit == kInitAll && g->n_static_hubs) {
+    PCK(cudaMemcpyAsync(g->listH[0], g->static_hubs, 4ull * g->n_static_hubs, cudaMemcpyDeviceToDevice, s));
+    PCK(cudaMemcpyAsync(g->chkA_h[0], g->static_chk_h, 4ull * g->n_static_chunks, cudaMemcpyDeviceToDevice, s));
+    PCK(cudaMemcpyAsync(g->chkA_c[0], g->static_chk_c, 4ull * g->n_static_chunks, cudaMemcpyDeviceToDevice, s));
+  }
+  // BFS runs unfused here (apply, exchange, activate), so its A lists are built
+  // by the generic activation (hub chunks by in-degree).
+  k_init_frontier<Prog, OffT><<<1, kBlock, 0, s>>>(P, o->source, g->n_static_hubs, g->n_static_chunks);
+  launches += 3;
+  PCK(cudaGetLastError());
+  PCK(cudaMemsetAsync(&g->ctl->stop, 0, sizeof(uint32_t), s));  // the host decides termination
+  PCK(cudaMemcpyAsync(g->h_ctl, g->ctl, sizeof(Ctl), cudaMemcpyDeviceToHost, s));
+  PCK(cudaStreamSynchronize(s));
+  uint64_t active = 0;
+  XCK(global_sum(C, g->h_ctl->cnt_act[0], &active, s));
+  uint32_t t = 0;
+  std::vector<uint64_t> cnt(C->world), dsp(C->world), all(C->world);
+  const uint32_t grid = g->grid_frontier;
+  while (active > 0 && (o->max_iters == 0 || t < o->max_iters)) {
+    k_gather_apply<Prog, OffT><<<grid, kBlock, 0, s>>>(P);
+    PCK(cudaMemcpyAsync(g->h_ctl, g->ctl, sizeof(Ctl), cudaMemcpyDeviceToHost, s));
+    PCK(cudaStreamSynchronize(s));
+    // exchange the changed set C_t (vertex, new value)
+    const uint64_t mine = g->h_ctl->cnt_C;
+    XCK(C->allgather_small(&mine, 1, all.data(), s));
+    uint64_t tot = 0;
+    for (int q = 0; q < C->world; q++) {
+      cnt[q] = 4 * all[q];
+      dsp[q] = 4 * tot;
+      tot += all[q];
+    }
+    if (tot) {
+      XCK(C->allgatherv(g->C_v, g->X_v, cnt, dsp, s));
+      XCK(C->allgatherv(g->C_val, g->X_val, cnt, dsp, s));
+    }
+    PCK(cudaMemsetAsync(&g->ctl->cnt_C, 0, sizeof(uint32_t), s));
+    if (tot) k_classify<OffT><<<std::min<uint32_t>(grid, (uint32_t)((tot + kBlock - 1) / kBlock)), kBlock, 0, s>>>(
+        P, g->X_v, g->X_val, (uint32_t)tot);
+    k_activate<OffT><<<grid, kBlock, 0, s>>>(P, 0ull, 0);
+    launches += tot ? 3 : 2;
+    PCK(cudaGetLastError());
+    PCK(cudaMemcpyAsync(g->h_ctl, g->ctl, sizeof(Ctl), cudaMemcpyDeviceToHost, s));
+    PCK(cudaStreamSynchronize(s));
+    t = g->h_ctl->iter;
+    XCK(global_sum(C, g->h_ctl->cnt_act[t & 1u], &active, s));
+  }
+  const Ctl &c = *g->h_ctl;
+  uint64_t v[2] = {c.tot_gathered, c.tot_scattered}, av[64];
+  XCK(C->allgather_small(v, 2, av, s));
+  st->iterations = t;
+  st->edges_gathered = st->edges_scattered = 0;
+  for (int q = 0; q < C->world; q++) {
+    st->edges_gathered += av[2 * q];
+    st->edges_scattered += av[2 * q + 1];
+  }
+  st->kernel_launches += launches;
+  st->bytes_nvlink = C->bytes_in;
+  g->epoch_next = h.epoch_base + t + 2;
+  g->trace_rows = std::min<uint64_t>(t, g->trace_cap);
+  st->bytes_hbm_model = (Prog::kUsesWeights ? 5 : 4) * c.tot_gathered + 4 * c.tot_scattered;
+  return GR_OK;
+}
+
+template <class OffT>
+gr_status run_pagerank_part(gr_graph *g, const gr_run_opts *o, cudaStream_t s, gr_run_stats *st) {
+  Comm *C = g->comm;
+  const uint32_t iters = o->max_iters;
+  const float d = o->damping;
+  const uint32_t lo = (uint32_t)g->H.own_lo;
+  std::vector<uint64_t> cnt, dsp;
+  owner_bytes(g, 4, &cnt, &dsp);
+  k_pr_init<<<g->num_sms * 4, 256, 0, s>>>((uint32_t)g->H.n, g->inv_outdeg, g->contrib[0]);
+  for (uint32_t t = 0; t < iters; t++) {
+    PrArgs<OffT> a{};
+    a.n = (uint32_t)g->H.n;
+    a.own_lo = lo;
+    a.own_n = (uint32_t)g->H.own_n();
+    a.m_in = g->H.m_in;
+    a.in_off = (const OffT *)g->in_off;
+    a.in_src = g->in_src;
+    a.inv_outdeg = g->inv_outdeg;
+    a.contrib_in = g->contrib[t & 1];
+    a.contrib_out = g->contrib[(t + 1) & 1];
+    a.rank = g->rank;
+    a.carry_row = g->carry_row;
+    a.carry_val = g->carry_val;
+    a.head_row = g->head_row;
+    a.head_val = g->head_val;
+    a.tile_row = g->tile_row;
+    a.base = (1.0f - d) / (float)g->H.n;
+    a.d = d;
+    a.last = (t + 1 == iters) ? 1 : 0;
+    k_pr_gather_apply<OffT><<<std::max<uint32_t>(g->pr_tiles, 1), kPrThreads, 0, s>>>(a);
+    k_pr_fixup<OffT><<<std::max<uint32_t>((g->pr_tiles + 255) / 256, 1), 256, 0, s>>>(a, g->pr_tiles);
+    PCK(cudaGetLastError());
+    if (!a.last) {
+      float *out = g->contrib[(t + 1) & 1];
+      XCK(C->allgatherv(out + lo, out, cnt, dsp, s));  // owned slices -> every replica
+    }
+  }
+  PCK(cudaStreamSynchronize(s));
+  st->iterations = iters;
+  uint64_t mi = g->H.m_in, tot = 0;
+  XCK(global_sum(C, mi, &tot, s));
+  st->edges_gathered = (uint64_t)iters * tot;
+  st->kernel_launches += 1 + 2ull * iters;
+  st->bytes_nvlink = C->bytes_in;
+  st->bytes_hbm_model = (uint64_t)iters * (4 * g->H.m_in + 12 * g->H.own_n() + 4 * g->H.n);
+  g->trace_rows = iters;
+  return GR_OK;
+}
+
+// Collective fetches for partitioned graphs.
+gr_status part_fetch_values(gr_graph *g, void *dst, uint64_t bytes) {
+  const uint64_t n = g->H.n;
+  if (g->last_algo == GR_PAGERANK) {
+    std::vector<uint64_t> cnt, dsp;
+    owner_bytes(g, 4, &cnt, &dsp);
+    XCK(g->comm->allgatherv(g->rank, g->rank_all, cnt, dsp, g->stream));
+    PCK(cudaStreamSynchronize(g->stream));
+    PCK(cudaMemcpy(dst, g->rank_all, 4 * n, cudaMemcpyDeviceToHost));
+  } else {
+    PCK(cudaMemcpy(dst, g->val, 4 * n, cudaMemcpyDeviceToHost));
+  }
+  (void)bytes;
+  return GR_OK;
+}
+
+gr_status part_fetch_trace(gr_graph *g, uint64_t *dst, uint64_t max_rows, uint64_t *rows) {
+  Comm *C = g->comm;
+  const uint64_t r = std::min<uint64_t>(g->trace_rows, max_rows);
+  if (g->last_algo == GR_PAGERANK) {
+    uint64_t mi = g->H.m_in, tot = 0;
+    XCK(global_sum(C, mi, &tot, g->stream));
+    for (uint64_t t = 0; t < r; t++) {
+      dst[4 * t] = g->H.n;
+      dst[4 * t + 1] = g->H.n;
+      dst[4 * t + 2] = tot;
+      dst[4 * t + 3] = 0;
+    }
+    *rows = r;
+    return GR_OK;
+  }
+  std::vector<uint64_t> cnt(C->world, 32 * r), dsp(C->world);
+  for (int q = 0; q < C->world; q++) dsp[q] = 32 * r * q;
+  char *base = nullptr;
+  PCK(cudaMalloc((void **)&base, 32 * std::max<uint64_t>(r, 1) * C->world));
+  PCK(cudaMemcpyAsync(base + 32 * r * C->rank, g->trace, 32 * r, cudaMemcpyDeviceToDevice, g->stream));
+  gr_status xs = C->allgatherv(base + 32 * r * C->rank, base, cnt, dsp, g->stream);
+  std::vector<uint64_t> all(4 * r * C->world);
+  cudaError_t ce = cudaStreamSynchronize(g->stream);
+  if (xs == GR_OK && ce == cudaSuccess && r) ce = cudaMemcpy(all.data(), base, 32 * r * C->world, cudaMemcpyDeviceToHost);
+  cudaFree(base);
+  if (xs != GR_OK) return fail(xs, "trace exchange failed");
+  if (ce != cudaSuccess) return fail(GR_ECUDA, "trace exchange: %s", cudaGetErrorString(ce));
+  for (uint64_t i = 0; i < 4 * r; i++) {
+    uint64_t sum = 0;
+    for (int q = 0; q < C->world; q++) sum += all[q * 4 * r + i];
+    dst[i] = sum;
+  }
+  *rows = r;
+  return GR_OK;
+}
+
+gr_status run_part(gr_graph *g, const gr_run_opts *o, cudaStream_t s, gr_run_stats *st) {
+  switch (o->algo) {
+    case GR_BFS:
+      return g->off64 ? run_frontier_part<ProgBFS, uint64_t>(g, o, s, st) : run_frontier_part<ProgBFS, uint32_t>(g, o, s, st);
+    case GR_SSSP:
+      return g->off64 ? run_frontier_part<ProgSSSP, uint64_t>(g, o, s, st)
+                      : run_frontier_part<ProgSSSP, uint32_t>(g, o, s, st);
+    case GR_CC:
+      return g->off64 ? run_frontier_part<ProgCC, uint64_t>(g, o, s, st) : run_frontier_part<ProgCC, uint32_t>(g, o, s, st);
+    default:
+      return g->off64 ? run_pagerank_part<uint64_t>(g, o, s, st) : run_pagerank_part<uint32_t>(g, o, s, st);
+  }
+}
+
+}  // namespace gr

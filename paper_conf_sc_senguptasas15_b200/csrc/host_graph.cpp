@@ -185,6 +185,7 @@ gr_status build_host_graph(const gr_edges *E, uint64_t shard_edges, int world, i
   G->m_total = m;
   G->own_lo = owners[rank];
   G->own_hi = owners[rank + 1];
+  G->owners = owners;
   G->has_w = (w != nullptr);
   const uint64_t own_n = G->own_n();
 

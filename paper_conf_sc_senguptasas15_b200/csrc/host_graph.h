@@ -34,6 +34,7 @@ struct HostGraph {
   uint64_t n = 0;          // |V|
   uint64_t m_total = 0;    // |E| of the input
   uint64_t own_lo = 0, own_hi = 0;  // owned destination range [own_lo, own_hi)
+  std::vector<uint64_t> owners;     // owner range bounds of every rank (world + 1)
   uint64_t m_in = 0;       // in-edges with an owned destination
   bool has_w = false;
   // CSC over owned destinations: in-edges of v = in_src[in_off[v-own_lo] .. in_off[v-own_lo+1])

@@ -25,6 +25,8 @@
 
 namespace gr {
 
+constexpr int kBatch = 4;  // edges in flight per lane per memory phase
+
 // ----------------------------------------------------------------- helpers
 template <class Prog>
 __device__ __forceinline__ typename Prog::GatherT warp_reduce_prog(typename Prog::GatherT x) {
@@ -68,7 +70,9 @@ __device__ typename Prog::GatherT gather_warp(const Part<OffT> &P, bool valid, u
     r = warp_reduce_prog<Prog>(r);
     if ((int)lane == L) acc = r;
   }
-  // fine-grained: pack the edges of all lanes with degree <= 32, 32 per round
+  // fine-grained: pack the edges of all lanes with degree <= 32, 32 per round;
+  // kBatch rounds' loads (sources + weights, then source values) are issued
+  // together before their segmented reductions
   const uint32_t sd = (valid && deg <= 32) ? deg : 0u;
   const uint32_t incl = warp_incl_scan(sd);
   const uint32_t excl = incl - sd;
@@ -76,33 +80,52 @@ __device__ typename Prog::GatherT gather_warp(const Part<OffT> &P, bool valid, u
   if (total == 0) return acc;
   sred[lane] = Prog::identity();
   __syncwarp();
-  for (uint32_t r0 = 0; r0 < total; r0 += 32) {
-    const uint32_t k = r0 + lane;
-    int o = 0;
+  for (uint32_t rb = 0; rb < total; rb += 32u * kBatch) {
+    int own[kBatch];
+    uint32_t su[kBatch], sw[kBatch], dv[kBatch];
+    bool act[kBatch];
 #pragma unroll
-    for (int step = 16; step > 0; step >>= 1) {
-      const uint32_t e = __shfl_sync(0xffffffffu, excl, o + step);
-      if (e <= k) o += step;
-    }
-    const uint64_t ob = __shfl_sync(0xffffffffu, beg, o);
-    const uint32_t oe = __shfl_sync(0xffffffffu, excl, o);
-    const uint32_t odv = __shfl_sync(0xffffffffu, dval, o);
-    G x = (k < total) ? map_edge<Prog>(P, ob + (k - oe), odv, cx) : Prog::identity();
-    // segmented inclusive scan keyed by owner lane (owners are non-decreasing)
-    const int prev_o = __shfl_up_sync(0xffffffffu, o, 1);
-    uint32_t f = (lane == 0 || prev_o != o) ? 1u : 0u;
+    for (int q = 0; q < kBatch; q++) {
+      const uint32_t k = rb + q * 32u + lane;
+      int o = 0;
 #pragma unroll
-    for (int d = 1; d < 32; d <<= 1) {
-      const G y = __shfl_up_sync(0xffffffffu, x, d);
-      const uint32_t g = __shfl_up_sync(0xffffffffu, f, d);
-      if (lane >= (uint32_t)d) {
-        if (!f) x = Prog::gatherReduce(y, x);
-        f |= g;
+      for (int step = 16; step > 0; step >>= 1) {
+        const uint32_t e = __shfl_sync(0xffffffffu, excl, o + step);
+        if (e <= k) o += step;
       }
+      own[q] = o;
+      const uint64_t ob = __shfl_sync(0xffffffffu, beg, o);
+      const uint32_t oe = __shfl_sync(0xffffffffu, excl, o);
+      dv[q] = __shfl_sync(0xffffffffu, dval, o);
+      act[q] = k < total;
+      const uint64_t e = ob + (k - oe);
+      su[q] = act[q] ? ldg_nc(P.in_src + e) : 0u;
+      sw[q] = (act[q] && Prog::kUsesWeights) ? (uint32_t)ldg_nc_u8(P.in_w + e) : 0u;
     }
-    const int next_o = __shfl_down_sync(0xffffffffu, o, 1);
-    if (lane == 31 || next_o != o) sred[o] = Prog::gatherReduce(sred[o], x);
-    __syncwarp();
+    uint32_t sv[kBatch];
+#pragma unroll
+    for (int q = 0; q < kBatch; q++) sv[q] = act[q] ? P.val[su[q]] : 0u;
+#pragma unroll
+    for (int q = 0; q < kBatch; q++) {
+      if (rb + q * 32u >= total) break;  // warp-uniform
+      const int o = own[q];
+      G x = act[q] ? Prog::gatherMap(dv[q], sv[q], sw[q], cx) : Prog::identity();
+      // segmented inclusive scan keyed by owner lane (owners are non-decreasing)
+      const int prev_o = __shfl_up_sync(0xffffffffu, o, 1);
+      uint32_t f = (lane == 0 || prev_o != o) ? 1u : 0u;
+#pragma unroll
+      for (int dd = 1; dd < 32; dd <<= 1) {
+        const G y = __shfl_up_sync(0xffffffffu, x, dd);
+        const uint32_t g = __shfl_up_sync(0xffffffffu, f, dd);
+        if (lane >= (uint32_t)dd) {
+          if (!f) x = Prog::gatherReduce(y, x);
+          f |= g;
+        }
+      }
+      const int next_o = __shfl_down_sync(0xffffffffu, o, 1);
+      if (lane == 31 || next_o != o) sred[o] = Prog::gatherReduce(sred[o], x);
+      __syncwarp();
+    }
   }
   if (sd > 0) acc = sred[lane];
   __syncwarp();
@@ -170,94 +193,146 @@ __device__ void append_hub_C(const Part<OffT> &P, uint32_t v, uint32_t nv) {
   }
 }
 
-// FrontierActivate of out-edge targets x (one per lane, `act` marks real ones):
-// stamp with `epoch`; the first stamper appends x (BFS: only if still unvisited).
+// FrontierActivate of up to kBatch targets per lane (`act` marks real ones).
+// Each memory phase (stamp read, first-stamper atomic, BFS filter read, hub
+// bit) is issued for the whole batch before any result is consumed, so a lane
+// keeps kBatch independent requests in flight instead of one dependent chain.
+// The first stamper of x appends it (BFS: only if still unvisited).
 template <bool kBfsFilter, class OffT>
-__device__ __forceinline__ uint32_t activate_lanes(const Part<OffT> &P, bool act, uint32_t x, uint32_t epoch,
-                                                   const uint32_t *hub_bits, WarpQueue &qA,
-                                                   uint32_t slot) {
-  bool newly = false;
-  if (act) {
-    const uint32_t lx = x - P.own_lo;
-    newly = atomicExch(P.stamp + lx, epoch) != epoch;
+__device__ __forceinline__ uint32_t activate_batch(const Part<OffT> &P, const bool (&act)[kBatch],
+                                                   const uint32_t (&x)[kBatch], uint32_t epoch,
+                                                   const uint32_t *hub_bits, WarpQueue &qA, uint32_t slot) {
+  uint32_t st[kBatch];
+#pragma unroll
+  for (int q = 0; q < kBatch; q++) st[q] = act[q] ? ld_cg(P.stamp + (x[q] - P.own_lo)) : epoch;
+  bool nw[kBatch];
+#pragma unroll
+  for (int q = 0; q < kBatch; q++) {
+    const uint32_t old = (st[q] != epoch) ? atomicExch(P.stamp + (x[q] - P.own_lo), epoch) : epoch;
+    nw[q] = old != epoch;
   }
-  bool keep = newly;
-  if (kBfsFilter && keep) keep = (*(volatile uint32_t *)(P.val + x) == kInf);
-  const bool hub = keep && test_bit(hub_bits, kBfsFilter ? x : x - P.own_lo);
-  qA.push(keep && !hub, x, 0, P.listA[slot], nullptr, &P.ctl->cnt_A[slot]);
-  if (hub) append_hub_A<kBfsFilter>(P, x, slot);
-  return __popc(__ballot_sync(0xffffffffu, newly));
+  bool keep[kBatch];
+#pragma unroll
+  for (int q = 0; q < kBatch; q++) {
+    if (kBfsFilter) keep[q] = nw[q] && (*(volatile uint32_t *)(P.val + x[q]) == kInf);
+    else keep[q] = nw[q];
+  }
+  uint32_t cnt = 0;
+#pragma unroll
+  for (int q = 0; q < kBatch; q++) {
+    const bool hub = keep[q] && test_bit(hub_bits, kBfsFilter ? x[q] : x[q] - P.own_lo);
+    if (hub) append_hub_A<kBfsFilter>(P, x[q], slot);
+    qA.push(keep[q] && !hub, x[q], 0, P.listA[slot], nullptr, &P.ctl->cnt_A[slot]);
+    cnt += __popc(__ballot_sync(0xffffffffu, nw[q]));
+  }
+  return cnt;
 }
 
-// Expand the out-edges of up to 32 source vertices (one per lane).
+// Expand the out-edges of up to 32 source vertices (one per lane, degree <=
+// kHubDegree): their edge ranges are concatenated and walked 32*kBatch edges at
+// a time; each element finds its source lane by a shuffle binary search over
+// the warp's exclusive degree prefix.
 template <bool kBfsFilter, class OffT>
 __device__ uint32_t expand_warp(const Part<OffT> &P, bool valid, uint64_t beg, uint32_t deg, uint32_t epoch,
                                 const uint32_t *hub_bits, WarpQueue &qA, uint32_t slot) {
   const uint32_t lane = lane_id();
-  uint32_t nact = 0;
-  uint32_t big = __ballot_sync(0xffffffffu, valid && deg > 32);
-  while (big) {
-    const int L = __ffs(big) - 1;
-    big &= big - 1;
-    const uint64_t b = __shfl_sync(0xffffffffu, beg, L);
-    const uint32_t d = __shfl_sync(0xffffffffu, deg, L);
-    for (uint32_t r0 = 0; r0 < d; r0 += 32) {
-      const uint32_t k = r0 + lane;
-      const bool act = k < d;
-      const uint32_t x = act ? ldg_nc(P.out_dst + b + k) : 0u;
-      nact += activate_lanes<kBfsFilter>(P, act, x, epoch, hub_bits, qA, slot);
-    }
-  }
-  const uint32_t sd = (valid && deg <= 32) ? deg : 0u;
-  const uint32_t incl = warp_incl_scan(sd);
-  const uint32_t excl = incl - sd;
+  const uint32_t d = valid ? deg : 0u;
+  const uint32_t incl = warp_incl_scan(d);
+  const uint32_t excl = incl - d;
   const uint32_t total = __shfl_sync(0xffffffffu, incl, 31);
-  for (uint32_t r0 = 0; r0 < total; r0 += 32) {
-    const uint32_t k = r0 + lane;
-    int o = 0;
+  uint32_t nact = 0;
+  for (uint32_t r0 = 0; r0 < total; r0 += 32u * kBatch) {
+    bool act[kBatch];
+    uint32_t x[kBatch];
 #pragma unroll
-    for (int step = 16; step > 0; step >>= 1) {
-      const uint32_t e = __shfl_sync(0xffffffffu, excl, o + step);
-      if (e <= k) o += step;
+    for (int q = 0; q < kBatch; q++) {
+      const uint32_t k = r0 + q * 32u + lane;
+      int o = 0;
+#pragma unroll
+      for (int step = 16; step > 0; step >>= 1) {
+        const uint32_t e = __shfl_sync(0xffffffffu, excl, o + step);
+        if (e <= k) o += step;
+      }
+      const uint64_t ob = __shfl_sync(0xffffffffu, beg, o);
+      const uint32_t oe = __shfl_sync(0xffffffffu, excl, o);
+      act[q] = k < total;
+      x[q] = act[q] ? ldg_nc(P.out_dst + ob + (k - oe)) : 0u;
     }
-    const uint64_t ob = __shfl_sync(0xffffffffu, beg, o);
-    const uint32_t oe = __shfl_sync(0xffffffffu, excl, o);
-    const bool act = k < total;
-    const uint32_t x = act ? ldg_nc(P.out_dst + ob + (k - oe)) : 0u;
-    nact += activate_lanes<kBfsFilter>(P, act, x, epoch, hub_bits, qA, slot);
+    nact += activate_batch<kBfsFilter>(P, act, x, epoch, hub_bits, qA, slot);
   }
   return nact;  // warp-uniform
 }
 
-// Block-wide expansion of one hub source (all warps, uniform rounds).
+// Block-wide expansion of one hub chunk (contiguous out-edges).
 template <bool kBfsFilter, class OffT>
 __device__ uint32_t expand_block(const Part<OffT> &P, uint64_t beg, uint32_t deg, uint32_t epoch,
                                  const uint32_t *hub_bits, WarpQueue &qA, uint32_t slot) {
   uint32_t nact = 0;
-  for (uint32_t r0 = 0; r0 < deg; r0 += kBlock) {
-    const uint32_t k = r0 + threadIdx.x;
-    const bool act = k < deg;
-    const uint32_t x = act ? ldg_nc(P.out_dst + beg + k) : 0u;
-    nact += activate_lanes<kBfsFilter>(P, act, x, epoch, hub_bits, qA, slot);
+  for (uint32_t r0 = 0; r0 < deg; r0 += kBlock * kBatch) {
+    bool act[kBatch];
+    uint32_t x[kBatch];
+#pragma unroll
+    for (int q = 0; q < kBatch; q++) {
+      const uint32_t k = r0 + q * kBlock + threadIdx.x;
+      act[q] = k < deg;
+      x[q] = act[q] ? ldg_nc(P.out_dst + beg + k) : 0u;
+    }
+    nact += activate_batch<kBfsFilter>(P, act, x, epoch, hub_bits, qA, slot);
   }
   return nact;  // per-warp count
 }
 
-// Last CTA of the superstep's final kernel closes superstep t.
+// Last CTA of the superstep's final kernel closes superstep t. The ticket is
+// two-level (groups of 32 CTAs) so no single address takes one atomic per CTA;
+// the whole last CTA sums the spread counter slots in parallel.
 template <class OffT>
 __device__ void finish_superstep(const Part<OffT> &P, unsigned long long cond_handle, int use_graph) {
   __shared__ bool s_last;
+  __shared__ unsigned long long s_red[4][kWarpsPerBlock];
   __syncthreads();
   if (threadIdx.x == 0) {
     __threadfence();
-    const uint32_t tk = atomicAdd(&P.ctl->done_blocks, 1u);
-    s_last = (tk == gridDim.x - 1);
+    Ctl *cc = P.ctl;
+    const uint32_t grp = blockIdx.x >> 5, ngrp = (gridDim.x + 31) >> 5;
+    const uint32_t gsize = min(32u, gridDim.x - grp * 32u);
+    bool last = false;
+    if (atomicAdd(&cc->tick1[grp], 1u) == gsize - 1) {
+      cc->tick1[grp] = 0;
+      __threadfence();
+      if (atomicAdd(&cc->tick2, 1u) == ngrp - 1) {
+        cc->tick2 = 0;
+        last = true;
+      }
+    }
+    s_last = last;
   }
   __syncthreads();
-  if (!s_last || threadIdx.x != 0) return;
+  if (!s_last) return;
   __threadfence();
   volatile Ctl *c = P.ctl;
+  {
+    unsigned long long v[4] = {0, 0, 0, 0};
+    if (threadIdx.x < kSlots) {
+      const uint32_t i = threadIdx.x;
+      v[0] = c->part_g[i]; v[1] = c->part_c[i]; v[2] = c->part_s[i]; v[3] = c->part_a[i];
+      c->part_g[i] = 0; c->part_c[i] = 0; c->part_s[i] = 0; c->part_a[i] = 0;
+    }
+#pragma unroll
+    for (int k = 0; k < 4; k++) {
+#pragma unroll
+      for (int o = 16; o > 0; o >>= 1) v[k] += __shfl_xor_sync(0xffffffffu, v[k], o);
+      if (lane_id() == 0) s_red[k][threadIdx.x >> 5] = v[k];
+    }
+  }
+  __syncthreads();
+  if (threadIdx.x != 0) return;
+  unsigned long long sg = 0, sc = 0, ss = 0, sa = 0;
+  for (int w = 0; w < kWarpsPerBlock; w++) { sg += s_red[0][w]; sc += s_red[1][w]; ss += s_red[2][w]; sa += s_red[3][w]; }
   const uint32_t t = c->iter, slot = t & 1u, ns = slot ^ 1u;
+  c->gathered = c->gathered + sg;
+  c->changed = c->changed + sc;
+  c->scattered = c->scattered + ss;
+  c->cnt_act[ns] = c->cnt_act[ns] + (uint32_t)sa;
   if (t < c->trace_cap) {
     volatile unsigned long long *row = P.trace + 4ull * t;
     row[0] = c->cnt_act[slot];
@@ -286,9 +361,8 @@ __device__ void finish_superstep(const Part<OffT> &P, unsigned long long cond_ha
   c->cnt_A[slot] = 0;
   c->cnt_H[slot] = 0;
   c->cnt_act[slot] = 0;
-  c->done_blocks = 0;
   c->iter = t + 1;
-  const bool stop = (c->cnt_act[ns] == 0) || (c->max_iters != 0 && t + 1 >= c->max_iters);
+  const bool stop = !c->ext_loop && ((c->cnt_act[ns] == 0) || (c->max_iters != 0 && t + 1 >= c->max_iters));
   c->stop = stop ? 1u : 0u;
   __threadfence();
   if (use_graph) cudaGraphSetConditional((cudaGraphConditionalHandle)cond_handle, stop ? 0u : 1u);
@@ -308,12 +382,15 @@ __global__ void __launch_bounds__(kBlock) k_gather_apply(const __grid_constant__
   const uint32_t nK = *(volatile uint32_t *)&ctl->cnt_K[slot];
   const uint32_t *LA = P.listA[slot];
   const uint32_t *LH = P.listH[slot];
+  const bool no_hub_c = ctl->no_hub_c != 0;
   prof_begin(ctl, 0);
 
   __shared__ uint32_t sq[kWarpsPerBlock][2][kQueueCap];
   __shared__ uint32_t sred[kWarpsPerBlock][32];
   __shared__ G sblk[kWarpsPerBlock];
   __shared__ uint32_t s_h;
+  __shared__ uint32_t s_off[kWarpsPerBlock + 1];
+  __shared__ unsigned long long s8[kWarpsPerBlock];
   const uint32_t warp = threadIdx.x / 32, lane = lane_id();
   WarpQueue qC{sq[warp][0], sq[warp][1], 0};
   unsigned long long my_g = 0, my_c = 0;
@@ -330,23 +407,25 @@ __global__ void __launch_bounds__(kBlock) k_gather_apply(const __grid_constant__
     uint64_t beg = 0;
     uint32_t deg = 0, cur = 0;
     if (valid) {
-      beg = (uint64_t)P.in_off[lv];
-      deg = (uint32_t)((uint64_t)P.in_off[lv + 1] - beg);
+      if (Prog::kHasGather) {
+        beg = (uint64_t)P.in_off[lv];
+        deg = (uint32_t)((uint64_t)P.in_off[lv + 1] - beg);
+      }
       cur = P.val[v];
     }
-    const G acc = gather_warp<Prog>(P, valid, beg, deg, cur, sred[warp], cx);
+    const G acc = Prog::kHasGather ? gather_warp<Prog>(P, valid, beg, deg, cur, sred[warp], cx) : Prog::identity();
     bool changed = false;
     uint32_t nv = cur;
     if (valid) {
       changed = Prog::apply(&nv, acc, cx);
       my_g += deg;
     }
-    const bool hubo = changed && test_bit(P.hub_out, v);
+    const bool hubo = changed && !no_hub_c && test_bit(P.hub_out, v);
     if (hubo) append_hub_C(P, v, nv);
     qC.push(changed && !hubo, v, nv, P.C_v, P.C_val, &ctl->cnt_C);
     my_c += changed ? 1 : 0;
   }
-  qC.flush(P.C_v, P.C_val, &ctl->cnt_C);
+  qC.block_flush(P.C_v, P.C_val, &ctl->cnt_C, s_off);
 
   // Phase 2: hub chunks (kChunk in-edges each), dynamic over CTAs. Chunk results
   // combine with Prog::atomicGather (exact for min); the last chunk applies.
@@ -363,10 +442,11 @@ __global__ void __launch_bounds__(kBlock) k_gather_apply(const __grid_constant__
     const uint64_t b = beg + (uint64_t)ci * kChunk;
     const uint32_t len = chunk_len(deg, ci);
     const uint32_t cur = P.val[v];
-    const G r = gather_block<Prog>(P, b, len, cur, sblk, cx);
+    if (!Prog::kHasGather && ci != 0) continue;  // no gather: chunk 0 applies
+    const G r = Prog::kHasGather ? gather_block<Prog>(P, b, len, cur, sblk, cx) : Prog::identity();
     if (threadIdx.x == 0) {
-      const uint32_t nch = (uint32_t)((deg + kChunk - 1) / kChunk);
-      if (ci == 0) my_g += deg;
+      const uint32_t nch = Prog::kHasGather ? (uint32_t)((deg + kChunk - 1) / kChunk) : 1u;
+      if (ci == 0 && Prog::kHasGather) my_g += deg;
       bool fin = (nch == 1);
       G acc = r;
       if (!fin) {
@@ -383,7 +463,7 @@ __global__ void __launch_bounds__(kBlock) k_gather_apply(const __grid_constant__
         uint32_t nv = cur;
         if (Prog::apply(&nv, acc, cx)) {
           my_c += 1;
-          if (test_bit(P.hub_out, v)) append_hub_C(P, v, nv);
+          if (!no_hub_c && test_bit(P.hub_out, v)) append_hub_C(P, v, nv);
           else {
             const uint32_t pos = atomicAdd(&ctl->cnt_C, 1u);
             P.C_v[pos] = v;
@@ -393,12 +473,10 @@ __global__ void __launch_bounds__(kBlock) k_gather_apply(const __grid_constant__
       }
     }
   }
-  my_g = warp_sum_u64(my_g);
-  my_c = warp_sum_u64(my_c);
-  if (lane == 0) {
-    if (my_g) atomicAdd(&ctl->gathered, my_g);
-    if (my_c) atomicAdd(&ctl->changed, my_c);
-  }
+  my_g = block_sum_u64(my_g, s8);
+  if (threadIdx.x == 0 && my_g) atomicAdd(&ctl->part_g[blockIdx.x % kSlots], my_g);
+  my_c = block_sum_u64(my_c, s8);
+  if (threadIdx.x == 0 && my_c) atomicAdd(&ctl->part_c[blockIdx.x % kSlots], my_c);
   prof_end(ctl, 0);
 }
 
@@ -420,6 +498,8 @@ __global__ void __launch_bounds__(kBlock) k_activate(const __grid_constant__ Par
 
   __shared__ uint32_t sq[kWarpsPerBlock][kQueueCap];
   __shared__ uint32_t s_h;
+  __shared__ uint32_t s_off[kWarpsPerBlock + 1];
+  __shared__ unsigned long long s8[kWarpsPerBlock];
   const uint32_t warp = threadIdx.x / 32, lane = lane_id();
   WarpQueue qA{sq[warp], nullptr, 0};
   unsigned long long my_s = 0, my_act = 0;
@@ -458,12 +538,11 @@ __global__ void __launch_bounds__(kBlock) k_activate(const __grid_constant__ Par
     const uint32_t a = expand_block<false>(P, beg + (uint64_t)ci * kChunk, len, epoch, P.hub_in, qA, ns);
     if (lane == 0) my_act += a;
   }
-  qA.flush(P.listA[ns], nullptr, &ctl->cnt_A[ns]);
-  my_s = warp_sum_u64(my_s);
-  if (lane == 0) {
-    if (my_s) atomicAdd(&ctl->scattered, my_s);
-    if (my_act) atomicAdd(&ctl->cnt_act[ns], (uint32_t)my_act);
-  }
+  qA.block_flush(P.listA[ns], nullptr, &ctl->cnt_A[ns], s_off);
+  my_s = block_sum_u64(my_s, s8);
+  if (threadIdx.x == 0 && my_s) atomicAdd(&ctl->part_s[blockIdx.x % kSlots], my_s);
+  my_act = block_sum_u64(lane == 0 ? my_act : 0ull, s8);
+  if (threadIdx.x == 0 && my_act) atomicAdd(&ctl->part_a[blockIdx.x % kSlots], my_act);
   prof_end(ctl, 1);
   finish_superstep(P, cond, use_graph);
 }
@@ -490,6 +569,8 @@ __global__ void __launch_bounds__(kBlock) k_bfs_expand(const __grid_constant__ P
   __shared__ uint32_t sq[kWarpsPerBlock][kQueueCap];
   __shared__ uint32_t s_h;
   __shared__ bool s_changed;
+  __shared__ uint32_t s_off[kWarpsPerBlock + 1];
+  __shared__ unsigned long long s8[kWarpsPerBlock];
   const uint32_t warp = threadIdx.x / 32, lane = lane_id();
   WarpQueue qA{sq[warp], nullptr, 0};
   unsigned long long my_s = 0, my_c = 0, my_act = 0;
@@ -540,16 +621,37 @@ __global__ void __launch_bounds__(kBlock) k_bfs_expand(const __grid_constant__ P
     const uint32_t a = expand_block<true>(P, beg + (uint64_t)ci * kChunk, len, epoch, P.hub_out, qA, ns);
     if (lane == 0) my_act += a;
   }
-  qA.flush(P.listA[ns], nullptr, &ctl->cnt_A[ns]);
-  my_s = warp_sum_u64(my_s);
-  my_c = warp_sum_u64(my_c);
-  if (lane == 0) {
-    if (my_s) atomicAdd(&ctl->scattered, my_s);
-    if (my_c) atomicAdd(&ctl->changed, my_c);
-    if (my_act) atomicAdd(&ctl->cnt_act[ns], (uint32_t)my_act);
-  }
+  qA.block_flush(P.listA[ns], nullptr, &ctl->cnt_A[ns], s_off);
+  my_s = block_sum_u64(my_s, s8);
+  if (threadIdx.x == 0 && my_s) atomicAdd(&ctl->part_s[blockIdx.x % kSlots], my_s);
+  my_c = block_sum_u64(my_c, s8);
+  if (threadIdx.x == 0 && my_c) atomicAdd(&ctl->part_c[blockIdx.x % kSlots], my_c);
+  my_act = block_sum_u64(lane == 0 ? my_act : 0ull, s8);
+  if (threadIdx.x == 0 && my_act) atomicAdd(&ctl->part_a[blockIdx.x % kSlots], my_act);
   prof_end(ctl, 1);
   finish_superstep(P, cond, use_graph);
+}
+
+// Partitioned runs: split the exchanged changed set (every rank's C_t) into
+// the local non-hub list and the local changed-hub chunks (hub-ness depends on
+// this rank's activation CSR).
+template <class OffT>
+__global__ void __launch_bounds__(kBlock) k_classify(const __grid_constant__ Part<OffT> P, const uint32_t *X_v,
+                                                     const uint32_t *X_val, uint32_t nX) {
+  __shared__ uint32_t sq[kWarpsPerBlock][2][kQueueCap];
+  __shared__ uint32_t s_off[kWarpsPerBlock + 1];
+  const uint32_t warp = threadIdx.x / 32, lane = lane_id();
+  WarpQueue qC{sq[warp][0], sq[warp][1], 0};
+  const uint32_t gw = blockIdx.x * kWarpsPerBlock + warp, nw = gridDim.x * kWarpsPerBlock;
+  for (uint32_t base = gw * 32u; base < nX; base += nw * 32u) {
+    const uint32_t i = base + lane;
+    const bool valid = i < nX;
+    const uint32_t u = valid ? X_v[i] : 0u, val = valid ? X_val[i] : 0u;
+    const bool hub = valid && test_bit(P.hub_out, u);
+    if (hub) append_hub_C(P, u, val);
+    qC.push(valid && !hub, u, val, P.C_v, P.C_val, &P.ctl->cnt_C);
+  }
+  qC.block_flush(P.C_v, P.C_val, &P.ctl->cnt_C, s_off);
 }
 
 // ----------------------------------------------------------- initialisation

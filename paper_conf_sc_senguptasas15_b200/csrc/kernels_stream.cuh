@@ -134,7 +134,7 @@ __global__ void __launch_bounds__(kBlock) k_s_activate(const __grid_constant__ P
     uint32_t big = __ballot_sync(0xffffffffu, valid && deg > 32);
     auto act_one = [&](bool act, uint32_t x) {
       bool newly = false;
-      if (act) newly = atomicExch(P.stamp + (x - P.own_lo), epoch_n) != epoch_n;
+      if (act) newly = stamp_first(P.stamp + (x - P.own_lo), epoch_n);
       if (newly) next_flags[shard_of(bounds, nshards, x)] = 1;
       return (uint32_t)__popc(__ballot_sync(0xffffffffu, newly));
     };
