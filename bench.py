@@ -28,6 +28,7 @@ CONFIG_NAMES = {
     2: "cfg2: PageRank x30 d=0.85 fp32, R-MAT s22 ef16 (4,194,304 V / 67,108,864 E), resident",
     3: "cfg3: SSSP from 0, road-like grid 4894x4894 weights 1-64, resident",
     4: "cfg4: CC, web-like power law n=18,520,486 (uk-2002 shape), symmetrized, resident",
+    5: "cfg5 shape: PageRank x30 on R-MAT ef16, host-streamed shards (K=2 slots) at 1 GPU",
 }
 
 
@@ -91,9 +92,14 @@ class ClockSampler:
                 "samples": len(sm)}
 
 
-def make_graph(cfg: int):
+def make_graph(cfg: int, scale: int = 26):
     import grgen
 
+    if cfg == 5:
+        # SURVEY §8(d) cfg5 is s = 31 (275 GB of COO): more than this box's 196 GB of host RAM,
+        # so the shape is kept (R-MAT ef16, seed 5) at the largest scale the host can build
+        g = grgen.rmat(scale, 16, seed=5)
+        return g, None, dict(algo="pagerank", max_iters=30, damping=0.85)
     g, run = grgen.config(cfg)
     w = g.get("w")
     if run["algo"] == "sssp" and w is None:
@@ -135,6 +141,24 @@ def cpu_oracle_sample(g, w, run, budget_s=20.0):
         og.close()
 
 
+def measure_h2d():
+    import torch
+
+    n = 1 << 30
+    h = torch.empty(n, dtype=torch.uint8).pin_memory()
+    d = torch.empty(n, dtype=torch.uint8, device="cuda")
+    best = 1e9
+    for _ in range(5):
+        a, b = torch.cuda.Event(enable_timing=True), torch.cuda.Event(enable_timing=True)
+        a.record()
+        d.copy_(h, non_blocking=True)
+        b.record()
+        torch.cuda.synchronize()
+        best = min(best, a.elapsed_time(b))
+    del h, d
+    return n / (best * 1e-3) / 1e9
+
+
 def load_traffic(kernel):
     p = os.path.join(ROOT, "profiles", "traffic.json")
     if os.path.exists(p):
@@ -151,8 +175,9 @@ def main():
     ap.add_argument("--impl", default="ours", choices=["ours", "reference"])
     ap.add_argument("--config", type=int, default=2)
     ap.add_argument("--e2e-steps", type=int, default=2)
+    ap.add_argument("--scale", type=int, default=26, help="R-MAT scale for --config 5")
     ap.add_argument("--no-cpu", action="store_true")
-    ap.add_argument("--loop", default="auto", choices=["auto", "host", "device"],
+    ap.add_argument("--loop", default="auto", choices=["auto", "host", "device", "persistent"],
                     help="superstep loop for frontier programs (host: profilable by ncu)")
     args = ap.parse_args()
 
@@ -163,7 +188,7 @@ def main():
     if args.impl == "reference":
         if rank != 0:
             return 0
-        g, w, run = make_graph(args.config)
+        g, w, run = make_graph(args.config, args.scale)
         per_step = []
         for i in range(args.warmup + args.steps):
             cb = cpu_oracle_sample(g, w, run)
@@ -190,12 +215,21 @@ def main():
     import paper_conf_sc_senguptasas15_b200 as gr
 
     t0 = time.perf_counter()
-    g, w, run = make_graph(args.config)
+    g, w, run = make_graph(args.config, args.scale)
     print(f"[bench] generated {g.name}: n={g.n} m={g.m} in {time.perf_counter() - t0:.1f}s", file=sys.stderr)
     algo = run["algo"]
     kw = dict(source=run.get("source", 0), max_iters=run.get("max_iters", 0), damping=run.get("damping", 0.85),
               loop=args.loop)
-    G = gr.GraphReduce(g.n, g.src, g.dst, w, device=local_rank, mode="resident")
+    part = {}
+    if world > 1:
+        # NCCL bootstrap: rank 0 creates the unique id, the torch process group broadcasts it
+        uid = torch.zeros(128, dtype=torch.uint8, device="cuda")
+        if rank == 0:
+            uid.copy_(torch.frombuffer(bytearray(gr.gr_get_unique_id()), dtype=torch.uint8))
+        torch.distributed.broadcast(uid, 0)
+        part = dict(world=world, rank=rank, nccl_unique_id=bytes(uid.cpu().numpy().tobytes()))
+    mode = "streamed" if args.config == 5 else "resident"
+    G = gr.GraphReduce(g.n, g.src, g.dst, w, device=local_rank, mode=mode, **part)
     info = G.info()
     print(f"[bench] loaded in {time.perf_counter() - t0:.1f}s total: {info}", file=sys.stderr)
     stream = torch.cuda.current_stream()
@@ -225,7 +259,7 @@ def main():
         torch.distributed.barrier()
     ms_step = ms / args.steps
     edges = metric_edges(run, stats, g.m)
-    value = edges * world / (ms_step * 1e-3) / 1e9
+    value = edges / (ms_step * 1e-3) / 1e9  # edges are global (whole job) in every mode
 
     # roofline of the dominant kernel (algorithmic bytes per launch / CUDA-event duration)
     peak, peak_src = peaks()
@@ -239,12 +273,22 @@ def main():
         bytes_per_launch = stats["bytes_hbm_model"] / launches_per_step
         kname = "k_gather_apply" if algo != "bfs" else "k_bfs_expand"
     avg_launch_s = (kms / args.steps) * 1e-3 / launches_per_step
+    if avg_launch_s <= 0:  # no per-kernel timing on this path: fall back to the whole step
+        avg_launch_s = ms_step * 1e-3 / launches_per_step
     achieved = bytes_per_launch / avg_launch_s / 1e9
     roof = {"bound": "hbm", "kernel": kname, "achieved": round(achieved, 1), "peak": peak, "unit": "GB/s",
             "frac": round(achieved / peak, 4), "peak_source": peak_src,
             "bytes_per_launch": int(bytes_per_launch), "avg_launch_us": round(avg_launch_s * 1e6, 2),
             "kernel_share_of_step": round(kms / ms, 4) if ms > 0 else None,
             "traffic": load_traffic(kname)}
+    if mode == "streamed":
+        h2d_peak = measure_h2d()
+        h2d_rate = stats["bytes_h2d"] / (ms_step * 1e-3) / 1e9
+        roof = {"bound": "host_link", "kernel": "H2D shard streamer (cudaMemcpyAsync, 2 slots)",
+                "achieved": round(h2d_rate, 2), "peak": round(h2d_peak, 2), "unit": "GB/s",
+                "frac": round(h2d_rate / h2d_peak, 4),
+                "peak_source": "measured in this run: pinned 1 GiB H2D cudaMemcpy, best of 5",
+                "bytes_per_step": stats["bytes_h2d"], "traffic": None}
     run_roof = {"bytes_hbm_model_per_step": stats["bytes_hbm_model"],
                 "frac_of_step": round(stats["bytes_hbm_model"] / (ms_step * 1e-3) / 1e9 / peak, 4)}
 
@@ -256,13 +300,13 @@ def main():
     out = torch.empty(n, dtype=torch.float32 if algo == "pagerank" else torch.int32).pin_memory().numpy()
     for i in range(args.e2e_steps):
         t0 = time.perf_counter()
-        H = gr.gr_graph_load(n, src_p, dst_p, w_p, device=local_rank, mode="resident")
+        H = gr.gr_graph_load(n, src_p, dst_p, w_p, device=local_rank, mode=mode, **part)
         gr.gr_run(H, algo, **kw)
         gr.gr_fetch_vertex_values(H, out)
         dt = time.perf_counter() - t0
         inf = gr.gr_graph_info_get(H)
         gr.gr_graph_free(H)
-        e2e_vals.append(edges * world / dt / 1e9)
+        e2e_vals.append(edges / dt / 1e9)
     h2d = int(8 * m + (m if w is not None else 0))  # CSC + CSR payloads (+weights) per load
     h2d += 8 * (n + 1) * 2 // (2 if not info["offsets_64bit"] else 1)
     e2e = {"value": float(np.median(e2e_vals)) if e2e_vals else None, "unit": "GTEPS", "h2d_bytes_per_step": h2d,
@@ -270,7 +314,7 @@ def main():
            "what": "gr_graph_load(host COO: shard build + H2D) + gr_run + gr_fetch_vertex_values, wall clock"}
 
     cpu = None
-    if rank == 0 and world == 1 and not args.no_cpu:
+    if rank == 0 and world == 1 and not args.no_cpu and args.config != 5:
         cpu = cpu_oracle_sample(g, w, run)
 
     G.close()
@@ -281,7 +325,8 @@ def main():
             "higher_is_better": True, "scaling": "strong", "vs_baseline": None,
             "dtype": "f32" if algo == "pagerank" else "u32", "data": "synthetic",
             "config": {"workload": CONFIG_NAMES[args.config], "n": n, "m": m, "shards": info["num_shards"],
-                       "mode": "resident", "l2": "inputs larger than L2 (CSC payload > 126 MB L2); no flush",
+                       "mode": mode, "parallelism": f"dst-interval partitions x{world}" if world > 1 else "1 GPU",
+                       "l2": "inputs larger than L2 (CSC payload > 126 MB L2); no flush",
                        "iterations": stats["iterations"]},
             "roofline": roof, "run_roofline": run_roof, "cpu_baseline": cpu, "e2e": e2e,
             "gpu_launches": launches, "clocks": ck,

@@ -65,9 +65,10 @@ typedef enum gr_mode {
 } gr_mode;
 
 typedef enum gr_loop {
-  GR_LOOP_AUTO = 0,   /* device-side loop where supported */
-  GR_LOOP_HOST = 1,   /* host reads the frontier count after every superstep */
-  GR_LOOP_DEVICE = 2  /* CUDA graph with a conditional WHILE node (no host round trip) */
+  GR_LOOP_AUTO = 0,       /* persistent loop where supported (single rank, resident), else host */
+  GR_LOOP_HOST = 1,       /* host reads the frontier count after every superstep */
+  GR_LOOP_DEVICE = 2,     /* CUDA graph with a conditional WHILE node (no host round trip) */
+  GR_LOOP_PERSISTENT = 3  /* one cooperative kernel runs every superstep; grid barriers between phases */
 } gr_loop;
 
 /* Input graph (caller-owned; the library copies what it needs during load). */

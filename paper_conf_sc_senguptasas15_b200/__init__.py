@@ -25,7 +25,7 @@ STATUS_NAMES = ["GR_OK", "GR_EINVAL", "GR_ENOMEM", "GR_ECUDA", "GR_ENCCL", "GR_E
 GR_FMT_COO, GR_FMT_CSR = 0, 1
 ALGOS = {"bfs": 0, "sssp": 1, "pagerank": 2, "cc": 3, "custom": 4}
 MODES = {"auto": 0, "resident": 1, "streamed": 2}
-LOOPS = {"auto": 0, "host": 1, "device": 2}
+LOOPS = {"auto": 0, "host": 1, "device": 2, "persistent": 3}
 INF = 0xFFFFFFFF
 
 EXPORTS = [

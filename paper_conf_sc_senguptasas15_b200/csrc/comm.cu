@@ -3,6 +3,7 @@
 
 #include <nccl.h>
 
+#include <chrono>
 #include <condition_variable>
 #include <cstring>
 #include <map>
@@ -58,17 +59,26 @@ struct SimGroup {
   std::vector<const void *> ptrs;
   std::vector<uint64_t> small;  // world * 8
   int members = 0;
+  bool poisoned = false;        // a rank failed: every waiter returns an error
 
-  void barrier() {
+  bool barrier() {
     std::unique_lock<std::mutex> lk(mu);
+    if (poisoned) return false;
     const uint64_t g = gen;
     if (++arrived == world) {
       arrived = 0;
       gen++;
       cv.notify_all();
     } else {
-      cv.wait(lk, [&] { return gen != g; });
+      cv.wait_for(lk, std::chrono::seconds(300), [&] { return gen != g || poisoned; });
+      if (gen == g) { poisoned = true; cv.notify_all(); return false; }
     }
+    return !poisoned;
+  }
+  void poison() {
+    std::lock_guard<std::mutex> lk(mu);
+    poisoned = true;
+    cv.notify_all();
   }
 };
 
@@ -82,30 +92,34 @@ struct SimComm : Comm {
     std::lock_guard<std::mutex> lk(g_sim_mu);
     if (--grp->members == 0) g_sim_groups.erase(key);
   }
+  gr_status fail_all(gr_status s) {
+    grp->poison();
+    return s;
+  }
   gr_status allgatherv(const void *send, void *recv, const std::vector<uint64_t> &counts,
                        const std::vector<uint64_t> &displs, cudaStream_t s) override {
-    if (cudaStreamSynchronize(s) != cudaSuccess) return GR_ECUDA;  // own data ready
+    if (cudaStreamSynchronize(s) != cudaSuccess) return fail_all(GR_ECUDA);  // own data ready
     grp->ptrs[rank] = send;
-    grp->barrier();
+    if (!grp->barrier()) return GR_ENCCL;
     for (int q = 0; q < world; q++) {
       char *dst = static_cast<char *>(recv) + displs[q];
       if (!counts[q] || grp->ptrs[q] == dst) continue;
       if (cudaMemcpyAsync(dst, grp->ptrs[q], counts[q], cudaMemcpyDeviceToDevice, s) != cudaSuccess)
-        return GR_ECUDA;
+        return fail_all(GR_ECUDA);
       if (q != rank) bytes_in += counts[q];
     }
-    if (cudaStreamSynchronize(s) != cudaSuccess) return GR_ECUDA;
-    grp->barrier();  // peers may reuse their send buffers only after everyone copied
+    if (cudaStreamSynchronize(s) != cudaSuccess) return fail_all(GR_ECUDA);
+    if (!grp->barrier()) return GR_ENCCL;  // peers may reuse their send buffers only after everyone copied
     return GR_OK;
   }
   gr_status allgather_small(const uint64_t *mine, int k, uint64_t *out, cudaStream_t s) override {
-    if (k > 8) return GR_EINVAL;
-    if (cudaStreamSynchronize(s) != cudaSuccess) return GR_ECUDA;
+    if (k > 8) return fail_all(GR_EINVAL);
+    if (cudaStreamSynchronize(s) != cudaSuccess) return fail_all(GR_ECUDA);
     for (int i = 0; i < k; i++) grp->small[rank * 8 + i] = mine[i];
-    grp->barrier();
+    if (!grp->barrier()) return GR_ENCCL;
     for (int q = 0; q < world; q++)
       for (int i = 0; i < k; i++) out[q * k + i] = grp->small[q * 8 + i];
-    grp->barrier();
+    if (!grp->barrier()) return GR_ENCCL;
     return GR_OK;
   }
 };
@@ -131,13 +145,13 @@ gr_status comm_create(int world, int rank, bool sim, const void *id128, int devi
         g->ptrs.assign(world, nullptr);
         g->small.assign(8ull * world, 0);
       }
+      g->members++;
+      c->grp = g;
       if (g->world != world) {
         delete c;
         *err = "simulated group world mismatch";
         return GR_EINVAL;
       }
-      g->members++;
-      c->grp = g;
     }
     *out = c;
     return GR_OK;

@@ -45,6 +45,7 @@ struct Ctl {
   uint32_t tick1[64];     // two-level last-CTA ticket: groups of 32 CTAs
   uint32_t tick2;
   uint32_t ext_loop;      // partitioned runs: the host decides termination (global counts)
+  uint32_t bar_count, bar_gen;  // grid barrier of the persistent loop
   uint32_t no_hub_c;      // partitioned runs: changed hubs are classified after the exchange
   unsigned long long prof;               // 1: kernels stamp %globaltimer
   unsigned long long kstart[2], kend[2]; // per-kernel span of the current superstep (ns)

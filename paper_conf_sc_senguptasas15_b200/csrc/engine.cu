@@ -14,6 +14,7 @@
 
 #include <algorithm>
 #include <cstdarg>
+#include <cstdlib>
 #include <cstdio>
 #include <cstring>
 #include <map>
@@ -155,10 +156,13 @@ gr_status load_device(gr_graph *g) {
     if ((s = dev_alloc(g, (void **)&g->listA[i], 4 * ow)) != GR_OK) return s;
     if ((s = dev_alloc(g, (void **)&g->listH[i], 4 * ow)) != GR_OK) return s;
   }
-  if ((s = dev_alloc(g, (void **)&g->C_v, 4 * ow)) != GR_OK) return s;
-  if ((s = dev_alloc(g, (void **)&g->C_val, 4 * ow)) != GR_OK) return s;
-  if ((s = dev_alloc(g, (void **)&g->CH_v, 4 * ow)) != GR_OK) return s;
-  if ((s = dev_alloc(g, (void **)&g->CH_val, 4 * ow)) != GR_OK) return s;
+  // changed lists: owned vertices only, except in partitioned runs where the
+  // exchanged changed set of every rank is classified into them
+  const size_t cw = H.owners.size() > 2 ? std::max<uint64_t>(n, 1) : ow;
+  if ((s = dev_alloc(g, (void **)&g->C_v, 4 * cw)) != GR_OK) return s;
+  if ((s = dev_alloc(g, (void **)&g->C_val, 4 * cw)) != GR_OK) return s;
+  if ((s = dev_alloc(g, (void **)&g->CH_v, 4 * cw)) != GR_OK) return s;
+  if ((s = dev_alloc(g, (void **)&g->CH_val, 4 * cw)) != GR_OK) return s;
   if ((s = dev_alloc(g, (void **)&g->ctl, sizeof(Ctl))) != GR_OK) return s;
   g->trace_cap = 1u << 20;
   if ((s = dev_alloc(g, (void **)&g->trace, 32ull * g->trace_cap)) != GR_OK) return s;
@@ -194,6 +198,9 @@ gr_status load_device(gr_graph *g) {
   int bps = 0;
   CK(cudaOccupancyMaxActiveBlocksPerMultiprocessor(&bps, k_gather_apply<ProgCC, uint32_t>, kBlock, 0));
   g->grid_frontier = g->num_sms * std::max(1, std::min(bps, 8));
+  int coop = 0;
+  cudaDeviceGetAttribute(&coop, cudaDevAttrCooperativeLaunch, g->device);
+  g->coop = coop != 0;
   return GR_OK;
 }
 
@@ -279,8 +286,18 @@ static gr_status run_frontier(gr_graph *g, const gr_run_opts *o, cudaStream_t s,
   k_init_frontier<Prog, OffT><<<1, kBlock, 0, s>>>(P, o->source, g->n_static_hubs, g->n_static_chunks);
   launches++;
   CK(cudaGetLastError());
-  const bool use_graph = (o->loop != GR_LOOP_HOST);
-  if (use_graph) {
+  const bool persistent = (o->loop == GR_LOOP_AUTO || o->loop == GR_LOOP_PERSISTENT) && g->coop;
+  const bool use_graph = !persistent && (o->loop == GR_LOOP_DEVICE || o->loop == GR_LOOP_AUTO);
+  if (persistent) {
+    int bps = 0;
+    CK(cudaOccupancyMaxActiveBlocksPerMultiprocessor(&bps, k_persistent<Prog, OffT>, kBlock, 0));
+    const uint32_t grid = (uint32_t)g->num_sms * (uint32_t)std::max(1, std::min(bps, 4));
+    void *args[] = {(void *)&P};
+    CK(cudaLaunchCooperativeKernel((const void *)k_persistent<Prog, OffT>, dim3(grid), dim3(kBlock), args, 0, s));
+    CK(cudaMemcpyAsync(g->h_ctl, g->ctl, sizeof(Ctl), cudaMemcpyDeviceToHost, s));
+    CK(cudaStreamSynchronize(s));
+    launches += 1;
+  } else if (use_graph) {
     cudaGraphExec_t ex;
     uint64_t per = 0;
     gr_status gs = get_while_graph<Prog, OffT>(g, key, &ex, &per);
@@ -345,12 +362,63 @@ template <class OffT> static PrArgs<OffT> pr_args(gr_graph *g, uint32_t t, uint3
   return a;
 }
 
+// Hot-source setup (once per graph): pick the kHotK vertices of largest
+// out-degree (the sources of the most in-edges), tag them in a PageRank copy
+// of the CSC payload, size the persistent grid from the occupancy calculator.
+template <class OffT> static gr_status pr_hot_setup(gr_graph *g) {
+  g->pr_hot = 0;
+  const char *env = getenv("GR_PR_HOT");
+  if (env && env[0] == '0') return GR_OK;
+  const HostGraph &H = g->H;
+  if (g->mode != GR_MODE_RESIDENT || g->comm || H.n >= 0x80000000ull || H.m_in < (1u << 20)) return GR_OK;
+  std::vector<uint32_t> idx(H.n);
+  for (uint64_t v = 0; v < H.n; v++) idx[v] = (uint32_t)v;
+  const uint64_t K = std::min<uint64_t>(kHotK, H.n);
+  std::partial_sort(idx.begin(), idx.begin() + K, idx.end(), [&](uint32_t a, uint32_t b) {
+    return H.outdeg[a] != H.outdeg[b] ? H.outdeg[a] > H.outdeg[b] : a < b;
+  });
+  std::vector<uint32_t> slot(H.n, 0xFFFFFFFFu), ids;
+  for (uint64_t k = 0; k < K && H.outdeg[idx[k]] > 0; k++) {
+    slot[idx[k]] = (uint32_t)k;
+    ids.push_back(idx[k]);
+  }
+  g->hot_k = (uint32_t)((ids.size() + 3) & ~size_t(3));
+  ids.resize(g->hot_k, ids.empty() ? 0u : ids[0]);
+  uint32_t *d_slot = nullptr;
+  gr_status s;
+  if ((s = upload(g, &g->hot_ids, ids.data(), ids.size())) != GR_OK) return s;
+  if ((s = dev_alloc(g, (void **)&g->hot_contrib, 4ull * std::max<uint32_t>(g->hot_k, 4))) != GR_OK) return s;
+  if ((s = dev_alloc(g, (void **)&g->pr_src, 4 * (H.m_in + 4))) != GR_OK) return s;
+  CK(cudaMalloc(&d_slot, 4 * H.n));
+  CK(cudaMemcpy(d_slot, slot.data(), 4 * H.n, cudaMemcpyHostToDevice));
+  k_pr_tag<<<g->num_sms * 8, 256, 0, g->stream>>>(g->in_src, H.m_in, d_slot, g->pr_src);
+  CK(cudaGetLastError());
+  CK(cudaStreamSynchronize(g->stream));
+  cudaFree(d_slot);
+  g->hot_smem = sizeof(PrSmem) + 4ull * g->hot_k;
+  CK(cudaFuncSetAttribute(k_pr_gather_apply_hot<OffT>, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)g->hot_smem));
+  int bps = 0;
+  CK(cudaOccupancyMaxActiveBlocksPerMultiprocessor(&bps, k_pr_gather_apply_hot<OffT>, kPrThreads, g->hot_smem));
+  if (bps < 1) return GR_OK;
+  g->hot_grid = (uint32_t)(g->num_sms * bps);
+  g->pr_hot = 1;
+  return GR_OK;
+}
+
 template <class OffT>
 static void pr_launch_iter(gr_graph *g, cudaStream_t s, uint32_t t, uint32_t iters, float d, cudaEvent_t e0,
                            cudaEvent_t e1) {
   PrArgs<OffT> a = pr_args<OffT>(g, t, iters, d);
-  if (e0) cudaEventRecord(e0, s);
-  k_pr_gather_apply<OffT><<<std::max<uint32_t>(g->pr_tiles, 1), kPrThreads, 0, s>>>(a);
+  if (g->pr_hot == 1) {
+    k_pr_hot_pack<<<(g->hot_k + 255) / 256, 256, 0, s>>>(a.contrib_in, g->hot_ids, g->hot_contrib, g->hot_k);
+    a.in_src = g->pr_src;
+    if (e0) cudaEventRecord(e0, s);
+    k_pr_gather_apply_hot<OffT><<<std::min(g->hot_grid, std::max<uint32_t>(g->pr_tiles, 1)), kPrThreads, g->hot_smem,
+                                  s>>>(a, g->hot_contrib, g->hot_k, g->pr_tiles);
+  } else {
+    if (e0) cudaEventRecord(e0, s);
+    k_pr_gather_apply<OffT><<<std::max<uint32_t>(g->pr_tiles, 1), kPrThreads, 0, s>>>(a);
+  }
   if (e1) cudaEventRecord(e1, s);
   k_pr_fixup<OffT><<<std::max<uint32_t>((g->pr_tiles + 255) / 256, 1), 256, 0, s>>>(a, g->pr_tiles);
 }
@@ -360,6 +428,10 @@ static gr_status run_pagerank(gr_graph *g, const gr_run_opts *o, cudaStream_t s,
   const uint32_t iters = o->max_iters;
   const float d = o->damping;
   const int prof = o->profile ? 1 : 0;
+  if (g->pr_hot < 0) {
+    gr_status hs = pr_hot_setup<OffT>(g);
+    if (hs != GR_OK) return hs;
+  }
   if (prof && g->prof_ev.size() < 2 * (size_t)iters + 2) {
     while (g->prof_ev.size() < 2 * (size_t)iters + 2) {
       cudaEvent_t e;
@@ -405,7 +477,7 @@ static gr_status run_pagerank(gr_graph *g, const gr_run_opts *o, cudaStream_t s,
   st->iterations = iters;
   st->edges_gathered = (uint64_t)iters * g->H.m_in;
   st->edges_scattered = 0;
-  st->kernel_launches += 1 + 2ull * iters;
+  st->kernel_launches += 1 + (g->pr_hot == 1 ? 3ull : 2ull) * iters;
   st->bytes_hbm_model = (uint64_t)iters * (4 * g->H.m_in + 12 * g->H.own_n() + 4 * g->H.n);
   g->trace_rows = iters;
   return GR_OK;

@@ -44,6 +44,7 @@ struct gr_graph {
   unsigned long long *trace = nullptr;
   uint32_t trace_cap = 0;
   int grid_frontier = 0;
+  bool coop = false;             // cooperative launch available (persistent loop)
 
   // PageRank state
   uint32_t *d_outdeg = nullptr;
@@ -57,6 +58,13 @@ struct gr_graph {
   float pr_exec_d = 0.f;
   int pr_exec_prof = -1;
   uint32_t pr_trace_iters = 0;
+  // PageRank hot-source path (resident, single rank): shared-memory table of the
+  // kHotK highest-out-degree sources, tagged payload pr_src
+  int pr_hot = -1;                 // -1 not set up, 0 disabled, 1 enabled
+  uint32_t *pr_src = nullptr, *hot_ids = nullptr;
+  float *hot_contrib = nullptr;
+  uint32_t hot_k = 0, hot_grid = 0;
+  size_t hot_smem = 0;
 
   // run bookkeeping
   int last_algo = -1;

@@ -282,32 +282,12 @@ __device__ uint32_t expand_block(const Part<OffT> &P, uint64_t beg, uint32_t deg
   return nact;  // per-warp count
 }
 
-// Last CTA of the superstep's final kernel closes superstep t. The ticket is
-// two-level (groups of 32 CTAs) so no single address takes one atomic per CTA;
-// the whole last CTA sums the spread counter slots in parallel.
+// Close superstep t (the whole CTA calls it; thread 0 writes): sum the spread
+// counters, write the trace row, reset the per-superstep counters, advance t,
+// decide termination and set the CUDA-graph loop condition.
 template <class OffT>
-__device__ void finish_superstep(const Part<OffT> &P, unsigned long long cond_handle, int use_graph) {
-  __shared__ bool s_last;
+__device__ void close_superstep(const Part<OffT> &P, unsigned long long cond_handle, int use_graph) {
   __shared__ unsigned long long s_red[4][kWarpsPerBlock];
-  __syncthreads();
-  if (threadIdx.x == 0) {
-    __threadfence();
-    Ctl *cc = P.ctl;
-    const uint32_t grp = blockIdx.x >> 5, ngrp = (gridDim.x + 31) >> 5;
-    const uint32_t gsize = min(32u, gridDim.x - grp * 32u);
-    bool last = false;
-    if (atomicAdd(&cc->tick1[grp], 1u) == gsize - 1) {
-      cc->tick1[grp] = 0;
-      __threadfence();
-      if (atomicAdd(&cc->tick2, 1u) == ngrp - 1) {
-        cc->tick2 = 0;
-        last = true;
-      }
-    }
-    s_last = last;
-  }
-  __syncthreads();
-  if (!s_last) return;
   __threadfence();
   volatile Ctl *c = P.ctl;
   {
@@ -368,12 +348,40 @@ __device__ void finish_superstep(const Part<OffT> &P, unsigned long long cond_ha
   if (use_graph) cudaGraphSetConditional((cudaGraphConditionalHandle)cond_handle, stop ? 0u : 1u);
 }
 
+
+// Last CTA of the superstep's final kernel closes superstep t. The ticket is
+// two-level (groups of 32 CTAs) so no single address takes one atomic per CTA.
+template <class OffT>
+__device__ void finish_superstep(const Part<OffT> &P, unsigned long long cond_handle, int use_graph) {
+  __shared__ bool s_last;
+  __syncthreads();
+  if (threadIdx.x == 0) {
+    __threadfence();
+    Ctl *cc = P.ctl;
+    const uint32_t grp = blockIdx.x >> 5, ngrp = (gridDim.x + 31) >> 5;
+    const uint32_t gsize = min(32u, gridDim.x - grp * 32u);
+    bool last = false;
+    if (atomicAdd(&cc->tick1[grp], 1u) == gsize - 1) {
+      cc->tick1[grp] = 0;
+      __threadfence();
+      if (atomicAdd(&cc->tick2, 1u) == ngrp - 1) {
+        cc->tick2 = 0;
+        last = true;
+      }
+    }
+    s_last = last;
+  }
+  __syncthreads();
+  if (!s_last) return;
+  close_superstep(P, cond_handle, use_graph);
+}
+
 // ------------------------------------------------------------- kernels
+// Gather + apply over A_t (one phase of superstep t).
 template <class Prog, class OffT>
-__global__ void __launch_bounds__(kBlock) k_gather_apply(const __grid_constant__ Part<OffT> P) {
+__device__ __forceinline__ void gather_phase(const Part<OffT> &P) {
   using G = typename Prog::GatherT;
   Ctl *ctl = P.ctl;
-  if (*(volatile uint32_t *)&ctl->stop) return;
   const uint32_t t = *(volatile uint32_t *)&ctl->iter;
   const uint32_t slot = t & 1u;
   const Ctx cx{t, P.n, ctl->source, ctl->damping};
@@ -480,15 +488,16 @@ __global__ void __launch_bounds__(kBlock) k_gather_apply(const __grid_constant__
   prof_end(ctl, 0);
 }
 
+template <class Prog, class OffT>
+__global__ void __launch_bounds__(kBlock) k_gather_apply(const __grid_constant__ Part<OffT> P) {
+  if (*(volatile uint32_t *)&P.ctl->stop) return;
+  gather_phase<Prog>(P);
+}
+
+// Commit C_t and FrontierActivate (the other phase of superstep t).
 template <class OffT>
-__global__ void __launch_bounds__(kBlock) k_activate(const __grid_constant__ Part<OffT> P, unsigned long long cond,
-                                                     int use_graph) {
+__device__ __forceinline__ void activate_phase(const Part<OffT> &P) {
   Ctl *ctl = P.ctl;
-  if (*(volatile uint32_t *)&ctl->stop) {
-    if (use_graph && blockIdx.x == 0 && threadIdx.x == 0)
-      cudaGraphSetConditional((cudaGraphConditionalHandle)cond, 0u);
-    return;
-  }
   const uint32_t t = *(volatile uint32_t *)&ctl->iter;
   const uint32_t ns = (t + 1) & 1u;
   const uint32_t epoch = ctl->epoch_base + t + 1;
@@ -544,19 +553,24 @@ __global__ void __launch_bounds__(kBlock) k_activate(const __grid_constant__ Par
   my_act = block_sum_u64(lane == 0 ? my_act : 0ull, s8);
   if (threadIdx.x == 0 && my_act) atomicAdd(&ctl->part_a[blockIdx.x % kSlots], my_act);
   prof_end(ctl, 1);
+}
+
+template <class OffT>
+__global__ void __launch_bounds__(kBlock) k_activate(const __grid_constant__ Part<OffT> P, unsigned long long cond,
+                                                     int use_graph) {
+  if (*(volatile uint32_t *)&P.ctl->stop) {
+    if (use_graph && blockIdx.x == 0 && threadIdx.x == 0)
+      cudaGraphSetConditional((cudaGraphConditionalHandle)cond, 0u);
+    return;
+  }
+  activate_phase(P);
   finish_superstep(P, cond, use_graph);
 }
 
 // BFS: apply (depth = t, L276) fused with FrontierActivate; no gather (L274).
 template <class OffT>
-__global__ void __launch_bounds__(kBlock) k_bfs_expand(const __grid_constant__ Part<OffT> P, unsigned long long cond,
-                                                       int use_graph) {
+__device__ __forceinline__ void bfs_phase(const Part<OffT> &P) {
   Ctl *ctl = P.ctl;
-  if (*(volatile uint32_t *)&ctl->stop) {
-    if (use_graph && blockIdx.x == 0 && threadIdx.x == 0)
-      cudaGraphSetConditional((cudaGraphConditionalHandle)cond, 0u);
-    return;
-  }
   const uint32_t t = *(volatile uint32_t *)&ctl->iter;
   const uint32_t slot = t & 1u, ns = slot ^ 1u;
   const uint32_t epoch = ctl->epoch_base + t + 1;
@@ -629,7 +643,60 @@ __global__ void __launch_bounds__(kBlock) k_bfs_expand(const __grid_constant__ P
   my_act = block_sum_u64(lane == 0 ? my_act : 0ull, s8);
   if (threadIdx.x == 0 && my_act) atomicAdd(&ctl->part_a[blockIdx.x % kSlots], my_act);
   prof_end(ctl, 1);
+}
+
+template <class OffT>
+__global__ void __launch_bounds__(kBlock) k_bfs_expand(const __grid_constant__ Part<OffT> P, unsigned long long cond,
+                                                       int use_graph) {
+  if (*(volatile uint32_t *)&P.ctl->stop) {
+    if (use_graph && blockIdx.x == 0 && threadIdx.x == 0)
+      cudaGraphSetConditional((cudaGraphConditionalHandle)cond, 0u);
+    return;
+  }
+  bfs_phase(P);
   finish_superstep(P, cond, use_graph);
+}
+
+// Software grid barrier for the persistent loop (cooperative launch guarantees
+// that every CTA is resident). Sense by generation counter.
+__device__ __forceinline__ void grid_sync(Ctl *c) {
+  __syncthreads();
+  if (threadIdx.x == 0) {
+    volatile uint32_t *gen = &c->bar_gen;
+    const uint32_t g = *gen;
+    __threadfence();
+    if (atomicAdd(&c->bar_count, 1u) == gridDim.x - 1) {
+      c->bar_count = 0;
+      __threadfence();
+      atomicAdd(&c->bar_gen, 1u);
+    } else {
+      while (*gen == g) __nanosleep(32);
+    }
+    __threadfence();
+  }
+  __syncthreads();
+}
+
+// Persistent device-side BSP loop (one cooperative launch per run): phases are
+// separated by grid barriers instead of kernel boundaries, and CTA 0 closes
+// each superstep while the others wait — no launch or host round trip per
+// superstep (the latency floor of high-diameter graphs, cfg3).
+template <class Prog, class OffT>
+__global__ void __launch_bounds__(kBlock) k_persistent(const __grid_constant__ Part<OffT> P) {
+  Ctl *ctl = P.ctl;
+  for (;;) {
+    if (*(volatile uint32_t *)&ctl->stop) break;
+    if (Prog::kHasGather) {
+      gather_phase<Prog>(P);
+      grid_sync(ctl);
+      activate_phase(P);
+    } else {
+      bfs_phase(P);
+    }
+    grid_sync(ctl);
+    if (blockIdx.x == 0) close_superstep(P, 0ull, 0);
+    grid_sync(ctl);
+  }
 }
 
 // Partitioned runs: split the exchanged changed set (every rank's C_t) into

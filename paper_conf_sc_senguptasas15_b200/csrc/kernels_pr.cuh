@@ -70,36 +70,44 @@ __device__ __forceinline__ uint32_t merge_path_rows(const OffT *in_off, uint64_t
   return (uint32_t)lo;
 }
 
-template <class OffT>
-__global__ void __launch_bounds__(kPrThreads, 6) k_pr_gather_apply(const __grid_constant__ PrArgs<OffT> a) {
-  __shared__ uint32_t s_end[kPrTile + 1 + kPrPad];  // row ends, local to the tile's first edge (padded)
-  __shared__ float s_val[kPrTile + kPrPad];         // contrib[src] of the tile's edges (padded)
-  __shared__ float s_tot[kPrTile + kPrPad];         // per-row partial totals (padded)
-  __shared__ uint32_t s_crow[kPrThreads];
-  __shared__ float s_cval[kPrThreads];
-  __shared__ uint32_t s_wkey_first[kPrThreads / 32], s_wkey_last[kPrThreads / 32];
-  __shared__ float s_wval_last[kPrThreads / 32];
-  __shared__ uint64_t s_i0, s_i1, s_j0, s_j1, s_rowstart0;
+constexpr uint32_t kHotTag = 0x80000000u;  // in the PageRank payload: source is hot, low bits = slot
+constexpr int kHotK = 16384;                 // hot sources held in shared memory per CTA (64 KB)
 
+struct PrSmem {
+  uint32_t s_end[kPrTile + 1 + kPrPad];  // row ends, local to the tile's first edge (padded)
+  float s_val[kPrTile + kPrPad];         // contrib[src] of the tile's edges (padded)
+  float s_tot[kPrTile + kPrPad];         // per-row partial totals (padded)
+  uint32_t s_crow[kPrThreads];
+  float s_cval[kPrThreads];
+  uint32_t s_wkey_first[kPrThreads / 32], s_wkey_last[kPrThreads / 32];
+  float s_wval_last[kPrThreads / 32];
+  uint64_t s_i0, s_i1, s_j0, s_j1, s_rowstart0;
+};
+
+// One merge-path tile: stage, walk, join, apply. kHot: sources tagged with
+// kHotTag read their contribution from the CTA's shared hot table.
+template <class OffT, bool kHot>
+__device__ __forceinline__ void pr_tile(const PrArgs<OffT> &a, uint32_t tile, PrSmem &S, const float *s_hot) {
   const uint32_t tid = threadIdx.x, lane = tid & 31, warp = tid >> 5;
   const uint64_t total = (uint64_t)a.own_n + a.m_in;
-  const uint64_t d0 = (uint64_t)blockIdx.x * kPrTile;
+  const uint64_t d0 = (uint64_t)tile * kPrTile;
   const uint64_t d1 = d0 + kPrTile < total ? d0 + kPrTile : total;
+  __syncthreads();  // the previous tile's readers are done with S
   if (tid < 2) {
     const uint64_t diag = tid == 0 ? d0 : d1;
-    const uint32_t i = __ldg(a.tile_row + blockIdx.x + tid);  // == merge_path_rows(diag), precomputed
-    if (tid == 0) { s_i0 = i; s_j0 = diag - i; s_rowstart0 = (uint64_t)a.in_off[i] - a.e_base; }
-    else { s_i1 = i; s_j1 = diag - i; }
+    const uint32_t i = __ldg(a.tile_row + tile + tid);  // == merge_path_rows(diag), precomputed
+    if (tid == 0) { S.s_i0 = i; S.s_j0 = diag - i; S.s_rowstart0 = (uint64_t)a.in_off[i] - a.e_base; }
+    else { S.s_i1 = i; S.s_j1 = diag - i; }
   }
   __syncthreads();
-  const uint64_t i0 = s_i0, j0 = s_j0;
-  const uint32_t ni = (uint32_t)(s_i1 - i0), nj = (uint32_t)(s_j1 - j0);
+  const uint64_t i0 = S.s_i0, j0 = S.s_j0;
+  const uint32_t ni = (uint32_t)(S.s_i1 - i0), nj = (uint32_t)(S.s_j1 - j0);
 
   // stage row ends (local) and gathered contributions
   for (uint32_t k = tid; k <= ni; k += kPrThreads) {
     const uint64_t r = i0 + k;
     uint64_t e = r < a.own_n ? (uint64_t)a.in_off[r + 1] - a.e_base - j0 : (uint64_t)nj;
-    s_end[pr_pad(k)] = (uint32_t)(e < nj ? e : nj);
+    S.s_end[pr_pad(k)] = (uint32_t)(e < nj ? e : nj);
   }
   {
     uint32_t src[kPrIpt];
@@ -112,12 +120,13 @@ __global__ void __launch_bounds__(kPrThreads, 6) k_pr_gather_apply(const __grid_
 #pragma unroll
     for (int q = 0; q < kPrIpt; q++) {
       const uint32_t k = tid + q * kPrThreads;
-      v[q] = k < nj ? __ldg(a.contrib_in + src[q]) : 0.f;
+      if (kHot && (src[q] & kHotTag)) v[q] = s_hot[src[q] & ~kHotTag];
+      else v[q] = k < nj ? __ldg(a.contrib_in + src[q]) : 0.f;
     }
 #pragma unroll
     for (int q = 0; q < kPrIpt; q++) {
       const uint32_t k = tid + q * kPrThreads;
-      if (k < nj) s_val[pr_pad(k)] = v[q];
+      if (k < nj) S.s_val[pr_pad(k)] = v[q];
     }
   }
   __syncthreads();
@@ -128,7 +137,7 @@ __global__ void __launch_bounds__(kPrThreads, 6) k_pr_gather_apply(const __grid_
   uint32_t lo = dt > nj ? dt - nj : 0, hi = dt < ni ? dt : ni;
   while (lo < hi) {
     const uint32_t p = (lo + hi) >> 1;
-    if (s_end[pr_pad(p)] <= dt - p - 1) lo = p + 1;
+    if (S.s_end[pr_pad(p)] <= dt - p - 1) lo = p + 1;
     else hi = p;
   }
   uint32_t i = lo, j = dt - lo;
@@ -137,11 +146,11 @@ __global__ void __launch_bounds__(kPrThreads, 6) k_pr_gather_apply(const __grid_
 #pragma unroll
   for (int q = 0; q < kPrIpt; q++) {
     if (dt + q < dend) {
-      if (j < s_end[pr_pad(i)]) { run += s_val[pr_pad(j)]; ++j; }
-      else { s_tot[pr_pad(i)] = run; run = 0.f; ++i; }
+      if (j < S.s_end[pr_pad(i)]) { run += S.s_val[pr_pad(j)]; ++j; }
+      else { S.s_tot[pr_pad(i)] = run; run = 0.f; ++i; }
     }
   }
-  s_crow[tid] = i;
+  S.s_crow[tid] = i;
 
   // segmented inclusive scan of the thread carries (keys non-decreasing)
   float x = run;
@@ -151,35 +160,74 @@ __global__ void __launch_bounds__(kPrThreads, 6) k_pr_gather_apply(const __grid_
     const uint32_t ky = __shfl_up_sync(0xffffffffu, i, o);
     if (lane >= (uint32_t)o && ky == i) x += y;
   }
-  if (lane == 0) s_wkey_first[warp] = i;
-  if (lane == 31) { s_wkey_last[warp] = i; s_wval_last[warp] = x; }
+  if (lane == 0) S.s_wkey_first[warp] = i;
+  if (lane == 31) { S.s_wkey_last[warp] = i; S.s_wval_last[warp] = x; }
   __syncthreads();
-  if (i == s_wkey_first[warp]) {
+  if (i == S.s_wkey_first[warp]) {
     for (int w = (int)warp - 1; w >= 0; w--) {
-      if (s_wkey_last[w] != i) break;
-      x += s_wval_last[w];
-      if (s_wkey_first[w] != i) break;
+      if (S.s_wkey_last[w] != i) break;
+      x += S.s_wval_last[w];
+      if (S.s_wkey_first[w] != i) break;
     }
   }
-  s_cval[tid] = x;
+  S.s_cval[tid] = x;
   __syncthreads();
   // the last thread of each carry run adds it to the row finished by the next thread
-  const bool run_end = (tid == kPrThreads - 1) || (s_crow[tid + 1] != i);
-  if (run_end && i < ni) s_tot[pr_pad(i)] += x;
+  const bool run_end = (tid == kPrThreads - 1) || (S.s_crow[tid + 1] != i);
+  if (run_end && i < ni) S.s_tot[pr_pad(i)] += x;
   __syncthreads();
 
   // apply the rows whose end lies in this tile (coalesced over destinations)
-  const bool head = (ni > 0) && (s_rowstart0 < j0);  // row i0 began in an earlier tile
+  const bool head = (ni > 0) && (S.s_rowstart0 < j0);  // row i0 began in an earlier tile
   for (uint32_t k = tid; k < ni; k += kPrThreads) {
     if (k == 0 && head) continue;
-    pr_apply_row(a, (uint32_t)(i0 + k), s_tot[pr_pad(k)]);
+    pr_apply_row(a, (uint32_t)(i0 + k), S.s_tot[pr_pad(k)]);
   }
   if (tid == 0) {
-    a.head_row[blockIdx.x] = head ? (uint32_t)i0 : kNoRow;
-    a.head_val[blockIdx.x] = head ? s_tot[pr_pad(0)] : 0.f;
-    const uint64_t i1 = s_i1;
-    a.carry_row[blockIdx.x] = i1 < a.own_n ? (uint32_t)i1 : kNoRow;
-    a.carry_val[blockIdx.x] = s_cval[kPrThreads - 1];
+    a.head_row[tile] = head ? (uint32_t)i0 : kNoRow;
+    a.head_val[tile] = head ? S.s_tot[pr_pad(0)] : 0.f;
+    const uint64_t i1 = S.s_i1;
+    a.carry_row[tile] = i1 < a.own_n ? (uint32_t)i1 : kNoRow;
+    a.carry_val[tile] = S.s_cval[kPrThreads - 1];
+  }
+}
+
+template <class OffT>
+__global__ void __launch_bounds__(kPrThreads, 6) k_pr_gather_apply(const __grid_constant__ PrArgs<OffT> a) {
+  __shared__ PrSmem S;
+  pr_tile<OffT, false>(a, blockIdx.x, S, nullptr);
+}
+
+// Persistent variant (2 CTAs per SM): the CTA first copies the hot sources'
+// contributions (hot_contrib[kHotK], packed by k_pr_hot_pack) into shared
+// memory, then walks tiles blockIdx.x, +gridDim.x, ...; a.in_src is the
+// tagged PageRank payload.
+template <class OffT>
+__global__ void __launch_bounds__(kPrThreads, 2) k_pr_gather_apply_hot(const __grid_constant__ PrArgs<OffT> a,
+                                                                        const float *hot_contrib, uint32_t hot_k,
+                                                                        uint32_t num_tiles) {
+  extern __shared__ __align__(16) unsigned char smem_raw[];
+  PrSmem &S = *reinterpret_cast<PrSmem *>(smem_raw);
+  float *s_hot = reinterpret_cast<float *>(smem_raw + sizeof(PrSmem));
+  for (uint32_t k = threadIdx.x * 4; k < hot_k; k += kPrThreads * 4) {
+    const float4 v = __ldg(reinterpret_cast<const float4 *>(hot_contrib + k));
+    *reinterpret_cast<float4 *>(s_hot + k) = v;
+  }
+  for (uint32_t tile = blockIdx.x; tile < num_tiles; tile += gridDim.x) pr_tile<OffT, true>(a, tile, S, s_hot);
+}
+
+// hot_contrib[k] = contrib[hot_ids[k]] (after the previous superstep finished)
+static __global__ void k_pr_hot_pack(const float *contrib, const uint32_t *hot_ids, float *hot_contrib, uint32_t k) {
+  for (uint32_t i = blockIdx.x * blockDim.x + threadIdx.x; i < k; i += gridDim.x * blockDim.x)
+    hot_contrib[i] = contrib[hot_ids[i]];
+}
+
+// PageRank payload: in_src with hot sources replaced by kHotTag | slot.
+static __global__ void k_pr_tag(const uint32_t *in_src, uint64_t m, const uint32_t *hot_slot, uint32_t *pr_src) {
+  for (uint64_t e = blockIdx.x * (uint64_t)blockDim.x + threadIdx.x; e < m; e += (uint64_t)gridDim.x * blockDim.x) {
+    const uint32_t u = in_src[e];
+    const uint32_t sl = hot_slot[u];
+    pr_src[e] = sl != 0xFFFFFFFFu ? (kHotTag | sl) : u;
   }
 }
 
