@@ -67,17 +67,42 @@ __device__ __forceinline__ unsigned long long block_sum_u64(unsigned long long x
   return t;
 }
 
+// Per-CTA snapshot of the control block: thread 0 issues every load at once
+// (both parities, no load depends on another), the CTA reads shared memory.
+// Avoids thousands of warps queueing on the same L2 line with a dependent chain.
+struct View {
+  uint32_t stop, t, epoch_base, implicit0, no_hub_c, source, prof;
+  uint32_t cntA[2], cntK[2], cntC, cntKC;
+  float damping;
+};
+
+__device__ __forceinline__ void load_view(const Ctl *c, View &v) {
+  __syncthreads();  // a previous snapshot in the same shared slot is no longer read
+  if (threadIdx.x == 0) {
+    const volatile Ctl *vc = c;
+    const uint32_t a0 = vc->cnt_A[0], a1 = vc->cnt_A[1], k0 = vc->cnt_K[0], k1 = vc->cnt_K[1];
+    const uint32_t st = vc->stop, t = vc->iter, eb = vc->epoch_base, im = vc->implicit0, nh = vc->no_hub_c;
+    const uint32_t so = vc->source, cc = vc->cnt_C, kc = vc->cnt_KC;
+    const float dm = vc->damping;
+    const uint32_t pr = (uint32_t)vc->prof;
+    v.cntA[0] = a0; v.cntA[1] = a1; v.cntK[0] = k0; v.cntK[1] = k1;
+    v.stop = st; v.t = t; v.epoch_base = eb; v.implicit0 = im; v.no_hub_c = nh;
+    v.source = so; v.cntC = cc; v.cntKC = kc; v.damping = dm; v.prof = pr;
+  }
+  __syncthreads();
+}
+
 __device__ __forceinline__ unsigned long long gtimer() {
   unsigned long long t;
   asm volatile("mov.u64 %0, %%globaltimer;" : "=l"(t));
   return t;
 }
 // device-side kernel timing inside CUDA-graph loops (first block start .. last block end)
-__device__ __forceinline__ void prof_begin(Ctl *c, int k) {
-  if (c->prof && threadIdx.x == 0) atomicMin(&c->kstart[k], gtimer());
+__device__ __forceinline__ void prof_begin(Ctl *c, const View &v, int k) {
+  if (v.prof && threadIdx.x == 0) atomicMin(&c->kstart[k], gtimer());
 }
-__device__ __forceinline__ void prof_end(Ctl *c, int k) {
-  if (c->prof) {
+__device__ __forceinline__ void prof_end(Ctl *c, const View &v, int k) {
+  if (v.prof) {
     __syncthreads();
     if (threadIdx.x == 0) atomicMax(&c->kend[k], gtimer());
   }

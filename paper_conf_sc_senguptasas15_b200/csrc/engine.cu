@@ -177,7 +177,9 @@ gr_status load_device(gr_graph *g) {
   if ((s = dev_alloc(g, (void **)&g->rank, 4 * ow)) != GR_OK) return s;
   const uint64_t items = own_n + mi;
   g->pr_tiles = (uint32_t)((items + kPrTile - 1) / kPrTile);
-  const size_t tb = 4ull * std::max<uint32_t>(g->pr_tiles, 1);
+  g->pr_wtiles = (uint32_t)((items + kWTile - 1) / kWTile);
+  // head/carry records: one per tile (block/warp kernels) or per persistent warp (range kernels)
+  const size_t tb = 4ull * (std::max<uint32_t>(std::max(g->pr_tiles, g->pr_wtiles), 1) + 64ull * g->num_sms);
   if ((s = dev_alloc(g, (void **)&g->carry_row, tb)) != GR_OK) return s;
   if ((s = dev_alloc(g, (void **)&g->carry_val, tb)) != GR_OK) return s;
   if ((s = dev_alloc(g, (void **)&g->head_row, tb)) != GR_OK) return s;
@@ -190,6 +192,13 @@ gr_status load_device(gr_graph *g) {
     else
       k_pr_tiles<uint32_t><<<(g->pr_tiles + 256) / 256, 256, 0, g->stream>>>(
           (const uint32_t *)g->in_off, 0, (uint32_t)own_n, mi, g->pr_tiles, g->tile_row);
+    if ((s = dev_alloc(g, (void **)&g->wtile_row, 4ull * (g->pr_wtiles + 1))) != GR_OK) return s;
+    if (g->off64)
+      k_pr_tiles<uint64_t><<<(g->pr_wtiles + 256) / 256, 256, 0, g->stream>>>(
+          (const uint64_t *)g->in_off, 0, (uint32_t)own_n, mi, g->pr_wtiles, g->wtile_row, (uint32_t)kWTile);
+    else
+      k_pr_tiles<uint32_t><<<(g->pr_wtiles + 256) / 256, 256, 0, g->stream>>>(
+          (const uint32_t *)g->in_off, 0, (uint32_t)own_n, mi, g->pr_wtiles, g->wtile_row, (uint32_t)kWTile);
     CK(cudaGetLastError());
   }
   CK(cudaStreamSynchronize(g->stream));
@@ -367,10 +376,27 @@ template <class OffT> static PrArgs<OffT> pr_args(gr_graph *g, uint32_t t, uint3
 // of the CSC payload, size the persistent grid from the occupancy calculator.
 template <class OffT> static gr_status pr_hot_setup(gr_graph *g) {
   g->pr_hot = 0;
-  const char *env = getenv("GR_PR_HOT");
-  if (env && env[0] == '0') return GR_OK;
+  // kernel variant (GR_PR_KERNEL = block | blockhot | warp | warphot | range | rangehot; default rangehot)
+  g->pr_kernel = 5;
+  if (const char *k = getenv("GR_PR_KERNEL")) {
+    const std::string v(k);
+    g->pr_kernel = v == "block" ? 0 : v == "blockhot" ? 1 : v == "warp" ? 2 : v == "warphot" ? 3 : v == "range" ? 4 : 5;
+  }
+  if (g->pr_kernel == 4) {
+    g->hot_smem = 32 * sizeof(PrWarpSmem);
+    CK(cudaFuncSetAttribute(k_pr_warp_range<OffT, false>, cudaFuncAttributeMaxDynamicSharedMemorySize,
+                            (int)g->hot_smem));
+    int bps = 0;
+    CK(cudaOccupancyMaxActiveBlocksPerMultiprocessor(&bps, k_pr_warp_range<OffT, false>, 1024, g->hot_smem));
+    g->hot_grid = (uint32_t)(g->num_sms * std::max(bps, 1));
+    return GR_OK;
+  }
+  if (g->pr_kernel != 1 && g->pr_kernel != 3 && g->pr_kernel != 5) return GR_OK;
   const HostGraph &H = g->H;
-  if (g->mode != GR_MODE_RESIDENT || g->comm || H.n >= 0x80000000ull || H.m_in < (1u << 20)) return GR_OK;
+  if (g->mode != GR_MODE_RESIDENT || g->comm || H.n >= 0x80000000ull || H.m_in < (1u << 20)) {
+    g->pr_kernel -= 1;
+    return GR_OK;
+  }
   std::vector<uint32_t> idx(H.n);
   for (uint64_t v = 0; v < H.n; v++) idx[v] = (uint32_t)v;
   const uint64_t K = std::min<uint64_t>(kHotK, H.n);
@@ -395,11 +421,26 @@ template <class OffT> static gr_status pr_hot_setup(gr_graph *g) {
   CK(cudaGetLastError());
   CK(cudaStreamSynchronize(g->stream));
   cudaFree(d_slot);
-  g->hot_smem = sizeof(PrSmem) + 4ull * g->hot_k;
-  CK(cudaFuncSetAttribute(k_pr_gather_apply_hot<OffT>, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)g->hot_smem));
   int bps = 0;
-  CK(cudaOccupancyMaxActiveBlocksPerMultiprocessor(&bps, k_pr_gather_apply_hot<OffT>, kPrThreads, g->hot_smem));
-  if (bps < 1) return GR_OK;
+  if (g->pr_kernel == 5) {
+    g->hot_smem = 4ull * g->hot_k + 32 * sizeof(PrWarpSmem);
+    CK(cudaFuncSetAttribute(k_pr_warp_range<OffT, true>, cudaFuncAttributeMaxDynamicSharedMemorySize,
+                            (int)g->hot_smem));
+    CK(cudaOccupancyMaxActiveBlocksPerMultiprocessor(&bps, k_pr_warp_range<OffT, true>, 1024, g->hot_smem));
+  } else if (g->pr_kernel == 1) {
+    g->hot_smem = sizeof(PrSmem) + 4ull * g->hot_k;
+    CK(cudaFuncSetAttribute(k_pr_gather_apply_hot<OffT>, cudaFuncAttributeMaxDynamicSharedMemorySize,
+                            (int)g->hot_smem));
+    CK(cudaOccupancyMaxActiveBlocksPerMultiprocessor(&bps, k_pr_gather_apply_hot<OffT>, kPrThreads, g->hot_smem));
+  } else {
+    g->hot_smem = 4ull * g->hot_k + 32 * sizeof(PrWarpSmem);
+    CK(cudaFuncSetAttribute(k_pr_warp_hot<OffT>, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)g->hot_smem));
+    CK(cudaOccupancyMaxActiveBlocksPerMultiprocessor(&bps, k_pr_warp_hot<OffT>, 1024, g->hot_smem));
+  }
+  if (bps < 1) {
+    g->pr_kernel -= 1;
+    return GR_OK;
+  }
   g->hot_grid = (uint32_t)(g->num_sms * bps);
   g->pr_hot = 1;
   return GR_OK;
@@ -409,18 +450,43 @@ template <class OffT>
 static void pr_launch_iter(gr_graph *g, cudaStream_t s, uint32_t t, uint32_t iters, float d, cudaEvent_t e0,
                            cudaEvent_t e1) {
   PrArgs<OffT> a = pr_args<OffT>(g, t, iters, d);
+  const bool warp = g->pr_kernel >= 2;
+  const bool range = g->pr_kernel >= 4;
+  if (warp) a.tile_row = g->wtile_row;
+  const uint32_t tiles = warp ? g->pr_wtiles : g->pr_tiles;
+  const uint32_t ranges = g->hot_grid * 32;
   if (g->pr_hot == 1) {
     k_pr_hot_pack<<<(g->hot_k + 255) / 256, 256, 0, s>>>(a.contrib_in, g->hot_ids, g->hot_contrib, g->hot_k);
     a.in_src = g->pr_src;
-    if (e0) cudaEventRecord(e0, s);
-    k_pr_gather_apply_hot<OffT><<<std::min(g->hot_grid, std::max<uint32_t>(g->pr_tiles, 1)), kPrThreads, g->hot_smem,
-                                  s>>>(a, g->hot_contrib, g->hot_k, g->pr_tiles);
-  } else {
-    if (e0) cudaEventRecord(e0, s);
-    k_pr_gather_apply<OffT><<<std::max<uint32_t>(g->pr_tiles, 1), kPrThreads, 0, s>>>(a);
+  }
+  if (e0) cudaEventRecord(e0, s);
+  switch (g->pr_kernel) {
+    case 0:
+      k_pr_gather_apply<OffT><<<std::max<uint32_t>(tiles, 1), kPrThreads, 0, s>>>(a);
+      break;
+    case 1:
+      k_pr_gather_apply_hot<OffT><<<std::min(g->hot_grid, std::max<uint32_t>(tiles, 1)), kPrThreads, g->hot_smem, s>>>(
+          a, g->hot_contrib, g->hot_k, tiles);
+      break;
+    case 3:
+      k_pr_warp_hot<OffT><<<g->hot_grid, 1024, g->hot_smem, s>>>(a, g->hot_contrib, g->hot_k, tiles);
+      break;
+    case 4:
+      k_pr_warp_range<OffT, false><<<g->hot_grid, 1024, g->hot_smem, s>>>(a, nullptr, 0, tiles);
+      break;
+    case 5:
+      k_pr_warp_range<OffT, true><<<g->hot_grid, 1024, g->hot_smem, s>>>(a, g->hot_contrib, g->hot_k, tiles);
+      break;
+    default:
+      k_pr_warp<OffT><<<std::max<uint32_t>((tiles + 7) / 8, 1), 256, 0, s>>>(a, tiles);
   }
   if (e1) cudaEventRecord(e1, s);
-  k_pr_fixup<OffT><<<std::max<uint32_t>((g->pr_tiles + 255) / 256, 1), 256, 0, s>>>(a, g->pr_tiles);
+  if (range)
+    k_pr_fixup<OffT><<<(ranges + 255) / 256, 256, 0, s>>>(a, ranges);
+  else if (warp)
+    k_pr_fixup_warp<OffT><<<std::max<uint32_t>((tiles + 7) / 8, 1), 256, 0, s>>>(a, tiles);
+  else
+    k_pr_fixup<OffT><<<std::max<uint32_t>((tiles + 255) / 256, 1), 256, 0, s>>>(a, tiles);
 }
 
 template <class OffT>
@@ -478,6 +544,7 @@ static gr_status run_pagerank(gr_graph *g, const gr_run_opts *o, cudaStream_t s,
   st->edges_gathered = (uint64_t)iters * g->H.m_in;
   st->edges_scattered = 0;
   st->kernel_launches += 1 + (g->pr_hot == 1 ? 3ull : 2ull) * iters;
+  st->kernel_ms[3] = (double)g->pr_kernel;  // which PageRank gather variant ran (0 block .. 3 warp+hot)
   st->bytes_hbm_model = (uint64_t)iters * (4 * g->H.m_in + 12 * g->H.own_n() + 4 * g->H.n);
   g->trace_rows = iters;
   return GR_OK;

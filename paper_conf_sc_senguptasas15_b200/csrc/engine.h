@@ -53,6 +53,9 @@ struct gr_graph {
   float *carry_val = nullptr, *head_val = nullptr;
   uint32_t pr_tiles = 0;
   uint32_t *tile_row = nullptr;  // merge-path tile starts (resident: [pr_tiles+1]; streamed: per shard)
+  uint32_t pr_wtiles = 0;          // warp-granular tiles (kWTile items)
+  uint32_t *wtile_row = nullptr;
+  int pr_kernel = -1;              // 0 block, 1 block+hot, 2 warp, 3 warp+hot
   cudaGraphExec_t pr_exec = nullptr;
   uint32_t pr_exec_iters = 0;
   float pr_exec_d = 0.f;

@@ -379,19 +379,19 @@ __device__ void finish_superstep(const Part<OffT> &P, unsigned long long cond_ha
 // ------------------------------------------------------------- kernels
 // Gather + apply over A_t (one phase of superstep t).
 template <class Prog, class OffT>
-__device__ __forceinline__ void gather_phase(const Part<OffT> &P) {
+__device__ __forceinline__ void gather_phase(const Part<OffT> &P, const View &V) {
   using G = typename Prog::GatherT;
   Ctl *ctl = P.ctl;
-  const uint32_t t = *(volatile uint32_t *)&ctl->iter;
+  const uint32_t t = V.t;
   const uint32_t slot = t & 1u;
-  const Ctx cx{t, P.n, ctl->source, ctl->damping};
-  const bool implicit = ctl->implicit0 && t == 0;
-  const uint32_t nA = implicit ? P.own_n : *(volatile uint32_t *)&ctl->cnt_A[slot];
-  const uint32_t nK = *(volatile uint32_t *)&ctl->cnt_K[slot];
+  const Ctx cx{t, P.n, V.source, V.damping};
+  const bool implicit = V.implicit0 && t == 0;
+  const uint32_t nA = implicit ? P.own_n : V.cntA[slot];
+  const uint32_t nK = V.cntK[slot];
   const uint32_t *LA = P.listA[slot];
   const uint32_t *LH = P.listH[slot];
-  const bool no_hub_c = ctl->no_hub_c != 0;
-  prof_begin(ctl, 0);
+  const bool no_hub_c = V.no_hub_c != 0;
+  prof_begin(ctl, V, 0);
 
   __shared__ uint32_t sq[kWarpsPerBlock][2][kQueueCap];
   __shared__ uint32_t sred[kWarpsPerBlock][32];
@@ -485,25 +485,27 @@ __device__ __forceinline__ void gather_phase(const Part<OffT> &P) {
   if (threadIdx.x == 0 && my_g) atomicAdd(&ctl->part_g[blockIdx.x % kSlots], my_g);
   my_c = block_sum_u64(my_c, s8);
   if (threadIdx.x == 0 && my_c) atomicAdd(&ctl->part_c[blockIdx.x % kSlots], my_c);
-  prof_end(ctl, 0);
+  prof_end(ctl, V, 0);
 }
 
 template <class Prog, class OffT>
 __global__ void __launch_bounds__(kBlock) k_gather_apply(const __grid_constant__ Part<OffT> P) {
-  if (*(volatile uint32_t *)&P.ctl->stop) return;
-  gather_phase<Prog>(P);
+  __shared__ View V;
+  load_view(P.ctl, V);
+  if (V.stop) return;
+  gather_phase<Prog>(P, V);
 }
 
 // Commit C_t and FrontierActivate (the other phase of superstep t).
 template <class OffT>
-__device__ __forceinline__ void activate_phase(const Part<OffT> &P) {
+__device__ __forceinline__ void activate_phase(const Part<OffT> &P, const View &V) {
   Ctl *ctl = P.ctl;
-  const uint32_t t = *(volatile uint32_t *)&ctl->iter;
+  const uint32_t t = V.t;
   const uint32_t ns = (t + 1) & 1u;
-  const uint32_t epoch = ctl->epoch_base + t + 1;
-  const uint32_t nC = *(volatile uint32_t *)&ctl->cnt_C;
-  const uint32_t nKC = *(volatile uint32_t *)&ctl->cnt_KC;
-  prof_begin(ctl, 1);
+  const uint32_t epoch = V.epoch_base + t + 1;
+  const uint32_t nC = V.cntC;
+  const uint32_t nKC = V.cntKC;
+  prof_begin(ctl, V, 1);
 
   __shared__ uint32_t sq[kWarpsPerBlock][kQueueCap];
   __shared__ uint32_t s_h;
@@ -552,33 +554,35 @@ __device__ __forceinline__ void activate_phase(const Part<OffT> &P) {
   if (threadIdx.x == 0 && my_s) atomicAdd(&ctl->part_s[blockIdx.x % kSlots], my_s);
   my_act = block_sum_u64(lane == 0 ? my_act : 0ull, s8);
   if (threadIdx.x == 0 && my_act) atomicAdd(&ctl->part_a[blockIdx.x % kSlots], my_act);
-  prof_end(ctl, 1);
+  prof_end(ctl, V, 1);
 }
 
 template <class OffT>
 __global__ void __launch_bounds__(kBlock) k_activate(const __grid_constant__ Part<OffT> P, unsigned long long cond,
                                                      int use_graph) {
-  if (*(volatile uint32_t *)&P.ctl->stop) {
+  __shared__ View V;
+  load_view(P.ctl, V);
+  if (V.stop) {
     if (use_graph && blockIdx.x == 0 && threadIdx.x == 0)
       cudaGraphSetConditional((cudaGraphConditionalHandle)cond, 0u);
     return;
   }
-  activate_phase(P);
+  activate_phase(P, V);
   finish_superstep(P, cond, use_graph);
 }
 
 // BFS: apply (depth = t, L276) fused with FrontierActivate; no gather (L274).
 template <class OffT>
-__device__ __forceinline__ void bfs_phase(const Part<OffT> &P) {
+__device__ __forceinline__ void bfs_phase(const Part<OffT> &P, const View &V) {
   Ctl *ctl = P.ctl;
-  const uint32_t t = *(volatile uint32_t *)&ctl->iter;
+  const uint32_t t = V.t;
   const uint32_t slot = t & 1u, ns = slot ^ 1u;
-  const uint32_t epoch = ctl->epoch_base + t + 1;
-  const uint32_t nA = *(volatile uint32_t *)&ctl->cnt_A[slot];
-  const uint32_t nK = *(volatile uint32_t *)&ctl->cnt_K[slot];
+  const uint32_t epoch = V.epoch_base + t + 1;
+  const uint32_t nA = V.cntA[slot];
+  const uint32_t nK = V.cntK[slot];
   const uint32_t *LA = P.listA[slot];
   const uint32_t *LH = P.listH[slot];
-  prof_begin(ctl, 1);
+  prof_begin(ctl, V, 1);
 
   __shared__ uint32_t sq[kWarpsPerBlock][kQueueCap];
   __shared__ uint32_t s_h;
@@ -642,18 +646,20 @@ __device__ __forceinline__ void bfs_phase(const Part<OffT> &P) {
   if (threadIdx.x == 0 && my_c) atomicAdd(&ctl->part_c[blockIdx.x % kSlots], my_c);
   my_act = block_sum_u64(lane == 0 ? my_act : 0ull, s8);
   if (threadIdx.x == 0 && my_act) atomicAdd(&ctl->part_a[blockIdx.x % kSlots], my_act);
-  prof_end(ctl, 1);
+  prof_end(ctl, V, 1);
 }
 
 template <class OffT>
 __global__ void __launch_bounds__(kBlock) k_bfs_expand(const __grid_constant__ Part<OffT> P, unsigned long long cond,
                                                        int use_graph) {
-  if (*(volatile uint32_t *)&P.ctl->stop) {
+  __shared__ View V;
+  load_view(P.ctl, V);
+  if (V.stop) {
     if (use_graph && blockIdx.x == 0 && threadIdx.x == 0)
       cudaGraphSetConditional((cudaGraphConditionalHandle)cond, 0u);
     return;
   }
-  bfs_phase(P);
+  bfs_phase(P, V);
   finish_superstep(P, cond, use_graph);
 }
 
@@ -684,14 +690,17 @@ __device__ __forceinline__ void grid_sync(Ctl *c) {
 template <class Prog, class OffT>
 __global__ void __launch_bounds__(kBlock) k_persistent(const __grid_constant__ Part<OffT> P) {
   Ctl *ctl = P.ctl;
+  __shared__ View V;
   for (;;) {
-    if (*(volatile uint32_t *)&ctl->stop) break;
+    load_view(ctl, V);
+    if (V.stop) break;
     if (Prog::kHasGather) {
-      gather_phase<Prog>(P);
+      gather_phase<Prog>(P, V);
       grid_sync(ctl);
-      activate_phase(P);
+      load_view(ctl, V);
+      activate_phase(P, V);
     } else {
-      bfs_phase(P);
+      bfs_phase(P, V);
     }
     grid_sync(ctl);
     if (blockIdx.x == 0) close_superstep(P, 0ull, 0);

@@ -216,6 +216,292 @@ __global__ void __launch_bounds__(kPrThreads, 2) k_pr_gather_apply_hot(const __g
   for (uint32_t tile = blockIdx.x; tile < num_tiles; tile += gridDim.x) pr_tile<OffT, true>(a, tile, S, s_hot);
 }
 
+
+// ---------------------------------------------------------------------------
+// Warp-granular merge path: a tile of kWTile = 256 items belongs to ONE warp
+// (8 items per lane). Staging, the merge walk, the segmented join and the
+// apply are warp-local (shuffles + __syncwarp), so warps never wait at a CTA
+// barrier and every warp's memory phases overlap with its neighbours'.
+// Rows spanning warp tiles are finished by k_pr_fixup_warp.
+constexpr int kWIpt = 8;
+constexpr int kWTile = 32 * kWIpt;
+constexpr int kWPad = kWTile / kWIpt;
+
+struct PrWarpSmem {
+  uint32_t s_end[kWTile + 1 + kWPad + 1];
+  float s_val[kWTile + kWPad];
+  float s_tot[kWTile + kWPad];
+};
+
+template <class OffT, bool kHot>
+__device__ __forceinline__ void pr_warp_tile(const PrArgs<OffT> &a, uint32_t tile, PrWarpSmem &S,
+                                             const float *s_hot) {
+  const uint32_t lane = threadIdx.x & 31;
+  const uint64_t total = (uint64_t)a.own_n + a.m_in;
+  const uint64_t d0 = (uint64_t)tile * kWTile;
+  const uint64_t d1 = d0 + kWTile < total ? d0 + kWTile : total;
+  const uint32_t i0 = __ldg(a.tile_row + tile), i1 = __ldg(a.tile_row + tile + 1);
+  const uint64_t j0 = d0 - i0;
+  const uint32_t ni = i1 - i0, nj = (uint32_t)((d1 - i1) - j0);
+  const uint64_t rowstart0 = (uint64_t)a.in_off[i0] - a.e_base;
+  __syncwarp();  // the previous tile's readers are done with S
+  for (uint32_t k = lane; k <= ni; k += 32) {
+    const uint64_t r = (uint64_t)i0 + k;
+    const uint64_t e = r < a.own_n ? (uint64_t)a.in_off[r + 1] - a.e_base - j0 : (uint64_t)nj;
+    S.s_end[pr_pad(k)] = (uint32_t)(e < nj ? e : nj);
+  }
+  {
+    uint32_t src[kWIpt];
+#pragma unroll
+    for (int q = 0; q < kWIpt; q++) {
+      const uint32_t k = lane + 32u * q;
+      src[q] = k < nj ? ldg_nc(a.in_src + j0 + k) : 0u;
+    }
+    float v[kWIpt];
+#pragma unroll
+    for (int q = 0; q < kWIpt; q++) {
+      const uint32_t k = lane + 32u * q;
+      if (kHot && (src[q] & kHotTag)) v[q] = s_hot[src[q] & ~kHotTag];
+      else v[q] = k < nj ? __ldg(a.contrib_in + src[q]) : 0.f;
+    }
+#pragma unroll
+    for (int q = 0; q < kWIpt; q++) {
+      const uint32_t k = lane + 32u * q;
+      if (k < nj) S.s_val[pr_pad(k)] = v[q];
+    }
+  }
+  __syncwarp();
+  const uint32_t items = ni + nj;
+  const uint32_t dt = min(lane * kWIpt, items);
+  uint32_t lo = dt > nj ? dt - nj : 0, hi = dt < ni ? dt : ni;
+  while (lo < hi) {
+    const uint32_t p = (lo + hi) >> 1;
+    if (S.s_end[pr_pad(p)] <= dt - p - 1) lo = p + 1;
+    else hi = p;
+  }
+  uint32_t i = lo, j = dt - lo;
+  float run = 0.f;
+  const uint32_t dend = min(dt + kWIpt, items);
+#pragma unroll
+  for (int q = 0; q < kWIpt; q++) {
+    if (dt + q < dend) {
+      if (j < S.s_end[pr_pad(i)]) { run += S.s_val[pr_pad(j)]; ++j; }
+      else { S.s_tot[pr_pad(i)] = run; run = 0.f; ++i; }
+    }
+  }
+  float x = run;
+#pragma unroll
+  for (int o = 1; o < 32; o <<= 1) {
+    const float y = __shfl_up_sync(0xffffffffu, x, o);
+    const uint32_t ky = __shfl_up_sync(0xffffffffu, i, o);
+    if (lane >= (uint32_t)o && ky == i) x += y;
+  }
+  const uint32_t inext = __shfl_down_sync(0xffffffffu, i, 1);
+  const float carry = __shfl_sync(0xffffffffu, x, 31);
+  __syncwarp();  // every s_tot written by the walk is visible
+  const bool run_end = (lane == 31) || (inext != i);
+  if (run_end && i < ni) S.s_tot[pr_pad(i)] += x;
+  __syncwarp();
+  const bool head = (ni > 0) && (rowstart0 < j0);
+  for (uint32_t k = lane; k < ni; k += 32) {
+    if (k == 0 && head) continue;
+    pr_apply_row(a, i0 + k, S.s_tot[pr_pad(k)]);
+  }
+  if (lane == 0) {
+    a.head_row[tile] = head ? i0 : kNoRow;
+    a.head_val[tile] = head ? S.s_tot[pr_pad(0)] : 0.f;
+    a.carry_row[tile] = i1 < a.own_n ? i1 : kNoRow;
+    a.carry_val[tile] = carry;
+  }
+}
+
+template <class OffT>
+__global__ void __launch_bounds__(256) k_pr_warp(const __grid_constant__ PrArgs<OffT> a, uint32_t num_tiles) {
+  __shared__ PrWarpSmem S[8];
+  const uint32_t w = threadIdx.x >> 5;
+  const uint32_t tile = blockIdx.x * 8u + w;
+  if (tile < num_tiles) pr_warp_tile<OffT, false>(a, tile, S[w], nullptr);
+}
+
+// 1024-thread persistent CTAs: one shared hot table per SM, 32 warp-tile walkers.
+template <class OffT>
+__global__ void __launch_bounds__(1024, 1) k_pr_warp_hot(const __grid_constant__ PrArgs<OffT> a,
+                                                        const float *hot_contrib, uint32_t hot_k,
+                                                        uint32_t num_tiles) {
+  extern __shared__ __align__(16) unsigned char smem_raw[];
+  float *s_hot = reinterpret_cast<float *>(smem_raw);
+  PrWarpSmem *S = reinterpret_cast<PrWarpSmem *>(smem_raw + 4ull * hot_k);
+  for (uint32_t k = threadIdx.x * 4; k < hot_k; k += blockDim.x * 4)
+    *reinterpret_cast<float4 *>(s_hot + k) = __ldg(reinterpret_cast<const float4 *>(hot_contrib + k));
+  __syncthreads();
+  const uint32_t w = threadIdx.x >> 5, nw = blockDim.x >> 5;
+  for (uint32_t tile = blockIdx.x * nw + w; tile < num_tiles; tile += gridDim.x * nw)
+    pr_warp_tile<OffT, true>(a, tile, S[w], s_hot);
+}
+
+// Rows spanning warp tiles: one warp per tile with a head; the preceding
+// tiles' carries of the same row are summed 32 at a time (coalesced, ballot
+// for the run end) in a fixed order.
+template <class OffT>
+__global__ void k_pr_fixup_warp(const __grid_constant__ PrArgs<OffT> a, uint32_t num_tiles) {
+  const uint32_t lane = threadIdx.x & 31;
+  const uint32_t nw = (gridDim.x * blockDim.x) >> 5;
+  for (uint32_t c = (blockIdx.x * blockDim.x + threadIdx.x) >> 5; c < num_tiles; c += nw) {
+    const uint32_t row = a.head_row[c];
+    if (row == kNoRow) continue;
+    float acc = 0.f;
+    for (int64_t base = (int64_t)c - 1; base >= 0; base -= 32) {
+      const int64_t p = base - lane;
+      const bool ok = p >= 0 && a.carry_row[p] == row;
+      const uint32_t mask = __ballot_sync(0xffffffffu, ok);
+      const uint32_t run = mask == 0xffffffffu ? 32u : (uint32_t)(__ffs(~mask) - 1);
+      if (lane < run) acc += a.carry_val[p];
+      if (run < 32) break;
+    }
+#pragma unroll
+    for (int o = 16; o > 0; o >>= 1) acc += __shfl_xor_sync(0xffffffffu, acc, o);
+    if (lane == 0) pr_apply_row(a, row, a.head_val[c] + acc);
+  }
+}
+
+
+// ---------------------------------------------------------------------------
+// Persistent warp-range kernel: warp w walks the CONTIGUOUS tiles
+// [w*T, (w+1)*T) and carries the open row's partial sum in registers from one
+// tile to the next, so a row split between two tiles of the same warp is
+// finished by that warp. Only rows that cross a warp-range boundary are left to
+// k_pr_fixup (one head/carry record per warp range, indexed by the global warp).
+template <class OffT, bool kHot>
+__device__ __forceinline__ void pr_warp_range(const PrArgs<OffT> &a, uint32_t wid, uint32_t t0, uint32_t t1,
+                                              PrWarpSmem &S, const float *s_hot) {
+  const uint32_t lane = threadIdx.x & 31;
+  const uint64_t total = (uint64_t)a.own_n + a.m_in;
+  uint32_t pend_row = kNoRow;  // row whose partial sum is carried into the next tile
+  float pend_val = 0.f;
+  bool range_head = false;     // pend_row began before this warp's range
+  bool head_written = false;
+  for (uint32_t tile = t0; tile < t1; tile++) {
+    const uint64_t d0 = (uint64_t)tile * kWTile;
+    const uint64_t d1 = d0 + kWTile < total ? d0 + kWTile : total;
+    const uint32_t i0 = __ldg(a.tile_row + tile), i1 = __ldg(a.tile_row + tile + 1);
+    const uint64_t j0 = d0 - i0;
+    const uint32_t ni = i1 - i0, nj = (uint32_t)((d1 - i1) - j0);
+    const bool started_before = ((uint64_t)a.in_off[i0] - a.e_base) < j0;
+    if (tile == t0) {
+      pend_row = i0;
+      pend_val = 0.f;
+      range_head = started_before;
+    }
+    __syncwarp();
+    for (uint32_t k = lane; k <= ni; k += 32) {
+      const uint64_t r = (uint64_t)i0 + k;
+      const uint64_t e = r < a.own_n ? (uint64_t)a.in_off[r + 1] - a.e_base - j0 : (uint64_t)nj;
+      S.s_end[pr_pad(k)] = (uint32_t)(e < nj ? e : nj);
+    }
+    {
+      uint32_t src[kWIpt];
+#pragma unroll
+      for (int q = 0; q < kWIpt; q++) {
+        const uint32_t k = lane + 32u * q;
+        src[q] = k < nj ? ldg_nc(a.in_src + j0 + k) : 0u;
+      }
+      float v[kWIpt];
+#pragma unroll
+      for (int q = 0; q < kWIpt; q++) {
+        const uint32_t k = lane + 32u * q;
+        if (kHot && (src[q] & kHotTag)) v[q] = s_hot[src[q] & ~kHotTag];
+        else v[q] = k < nj ? __ldg(a.contrib_in + src[q]) : 0.f;
+      }
+#pragma unroll
+      for (int q = 0; q < kWIpt; q++) {
+        const uint32_t k = lane + 32u * q;
+        if (k < nj) S.s_val[pr_pad(k)] = v[q];
+      }
+    }
+    __syncwarp();
+    const uint32_t items = ni + nj;
+    const uint32_t dt = min(lane * kWIpt, items);
+    uint32_t lo = dt > nj ? dt - nj : 0, hi = dt < ni ? dt : ni;
+    while (lo < hi) {
+      const uint32_t p = (lo + hi) >> 1;
+      if (S.s_end[pr_pad(p)] <= dt - p - 1) lo = p + 1;
+      else hi = p;
+    }
+    uint32_t i = lo, j = dt - lo;
+    float run = 0.f;
+    const uint32_t dend = min(dt + kWIpt, items);
+#pragma unroll
+    for (int q = 0; q < kWIpt; q++) {
+      if (dt + q < dend) {
+        if (j < S.s_end[pr_pad(i)]) { run += S.s_val[pr_pad(j)]; ++j; }
+        else { S.s_tot[pr_pad(i)] = run; run = 0.f; ++i; }
+      }
+    }
+    float x = run;
+#pragma unroll
+    for (int o = 1; o < 32; o <<= 1) {
+      const float y = __shfl_up_sync(0xffffffffu, x, o);
+      const uint32_t ky = __shfl_up_sync(0xffffffffu, i, o);
+      if (lane >= (uint32_t)o && ky == i) x += y;
+    }
+    const uint32_t inext = __shfl_down_sync(0xffffffffu, i, 1);
+    const float cx = __shfl_sync(0xffffffffu, x, 31);  // partial of row i1 inside this tile
+    __syncwarp();
+    const bool run_end = (lane == 31) || (inext != i);
+    if (run_end && i < ni) S.s_tot[pr_pad(i)] += x;
+    __syncwarp();
+    if (ni > 0) {
+      // row i0: add the partial carried from this warp's previous tile
+      const float tot0 = S.s_tot[pr_pad(0)] + (started_before && pend_row == i0 ? pend_val : 0.f);
+      const bool is_head = started_before && range_head;
+      if (lane == 0) {
+        if (is_head) {
+          a.head_row[wid] = i0;
+          a.head_val[wid] = tot0;
+        } else {
+          pr_apply_row(a, i0, tot0);
+        }
+      }
+      head_written |= is_head;
+      for (uint32_t k = 1 + lane; k < ni; k += 32) pr_apply_row(a, i0 + k, S.s_tot[pr_pad(k)]);
+      pend_row = i1;
+      pend_val = cx;
+      range_head = false;
+    } else {
+      pend_val = (pend_row == i0 ? pend_val : 0.f) + cx;
+      pend_row = i0;
+    }
+  }
+  if (lane == 0 && t0 < t1) {
+    if (!head_written) a.head_row[wid] = kNoRow;
+    a.carry_row[wid] = pend_row < a.own_n ? pend_row : kNoRow;
+    a.carry_val[wid] = pend_val;
+  } else if (lane == 0) {
+    a.head_row[wid] = kNoRow;
+    a.carry_row[wid] = kNoRow;
+    a.carry_val[wid] = 0.f;
+  }
+}
+
+template <class OffT, bool kHot>
+__global__ void __launch_bounds__(1024, 1) k_pr_warp_range(const __grid_constant__ PrArgs<OffT> a,
+                                                          const float *hot_contrib, uint32_t hot_k,
+                                                          uint32_t num_tiles) {
+  extern __shared__ __align__(16) unsigned char smem_raw[];
+  float *s_hot = reinterpret_cast<float *>(smem_raw);
+  PrWarpSmem *S = reinterpret_cast<PrWarpSmem *>(smem_raw + (kHot ? 4ull * hot_k : 0ull));
+  if (kHot) {
+    for (uint32_t k = threadIdx.x * 4; k < hot_k; k += blockDim.x * 4)
+      *reinterpret_cast<float4 *>(s_hot + k) = __ldg(reinterpret_cast<const float4 *>(hot_contrib + k));
+    __syncthreads();
+  }
+  const uint32_t w = threadIdx.x >> 5, nw = blockDim.x >> 5;
+  const uint32_t wid = blockIdx.x * nw + w, W = gridDim.x * nw;
+  const uint32_t per = (num_tiles + W - 1) / W;
+  const uint32_t t0 = min(wid * per, num_tiles), t1 = min(t0 + per, num_tiles);
+  pr_warp_range<OffT, kHot>(a, wid, t0, t1, S[w], s_hot);
+}
+
 // hot_contrib[k] = contrib[hot_ids[k]] (after the previous superstep finished)
 static __global__ void k_pr_hot_pack(const float *contrib, const uint32_t *hot_ids, float *hot_contrib, uint32_t k) {
   for (uint32_t i = blockIdx.x * blockDim.x + threadIdx.x; i < k; i += gridDim.x * blockDim.x)
@@ -247,10 +533,10 @@ __global__ void k_pr_fixup(const __grid_constant__ PrArgs<OffT> a, uint32_t num_
 // = rows consumed before diagonal c * kPrTile (the last entry is the end).
 template <class OffT>
 __global__ void k_pr_tiles(const OffT *in_off, uint64_t e_base, uint32_t rows, uint64_t nnz, uint32_t num_tiles,
-                           uint32_t *tile_row) {
+                           uint32_t *tile_row, uint32_t tile_items = kPrTile) {
   const uint64_t total = (uint64_t)rows + nnz;
   for (uint32_t c = blockIdx.x * blockDim.x + threadIdx.x; c <= num_tiles; c += gridDim.x * blockDim.x) {
-    uint64_t diag = (uint64_t)c * kPrTile;
+    uint64_t diag = (uint64_t)c * tile_items;
     if (diag > total) diag = total;
     tile_row[c] = merge_path_rows(in_off, e_base, rows, nnz, diag);
   }

@@ -28,10 +28,12 @@ __global__ void __launch_bounds__(kBlock) k_s_gather_apply(const __grid_constant
                                                            uint32_t *cstamp) {
   using G = typename Prog::GatherT;
   Ctl *ctl = P.ctl;
-  const uint32_t t = ctl->iter;
-  const Ctx cx{t, P.n, ctl->source, ctl->damping};
-  const bool implicit = ctl->implicit0 && t == 0;
-  const uint32_t epoch_t = ctl->epoch_base + t;
+  __shared__ View V;
+  load_view(ctl, V);
+  const uint32_t t = V.t;
+  const Ctx cx{t, P.n, V.source, V.damping};
+  const bool implicit = V.implicit0 && t == 0;
+  const uint32_t epoch_t = V.epoch_base + t;
   __shared__ uint32_t sq[kWarpsPerBlock][2][kQueueCap];
   __shared__ uint32_t sred[kWarpsPerBlock][32];
   __shared__ int s_any;
