@@ -91,7 +91,14 @@ typedef struct gr_load_opts {
   const void *nccl_unique_id;    /* world > 1: 128 bytes from gr_get_unique_id() on rank 0, broadcast */
   int32_t host_threads;          /* shard-builder threads; 0 = all cores */
   int32_t sim_ranks;             /* > 1: emulate this many owner partitions on ONE device (tests) */
+  int32_t build;                 /* gr_build: where the shard layout is built */
 } gr_load_opts;
+
+typedef enum gr_build {
+  GR_BUILD_AUTO = 0,   /* device for resident single-rank COO inputs, else host */
+  GR_BUILD_HOST = 1,   /* multithreaded host builder (always used for streamed / multi-rank graphs) */
+  GR_BUILD_DEVICE = 2  /* upload the COO and sort it on the GPU (resident, single rank, COO only) */
+} gr_build;
 
 typedef struct gr_run_opts {
   int32_t algo;       /* gr_algo */

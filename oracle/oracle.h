@@ -10,7 +10,7 @@
 extern "C" {
 #endif
 
-enum { OR_BFS = 0, OR_SSSP = 1, OR_PAGERANK = 2, OR_CC = 3 };
+enum { OR_BFS = 0, OR_SSSP = 1, OR_PAGERANK = 2, OR_CC = 3, OR_WIDEST = 4 };
 #define OR_INF 0xFFFFFFFFu
 
 typedef struct or_graph or_graph;
@@ -23,7 +23,9 @@ or_graph *or_graph_build(uint64_t n, uint64_t m, const uint32_t *src, const uint
 void or_graph_free(or_graph *g);
 
 /* Run one program to termination (or max_iters supersteps; 0 = unlimited).
- * values_out: uint32_t[n] for BFS/SSSP/CC, double[n] for PAGERANK.
+ * values_out: uint32_t[n] for BFS/SSSP/CC/WIDEST, double[n] for PAGERANK.
+ * OR_WIDEST: single-source widest path (max over paths of the min edge weight),
+ * a user GAS program (§4.1) used to check GR_CUSTOM programs.
  * trace_out (nullable): rows of 4 uint64 per superstep t:
  *   |A_t|, |C_t|, sum_{v in A_t} indeg(v) (0 when gather is eliminated),
  *   sum_{u in C_t} outdeg(u) (0 when FrontierActivate is eliminated).

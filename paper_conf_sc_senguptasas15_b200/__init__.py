@@ -26,6 +26,7 @@ GR_FMT_COO, GR_FMT_CSR = 0, 1
 ALGOS = {"bfs": 0, "sssp": 1, "pagerank": 2, "cc": 3, "custom": 4}
 MODES = {"auto": 0, "resident": 1, "streamed": 2}
 LOOPS = {"auto": 0, "host": 1, "device": 2, "persistent": 3}
+BUILDS = {"auto": 0, "host": 1, "device": 2}
 INF = 0xFFFFFFFF
 
 EXPORTS = [
@@ -51,7 +52,7 @@ class gr_load_opts(ctypes.Structure):
     _fields_ = [("shard_edges", ctypes.c_uint64), ("device_budget_bytes", ctypes.c_uint64),
                 ("mode", ctypes.c_int32), ("device", ctypes.c_int32), ("rank", ctypes.c_int32),
                 ("world", ctypes.c_int32), ("nccl_unique_id", ctypes.c_void_p), ("host_threads", ctypes.c_int32),
-                ("sim_ranks", ctypes.c_int32)]
+                ("sim_ranks", ctypes.c_int32), ("build", ctypes.c_int32)]
 
 
 class gr_run_opts(ctypes.Structure):
@@ -157,7 +158,7 @@ def _edges(n, src=None, dst=None, weights=None, row_offsets=None, col_idx=None):
 
 
 def _load_opts(shard_edges=0, device_budget_bytes=0, mode="auto", device=0, rank=0, world=1,
-               nccl_unique_id=None, host_threads=0, sim_ranks=0):
+               nccl_unique_id=None, host_threads=0, sim_ranks=0, build="auto"):
     o = gr_load_opts()
     o.shard_edges, o.device_budget_bytes = int(shard_edges), int(device_budget_bytes)
     o.mode = MODES[mode] if isinstance(mode, str) else int(mode)
@@ -167,6 +168,7 @@ def _load_opts(shard_edges=0, device_budget_bytes=0, mode="auto", device=0, rank
         uid = ctypes.create_string_buffer(bytes(nccl_unique_id), 128)
         o.nccl_unique_id = ctypes.cast(uid, ctypes.c_void_p)
     o.host_threads, o.sim_ranks = int(host_threads), int(sim_ranks)
+    o.build = BUILDS[build] if isinstance(build, str) else int(build)
     return o, uid
 
 

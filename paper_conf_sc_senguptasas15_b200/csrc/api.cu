@@ -69,10 +69,27 @@ gr_status gr_graph_load(const gr_edges *edges, const gr_load_opts *opts_in, gr_g
   gr_graph *g = new gr_graph();
   g->device = opts.device;
   std::string err;
-  gr_status s = build_host_graph(edges, opts.shard_edges, opts.world, opts.rank, opts.host_threads, &g->H, &err);
-  if (s != GR_OK) {
+  gr_status s = GR_OK;
+  size_t free_b = 0, total_b = 0;
+  cudaMemGetInfo(&free_b, &total_b);
+  uint64_t budget = opts.device_budget_bytes ? opts.device_budget_bytes
+                                             : (free_b > (4ull << 30) ? free_b - (4ull << 30) : free_b / 2);
+  // device build: resident, single rank, COO input, and room for the sort buffers (~34 B/edge peak)
+  const uint64_t n0 = edges->num_vertices, m0 = edges->num_edges;
+  const bool dev_ok = opts.world == 1 && edges->fmt == GR_FMT_COO && opts.mode != GR_MODE_STREAMED && n0 >= 1 &&
+                      n0 < 0xFFFFFFFFull && (m0 == 0 || (edges->src && edges->dst)) &&
+                      34 * m0 + 64 * n0 + (64ull << 20) <= budget;
+  const bool dev_build = opts.build == GR_BUILD_DEVICE || (opts.build == GR_BUILD_AUTO && dev_ok);
+  if (opts.build == GR_BUILD_DEVICE && !dev_ok) {
     delete g;
-    return fail(s, "%s", err.c_str());
+    return fail(GR_EUNSUPPORTED, "device build needs a resident single-rank COO graph that fits the device budget");
+  }
+  if (!dev_build) {
+    s = build_host_graph(edges, opts.shard_edges, opts.world, opts.rank, opts.host_threads, &g->H, &err);
+    if (s != GR_OK) {
+      delete g;
+      return fail(s, "%s", err.c_str());
+    }
   }
   cudaDeviceProp prop;
   cudaGetDeviceProperties(&prop, g->device);
@@ -88,13 +105,20 @@ gr_status gr_graph_load(const gr_edges *edges, const gr_load_opts *opts_in, gr_g
     cudaEventCreate(&e);
     g->prof_ev.push_back(e);
   }
-  size_t free_b = 0, total_b = 0;
-  cudaMemGetInfo(&free_b, &total_b);
-  uint64_t budget = opts.device_budget_bytes ? opts.device_budget_bytes
-                                             : (free_b > (4ull << 30) ? free_b - (4ull << 30) : free_b / 2);
-  const uint64_t need = resident_bytes_estimate(g->H);
-  if (opts.mode == GR_MODE_AUTO) g->mode = (need <= budget || opts.world > 1) ? GR_MODE_RESIDENT : GR_MODE_STREAMED;
-  else g->mode = opts.mode;
+  if (dev_build) {
+    g->mode = GR_MODE_RESIDENT;
+    g->dev_built = true;
+    s = device_build(g, edges, opts.shard_edges);
+    if (s != GR_OK) {
+      std::string keep = gr::last_error();
+      destroy(g);
+      return fail(s, "%s", keep.c_str());
+    }
+  } else {
+    const uint64_t need = resident_bytes_estimate(g->H);
+    if (opts.mode == GR_MODE_AUTO) g->mode = (need <= budget || opts.world > 1) ? GR_MODE_RESIDENT : GR_MODE_STREAMED;
+    else g->mode = opts.mode;
+  }
   g->sim = sim;
   s = load_device(g);
   if (s == GR_OK && g->mode == GR_MODE_STREAMED) s = stream_setup(g, budget);

@@ -92,8 +92,16 @@ static void build_hub_bits(const std::vector<uint64_t> &off, uint64_t count, std
 gr_status load_device(gr_graph *g) {
   HostGraph &H = g->H;
   const uint64_t n = H.n, own_n = H.own_n(), mi = H.m_in;
-  g->off64 = (mi >= 0xFFFFFFFFull);
   gr_status s;
+  uint64_t hubs_in = 0, chunks_in = 0, hubs_out = 0, chunks_out = 0;
+  if (g->dev_built) {
+    // offsets, payloads, hub bitmaps and static hub chunks already on the device
+    hubs_in = g->dev_hubs_in;
+    chunks_in = g->dev_chunks_in;
+    hubs_out = g->dev_hubs_out;
+    chunks_out = g->dev_chunks_out;
+  } else {
+  g->off64 = (mi >= 0xFFFFFFFFull);
   // static per-vertex metadata (both modes)
   if (g->off64) {
     if ((s = upload_offsets<uint64_t>(g, &g->in_off, H.in_off)) != GR_OK) return s;
@@ -110,7 +118,7 @@ gr_status load_device(gr_graph *g) {
   g->n_static_hubs = (uint32_t)hubs.size();
   if ((s = upload(g, &g->static_hubs, hubs.data(), hubs.size())) != GR_OK) return s;
   // hub chunk capacities: every hub appears at most once per list
-  uint64_t hubs_in = 0, chunks_in = 0, hubs_out = 0, chunks_out = 0;
+  {
   std::vector<uint32_t> sch_h, sch_c;
   for (uint64_t i = 0; i < own_n; i++) {
     const uint64_t d = H.in_off[i + 1] - H.in_off[i];
@@ -128,6 +136,15 @@ gr_status load_device(gr_graph *g) {
   g->n_static_chunks = (uint32_t)sch_h.size();
   if ((s = upload(g, &g->static_chk_h, sch_h.data(), sch_h.size())) != GR_OK) return s;
   if ((s = upload(g, &g->static_chk_c, sch_c.data(), sch_c.size())) != GR_OK) return s;
+  }
+  // edge payloads: resident copies (streamed mode keeps them in pinned host memory)
+  if (g->mode == GR_MODE_RESIDENT) {
+    if ((s = upload(g, &g->in_src, H.in_src.as<uint32_t>(), mi + 4)) != GR_OK) return s;
+    if ((s = upload(g, &g->out_dst, H.out_dst.as<uint32_t>(), mi + 4)) != GR_OK) return s;
+    if (H.has_w && (s = upload(g, &g->in_w, H.in_w.as<uint8_t>(), mi + 16)) != GR_OK) return s;
+  }
+  if ((s = upload(g, &g->d_outdeg, H.outdeg.data(), n)) != GR_OK) return s;
+  }
   const uint64_t chk_cap = std::max<uint64_t>(std::max(chunks_in, chunks_out), 1);
   for (int i = 0; i < 2; i++) {
     if ((s = dev_alloc(g, (void **)&g->chkA_h[i], 4 * chk_cap)) != GR_OK) return s;
@@ -139,13 +156,6 @@ gr_status load_device(gr_graph *g) {
   if ((s = dev_alloc(g, (void **)&g->hub_acc, 4ull * g->hub_cap)) != GR_OK) return s;
   if ((s = dev_alloc(g, (void **)&g->hub_done, 4ull * g->hub_cap)) != GR_OK) return s;
   CK(cudaMemset(g->hub_done, 0, 4ull * g->hub_cap));
-
-  // edge payloads: resident copies (streamed mode keeps them in pinned host memory)
-  if (g->mode == GR_MODE_RESIDENT) {
-    if ((s = upload(g, &g->in_src, H.in_src.as<uint32_t>(), mi + 4)) != GR_OK) return s;
-    if ((s = upload(g, &g->out_dst, H.out_dst.as<uint32_t>(), mi + 4)) != GR_OK) return s;
-    if (H.has_w && (s = upload(g, &g->in_w, H.in_w.as<uint8_t>(), mi + 16)) != GR_OK) return s;
-  }
 
   // vertex state (replicated values, owned frontier structures)
   const size_t ow = std::max<uint64_t>(own_n, 1);
@@ -168,7 +178,6 @@ gr_status load_device(gr_graph *g) {
   if ((s = dev_alloc(g, (void **)&g->trace, 32ull * g->trace_cap)) != GR_OK) return s;
 
   // PageRank state
-  if ((s = upload(g, &g->d_outdeg, H.outdeg.data(), n)) != GR_OK) return s;
   if ((s = dev_alloc(g, (void **)&g->inv_outdeg, 4 * n)) != GR_OK) return s;
   k_inv_outdeg<<<g->num_sms * 4, 256, 0, g->stream>>>((uint32_t)n, g->d_outdeg, g->inv_outdeg);
   CK(cudaGetLastError());
@@ -382,6 +391,9 @@ template <class OffT> static gr_status pr_hot_setup(gr_graph *g) {
     const std::string v(k);
     g->pr_kernel = v == "block" ? 0 : v == "blockhot" ? 1 : v == "warp" ? 2 : v == "warphot" ? 3 : v == "range" ? 4 : 5;
   }
+  const HostGraph &H = g->H;
+  const bool hot_ok = g->mode == GR_MODE_RESIDENT && !g->comm && H.n < 0x80000000ull && H.m_in >= (1u << 20);
+  if ((g->pr_kernel == 1 || g->pr_kernel == 3 || g->pr_kernel == 5) && !hot_ok) g->pr_kernel -= 1;
   if (g->pr_kernel == 4) {
     g->hot_smem = 32 * sizeof(PrWarpSmem);
     CK(cudaFuncSetAttribute(k_pr_warp_range<OffT, false>, cudaFuncAttributeMaxDynamicSharedMemorySize,
@@ -392,11 +404,6 @@ template <class OffT> static gr_status pr_hot_setup(gr_graph *g) {
     return GR_OK;
   }
   if (g->pr_kernel != 1 && g->pr_kernel != 3 && g->pr_kernel != 5) return GR_OK;
-  const HostGraph &H = g->H;
-  if (g->mode != GR_MODE_RESIDENT || g->comm || H.n >= 0x80000000ull || H.m_in < (1u << 20)) {
-    g->pr_kernel -= 1;
-    return GR_OK;
-  }
   std::vector<uint32_t> idx(H.n);
   for (uint64_t v = 0; v < H.n; v++) idx[v] = (uint32_t)v;
   const uint64_t K = std::min<uint64_t>(kHotK, H.n);
@@ -438,7 +445,7 @@ template <class OffT> static gr_status pr_hot_setup(gr_graph *g) {
     CK(cudaOccupancyMaxActiveBlocksPerMultiprocessor(&bps, k_pr_warp_hot<OffT>, 1024, g->hot_smem));
   }
   if (bps < 1) {
-    g->pr_kernel -= 1;
+    g->pr_kernel = 0;  // shared-memory table does not fit: CTA merge-path kernel
     return GR_OK;
   }
   g->hot_grid = (uint32_t)(g->num_sms * bps);
@@ -454,7 +461,7 @@ static void pr_launch_iter(gr_graph *g, cudaStream_t s, uint32_t t, uint32_t ite
   const bool range = g->pr_kernel >= 4;
   if (warp) a.tile_row = g->wtile_row;
   const uint32_t tiles = warp ? g->pr_wtiles : g->pr_tiles;
-  const uint32_t ranges = g->hot_grid * 32;
+  const uint32_t ranges = (tiles + kRangeTiles - 1) / kRangeTiles;
   if (g->pr_hot == 1) {
     k_pr_hot_pack<<<(g->hot_k + 255) / 256, 256, 0, s>>>(a.contrib_in, g->hot_ids, g->hot_contrib, g->hot_k);
     a.in_src = g->pr_src;
@@ -560,7 +567,15 @@ gr_status run(gr_graph *g, const gr_run_opts *oin, gr_run_stats *st) {
     return fail(GR_EINVAL, "source %u >= num_vertices %llu", o.source, (unsigned long long)g->H.n);
   if (o.algo == GR_SSSP && !g->H.has_w) return fail(GR_EINVAL, "SSSP needs edge weights");
   if (o.algo < GR_BFS || o.algo > GR_CUSTOM) return fail(GR_EINVAL, "unknown algo %d", o.algo);
-  if (o.algo == GR_CUSTOM) return fail(GR_EUNSUPPORTED, "no custom program with id %d is registered", o.custom_id);
+  if (o.algo == GR_CUSTOM) {
+    bool known = false, uses_w = false;
+#define GR_X(id, T) if (o.custom_id == id) { known = true; uses_w = T::kUsesWeights; }
+    GR_CUSTOM_PROGRAMS(GR_X)
+#undef GR_X
+    if (!known) return fail(GR_EUNSUPPORTED, "no custom program with id %d is registered", o.custom_id);
+    if (uses_w && !g->H.has_w) return fail(GR_EINVAL, "custom program %d needs edge weights", o.custom_id);
+    if (o.source >= g->H.n) return fail(GR_EINVAL, "source %u >= num_vertices", o.source);
+  }
   if (g->mode == GR_MODE_STREAMED) return run_streamed(g, &o, st);
   cudaStream_t s = o.stream ? (cudaStream_t)o.stream : g->stream;
   CK(cudaEventRecord(g->ev_start, s));
@@ -586,6 +601,14 @@ gr_status run(gr_graph *g, const gr_run_opts *oin, gr_run_stats *st) {
       break;
     case GR_CC:
       r = g->off64 ? run_frontier<ProgCC, uint64_t>(g, &o, s, st, 3) : run_frontier<ProgCC, uint32_t>(g, &o, s, st, 3);
+      break;
+    case GR_CUSTOM:
+      r = GR_EUNSUPPORTED;
+#define GR_X(id, T)                                                                                        \
+  if (o.custom_id == id)                                                                                   \
+    r = g->off64 ? run_frontier<T, uint64_t>(g, &o, s, st, 16 + id) : run_frontier<T, uint32_t>(g, &o, s, st, 16 + id);
+      GR_CUSTOM_PROGRAMS(GR_X)
+#undef GR_X
       break;
     default:
       r = g->off64 ? run_pagerank<uint64_t>(g, &o, s, st) : run_pagerank<uint32_t>(g, &o, s, st);

@@ -34,6 +34,8 @@ struct gr_graph {
   uint32_t *hub_acc = nullptr, *hub_done = nullptr;
   uint32_t *static_chk_h = nullptr, *static_chk_c = nullptr;
   uint32_t n_static_chunks = 0, hub_cap = 0;
+  bool dev_built = false;        // layout built on the GPU (device_build.cu)
+  uint64_t dev_hubs_in = 0, dev_chunks_in = 0, dev_hubs_out = 0, dev_chunks_out = 0;
 
   // frontier-program state
   uint32_t *val = nullptr, *stamp = nullptr;
@@ -119,6 +121,7 @@ const char *last_error();
 void clear_error();
 gr_status dev_alloc(gr_graph *g, void **p, size_t bytes);
 gr_status load_device(gr_graph *g);
+gr_status device_build(gr_graph *g, const gr_edges *E, uint64_t shard_edges);
 gr_status run(gr_graph *g, const gr_run_opts *o, gr_run_stats *st);
 gr_status fetch_values(gr_graph *g, void *dst, uint64_t bytes);
 gr_status fetch_trace(gr_graph *g, uint64_t *dst, uint64_t max_rows, uint64_t *rows);

@@ -261,6 +261,13 @@ gr_status run_part(gr_graph *g, const gr_run_opts *o, cudaStream_t s, gr_run_sta
                       : run_frontier_part<ProgSSSP, uint32_t>(g, o, s, st);
     case GR_CC:
       return g->off64 ? run_frontier_part<ProgCC, uint64_t>(g, o, s, st) : run_frontier_part<ProgCC, uint32_t>(g, o, s, st);
+    case GR_CUSTOM:
+#define GR_X(id, T)                                                                                         \
+  if (o->custom_id == id)                                                                                   \
+    return g->off64 ? run_frontier_part<T, uint64_t>(g, o, s, st) : run_frontier_part<T, uint32_t>(g, o, s, st);
+      GR_CUSTOM_PROGRAMS(GR_X)
+#undef GR_X
+      return fail(GR_EUNSUPPORTED, "no custom program %d", o->custom_id);
     default:
       return g->off64 ? run_pagerank_part<uint64_t>(g, o, s, st) : run_pagerank_part<uint32_t>(g, o, s, st);
   }

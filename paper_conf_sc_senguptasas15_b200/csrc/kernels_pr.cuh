@@ -371,6 +371,8 @@ __global__ void k_pr_fixup_warp(const __grid_constant__ PrArgs<OffT> a, uint32_t
 // tile to the next, so a row split between two tiles of the same warp is
 // finished by that warp. Only rows that cross a warp-range boundary are left to
 // k_pr_fixup (one head/carry record per warp range, indexed by the global warp).
+constexpr uint32_t kRangeTiles = 8;  // warp tiles per chunk (2048 items)
+
 template <class OffT, bool kHot>
 __device__ __forceinline__ void pr_warp_range(const PrArgs<OffT> &a, uint32_t wid, uint32_t t0, uint32_t t1,
                                               PrWarpSmem &S, const float *s_hot) {
@@ -495,11 +497,16 @@ __global__ void __launch_bounds__(1024, 1) k_pr_warp_range(const __grid_constant
       *reinterpret_cast<float4 *>(s_hot + k) = __ldg(reinterpret_cast<const float4 *>(hot_contrib + k));
     __syncthreads();
   }
+  // interleaved chunks of kRangeTiles contiguous tiles: balanced across warps
+  // (hot/cold source mix varies along the graph), carries stay in registers
+  // inside a chunk, one head/carry record per chunk for k_pr_fixup
   const uint32_t w = threadIdx.x >> 5, nw = blockDim.x >> 5;
   const uint32_t wid = blockIdx.x * nw + w, W = gridDim.x * nw;
-  const uint32_t per = (num_tiles + W - 1) / W;
-  const uint32_t t0 = min(wid * per, num_tiles), t1 = min(t0 + per, num_tiles);
-  pr_warp_range<OffT, kHot>(a, wid, t0, t1, S[w], s_hot);
+  const uint32_t nchunks = (num_tiles + kRangeTiles - 1) / kRangeTiles;
+  for (uint32_t c = wid; c < nchunks; c += W) {
+    const uint32_t t0 = c * kRangeTiles, t1 = min(t0 + kRangeTiles, num_tiles);
+    pr_warp_range<OffT, kHot>(a, c, t0, t1, S[w], s_hot);
+  }
 }
 
 // hot_contrib[k] = contrib[hot_ids[k]] (after the previous superstep finished)

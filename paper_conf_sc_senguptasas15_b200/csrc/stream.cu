@@ -359,6 +359,14 @@ gr_status run_streamed(gr_graph *g, const gr_run_opts *o, gr_run_stats *st) {
     case GR_CC:
       r = g->off64 ? stream_frontier<ProgCC, uint64_t>(g, o, cs, st) : stream_frontier<ProgCC, uint32_t>(g, o, cs, st);
       break;
+    case GR_CUSTOM:
+      r = GR_EUNSUPPORTED;
+#define GR_X(id, T)                                                                                           \
+  if (o->custom_id == id)                                                                                     \
+    r = g->off64 ? stream_frontier<T, uint64_t>(g, o, cs, st) : stream_frontier<T, uint32_t>(g, o, cs, st);
+      GR_CUSTOM_PROGRAMS(GR_X)
+#undef GR_X
+      break;
     default:
       r = g->off64 ? stream_pagerank<uint64_t>(g, o, cs, st) : stream_pagerank<uint32_t>(g, o, cs, st);
   }

@@ -88,3 +88,35 @@ def test_sim_ranks_hubs_and_configs():
     for st, vals, tr, info in run_sim_ranks(g.n, g.src, g.dst, g.w, 2, "sssp", source=0):
         np.testing.assert_array_equal(vals, ref)
         np.testing.assert_array_equal(tr, rtr)
+
+
+@pytest.mark.timeout(600)
+def test_sim_ranks_custom_program():
+    g = grgen.rmat(12, 16, seed=3)
+    w = grgen.weights(g.m, 1, 64, seed=4)
+    ref, rtr, rit = oracle.run(g.n, g.src, g.dst, "widest", w=w, source=0)
+    import os
+    import threading
+
+    key = os.urandom(128)
+    out, errs = [None] * 2, []
+
+    def worker(r):
+        h = None
+        try:
+            h = gr.gr_graph_load(g.n, g.src, g.dst, w, world=2, rank=r, sim_ranks=2, nccl_unique_id=key)
+            gr.gr_run(h, "custom", custom_id=0, source=0)
+            out[r] = (gr.gr_fetch_vertex_values(h), gr.gr_fetch_frontier_trace(h))
+        except Exception as e:
+            errs.append(e)
+        finally:
+            if h:
+                gr.gr_graph_free(h)
+
+    th = [threading.Thread(target=worker, args=(r,)) for r in range(2)]
+    [t.start() for t in th]
+    [t.join(timeout=300) for t in th]
+    assert not errs, errs
+    for vals, tr in out:
+        np.testing.assert_array_equal(vals, ref)
+        np.testing.assert_array_equal(tr, rtr)

@@ -232,3 +232,54 @@ def test_pagerank_kernel_variants(variant, monkeypatch):
     with gr.GraphReduce(n, src, dst) as G:
         G.run("pagerank")
         check_pr(G.values("pagerank"), ref, n)
+
+
+@pytest.mark.parametrize("seed", [1, 2])
+def test_device_build_matches_host_build(seed):
+    """The GPU shard builder produces the host builder's layout exactly: every
+    program (PageRank included, same fp32 summation order) is bit-identical,
+    and the shard tables agree."""
+    g = grgen.rmat(14, 16, seed=seed)
+    w = grgen.weights(g.m, 1, 64, seed=seed)
+    src = np.concatenate([g.src, g.src[:5000]])  # extra duplicates with other weights
+    dst = np.concatenate([g.dst, g.dst[:5000]])
+    w = np.concatenate([w, (w[:5000] % 7) + 1]).astype(np.uint32)
+    res = {}
+    for build in ("host", "device"):
+        with gr.GraphReduce(g.n, src, dst, w, build=build, shard_edges=50000) as G:
+            info = G.info()
+            shards = [gr.gr_shard_info(G.h, s) for s in range(info["num_shards"])]
+            out = {"shards": shards}
+            for algo in ("bfs", "sssp", "cc", "pagerank"):
+                G.run(algo, source=3)
+                out[algo] = (G.values(algo), G.trace())
+            res[build] = out
+    assert res["host"]["shards"] == res["device"]["shards"]
+    for algo in ("bfs", "sssp", "cc", "pagerank"):
+        np.testing.assert_array_equal(res["host"][algo][0], res["device"][algo][0])
+        np.testing.assert_array_equal(res["host"][algo][1], res["device"][algo][1])
+    with pytest.raises(gr.GrError):
+        gr.GraphReduce(4, np.array([0, 9], np.uint32), np.array([1, 2], np.uint32), build="device")
+
+
+@pytest.mark.parametrize("mode", ["resident", "streamed"])
+def test_custom_program_widest_path(mode):
+    """A user program registered with GR_CUSTOM_PROGRAMS (include/gr/program.cuh)
+    runs through the same engine and equals the oracle's widest path exactly."""
+    for seed in (1, 2):
+        g = grgen.rmat(12, 16, seed=seed)
+        w = grgen.weights(g.m, 1, 64, seed=seed + 7)
+        ref, rtr, rit = oracle.run(g.n, g.src, g.dst, "widest", w=w, source=0)
+        kw = dict(mode=mode, shard_edges=6000) if mode == "streamed" else {}
+        with gr.GraphReduce(g.n, g.src, g.dst, w, **kw) as G:
+            for loop in (("auto", "device", "host") if mode == "resident" else ("host",)):
+                st = G.run("custom", custom_id=0, source=0, loop=loop)
+                assert st["iterations"] == rit
+                np.testing.assert_array_equal(G.values(), ref)
+                np.testing.assert_array_equal(G.trace(), rtr)
+    n, src, dst, w = hub_graph()
+    ref, rtr, _ = oracle.run(n, src, dst, "widest", w=w, source=5)
+    with gr.GraphReduce(n, src, dst, w) as G:
+        G.run("custom", custom_id=0, source=5)
+        np.testing.assert_array_equal(G.values(), ref)
+        np.testing.assert_array_equal(G.trace(), rtr)

@@ -415,3 +415,44 @@ def test_trace_vs_bruteforce(algo, seed):
 def test_oracle_rejects_bad_input():
     with pytest.raises(ValueError):
         oracle.OracleGraph(4, np.array([0, 5], np.uint32), np.array([1, 2], np.uint32))
+
+
+# ------------------------------------------------- widest path (user program)
+def maxmin_dijkstra(n, src, dst, w, s):
+    """Textbook widest path: Dijkstra on the (max, min) semiring."""
+    adj = collections.defaultdict(list)
+    for a, b, c in zip(src.tolist(), dst.tolist(), w.tolist()):
+        adj[a].append((b, c))
+    width = [0] * n
+    width[s] = INF
+    h = [(-INF, s)]
+    while h:
+        negw, u = heapq.heappop(h)
+        if -negw < width[u]:
+            continue
+        for x, c in adj[u]:
+            cand = min(width[u], c)
+            if cand > width[x]:
+                width[x] = cand
+                heapq.heappush(h, (-cand, x))
+    return np.array(width, np.uint32)
+
+
+@pytest.mark.parametrize("seed", range(10))
+def test_widest_vs_maxmin_dijkstra(seed):
+    rng = np.random.default_rng(700 + seed)
+    n = int(rng.integers(2, 60))
+    src, dst, w = rand_graph(rng, n, int(rng.integers(0, 4 * n)), wmax=64)
+    s = int(rng.integers(0, n))
+    vals, tr, _ = oracle.run(n, src, dst, "widest", w=w, source=s)
+    np.testing.assert_array_equal(vals, maxmin_dijkstra(n, src, dst, w, s))
+
+
+def test_widest_path_prefix_min():
+    rng = np.random.default_rng(9)
+    n = 30
+    w = rng.integers(1, 65, n - 1).astype(np.uint32)
+    src = np.arange(n - 1, dtype=np.uint32)
+    vals, _, _ = oracle.run(n, src, src + 1, "widest", w=w, source=0)
+    exp = np.concatenate([[INF], np.minimum.accumulate(w)]).astype(np.uint32)
+    np.testing.assert_array_equal(vals, exp)
