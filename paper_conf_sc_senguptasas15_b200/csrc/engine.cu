@@ -64,10 +64,16 @@ gr_status dev_alloc(gr_graph *g, void **p, size_t bytes) {
   return GR_OK;
 }
 
+// Every setup transfer is ordered on the graph's (non-blocking) stream: a plain
+// cudaMemcpy from pageable memory may return before its DMA lands, and
+// cudaMemset is asynchronous — neither is ordered with kernels on g->stream.
 template <class T> static gr_status upload(gr_graph *g, T **dst, const T *src, size_t count) {
   gr_status s = dev_alloc(g, (void **)dst, count * sizeof(T));
   if (s != GR_OK) return s;
-  if (count) CK(cudaMemcpy(*dst, src, count * sizeof(T), cudaMemcpyHostToDevice));
+  if (count) {
+    CK(cudaMemcpyAsync(*dst, src, count * sizeof(T), cudaMemcpyHostToDevice, g->stream));
+    CK(cudaStreamSynchronize(g->stream));  // the host buffer may be freed on return
+  }
   return GR_OK;
 }
 
@@ -155,13 +161,13 @@ gr_status load_device(gr_graph *g) {
   g->hub_cap = (uint32_t)std::max<uint64_t>(std::max(hubs_in, hubs_out), 1);
   if ((s = dev_alloc(g, (void **)&g->hub_acc, 4ull * g->hub_cap)) != GR_OK) return s;
   if ((s = dev_alloc(g, (void **)&g->hub_done, 4ull * g->hub_cap)) != GR_OK) return s;
-  CK(cudaMemset(g->hub_done, 0, 4ull * g->hub_cap));
+  CK(cudaMemsetAsync(g->hub_done, 0, 4ull * g->hub_cap, g->stream));
 
   // vertex state (replicated values, owned frontier structures)
   const size_t ow = std::max<uint64_t>(own_n, 1);
   if ((s = dev_alloc(g, (void **)&g->val, 4 * n)) != GR_OK) return s;
   if ((s = dev_alloc(g, (void **)&g->stamp, 4 * ow)) != GR_OK) return s;
-  CK(cudaMemset(g->stamp, 0, 4 * ow));
+  CK(cudaMemsetAsync(g->stamp, 0, 4 * ow, g->stream));
   for (int i = 0; i < 2; i++) {
     if ((s = dev_alloc(g, (void **)&g->listA[i], 4 * ow)) != GR_OK) return s;
     if ((s = dev_alloc(g, (void **)&g->listH[i], 4 * ow)) != GR_OK) return s;
@@ -202,13 +208,29 @@ gr_status load_device(gr_graph *g) {
       k_pr_tiles<uint32_t><<<(g->pr_tiles + 256) / 256, 256, 0, g->stream>>>(
           (const uint32_t *)g->in_off, 0, (uint32_t)own_n, mi, g->pr_tiles, g->tile_row);
     if ((s = dev_alloc(g, (void **)&g->wtile_row, 4ull * (g->pr_wtiles + 1))) != GR_OK) return s;
-    if (g->off64)
+    if ((s = dev_alloc(g, (void **)&g->w_is_long, g->pr_wtiles + 16)) != GR_OK) return s;
+    if ((s = dev_alloc(g, (void **)&g->long_c, 4ull * (g->pr_wtiles + 1))) != GR_OK) return s;
+    if ((s = dev_alloc(g, (void **)&g->long_f, 4ull * (g->pr_wtiles + 1))) != GR_OK) return s;
+    uint32_t *d_nlong = nullptr;
+    CK(cudaMalloc(&d_nlong, 4));
+    CK(cudaMemsetAsync(d_nlong, 0, 4, g->stream));
+    if (g->off64) {
       k_pr_tiles<uint64_t><<<(g->pr_wtiles + 256) / 256, 256, 0, g->stream>>>(
           (const uint64_t *)g->in_off, 0, (uint32_t)own_n, mi, g->pr_wtiles, g->wtile_row, (uint32_t)kWTile);
-    else
+      k_pr_long_heads<uint64_t><<<(g->pr_wtiles + 255) / 256 + 1, 256, 0, g->stream>>>(
+          (const uint64_t *)g->in_off, own_n, mi, g->wtile_row, g->pr_wtiles, kWTile, g->w_is_long, g->long_c,
+          g->long_f, d_nlong);
+    } else {
       k_pr_tiles<uint32_t><<<(g->pr_wtiles + 256) / 256, 256, 0, g->stream>>>(
           (const uint32_t *)g->in_off, 0, (uint32_t)own_n, mi, g->pr_wtiles, g->wtile_row, (uint32_t)kWTile);
+      k_pr_long_heads<uint32_t><<<(g->pr_wtiles + 255) / 256 + 1, 256, 0, g->stream>>>(
+          (const uint32_t *)g->in_off, own_n, mi, g->wtile_row, g->pr_wtiles, kWTile, g->w_is_long, g->long_c,
+          g->long_f, d_nlong);
+    }
     CK(cudaGetLastError());
+    CK(cudaMemcpyAsync(&g->n_long, d_nlong, 4, cudaMemcpyDeviceToHost, g->stream));
+    CK(cudaStreamSynchronize(g->stream));
+    cudaFree(d_nlong);
   }
   CK(cudaStreamSynchronize(g->stream));
 
@@ -348,7 +370,8 @@ static gr_status run_frontier(gr_graph *g, const gr_run_opts *o, cudaStream_t s,
   // 4 B per activated out-edge, 8 B per changed vertex (value commit + offsets)
   std::vector<unsigned long long> tr(4 * g->trace_rows);
   if (g->trace_rows)
-    CK(cudaMemcpy(tr.data(), g->trace, 32 * g->trace_rows, cudaMemcpyDeviceToHost));
+    CK(cudaMemcpyAsync(tr.data(), g->trace, 32 * g->trace_rows, cudaMemcpyDeviceToHost, s));
+  CK(cudaStreamSynchronize(s));
   uint64_t sumA = 0, sumC = 0;
   for (uint64_t t = 0; t < g->trace_rows; t++) { sumA += tr[4 * t]; sumC += tr[4 * t + 1]; }
   const uint64_t wb = Prog::kUsesWeights ? 5 : 4;
@@ -385,15 +408,15 @@ template <class OffT> static PrArgs<OffT> pr_args(gr_graph *g, uint32_t t, uint3
 // of the CSC payload, size the persistent grid from the occupancy calculator.
 template <class OffT> static gr_status pr_hot_setup(gr_graph *g) {
   g->pr_hot = 0;
-  // kernel variant (GR_PR_KERNEL = block | blockhot | warp | warphot | range | rangehot; default rangehot)
-  g->pr_kernel = 5;
+  // kernel variant (GR_PR_KERNEL = block | warp | warphot | range | rangehot; default warphot)
+  g->pr_kernel = 3;
   if (const char *k = getenv("GR_PR_KERNEL")) {
     const std::string v(k);
-    g->pr_kernel = v == "block" ? 0 : v == "blockhot" ? 1 : v == "warp" ? 2 : v == "warphot" ? 3 : v == "range" ? 4 : 5;
+    g->pr_kernel = v == "block" || v == "blockhot" ? 0 : v == "warp" ? 2 : v == "warphot" ? 3 : v == "range" ? 4 : 5;
   }
   const HostGraph &H = g->H;
   const bool hot_ok = g->mode == GR_MODE_RESIDENT && !g->comm && H.n < 0x80000000ull && H.m_in >= (1u << 20);
-  if ((g->pr_kernel == 1 || g->pr_kernel == 3 || g->pr_kernel == 5) && !hot_ok) g->pr_kernel -= 1;
+  if ((g->pr_kernel == 3 || g->pr_kernel == 5) && !hot_ok) g->pr_kernel -= 1;
   if (g->pr_kernel == 4) {
     g->hot_smem = 32 * sizeof(PrWarpSmem);
     CK(cudaFuncSetAttribute(k_pr_warp_range<OffT, false>, cudaFuncAttributeMaxDynamicSharedMemorySize,
@@ -403,10 +426,12 @@ template <class OffT> static gr_status pr_hot_setup(gr_graph *g) {
     g->hot_grid = (uint32_t)(g->num_sms * std::max(bps, 1));
     return GR_OK;
   }
-  if (g->pr_kernel != 1 && g->pr_kernel != 3 && g->pr_kernel != 5) return GR_OK;
+  if (g->pr_kernel != 3 && g->pr_kernel != 5) return GR_OK;
   std::vector<uint32_t> idx(H.n);
   for (uint64_t v = 0; v < H.n; v++) idx[v] = (uint32_t)v;
-  const uint64_t K = std::min<uint64_t>(kHotK, H.n);
+  uint64_t K = kHotK;
+  if (const char *hk = getenv("GR_PR_HOTK")) K = std::max<uint64_t>(4, std::min<uint64_t>(strtoull(hk, nullptr, 10), 49152));
+  K = std::min<uint64_t>(K, H.n);
   std::partial_sort(idx.begin(), idx.begin() + K, idx.end(), [&](uint32_t a, uint32_t b) {
     return H.outdeg[a] != H.outdeg[b] ? H.outdeg[a] > H.outdeg[b] : a < b;
   });
@@ -423,7 +448,7 @@ template <class OffT> static gr_status pr_hot_setup(gr_graph *g) {
   if ((s = dev_alloc(g, (void **)&g->hot_contrib, 4ull * std::max<uint32_t>(g->hot_k, 4))) != GR_OK) return s;
   if ((s = dev_alloc(g, (void **)&g->pr_src, 4 * (H.m_in + 4))) != GR_OK) return s;
   CK(cudaMalloc(&d_slot, 4 * H.n));
-  CK(cudaMemcpy(d_slot, slot.data(), 4 * H.n, cudaMemcpyHostToDevice));
+  CK(cudaMemcpyAsync(d_slot, slot.data(), 4 * H.n, cudaMemcpyHostToDevice, g->stream));
   k_pr_tag<<<g->num_sms * 8, 256, 0, g->stream>>>(g->in_src, H.m_in, d_slot, g->pr_src);
   CK(cudaGetLastError());
   CK(cudaStreamSynchronize(g->stream));
@@ -434,15 +459,12 @@ template <class OffT> static gr_status pr_hot_setup(gr_graph *g) {
     CK(cudaFuncSetAttribute(k_pr_warp_range<OffT, true>, cudaFuncAttributeMaxDynamicSharedMemorySize,
                             (int)g->hot_smem));
     CK(cudaOccupancyMaxActiveBlocksPerMultiprocessor(&bps, k_pr_warp_range<OffT, true>, 1024, g->hot_smem));
-  } else if (g->pr_kernel == 1) {
-    g->hot_smem = sizeof(PrSmem) + 4ull * g->hot_k;
-    CK(cudaFuncSetAttribute(k_pr_gather_apply_hot<OffT>, cudaFuncAttributeMaxDynamicSharedMemorySize,
-                            (int)g->hot_smem));
-    CK(cudaOccupancyMaxActiveBlocksPerMultiprocessor(&bps, k_pr_gather_apply_hot<OffT>, kPrThreads, g->hot_smem));
   } else {
-    g->hot_smem = 4ull * g->hot_k + 32 * sizeof(PrWarpSmem);
+    g->hot_cta = 1024;
+    if (const char *ct = getenv("GR_PR_CTA")) g->hot_cta = std::max(64, std::min(1024, atoi(ct))) & ~31;
+    g->hot_smem = 4ull * g->hot_k + (g->hot_cta / 32) * sizeof(PrWarpSmem);
     CK(cudaFuncSetAttribute(k_pr_warp_hot<OffT>, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)g->hot_smem));
-    CK(cudaOccupancyMaxActiveBlocksPerMultiprocessor(&bps, k_pr_warp_hot<OffT>, 1024, g->hot_smem));
+    CK(cudaOccupancyMaxActiveBlocksPerMultiprocessor(&bps, k_pr_warp_hot<OffT>, g->hot_cta, g->hot_smem));
   }
   if (bps < 1) {
     g->pr_kernel = 0;  // shared-memory table does not fit: CTA merge-path kernel
@@ -471,12 +493,8 @@ static void pr_launch_iter(gr_graph *g, cudaStream_t s, uint32_t t, uint32_t ite
     case 0:
       k_pr_gather_apply<OffT><<<std::max<uint32_t>(tiles, 1), kPrThreads, 0, s>>>(a);
       break;
-    case 1:
-      k_pr_gather_apply_hot<OffT><<<std::min(g->hot_grid, std::max<uint32_t>(tiles, 1)), kPrThreads, g->hot_smem, s>>>(
-          a, g->hot_contrib, g->hot_k, tiles);
-      break;
     case 3:
-      k_pr_warp_hot<OffT><<<g->hot_grid, 1024, g->hot_smem, s>>>(a, g->hot_contrib, g->hot_k, tiles);
+      k_pr_warp_hot<OffT><<<g->hot_grid, g->hot_cta, g->hot_smem, s>>>(a, g->hot_contrib, g->hot_k, tiles);
       break;
     case 4:
       k_pr_warp_range<OffT, false><<<g->hot_grid, 1024, g->hot_smem, s>>>(a, nullptr, 0, tiles);
@@ -490,8 +508,10 @@ static void pr_launch_iter(gr_graph *g, cudaStream_t s, uint32_t t, uint32_t ite
   if (e1) cudaEventRecord(e1, s);
   if (range)
     k_pr_fixup<OffT><<<(ranges + 255) / 256, 256, 0, s>>>(a, ranges);
-  else if (warp)
-    k_pr_fixup_warp<OffT><<<std::max<uint32_t>((tiles + 7) / 8, 1), 256, 0, s>>>(a, tiles);
+  else if (warp) {
+    k_pr_fixup_short<OffT><<<std::max<uint32_t>((tiles + 255) / 256, 1), 256, 0, s>>>(a, tiles, g->w_is_long);
+    if (g->n_long) k_pr_fixup_long<OffT><<<(g->n_long + 7) / 8, 256, 0, s>>>(a, g->long_c, g->long_f, g->n_long);
+  }
   else
     k_pr_fixup<OffT><<<std::max<uint32_t>((tiles + 255) / 256, 1), 256, 0, s>>>(a, tiles);
 }
@@ -632,8 +652,9 @@ gr_status fetch_values(gr_graph *g, void *dst, uint64_t bytes) {
   if (bytes < 4 * n) return fail(GR_EINVAL, "buffer of %llu bytes < 4*n = %llu", (unsigned long long)bytes,
                                  (unsigned long long)(4 * n));
   if (g->comm) return part_fetch_values(g, dst, bytes);
-  if (g->last_algo == GR_PAGERANK) CK(cudaMemcpy(dst, g->rank, 4 * n, cudaMemcpyDeviceToHost));
-  else CK(cudaMemcpy(dst, g->val, 4 * n, cudaMemcpyDeviceToHost));
+  CK(cudaMemcpyAsync(dst, g->last_algo == GR_PAGERANK ? (const void *)g->rank : (const void *)g->val, 4 * n,
+                     cudaMemcpyDeviceToHost, g->stream));
+  CK(cudaStreamSynchronize(g->stream));
   return GR_OK;
 }
 
@@ -650,7 +671,8 @@ gr_status fetch_trace(gr_graph *g, uint64_t *dst, uint64_t max_rows, uint64_t *r
       dst[4 * t + 3] = 0;
     }
   } else if (r) {
-    CK(cudaMemcpy(dst, g->trace, 32 * r, cudaMemcpyDeviceToHost));
+    CK(cudaMemcpyAsync(dst, g->trace, 32 * r, cudaMemcpyDeviceToHost, g->stream));
+    CK(cudaStreamSynchronize(g->stream));
   }
   *rows = r;
   return GR_OK;

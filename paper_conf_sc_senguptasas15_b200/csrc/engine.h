@@ -57,7 +57,10 @@ struct gr_graph {
   uint32_t *tile_row = nullptr;  // merge-path tile starts (resident: [pr_tiles+1]; streamed: per shard)
   uint32_t pr_wtiles = 0;          // warp-granular tiles (kWTile items)
   uint32_t *wtile_row = nullptr;
-  int pr_kernel = -1;              // 0 block, 1 block+hot, 2 warp, 3 warp+hot
+  int pr_kernel = -1;              // 0 block, 2 warp, 3 warp+hot, 4 warp range, 5 warp range+hot
+  uint8_t *w_is_long = nullptr;    // warp tiles whose head row began > kShortChain tiles earlier
+  uint32_t *long_c = nullptr, *long_f = nullptr, n_long = 0;
+  int hot_cta = 1024;
   cudaGraphExec_t pr_exec = nullptr;
   uint32_t pr_exec_iters = 0;
   float pr_exec_d = 0.f;

@@ -208,9 +208,11 @@ gr_status part_fetch_values(gr_graph *g, void *dst, uint64_t bytes) {
     owner_bytes(g, 4, &cnt, &dsp);
     XCK(g->comm->allgatherv(g->rank, g->rank_all, cnt, dsp, g->stream));
     PCK(cudaStreamSynchronize(g->stream));
-    PCK(cudaMemcpy(dst, g->rank_all, 4 * n, cudaMemcpyDeviceToHost));
+    PCK(cudaMemcpyAsync(dst, g->rank_all, 4 * n, cudaMemcpyDeviceToHost, g->stream));
+    PCK(cudaStreamSynchronize(g->stream));
   } else {
-    PCK(cudaMemcpy(dst, g->val, 4 * n, cudaMemcpyDeviceToHost));
+    PCK(cudaMemcpyAsync(dst, g->val, 4 * n, cudaMemcpyDeviceToHost, g->stream));
+    PCK(cudaStreamSynchronize(g->stream));
   }
   (void)bytes;
   return GR_OK;
@@ -235,11 +237,15 @@ gr_status part_fetch_trace(gr_graph *g, uint64_t *dst, uint64_t max_rows, uint64
   for (int q = 0; q < C->world; q++) dsp[q] = 32 * r * q;
   char *base = nullptr;
   PCK(cudaMalloc((void **)&base, 32 * std::max<uint64_t>(r, 1) * C->world));
+  PCK(cudaStreamSynchronize(g->stream));  // the trace of the last run is complete
   PCK(cudaMemcpyAsync(base + 32 * r * C->rank, g->trace, 32 * r, cudaMemcpyDeviceToDevice, g->stream));
   gr_status xs = C->allgatherv(base + 32 * r * C->rank, base, cnt, dsp, g->stream);
   std::vector<uint64_t> all(4 * r * C->world);
   cudaError_t ce = cudaStreamSynchronize(g->stream);
-  if (xs == GR_OK && ce == cudaSuccess && r) ce = cudaMemcpy(all.data(), base, 32 * r * C->world, cudaMemcpyDeviceToHost);
+  if (xs == GR_OK && ce == cudaSuccess && r) {
+    ce = cudaMemcpyAsync(all.data(), base, 32 * r * C->world, cudaMemcpyDeviceToHost, g->stream);
+    if (ce == cudaSuccess) ce = cudaStreamSynchronize(g->stream);
+  }
   cudaFree(base);
   if (xs != GR_OK) return fail(xs, "trace exchange failed");
   if (ce != cudaSuccess) return fail(GR_ECUDA, "trace exchange: %s", cudaGetErrorString(ce));

@@ -203,8 +203,12 @@ __device__ __forceinline__ uint32_t activate_batch(const Part<OffT> &P, const bo
                                                    const uint32_t (&x)[kBatch], uint32_t epoch,
                                                    const uint32_t *hub_bits, WarpQueue &qA, uint32_t slot) {
   uint32_t st[kBatch];
+  bool hb[kBatch];
 #pragma unroll
-  for (int q = 0; q < kBatch; q++) st[q] = act[q] ? ld_cg(P.stamp + (x[q] - P.own_lo)) : epoch;
+  for (int q = 0; q < kBatch; q++) {
+    st[q] = act[q] ? ld_cg(P.stamp + (x[q] - P.own_lo)) : epoch;
+    hb[q] = act[q] && test_bit(hub_bits, kBfsFilter ? x[q] : x[q] - P.own_lo);  // issued with the stamp read
+  }
   bool nw[kBatch];
 #pragma unroll
   for (int q = 0; q < kBatch; q++) {
@@ -220,7 +224,7 @@ __device__ __forceinline__ uint32_t activate_batch(const Part<OffT> &P, const bo
   uint32_t cnt = 0;
 #pragma unroll
   for (int q = 0; q < kBatch; q++) {
-    const bool hub = keep[q] && test_bit(hub_bits, kBfsFilter ? x[q] : x[q] - P.own_lo);
+    const bool hub = keep[q] && hb[q];
     if (hub) append_hub_A<kBfsFilter>(P, x[q], slot);
     qA.push(keep[q] && !hub, x[q], 0, P.listA[slot], nullptr, &P.ctl->cnt_A[slot]);
     cnt += __popc(__ballot_sync(0xffffffffu, nw[q]));
@@ -414,12 +418,14 @@ __device__ __forceinline__ void gather_phase(const Part<OffT> &P, const View &V)
     if (valid && implicit && test_bit(P.hub_in, lv)) valid = false;  // served by the hub chunks
     uint64_t beg = 0;
     uint32_t deg = 0, cur = 0;
+    bool hubv = false;
     if (valid) {
       if (Prog::kHasGather) {
         beg = (uint64_t)P.in_off[lv];
         deg = (uint32_t)((uint64_t)P.in_off[lv + 1] - beg);
       }
       cur = P.val[v];
+      hubv = !no_hub_c && test_bit(P.hub_out, v);  // issued with the offsets, used after apply
     }
     const G acc = Prog::kHasGather ? gather_warp<Prog>(P, valid, beg, deg, cur, sred[warp], cx) : Prog::identity();
     bool changed = false;
@@ -428,7 +434,7 @@ __device__ __forceinline__ void gather_phase(const Part<OffT> &P, const View &V)
       changed = Prog::apply(&nv, acc, cx);
       my_g += deg;
     }
-    const bool hubo = changed && !no_hub_c && test_bit(P.hub_out, v);
+    const bool hubo = changed && hubv;
     if (hubo) append_hub_C(P, v, nv);
     qC.push(changed && !hubo, v, nv, P.C_v, P.C_val, &ctl->cnt_C);
     my_c += changed ? 1 : 0;

@@ -198,23 +198,6 @@ __global__ void __launch_bounds__(kPrThreads, 6) k_pr_gather_apply(const __grid_
   pr_tile<OffT, false>(a, blockIdx.x, S, nullptr);
 }
 
-// Persistent variant (2 CTAs per SM): the CTA first copies the hot sources'
-// contributions (hot_contrib[kHotK], packed by k_pr_hot_pack) into shared
-// memory, then walks tiles blockIdx.x, +gridDim.x, ...; a.in_src is the
-// tagged PageRank payload.
-template <class OffT>
-__global__ void __launch_bounds__(kPrThreads, 2) k_pr_gather_apply_hot(const __grid_constant__ PrArgs<OffT> a,
-                                                                        const float *hot_contrib, uint32_t hot_k,
-                                                                        uint32_t num_tiles) {
-  extern __shared__ __align__(16) unsigned char smem_raw[];
-  PrSmem &S = *reinterpret_cast<PrSmem *>(smem_raw);
-  float *s_hot = reinterpret_cast<float *>(smem_raw + sizeof(PrSmem));
-  for (uint32_t k = threadIdx.x * 4; k < hot_k; k += kPrThreads * 4) {
-    const float4 v = __ldg(reinterpret_cast<const float4 *>(hot_contrib + k));
-    *reinterpret_cast<float4 *>(s_hot + k) = v;
-  }
-  for (uint32_t tile = blockIdx.x; tile < num_tiles; tile += gridDim.x) pr_tile<OffT, true>(a, tile, S, s_hot);
-}
 
 
 // ---------------------------------------------------------------------------
@@ -337,6 +320,64 @@ __global__ void __launch_bounds__(1024, 1) k_pr_warp_hot(const __grid_constant__
   const uint32_t w = threadIdx.x >> 5, nw = blockDim.x >> 5;
   for (uint32_t tile = blockIdx.x * nw + w; tile < num_tiles; tile += gridDim.x * nw)
     pr_warp_tile<OffT, true>(a, tile, S[w], s_hot);
+}
+
+// Long chains (a head whose row began more than kShortChain tiles earlier) are
+// listed once per graph by k_pr_long_heads and finished one warp each by
+// k_pr_fixup_long; every other head is finished by one thread (k_pr_fixup_short).
+constexpr uint32_t kShortChain = 8;
+
+template <class OffT>
+__global__ void k_pr_long_heads(const OffT *in_off, uint64_t rows, uint64_t nnz, const uint32_t *tile_row,
+                                uint32_t num_tiles, uint32_t tile_items, uint8_t *is_long, uint32_t *long_c,
+                                uint32_t *long_f, uint32_t *long_n) {
+  const uint64_t total = rows + nnz;
+  for (uint32_t c = blockIdx.x * blockDim.x + threadIdx.x; c < num_tiles; c += gridDim.x * blockDim.x) {
+    const uint32_t i0 = tile_row[c], i1 = tile_row[c + 1];
+    const uint64_t d0 = (uint64_t)c * tile_items;
+    const uint64_t j0 = d0 - i0;
+    const uint64_t rs = (uint64_t)in_off[i0];
+    bool lng = false;
+    if (i1 > i0 && rs < j0) {
+      // the row's first item sits on merge-path diagonal i0 + rs
+      const uint32_t f = (uint32_t)(((uint64_t)i0 + rs) / tile_items);
+      if (c - f > kShortChain) {
+        lng = true;
+        const uint32_t pos = atomicAdd(long_n, 1u);
+        long_c[pos] = c;
+        long_f[pos] = f;
+      }
+    }
+    is_long[c] = lng ? 1 : 0;
+    (void)total;
+  }
+}
+
+template <class OffT>
+__global__ void k_pr_fixup_short(const __grid_constant__ PrArgs<OffT> a, uint32_t num_tiles, const uint8_t *is_long) {
+  for (uint32_t c = blockIdx.x * blockDim.x + threadIdx.x; c < num_tiles; c += gridDim.x * blockDim.x) {
+    const uint32_t row = a.head_row[c];
+    if (row == kNoRow || is_long[c]) continue;
+    float acc = a.head_val[c];
+    for (int64_t p = (int64_t)c - 1; p >= 0 && a.carry_row[p] == row; p--) acc += a.carry_val[p];
+    pr_apply_row(a, row, acc);
+  }
+}
+
+template <class OffT>
+__global__ void k_pr_fixup_long(const __grid_constant__ PrArgs<OffT> a, const uint32_t *long_c, const uint32_t *long_f,
+                                uint32_t n_long) {
+  const uint32_t lane = threadIdx.x & 31;
+  const uint32_t nw = (gridDim.x * blockDim.x) >> 5;
+  for (uint32_t i = (blockIdx.x * blockDim.x + threadIdx.x) >> 5; i < n_long; i += nw) {
+    const uint32_t c = long_c[i], f = long_f[i];
+    const uint32_t row = a.head_row[c];
+    float acc = 0.f;
+    for (uint32_t p = f + lane; p < c; p += 32) acc += a.carry_val[p];  // tiles f..c-1 all carry this row
+#pragma unroll
+    for (int o = 16; o > 0; o >>= 1) acc += __shfl_xor_sync(0xffffffffu, acc, o);
+    if (lane == 0 && row != kNoRow) pr_apply_row(a, row, a.head_val[c] + acc);
+  }
 }
 
 // Rows spanning warp tiles: one warp per tile with a head; the preceding

@@ -93,12 +93,12 @@ gr_status stream_setup(gr_graph *g, uint64_t budget) {
   }
   SCK(cudaStreamCreateWithFlags(&S->copy_s, cudaStreamNonBlocking));
   if ((st = dev_alloc(g, (void **)&S->d_bounds, 8ull * (S->P + 1))) != GR_OK) return st;
-  SCK(cudaMemcpy(S->d_bounds, H.bounds.data(), 8ull * (S->P + 1), cudaMemcpyHostToDevice));
+  SCK(cudaMemcpyAsync(S->d_bounds, H.bounds.data(), 8ull * (S->P + 1), cudaMemcpyHostToDevice, g->stream));
   if ((st = dev_alloc(g, (void **)&S->d_next, S->P)) != GR_OK) return st;
   if ((st = dev_alloc(g, (void **)&S->d_changed, S->P)) != GR_OK) return st;
   SCK(cudaMallocHost((void **)&S->h_flags, 2ull * S->P + 16));
   if ((st = dev_alloc(g, (void **)&S->cstamp, 4ull * std::max<uint64_t>(H.own_n(), 1))) != GR_OK) return st;
-  SCK(cudaMemset(S->cstamp, 0, 4ull * std::max<uint64_t>(H.own_n(), 1)));
+  SCK(cudaMemsetAsync(S->cstamp, 0, 4ull * std::max<uint64_t>(H.own_n(), 1), g->stream));
   if ((st = dev_alloc(g, (void **)&S->d_list, 4ull * std::max<uint64_t>(H.own_n(), 1))) != GR_OK) return st;
   // PageRank carries per shard
   if (S->tile_base[S->P] > g->pr_tiles) {

@@ -65,7 +65,8 @@ def full(rep, out, key=None):
         lines.append("")
         rd = to_bytes(r[h.index("dram__bytes_read.sum")], units[h.index("dram__bytes_read.sum")])
         wr = to_bytes(r[h.index("dram__bytes_write.sum")], units[h.index("dram__bytes_write.sum")])
-        traffic.append(rd + wr)
+        if key and key in name:
+            traffic.append(rd + wr)
     open(out, "w").write("\n".join(lines) + "\n")
     if key and traffic:
         p = os.path.join(os.path.dirname(out), "traffic.json")
