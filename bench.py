@@ -243,10 +243,13 @@ def main():
     clocks.start()
     e0, e1 = torch.cuda.Event(enable_timing=True), torch.cuda.Event(enable_timing=True)
     kms, launches, stats = 0.0, 0, None
+    phase_ms = [0.0, 0.0]
     e0.record(stream)
     for _ in range(args.steps):
         stats = G.run(algo, stream=sp, profile=True, **kw)
         kms += stats["kernel_ms"][0] if algo != "bfs" else stats["kernel_ms"][1]
+        phase_ms[0] += stats["kernel_ms"][0]
+        phase_ms[1] += stats["kernel_ms"][1]
         launches += stats["kernel_launches"]
     e1.record(stream)
     torch.cuda.synchronize()
@@ -330,6 +333,8 @@ def main():
                        "l2": "inputs larger than L2 (CSC payload > 126 MB L2); no flush",
                        "iterations": stats["iterations"]},
             "roofline": roof, "run_roofline": run_roof, "cpu_baseline": cpu, "e2e": e2e,
+            "phase_ms_per_step": {"gather_apply": round(phase_ms[0] / args.steps, 4),
+                                  "activate_or_bfs": round(phase_ms[1] / args.steps, 4)},
             "gpu_launches": launches, "clocks": ck,
         }
         print(json.dumps(line), flush=True)
