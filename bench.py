@@ -311,8 +311,11 @@ def main():
         inf = gr.gr_graph_info_get(H)
         gr.gr_graph_free(H)
         e2e_vals.append(edges / dt / 1e9)
-    h2d = int(8 * m + (m if w is not None else 0))  # CSC + CSR payloads (+weights) per load
-    h2d += 8 * (n + 1) * 2 // (2 if not info["offsets_64bit"] else 1)
+    if inf["built_on_device"]:  # the COO goes up once; the GPU builds CSC/CSR/offsets
+        h2d = int(8 * m + (4 * m if w is not None else 0))
+    else:  # host-built layout: CSC + CSR payloads (+weights) and offsets
+        h2d = int(8 * m + (m if w is not None else 0))
+        h2d += 8 * (n + 1) * 2 // (2 if not info["offsets_64bit"] else 1)
     e2e = {"value": float(np.median(e2e_vals)) if e2e_vals else None, "unit": "GTEPS", "h2d_bytes_per_step": h2d,
            "d2h_bytes_per_step": 4 * n,
            "what": "gr_graph_load(host COO: shard build + H2D) + gr_run + gr_fetch_vertex_values, wall clock"}

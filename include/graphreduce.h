@@ -133,6 +133,8 @@ typedef struct gr_graph_info {
   uint64_t pinned_bytes;     /* pinned host memory held by the graph */
   int32_t offsets_64bit;     /* 1 if edge offsets are stored as uint64 on the device */
   int32_t has_weights;
+  int32_t built_on_device;   /* 1 if the layout was built by the GPU build path (GR_BUILD_DEVICE) */
+  int32_t reserved;
 } gr_graph_info;
 
 /* One destination-interval shard (Fig. 7, §4.2). */

@@ -79,7 +79,8 @@ class gr_graph_info(ctypes.Structure):
                 ("mode", ctypes.c_int32), ("rank", ctypes.c_int32), ("world", ctypes.c_int32),
                 ("sim_ranks", ctypes.c_int32), ("own_lo", ctypes.c_uint64), ("own_hi", ctypes.c_uint64),
                 ("device_bytes", ctypes.c_uint64), ("pinned_bytes", ctypes.c_uint64),
-                ("offsets_64bit", ctypes.c_int32), ("has_weights", ctypes.c_int32)]
+                ("offsets_64bit", ctypes.c_int32), ("has_weights", ctypes.c_int32),
+                ("built_on_device", ctypes.c_int32), ("reserved", ctypes.c_int32)]
 
 
 class gr_shard_desc(ctypes.Structure):

@@ -66,6 +66,7 @@ gr_status gr_graph_load(const gr_edges *edges, const gr_load_opts *opts_in, gr_g
   if (opts.device < 0 || opts.device >= ndev) return fail(GR_EINVAL, "device %d out of range", opts.device);
   if (cudaSetDevice(opts.device) != cudaSuccess) return fail(GR_ECUDA, "cudaSetDevice failed");
 
+  tmark("load: enter");
   gr_graph *g = new gr_graph();
   g->device = opts.device;
   std::string err;
@@ -91,9 +92,7 @@ gr_status gr_graph_load(const gr_edges *edges, const gr_load_opts *opts_in, gr_g
       return fail(s, "%s", err.c_str());
     }
   }
-  cudaDeviceProp prop;
-  cudaGetDeviceProperties(&prop, g->device);
-  g->num_sms = prop.multiProcessorCount;
+  cudaDeviceGetAttribute(&g->num_sms, cudaDevAttrMultiProcessorCount, g->device);
   if (cudaStreamCreateWithFlags(&g->stream, cudaStreamNonBlocking) != cudaSuccess ||
       cudaEventCreate(&g->ev_start) != cudaSuccess || cudaEventCreate(&g->ev_stop) != cudaSuccess ||
       cudaMallocHost((void **)&g->h_ctl, sizeof(Ctl)) != cudaSuccess) {
@@ -105,10 +104,12 @@ gr_status gr_graph_load(const gr_edges *edges, const gr_load_opts *opts_in, gr_g
     cudaEventCreate(&e);
     g->prof_ev.push_back(e);
   }
+  tmark("load: host build / setup");
   if (dev_build) {
     g->mode = GR_MODE_RESIDENT;
     g->dev_built = true;
     s = device_build(g, edges, opts.shard_edges);
+    tmark("load: device build");
     if (s != GR_OK) {
       std::string keep = gr::last_error();
       destroy(g);
@@ -121,6 +122,7 @@ gr_status gr_graph_load(const gr_edges *edges, const gr_load_opts *opts_in, gr_g
   }
   g->sim = sim;
   s = load_device(g);
+  tmark("load: load_device");
   if (s == GR_OK && g->mode == GR_MODE_STREAMED) s = stream_setup(g, budget);
   if (s == GR_OK && opts.world > 1) {
     std::string cerr;
@@ -178,12 +180,20 @@ gr_status gr_graph_info_get(const gr_graph *g, gr_graph_info *o) {
   o->pinned_bytes = g->pinned_bytes;
   o->offsets_64bit = g->off64 ? 1 : 0;
   o->has_weights = g->H.has_w ? 1 : 0;
+  o->built_on_device = g->dev_built ? 1 : 0;
   return GR_OK;
 }
 
 static void shard_desc(const HostGraph &H, uint32_t s, gr_shard_desc *o) {
   o->v_lo = H.bounds[s];
   o->v_hi = H.bounds[s + 1];
+  if (H.in_off.empty()) {  // device-built: offsets kept only at the bounds
+    o->in_begin = H.bound_in[s];
+    o->in_end = H.bound_in[s + 1];
+    o->out_begin = H.bound_out[s];
+    o->out_end = H.bound_out[s + 1];
+    return;
+  }
   o->in_begin = H.in_off[o->v_lo - H.own_lo];
   o->in_end = H.in_off[o->v_hi - H.own_lo];
   o->out_begin = H.out_off[o->v_lo];

@@ -13,6 +13,7 @@
 #include <cuda_runtime.h>
 
 #include <algorithm>
+#include <chrono>
 #include <cstdarg>
 #include <cstdlib>
 #include <cstdio>
@@ -40,6 +41,18 @@ gr_status fail(gr_status s, const char *fmt, ...) {
 }
 
 const char *last_error() { return t_err.c_str(); }
+
+void tmark(const char *what) {
+  static const bool on = [] {
+    const char *e = getenv("GR_TIMING");
+    return e && e[0] == '1';
+  }();
+  if (!on) return;
+  static thread_local std::chrono::steady_clock::time_point last = std::chrono::steady_clock::now();
+  const auto now = std::chrono::steady_clock::now();
+  fprintf(stderr, "[gr timing] %-34s %9.3f ms\n", what, std::chrono::duration<double, std::milli>(now - last).count());
+  last = now;
+}
 void clear_error() { t_err.clear(); }
 
 #define CK(call)                                                                              \
@@ -50,10 +63,29 @@ void clear_error() { t_err.clear(); }
                   cudaGetErrorString(e_), __FILE__, __LINE__);                                \
   } while (0)
 
+void pool_init(int device) {
+  static bool done[64] = {};
+  if (device < 0 || device >= 64 || done[device]) return;
+  cudaMemPool_t pool;
+  if (cudaDeviceGetDefaultMemPool(&pool, device) == cudaSuccess) {
+    uint64_t keep = ~0ull;
+    cudaMemPoolSetAttribute(pool, cudaMemPoolAttrReleaseThreshold, &keep);
+  }
+  cudaGetLastError();
+  done[device] = true;
+}
+
 gr_status dev_alloc(gr_graph *g, void **p, size_t bytes) {
   *p = nullptr;
   if (bytes == 0) bytes = 16;
-  cudaError_t e = cudaMalloc(p, bytes);
+  cudaError_t e = cudaMallocAsync(p, bytes, g->stream);
+  if (e != cudaSuccess) {  // give cached pool memory back to the device and retry once
+    cudaGetLastError();
+    cudaDeviceSynchronize();
+    cudaMemPool_t pool;
+    if (cudaDeviceGetDefaultMemPool(&pool, g->device) == cudaSuccess) cudaMemPoolTrimTo(pool, 0);
+    e = cudaMallocAsync(p, bytes, g->stream);
+  }
   if (e != cudaSuccess) {
     *p = nullptr;
     cudaGetLastError();
@@ -212,7 +244,7 @@ gr_status load_device(gr_graph *g) {
     if ((s = dev_alloc(g, (void **)&g->long_c, 4ull * (g->pr_wtiles + 1))) != GR_OK) return s;
     if ((s = dev_alloc(g, (void **)&g->long_f, 4ull * (g->pr_wtiles + 1))) != GR_OK) return s;
     uint32_t *d_nlong = nullptr;
-    CK(cudaMalloc(&d_nlong, 4));
+    CK(pmalloc(&d_nlong, 4, g->stream));
     CK(cudaMemsetAsync(d_nlong, 0, 4, g->stream));
     if (g->off64) {
       k_pr_tiles<uint64_t><<<(g->pr_wtiles + 256) / 256, 256, 0, g->stream>>>(
@@ -230,7 +262,7 @@ gr_status load_device(gr_graph *g) {
     CK(cudaGetLastError());
     CK(cudaMemcpyAsync(&g->n_long, d_nlong, 4, cudaMemcpyDeviceToHost, g->stream));
     CK(cudaStreamSynchronize(g->stream));
-    cudaFree(d_nlong);
+    pfree(d_nlong, g->stream);
   }
   CK(cudaStreamSynchronize(g->stream));
 
@@ -427,32 +459,17 @@ template <class OffT> static gr_status pr_hot_setup(gr_graph *g) {
     return GR_OK;
   }
   if (g->pr_kernel != 3 && g->pr_kernel != 5) return GR_OK;
-  std::vector<uint32_t> idx(H.n);
-  for (uint64_t v = 0; v < H.n; v++) idx[v] = (uint32_t)v;
   uint64_t K = kHotK;
   if (const char *hk = getenv("GR_PR_HOTK")) K = std::max<uint64_t>(4, std::min<uint64_t>(strtoull(hk, nullptr, 10), 49152));
   K = std::min<uint64_t>(K, H.n);
-  std::partial_sort(idx.begin(), idx.begin() + K, idx.end(), [&](uint32_t a, uint32_t b) {
-    return H.outdeg[a] != H.outdeg[b] ? H.outdeg[a] > H.outdeg[b] : a < b;
-  });
-  std::vector<uint32_t> slot(H.n, 0xFFFFFFFFu), ids;
-  for (uint64_t k = 0; k < K && H.outdeg[idx[k]] > 0; k++) {
-    slot[idx[k]] = (uint32_t)k;
-    ids.push_back(idx[k]);
-  }
-  g->hot_k = (uint32_t)((ids.size() + 3) & ~size_t(3));
-  ids.resize(g->hot_k, ids.empty() ? 0u : ids[0]);
   uint32_t *d_slot = nullptr;
   gr_status s;
-  if ((s = upload(g, &g->hot_ids, ids.data(), ids.size())) != GR_OK) return s;
+  if ((s = select_hot(g, K, &g->hot_ids, &g->hot_k, &d_slot)) != GR_OK) return s;
   if ((s = dev_alloc(g, (void **)&g->hot_contrib, 4ull * std::max<uint32_t>(g->hot_k, 4))) != GR_OK) return s;
   if ((s = dev_alloc(g, (void **)&g->pr_src, 4 * (H.m_in + 4))) != GR_OK) return s;
-  CK(cudaMalloc(&d_slot, 4 * H.n));
-  CK(cudaMemcpyAsync(d_slot, slot.data(), 4 * H.n, cudaMemcpyHostToDevice, g->stream));
   k_pr_tag<<<g->num_sms * 8, 256, 0, g->stream>>>(g->in_src, H.m_in, d_slot, g->pr_src);
   CK(cudaGetLastError());
   CK(cudaStreamSynchronize(g->stream));
-  cudaFree(d_slot);
   int bps = 0;
   if (g->pr_kernel == 5) {
     g->hot_smem = 4ull * g->hot_k + 32 * sizeof(PrWarpSmem);
@@ -522,8 +539,10 @@ static gr_status run_pagerank(gr_graph *g, const gr_run_opts *o, cudaStream_t s,
   const float d = o->damping;
   const int prof = o->profile ? 1 : 0;
   if (g->pr_hot < 0) {
+    tmark("pagerank: before hot setup");
     gr_status hs = pr_hot_setup<OffT>(g);
     if (hs != GR_OK) return hs;
+    tmark("pagerank: hot setup");
   }
   if (prof && g->prof_ev.size() < 2 * (size_t)iters + 2) {
     while (g->prof_ev.size() < 2 * (size_t)iters + 2) {
@@ -564,8 +583,10 @@ static gr_status run_pagerank(gr_graph *g, const gr_run_opts *o, cudaStream_t s,
       g->pr_exec_iters = iters;
       g->pr_exec_d = d;
     }
+    tmark("pagerank: graph ready");
     CK(cudaGraphLaunch(g->pr_exec, s));
     CK(cudaStreamSynchronize(s));
+    tmark("pagerank: 30 supersteps");
   }
   st->iterations = iters;
   st->edges_gathered = (uint64_t)iters * g->H.m_in;
@@ -690,7 +711,8 @@ void destroy(gr_graph *g) {
   stream_destroy(g);
   delete g->comm;
   g->comm = nullptr;
-  for (void *p : g->allocs) cudaFree(p);
+  for (void *p : g->allocs) cudaFreeAsync(p, g->stream);
+  cudaStreamSynchronize(g->stream);
   if (g->h_ctl) cudaFreeHost(g->h_ctl);
   if (g->stream) cudaStreamDestroy(g->stream);
   delete g;

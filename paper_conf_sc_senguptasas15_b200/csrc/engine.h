@@ -120,11 +120,24 @@ template <class OffT> inline Part<OffT> make_part(gr_graph *g) {
 }
 
 gr_status fail(gr_status s, const char *fmt, ...);
+// GR_TIMING=1: host wall-clock marks of the load/run phases on stderr
+void tmark(const char *what);
 const char *last_error();
 void clear_error();
 gr_status dev_alloc(gr_graph *g, void **p, size_t bytes);
+// Stream-ordered allocations from the device's default memory pool. The pool
+// keeps freed memory (release threshold = max), so a reload or a temporary
+// buffer costs no cudaMalloc/cudaFree (each of which synchronises the device).
+void pool_init(int device);
+template <class T> inline cudaError_t pmalloc(T **p, size_t bytes, cudaStream_t s) {
+  return cudaMallocAsync((void **)p, bytes ? bytes : 16, s);
+}
+inline void pfree(void *p, cudaStream_t s) {
+  if (p) cudaFreeAsync(p, s);
+}
 gr_status load_device(gr_graph *g);
 gr_status device_build(gr_graph *g, const gr_edges *E, uint64_t shard_edges);
+gr_status select_hot(gr_graph *g, uint64_t K, uint32_t **hot_ids, uint32_t *hot_k, uint32_t **d_slot);
 gr_status run(gr_graph *g, const gr_run_opts *o, gr_run_stats *st);
 gr_status fetch_values(gr_graph *g, void *dst, uint64_t bytes);
 gr_status fetch_trace(gr_graph *g, uint64_t *dst, uint64_t max_rows, uint64_t *rows);

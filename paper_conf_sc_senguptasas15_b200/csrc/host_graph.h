@@ -49,6 +49,9 @@ struct HostGraph {
   std::vector<uint32_t> outdeg;  // global out-degree of every vertex (PageRank n_j, L74)
   // Shards: intervals [bounds[s], bounds[s+1]) of the owned range
   std::vector<uint64_t> bounds;  // P + 1
+  // Device-built graphs keep no host in_off/out_off: the offsets at the shard
+  // bounds (in_off[bounds[s]-own_lo], out_off[bounds[s]]) are stored instead.
+  std::vector<uint64_t> bound_in, bound_out;
   uint32_t num_shards() const { return bounds.empty() ? 0 : (uint32_t)(bounds.size() - 1); }
   uint64_t own_n() const { return own_hi - own_lo; }
 };
