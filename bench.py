@@ -179,6 +179,8 @@ def main():
     ap.add_argument("--no-cpu", action="store_true")
     ap.add_argument("--loop", default="auto", choices=["auto", "host", "device", "persistent"],
                     help="superstep loop for frontier programs (host: profilable by ncu)")
+    ap.add_argument("--direction", default="auto", choices=["auto", "push", "pull"],
+                    help="FrontierActivate direction for frontier programs (auto: pull when |C_t| > |V|/16)")
     args = ap.parse_args()
 
     rank = int(os.environ.get("RANK", "0"))
@@ -219,7 +221,7 @@ def main():
     print(f"[bench] generated {g.name}: n={g.n} m={g.m} in {time.perf_counter() - t0:.1f}s", file=sys.stderr)
     algo = run["algo"]
     kw = dict(source=run.get("source", 0), max_iters=run.get("max_iters", 0), damping=run.get("damping", 0.85),
-              loop=args.loop)
+              loop=args.loop, direction=args.direction)
     part = {}
     if world > 1:
         # NCCL bootstrap: rank 0 creates the unique id, the torch process group broadcasts it
@@ -311,7 +313,7 @@ def main():
         inf = gr.gr_graph_info_get(H)
         gr.gr_graph_free(H)
         e2e_vals.append(edges / dt / 1e9)
-    if inf["built_on_device"]:  # the COO goes up once; the GPU builds CSC/CSR/offsets
+    if info["built_on_device"]:  # the COO goes up once; the GPU builds CSC/CSR/offsets
         h2d = int(8 * m + (4 * m if w is not None else 0))
     else:  # host-built layout: CSC + CSR payloads (+weights) and offsets
         h2d = int(8 * m + (m if w is not None else 0))
@@ -334,7 +336,9 @@ def main():
             "config": {"workload": CONFIG_NAMES[args.config], "n": n, "m": m, "shards": info["num_shards"],
                        "mode": mode, "parallelism": f"dst-interval partitions x{world}" if world > 1 else "1 GPU",
                        "l2": "inputs larger than L2 (CSC payload > 126 MB L2); no flush",
-                       "iterations": stats["iterations"]},
+                       "iterations": stats["iterations"],
+                       **({} if algo == "pagerank" else {"direction": args.direction,
+                                                          "pull_supersteps": stats["pull_supersteps"]})},
             "roofline": roof, "run_roofline": run_roof, "cpu_baseline": cpu, "e2e": e2e,
             "phase_ms_per_step": {"gather_apply": round(phase_ms[0] / args.steps, 4),
                                   "activate_or_bfs": round(phase_ms[1] / args.steps, 4)},

@@ -109,7 +109,17 @@ typedef struct gr_run_opts {
   int32_t loop;       /* gr_loop */
   void *stream;       /* cudaStream_t to order the run on (device work only); NULL = library stream */
   int32_t profile;    /* 1: time the per-phase kernels with CUDA events (stats.kernel_ms) */
+  int32_t direction;  /* gr_direction: how FrontierActivate reaches the out-neighbours of C_t */
+  uint32_t pull_div;  /* GR_DIR_AUTO: pull when |C_t| * pull_div > |V|; 0 = library default (16) */
 } gr_run_opts;
+
+/* FrontierActivate direction (resident single-rank frontier programs; the
+ * activated set and the trace are identical either way — only the cost differs). */
+typedef enum gr_direction {
+  GR_DIR_AUTO = 0,  /* pull when the changed set is large (|C_t| * pull_div > |V|), else push */
+  GR_DIR_PUSH = 1,  /* always expand the out-edges of C_t (stamps + atomics) */
+  GR_DIR_PULL = 2   /* always scan the in-edges of every vertex for a changed source */
+} gr_direction;
 
 typedef struct gr_run_stats {
   uint32_t iterations;       /* supersteps executed */
@@ -121,6 +131,8 @@ typedef struct gr_run_stats {
   uint64_t bytes_hbm_model;  /* algorithmic (compulsory) HBM bytes */
   uint64_t kernel_launches;  /* library kernel launches issued by this run */
   double kernel_ms[4];       /* profile: [0] gather(+apply), [1] activate/expand, [2] exchange, [3] other */
+  uint32_t pull_supersteps;  /* supersteps whose FrontierActivate ran by pull */
+  uint32_t reserved;
 } gr_run_stats;
 
 typedef struct gr_graph_info {

@@ -27,6 +27,7 @@ ALGOS = {"bfs": 0, "sssp": 1, "pagerank": 2, "cc": 3, "custom": 4}
 MODES = {"auto": 0, "resident": 1, "streamed": 2}
 LOOPS = {"auto": 0, "host": 1, "device": 2, "persistent": 3}
 BUILDS = {"auto": 0, "host": 1, "device": 2}
+DIRECTIONS = {"auto": 0, "push": 1, "pull": 2}
 INF = 0xFFFFFFFF
 
 EXPORTS = [
@@ -58,7 +59,8 @@ class gr_load_opts(ctypes.Structure):
 class gr_run_opts(ctypes.Structure):
     _fields_ = [("algo", ctypes.c_int32), ("source", ctypes.c_uint32), ("max_iters", ctypes.c_uint32),
                 ("damping", ctypes.c_float), ("custom_id", ctypes.c_int32), ("loop", ctypes.c_int32),
-                ("stream", ctypes.c_void_p), ("profile", ctypes.c_int32)]
+                ("stream", ctypes.c_void_p), ("profile", ctypes.c_int32), ("direction", ctypes.c_int32),
+                ("pull_div", ctypes.c_uint32)]
 
 
 class gr_run_stats(ctypes.Structure):
@@ -66,7 +68,8 @@ class gr_run_stats(ctypes.Structure):
                 ("edges_gathered", ctypes.c_uint64), ("edges_scattered", ctypes.c_uint64),
                 ("bytes_h2d", ctypes.c_uint64), ("bytes_nvlink", ctypes.c_uint64),
                 ("bytes_hbm_model", ctypes.c_uint64), ("kernel_launches", ctypes.c_uint64),
-                ("kernel_ms", ctypes.c_double * 4)]
+                ("kernel_ms", ctypes.c_double * 4), ("pull_supersteps", ctypes.c_uint32),
+                ("reserved", ctypes.c_uint32)]
 
     def as_dict(self):
         d = {k: getattr(self, k) for k, _ in self._fields_ if k != "kernel_ms"}
@@ -191,13 +194,15 @@ def gr_graph_load(n, src=None, dst=None, weights=None, row_offsets=None, col_idx
 
 
 def gr_run(h, algo, source=0, max_iters=0, damping=0.85, custom_id=0, loop="auto", stream=None,
-           profile=False) -> dict:
+           profile=False, direction="auto", pull_div=0) -> dict:
     o = gr_run_opts()
     o.algo = ALGOS[algo] if isinstance(algo, str) else int(algo)
     o.source, o.max_iters, o.damping, o.custom_id = int(source), int(max_iters), float(damping), int(custom_id)
     o.loop = LOOPS[loop] if isinstance(loop, str) else int(loop)
     o.stream = stream
     o.profile = 1 if profile else 0
+    o.direction = DIRECTIONS[direction] if isinstance(direction, str) else int(direction)
+    o.pull_div = int(pull_div)
     st = gr_run_stats()
     _check(lib().gr_run(h, ctypes.byref(o), ctypes.byref(st)))
     return st.as_dict()

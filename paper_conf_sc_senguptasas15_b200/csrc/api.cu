@@ -65,6 +65,7 @@ gr_status gr_graph_load(const gr_edges *edges, const gr_load_opts *opts_in, gr_g
   }
   if (opts.device < 0 || opts.device >= ndev) return fail(GR_EINVAL, "device %d out of range", opts.device);
   if (cudaSetDevice(opts.device) != cudaSuccess) return fail(GR_ECUDA, "cudaSetDevice failed");
+  pool_init(opts.device);
 
   tmark("load: enter");
   gr_graph *g = new gr_graph();

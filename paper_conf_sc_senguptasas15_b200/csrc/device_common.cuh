@@ -50,6 +50,13 @@ struct Ctl {
   unsigned long long prof;               // 1: kernels stamp %globaltimer
   unsigned long long kstart[2], kend[2]; // per-kernel span of the current superstep (ns)
   unsigned long long kns[2];             // accumulated kernel ns: [0] gather+apply, [1] activate / BFS expand
+  // Activation direction: pull (scan every owned vertex's in-edges for a
+  // changed source) when |changed| * pull_div > own_n; 0 = always push.
+  uint32_t pull_div;
+  uint32_t pull_pending;  // split-kernel loops: this superstep's pull kernel has work
+  uint32_t dirty[2];      // changed-bitmap b holds bits of an earlier pull and must be cleared
+  uint32_t tot_pull;      // supersteps that activated by pull
+  uint32_t dense;         // superstep `iter` gathers densely (previous activation was by pull)
 };
 
 constexpr int kSlots = 64;
@@ -72,7 +79,8 @@ __device__ __forceinline__ unsigned long long block_sum_u64(unsigned long long x
 // Avoids thousands of warps queueing on the same L2 line with a dependent chain.
 struct View {
   uint32_t stop, t, epoch_base, implicit0, no_hub_c, source, prof;
-  uint32_t cntA[2], cntK[2], cntC, cntKC;
+  uint32_t cntA[2], cntK[2], cntH[2], cntC, cntCH, cntKC;
+  uint32_t pull_div, pull_pending, dirty[2], dense;
   float damping;
 };
 
@@ -85,6 +93,10 @@ __device__ __forceinline__ void load_view(const Ctl *c, View &v) {
     const uint32_t so = vc->source, cc = vc->cnt_C, kc = vc->cnt_KC;
     const float dm = vc->damping;
     const uint32_t pr = (uint32_t)vc->prof;
+    const uint32_t h0 = vc->cnt_H[0], h1 = vc->cnt_H[1], ch = vc->cnt_CH;
+    const uint32_t pd = vc->pull_div, pp = vc->pull_pending, d0 = vc->dirty[0], d1 = vc->dirty[1], dn = vc->dense;
+    v.cntH[0] = h0; v.cntH[1] = h1; v.cntCH = ch;
+    v.pull_div = pd; v.pull_pending = pp; v.dirty[0] = d0; v.dirty[1] = d1; v.dense = dn;
     v.cntA[0] = a0; v.cntA[1] = a1; v.cntK[0] = k0; v.cntK[1] = k1;
     v.stop = st; v.t = t; v.epoch_base = eb; v.implicit0 = im; v.no_hub_c = nh;
     v.source = so; v.cntC = cc; v.cntKC = kc; v.damping = dm; v.prof = pr;
@@ -128,6 +140,10 @@ template <class OffT> struct Part {
   uint32_t *chkA_h[2], *chkA_c[2]; // A_t hub chunks: (position in listH, chunk index)
   uint32_t *chkC_h, *chkC_c;       // changed-hub chunks: (position in CH list, chunk index)
   uint32_t *hub_acc, *hub_done;    // per A-hub position: chunk-combined gather result, chunks done
+  uint32_t *cbits[2];     // changed-set bitmaps over V for pull activation (by superstep parity)
+  uint32_t *hub_act;      // per static hub: some chunk saw a marked source (dense gathers)
+  const uint32_t *s_hubs, *s_chk_h, *s_chk_c;  // static in-hub list and its chunks (dense gathers)
+  uint32_t n_s_hubs, n_s_chunks;
   Ctl *ctl;
   unsigned long long *trace; // [trace_cap][4]
 };
@@ -166,6 +182,10 @@ __device__ __forceinline__ bool stamp_first(uint32_t *stamp, uint32_t epoch) {
 
 __device__ __forceinline__ bool test_bit(const uint32_t *bits, uint32_t i) {
   return (__ldg(bits + (i >> 5)) >> (i & 31)) & 1u;
+}
+// bit test on a bitmap written earlier in the same kernel (L2, not the nc path)
+__device__ __forceinline__ bool test_bit_cg(const uint32_t *bits, uint32_t i) {
+  return (ld_cg(bits + (i >> 5)) >> (i & 31)) & 1u;
 }
 
 // Warp-inclusive scan of a uint32 (all lanes participate).

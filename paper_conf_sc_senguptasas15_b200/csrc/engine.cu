@@ -194,6 +194,14 @@ gr_status load_device(gr_graph *g) {
   if ((s = dev_alloc(g, (void **)&g->hub_acc, 4ull * g->hub_cap)) != GR_OK) return s;
   if ((s = dev_alloc(g, (void **)&g->hub_done, 4ull * g->hub_cap)) != GR_OK) return s;
   CK(cudaMemsetAsync(g->hub_done, 0, 4ull * g->hub_cap, g->stream));
+  if ((s = dev_alloc(g, (void **)&g->hub_act, 4ull * g->hub_cap)) != GR_OK) return s;
+  CK(cudaMemsetAsync(g->hub_act, 0, 4ull * g->hub_cap, g->stream));
+  // changed-set bitmaps for pull activation (resident single-rank runs)
+  if (g->mode == GR_MODE_RESIDENT && H.owners.size() <= 2) {
+    g->cbits_words = cbits_words_n(n);
+    for (int i = 0; i < 2; i++)
+      if ((s = dev_alloc(g, (void **)&g->cbits[i], 4 * g->cbits_words)) != GR_OK) return s;
+  }
 
   // vertex state (replicated values, owned frontier structures)
   const size_t ow = std::max<uint64_t>(own_n, 1);
@@ -288,6 +296,10 @@ static void launch_body(gr_graph *g, cudaStream_t s, unsigned long long cond, in
     k_bfs_expand<OffT><<<g->grid_frontier, kBlock, 0, s>>>(P, cond, use_graph);
     *launches += 1;
   }
+  if (!Prog::kHasGather && g->cbits[0]) {  // BFS: scan half of a pull superstep (returns at once after a push)
+    k_pull<true, OffT><<<g->grid_frontier, kBlock, 0, s>>>(P, cond, use_graph);
+    *launches += 1;
+  }
 }
 
 template <class Prog, class OffT>
@@ -344,6 +356,14 @@ static gr_status run_frontier(gr_graph *g, const gr_run_opts *o, cudaStream_t s,
   h.damping = o->damping;
   h.prof = o->profile ? 1 : 0;
   h.kstart[0] = h.kstart[1] = ~0ull;
+  // activation direction (gr_direction); pull needs the bitmaps (resident, one rank)
+  if (g->cbits[0] && o->direction != GR_DIR_PUSH) {
+    uint32_t div = o->pull_div ? o->pull_div : kPullDivDefault;
+    if (const char *e = getenv("GR_PULL_DIV")) div = (uint32_t)strtoul(e, nullptr, 10);
+    h.pull_div = o->direction == GR_DIR_PULL ? 0xFFFFFFFFu : div;
+    CK(cudaMemsetAsync(g->cbits[0], 0, 4 * g->cbits_words, s));
+    CK(cudaMemsetAsync(g->cbits[1], 0, 4 * g->cbits_words, s));
+  }
   CK(cudaMemcpyAsync(g->ctl, &h, sizeof h, cudaMemcpyHostToDevice, s));
   k_init_values<Prog, OffT><<<g->num_sms * 4, 256, 0, s>>>(P, o->source);
   k_fill_u32<<<std::min<uint32_t>((g->hub_cap + 255) / 256, 1024), 256, 0, s>>>(g->hub_acc, Prog::identity_host(),
@@ -393,6 +413,7 @@ static gr_status run_frontier(gr_graph *g, const gr_run_opts *o, cudaStream_t s,
     st->kernel_ms[1] += c.kns[1] * 1e-6;
   }
   st->iterations = c.iter;
+  st->pull_supersteps = c.tot_pull;
   st->edges_gathered = c.tot_gathered;
   st->edges_scattered = c.tot_scattered;
   st->kernel_launches += launches;
@@ -608,6 +629,7 @@ gr_status run(gr_graph *g, const gr_run_opts *oin, gr_run_stats *st) {
     return fail(GR_EINVAL, "source %u >= num_vertices %llu", o.source, (unsigned long long)g->H.n);
   if (o.algo == GR_SSSP && !g->H.has_w) return fail(GR_EINVAL, "SSSP needs edge weights");
   if (o.algo < GR_BFS || o.algo > GR_CUSTOM) return fail(GR_EINVAL, "unknown algo %d", o.algo);
+  if (o.direction < GR_DIR_AUTO || o.direction > GR_DIR_PULL) return fail(GR_EINVAL, "unknown direction %d", o.direction);
   if (o.algo == GR_CUSTOM) {
     bool known = false, uses_w = false;
 #define GR_X(id, T) if (o.custom_id == id) { known = true; uses_w = T::kUsesWeights; }

@@ -32,6 +32,9 @@ struct gr_graph {
   uint32_t *chkA_h[2] = {nullptr, nullptr}, *chkA_c[2] = {nullptr, nullptr};
   uint32_t *chkC_h = nullptr, *chkC_c = nullptr;
   uint32_t *hub_acc = nullptr, *hub_done = nullptr;
+  uint32_t *cbits[2] = {nullptr, nullptr};  // changed-set bitmaps (pull activation)
+  uint32_t *hub_act = nullptr;
+  size_t cbits_words = 0;
   uint32_t *static_chk_h = nullptr, *static_chk_c = nullptr;
   uint32_t n_static_chunks = 0, hub_cap = 0;
   bool dev_built = false;        // layout built on the GPU (device_build.cu)
@@ -114,6 +117,10 @@ template <class OffT> inline Part<OffT> make_part(gr_graph *g) {
   for (int i = 0; i < 2; i++) { P.chkA_h[i] = g->chkA_h[i]; P.chkA_c[i] = g->chkA_c[i]; }
   P.chkC_h = g->chkC_h; P.chkC_c = g->chkC_c;
   P.hub_acc = g->hub_acc; P.hub_done = g->hub_done;
+  P.cbits[0] = g->cbits[0]; P.cbits[1] = g->cbits[1];
+  P.hub_act = g->hub_act;
+  P.s_hubs = g->static_hubs; P.s_chk_h = g->static_chk_h; P.s_chk_c = g->static_chk_c;
+  P.n_s_hubs = g->n_static_hubs; P.n_s_chunks = g->n_static_chunks;
   P.ctl = g->ctl;
   P.trace = g->trace;
   return P;

@@ -26,6 +26,10 @@
 namespace gr {
 
 constexpr int kBatch = 4;  // edges in flight per lane per memory phase
+// how superstep t's FrontierActivate ran (close_superstep)
+constexpr int kPush = 0;       // out-edge expansion of C_t with stamps
+constexpr int kPullScan = 1;   // BFS: in-edge scan of every vertex for a C_t source -> A_{t+1} list
+constexpr int kPullDense = 2;  // gather programs: C_t marked only; superstep t+1 gathers densely
 
 // ----------------------------------------------------------------- helpers
 template <class Prog>
@@ -44,13 +48,17 @@ __device__ __forceinline__ typename Prog::GatherT map_edge(const Part<OffT> &P, 
 }
 
 // Gather for up to 32 vertices held one per lane (valid, beg, deg, dval).
-// Returns the gatherReduce result of the lane's own vertex.
-template <class Prog, class OffT>
+// Returns the gatherReduce result of the lane's own vertex. kDense (pull
+// supersteps): also sets `act` iff some in-edge source is marked in `bits`
+// (the changed set of the previous superstep), i.e. the vertex is in A_t.
+template <class Prog, bool kDense, class OffT>
 __device__ typename Prog::GatherT gather_warp(const Part<OffT> &P, bool valid, uint64_t beg, uint32_t deg,
-                                              uint32_t dval, uint32_t *sred, const Ctx &cx) {
+                                              uint32_t dval, uint32_t *sred, const Ctx &cx, const uint32_t *bits,
+                                              bool &act) {
   using G = typename Prog::GatherT;
   const uint32_t lane = lane_id();
   G acc = Prog::identity();
+  act = false;
   // warp-cooperative: one vertex of degree in (32, kHubDegree] at a time
   uint32_t big = __ballot_sync(0xffffffffu, valid && deg > 32);
   while (big) {
@@ -60,15 +68,39 @@ __device__ typename Prog::GatherT gather_warp(const Part<OffT> &P, bool valid, u
     const uint32_t d = __shfl_sync(0xffffffffu, deg, L);
     const uint32_t dv = __shfl_sync(0xffffffffu, dval, L);
     G r = Prog::identity();
+    bool hit = false;
     uint32_t k = lane;
     for (; k + 96 < d; k += 128) {  // 4 independent loads in flight per lane
-      G a0 = map_edge<Prog>(P, b + k, dv, cx), a1 = map_edge<Prog>(P, b + k + 32, dv, cx);
-      G a2 = map_edge<Prog>(P, b + k + 64, dv, cx), a3 = map_edge<Prog>(P, b + k + 96, dv, cx);
-      r = Prog::gatherReduce(r, Prog::gatherReduce(Prog::gatherReduce(a0, a1), Prog::gatherReduce(a2, a3)));
+      uint32_t u[4], w[4];
+#pragma unroll
+      for (int q = 0; q < 4; q++) {
+        u[q] = ldg_nc(P.in_src + b + k + 32 * q);
+        w[q] = Prog::kUsesWeights ? (uint32_t)ldg_nc_u8(P.in_w + b + k + 32 * q) : 0u;
+      }
+      uint32_t v[4], bw[4];
+#pragma unroll
+      for (int q = 0; q < 4; q++) {
+        v[q] = P.val[u[q]];
+        if (kDense) bw[q] = ld_cg(bits + (u[q] >> 5));
+      }
+#pragma unroll
+      for (int q = 0; q < 4; q++) {
+        r = Prog::gatherReduce(r, Prog::gatherMap(dv, v[q], w[q], cx));
+        if (kDense) hit |= (bw[q] >> (u[q] & 31)) & 1u;
+      }
     }
-    for (; k < d; k += 32) r = Prog::gatherReduce(r, map_edge<Prog>(P, b + k, dv, cx));
+    for (; k < d; k += 32) {
+      const uint32_t u = ldg_nc(P.in_src + b + k);
+      const uint32_t w = Prog::kUsesWeights ? (uint32_t)ldg_nc_u8(P.in_w + b + k) : 0u;
+      r = Prog::gatherReduce(r, Prog::gatherMap(dv, P.val[u], w, cx));
+      if (kDense) hit |= test_bit_cg(bits, u);
+    }
     r = warp_reduce_prog<Prog>(r);
-    if ((int)lane == L) acc = r;
+    const bool any = kDense ? (__any_sync(0xffffffffu, hit) != 0) : false;
+    if ((int)lane == L) {
+      acc = r;
+      act = any;
+    }
   }
   // fine-grained: pack the edges of all lanes with degree <= 32, 32 per round;
   // kBatch rounds' loads (sources + weights, then source values) are issued
@@ -79,11 +111,12 @@ __device__ typename Prog::GatherT gather_warp(const Part<OffT> &P, bool valid, u
   const uint32_t total = __shfl_sync(0xffffffffu, incl, 31);
   if (total == 0) return acc;
   sred[lane] = Prog::identity();
+  uint32_t hitmask = 0;  // kDense: owner lanes with a marked source (warp-uniform)
   __syncwarp();
   for (uint32_t rb = 0; rb < total; rb += 32u * kBatch) {
     int own[kBatch];
     uint32_t su[kBatch], sw[kBatch], dv[kBatch];
-    bool act[kBatch];
+    bool act_q[kBatch];
 #pragma unroll
     for (int q = 0; q < kBatch; q++) {
       const uint32_t k = rb + q * 32u + lane;
@@ -97,19 +130,30 @@ __device__ typename Prog::GatherT gather_warp(const Part<OffT> &P, bool valid, u
       const uint64_t ob = __shfl_sync(0xffffffffu, beg, o);
       const uint32_t oe = __shfl_sync(0xffffffffu, excl, o);
       dv[q] = __shfl_sync(0xffffffffu, dval, o);
-      act[q] = k < total;
+      act_q[q] = k < total;
       const uint64_t e = ob + (k - oe);
-      su[q] = act[q] ? ldg_nc(P.in_src + e) : 0u;
-      sw[q] = (act[q] && Prog::kUsesWeights) ? (uint32_t)ldg_nc_u8(P.in_w + e) : 0u;
+      su[q] = act_q[q] ? ldg_nc(P.in_src + e) : 0u;
+      sw[q] = (act_q[q] && Prog::kUsesWeights) ? (uint32_t)ldg_nc_u8(P.in_w + e) : 0u;
     }
-    uint32_t sv[kBatch];
+    uint32_t sv[kBatch], sb[kBatch];
 #pragma unroll
-    for (int q = 0; q < kBatch; q++) sv[q] = act[q] ? P.val[su[q]] : 0u;
+    for (int q = 0; q < kBatch; q++) {
+      sv[q] = act_q[q] ? P.val[su[q]] : 0u;
+      if (kDense) sb[q] = act_q[q] ? ld_cg(bits + (su[q] >> 5)) : 0u;
+    }
 #pragma unroll
     for (int q = 0; q < kBatch; q++) {
       if (rb + q * 32u >= total) break;  // warp-uniform
       const int o = own[q];
-      G x = act[q] ? Prog::gatherMap(dv[q], sv[q], sw[q], cx) : Prog::identity();
+      if (kDense) {
+        const bool h = act_q[q] && ((sb[q] >> (su[q] & 31)) & 1u);
+        // owners of hits: OR of (1 << owner) over the warp
+        uint32_t m = h ? (1u << o) : 0u;
+#pragma unroll
+        for (int dd = 16; dd > 0; dd >>= 1) m |= __shfl_xor_sync(0xffffffffu, m, dd);
+        hitmask |= m;
+      }
+      G x = act_q[q] ? Prog::gatherMap(dv[q], sv[q], sw[q], cx) : Prog::identity();
       // segmented inclusive scan keyed by owner lane (owners are non-decreasing)
       const int prev_o = __shfl_up_sync(0xffffffffu, o, 1);
       uint32_t f = (lane == 0 || prev_o != o) ? 1u : 0u;
@@ -127,24 +171,53 @@ __device__ typename Prog::GatherT gather_warp(const Part<OffT> &P, bool valid, u
       __syncwarp();
     }
   }
-  if (sd > 0) acc = sred[lane];
+  if (sd > 0) {
+    acc = sred[lane];
+    if (kDense) act = (hitmask >> lane) & 1u;
+  }
   __syncwarp();
   return acc;
 }
 
-// Block-wide gather of one hub vertex.
-template <class Prog, class OffT>
+// Block-wide gather of one hub vertex (chunk). kDense: *act (thread 0) = some
+// source in the chunk is marked in `bits`.
+template <class Prog, bool kDense, class OffT>
 __device__ typename Prog::GatherT gather_block(const Part<OffT> &P, uint64_t beg, uint32_t deg, uint32_t dval,
-                                               typename Prog::GatherT *sblk, const Ctx &cx) {
+                                               typename Prog::GatherT *sblk, const Ctx &cx, const uint32_t *bits,
+                                               bool *act) {
   using G = typename Prog::GatherT;
   G r = Prog::identity();
+  bool hit = false;
   uint32_t k = threadIdx.x;
   for (; k + 3 * kBlock < deg; k += 4 * kBlock) {
-    G a0 = map_edge<Prog>(P, beg + k, dval, cx), a1 = map_edge<Prog>(P, beg + k + kBlock, dval, cx);
-    G a2 = map_edge<Prog>(P, beg + k + 2 * kBlock, dval, cx), a3 = map_edge<Prog>(P, beg + k + 3 * kBlock, dval, cx);
-    r = Prog::gatherReduce(r, Prog::gatherReduce(Prog::gatherReduce(a0, a1), Prog::gatherReduce(a2, a3)));
+    uint32_t u[4], w[4];
+#pragma unroll
+    for (int q = 0; q < 4; q++) {
+      u[q] = ldg_nc(P.in_src + beg + k + q * kBlock);
+      w[q] = Prog::kUsesWeights ? (uint32_t)ldg_nc_u8(P.in_w + beg + k + q * kBlock) : 0u;
+    }
+    uint32_t v[4], bw[4];
+#pragma unroll
+    for (int q = 0; q < 4; q++) {
+      v[q] = P.val[u[q]];
+      if (kDense) bw[q] = ld_cg(bits + (u[q] >> 5));
+    }
+#pragma unroll
+    for (int q = 0; q < 4; q++) {
+      r = Prog::gatherReduce(r, Prog::gatherMap(dval, v[q], w[q], cx));
+      if (kDense) hit |= (bw[q] >> (u[q] & 31)) & 1u;
+    }
   }
-  for (; k < deg; k += kBlock) r = Prog::gatherReduce(r, map_edge<Prog>(P, beg + k, dval, cx));
+  for (; k < deg; k += kBlock) {
+    const uint32_t u = ldg_nc(P.in_src + beg + k);
+    const uint32_t w = Prog::kUsesWeights ? (uint32_t)ldg_nc_u8(P.in_w + beg + k) : 0u;
+    r = Prog::gatherReduce(r, Prog::gatherMap(dval, P.val[u], w, cx));
+    if (kDense) hit |= test_bit_cg(bits, u);
+  }
+  if (kDense) {
+    const int any = __syncthreads_or(hit ? 1 : 0);
+    if (threadIdx.x == 0) *act = any != 0;
+  }
   r = warp_reduce_prog<Prog>(r);
   if (lane_id() == 0) sblk[threadIdx.x / 32] = r;
   __syncthreads();
@@ -290,7 +363,7 @@ __device__ uint32_t expand_block(const Part<OffT> &P, uint64_t beg, uint32_t deg
 // counters, write the trace row, reset the per-superstep counters, advance t,
 // decide termination and set the CUDA-graph loop condition.
 template <class OffT>
-__device__ void close_superstep(const Part<OffT> &P, unsigned long long cond_handle, int use_graph) {
+__device__ void close_superstep(const Part<OffT> &P, unsigned long long cond_handle, int use_graph, int pulled) {
   __shared__ unsigned long long s_red[4][kWarpsPerBlock];
   __threadfence();
   volatile Ctl *c = P.ctl;
@@ -331,6 +404,7 @@ __device__ void close_superstep(const Part<OffT> &P, unsigned long long cond_han
       c->kend[k] = 0;
     }
   }
+  const unsigned long long scat = c->scattered;
   c->tot_gathered = c->tot_gathered + c->gathered;
   c->tot_scattered = c->tot_scattered + c->scattered;
   c->changed = 0;
@@ -345,8 +419,20 @@ __device__ void close_superstep(const Part<OffT> &P, unsigned long long cond_han
   c->cnt_A[slot] = 0;
   c->cnt_H[slot] = 0;
   c->cnt_act[slot] = 0;
+  // changed bitmaps: this superstep's activation cleared bitmap (t+1)&1; a
+  // pull left bits in bitmap t&1
+  c->dirty[ns] = 0;
+  if (pulled) {
+    c->dirty[slot] = 1;
+    c->tot_pull = c->tot_pull + 1;
+  }
+  c->pull_pending = 0;
+  // kPullDense: A_{t+1} is found by the dense gather of t+1; it is empty iff
+  // C_t has no out-edges
+  c->dense = (pulled == kPullDense) ? 1u : 0u;
   c->iter = t + 1;
-  const bool stop = !c->ext_loop && ((c->cnt_act[ns] == 0) || (c->max_iters != 0 && t + 1 >= c->max_iters));
+  const bool empty = (pulled == kPullDense) ? (scat == 0) : (c->cnt_act[ns] == 0);
+  const bool stop = !c->ext_loop && (empty || (c->max_iters != 0 && t + 1 >= c->max_iters));
   c->stop = stop ? 1u : 0u;
   __threadfence();
   if (use_graph) cudaGraphSetConditional((cudaGraphConditionalHandle)cond_handle, stop ? 0u : 1u);
@@ -356,7 +442,7 @@ __device__ void close_superstep(const Part<OffT> &P, unsigned long long cond_han
 // Last CTA of the superstep's final kernel closes superstep t. The ticket is
 // two-level (groups of 32 CTAs) so no single address takes one atomic per CTA.
 template <class OffT>
-__device__ void finish_superstep(const Part<OffT> &P, unsigned long long cond_handle, int use_graph) {
+__device__ void finish_superstep(const Part<OffT> &P, unsigned long long cond_handle, int use_graph, int pulled) {
   __shared__ bool s_last;
   __syncthreads();
   if (threadIdx.x == 0) {
@@ -377,23 +463,172 @@ __device__ void finish_superstep(const Part<OffT> &P, unsigned long long cond_ha
   }
   __syncthreads();
   if (!s_last) return;
-  close_superstep(P, cond_handle, use_graph);
+  close_superstep(P, cond_handle, use_graph, pulled);
+}
+
+// ------------------------------------------------- pull activation (dense)
+// When the changed set is a large fraction of V, FrontierActivate by pull:
+// commit C_t and mark it in a bitmap, then every owned vertex x scans its
+// in-edges for a changed source (early exit) — x is in A_{t+1} iff one exists,
+// the same set the push expansion produces (the out-neighbours of C_t), with
+// no per-edge atomics. Trace columns are unchanged.
+// words of one changed bitmap (a multiple of 4 for 16-byte clears; the host allocates the same)
+__host__ __device__ __forceinline__ size_t cbits_words_n(uint64_t n) { return (((n + 31) / 32 + 1) + 3) & ~size_t(3); }
+template <class OffT> __device__ __forceinline__ size_t cbits_words(const Part<OffT> &P) { return cbits_words_n(P.n); }
+
+__device__ __forceinline__ bool pull_mode(const View &V, uint32_t own_n, uint32_t frontier) {
+  return V.pull_div != 0 && (unsigned long long)frontier * V.pull_div > own_n;
+}
+__device__ __forceinline__ uint32_t frontier_gather(const View &V) { return V.cntC + V.cntCH; }
+__device__ __forceinline__ uint32_t frontier_bfs(const View &V) { return V.cntA[V.t & 1u] + V.cntH[V.t & 1u]; }
+
+// Zero the bitmap the next superstep may pull into (all CTAs; nobody reads it now).
+template <class OffT>
+__device__ __forceinline__ void clear_dirty(const Part<OffT> &P, const View &V, size_t words) {
+  const uint32_t nb = (V.t + 1) & 1u;
+  if (!V.dirty[nb]) return;
+  uint4 *w = reinterpret_cast<uint4 *>(P.cbits[nb]);
+  for (size_t i = blockIdx.x * (size_t)blockDim.x + threadIdx.x; i < words / 4; i += (size_t)gridDim.x * blockDim.x)
+    w[i] = make_uint4(0, 0, 0, 0);
+}
+
+__device__ __forceinline__ void set_bit(uint32_t *bits, uint32_t u) { atomicOr(bits + (u >> 5), 1u << (u & 31)); }
+
+// Pull mode, gather programs: commit C_t (non-hub and hub entries) and mark it.
+template <class OffT>
+__device__ __forceinline__ void commit_phase(const Part<OffT> &P, const View &V) {
+  uint32_t *bits = P.cbits[V.t & 1u];
+  __shared__ unsigned long long s8[kWarpsPerBlock];
+  unsigned long long my_s = 0;
+  const uint32_t nC = V.cntC, nCH = V.cntCH;
+  for (uint32_t i = blockIdx.x * blockDim.x + threadIdx.x; i < nC + nCH; i += gridDim.x * blockDim.x) {
+    const bool h = i >= nC;
+    const uint32_t u = h ? P.CH_v[i - nC] : P.C_v[i];
+    P.val[u] = h ? P.CH_val[i - nC] : P.C_val[i];  // BSP commit of superstep t
+    set_bit(bits, u);
+    my_s += (uint64_t)P.out_off[u + 1] - (uint64_t)P.out_off[u];
+  }
+  my_s = block_sum_u64(my_s, s8);
+  if (threadIdx.x == 0 && my_s) atomicAdd(&P.ctl->part_s[blockIdx.x % kSlots], my_s);
+}
+
+// Pull mode, BFS: apply A_t (depth = t, L276; hubs included) and mark C_t.
+template <class OffT>
+__device__ __forceinline__ void bfs_apply_phase(const Part<OffT> &P, const View &V) {
+  const uint32_t t = V.t, slot = t & 1u;
+  uint32_t *bits = P.cbits[slot];
+  __shared__ unsigned long long s8[kWarpsPerBlock];
+  unsigned long long my_s = 0, my_c = 0;
+  const uint32_t nA = V.cntA[slot], nH = V.cntH[slot];
+  for (uint32_t i = blockIdx.x * blockDim.x + threadIdx.x; i < nA + nH; i += gridDim.x * blockDim.x) {
+    const uint32_t v = i < nA ? P.listA[slot][i] : P.listH[slot][i - nA];
+    if (P.val[v] == kInf) {
+      P.val[v] = t;
+      set_bit(bits, v);
+      my_c += 1;
+      my_s += (uint64_t)P.out_off[v + 1] - (uint64_t)P.out_off[v];
+    }
+  }
+  my_s = block_sum_u64(my_s, s8);
+  if (threadIdx.x == 0 && my_s) atomicAdd(&P.ctl->part_s[blockIdx.x % kSlots], my_s);
+  my_c = block_sum_u64(my_c, s8);
+  if (threadIdx.x == 0 && my_c) atomicAdd(&P.ctl->part_c[blockIdx.x % kSlots], my_c);
+}
+
+// Pull mode: A_{t+1} = owned x with an in-neighbour in C_t. Each lane probes
+// the first kProbe in-edges of its vertex; the vertices still undecided are
+// then scanned by the whole warp, 32 edges per step, stopping at the first hit.
+// BFS keeps only unvisited vertices in the list (counts every activated one).
+constexpr uint32_t kProbe = 4;
+constexpr uint32_t kPullDivDefault = 16;  // GR_DIR_AUTO: pull when |C_t| > |V| / 16
+template <bool kBfs, class OffT>
+__device__ __forceinline__ void pull_phase(const Part<OffT> &P, const View &V) {
+  Ctl *ctl = P.ctl;
+  const uint32_t t = V.t, ns = (t + 1) & 1u;
+  const uint32_t *bits = P.cbits[t & 1u];
+  prof_begin(ctl, V, 1);
+  __shared__ uint32_t sq[kWarpsPerBlock][kQueueCap];
+  __shared__ uint32_t s_off[kWarpsPerBlock + 1];
+  __shared__ unsigned long long s8[kWarpsPerBlock];
+  const uint32_t warp = threadIdx.x / 32, lane = lane_id();
+  WarpQueue qA{sq[warp], nullptr, 0};
+  unsigned long long my_act = 0;
+  const uint32_t gw = blockIdx.x * kWarpsPerBlock + warp, nw = gridDim.x * kWarpsPerBlock;
+  for (uint32_t base = gw * 32u; base < P.own_n; base += nw * 32u) {
+    const uint32_t lx = base + lane;
+    const bool valid = lx < P.own_n;
+    const uint32_t x = P.own_lo + lx;
+    uint64_t beg = 0, end = 0;
+    if (valid) {
+      beg = (uint64_t)P.in_off[lx];
+      end = (uint64_t)P.in_off[lx + 1];
+    }
+    const uint64_t deg = end - beg;
+    uint32_t src[kProbe];
+#pragma unroll
+    for (uint32_t q = 0; q < kProbe; q++) src[q] = (q < deg) ? ldg_nc(P.in_src + beg + q) : 0u;
+    bool found = false;
+#pragma unroll
+    for (uint32_t q = 0; q < kProbe; q++) found |= (q < deg) && test_bit_cg(bits, src[q]);
+    uint32_t pend = __ballot_sync(0xffffffffu, !found && deg > kProbe);
+    uint32_t fm = 0;
+    while (pend) {
+      const int l = __ffs(pend) - 1;
+      pend &= pend - 1;
+      const uint64_t b = __shfl_sync(0xffffffffu, beg, l) + kProbe, e = __shfl_sync(0xffffffffu, end, l);
+      for (uint64_t k = b; k < e; k += 32) {
+        const uint64_t kk = k + lane;
+        const bool hit = kk < e && test_bit_cg(bits, ldg_nc(P.in_src + kk));
+        if (__ballot_sync(0xffffffffu, hit)) {
+          fm |= 1u << l;
+          break;
+        }
+      }
+    }
+    found = found || ((fm >> lane) & 1u);
+    my_act += __popc(__ballot_sync(0xffffffffu, found));
+    const bool keep = found && (!kBfs || *(volatile uint32_t *)(P.val + x) == kInf);
+    const bool hub = keep && test_bit(kBfs ? P.hub_out : P.hub_in, kBfs ? x : lx);
+    if (hub) append_hub_A<kBfs>(P, x, ns);
+    qA.push(keep && !hub, x, 0, P.listA[ns], nullptr, &ctl->cnt_A[ns]);
+  }
+  qA.block_flush(P.listA[ns], nullptr, &ctl->cnt_A[ns], s_off);
+  my_act = block_sum_u64(lane == 0 ? my_act : 0ull, s8);
+  if (threadIdx.x == 0 && my_act) atomicAdd(&ctl->part_a[blockIdx.x % kSlots], my_act);
+  prof_end(ctl, V, 1);
+}
+
+// Split-kernel loops: the pull half of a pull superstep (no-op otherwise).
+template <bool kBfs, class OffT>
+__global__ void __launch_bounds__(kBlock) k_pull(const __grid_constant__ Part<OffT> P, unsigned long long cond,
+                                                 int use_graph) {
+  __shared__ View V;
+  load_view(P.ctl, V);
+  if (V.stop || !V.pull_pending) return;
+  pull_phase<kBfs>(P, V);
+  finish_superstep(P, cond, use_graph, kPullScan);
 }
 
 // ------------------------------------------------------------- kernels
-// Gather + apply over A_t (one phase of superstep t).
-template <class Prog, class OffT>
+// Gather + apply over A_t (one phase of superstep t). kDense (the previous
+// superstep activated by pull): A_t is not materialised — every owned vertex
+// is gathered and is active iff one of its in-edge sources is marked in the
+// changed bitmap of t-1; only active vertices apply and count in the trace.
+template <class Prog, bool kDense, class OffT>
 __device__ __forceinline__ void gather_phase(const Part<OffT> &P, const View &V) {
   using G = typename Prog::GatherT;
   Ctl *ctl = P.ctl;
   const uint32_t t = V.t;
   const uint32_t slot = t & 1u;
   const Ctx cx{t, P.n, V.source, V.damping};
-  const bool implicit = V.implicit0 && t == 0;
+  const bool implicit = kDense || (V.implicit0 && t == 0);
   const uint32_t nA = implicit ? P.own_n : V.cntA[slot];
-  const uint32_t nK = V.cntK[slot];
+  const uint32_t nK = kDense ? P.n_s_chunks : V.cntK[slot];
   const uint32_t *LA = P.listA[slot];
-  const uint32_t *LH = P.listH[slot];
+  const uint32_t *LH = kDense ? P.s_hubs : P.listH[slot];
+  const uint32_t *KH = kDense ? P.s_chk_h : P.chkA_h[slot];
+  const uint32_t *KC = kDense ? P.s_chk_c : P.chkA_c[slot];
+  const uint32_t *bits = P.cbits[slot ^ 1u];  // C_{t-1} (dense only)
   const bool no_hub_c = V.no_hub_c != 0;
   prof_begin(ctl, V, 0);
 
@@ -401,11 +636,12 @@ __device__ __forceinline__ void gather_phase(const Part<OffT> &P, const View &V)
   __shared__ uint32_t sred[kWarpsPerBlock][32];
   __shared__ G sblk[kWarpsPerBlock];
   __shared__ uint32_t s_h;
+  __shared__ bool s_act;
   __shared__ uint32_t s_off[kWarpsPerBlock + 1];
   __shared__ unsigned long long s8[kWarpsPerBlock];
   const uint32_t warp = threadIdx.x / 32, lane = lane_id();
   WarpQueue qC{sq[warp][0], sq[warp][1], 0};
-  unsigned long long my_g = 0, my_c = 0;
+  unsigned long long my_g = 0, my_c = 0, my_a = 0;
 
   // Phase 1: non-hub active vertices, 32 per warp, static grid stride
   const uint32_t gw = blockIdx.x * kWarpsPerBlock + warp, nw = gridDim.x * kWarpsPerBlock;
@@ -427,12 +663,16 @@ __device__ __forceinline__ void gather_phase(const Part<OffT> &P, const View &V)
       cur = P.val[v];
       hubv = !no_hub_c && test_bit(P.hub_out, v);  // issued with the offsets, used after apply
     }
-    const G acc = Prog::kHasGather ? gather_warp<Prog>(P, valid, beg, deg, cur, sred[warp], cx) : Prog::identity();
+    bool hit = false;
+    const G acc = Prog::kHasGather ? gather_warp<Prog, kDense>(P, valid, beg, deg, cur, sred[warp], cx, bits, hit)
+                                   : Prog::identity();
+    const bool active = valid && (!kDense || hit);
     bool changed = false;
     uint32_t nv = cur;
-    if (valid) {
+    if (active) {
       changed = Prog::apply(&nv, acc, cx);
       my_g += deg;
+      my_a += 1;
     }
     const bool hubo = changed && hubv;
     if (hubo) append_hub_C(P, v, nv);
@@ -449,7 +689,7 @@ __device__ __forceinline__ void gather_phase(const Part<OffT> &P, const View &V)
     __syncthreads();
     const uint32_t i = s_h;
     if (i >= nK) break;
-    const uint32_t hp = P.chkA_h[slot][i], ci = P.chkA_c[slot][i];
+    const uint32_t hp = KH[i], ci = KC[i];
     const uint32_t v = LH[hp], lv = v - P.own_lo;
     const uint64_t beg = (uint64_t)P.in_off[lv];
     const uint64_t deg = (uint64_t)P.in_off[lv + 1] - beg;
@@ -457,23 +697,28 @@ __device__ __forceinline__ void gather_phase(const Part<OffT> &P, const View &V)
     const uint32_t len = chunk_len(deg, ci);
     const uint32_t cur = P.val[v];
     if (!Prog::kHasGather && ci != 0) continue;  // no gather: chunk 0 applies
-    const G r = Prog::kHasGather ? gather_block<Prog>(P, b, len, cur, sblk, cx) : Prog::identity();
+    const G r = Prog::kHasGather ? gather_block<Prog, kDense>(P, b, len, cur, sblk, cx, bits, &s_act)
+                                 : Prog::identity();
     if (threadIdx.x == 0) {
       const uint32_t nch = Prog::kHasGather ? (uint32_t)((deg + kChunk - 1) / kChunk) : 1u;
-      if (ci == 0 && Prog::kHasGather) my_g += deg;
       bool fin = (nch == 1);
+      bool hact = kDense ? s_act : true;
       G acc = r;
       if (!fin) {
         Prog::atomicGather(P.hub_acc + hp, r);
+        if (kDense && s_act) atomicOr(P.hub_act + hp, 1u);
         __threadfence();
         fin = (atomicAdd(P.hub_done + hp, 1u) == nch - 1);
         if (fin) {
           __threadfence();
           acc = atomicExch(P.hub_acc + hp, Prog::identity());
+          if (kDense) hact = atomicExch(P.hub_act + hp, 0u) != 0;
           P.hub_done[hp] = 0;
         }
       }
-      if (fin) {
+      if (fin && hact) {
+        if (Prog::kHasGather) my_g += deg;
+        my_a += 1;
         uint32_t nv = cur;
         if (Prog::apply(&nv, acc, cx)) {
           my_c += 1;
@@ -491,6 +736,10 @@ __device__ __forceinline__ void gather_phase(const Part<OffT> &P, const View &V)
   if (threadIdx.x == 0 && my_g) atomicAdd(&ctl->part_g[blockIdx.x % kSlots], my_g);
   my_c = block_sum_u64(my_c, s8);
   if (threadIdx.x == 0 && my_c) atomicAdd(&ctl->part_c[blockIdx.x % kSlots], my_c);
+  if (kDense) {  // |A_t| is only known now (one atomic per CTA)
+    my_a = block_sum_u64(my_a, s8);
+    if (threadIdx.x == 0 && my_a) atomicAdd(&ctl->cnt_act[slot], (uint32_t)my_a);
+  }
   prof_end(ctl, V, 0);
 }
 
@@ -499,7 +748,8 @@ __global__ void __launch_bounds__(kBlock) k_gather_apply(const __grid_constant__
   __shared__ View V;
   load_view(P.ctl, V);
   if (V.stop) return;
-  gather_phase<Prog>(P, V);
+  if (V.dense) gather_phase<Prog, true>(P, V);
+  else gather_phase<Prog, false>(P, V);
 }
 
 // Commit C_t and FrontierActivate (the other phase of superstep t).
@@ -573,8 +823,14 @@ __global__ void __launch_bounds__(kBlock) k_activate(const __grid_constant__ Par
       cudaGraphSetConditional((cudaGraphConditionalHandle)cond, 0u);
     return;
   }
+  clear_dirty(P, V, cbits_words(P));
+  if (pull_mode(V, P.own_n, frontier_gather(V))) {
+    commit_phase(P, V);  // superstep t+1 gathers densely
+    finish_superstep(P, cond, use_graph, kPullDense);
+    return;
+  }
   activate_phase(P, V);
-  finish_superstep(P, cond, use_graph);
+  finish_superstep(P, cond, use_graph, kPush);
 }
 
 // BFS: apply (depth = t, L276) fused with FrontierActivate; no gather (L274).
@@ -665,8 +921,14 @@ __global__ void __launch_bounds__(kBlock) k_bfs_expand(const __grid_constant__ P
       cudaGraphSetConditional((cudaGraphConditionalHandle)cond, 0u);
     return;
   }
+  clear_dirty(P, V, cbits_words(P));
+  if (pull_mode(V, P.own_n, frontier_bfs(V))) {
+    bfs_apply_phase(P, V);
+    if (blockIdx.x == 0 && threadIdx.x == 0) P.ctl->pull_pending = 1;
+    return;
+  }
   bfs_phase(P, V);
-  finish_superstep(P, cond, use_graph);
+  finish_superstep(P, cond, use_graph, kPush);
 }
 
 // Software grid barrier for the persistent loop (cooperative launch guarantees
@@ -700,16 +962,29 @@ __global__ void __launch_bounds__(kBlock) k_persistent(const __grid_constant__ P
   for (;;) {
     load_view(ctl, V);
     if (V.stop) break;
+    int pull;
     if (Prog::kHasGather) {
-      gather_phase<Prog>(P, V);
+      if (V.dense) gather_phase<Prog, true>(P, V);
+      else gather_phase<Prog, false>(P, V);
       grid_sync(ctl);
       load_view(ctl, V);
-      activate_phase(P, V);
+      clear_dirty(P, V, cbits_words(P));
+      pull = pull_mode(V, P.own_n, frontier_gather(V)) ? kPullDense : kPush;
+      if (pull) commit_phase(P, V);  // superstep t+1 gathers densely
+      else activate_phase(P, V);
     } else {
-      bfs_phase(P, V);
+      clear_dirty(P, V, cbits_words(P));
+      pull = pull_mode(V, P.own_n, frontier_bfs(V)) ? kPullScan : kPush;
+      if (pull) {
+        bfs_apply_phase(P, V);
+        grid_sync(ctl);
+        pull_phase<true>(P, V);
+      } else {
+        bfs_phase(P, V);
+      }
     }
     grid_sync(ctl);
-    if (blockIdx.x == 0) close_superstep(P, 0ull, 0);
+    if (blockIdx.x == 0) close_superstep(P, 0ull, 0, pull);
     grid_sync(ctl);
   }
 }

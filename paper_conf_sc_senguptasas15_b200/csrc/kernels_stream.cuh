@@ -55,7 +55,8 @@ __global__ void __launch_bounds__(kBlock) k_s_gather_apply(const __grid_constant
       deg = (uint32_t)((uint64_t)P.in_off[lv + 1] - beg);
       cur = P.val[v];
     }
-    const G acc = gather_warp<Prog>(P, valid, beg, deg, cur, sred[warp], cx);
+    bool unused;
+    const G acc = gather_warp<Prog, false>(P, valid, beg, deg, cur, sred[warp], cx, nullptr, unused);
     bool changed = false;
     uint32_t nv = cur;
     if (valid) {
@@ -177,7 +178,7 @@ __global__ void __launch_bounds__(kBlock) k_s_activate(const __grid_constant__ P
 
 // Close the superstep (one CTA): the same bookkeeping as the resident path.
 template <class OffT> __global__ void k_s_finish(const __grid_constant__ Part<OffT> P) {
-  finish_superstep(P, 0ull, 0);
+  finish_superstep(P, 0ull, 0, kPush);
 }
 
 // Stamp a host-computed starting frontier (SSSP: out-neighbours of the source).

@@ -28,23 +28,35 @@ def check_pr(got, ref, n):
     assert abs(got.sum() - ref.sum()) <= 1e-5
 
 
-def compare(n, src, dst, w, algo, source=0, max_iters=0, loops=("auto", "device", "host"), **load):
+DIRS = ("auto", "push", "pull")
+
+
+def compare(n, src, dst, w, algo, source=0, max_iters=0, loops=("auto", "device", "host"), directions=DIRS,
+            **load):
+    """Every loop driver x every FrontierActivate direction (push / pull / the
+    size heuristic) must reproduce the oracle's values and trace."""
     og = oracle.OracleGraph(n, src, dst, w)
     ref, rtr, rit = og.run(algo, source=source, max_iters=max_iters)
     og.close()
     with gr.GraphReduce(n, src, dst, w, **load) as G:
+        resident1 = G.info()["mode"] == gr.MODES["resident"] and G.info()["world"] == 1
         for loop in loops:
-            st = G.run(algo, source=source, max_iters=max_iters, loop=loop)
-            got = G.values(algo)
-            tr = G.trace()
-            assert st["iterations"] == rit, (loop, st["iterations"], rit)
-            if algo == "pagerank":
-                check_pr(got, ref, n)
-            else:
-                np.testing.assert_array_equal(got, ref)
-                np.testing.assert_array_equal(tr, rtr)
+            for d in (directions if algo != "pagerank" else ("auto",)):
+                st = G.run(algo, source=source, max_iters=max_iters, loop=loop, direction=d)
+                got = G.values(algo)
+                tr = G.trace()
+                assert st["iterations"] == rit, (loop, d, st["iterations"], rit)
+                if algo == "pagerank":
+                    check_pr(got, ref, n)
+                    continue
+                np.testing.assert_array_equal(got, ref, err_msg=f"{loop} {d}")
+                np.testing.assert_array_equal(tr, rtr, err_msg=f"{loop} {d}")
                 assert st["edges_gathered"] == int(rtr[:, 2].sum())
                 assert st["edges_scattered"] == int(rtr[:, 3].sum())
+                if d == "push" or not resident1:
+                    assert st["pull_supersteps"] == 0
+                elif d == "pull" and rtr[:, 1].sum() > 0:
+                    assert st["pull_supersteps"] > 0
     return st
 
 
