@@ -170,6 +170,20 @@ gr_status gr_get_unique_id(uint8_t out[128]);
  * keeps only its owned destination range. */
 gr_status gr_graph_load(const gr_edges *edges, const gr_load_opts *opts, gr_graph **out);
 
+/* Load from a canonical graph file (memory-mapped, read-only; every rank of a
+ * multi-GPU job maps the same file and keeps its owned range — SURVEY §8(b)).
+ * Little-endian layout, 32-byte header then the arrays, each 4-byte aligned:
+ *   char     magic[8] = "GRGRAPH1"
+ *   uint64_t num_vertices, num_edges
+ *   uint32_t fmt        (gr_format: 0 COO, 1 CSR by source)
+ *   uint32_t flags      (bit 0: weights present)
+ *   COO: uint32 src[m], uint32 dst[m]          CSR: uint64 row_offsets[n+1], uint32 col_idx[m]
+ *   then, if flags & 1: uint32 weights[m]
+ * GR_EINVAL: unreadable file, bad magic/format/flags, or a size that does not
+ * match the header; otherwise exactly gr_graph_load's behaviour. The mapping
+ * is released before returning. */
+gr_status gr_graph_load_file(const char *path, const gr_load_opts *opts, gr_graph **out);
+
 /* Run one program to termination (PAPER.md L62 stages 1-3). Synchronous: returns
  * when the results are on the device. */
 gr_status gr_run(gr_graph *g, const gr_run_opts *opts, gr_run_stats *stats);

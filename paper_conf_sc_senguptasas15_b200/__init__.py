@@ -31,7 +31,7 @@ DIRECTIONS = {"auto": 0, "push": 1, "pull": 2}
 INF = 0xFFFFFFFF
 
 EXPORTS = [
-    "gr_get_unique_id", "gr_graph_load", "gr_run", "gr_fetch_vertex_values", "gr_fetch_frontier_trace",
+    "gr_get_unique_id", "gr_graph_load", "gr_graph_load_file", "gr_run", "gr_fetch_vertex_values", "gr_fetch_frontier_trace",
     "gr_graph_info_get", "gr_shard_info", "gr_graph_free", "gr_last_error", "gr_plan_intervals",
     "gr_host_build", "gr_host_csc", "gr_host_csr", "gr_host_shards", "gr_host_free",
 ]
@@ -96,16 +96,20 @@ def lib():
     global _lib
     if _lib is not None:
         return _lib
-    if not os.path.exists(_SO) or _build.stale():
-        if not os.path.exists(_build.NVCC):
-            raise GrError(GR_EUNSUPPORTED, f"{_SO} is missing and nvcc is unavailable to build it")
-        _build.build()
-    L = ctypes.CDLL(_SO)
+    so = os.environ.get("GR_LIB")  # experiments: an alternative in-tree build of the same library
+    if not so:
+        so = _SO
+        if not os.path.exists(_SO) or _build.stale():
+            if not os.path.exists(_build.NVCC):
+                raise GrError(GR_EUNSUPPORTED, f"{_SO} is missing and nvcc is unavailable to build it")
+            _build.build()
+    L = ctypes.CDLL(so)
     vp, u64, u32, i32 = ctypes.c_void_p, ctypes.c_uint64, ctypes.c_uint32, ctypes.c_int32
     u64p = ctypes.POINTER(ctypes.c_uint64)
     sig = {
         "gr_get_unique_id": (i32, [vp]),
         "gr_graph_load": (i32, [ctypes.POINTER(gr_edges), ctypes.POINTER(gr_load_opts), ctypes.POINTER(vp)]),
+        "gr_graph_load_file": (i32, [ctypes.c_char_p, ctypes.POINTER(gr_load_opts), ctypes.POINTER(vp)]),
         "gr_run": (i32, [vp, ctypes.POINTER(gr_run_opts), ctypes.POINTER(gr_run_stats)]),
         "gr_fetch_vertex_values": (i32, [vp, vp, u64]),
         "gr_fetch_frontier_trace": (i32, [vp, u64p, u64, u64p]),
@@ -190,6 +194,45 @@ def gr_graph_load(n, src=None, dst=None, weights=None, row_offsets=None, col_idx
     h = ctypes.c_void_p()
     _check(lib().gr_graph_load(ctypes.byref(e), ctypes.byref(o), ctypes.byref(h)))
     del keep, uid
+    return h
+
+
+GRAPH_FILE_MAGIC = b"GRGRAPH1"
+
+
+def write_graph_file(path, n, src=None, dst=None, weights=None, row_offsets=None, col_idx=None):
+    """Write the canonical graph file read by gr_graph_load_file (layout in
+    include/graphreduce.h): 32-byte header, then COO src/dst (or CSR
+    row_offsets/col_idx), then optional uint32 weights."""
+    if row_offsets is not None:
+        ro = np.ascontiguousarray(row_offsets, dtype=np.uint64)
+        ci = np.ascontiguousarray(col_idx, dtype=np.uint32)
+        fmt, m, arrays = GR_FMT_CSR, ci.shape[0], [ro, ci]
+    else:
+        s_, d_ = np.ascontiguousarray(src, dtype=np.uint32), np.ascontiguousarray(dst, dtype=np.uint32)
+        if s_.shape != d_.shape:
+            raise ValueError("src and dst lengths differ")
+        fmt, m, arrays = GR_FMT_COO, s_.shape[0], [s_, d_]
+    flags = 0
+    if weights is not None:
+        w = np.ascontiguousarray(weights, dtype=np.uint32)
+        if w.shape[0] != m:
+            raise ValueError("weights length != number of edges")
+        arrays.append(w)
+        flags = 1
+    hdr = GRAPH_FILE_MAGIC + np.array([n, m], np.uint64).tobytes() + np.array([fmt, flags], np.uint32).tobytes()
+    with open(path, "wb") as f:
+        f.write(hdr)
+        for a in arrays:
+            a.tofile(f)
+
+
+def gr_graph_load_file(path, **opts):
+    """gr_graph_load from a canonical graph file (memory-mapped by the library)."""
+    o, uid = _load_opts(**opts)
+    h = ctypes.c_void_p()
+    _check(lib().gr_graph_load_file(os.fsencode(path), ctypes.byref(o), ctypes.byref(h)))
+    del uid
     return h
 
 
@@ -293,6 +336,13 @@ class GraphReduce:
     def __init__(self, n, src=None, dst=None, weights=None, **opts):
         self.n = int(n)
         self.h = gr_graph_load(n, src, dst, weights, **opts)
+
+    @classmethod
+    def from_file(cls, path, **opts):
+        self = cls.__new__(cls)
+        self.h = gr_graph_load_file(path, **opts)
+        self.n = gr_graph_info_get(self.h)["num_vertices"]
+        return self
 
     def run(self, algo, **kw) -> dict:
         return gr_run(self.h, algo, **kw)

@@ -41,14 +41,17 @@ def stale() -> bool:
     return any(os.path.getmtime(p) > t for p in _deps())
 
 
-def build(force: bool = False, verbose: bool = False) -> str:
-    if not force and not stale():
+def build(force: bool = False, verbose: bool = False, out: str | None = None, defines=()) -> str:
+    """Compile every csrc source and link `out` (default: the in-tree SO).
+    `defines` (e.g. ["GR_WIPT=4"]) select compile-time variants for experiments."""
+    so = out or SO
+    if out is None and not force and not stale():
         return SO
     nccl_inc, nccl_lib = _nccl_dirs()
-    objdir = os.path.join(PKG, "build")
+    objdir = os.path.join(PKG, "build" if not defines else "build_" + "_".join(d.replace("=", "") for d in defines))
     os.makedirs(objdir, exist_ok=True)
     common = ["-O3", "-std=c++17", "-lineinfo", "-Xcompiler", "-fPIC,-O3", "-I", INCLUDE, "-I", CSRC,
-              "-I", nccl_inc]
+              "-I", nccl_inc] + [f"-D{d}" for d in defines]
 
     def compile_one(src):
         obj = os.path.join(objdir, os.path.basename(src) + ".o")
@@ -67,14 +70,14 @@ def build(force: bool = False, verbose: bool = False) -> str:
         for _, err in results:
             if err:
                 print(err)
-    tmp = SO + f".tmp{os.getpid()}"
+    tmp = so + f".tmp{os.getpid()}"
     cmd = [NVCC, *ARCH, "-shared", "-cudart", "shared", "-o", tmp, *objs, "-L", nccl_lib, "-l:libnccl.so.2",
            "-Xlinker", f"-rpath,{nccl_lib}", "-lpthread"]
     r = subprocess.run(cmd, capture_output=True, text=True)
     if r.returncode != 0:
         raise RuntimeError(f"link failed:\n{r.stderr[-6000:]}")
-    os.replace(tmp, SO)
-    return SO
+    os.replace(tmp, so)
+    return so
 
 
 if __name__ == "__main__":

@@ -3,6 +3,11 @@
 #include <nccl.h>
 
 #include <cstring>
+#include <cerrno>
+#include <fcntl.h>
+#include <sys/mman.h>
+#include <sys/stat.h>
+#include <unistd.h>
 
 #include "engine.h"
 
@@ -210,6 +215,55 @@ gr_status gr_shard_info(const gr_graph *g, uint32_t s, gr_shard_desc *o) {
 }
 
 void gr_graph_free(gr_graph *g) { destroy(g); }
+
+gr_status gr_graph_load_file(const char *path, const gr_load_opts *opts, gr_graph **out) {
+  clear_error();
+  if (!path || !out) return fail(GR_EINVAL, "null argument");
+  *out = nullptr;
+  const int fd = open(path, O_RDONLY);
+  if (fd < 0) return fail(GR_EINVAL, "cannot open %s: %s", path, strerror(errno));
+  struct stat sb;
+  if (fstat(fd, &sb) != 0 || sb.st_size < 32) {
+    close(fd);
+    return fail(GR_EINVAL, "%s: not a graph file (size %lld)", path, (long long)sb.st_size);
+  }
+  const size_t size = (size_t)sb.st_size;
+  void *map = mmap(nullptr, size, PROT_READ, MAP_PRIVATE, fd, 0);
+  close(fd);
+  if (map == MAP_FAILED) return fail(GR_EINVAL, "mmap %s: %s", path, strerror(errno));
+  madvise(map, size, MADV_SEQUENTIAL);
+  const unsigned char *b = (const unsigned char *)map;
+  struct Hdr { char magic[8]; uint64_t n, m; uint32_t fmt, flags; } h;
+  std::memcpy(&h, b, sizeof h);
+  gr_status st = GR_OK;
+  gr_edges e{};
+  if (std::memcmp(h.magic, "GRGRAPH1", 8) != 0) st = fail(GR_EINVAL, "%s: bad magic", path);
+  else if (h.fmt > GR_FMT_CSR || (h.flags & ~1u)) st = fail(GR_EINVAL, "%s: bad fmt %u / flags %u", path, h.fmt, h.flags);
+  else if (h.n >= (1ull << 40) || h.m >= (1ull << 40)) st = fail(GR_EINVAL, "%s: implausible n/m", path);
+  else {
+    const uint64_t body = h.fmt == GR_FMT_COO ? 8 * h.m : 8 * (h.n + 1) + 4 * h.m;
+    const uint64_t need = 32 + body + ((h.flags & 1) ? 4 * h.m : 0);
+    if (need != size) st = fail(GR_EINVAL, "%s: size %zu != %llu expected from the header", path, size,
+                                (unsigned long long)need);
+    else {
+      e.fmt = (int32_t)h.fmt;
+      e.num_vertices = h.n;
+      e.num_edges = h.m;
+      const unsigned char *p = b + 32;
+      if (h.fmt == GR_FMT_COO) {
+        e.src = (const uint32_t *)p;
+        e.dst = (const uint32_t *)(p + 4 * h.m);
+      } else {
+        e.row_offsets = (const uint64_t *)p;
+        e.col_idx = (const uint32_t *)(p + 8 * (h.n + 1));
+      }
+      if (h.flags & 1) e.weights = (const uint32_t *)(b + 32 + body);
+    }
+  }
+  if (st == GR_OK) st = gr_graph_load(&e, opts, out);  // copies everything it keeps
+  munmap(map, size);
+  return st;
+}
 
 gr_status gr_host_build(const gr_edges *edges, const gr_load_opts *opts_in, gr_host_graph **out) {
   clear_error();

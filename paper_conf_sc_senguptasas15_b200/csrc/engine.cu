@@ -383,7 +383,9 @@ static gr_status run_frontier(gr_graph *g, const gr_run_opts *o, cudaStream_t s,
   if (persistent) {
     int bps = 0;
     CK(cudaOccupancyMaxActiveBlocksPerMultiprocessor(&bps, k_persistent<Prog, OffT>, kBlock, 0));
-    const uint32_t grid = (uint32_t)g->num_sms * (uint32_t)std::max(1, std::min(bps, 4));
+    int per_sm = std::min(bps, 4);
+    if (const char *e = getenv("GR_PERSIST_CTAS_PER_SM")) per_sm = std::min(bps, atoi(e));
+    const uint32_t grid = (uint32_t)g->num_sms * (uint32_t)std::max(1, per_sm);
     void *args[] = {(void *)&P};
     CK(cudaLaunchCooperativeKernel((const void *)k_persistent<Prog, OffT>, dim3(grid), dim3(kBlock), args, 0, s));
     CK(cudaMemcpyAsync(g->h_ctl, g->ctl, sizeof(Ctl), cudaMemcpyDeviceToHost, s));

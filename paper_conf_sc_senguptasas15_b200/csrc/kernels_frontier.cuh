@@ -535,11 +535,13 @@ __device__ __forceinline__ void bfs_apply_phase(const Part<OffT> &P, const View 
   if (threadIdx.x == 0 && my_c) atomicAdd(&P.ctl->part_c[blockIdx.x % kSlots], my_c);
 }
 
-// Pull mode: A_{t+1} = owned x with an in-neighbour in C_t. Each lane probes
-// the first kProbe in-edges of its vertex; the vertices still undecided are
-// then scanned by the whole warp, 32 edges per step, stopping at the first hit.
+// Pull mode (BFS): A_{t+1} = owned x with an in-neighbour in C_t. Each lane
+// scans its own vertex (kProbe loads in flight, stopping at the first hit);
+// vertices of in-degree > kPullLane are scanned by the whole warp, 32 edges
+// per step.
 // BFS keeps only unvisited vertices in the list (counts every activated one).
 constexpr uint32_t kProbe = 4;
+constexpr uint32_t kPullLane = 128;  // in-degree up to which a lane scans its vertex alone
 constexpr uint32_t kPullDivDefault = 16;  // GR_DIR_AUTO: pull when |C_t| > |V| / 16
 template <bool kBfs, class OffT>
 __device__ __forceinline__ void pull_phase(const Part<OffT> &P, const View &V) {
@@ -570,7 +572,16 @@ __device__ __forceinline__ void pull_phase(const Part<OffT> &P, const View &V) {
     bool found = false;
 #pragma unroll
     for (uint32_t q = 0; q < kProbe; q++) found |= (q < deg) && test_bit_cg(bits, src[q]);
-    uint32_t pend = __ballot_sync(0xffffffffu, !found && deg > kProbe);
+    // moderate degrees: each lane continues its own scan, kProbe loads in flight
+    for (uint64_t k = beg + kProbe; !found && deg <= kPullLane && k < end; k += kProbe) {
+      uint32_t u[kProbe];
+#pragma unroll
+      for (uint32_t q = 0; q < kProbe; q++) u[q] = (k + q < end) ? ldg_nc(P.in_src + k + q) : 0u;
+#pragma unroll
+      for (uint32_t q = 0; q < kProbe; q++) found |= (k + q < end) && test_bit_cg(bits, u[q]);
+    }
+    // large degrees: the whole warp scans one vertex at a time
+    uint32_t pend = __ballot_sync(0xffffffffu, !found && deg > kPullLane);
     uint32_t fm = 0;
     while (pend) {
       const int l = __ffs(pend) - 1;

@@ -206,7 +206,10 @@ __global__ void __launch_bounds__(kPrThreads, 6) k_pr_gather_apply(const __grid_
 // apply are warp-local (shuffles + __syncwarp), so warps never wait at a CTA
 // barrier and every warp's memory phases overlap with its neighbours'.
 // Rows spanning warp tiles are finished by k_pr_fixup_warp.
-constexpr int kWIpt = 8;
+#ifndef GR_WIPT
+#define GR_WIPT 8
+#endif
+constexpr int kWIpt = GR_WIPT;  // items per lane of a warp tile
 constexpr int kWTile = 32 * kWIpt;
 constexpr int kWPad = kWTile / kWIpt;
 

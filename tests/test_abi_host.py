@@ -134,3 +134,50 @@ def test_multirank_owner_ranges_partition_edges():
         assert np.all((p.out_dst >= lo[r]) & (p.out_dst < hi[r]))
         owned = (g.dst >= lo[r]) & (g.dst < hi[r])
         assert len(p.out_dst) == owned.sum()
+
+
+def test_graph_file_validation(tmp_path):
+    """gr_graph_load_file parses the canonical file before touching the device:
+    malformed files are GR_EINVAL; well-formed ones reach the device stage
+    (GR_ECUDA here, without a GPU)."""
+    import torch
+
+    g = grgen.rmat(8, 4, seed=1)
+    w = grgen.weights(g.m, 1, 64, seed=1)
+    good = tmp_path / "g.bin"
+    gr.write_graph_file(good, g.n, g.src, g.dst, w)
+    raw = good.read_bytes()
+    assert len(raw) == 32 + 12 * g.m and raw[:8] == b"GRGRAPH1"
+    hdr = np.frombuffer(raw[8:24], np.uint64)
+    assert hdr[0] == g.n and hdr[1] == g.m
+    np.testing.assert_array_equal(np.frombuffer(raw[32:32 + 4 * g.m], np.uint32), g.src)
+    np.testing.assert_array_equal(np.frombuffer(raw[32 + 8 * g.m:], np.uint32), w)
+    bad = {
+        "magic": b"XXGRAPH1" + raw[8:],
+        "truncated": raw[:-4],
+        "extra": raw + b"\0\0\0\0",
+        "fmt": raw[:24] + np.array([7, 1], np.uint32).tobytes() + raw[32:],
+        "flags": raw[:24] + np.array([0, 6], np.uint32).tobytes() + raw[32:],
+        "tiny": raw[:16],
+    }
+    for name, data in bad.items():
+        p = tmp_path / f"bad_{name}.bin"
+        p.write_bytes(data)
+        with pytest.raises(gr.GrError) as ei:
+            gr.gr_graph_load_file(p)
+        assert ei.value.status == gr.GR_EINVAL, name
+    with pytest.raises(gr.GrError) as ei:
+        gr.gr_graph_load_file(tmp_path / "missing.bin")
+    assert ei.value.status == gr.GR_EINVAL
+    # CSR form: header + row offsets + col idx
+    order = np.lexsort((g.dst, g.src))
+    ro = np.zeros(g.n + 1, np.uint64)
+    ro[1:] = np.cumsum(np.bincount(g.src, minlength=g.n))
+    csr = tmp_path / "csr.bin"
+    gr.write_graph_file(csr, g.n, row_offsets=ro, col_idx=g.dst[order])
+    assert csr.stat().st_size == 32 + 8 * (g.n + 1) + 4 * g.m
+    if not torch.cuda.is_available():
+        for p in (good, csr):
+            with pytest.raises(gr.GrError) as ei:
+                gr.gr_graph_load_file(p)
+            assert ei.value.status == gr.GR_ECUDA

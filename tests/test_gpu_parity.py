@@ -295,3 +295,30 @@ def test_custom_program_widest_path(mode):
         G.run("custom", custom_id=0, source=5)
         np.testing.assert_array_equal(G.values(), ref)
         np.testing.assert_array_equal(G.trace(), rtr)
+
+
+@pytest.mark.parametrize("fmt", ["coo", "csr"])
+def test_load_from_file(tmp_path, fmt):
+    """gr_graph_load_file (mmap of the canonical file) == in-memory load, both formats."""
+    g = grgen.rmat(13, 8, seed=4)
+    w = grgen.weights(g.m, 1, 64, seed=4)
+    path = tmp_path / "g.bin"
+    if fmt == "coo":
+        gr.write_graph_file(path, g.n, g.src, g.dst, w)
+    else:
+        order = np.lexsort((g.dst, g.src))
+        ro = np.zeros(g.n + 1, np.uint64)
+        ro[1:] = np.cumsum(np.bincount(g.src, minlength=g.n))
+        gr.write_graph_file(path, g.n, row_offsets=ro, col_idx=g.dst[order], weights=w[order])
+    og = oracle.OracleGraph(g.n, g.src, g.dst, w)
+    with gr.GraphReduce.from_file(path) as G:
+        assert G.n == g.n and G.info()["num_edges"] == g.m
+        for algo in ("bfs", "sssp", "pagerank"):
+            G.run(algo, source=1)
+            ref, rtr, _ = og.run(algo, source=1)
+            if algo == "pagerank":
+                check_pr(G.values(algo), ref, g.n)
+            else:
+                np.testing.assert_array_equal(G.values(algo), ref)
+                np.testing.assert_array_equal(G.trace(), rtr)
+    og.close()
