@@ -111,6 +111,10 @@ typedef struct gr_run_opts {
   int32_t profile;    /* 1: time the per-phase kernels with CUDA events (stats.kernel_ms) */
   int32_t direction;  /* gr_direction: how FrontierActivate reaches the out-neighbours of C_t */
   uint32_t pull_div;  /* GR_DIR_AUTO: pull when |C_t| * pull_div > |V|; 0 = library default (16) */
+  int32_t zero_copy;  /* streamed mode: how a superstep reads the active shards' edges —
+                         0 auto (in place over the host link when the frontier's edges are
+                         < 1/8 of the active shards' edges, else DMA whole shards into the
+                         device slots), 1 always in place, -1 never */
 } gr_run_opts;
 
 /* FrontierActivate direction (resident single-rank frontier programs; the
@@ -132,7 +136,8 @@ typedef struct gr_run_stats {
   uint64_t kernel_launches;  /* library kernel launches issued by this run */
   double kernel_ms[4];       /* profile: [0] gather(+apply), [1] activate/expand, [2] exchange, [3] other */
   uint32_t pull_supersteps;  /* supersteps whose FrontierActivate ran by pull */
-  uint32_t reserved;
+  uint32_t zero_copy_phases; /* streamed: gather / activate phases that read edges in place */
+  uint64_t bytes_h2d_zero_copy; /* part of bytes_h2d read in place by the kernels (4 B per edge, +1 B weight) */
 } gr_run_stats;
 
 typedef struct gr_graph_info {

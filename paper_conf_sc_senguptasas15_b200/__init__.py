@@ -60,7 +60,7 @@ class gr_run_opts(ctypes.Structure):
     _fields_ = [("algo", ctypes.c_int32), ("source", ctypes.c_uint32), ("max_iters", ctypes.c_uint32),
                 ("damping", ctypes.c_float), ("custom_id", ctypes.c_int32), ("loop", ctypes.c_int32),
                 ("stream", ctypes.c_void_p), ("profile", ctypes.c_int32), ("direction", ctypes.c_int32),
-                ("pull_div", ctypes.c_uint32)]
+                ("pull_div", ctypes.c_uint32), ("zero_copy", ctypes.c_int32)]
 
 
 class gr_run_stats(ctypes.Structure):
@@ -69,7 +69,7 @@ class gr_run_stats(ctypes.Structure):
                 ("bytes_h2d", ctypes.c_uint64), ("bytes_nvlink", ctypes.c_uint64),
                 ("bytes_hbm_model", ctypes.c_uint64), ("kernel_launches", ctypes.c_uint64),
                 ("kernel_ms", ctypes.c_double * 4), ("pull_supersteps", ctypes.c_uint32),
-                ("reserved", ctypes.c_uint32)]
+                ("zero_copy_phases", ctypes.c_uint32), ("bytes_h2d_zero_copy", ctypes.c_uint64)]
 
     def as_dict(self):
         d = {k: getattr(self, k) for k, _ in self._fields_ if k != "kernel_ms"}
@@ -237,7 +237,7 @@ def gr_graph_load_file(path, **opts):
 
 
 def gr_run(h, algo, source=0, max_iters=0, damping=0.85, custom_id=0, loop="auto", stream=None,
-           profile=False, direction="auto", pull_div=0) -> dict:
+           profile=False, direction="auto", pull_div=0, zero_copy=0) -> dict:
     o = gr_run_opts()
     o.algo = ALGOS[algo] if isinstance(algo, str) else int(algo)
     o.source, o.max_iters, o.damping, o.custom_id = int(source), int(max_iters), float(damping), int(custom_id)
@@ -246,6 +246,7 @@ def gr_run(h, algo, source=0, max_iters=0, damping=0.85, custom_id=0, loop="auto
     o.profile = 1 if profile else 0
     o.direction = DIRECTIONS[direction] if isinstance(direction, str) else int(direction)
     o.pull_div = int(pull_div)
+    o.zero_copy = int(zero_copy)
     st = gr_run_stats()
     _check(lib().gr_run(h, ctypes.byref(o), ctypes.byref(st)))
     return st.as_dict()

@@ -14,6 +14,7 @@
 #include <cuda_runtime.h>
 
 #include <algorithm>
+#include <cstdlib>
 #include <cstring>
 #include <vector>
 
@@ -46,7 +47,16 @@ struct Streamer {
   uint32_t *cstamp = nullptr;
   uint32_t *d_list = nullptr;
   uint64_t bytes_h2d = 0;
+  // zero-copy views of the pinned payloads (device addresses of the mapped host buffers)
+  const uint32_t *zc_in = nullptr, *zc_out = nullptr;
+  const uint8_t *zc_w = nullptr;
+  uint64_t bytes_zc = 0;
+  uint32_t zc_phases = 0;
 };
+
+// auto mode: read in place when the frontier's edges are < 1/kZcDiv of the
+// edges a whole-shard DMA of the active shards would move
+constexpr uint64_t kZcDiv = 8;
 
 static Streamer *S_(gr_graph *g) { return static_cast<Streamer *>(g->streamer); }
 
@@ -76,13 +86,18 @@ gr_status stream_setup(gr_graph *g, uint64_t budget) {
   // page-lock the host payloads for DMA
   for (HostBuf *b : {&H.in_src, &H.out_dst, &H.in_w}) {
     if (!b->p || !b->bytes) continue;
-    cudaError_t e = cudaHostRegister(b->p, b->bytes, cudaHostRegisterDefault);
+    cudaError_t e = cudaHostRegister(b->p, b->bytes, cudaHostRegisterMapped);
     if (e != cudaSuccess) {
       cudaGetLastError();
       return fail(GR_ENOMEM, "cudaHostRegister(%zu bytes): %s", b->bytes, cudaGetErrorString(e));
     }
     b->registered = true;
     g->pinned_bytes += b->bytes;
+    void *dp = nullptr;
+    SCK(cudaHostGetDevicePointer(&dp, b->p, 0));
+    if (b == &H.in_src) S->zc_in = (const uint32_t *)dp;
+    else if (b == &H.out_dst) S->zc_out = (const uint32_t *)dp;
+    else S->zc_w = (const uint8_t *)dp;
   }
   gr_status st;
   for (int k = 0; k < 2; k++) {
@@ -160,6 +175,26 @@ static gr_status stage(gr_graph *g, Streamer *S, cudaStream_t cs, bool in, uint3
   return GR_OK;
 }
 
+// Zero-copy view: the kernels read the whole pinned payload in place (global edge positions).
+template <class OffT> static Part<OffT> zc_part(gr_graph *g, Streamer *S, bool in) {
+  Part<OffT> P = make_part<OffT>(g);
+  if (in) {
+    P.in_src = S->zc_in;
+    P.in_w = S->zc_w;
+  } else {
+    P.out_dst = S->zc_out;
+  }
+  return P;
+}
+
+static bool want_zc(const gr_run_opts *o, uint64_t frontier_edges, uint64_t shard_edges) {
+  if (o->zero_copy > 0) return true;
+  if (o->zero_copy < 0) return false;
+  uint64_t div = kZcDiv;
+  if (const char *e = getenv("GR_ZC_DIV")) div = strtoull(e, nullptr, 10);
+  return div > 0 && frontier_edges * div < shard_edges;
+}
+
 template <class OffT> static Part<OffT> slot_part(gr_graph *g, Streamer *S, int k, bool in, uint32_t s) {
   Part<OffT> P = make_part<OffT>(g);
   const uint64_t b = in ? S->in_b[s] : S->out_b[s];
@@ -192,9 +227,13 @@ static gr_status stream_pagerank(gr_graph *g, const gr_run_opts *o, cudaStream_t
       const uint64_t r0 = H.bounds[s] - H.own_lo, rows = H.bounds[s + 1] - H.bounds[s];
       const uint64_t me = S->in_b[s + 1] - S->in_b[s];
       if (rows == 0) continue;
-      int k;
-      gr_status gs = stage(g, S, cs, true, s, false, &k);
-      if (gs != GR_OK) return gs;
+      int k = -1;  // PageRank reads every edge: DMA unless zero-copy is forced
+      if (o->zero_copy <= 0) {
+        gr_status gs = stage(g, S, cs, true, s, false, &k);
+        if (gs != GR_OK) return gs;
+      } else {
+        S->bytes_zc += 4 * me;
+      }
       PrArgs<OffT> a{};
       a.n = (uint32_t)H.n;
       a.own_lo = (uint32_t)H.bounds[s];
@@ -202,7 +241,7 @@ static gr_status stream_pagerank(gr_graph *g, const gr_run_opts *o, cudaStream_t
       a.m_in = me;
       a.e_base = S->in_b[s];
       a.in_off = (const OffT *)g->in_off + r0;
-      a.in_src = S->slot_idx[k];
+      a.in_src = k >= 0 ? S->slot_idx[k] : S->zc_in + S->in_b[s];
       a.inv_outdeg = g->inv_outdeg;
       a.contrib_in = g->contrib[t & 1];
       a.contrib_out = g->contrib[(t + 1) & 1];
@@ -218,13 +257,14 @@ static gr_status stream_pagerank(gr_graph *g, const gr_run_opts *o, cudaStream_t
       a.last = (t + 1 == iters) ? 1 : 0;
       k_pr_gather_apply<OffT><<<tiles, kPrThreads, 0, cs>>>(a);
       k_pr_fixup<OffT><<<(tiles + 255) / 256, 256, 0, cs>>>(a, tiles);
-      SCK(cudaEventRecord(S->freed[k], cs));
+      if (k >= 0) SCK(cudaEventRecord(S->freed[k], cs));
       launches += 2;
     }
   }
   SCK(cudaGetLastError());
   SCK(cudaStreamSynchronize(cs));
   st->iterations = iters;
+  if (o->zero_copy > 0) S->zc_phases += iters;
   st->edges_gathered = (uint64_t)iters * H.m_in;
   st->kernel_launches += launches;
   st->bytes_hbm_model = (uint64_t)iters * (4 * H.m_in + 12 * H.own_n() + 4 * H.n);
@@ -286,19 +326,37 @@ static gr_status stream_frontier(gr_graph *g, const gr_run_opts *o, cudaStream_t
   SCK(cudaMemcpyAsync(g->h_ctl, g->ctl, sizeof(Ctl), cudaMemcpyDeviceToHost, cs));
   SCK(cudaStreamSynchronize(cs));
   uint8_t *h_changed = S->h_flags, *h_next = S->h_flags + P;
+  const double avg_in = H.own_n() ? (double)H.m_in / (double)H.own_n() : 0.0;
+  const double avg_out = H.n ? (double)H.m_in / (double)H.n : 0.0;
+  const uint64_t wb = Prog::kUsesWeights ? 5 : 4;
   while (!g->h_ctl->stop) {
+    const uint64_t g0 = g->h_ctl->tot_gathered, s0 = g->h_ctl->tot_scattered;
     SCK(cudaMemsetAsync(S->d_changed, 0, P, cs));
+    // gather phase: whole-shard DMA, or in place when A_t's in-edges are few (f1)
+    bool zc_g = false;
+    if (Prog::kHasGather) {
+      uint64_t shard_e = 0;
+      for (uint32_t s = 0; s < P; s++)
+        if (act[s]) shard_e += S->in_b[s + 1] - S->in_b[s];
+      const uint32_t nA = g->h_ctl->iter == 0 && g->h_ctl->implicit0 ? (uint32_t)H.own_n()
+                                                                       : g->h_ctl->cnt_act[g->h_ctl->iter & 1u];
+      zc_g = want_zc(o, (uint64_t)(nA * avg_in), shard_e);
+      if (zc_g) S->zc_phases++;
+    }
+    const Part<OffT> Pz_in = zc_part<OffT>(g, S, true);
     for (uint32_t s = 0; s < P; s++) {
       if (!act[s]) continue;  // frontier skipping: no copy, no launch
       const uint32_t v0 = (uint32_t)H.bounds[s], v1 = (uint32_t)H.bounds[s + 1];
       if (Prog::kHasGather) {
-        int k;
-        gr_status gs = stage(g, S, cs, true, s, Prog::kUsesWeights, &k);
-        if (gs != GR_OK) return gs;
-        Part<OffT> Pk = slot_part<OffT>(g, S, k, true, s);
+        int k = -1;
+        if (!zc_g) {
+          gr_status gs = stage(g, S, cs, true, s, Prog::kUsesWeights, &k);
+          if (gs != GR_OK) return gs;
+        }
+        const Part<OffT> Pk = zc_g ? Pz_in : slot_part<OffT>(g, S, k, true, s);
         k_s_gather_apply<Prog, OffT><<<grid_for(g, (v1 - v0)), kBlock, 0, cs>>>(Pk, v0, v1, s, S->d_changed,
                                                                                    S->cstamp);
-        SCK(cudaEventRecord(S->freed[k], cs));
+        if (k >= 0) SCK(cudaEventRecord(S->freed[k], cs));
       } else {
         k_s_bfs_apply<OffT><<<grid_for(g, v1 - v0), kBlock, 0, cs>>>(P0, v0, v1, s, S->d_changed, S->cstamp);
       }
@@ -309,17 +367,27 @@ static gr_status stream_frontier(gr_graph *g, const gr_run_opts *o, cudaStream_t
       launches++;
     }
     SCK(cudaMemcpyAsync(h_changed, S->d_changed, P, cudaMemcpyDeviceToHost, cs));
+    SCK(cudaMemcpyAsync(g->h_ctl, g->ctl, sizeof(Ctl), cudaMemcpyDeviceToHost, cs));
     SCK(cudaMemsetAsync(S->d_next, 0, P, cs));
     SCK(cudaStreamSynchronize(cs));
+    // FrontierActivate: the same choice over the changed vertices' out-edges
+    uint64_t shard_o = 0;
+    for (uint32_t s = 0; s < P; s++)
+      if (h_changed[s]) shard_o += S->out_b[s + 1] - S->out_b[s];
+    const bool zc_a = want_zc(o, (uint64_t)((double)g->h_ctl->changed * avg_out), shard_o);
+    if (zc_a && shard_o) S->zc_phases++;
+    const Part<OffT> Pz_out = zc_part<OffT>(g, S, false);
     for (uint32_t s = 0; s < P; s++) {
       if (!h_changed[s]) continue;
       const uint32_t u0 = (uint32_t)H.bounds[s], u1 = (uint32_t)H.bounds[s + 1];
-      int k;
-      gr_status gs = stage(g, S, cs, false, s, false, &k);
-      if (gs != GR_OK) return gs;
-      Part<OffT> Pk = slot_part<OffT>(g, S, k, false, s);
+      int k = -1;
+      if (!zc_a) {
+        gr_status gs = stage(g, S, cs, false, s, false, &k);
+        if (gs != GR_OK) return gs;
+      }
+      const Part<OffT> Pk = zc_a ? Pz_out : slot_part<OffT>(g, S, k, false, s);
       k_s_activate<OffT><<<grid_for(g, u1 - u0), kBlock, 0, cs>>>(Pk, u0, u1, S->d_bounds, P, S->d_next, S->cstamp);
-      SCK(cudaEventRecord(S->freed[k], cs));
+      if (k >= 0) SCK(cudaEventRecord(S->freed[k], cs));
       launches++;
     }
     k_s_finish<OffT><<<1, kBlock, 0, cs>>>(P0);
@@ -329,6 +397,9 @@ static gr_status stream_frontier(gr_graph *g, const gr_run_opts *o, cudaStream_t
     SCK(cudaMemcpyAsync(h_next, S->d_next, P, cudaMemcpyDeviceToHost, cs));
     SCK(cudaStreamSynchronize(cs));
     for (uint32_t s = 0; s < P; s++) act[s] = h_next[s];
+    // bytes read in place this superstep (exact: the edges the kernels touched)
+    if (zc_g) S->bytes_zc += wb * (g->h_ctl->tot_gathered - g0);
+    if (zc_a) S->bytes_zc += 4 * (g->h_ctl->tot_scattered - s0);
   }
   const Ctl &c = *g->h_ctl;
   st->iterations = c.iter;
@@ -346,6 +417,8 @@ gr_status run_streamed(gr_graph *g, const gr_run_opts *o, gr_run_stats *st) {
   if (!S) return fail(GR_ESTATE, "streamer not initialised");
   cudaStream_t cs = o->stream ? (cudaStream_t)o->stream : g->stream;
   S->bytes_h2d = 0;
+  S->bytes_zc = 0;
+  S->zc_phases = 0;
   SCK(cudaEventRecord(g->ev_start, cs));
   gr_status r;
   switch (o->algo) {
@@ -376,7 +449,9 @@ gr_status run_streamed(gr_graph *g, const gr_run_opts *o, gr_run_stats *st) {
   float ms = 0;
   SCK(cudaEventElapsedTime(&ms, g->ev_start, g->ev_stop));
   st->seconds = ms * 1e-3;
-  st->bytes_h2d = S->bytes_h2d;
+  st->bytes_h2d = S->bytes_h2d + S->bytes_zc;
+  st->bytes_h2d_zero_copy = S->bytes_zc;
+  st->zero_copy_phases = S->zc_phases;
   g->last_algo = o->algo;
   g->last_iters = st->iterations;
   return GR_OK;

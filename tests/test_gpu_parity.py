@@ -32,7 +32,7 @@ DIRS = ("auto", "push", "pull")
 
 
 def compare(n, src, dst, w, algo, source=0, max_iters=0, loops=("auto", "device", "host"), directions=DIRS,
-            **load):
+            run_kw=None, **load):
     """Every loop driver x every FrontierActivate direction (push / pull / the
     size heuristic) must reproduce the oracle's values and trace."""
     og = oracle.OracleGraph(n, src, dst, w)
@@ -42,7 +42,7 @@ def compare(n, src, dst, w, algo, source=0, max_iters=0, loops=("auto", "device"
         resident1 = G.info()["mode"] == gr.MODES["resident"] and G.info()["world"] == 1
         for loop in loops:
             for d in (directions if algo != "pagerank" else ("auto",)):
-                st = G.run(algo, source=source, max_iters=max_iters, loop=loop, direction=d)
+                st = G.run(algo, source=source, max_iters=max_iters, loop=loop, direction=d, **(run_kw or {}))
                 got = G.values(algo)
                 tr = G.trace()
                 assert st["iterations"] == rit, (loop, d, st["iterations"], rit)
@@ -180,14 +180,27 @@ def test_errors_through_abi():
 # ---------------------------------------------------------------- streamed mode
 @pytest.mark.parametrize("algo", ["bfs", "sssp", "cc", "pagerank"])
 @pytest.mark.parametrize("shard_edges", [3000, 40000])
-def test_streamed_equals_oracle(algo, shard_edges):
+@pytest.mark.parametrize("zero_copy", [-1, 0, 1])
+def test_streamed_equals_oracle(algo, shard_edges, zero_copy):
+    """Whole-shard DMA (-1), in-place reads over the host link (1) and the
+    per-phase choice (0) all reproduce the oracle."""
     g = grgen.rmat(13, 16, seed=4)
     src, dst = g.src, g.dst
     if algo == "cc":
         src, dst = np.concatenate([g.src, g.dst]), np.concatenate([g.dst, g.src])
     w = grgen.weights(len(src), 1, 64, seed=5)
-    st = compare(g.n, src, dst, w, algo, source=1, loops=("host",), mode="streamed", shard_edges=shard_edges)
+    st = compare(g.n, src, dst, w, algo, source=1, loops=("host",), mode="streamed", shard_edges=shard_edges,
+                 run_kw={"zero_copy": zero_copy})
     assert st["bytes_h2d"] > 0
+    if zero_copy < 0:
+        assert st["bytes_h2d_zero_copy"] == 0 and st["zero_copy_phases"] == 0
+    if zero_copy > 0:  # nothing staged: every byte was read in place
+        assert st["bytes_h2d"] == st["bytes_h2d_zero_copy"] > 0
+        wb = 5 if algo == "sssp" else 4
+        if algo == "pagerank":
+            assert st["bytes_h2d"] == 4 * len(src) * st["iterations"]
+        else:
+            assert st["bytes_h2d"] == wb * st["edges_gathered"] + 4 * st["edges_scattered"]
 
 
 @pytest.mark.parametrize("algo", ["bfs", "sssp", "cc", "pagerank"])
@@ -216,7 +229,7 @@ def test_streamed_frontier_skips_inactive_shards():
         shards = [gr.gr_shard_info(G.h, s) for s in range(info["num_shards"])]
         first = [s for s in shards if s["v_lo"] < k]
         max_first = max(4 * (s["out_end"] - s["out_begin"]) for s in first)
-        st = G.run("bfs", source=0)
+        st = G.run("bfs", source=0, zero_copy=-1)
         assert st["iterations"] == k
         # one changed vertex per superstep => at most one shard's out-edges copied per superstep
         assert st["bytes_h2d"] <= st["iterations"] * max_first
@@ -225,6 +238,12 @@ def test_streamed_frontier_skips_inactive_shards():
         assert st["bytes_h2d"] < st["iterations"] * whole / 4
         d = G.values()
         assert d[k - 1] == k - 1 and d[k] == gr.INF
+        # f1: with one frontier vertex per superstep the auto policy reads its
+        # single out-edge in place instead of DMA-ing a shard
+        st2 = G.run("bfs", source=0, zero_copy=0)
+        assert st2["zero_copy_phases"] == st2["iterations"]  # one (activation) phase per superstep
+        assert st2["bytes_h2d"] == st2["bytes_h2d_zero_copy"] == 4 * (k - 1)
+        np.testing.assert_array_equal(G.values(), d)
 
 
 @pytest.mark.parametrize("variant", ["block", "warp", "warphot", "range", "rangehot"])
