@@ -22,10 +22,14 @@ __device__ __forceinline__ uint32_t shard_of(const uint64_t *bounds, uint32_t P,
 }
 
 // Gather + apply over the active vertices of one shard [v0, v1); in-edges in a slot.
+// shard == kAllShards: one launch over every shard's interval (zero-copy
+// phases); changed flags are then set per vertex through `bounds`.
+constexpr uint32_t kAllShards = 0xFFFFFFFFu;
 template <class Prog, class OffT>
 __global__ void __launch_bounds__(kBlock) k_s_gather_apply(const __grid_constant__ Part<OffT> P, uint32_t v0,
                                                            uint32_t v1, uint32_t shard, uint8_t *changed_flags,
-                                                           uint32_t *cstamp) {
+                                                           uint32_t *cstamp, const uint64_t *bounds,
+                                                           uint32_t nshards) {
   using G = typename Prog::GatherT;
   Ctl *ctl = P.ctl;
   __shared__ View V;
@@ -62,7 +66,10 @@ __global__ void __launch_bounds__(kBlock) k_s_gather_apply(const __grid_constant
     if (valid) {
       changed = Prog::apply(&nv, acc, cx);
       my_g += deg;
-      if (changed) cstamp[lv] = epoch_t;
+      if (changed) {
+        cstamp[lv] = epoch_t;
+        if (shard == kAllShards) changed_flags[shard_of(bounds, nshards, v)] = 1;
+      }
     }
     qC.push(changed, v, nv, P.C_v, P.C_val, &ctl->cnt_C);
     my_c += changed ? 1 : 0;
@@ -75,7 +82,7 @@ __global__ void __launch_bounds__(kBlock) k_s_gather_apply(const __grid_constant
     if (my_c) { atomicAdd(&ctl->changed, my_c); s_any = 1; }
   }
   __syncthreads();
-  if (threadIdx.x == 0 && s_any) changed_flags[shard] = 1;
+  if (threadIdx.x == 0 && s_any && shard != kAllShards) changed_flags[shard] = 1;
 }
 
 // BSP commit of superstep t: val[u] = new for u in C_t.

@@ -329,6 +329,9 @@ static gr_status stream_frontier(gr_graph *g, const gr_run_opts *o, cudaStream_t
   const double avg_in = H.own_n() ? (double)H.m_in / (double)H.own_n() : 0.0;
   const double avg_out = H.n ? (double)H.m_in / (double)H.n : 0.0;
   const uint64_t wb = Prog::kUsesWeights ? 5 : 4;
+  // ablation knob (Fig. 15): GR_STREAM_NO_SKIP=1 moves and scans every shard every superstep
+  const bool no_skip = getenv("GR_STREAM_NO_SKIP") && getenv("GR_STREAM_NO_SKIP")[0] == '1';
+  if (no_skip) std::fill(act.begin(), act.end(), 1);
   while (!g->h_ctl->stop) {
     const uint64_t g0 = g->h_ctl->tot_gathered, s0 = g->h_ctl->tot_scattered;
     SCK(cudaMemsetAsync(S->d_changed, 0, P, cs));
@@ -337,15 +340,21 @@ static gr_status stream_frontier(gr_graph *g, const gr_run_opts *o, cudaStream_t
     if (Prog::kHasGather) {
       uint64_t shard_e = 0;
       for (uint32_t s = 0; s < P; s++)
-        if (act[s]) shard_e += S->in_b[s + 1] - S->in_b[s];
+        if (act[s] || no_skip) shard_e += S->in_b[s + 1] - S->in_b[s];
       const uint32_t nA = g->h_ctl->iter == 0 && g->h_ctl->implicit0 ? (uint32_t)H.own_n()
                                                                        : g->h_ctl->cnt_act[g->h_ctl->iter & 1u];
       zc_g = want_zc(o, (uint64_t)(nA * avg_in), shard_e);
       if (zc_g) S->zc_phases++;
     }
     const Part<OffT> Pz_in = zc_part<OffT>(g, S, true);
-    for (uint32_t s = 0; s < P; s++) {
-      if (!act[s]) continue;  // frontier skipping: no copy, no launch
+    if (zc_g) {  // in place: one launch over every shard (stamps select A_t)
+      const uint32_t v0 = (uint32_t)H.own_lo, v1 = (uint32_t)H.own_hi;
+      k_s_gather_apply<Prog, OffT><<<grid_for(g, v1 - v0), kBlock, 0, cs>>>(Pz_in, v0, v1, kAllShards, S->d_changed,
+                                                                            S->cstamp, S->d_bounds, P);
+      launches++;
+    }
+    for (uint32_t s = 0; s < P && !zc_g; s++) {
+      if (!act[s] && !no_skip) continue;  // frontier skipping: no copy, no launch
       const uint32_t v0 = (uint32_t)H.bounds[s], v1 = (uint32_t)H.bounds[s + 1];
       if (Prog::kHasGather) {
         int k = -1;
@@ -355,7 +364,7 @@ static gr_status stream_frontier(gr_graph *g, const gr_run_opts *o, cudaStream_t
         }
         const Part<OffT> Pk = zc_g ? Pz_in : slot_part<OffT>(g, S, k, true, s);
         k_s_gather_apply<Prog, OffT><<<grid_for(g, (v1 - v0)), kBlock, 0, cs>>>(Pk, v0, v1, s, S->d_changed,
-                                                                                   S->cstamp);
+                                                                                   S->cstamp, S->d_bounds, P);
         if (k >= 0) SCK(cudaEventRecord(S->freed[k], cs));
       } else {
         k_s_bfs_apply<OffT><<<grid_for(g, v1 - v0), kBlock, 0, cs>>>(P0, v0, v1, s, S->d_changed, S->cstamp);
@@ -373,12 +382,18 @@ static gr_status stream_frontier(gr_graph *g, const gr_run_opts *o, cudaStream_t
     // FrontierActivate: the same choice over the changed vertices' out-edges
     uint64_t shard_o = 0;
     for (uint32_t s = 0; s < P; s++)
-      if (h_changed[s]) shard_o += S->out_b[s + 1] - S->out_b[s];
+      if (h_changed[s] || no_skip) shard_o += S->out_b[s + 1] - S->out_b[s];
     const bool zc_a = want_zc(o, (uint64_t)((double)g->h_ctl->changed * avg_out), shard_o);
     if (zc_a && shard_o) S->zc_phases++;
     const Part<OffT> Pz_out = zc_part<OffT>(g, S, false);
-    for (uint32_t s = 0; s < P; s++) {
-      if (!h_changed[s]) continue;
+    if (zc_a && shard_o) {  // in place: one launch over every shard (changed stamps select C_t)
+      const uint32_t u0 = (uint32_t)H.bounds[0], u1 = (uint32_t)H.bounds[P];
+      k_s_activate<OffT><<<grid_for(g, u1 - u0), kBlock, 0, cs>>>(Pz_out, u0, u1, S->d_bounds, P, S->d_next,
+                                                                  S->cstamp);
+      launches++;
+    }
+    for (uint32_t s = 0; s < P && !zc_a; s++) {
+      if (!h_changed[s] && !no_skip) continue;
       const uint32_t u0 = (uint32_t)H.bounds[s], u1 = (uint32_t)H.bounds[s + 1];
       int k = -1;
       if (!zc_a) {
