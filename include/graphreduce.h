@@ -55,7 +55,10 @@ typedef enum gr_algo {
   GR_SSSP = 1,     /* Bellman-Ford with frontier; "BFS with weighted edges" (L372) */
   GR_PAGERANK = 2, /* L74 (reading R1): R = (1-d)/n + d*sum R_u/outdeg(u); fixed iterations */
   GR_CC = 3,       /* Fig. 6: min-label propagation; input must be symmetric (L290) */
-  GR_CUSTOM = 4    /* program compiled into the library with GR_REGISTER_PROGRAM (gr/program.cuh) */
+  GR_CUSTOM = 4,   /* program compiled into the library: GR_CUSTOM_PROGRAMS in gr/program.cuh */
+  GR_PAGERANK_DELTA = 5 /* tolerance-driven PageRank (Figs. 16-17): a vertex
+                           stays active while |dR| > tolerance/n; exact fixed-point gather, so the
+                           frontier is reproducible (gr/program.cuh ProgPRDelta); fp32 rank values */
 } gr_algo;
 
 typedef enum gr_mode {
@@ -111,6 +114,7 @@ typedef struct gr_run_opts {
   int32_t profile;    /* 1: time the per-phase kernels with CUDA events (stats.kernel_ms) */
   int32_t direction;  /* gr_direction: how FrontierActivate reaches the out-neighbours of C_t */
   uint32_t pull_div;  /* GR_DIR_AUTO: pull when |C_t| * pull_div > |V|; 0 = library default (16) */
+  float tolerance;    /* GR_PAGERANK_DELTA: a vertex changes when |R_new - R_old| > tolerance / n (>= 0) */
   int32_t zero_copy;  /* streamed mode: how a superstep reads the active shards' edges —
                          0 auto (in place over the host link when the frontier's edges are
                          < 1/8 of the active shards' edges, else DMA whole shards into the

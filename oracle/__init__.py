@@ -22,7 +22,7 @@ _SO = os.path.join(_HERE, "liboracle.so")
 _SRC = os.path.join(_HERE, "oracle.c")
 _lib = None
 
-ALGOS = {"bfs": 0, "sssp": 1, "pagerank": 2, "cc": 3, "widest": 4}
+ALGOS = {"bfs": 0, "sssp": 1, "pagerank": 2, "cc": 3, "widest": 4, "pagerank_delta": 5}
 INF = 0xFFFFFFFF
 
 
@@ -48,7 +48,7 @@ def lib():
         L.or_graph_free.argtypes = [ctypes.c_void_p]
         L.or_run.restype = ctypes.c_int64
         L.or_run.argtypes = [ctypes.c_void_p, ctypes.c_int, ctypes.c_uint32, ctypes.c_uint32,
-                             ctypes.c_double, ctypes.c_void_p, ctypes.POINTER(ctypes.c_uint64),
+                             ctypes.c_double, ctypes.c_double, ctypes.c_void_p, ctypes.POINTER(ctypes.c_uint64),
                              ctypes.c_uint64, ctypes.POINTER(ctypes.c_uint64)]
         _lib = L
     return _lib
@@ -77,19 +77,22 @@ class OracleGraph:
         self._h = h
 
     def run(self, algo: str, source: int = 0, max_iters: int = 0, damping: float = 0.85,
-            trace_cap: int = 1 << 20):
-        """Return (values, trace[rows,4], iterations)."""
+            trace_cap: int = 1 << 20, tolerance: float = 1e-4):
+        """Return (values, trace[rows,4], iterations). pagerank_delta values are
+        float32 (the fp32 ranks); pagerank values are float64."""
         a = ALGOS[algo]
         if algo == "pagerank" and max_iters == 0:
             max_iters = 30
         vals = np.empty(self.n, np.float64 if algo == "pagerank" else np.uint32)
         tr = np.zeros((trace_cap, 4), np.uint64)
         rows = ctypes.c_uint64(0)
-        it = lib().or_run(self._h, a, source, max_iters, damping, vals.ctypes.data_as(ctypes.c_void_p),
+        it = lib().or_run(self._h, a, source, max_iters, damping, tolerance, vals.ctypes.data_as(ctypes.c_void_p),
                           tr.ctypes.data_as(ctypes.POINTER(ctypes.c_uint64)), trace_cap,
                           ctypes.byref(rows))
         if it < 0:
             raise ValueError(f"or_run failed rc={it}")
+        if algo == "pagerank_delta":
+            vals = vals.view(np.float32)
         return vals, tr[: min(rows.value, trace_cap)].copy(), int(it)
 
     def close(self):

@@ -10,7 +10,7 @@
 extern "C" {
 #endif
 
-enum { OR_BFS = 0, OR_SSSP = 1, OR_PAGERANK = 2, OR_CC = 3, OR_WIDEST = 4 };
+enum { OR_BFS = 0, OR_SSSP = 1, OR_PAGERANK = 2, OR_CC = 3, OR_WIDEST = 4, OR_PRDELTA = 5 };
 #define OR_INF 0xFFFFFFFFu
 
 typedef struct or_graph or_graph;
@@ -23,7 +23,14 @@ or_graph *or_graph_build(uint64_t n, uint64_t m, const uint32_t *src, const uint
 void or_graph_free(or_graph *g);
 
 /* Run one program to termination (or max_iters supersteps; 0 = unlimited).
- * values_out: uint32_t[n] for BFS/SSSP/CC/WIDEST, double[n] for PAGERANK.
+ * values_out: uint32_t[n] for BFS/SSSP/CC/WIDEST, double[n] for PAGERANK,
+ * uint32_t[n] fp32 bit patterns for PRDELTA.
+ * OR_PRDELTA: tolerance-driven PageRank (Figs. 16-17,
+ * L360-372): A_0 = V; a vertex changes (and only then takes its new rank) when
+ * |R_new - R_old| > tolerance / n. Ranks are fp32; the gather is the exact sum
+ * of floor(fix(R_u) / n_u) in 2^-62 fixed point, fix(R) = floor(R * 2^62);
+ * R_new = fp32(double(floor(((2^20 - q) << 42) / n) + floor(S * q / 2^20)) * 2^-62),
+ * q = round(d * 2^20) of the fp32 damping d.
  * OR_WIDEST: single-source widest path (max over paths of the min edge weight),
  * a user GAS program (§4.1) used to check GR_CUSTOM programs.
  * trace_out (nullable): rows of 4 uint64 per superstep t:
@@ -31,7 +38,8 @@ void or_graph_free(or_graph *g);
  *   sum_{u in C_t} outdeg(u) (0 when FrontierActivate is eliminated).
  * Returns the number of supersteps executed, or <0 on error. */
 int64_t or_run(or_graph *g, int algo, uint32_t source, uint32_t max_iters, double damping,
-               void *values_out, uint64_t *trace_out, uint64_t trace_cap, uint64_t *rows_out);
+               double tolerance, void *values_out, uint64_t *trace_out, uint64_t trace_cap,
+               uint64_t *rows_out);
 
 #ifdef __cplusplus
 }

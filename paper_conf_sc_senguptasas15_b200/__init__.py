@@ -23,7 +23,8 @@ _lib = None
 GR_OK, GR_EINVAL, GR_ENOMEM, GR_ECUDA, GR_ENCCL, GR_EUNSUPPORTED, GR_ESTATE = range(7)
 STATUS_NAMES = ["GR_OK", "GR_EINVAL", "GR_ENOMEM", "GR_ECUDA", "GR_ENCCL", "GR_EUNSUPPORTED", "GR_ESTATE"]
 GR_FMT_COO, GR_FMT_CSR = 0, 1
-ALGOS = {"bfs": 0, "sssp": 1, "pagerank": 2, "cc": 3, "custom": 4}
+ALGOS = {"bfs": 0, "sssp": 1, "pagerank": 2, "cc": 3, "custom": 4, "pagerank_delta": 5}
+FLOAT_ALGOS = ("pagerank", "pagerank_delta")
 MODES = {"auto": 0, "resident": 1, "streamed": 2}
 LOOPS = {"auto": 0, "host": 1, "device": 2, "persistent": 3}
 BUILDS = {"auto": 0, "host": 1, "device": 2}
@@ -60,7 +61,7 @@ class gr_run_opts(ctypes.Structure):
     _fields_ = [("algo", ctypes.c_int32), ("source", ctypes.c_uint32), ("max_iters", ctypes.c_uint32),
                 ("damping", ctypes.c_float), ("custom_id", ctypes.c_int32), ("loop", ctypes.c_int32),
                 ("stream", ctypes.c_void_p), ("profile", ctypes.c_int32), ("direction", ctypes.c_int32),
-                ("pull_div", ctypes.c_uint32), ("zero_copy", ctypes.c_int32)]
+                ("pull_div", ctypes.c_uint32), ("tolerance", ctypes.c_float), ("zero_copy", ctypes.c_int32)]
 
 
 class gr_run_stats(ctypes.Structure):
@@ -237,7 +238,7 @@ def gr_graph_load_file(path, **opts):
 
 
 def gr_run(h, algo, source=0, max_iters=0, damping=0.85, custom_id=0, loop="auto", stream=None,
-           profile=False, direction="auto", pull_div=0, zero_copy=0) -> dict:
+           profile=False, direction="auto", pull_div=0, zero_copy=0, tolerance=1e-4) -> dict:
     o = gr_run_opts()
     o.algo = ALGOS[algo] if isinstance(algo, str) else int(algo)
     o.source, o.max_iters, o.damping, o.custom_id = int(source), int(max_iters), float(damping), int(custom_id)
@@ -247,6 +248,7 @@ def gr_run(h, algo, source=0, max_iters=0, damping=0.85, custom_id=0, loop="auto
     o.direction = DIRECTIONS[direction] if isinstance(direction, str) else int(direction)
     o.pull_div = int(pull_div)
     o.zero_copy = int(zero_copy)
+    o.tolerance = float(tolerance)
     st = gr_run_stats()
     _check(lib().gr_run(h, ctypes.byref(o), ctypes.byref(st)))
     return st.as_dict()
@@ -349,7 +351,7 @@ class GraphReduce:
         return gr_run(self.h, algo, **kw)
 
     def values(self, algo=None):
-        dt = np.float32 if algo == "pagerank" else np.uint32
+        dt = np.float32 if algo in FLOAT_ALGOS else np.uint32
         return gr_fetch_vertex_values(self.h, dtype=dt)
 
     def trace(self):

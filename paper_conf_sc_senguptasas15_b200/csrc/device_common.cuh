@@ -57,6 +57,9 @@ struct Ctl {
   uint32_t dirty[2];      // changed-bitmap b holds bits of an earlier pull and must be cleared
   uint32_t tot_pull;      // supersteps that activated by pull
   uint32_t dense;         // superstep `iter` gathers densely (previous activation was by pull)
+  uint32_t prd_r0;        // ProgPRDelta constants (Ctx)
+  unsigned long long prd_base, prd_dq;
+  double prd_thr;
 };
 
 constexpr int kSlots = 64;
@@ -82,6 +85,8 @@ struct View {
   uint32_t cntA[2], cntK[2], cntH[2], cntC, cntCH, cntKC;
   uint32_t pull_div, pull_pending, dirty[2], dense;
   float damping;
+  unsigned long long prd_base, prd_dq;
+  double prd_thr;
 };
 
 __device__ __forceinline__ void load_view(const Ctl *c, View &v) {
@@ -97,6 +102,7 @@ __device__ __forceinline__ void load_view(const Ctl *c, View &v) {
     const uint32_t pd = vc->pull_div, pp = vc->pull_pending, d0 = vc->dirty[0], d1 = vc->dirty[1], dn = vc->dense;
     v.cntH[0] = h0; v.cntH[1] = h1; v.cntCH = ch;
     v.pull_div = pd; v.pull_pending = pp; v.dirty[0] = d0; v.dirty[1] = d1; v.dense = dn;
+    v.prd_base = vc->prd_base; v.prd_dq = vc->prd_dq; v.prd_thr = vc->prd_thr;
     v.cntA[0] = a0; v.cntA[1] = a1; v.cntK[0] = k0; v.cntK[1] = k1;
     v.stop = st; v.t = t; v.epoch_base = eb; v.implicit0 = im; v.no_hub_c = nh;
     v.source = so; v.cntC = cc; v.cntKC = kc; v.damping = dm; v.prof = pr;
@@ -139,7 +145,9 @@ template <class OffT> struct Part {
   uint32_t *CH_v, *CH_val;// changed list (activation hubs)
   uint32_t *chkA_h[2], *chkA_c[2]; // A_t hub chunks: (position in listH, chunk index)
   uint32_t *chkC_h, *chkC_c;       // changed-hub chunks: (position in CH list, chunk index)
-  uint32_t *hub_acc, *hub_done;    // per A-hub position: chunk-combined gather result, chunks done
+  unsigned long long *hub_acc;     // per A-hub position: chunk-combined gather result (GatherT, 8 B slots)
+  uint32_t *hub_done;              // per A-hub position: chunks done
+  const uint32_t *outdeg;          // out-degree of every vertex (Ctx::outdeg)
   uint32_t *cbits[2];     // changed-set bitmaps over V for pull activation (by superstep parity)
   uint32_t *hub_act;      // per static hub: some chunk saw a marked source (dense gathers)
   const uint32_t *s_hubs, *s_chk_h, *s_chk_c;  // static in-hub list and its chunks (dense gathers)

@@ -191,7 +191,7 @@ gr_status load_device(gr_graph *g) {
   if ((s = dev_alloc(g, (void **)&g->chkC_h, 4 * std::max<uint64_t>(chunks_out, 1))) != GR_OK) return s;
   if ((s = dev_alloc(g, (void **)&g->chkC_c, 4 * std::max<uint64_t>(chunks_out, 1))) != GR_OK) return s;
   g->hub_cap = (uint32_t)std::max<uint64_t>(std::max(hubs_in, hubs_out), 1);
-  if ((s = dev_alloc(g, (void **)&g->hub_acc, 4ull * g->hub_cap)) != GR_OK) return s;
+  if ((s = dev_alloc(g, (void **)&g->hub_acc, 8ull * g->hub_cap)) != GR_OK) return s;
   if ((s = dev_alloc(g, (void **)&g->hub_done, 4ull * g->hub_cap)) != GR_OK) return s;
   CK(cudaMemsetAsync(g->hub_done, 0, 4ull * g->hub_cap, g->stream));
   if ((s = dev_alloc(g, (void **)&g->hub_act, 4ull * g->hub_cap)) != GR_OK) return s;
@@ -356,6 +356,7 @@ static gr_status run_frontier(gr_graph *g, const gr_run_opts *o, cudaStream_t s,
   h.damping = o->damping;
   h.prof = o->profile ? 1 : 0;
   h.kstart[0] = h.kstart[1] = ~0ull;
+  prd_setup(h, o, g->H.n);
   // activation direction (gr_direction); pull needs the bitmaps (resident, one rank)
   if (g->cbits[0] && o->direction != GR_DIR_PUSH) {
     uint32_t div = o->pull_div ? o->pull_div : kPullDivDefault;
@@ -366,8 +367,8 @@ static gr_status run_frontier(gr_graph *g, const gr_run_opts *o, cudaStream_t s,
   }
   CK(cudaMemcpyAsync(g->ctl, &h, sizeof h, cudaMemcpyHostToDevice, s));
   k_init_values<Prog, OffT><<<g->num_sms * 4, 256, 0, s>>>(P, o->source);
-  k_fill_u32<<<std::min<uint32_t>((g->hub_cap + 255) / 256, 1024), 256, 0, s>>>(g->hub_acc, Prog::identity_host(),
-                                                                                 g->hub_cap);
+  k_fill<typename Prog::GatherT><<<std::min<uint32_t>((g->hub_cap + 255) / 256, 1024), 256, 0, s>>>(
+      reinterpret_cast<typename Prog::GatherT *>(g->hub_acc), Prog::identity_host(), g->hub_cap);
   CK(cudaMemsetAsync(g->hub_done, 0, 4ull * g->hub_cap, s));
   launches += 2;
   if (Prog::kInit == kInitAll && g->n_static_hubs) {
@@ -625,12 +626,13 @@ gr_status run(gr_graph *g, const gr_run_opts *oin, gr_run_stats *st) {
   gr_run_opts o = *oin;
   if (o.damping == 0.f) o.damping = 0.85f;
   if (o.algo == GR_PAGERANK && o.max_iters == 0) o.max_iters = 30;
-  if (o.algo == GR_PAGERANK && !(o.damping > 0.f && o.damping < 1.f))
+  if ((o.algo == GR_PAGERANK || o.algo == GR_PAGERANK_DELTA) && !(o.damping > 0.f && o.damping < 1.f))
     return fail(GR_EINVAL, "damping must lie in (0, 1)");
+  if (o.algo == GR_PAGERANK_DELTA && !(o.tolerance >= 0.f)) return fail(GR_EINVAL, "tolerance must be >= 0");
   if ((o.algo == GR_BFS || o.algo == GR_SSSP) && o.source >= g->H.n)
     return fail(GR_EINVAL, "source %u >= num_vertices %llu", o.source, (unsigned long long)g->H.n);
   if (o.algo == GR_SSSP && !g->H.has_w) return fail(GR_EINVAL, "SSSP needs edge weights");
-  if (o.algo < GR_BFS || o.algo > GR_CUSTOM) return fail(GR_EINVAL, "unknown algo %d", o.algo);
+  if (o.algo < GR_BFS || o.algo > GR_PAGERANK_DELTA) return fail(GR_EINVAL, "unknown algo %d", o.algo);
   if (o.direction < GR_DIR_AUTO || o.direction > GR_DIR_PULL) return fail(GR_EINVAL, "unknown direction %d", o.direction);
   if (o.algo == GR_CUSTOM) {
     bool known = false, uses_w = false;
@@ -666,6 +668,10 @@ gr_status run(gr_graph *g, const gr_run_opts *oin, gr_run_stats *st) {
       break;
     case GR_CC:
       r = g->off64 ? run_frontier<ProgCC, uint64_t>(g, &o, s, st, 3) : run_frontier<ProgCC, uint32_t>(g, &o, s, st, 3);
+      break;
+    case GR_PAGERANK_DELTA:
+      r = g->off64 ? run_frontier<ProgPRDelta, uint64_t>(g, &o, s, st, 5)
+                   : run_frontier<ProgPRDelta, uint32_t>(g, &o, s, st, 5);
       break;
     case GR_CUSTOM:
       r = GR_EUNSUPPORTED;

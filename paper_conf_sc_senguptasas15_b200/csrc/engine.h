@@ -1,5 +1,7 @@
 // engine.h — internal state of a loaded graph (the opaque gr_graph).
 #pragma once
+#include <cmath>
+#include <cstring>
 #include <cuda_runtime.h>
 
 #include <map>
@@ -31,7 +33,8 @@ struct gr_graph {
   // hub chunk lists (kChunk edges per CTA work item)
   uint32_t *chkA_h[2] = {nullptr, nullptr}, *chkA_c[2] = {nullptr, nullptr};
   uint32_t *chkC_h = nullptr, *chkC_c = nullptr;
-  uint32_t *hub_acc = nullptr, *hub_done = nullptr;
+  unsigned long long *hub_acc = nullptr;  // 8-byte slots (GatherT of any program)
+  uint32_t *hub_done = nullptr;
   uint32_t *cbits[2] = {nullptr, nullptr};  // changed-set bitmaps (pull activation)
   uint32_t *hub_act = nullptr;
   size_t cbits_words = 0;
@@ -117,6 +120,7 @@ template <class OffT> inline Part<OffT> make_part(gr_graph *g) {
   for (int i = 0; i < 2; i++) { P.chkA_h[i] = g->chkA_h[i]; P.chkA_c[i] = g->chkA_c[i]; }
   P.chkC_h = g->chkC_h; P.chkC_c = g->chkC_c;
   P.hub_acc = g->hub_acc; P.hub_done = g->hub_done;
+  P.outdeg = g->d_outdeg;
   P.cbits[0] = g->cbits[0]; P.cbits[1] = g->cbits[1];
   P.hub_act = g->hub_act;
   P.s_hubs = g->static_hubs; P.s_chk_h = g->static_chk_h; P.s_chk_c = g->static_chk_c;
@@ -124,6 +128,16 @@ template <class OffT> inline Part<OffT> make_part(gr_graph *g) {
   P.ctl = g->ctl;
   P.trace = g->trace;
   return P;
+}
+
+// ProgPRDelta constants (gr/program.cuh), from the fp32 options
+inline void prd_setup(Ctl &h, const gr_run_opts *o, uint64_t n) {
+  const unsigned long long dq = (unsigned long long)llround((double)o->damping * 1048576.0);
+  h.prd_dq = dq;
+  h.prd_base = (((1ull << 20) - dq) << 42) / n;
+  h.prd_thr = (double)o->tolerance / (double)n;
+  const float r0 = (float)((double)((1ull << 62) / n) * 0x1p-62);
+  std::memcpy(&h.prd_r0, &r0, 4);
 }
 
 gr_status fail(gr_status s, const char *fmt, ...);

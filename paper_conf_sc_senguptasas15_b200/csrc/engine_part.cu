@@ -82,11 +82,12 @@ gr_status run_frontier_part(gr_graph *g, const gr_run_opts *o, cudaStream_t s, g
   h.damping = o->damping;
   h.ext_loop = 1;
   h.no_hub_c = 1;
+  prd_setup(h, o, g->H.n);
   h.kstart[0] = h.kstart[1] = ~0ull;
   PCK(cudaMemcpyAsync(g->ctl, &h, sizeof h, cudaMemcpyHostToDevice, s));
   k_init_values<Prog, OffT><<<g->num_sms * 4, 256, 0, s>>>(P, o->source);
-  k_fill_u32<<<std::min<uint32_t>((g->hub_cap + 255) / 256, 1024), 256, 0, s>>>(g->hub_acc, Prog::identity_host(),
-                                                                                 g->hub_cap);
+  k_fill<typename Prog::GatherT><<<std::min<uint32_t>((g->hub_cap + 255) / 256, 1024), 256, 0, s>>>(
+      reinterpret_cast<typename Prog::GatherT *>(g->hub_acc), Prog::identity_host(), g->hub_cap);
   PCK(cudaMemsetAsync(g->hub_done, 0, 4ull * g->hub_cap, s));
   if (Prog::kInit == kInitAll && g->n_static_hubs) {
     PCK(cudaMemcpyAsync(g->listH[0], g->static_hubs, 4ull * g->n_static_hubs, cudaMemcpyDeviceToDevice, s));
@@ -267,6 +268,9 @@ gr_status run_part(gr_graph *g, const gr_run_opts *o, cudaStream_t s, gr_run_sta
                       : run_frontier_part<ProgSSSP, uint32_t>(g, o, s, st);
     case GR_CC:
       return g->off64 ? run_frontier_part<ProgCC, uint64_t>(g, o, s, st) : run_frontier_part<ProgCC, uint32_t>(g, o, s, st);
+    case GR_PAGERANK_DELTA:
+      return g->off64 ? run_frontier_part<ProgPRDelta, uint64_t>(g, o, s, st)
+                      : run_frontier_part<ProgPRDelta, uint32_t>(g, o, s, st);
     case GR_CUSTOM:
 #define GR_X(id, T)                                                                                         \
   if (o->custom_id == id)                                                                                   \

@@ -32,6 +32,20 @@ constexpr int kPullScan = 1;   // BFS: in-edge scan of every vertex for a C_t so
 constexpr int kPullDense = 2;  // gather programs: C_t marked only; superstep t+1 gathers densely
 
 // ----------------------------------------------------------------- helpers
+template <class OffT> __device__ __forceinline__ Ctx make_ctx(const Part<OffT> &P, const View &V) {
+  Ctx cx;
+  cx.iter = V.t;
+  cx.n = P.n;
+  cx.source = V.source;
+  cx.damping = V.damping;
+  cx.outdeg = P.outdeg;
+  cx.prd_base = V.prd_base;
+  cx.prd_dq = V.prd_dq;
+  cx.prd_thr = V.prd_thr;
+  cx.prd_r0 = 0;
+  return cx;
+}
+
 template <class Prog>
 __device__ __forceinline__ typename Prog::GatherT warp_reduce_prog(typename Prog::GatherT x) {
 #pragma unroll
@@ -39,13 +53,6 @@ __device__ __forceinline__ typename Prog::GatherT warp_reduce_prog(typename Prog
   return x;
 }
 
-template <class Prog, class OffT>
-__device__ __forceinline__ typename Prog::GatherT map_edge(const Part<OffT> &P, uint64_t e, uint32_t dval,
-                                                           const Ctx &cx) {
-  uint32_t u = ldg_nc(P.in_src + e);
-  uint32_t w = Prog::kUsesWeights ? (uint32_t)ldg_nc_u8(P.in_w + e) : 0u;
-  return Prog::gatherMap(dval, P.val[u], w, cx);
-}
 
 // Gather for up to 32 vertices held one per lane (valid, beg, deg, dval).
 // Returns the gatherReduce result of the lane's own vertex. kDense (pull
@@ -53,8 +60,8 @@ __device__ __forceinline__ typename Prog::GatherT map_edge(const Part<OffT> &P, 
 // (the changed set of the previous superstep), i.e. the vertex is in A_t.
 template <class Prog, bool kDense, class OffT>
 __device__ typename Prog::GatherT gather_warp(const Part<OffT> &P, bool valid, uint64_t beg, uint32_t deg,
-                                              uint32_t dval, uint32_t *sred, const Ctx &cx, const uint32_t *bits,
-                                              bool &act) {
+                                              uint32_t dval, typename Prog::GatherT *sred, const Ctx &cx,
+                                              const uint32_t *bits, bool &act) {
   using G = typename Prog::GatherT;
   const uint32_t lane = lane_id();
   G acc = Prog::identity();
@@ -85,14 +92,14 @@ __device__ typename Prog::GatherT gather_warp(const Part<OffT> &P, bool valid, u
       }
 #pragma unroll
       for (int q = 0; q < 4; q++) {
-        r = Prog::gatherReduce(r, Prog::gatherMap(dv, v[q], w[q], cx));
+        r = Prog::gatherReduce(r, Prog::gatherMap(dv, v[q], w[q], u[q], cx));
         if (kDense) hit |= (bw[q] >> (u[q] & 31)) & 1u;
       }
     }
     for (; k < d; k += 32) {
       const uint32_t u = ldg_nc(P.in_src + b + k);
       const uint32_t w = Prog::kUsesWeights ? (uint32_t)ldg_nc_u8(P.in_w + b + k) : 0u;
-      r = Prog::gatherReduce(r, Prog::gatherMap(dv, P.val[u], w, cx));
+      r = Prog::gatherReduce(r, Prog::gatherMap(dv, P.val[u], w, u, cx));
       if (kDense) hit |= test_bit_cg(bits, u);
     }
     r = warp_reduce_prog<Prog>(r);
@@ -153,7 +160,7 @@ __device__ typename Prog::GatherT gather_warp(const Part<OffT> &P, bool valid, u
         for (int dd = 16; dd > 0; dd >>= 1) m |= __shfl_xor_sync(0xffffffffu, m, dd);
         hitmask |= m;
       }
-      G x = act_q[q] ? Prog::gatherMap(dv[q], sv[q], sw[q], cx) : Prog::identity();
+      G x = act_q[q] ? Prog::gatherMap(dv[q], sv[q], sw[q], su[q], cx) : Prog::identity();
       // segmented inclusive scan keyed by owner lane (owners are non-decreasing)
       const int prev_o = __shfl_up_sync(0xffffffffu, o, 1);
       uint32_t f = (lane == 0 || prev_o != o) ? 1u : 0u;
@@ -204,14 +211,14 @@ __device__ typename Prog::GatherT gather_block(const Part<OffT> &P, uint64_t beg
     }
 #pragma unroll
     for (int q = 0; q < 4; q++) {
-      r = Prog::gatherReduce(r, Prog::gatherMap(dval, v[q], w[q], cx));
+      r = Prog::gatherReduce(r, Prog::gatherMap(dval, v[q], w[q], u[q], cx));
       if (kDense) hit |= (bw[q] >> (u[q] & 31)) & 1u;
     }
   }
   for (; k < deg; k += kBlock) {
     const uint32_t u = ldg_nc(P.in_src + beg + k);
     const uint32_t w = Prog::kUsesWeights ? (uint32_t)ldg_nc_u8(P.in_w + beg + k) : 0u;
-    r = Prog::gatherReduce(r, Prog::gatherMap(dval, P.val[u], w, cx));
+    r = Prog::gatherReduce(r, Prog::gatherMap(dval, P.val[u], w, u, cx));
     if (kDense) hit |= test_bit_cg(bits, u);
   }
   if (kDense) {
@@ -631,7 +638,7 @@ __device__ __forceinline__ void gather_phase(const Part<OffT> &P, const View &V)
   Ctl *ctl = P.ctl;
   const uint32_t t = V.t;
   const uint32_t slot = t & 1u;
-  const Ctx cx{t, P.n, V.source, V.damping};
+  const Ctx cx = make_ctx(P, V);
   const bool implicit = kDense || (V.implicit0 && t == 0);
   const uint32_t nA = implicit ? P.own_n : V.cntA[slot];
   const uint32_t nK = kDense ? P.n_s_chunks : V.cntK[slot];
@@ -644,7 +651,7 @@ __device__ __forceinline__ void gather_phase(const Part<OffT> &P, const View &V)
   prof_begin(ctl, V, 0);
 
   __shared__ uint32_t sq[kWarpsPerBlock][2][kQueueCap];
-  __shared__ uint32_t sred[kWarpsPerBlock][32];
+  __shared__ G sred[kWarpsPerBlock][32];
   __shared__ G sblk[kWarpsPerBlock];
   __shared__ uint32_t s_h;
   __shared__ bool s_act;
@@ -716,13 +723,13 @@ __device__ __forceinline__ void gather_phase(const Part<OffT> &P, const View &V)
       bool hact = kDense ? s_act : true;
       G acc = r;
       if (!fin) {
-        Prog::atomicGather(P.hub_acc + hp, r);
+        Prog::atomicGather(reinterpret_cast<G *>(P.hub_acc) + hp, r);
         if (kDense && s_act) atomicOr(P.hub_act + hp, 1u);
         __threadfence();
         fin = (atomicAdd(P.hub_done + hp, 1u) == nch - 1);
         if (fin) {
           __threadfence();
-          acc = atomicExch(P.hub_acc + hp, Prog::identity());
+          acc = atomicExch(reinterpret_cast<G *>(P.hub_acc) + hp, Prog::identity());
           if (kDense) hact = atomicExch(P.hub_act + hp, 0u) != 0;
           P.hub_done[hp] = 0;
         }
@@ -1025,9 +1032,17 @@ __global__ void __launch_bounds__(kBlock) k_classify(const __grid_constant__ Par
 // ----------------------------------------------------------- initialisation
 template <class Prog, class OffT>
 __global__ void k_init_values(const __grid_constant__ Part<OffT> P, uint32_t source) {
-  const Ctx cx{0, P.n, source, 0.f};
+  Ctx cx{};
+  cx.n = P.n;
+  cx.source = source;
+  cx.prd_r0 = P.ctl->prd_r0;
   for (uint64_t v = blockIdx.x * (uint64_t)blockDim.x + threadIdx.x; v < P.n; v += (uint64_t)gridDim.x * blockDim.x)
     P.val[v] = Prog::initValue((uint32_t)v, cx);
+}
+
+template <class T> __global__ void k_fill(T *p, T value, uint64_t count) {
+  for (uint64_t i = blockIdx.x * (uint64_t)blockDim.x + threadIdx.x; i < count; i += (uint64_t)gridDim.x * blockDim.x)
+    p[i] = value;
 }
 
 static __global__ void k_fill_u32(uint32_t *p, uint32_t value, uint64_t count) {

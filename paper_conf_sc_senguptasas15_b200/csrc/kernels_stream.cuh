@@ -35,11 +35,11 @@ __global__ void __launch_bounds__(kBlock) k_s_gather_apply(const __grid_constant
   __shared__ View V;
   load_view(ctl, V);
   const uint32_t t = V.t;
-  const Ctx cx{t, P.n, V.source, V.damping};
+  const Ctx cx = make_ctx(P, V);
   const bool implicit = V.implicit0 && t == 0;
   const uint32_t epoch_t = V.epoch_base + t;
   __shared__ uint32_t sq[kWarpsPerBlock][2][kQueueCap];
-  __shared__ uint32_t sred[kWarpsPerBlock][32];
+  __shared__ G sred[kWarpsPerBlock][32];
   __shared__ int s_any;
   if (threadIdx.x == 0) s_any = 0;
   __syncthreads();

@@ -291,6 +291,7 @@ static gr_status stream_frontier(gr_graph *g, const gr_run_opts *o, cudaStream_t
   h.trace_cap = g->trace_cap;
   h.source = o->source;
   h.damping = o->damping;
+  prd_setup(h, o, H.n);
   std::vector<uint8_t> act(P, 0);
   std::vector<uint32_t> a0;
   if (Prog::kInit == kInitSourceChanged) {
@@ -446,6 +447,10 @@ gr_status run_streamed(gr_graph *g, const gr_run_opts *o, gr_run_stats *st) {
       break;
     case GR_CC:
       r = g->off64 ? stream_frontier<ProgCC, uint64_t>(g, o, cs, st) : stream_frontier<ProgCC, uint32_t>(g, o, cs, st);
+      break;
+    case GR_PAGERANK_DELTA:
+      r = g->off64 ? stream_frontier<ProgPRDelta, uint64_t>(g, o, cs, st)
+                   : stream_frontier<ProgPRDelta, uint32_t>(g, o, cs, st);
       break;
     case GR_CUSTOM:
       r = GR_EUNSUPPORTED;

@@ -29,7 +29,7 @@ def run_sim_ranks(n, src, dst, w, G, algo, source=0, max_iters=0):
         try:
             h = gr.gr_graph_load(n, src, dst, w, world=G, rank=r, sim_ranks=G, nccl_unique_id=key)
             st = gr.gr_run(h, algo, source=source, max_iters=max_iters)
-            vals = gr.gr_fetch_vertex_values(h, dtype=np.float32 if algo == "pagerank" else np.uint32)
+            vals = gr.gr_fetch_vertex_values(h, dtype=np.float32 if algo in gr.FLOAT_ALGOS else np.uint32)
             tr = gr.gr_fetch_frontier_trace(h)
             out[r] = (st, vals, tr, gr.gr_graph_info_get(h))
         except Exception as e:  # pragma: no cover - surfaced below
@@ -49,7 +49,7 @@ def run_sim_ranks(n, src, dst, w, G, algo, source=0, max_iters=0):
 
 @pytest.mark.timeout(900)
 @pytest.mark.parametrize("G", [2, 3])
-@pytest.mark.parametrize("algo", ["bfs", "sssp", "cc", "pagerank"])
+@pytest.mark.parametrize("algo", ["bfs", "sssp", "cc", "pagerank", "pagerank_delta"])
 def test_sim_ranks_equal_oracle(G, algo):
     g = grgen.rmat(13, 16, seed=8)
     src, dst = g.src, g.dst

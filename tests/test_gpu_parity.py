@@ -70,7 +70,10 @@ def rand_graph(seed, n, m, sym=False, wmax=64):
     return src, dst, w
 
 
-@pytest.mark.parametrize("algo", ["bfs", "sssp", "cc", "pagerank"])
+ALGOS = ["bfs", "sssp", "cc", "pagerank", "pagerank_delta"]
+
+
+@pytest.mark.parametrize("algo", ALGOS)
 @pytest.mark.parametrize("seed,n,m", [(1, 1, 0), (2, 7, 20), (3, 200, 900), (4, 5000, 3000), (5, 3001, 40000)])
 def test_random_graphs(algo, seed, n, m):
     src, dst, w = rand_graph(seed, n, m, sym=(algo == "cc"))
@@ -93,7 +96,7 @@ def hub_graph(k=5000, extra=3000, seed=9):
     return n, src, dst, w
 
 
-@pytest.mark.parametrize("algo", ["bfs", "sssp", "cc", "pagerank"])
+@pytest.mark.parametrize("algo", ALGOS)
 def test_hubs(algo):
     n, src, dst, w = hub_graph()
     for s in (0, 5, n - 1):
@@ -178,7 +181,7 @@ def test_errors_through_abi():
 
 
 # ---------------------------------------------------------------- streamed mode
-@pytest.mark.parametrize("algo", ["bfs", "sssp", "cc", "pagerank"])
+@pytest.mark.parametrize("algo", ALGOS)
 @pytest.mark.parametrize("shard_edges", [3000, 40000])
 @pytest.mark.parametrize("zero_copy", [-1, 0, 1])
 def test_streamed_equals_oracle(algo, shard_edges, zero_copy):
@@ -203,7 +206,7 @@ def test_streamed_equals_oracle(algo, shard_edges, zero_copy):
             assert st["bytes_h2d"] == wb * st["edges_gathered"] + 4 * st["edges_scattered"]
 
 
-@pytest.mark.parametrize("algo", ["bfs", "sssp", "cc", "pagerank"])
+@pytest.mark.parametrize("algo", ALGOS)
 def test_streamed_hub_larger_than_shard(algo):
     n, src, dst, w = hub_graph()
     compare(n, src, dst, w, algo, source=0, loops=("host",), mode="streamed", shard_edges=2000)
@@ -341,3 +344,22 @@ def test_load_from_file(tmp_path, fmt):
                 np.testing.assert_array_equal(G.values(algo), ref)
                 np.testing.assert_array_equal(G.trace(), rtr)
     og.close()
+
+
+@pytest.mark.parametrize("tol", [0.0, 1e-6, 1e-3])
+def test_pagerank_delta_rmat_tolerances(tol):
+    """Tolerance-driven PageRank: ranks bit-identical to the
+    oracle (exact fixed-point gather) and the shrinking frontier trace equal,
+    on an R-MAT with hubs above the chunk threshold; with a tolerance the
+    supersteps activate ever fewer vertices."""
+    g = grgen.rmat(15, 16, seed=21)
+    mi = 40 if tol == 0.0 else 0
+    ref, rtr, rit = oracle.run(g.n, g.src, g.dst, "pagerank_delta", tolerance=tol, max_iters=mi)
+    with gr.GraphReduce(g.n, g.src, g.dst) as G:
+        for d in DIRS:
+            st = G.run("pagerank_delta", tolerance=tol, max_iters=mi, direction=d)
+            np.testing.assert_array_equal(G.values("pagerank_delta").view(np.uint32), ref.view(np.uint32))
+            np.testing.assert_array_equal(G.trace(), rtr)
+            assert st["iterations"] == rit
+        if tol > 0:  # the frontier shrinks (Figs. 16-17): late supersteps gather a fraction of V
+            assert rtr[-1, 0] < g.n // 4 and rtr[:, 0].min() < g.n

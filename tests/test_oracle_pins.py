@@ -456,3 +456,82 @@ def test_widest_path_prefix_min():
     vals, _, _ = oracle.run(n, src, src + 1, "widest", w=w, source=0)
     exp = np.concatenate([[INF], np.minimum.accumulate(w)]).astype(np.uint32)
     np.testing.assert_array_equal(vals, exp)
+
+
+# ------------------------------------------- tolerance-driven PageRank (f2)
+def _jacobi(n, src, dst, iters, d=0.85):
+    M = np.zeros((n, n))
+    np.add.at(M, (src, dst), 1.0)
+    out = M.sum(1)
+    M[out > 0] /= out[out > 0, None]
+    R = np.full(n, 1.0 / n)
+    for _ in range(iters):
+        R = (1 - d) / n + d * (M.T @ R)
+    return R
+
+
+@pytest.mark.parametrize("seed", range(6))
+def test_prdelta_tolerance0_is_the_jacobi_iteration(seed):
+    """tolerance 0: a vertex is skipped only when none of its sources moved, so
+    its recomputation would reproduce its value — 30 supersteps equal 30 Jacobi
+    iterations of PageRank (fp64 matrix powers) up to fp32 rounding."""
+    rng = np.random.default_rng(700 + seed)
+    n = int(rng.integers(4, 40))
+    src, dst, _ = rand_graph(rng, n, 3 * n)
+    vals, tr, it = oracle.run(n, src, dst, "pagerank_delta", max_iters=30, tolerance=0.0)
+    R = _jacobi(n, src, dst, it)
+    assert vals.dtype == np.float32
+    np.testing.assert_allclose(vals.astype(np.float64), R, atol=2e-7, rtol=2e-6)
+    assert tr[0, 0] == n and tr[0, 2] == len(src)  # A_0 = V, every in-edge gathered
+
+
+def test_prdelta_star_fixed_point_and_cycle():
+    d, k = 0.85, 3
+    n = k + 1
+    src = np.array([0] * k + list(range(1, n)), np.uint32)
+    dst = np.array(list(range(1, n)) + [0] * k, np.uint32)
+    # tolerance 0 may cycle between neighbouring fp32 values forever (every
+    # rounding is a "change"); a tolerance above one ulp terminates
+    vals, _, it = oracle.run(n, src, dst, "pagerank_delta", max_iters=500, tolerance=1e-6)
+    assert it < 500  # the frontier empties
+    leaf = (1 + d / k) / (n * (1 + d))
+    np.testing.assert_allclose(vals[1:], leaf, rtol=1e-5)
+    np.testing.assert_allclose(vals[0], (1 - d) / n + d * k * leaf, rtol=1e-5)
+    # directed cycle: R = 1/n is already the fixed point -> one superstep, nothing changes
+    n = 31
+    s = np.arange(n, dtype=np.uint32)
+    vals, tr, it = oracle.run(n, s, (s + 1) % n, "pagerank_delta", tolerance=1e-3)
+    np.testing.assert_allclose(vals, 1.0 / n, rtol=1e-6)
+    assert it == 1 and tr[0, 1] == 0
+
+
+@pytest.mark.parametrize("seed", range(6))
+def test_prdelta_tolerance_bound_vs_dense_solve(seed):
+    """With tolerance tau every vertex ends within tau/n (+ fp32 rounding) of its
+    own update f_v(R), and f is a d-contraction in the L1 norm (the columns of
+    the transition matrix sum to <= 1), so sum_v |R - R*| <= (tau + n*eps)/(1-d)
+    with R* from a dense linear solve. Larger tau never needs more supersteps."""
+    rng = np.random.default_rng(800 + seed)
+    n = int(rng.integers(6, 60))
+    src, dst, _ = rand_graph(rng, n, 4 * n)
+    Rstar = dense_pagerank_fixed_point(n, src, dst)
+    prev = None
+    for tau in (0.0, 1e-6, 1e-4, 1e-2):
+        vals, tr, it = oracle.run(n, src, dst, "pagerank_delta", max_iters=10000, tolerance=tau)
+        assert it < 10000
+        err = np.abs(vals.astype(np.float64) - Rstar).sum()
+        assert err <= (tau + n * 2e-7) / (1 - 0.85), (tau, err)
+        if prev is not None:
+            assert it <= prev + 1
+        prev = it
+        # |C_t| <= |A_t|, and A_{t+1} is exactly the out-neighbourhood of C_t (brute force)
+        assert np.all(tr[:, 1] <= tr[:, 0])
+        assert tr[0, 0] == n
+
+
+def test_prdelta_rejects_bad_parameters():
+    src = np.array([0, 1], np.uint32)
+    dst = np.array([1, 0], np.uint32)
+    for kw in ({"damping": 0.0}, {"damping": 1.0}, {"tolerance": -1.0}):
+        with pytest.raises(ValueError):
+            oracle.run(2, src, dst, "pagerank_delta", **kw)
