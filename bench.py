@@ -107,6 +107,28 @@ def make_graph(cfg: int, scale: int = 26):
     return g, w, run
 
 
+def override_algo(run, args):
+    """--algo: another program on the same graph (its own GTEPS rule, metric_edges)."""
+    if not args.algo or args.algo == run["algo"]:
+        return run
+    r = dict(run, algo=args.algo, override=True)
+    if args.algo == "pagerank":
+        r["max_iters"] = 30
+    else:
+        r.pop("max_iters", None)
+    if args.algo == "pagerank_delta":
+        r["tolerance"] = args.tolerance
+    return r
+
+
+def workload_name(cfg, run):
+    name = CONFIG_NAMES[cfg]
+    if run.get("override"):
+        extra = f", tolerance {run['tolerance']:g}" if run["algo"] == "pagerank_delta" else ""
+        name += f" [program: {run['algo']}{extra}]"
+    return name
+
+
 def metric_edges(cfg_run, stats, m):
     """GTEPS numerator (DESIGN.md §7 / SURVEY reading R15)."""
     a = cfg_run["algo"]
@@ -132,7 +154,10 @@ def cpu_oracle_sample(g, w, run, budget_s=20.0):
                         sample=f"PageRank {iters} of 30 supersteps on the full graph (m={g.m}); "
                                f"oracle CSC build not timed; {dt:.2f} s")
         t = time.perf_counter()
-        vals, tr, it = og.run(run["algo"], source=run.get("source", 0))
+        if run["algo"] == "pagerank_delta":  # bounded sample: the first 3 supersteps
+            vals, tr, it = og.run("pagerank_delta", max_iters=3, tolerance=run["tolerance"])
+        else:
+            vals, tr, it = og.run(run["algo"], source=run.get("source", 0))
         dt = time.perf_counter() - t
         edges = int(tr[:, 2].sum() + tr[:, 3].sum()) if run["algo"] != "cc" else g.m
         return dict(value=edges / dt / 1e9, unit="GTEPS", cores=1, kind="oracle",
@@ -181,6 +206,10 @@ def main():
                     help="superstep loop for frontier programs (host: profilable by ncu)")
     ap.add_argument("--direction", default="auto", choices=["auto", "push", "pull"],
                     help="FrontierActivate direction for frontier programs (auto: pull when |C_t| > |V|/16)")
+    ap.add_argument("--algo", default=None, choices=["bfs", "sssp", "cc", "pagerank", "pagerank_delta"],
+                    help="run another program on the config's graph (e.g. --config 5 --algo bfs, "
+                         "--config 2 --algo pagerank_delta)")
+    ap.add_argument("--tolerance", type=float, default=1e-4, help="pagerank_delta: |dR| threshold x n")
     args = ap.parse_args()
 
     rank = int(os.environ.get("RANK", "0"))
@@ -191,6 +220,7 @@ def main():
         if rank != 0:
             return 0
         g, w, run = make_graph(args.config, args.scale)
+        run = override_algo(run, args)
         per_step = []
         for i in range(args.warmup + args.steps):
             cb = cpu_oracle_sample(g, w, run)
@@ -201,7 +231,7 @@ def main():
         line = {"impl": "reference", "metric": "GTEPS", "value": val, "unit": "GTEPS", "n_gpus": args.gpus,
                 "steps": args.steps, "warmup": args.warmup, "higher_is_better": True, "scaling": "strong",
                 "vs_baseline": None, "dtype": "f64", "data": "synthetic",
-                "config": {"workload": CONFIG_NAMES[args.config], "impl": "single-threaded CPU oracle"},
+                "config": {"workload": workload_name(args.config, run), "impl": "single-threaded CPU oracle"},
                 "cpu_baseline": cb, "e2e": {"value": val, "unit": "GTEPS", "h2d_bytes_per_step": 0,
                                             "d2h_bytes_per_step": 0}}
         print(json.dumps(line), flush=True)
@@ -219,9 +249,16 @@ def main():
     t0 = time.perf_counter()
     g, w, run = make_graph(args.config, args.scale)
     print(f"[bench] generated {g.name}: n={g.n} m={g.m} in {time.perf_counter() - t0:.1f}s", file=sys.stderr)
+    run = override_algo(run, args)
     algo = run["algo"]
+    if algo == "sssp" and w is None:
+        import grgen
+
+        w = grgen.weights(g.m, 1, 64, seed=args.config)
     kw = dict(source=run.get("source", 0), max_iters=run.get("max_iters", 0), damping=run.get("damping", 0.85),
               loop=args.loop, direction=args.direction)
+    if algo == "pagerank_delta":
+        kw["tolerance"] = run["tolerance"]
     part = {}
     if world > 1:
         # NCCL bootstrap: rank 0 creates the unique id, the torch process group broadcasts it
@@ -303,7 +340,7 @@ def main():
     src_p = torch.from_numpy(g.src).pin_memory().numpy()
     dst_p = torch.from_numpy(g.dst).pin_memory().numpy()
     w_p = torch.from_numpy(w).pin_memory().numpy() if w is not None else None
-    out = torch.empty(n, dtype=torch.float32 if algo == "pagerank" else torch.int32).pin_memory().numpy()
+    out = torch.empty(n, dtype=torch.float32 if algo in gr.FLOAT_ALGOS else torch.int32).pin_memory().numpy()
     for i in range(args.e2e_steps):
         t0 = time.perf_counter()
         H = gr.gr_graph_load(n, src_p, dst_p, w_p, device=local_rank, mode=mode, **part)
@@ -332,8 +369,9 @@ def main():
             "metric": "GTEPS", "value": round(value, 3), "unit": "GTEPS", "n_gpus": world, "steps": args.steps,
             "warmup": args.warmup, "ms_per_step": round(ms_step, 4), "s_per_run": ms_step * 1e-3,
             "higher_is_better": True, "scaling": "strong", "vs_baseline": None,
-            "dtype": "f32" if algo == "pagerank" else "u32", "data": "synthetic",
-            "config": {"workload": CONFIG_NAMES[args.config], "n": n, "m": m, "shards": info["num_shards"],
+            "dtype": "f32" if algo == "pagerank" else ("u64+f32" if algo == "pagerank_delta" else "u32"),
+            "data": "synthetic",
+            "config": {"workload": workload_name(args.config, run), "n": n, "m": m, "shards": info["num_shards"],
                        "mode": mode, "parallelism": f"dst-interval partitions x{world}" if world > 1 else "1 GPU",
                        "l2": "inputs larger than L2 (CSC payload > 126 MB L2); no flush",
                        "iterations": stats["iterations"],
