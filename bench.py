@@ -310,7 +310,7 @@ def main():
         launches_per_step = run.get("max_iters", 30)
         bytes_per_launch = 4 * m + 16 * n
         kname = {0: "k_pr_gather_apply", 2: "k_pr_warp", 3: "k_pr_warp_hot", 4: "k_pr_warp_range",
-                 5: "k_pr_warp_range"}.get(int(stats["kernel_ms"][3]), "k_pr_gather_apply")
+                 5: "k_pr_warp_range", 6: "k_pr_warp_pipe", 7: "k_pr_seg"}.get(int(stats["kernel_ms"][3]), "k_pr_gather_apply")
     else:
         launches_per_step = max(1, stats["iterations"])
         bytes_per_launch = stats["bytes_hbm_model"] / launches_per_step

@@ -168,6 +168,11 @@ __device__ __forceinline__ uint32_t ldg_nc(const uint32_t *p) {
   asm volatile("ld.global.nc.L1::no_allocate.u32 %0, [%1];" : "=r"(v) : "l"(p));
   return v;
 }
+__device__ __forceinline__ float ldg_na(const float *p) {  // read-only, no L1 allocation, reorderable
+  float v;
+  asm("ld.global.nc.L1::no_allocate.f32 %0, [%1];" : "=f"(v) : "l"(p));
+  return v;
+}
 __device__ __forceinline__ uint8_t ldg_nc_u8(const uint8_t *p) {
   uint16_t v;
   asm volatile("ld.global.nc.L1::no_allocate.u8 %0, [%1];" : "=h"(v) : "l"(p));

@@ -12,6 +12,8 @@
 //     host (GR_LOOP_HOST).
 #include <cuda_runtime.h>
 
+#include <cub/cub.cuh>
+
 #include <algorithm>
 #include <chrono>
 #include <cstdarg>
@@ -459,20 +461,82 @@ template <class OffT> static PrArgs<OffT> pr_args(gr_graph *g, uint32_t t, uint3
   return a;
 }
 
-// Hot-source setup (once per graph): pick the kHotK vertices of largest
+// Edge-segmented layout for k_pr_seg (once per graph): item offsets
+// seg_off = scan(max(indeg, 1)), the tagged sources placed at their items
+// (an empty row's item reads the zero slot), one head bit per item, the first
+// row of every 256-item tile and the long fix-up chains.
+template <class OffT> static gr_status pr_seg_setup(gr_graph *g) {
+  const HostGraph &H = g->H;
+  cudaStream_t s = g->stream;
+  const uint32_t rows = (uint32_t)H.own_n();
+  const OffT *in_off = (const OffT *)g->in_off;
+  gr_status st;
+  if ((st = dev_alloc(g, (void **)&g->seg_off, 4ull * (rows + 1))) != GR_OK) return st;
+  uint32_t *degp = nullptr;
+  void *tmp = nullptr;
+  size_t need = 0;
+  CK(pmalloc(&degp, 4ull * std::max<uint32_t>(rows, 1), s));
+  k_seg_deg<OffT><<<g->num_sms * 8, 256, 0, s>>>(in_off, rows, degp);
+  CK(cub::DeviceScan::InclusiveSum(nullptr, need, degp, g->seg_off + 1, (int64_t)rows, s));
+  CK(pmalloc(&tmp, std::max<size_t>(need, 16), s));
+  CK(cub::DeviceScan::InclusiveSum(tmp, need, degp, g->seg_off + 1, (int64_t)rows, s));
+  CK(cudaMemsetAsync(g->seg_off, 0, 4, s));
+  uint32_t items = 0;
+  CK(cudaMemcpyAsync(&items, g->seg_off + rows, 4, cudaMemcpyDeviceToHost, s));
+  CK(cudaStreamSynchronize(s));
+  pfree(degp, s);
+  pfree(tmp, s);
+  g->seg_items = items;
+  g->seg_tiles = (uint32_t)((items + kSegTile - 1) / kSegTile);
+  const uint64_t padded = (uint64_t)g->seg_tiles * kSegTile;
+  if ((st = dev_alloc(g, (void **)&g->seg_src, 4ull * padded + 16)) != GR_OK) return st;
+  if ((st = dev_alloc(g, (void **)&g->seg_flags, 4ull * (g->seg_tiles + 2) * 8)) != GR_OK) return st;
+  if ((st = dev_alloc(g, (void **)&g->seg_row, 4ull * (g->seg_tiles + 1))) != GR_OK) return st;
+  CK(cudaMemsetAsync(g->seg_flags, 0, 4ull * (g->seg_tiles + 2) * 8, s));
+  k_seg_fill<OffT><<<g->num_sms * 16, 256, 0, s>>>(in_off, rows, H.m_in, g->pr_src, g->seg_off, g->seg_src);
+  k_seg_rows<OffT><<<g->num_sms * 8, 256, 0, s>>>(in_off, rows, g->seg_off, g->seg_src, g->seg_flags,
+                                                   kHotTag | g->hot_k, padded);
+  uint32_t *d_nlong = nullptr;
+  CK(pmalloc(&d_nlong, 4, s));
+  CK(cudaMemsetAsync(d_nlong, 0, 4, s));
+  k_seg_tiles<<<(g->seg_tiles + 255) / 256, 256, 0, s>>>(g->seg_off, rows, g->seg_tiles, g->seg_row, g->w_is_long,
+                                                         g->long_c, g->long_f, d_nlong);
+  CK(cudaGetLastError());
+  CK(cudaMemcpyAsync(&g->n_long, d_nlong, 4, cudaMemcpyDeviceToHost, s));
+  CK(cudaStreamSynchronize(s));
+  pfree(d_nlong, s);
+  return GR_OK;
+}
+
+template <class OffT>
+using SegKernel = void (*)(const PrArgs<OffT>, const uint32_t *, const uint32_t *, const uint32_t *, const float *,
+                           uint32_t, uint32_t);
+template <class OffT> static SegKernel<OffT> seg_kernel(int var) {
+  static const SegKernel<OffT> tab[16] = {
+      k_pr_seg<OffT, 0>,  k_pr_seg<OffT, 1>,  k_pr_seg<OffT, 2>,  k_pr_seg<OffT, 3>,  k_pr_seg<OffT, 4>,  k_pr_seg<OffT, 5>,
+      k_pr_seg<OffT, 6>,  k_pr_seg<OffT, 7>,  k_pr_seg<OffT, 8>,  k_pr_seg<OffT, 9>,  k_pr_seg<OffT, 10>, k_pr_seg<OffT, 11>,
+      k_pr_seg<OffT, 12>, k_pr_seg<OffT, 13>, k_pr_seg<OffT, 14>, k_pr_seg<OffT, 15>};
+  return tab[var & 15];
+}
+
+// Hot-source setup (once per graph): pick the K vertices of largest
 // out-degree (the sources of the most in-edges), tag them in a PageRank copy
 // of the CSC payload, size the persistent grid from the occupancy calculator.
 template <class OffT> static gr_status pr_hot_setup(gr_graph *g) {
   g->pr_hot = 0;
-  // kernel variant (GR_PR_KERNEL = block | warp | warphot | range | rangehot; default warphot)
-  g->pr_kernel = 3;
-  if (const char *k = getenv("GR_PR_KERNEL")) {
-    const std::string v(k);
-    g->pr_kernel = v == "block" || v == "blockhot" ? 0 : v == "warp" ? 2 : v == "warphot" ? 3 : v == "range" ? 4 : 5;
-  }
   const HostGraph &H = g->H;
   const bool hot_ok = g->mode == GR_MODE_RESIDENT && !g->comm && H.n < 0x80000000ull && H.m_in >= (1u << 20);
+  const bool seg_ok = hot_ok && (uint64_t)H.own_n() + H.m_in + 2 * kSegTile < 0xFFFFFFFFull;
+  // kernel variant (GR_PR_KERNEL = block | warp | warphot | range | rangehot | pipe | seg; default seg)
+  g->pr_kernel = seg_ok ? 7 : 3;
+  if (const char *k = getenv("GR_PR_KERNEL")) {
+    const std::string v(k);
+    g->pr_kernel = v == "block" || v == "blockhot" ? 0 : v == "warp" ? 2 : v == "warphot" ? 3 : v == "range" ? 4
+                 : v == "pipe" ? 6 : v == "seg" ? 7 : 5;
+  }
   if ((g->pr_kernel == 3 || g->pr_kernel == 5) && !hot_ok) g->pr_kernel -= 1;
+  if (g->pr_kernel == 6 && !hot_ok) g->pr_kernel = 2;
+  if (g->pr_kernel == 7 && !seg_ok) g->pr_kernel = hot_ok ? 3 : 2;
   if (g->pr_kernel == 4) {
     g->hot_smem = 32 * sizeof(PrWarpSmem);
     CK(cudaFuncSetAttribute(k_pr_warp_range<OffT, false>, cudaFuncAttributeMaxDynamicSharedMemorySize,
@@ -482,9 +546,10 @@ template <class OffT> static gr_status pr_hot_setup(gr_graph *g) {
     g->hot_grid = (uint32_t)(g->num_sms * std::max(bps, 1));
     return GR_OK;
   }
-  if (g->pr_kernel != 3 && g->pr_kernel != 5) return GR_OK;
-  uint64_t K = kHotK;
-  if (const char *hk = getenv("GR_PR_HOTK")) K = std::max<uint64_t>(4, std::min<uint64_t>(strtoull(hk, nullptr, 10), 49152));
+  if (g->pr_kernel != 3 && g->pr_kernel != 5 && g->pr_kernel != 6 && g->pr_kernel != 7) return GR_OK;
+  // the seg kernel stages nothing in shared memory: its table can be ~3x larger
+  uint64_t K = g->pr_kernel == 7 ? kSegHotK : kHotK;
+  if (const char *hk = getenv("GR_PR_HOTK")) K = std::max<uint64_t>(4, std::min<uint64_t>(strtoull(hk, nullptr, 10), 57344));
   K = std::min<uint64_t>(K, H.n);
   uint32_t *d_slot = nullptr;
   gr_status s;
@@ -495,7 +560,17 @@ template <class OffT> static gr_status pr_hot_setup(gr_graph *g) {
   CK(cudaGetLastError());
   CK(cudaStreamSynchronize(g->stream));
   int bps = 0;
-  if (g->pr_kernel == 5) {
+  if (g->pr_kernel == 7) {
+    if ((s = pr_seg_setup<OffT>(g)) != GR_OK) return s;
+    g->hot_cta = 1024;
+    g->seg_var = kSegDefaultVar;
+    if (const char *sv = getenv("GR_PR_SEG_VAR")) g->seg_var = atoi(sv) & 15;
+    // the table plus (kSegBuf) 32 floats per warp; what is left of the SM's 256 KB is L1
+    g->hot_smem = 4ull * (g->hot_k + 4) + ((g->seg_var & kSegBuf) ? 4ull * 32 * (g->hot_cta / 32) : 0);
+    CK(cudaFuncSetAttribute(seg_kernel<OffT>(g->seg_var), cudaFuncAttributeMaxDynamicSharedMemorySize,
+                            (int)g->hot_smem));
+    CK(cudaOccupancyMaxActiveBlocksPerMultiprocessor(&bps, seg_kernel<OffT>(g->seg_var), g->hot_cta, g->hot_smem));
+  } else if (g->pr_kernel == 5) {
     g->hot_smem = 4ull * g->hot_k + 32 * sizeof(PrWarpSmem);
     CK(cudaFuncSetAttribute(k_pr_warp_range<OffT, true>, cudaFuncAttributeMaxDynamicSharedMemorySize,
                             (int)g->hot_smem));
@@ -504,8 +579,13 @@ template <class OffT> static gr_status pr_hot_setup(gr_graph *g) {
     g->hot_cta = 1024;
     if (const char *ct = getenv("GR_PR_CTA")) g->hot_cta = std::max(64, std::min(1024, atoi(ct))) & ~31;
     g->hot_smem = 4ull * g->hot_k + (g->hot_cta / 32) * sizeof(PrWarpSmem);
-    CK(cudaFuncSetAttribute(k_pr_warp_hot<OffT>, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)g->hot_smem));
-    CK(cudaOccupancyMaxActiveBlocksPerMultiprocessor(&bps, k_pr_warp_hot<OffT>, g->hot_cta, g->hot_smem));
+    if (g->pr_kernel == 6) {
+      CK(cudaFuncSetAttribute(k_pr_warp_pipe<OffT>, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)g->hot_smem));
+      CK(cudaOccupancyMaxActiveBlocksPerMultiprocessor(&bps, k_pr_warp_pipe<OffT>, g->hot_cta, g->hot_smem));
+    } else {
+      CK(cudaFuncSetAttribute(k_pr_warp_hot<OffT>, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)g->hot_smem));
+      CK(cudaOccupancyMaxActiveBlocksPerMultiprocessor(&bps, k_pr_warp_hot<OffT>, g->hot_cta, g->hot_smem));
+    }
   }
   if (bps < 1) {
     g->pr_kernel = 0;  // shared-memory table does not fit: CTA merge-path kernel
@@ -521,9 +601,9 @@ static void pr_launch_iter(gr_graph *g, cudaStream_t s, uint32_t t, uint32_t ite
                            cudaEvent_t e1) {
   PrArgs<OffT> a = pr_args<OffT>(g, t, iters, d);
   const bool warp = g->pr_kernel >= 2;
-  const bool range = g->pr_kernel >= 4;
+  const bool range = g->pr_kernel == 4 || g->pr_kernel == 5;
   if (warp) a.tile_row = g->wtile_row;
-  const uint32_t tiles = warp ? g->pr_wtiles : g->pr_tiles;
+  const uint32_t tiles = g->pr_kernel == 7 ? g->seg_tiles : warp ? g->pr_wtiles : g->pr_tiles;
   const uint32_t ranges = (tiles + kRangeTiles - 1) / kRangeTiles;
   if (g->pr_hot == 1) {
     k_pr_hot_pack<<<(g->hot_k + 255) / 256, 256, 0, s>>>(a.contrib_in, g->hot_ids, g->hot_contrib, g->hot_k);
@@ -536,6 +616,13 @@ static void pr_launch_iter(gr_graph *g, cudaStream_t s, uint32_t t, uint32_t ite
       break;
     case 3:
       k_pr_warp_hot<OffT><<<g->hot_grid, g->hot_cta, g->hot_smem, s>>>(a, g->hot_contrib, g->hot_k, tiles);
+      break;
+    case 7:
+      seg_kernel<OffT>(g->seg_var)<<<g->hot_grid, g->hot_cta, g->hot_smem, s>>>(
+          a, g->seg_src, g->seg_flags, g->seg_row, g->hot_contrib, g->hot_k, tiles);
+      break;
+    case 6:
+      k_pr_warp_pipe<OffT><<<g->hot_grid, g->hot_cta, g->hot_smem, s>>>(a, g->hot_contrib, g->hot_k, tiles);
       break;
     case 4:
       k_pr_warp_range<OffT, false><<<g->hot_grid, 1024, g->hot_smem, s>>>(a, nullptr, 0, tiles);

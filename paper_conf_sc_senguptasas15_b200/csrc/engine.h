@@ -63,7 +63,7 @@ struct gr_graph {
   uint32_t *tile_row = nullptr;  // merge-path tile starts (resident: [pr_tiles+1]; streamed: per shard)
   uint32_t pr_wtiles = 0;          // warp-granular tiles (kWTile items)
   uint32_t *wtile_row = nullptr;
-  int pr_kernel = -1;              // 0 block, 2 warp, 3 warp+hot, 4 warp range, 5 warp range+hot
+  int pr_kernel = -1;              // 0 block, 2 warp, 3 warp+hot, 4 warp range, 5 warp range+hot, 6 pipe, 7 seg
   uint8_t *w_is_long = nullptr;    // warp tiles whose head row began > kShortChain tiles earlier
   uint32_t *long_c = nullptr, *long_f = nullptr, n_long = 0;
   int hot_cta = 1024;
@@ -79,6 +79,11 @@ struct gr_graph {
   float *hot_contrib = nullptr;
   uint32_t hot_k = 0, hot_grid = 0;
   size_t hot_smem = 0;
+  // edge-segmented PageRank layout (pr_kernel 7, kernels_pr.cuh k_pr_seg)
+  uint32_t *seg_src = nullptr, *seg_flags = nullptr, *seg_row = nullptr, *seg_off = nullptr;
+  uint32_t seg_tiles = 0;
+  int seg_var = 0;                 // k_pr_seg variant bits (kernels_pr.cuh)
+  uint64_t seg_items = 0;
 
   // run bookkeeping
   int last_algo = -1;

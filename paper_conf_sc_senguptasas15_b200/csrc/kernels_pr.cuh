@@ -325,10 +325,403 @@ __global__ void __launch_bounds__(1024, 1) k_pr_warp_hot(const __grid_constant__
     pr_warp_tile<OffT, true>(a, tile, S[w], s_hot);
 }
 
+// Software-pipelined warp tiles (same tiles, same hot table, same sums as
+// k_pr_warp_hot): while a warp walks tile T it already has tile T+1's source
+// ids and tile T+2's merge-path coordinates in registers, so the only
+// dependent global round trips left per tile are the contribution gathers
+// (issued together with the row-offset loads) and the apply's stores. The
+// 1/outdeg of the tile's first 32 rows is loaded before the walk.
+template <class OffT>
+__device__ __forceinline__ void pr_load_src(const PrArgs<OffT> &a, uint32_t tile, uint32_t i0, uint32_t i1,
+                                            uint32_t (&src)[kWIpt]) {
+  const uint64_t total = (uint64_t)a.own_n + a.m_in;
+  const uint64_t d0 = (uint64_t)tile * kWTile;
+  const uint64_t d1 = d0 + kWTile < total ? d0 + kWTile : total;
+  const uint64_t j0 = d0 - i0;
+  const uint32_t nj = (uint32_t)((d1 - i1) - j0);
+  const uint32_t lane = threadIdx.x & 31;
+#pragma unroll
+  for (int q = 0; q < kWIpt; q++) {
+    const uint32_t k = lane + 32u * q;
+    src[q] = k < nj ? ldg_nc(a.in_src + j0 + k) : 0u;
+  }
+}
+
+template <class OffT>
+__global__ void __launch_bounds__(1024, 1) k_pr_warp_pipe(const __grid_constant__ PrArgs<OffT> a,
+                                                         const float *hot_contrib, uint32_t hot_k,
+                                                         uint32_t num_tiles) {
+  extern __shared__ __align__(16) unsigned char smem_raw[];
+  float *s_hot = reinterpret_cast<float *>(smem_raw);
+  for (uint32_t k = threadIdx.x * 4; k < hot_k; k += blockDim.x * 4)
+    *reinterpret_cast<float4 *>(s_hot + k) = __ldg(reinterpret_cast<const float4 *>(hot_contrib + k));
+  __syncthreads();
+  const uint32_t lane = threadIdx.x & 31, w = threadIdx.x >> 5, nw = blockDim.x >> 5;
+  PrWarpSmem &S = reinterpret_cast<PrWarpSmem *>(smem_raw + 4ull * hot_k)[w];
+  const uint32_t stride = gridDim.x * nw;
+  const uint64_t total = (uint64_t)a.own_n + a.m_in;
+  uint32_t tile = blockIdx.x * nw + w;
+  if (tile >= num_tiles) return;
+  uint32_t i0 = __ldg(a.tile_row + tile), i1 = __ldg(a.tile_row + tile + 1);
+  uint32_t src[kWIpt];
+  pr_load_src(a, tile, i0, i1, src);
+  uint32_t ntile = tile + stride, n_i0 = 0, n_i1 = 0;
+  if (ntile < num_tiles) { n_i0 = __ldg(a.tile_row + ntile); n_i1 = __ldg(a.tile_row + ntile + 1); }
+  for (;;) {
+    const uint64_t d0 = (uint64_t)tile * kWTile;
+    const uint64_t d1 = d0 + kWTile < total ? d0 + kWTile : total;
+    const uint64_t j0 = d0 - i0;
+    const uint32_t ni = i1 - i0, nj = (uint32_t)((d1 - i1) - j0);
+    // 1) this tile's gathers (sources already in registers)
+    float v[kWIpt];
+#pragma unroll
+    for (int q = 0; q < kWIpt; q++) {
+      const uint32_t k = lane + 32u * q;
+      if (src[q] & kHotTag) v[q] = s_hot[src[q] & ~kHotTag];
+      else v[q] = k < nj ? __ldg(a.contrib_in + src[q]) : 0.f;
+    }
+    // 2) next tile's sources, the tile after next's coordinates, this tile's first row start and 1/outdeg
+    const uint32_t nntile = ntile + stride;
+    uint32_t nn_i0 = 0, nn_i1 = 0;
+    if (ntile < num_tiles) pr_load_src(a, ntile, n_i0, n_i1, src);
+    if (nntile < num_tiles) { nn_i0 = __ldg(a.tile_row + nntile); nn_i1 = __ldg(a.tile_row + nntile + 1); }
+    const uint64_t rowstart0 = (uint64_t)a.in_off[i0] - a.e_base;
+    const float inv0 = (!a.last && lane < ni) ? __ldg(a.inv_outdeg + a.own_lo + i0 + lane) : 0.f;
+    // 3) stage row ends and contributions
+    __syncwarp();  // the previous tile's readers are done with S
+    for (uint32_t k = lane; k <= ni; k += 32) {
+      const uint64_t r = (uint64_t)i0 + k;
+      const uint64_t e = r < a.own_n ? (uint64_t)a.in_off[r + 1] - a.e_base - j0 : (uint64_t)nj;
+      S.s_end[pr_pad(k)] = (uint32_t)(e < nj ? e : nj);
+    }
+#pragma unroll
+    for (int q = 0; q < kWIpt; q++) {
+      const uint32_t k = lane + 32u * q;
+      if (k < nj) S.s_val[pr_pad(k)] = v[q];
+    }
+    __syncwarp();
+    // 4) merge walk + segmented warp scan (as pr_warp_tile)
+    const uint32_t items = ni + nj;
+    const uint32_t dt = min(lane * kWIpt, items);
+    uint32_t lo = dt > nj ? dt - nj : 0, hi = dt < ni ? dt : ni;
+    while (lo < hi) {
+      const uint32_t p = (lo + hi) >> 1;
+      if (S.s_end[pr_pad(p)] <= dt - p - 1) lo = p + 1;
+      else hi = p;
+    }
+    uint32_t i = lo, j = dt - lo;
+    float run = 0.f;
+    const uint32_t dend = min(dt + kWIpt, items);
+#pragma unroll
+    for (int q = 0; q < kWIpt; q++) {
+      if (dt + q < dend) {
+        if (j < S.s_end[pr_pad(i)]) { run += S.s_val[pr_pad(j)]; ++j; }
+        else { S.s_tot[pr_pad(i)] = run; run = 0.f; ++i; }
+      }
+    }
+    float x = run;
+#pragma unroll
+    for (int o = 1; o < 32; o <<= 1) {
+      const float y = __shfl_up_sync(0xffffffffu, x, o);
+      const uint32_t ky = __shfl_up_sync(0xffffffffu, i, o);
+      if (lane >= (uint32_t)o && ky == i) x += y;
+    }
+    const uint32_t inext = __shfl_down_sync(0xffffffffu, i, 1);
+    const float carry = __shfl_sync(0xffffffffu, x, 31);
+    __syncwarp();
+    const bool run_end = (lane == 31) || (inext != i);
+    if (run_end && i < ni) S.s_tot[pr_pad(i)] += x;
+    __syncwarp();
+    // 5) apply
+    const bool head = (ni > 0) && (rowstart0 < j0);
+    for (uint32_t k = lane; k < ni; k += 32) {
+      if (k == 0 && head) continue;
+      const float R = a.base + a.d * S.s_tot[pr_pad(k)];
+      const uint32_t lrow = i0 + k;
+      if (a.last) a.rank[lrow] = R;
+      else a.contrib_out[a.own_lo + lrow] = R * (k < 32 ? inv0 : __ldg(a.inv_outdeg + a.own_lo + lrow));
+    }
+    if (lane == 0) {
+      a.head_row[tile] = head ? i0 : kNoRow;
+      a.head_val[tile] = head ? S.s_tot[pr_pad(0)] : 0.f;
+      a.carry_row[tile] = i1 < a.own_n ? i1 : kNoRow;
+      a.carry_val[tile] = carry;
+    }
+    if (ntile >= num_tiles) break;
+    tile = ntile;
+    i0 = n_i0;
+    i1 = n_i1;
+    ntile = nntile;
+    n_i0 = nn_i0;
+    n_i1 = nn_i1;
+  }
+}
+
+// ---------------------------------------------------------------------------
+// Edge-segmented warp tiles (`seg`, the default on resident single-GPU runs).
+// The PageRank payload is re-laid out once per graph as an item stream in CSC
+// order where every destination row owns max(indeg, 1) consecutive items (an
+// empty row gets one item reading a zero slot of the hot table), plus one head
+// bit per item marking the first item of each row. A warp tile is 256
+// consecutive items, lane L owning items 8L..8L+7, loaded with two 128-bit
+// loads. Rows are recovered from the head bits (row = first row of the tile +
+// heads so far), so there is no merge-path search and no shared-memory
+// staging: the per-lane sums run in registers, one segmented shuffle scan over
+// the 32 lane tails joins rows split between lanes, and rows split between
+// tiles go to the same head/carry fix-up as the other warp kernels. All of the
+// shared memory is left to the hot-source table (up to ~56K sources instead of
+// 16K next to the staging buffers).
+constexpr int kSegIpt = 8;
+constexpr int kSegHotK = 32768;  // hot sources of the seg kernel (128 KB of shared memory; measured best of 16K-56K)
+constexpr int kSegTile = 32 * kSegIpt;
+
+__device__ __forceinline__ float lds_f32(uint32_t saddr) {
+  float v;
+  asm("ld.shared.f32 %0, [%1];" : "=f"(v) : "r"(saddr));
+  return v;
+}
+
+// Variant bits of k_pr_seg (GR_PR_SEG_VAR; measured in profiles/README.md):
+constexpr int kSegBallot = 1;   // segment starts of the lane scan from one ballot (1 shuffle per step, not 3)
+constexpr int kSegBuf = 2;      // finished rows through a per-warp buffer: coalesced apply, 1/outdeg preloaded
+constexpr int kSegPreFlag = 4;  // head bits loaded one tile ahead
+constexpr int kSegGeneric = 8;  // hot table read through a generic pointer instead of ld.shared
+constexpr int kSegDefaultVar = kSegBallot;  // measured best of the 16 (profiles/README.md)
+
+// contributions of my 8 items: hot sources from the shared table, the rest
+// from global memory (L2-resident)
+template <int kVar>
+__device__ __forceinline__ void seg_gather(const uint4 &s0, const uint4 &s1, const float *s_hot, uint32_t hot_sbase,
+                                           const float *__restrict__ contrib, float (&v)[kSegIpt]) {
+  const uint32_t src[kSegIpt] = {s0.x, s0.y, s0.z, s0.w, s1.x, s1.y, s1.z, s1.w};
+#pragma unroll
+  for (int k = 0; k < kSegIpt; k++) {
+    if (kVar & kSegGeneric) v[k] = (src[k] & kHotTag) ? s_hot[src[k] & ~kHotTag] : __ldg(contrib + src[k]);
+    else v[k] = (src[k] & kHotTag) ? lds_f32(hot_sbase + 4u * (src[k] & ~kHotTag)) : __ldg(contrib + src[k]);
+  }
+}
+
+// One tile's reduction and apply from the gathered values v (lane L: items
+// 8L..8L+7; b = my head bits, fnext = the item after the tile starts a row).
+// No staging of items: each lane sums its items in registers, rows split
+// between lanes are joined by one segmented shuffle scan of the lane tails
+// (a segment starts at a lane holding a head), and rows split between tiles
+// get head/carry records for the fix-up kernels.
+template <class OffT, int kVar>
+__device__ __forceinline__ void seg_tile(const PrArgs<OffT> &a, uint32_t tile, uint32_t r0, uint32_t b, uint32_t fnext,
+                                         float pre_inv, const float (&v)[kSegIpt], float *s_R) {
+  const uint32_t lane = threadIdx.x & 31;
+  uint32_t bn = __shfl_down_sync(0xffffffffu, b, 1) & 1u;
+  if (lane == 31) bn = fnext;
+  const uint32_t ends = (b >> 1) | (bn << 7);  // bit k: my item k ends a row
+  // lane tail: sum after my last head (all 8 items when I have none)
+  float tail = 0.f;
+#pragma unroll
+  for (int k = 0; k < kSegIpt; k++) {
+    if ((b >> k) & 1u) tail = 0.f;
+    tail += v[k];
+  }
+  // inclusive prefix count of heads and segmented inclusive scan of the tails over lanes
+  uint32_t cnt = __popc(b);
+  float x = tail;
+  if (kVar & kSegBallot) {
+    const uint32_t hl = __ballot_sync(0xffffffffu, b != 0u) & (0xFFFFFFFFu >> (31 - lane));
+    const int seg0 = hl ? 31 - __clz(hl) : 0;
+#pragma unroll
+    for (int o = 1; o < 32; o <<= 1) {
+      const float y = __shfl_up_sync(0xffffffffu, x, o);
+      const uint32_t c = __shfl_up_sync(0xffffffffu, cnt, o);
+      if ((int)lane - o >= seg0) x += y;
+      if (lane >= (uint32_t)o) cnt += c;
+    }
+  } else {
+    uint32_t hf = b != 0u;
+#pragma unroll
+    for (int o = 1; o < 32; o <<= 1) {
+      const float y = __shfl_up_sync(0xffffffffu, x, o);
+      const uint32_t f = __shfl_up_sync(0xffffffffu, hf, o);
+      const uint32_t c = __shfl_up_sync(0xffffffffu, cnt, o);
+      if (lane >= (uint32_t)o) {
+        if (!hf) x += y;
+        hf |= f;
+        cnt += c;
+      }
+    }
+  }
+  float run = __shfl_up_sync(0xffffffffu, x, 1);
+  if (lane == 0) run = 0.f;
+  const uint32_t total_heads = __shfl_sync(0xffffffffu, cnt, 31);
+  const uint32_t h0 = __shfl_sync(0xffffffffu, b, 0) & 1u;
+  uint32_t row = r0 - h0 + (cnt - __popc(b));  // row of the item before my first head
+  const bool head_exists = !h0 && (total_heads > 0 || fnext);
+  if (lane == 0 && !head_exists) a.head_row[tile] = kNoRow;
+#pragma unroll
+  for (int k = 0; k < kSegIpt; k++) {
+    if ((b >> k) & 1u) { run = 0.f; ++row; }
+    run += v[k];
+    if (((ends >> k) & 1u) && row < a.own_n) {
+      const uint32_t idx = row - r0;
+      if (!h0 && idx == 0) {  // row r0 began in an earlier tile: fix-up
+        a.head_row[tile] = r0;
+        a.head_val[tile] = run;
+      } else if ((kVar & kSegBuf) && idx < 32u) {
+        s_R[idx] = a.base + a.d * run;
+      } else {
+        const float R = a.base + a.d * run;
+        if (a.last) a.rank[row] = R;
+        else a.contrib_out[a.own_lo + row] = R * __ldg(a.inv_outdeg + a.own_lo + row);
+      }
+    }
+  }
+  if (lane == 31) {
+    const bool open = !fnext && row < a.own_n;
+    a.carry_row[tile] = open ? row : kNoRow;
+    a.carry_val[tile] = run;
+  }
+  if (kVar & kSegBuf) {
+    __syncwarp();
+    // coalesced apply of the finished rows r0 + [first, lastc] among the tile's first 32
+    const int first = h0 ? 0 : 1;
+    const int lastc = (int)(total_heads - h0) - (fnext ? 0 : 1);
+    const uint32_t myrow = r0 + lane;
+    if ((int)lane >= first && (int)lane <= lastc && myrow < a.own_n) {
+      const float R = s_R[lane];
+      if (a.last) a.rank[myrow] = R;
+      else a.contrib_out[a.own_lo + myrow] = R * pre_inv;
+    }
+    __syncwarp();
+  }
+}
+
+template <class OffT, int kVar>
+__global__ void __launch_bounds__(1024, 1) k_pr_seg(const __grid_constant__ PrArgs<OffT> a,
+                                                   const uint32_t *__restrict__ seg_src,
+                                                   const uint32_t *__restrict__ seg_flags,
+                                                   const uint32_t *__restrict__ seg_row, const float *hot_contrib,
+                                                   uint32_t hot_k, uint32_t num_tiles) {
+  extern __shared__ __align__(16) float s_hot[];  // [hot_k + 4] table, then 32 floats per warp
+  for (uint32_t k = threadIdx.x * 4; k < hot_k; k += blockDim.x * 4)
+    *reinterpret_cast<float4 *>(s_hot + k) = __ldg(reinterpret_cast<const float4 *>(hot_contrib + k));
+  if (threadIdx.x < 4) s_hot[hot_k + threadIdx.x] = 0.f;  // the empty rows' item reads slot hot_k
+  __syncthreads();
+  const uint32_t hot_sbase = (uint32_t)__cvta_generic_to_shared(s_hot);
+  const uint32_t lane = threadIdx.x & 31, w = threadIdx.x >> 5, nw = blockDim.x >> 5;
+  float *s_R = s_hot + hot_k + 4 + 32 * w;
+  const uint32_t stride = gridDim.x * nw;
+  uint32_t tile = blockIdx.x * nw + w;
+  if (tile >= num_tiles) return;
+  const uint4 *src4 = reinterpret_cast<const uint4 *>(seg_src) + 2 * lane;
+  uint4 s0 = __ldg(src4 + (uint64_t)tile * (kSegTile / 4));
+  uint4 s1 = __ldg(src4 + (uint64_t)tile * (kSegTile / 4) + 1);
+  uint32_t r0 = __ldg(seg_row + tile);
+  uint32_t fw = 0, fnext = 0;
+  if (kVar & kSegPreFlag) {
+    fw = __ldg(seg_flags + (uint64_t)tile * 8 + (lane >> 2));
+    fnext = __ldg(seg_flags + (uint64_t)tile * 8 + 8) & 1u;
+  }
+  for (;;) {
+    if (!(kVar & kSegPreFlag)) {  // this tile's head bits, in flight together with the gathers
+      fw = __ldg(seg_flags + (uint64_t)tile * 8 + (lane >> 2));
+      fnext = __ldg(seg_flags + (uint64_t)tile * 8 + 8) & 1u;
+    }
+    float v[kSegIpt];
+    seg_gather<kVar>(s0, s1, s_hot, hot_sbase, a.contrib_in, v);
+    float pre_inv = 0.f;
+    if (kVar & kSegBuf) {
+      const uint32_t prow = r0 + lane;
+      pre_inv = (!a.last && prow < a.own_n) ? __ldg(a.inv_outdeg + a.own_lo + prow) : 0.f;
+    }
+    const uint32_t b = (fw >> ((lane & 3) * 8)) & 0xFFu;  // bit k: my item k starts a row
+    const uint32_t fn = fnext;
+    // next tile's items and first row (and head bits)
+    const uint32_t ntile = tile + stride;
+    uint32_t nr0 = 0;
+    if (ntile < num_tiles) {
+      s0 = __ldg(src4 + (uint64_t)ntile * (kSegTile / 4));
+      s1 = __ldg(src4 + (uint64_t)ntile * (kSegTile / 4) + 1);
+      nr0 = __ldg(seg_row + ntile);
+      if (kVar & kSegPreFlag) {
+        fw = __ldg(seg_flags + (uint64_t)ntile * 8 + (lane >> 2));
+        fnext = __ldg(seg_flags + (uint64_t)ntile * 8 + 8) & 1u;
+      }
+    }
+    seg_tile<OffT, kVar>(a, tile, r0, b, fn, pre_inv, v, s_R);
+    if (ntile >= num_tiles) break;
+    tile = ntile;
+    r0 = nr0;
+  }
+}
+
+// --- seg layout builders (once per graph) ---
+template <class OffT>
+__global__ void k_seg_deg(const OffT *in_off, uint32_t rows, uint32_t *degp) {
+  for (uint32_t r = blockIdx.x * blockDim.x + threadIdx.x; r < rows; r += gridDim.x * blockDim.x) {
+    const uint64_t d = (uint64_t)in_off[r + 1] - (uint64_t)in_off[r];
+    degp[r] = d ? (uint32_t)d : 1u;
+  }
+}
+
+// item of edge e = seg_off[row(e)] + (e - in_off[row(e)]); row(e) by binary search
+template <class OffT>
+__global__ void k_seg_fill(const OffT *in_off, uint32_t rows, uint64_t m, const uint32_t *pr_src,
+                           const uint32_t *seg_off, uint32_t *seg_src) {
+  for (uint64_t e = blockIdx.x * (uint64_t)blockDim.x + threadIdx.x; e < m; e += (uint64_t)gridDim.x * blockDim.x) {
+    uint32_t lo = 0, hi = rows;  // last r with in_off[r] <= e
+    while (hi - lo > 1) {
+      const uint32_t mid = (lo + hi) >> 1;
+      if ((uint64_t)in_off[mid] <= e) lo = mid;
+      else hi = mid;
+    }
+    seg_src[seg_off[lo] + (e - (uint64_t)in_off[lo])] = pr_src[e];
+  }
+}
+
+template <class OffT>
+__global__ void k_seg_rows(const OffT *in_off, uint32_t rows, const uint32_t *seg_off, uint32_t *seg_src,
+                           uint32_t *seg_flags, uint32_t zero_tag, uint64_t padded_items) {
+  const uint64_t tid = blockIdx.x * (uint64_t)blockDim.x + threadIdx.x, nt = (uint64_t)gridDim.x * blockDim.x;
+  for (uint64_t r = tid; r < rows; r += nt) {
+    const uint32_t p = seg_off[r];
+    atomicOr(seg_flags + (p >> 5), 1u << (p & 31));
+    if (in_off[r + 1] == in_off[r]) seg_src[p] = zero_tag;
+  }
+  const uint64_t total = seg_off[rows];
+  if (tid == 0) atomicOr(seg_flags + (total >> 5), 1u << (total & 31));  // sentinel: ends the last row
+  for (uint64_t i = total + tid; i < padded_items; i += nt) seg_src[i] = zero_tag;
+}
+
+
 // Long chains (a head whose row began more than kShortChain tiles earlier) are
 // listed once per graph by k_pr_long_heads and finished one warp each by
 // k_pr_fixup_long; every other head is finished by one thread (k_pr_fixup_short).
 constexpr uint32_t kShortChain = 8;
+
+static __global__ void k_seg_tiles(const uint32_t *seg_off, uint32_t rows, uint32_t num_tiles, uint32_t *seg_row,
+                            uint8_t *is_long, uint32_t *long_c, uint32_t *long_f, uint32_t *long_n) {
+  for (uint32_t c = blockIdx.x * blockDim.x + threadIdx.x; c < num_tiles; c += gridDim.x * blockDim.x) {
+    const uint64_t i0 = (uint64_t)c * kSegTile;
+    uint32_t lo = 0, hi = rows;  // last r with seg_off[r] <= i0
+    while (hi - lo > 1) {
+      const uint32_t mid = (lo + hi) >> 1;
+      if (seg_off[mid] <= i0) lo = mid;
+      else hi = mid;
+    }
+    seg_row[c] = lo;
+    const bool h0 = seg_off[lo] == i0;
+    const bool ends = (uint64_t)seg_off[lo + 1] <= i0 + kSegTile;
+    bool lng = false;
+    if (!h0 && ends) {
+      const uint32_t f = seg_off[lo] / kSegTile;
+      if (c - f > kShortChain) {
+        lng = true;
+        const uint32_t pos = atomicAdd(long_n, 1u);
+        long_c[pos] = c;
+        long_f[pos] = f;
+      }
+    }
+    is_long[c] = lng ? 1 : 0;
+  }
+}
 
 template <class OffT>
 __global__ void k_pr_long_heads(const OffT *in_off, uint64_t rows, uint64_t nnz, const uint32_t *tile_row,

@@ -249,7 +249,7 @@ def test_streamed_frontier_skips_inactive_shards():
         np.testing.assert_array_equal(G.values(), d)
 
 
-@pytest.mark.parametrize("variant", ["block", "warp", "warphot", "range", "rangehot"])
+@pytest.mark.parametrize("variant", ["block", "warp", "warphot", "range", "rangehot", "pipe", "seg"])
 def test_pagerank_kernel_variants(variant, monkeypatch):
     """Every PageRank gather variant (CTA / warp merge-path tiles, with or without
     the shared-memory hot-source table) meets the PageRank bar."""
@@ -259,7 +259,7 @@ def test_pagerank_kernel_variants(variant, monkeypatch):
     with gr.GraphReduce(g.n, g.src, g.dst) as G:
         st = G.run("pagerank")
         assert st["kernel_ms"][3] == {"block": 0, "warp": 2, "warphot": 3, "range": 4,
-                                      "rangehot": 5}[variant]
+                                      "rangehot": 5, "pipe": 6, "seg": 7}[variant]
         check_pr(G.values("pagerank"), ref, g.n)
     n, src, dst, _ = hub_graph(k=70000, extra=1_200_000)
     ref, _, _ = oracle.run(n, src, dst, "pagerank", max_iters=30)

@@ -21,7 +21,7 @@ for name, order in perms.items():
     newid = np.empty(n, np.uint32)
     newid[order] = np.arange(n, dtype=np.uint32)
     src, dst = newid[g.src], newid[g.dst]
-    for kern in ("warphot", "block"):
+    for kern in ("seg", "warphot"):
         os.environ["GR_PR_KERNEL"] = kern
         with gr.GraphReduce(n, src, dst) as G:
             s = torch.cuda.current_stream()
