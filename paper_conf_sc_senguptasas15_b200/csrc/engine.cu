@@ -511,6 +511,17 @@ template <class OffT> static gr_status pr_seg_setup(gr_graph *g) {
 template <class OffT>
 using SegKernel = void (*)(const PrArgs<OffT>, const uint32_t *, const uint32_t *, const uint32_t *, const float *,
                            uint32_t, uint32_t);
+template <class OffT>
+using SegLoopKernel = void (*)(const PrArgs<OffT>, const PrLoop);
+template <class OffT> static SegLoopKernel<OffT> seg_loop_kernel(int var) {
+  static const SegLoopKernel<OffT> tab[16] = {
+      k_pr_seg_loop<OffT, 0>,  k_pr_seg_loop<OffT, 1>,  k_pr_seg_loop<OffT, 2>,  k_pr_seg_loop<OffT, 3>,
+      k_pr_seg_loop<OffT, 4>,  k_pr_seg_loop<OffT, 5>,  k_pr_seg_loop<OffT, 6>,  k_pr_seg_loop<OffT, 7>,
+      k_pr_seg_loop<OffT, 8>,  k_pr_seg_loop<OffT, 9>,  k_pr_seg_loop<OffT, 10>, k_pr_seg_loop<OffT, 11>,
+      k_pr_seg_loop<OffT, 12>, k_pr_seg_loop<OffT, 13>, k_pr_seg_loop<OffT, 14>, k_pr_seg_loop<OffT, 15>};
+  return tab[var & 15];
+}
+
 template <class OffT> static SegKernel<OffT> seg_kernel(int var) {
   static const SegKernel<OffT> tab[16] = {
       k_pr_seg<OffT, 0>,  k_pr_seg<OffT, 1>,  k_pr_seg<OffT, 2>,  k_pr_seg<OffT, 3>,  k_pr_seg<OffT, 4>,  k_pr_seg<OffT, 5>,
@@ -570,6 +581,29 @@ template <class OffT> static gr_status pr_hot_setup(gr_graph *g) {
     CK(cudaFuncSetAttribute(seg_kernel<OffT>(g->seg_var), cudaFuncAttributeMaxDynamicSharedMemorySize,
                             (int)g->hot_smem));
     CK(cudaOccupancyMaxActiveBlocksPerMultiprocessor(&bps, seg_kernel<OffT>(g->seg_var), g->hot_cta, g->hot_smem));
+    // persistent loop: one cooperative launch for all supersteps (GR_PR_LOOP=0: one launch per phase)
+    g->pr_loop = g->coop ? 1 : 0;
+    if (const char *pl = getenv("GR_PR_LOOP")) g->pr_loop = g->coop && atoi(pl) != 0;
+    if (g->pr_loop) {
+      int lbps = 0;
+      CK(cudaFuncSetAttribute(seg_loop_kernel<OffT>(g->seg_var), cudaFuncAttributeMaxDynamicSharedMemorySize,
+                              (int)g->hot_smem));
+      CK(cudaOccupancyMaxActiveBlocksPerMultiprocessor(&lbps, seg_loop_kernel<OffT>(g->seg_var), g->hot_cta,
+                                                       g->hot_smem));
+      if (lbps < 1) g->pr_loop = 0;
+    }
+    if (g->pr_loop) {
+      g->hot_slot = d_slot;
+      if ((s = dev_alloc(g, (void **)&g->hot_split, g->hot_k + 16)) != GR_OK) return s;
+      for (int i = 0; i < 2; i++)
+        if ((s = dev_alloc(g, (void **)&g->hot_buf[i], 4ull * (g->hot_k + 4))) != GR_OK) return s;
+      if ((s = dev_alloc(g, (void **)&g->pr_bar, 64)) != GR_OK) return s;
+      CK(cudaMemsetAsync(g->pr_bar, 0, 64, g->stream));
+      k_seg_hot_split<<<(g->hot_k + 255) / 256 + 1, 256, 0, g->stream>>>(g->hot_ids, g->hot_k, g->seg_off,
+                                                                         g->hot_split);
+      CK(cudaGetLastError());
+      CK(cudaStreamSynchronize(g->stream));
+    }
   } else if (g->pr_kernel == 5) {
     g->hot_smem = 4ull * g->hot_k + 32 * sizeof(PrWarpSmem);
     CK(cudaFuncSetAttribute(k_pr_warp_range<OffT, true>, cudaFuncAttributeMaxDynamicSharedMemorySize,
@@ -662,7 +696,43 @@ static gr_status run_pagerank(gr_graph *g, const gr_run_opts *o, cudaStream_t s,
       g->prof_ev.push_back(e);
     }
   }
-  if (prof) {
+  if (g->pr_kernel == 7 && g->pr_loop) {
+    // persistent loop: init, pack of the first hot table, ONE cooperative launch for all supersteps
+    PrArgs<OffT> a = pr_args<OffT>(g, 0, iters, d);
+    PrLoop L{};
+    L.seg_src = g->seg_src;
+    L.seg_flags = g->seg_flags;
+    L.seg_row = g->seg_row;
+    L.hot_ids = g->hot_ids;
+    L.hot_slot = g->hot_slot;
+    L.hot_split = g->hot_split;
+    L.hot_buf[0] = g->hot_buf[0];
+    L.hot_buf[1] = g->hot_buf[1];
+    L.contrib[0] = g->contrib[0];
+    L.contrib[1] = g->contrib[1];
+    L.is_long = g->w_is_long;
+    L.long_c = g->long_c;
+    L.long_f = g->long_f;
+    L.n_long = g->n_long;
+    L.hot_k = g->hot_k;
+    L.num_tiles = g->seg_tiles;
+    L.iters = iters;
+    L.bar = g->pr_bar;
+    k_pr_init<<<g->num_sms * 4, 256, 0, s>>>((uint32_t)g->H.n, g->inv_outdeg, g->contrib[0]);
+    k_pr_hot_pack<<<(g->hot_k + 255) / 256, 256, 0, s>>>(g->contrib[0], g->hot_ids, g->hot_buf[0], g->hot_k);
+    if (prof) CK(cudaEventRecord(g->prof_ev[0], s));
+    void *args[] = {(void *)&a, (void *)&L};
+    CK(cudaLaunchCooperativeKernel((const void *)seg_loop_kernel<OffT>(g->seg_var), dim3(g->hot_grid),
+                                   dim3(g->hot_cta), args, g->hot_smem, s));
+    if (prof) CK(cudaEventRecord(g->prof_ev[1], s));
+    CK(cudaStreamSynchronize(s));
+    if (prof) {
+      float ms = 0;
+      CK(cudaEventElapsedTime(&ms, g->prof_ev[0], g->prof_ev[1]));
+      st->kernel_ms[0] += ms;
+    }
+    st->kernel_launches += 3;
+  } else if (prof) {
     // direct launches with a CUDA event pair around every gather launch (events
     // recorded inside a captured graph cannot be timed); the host enqueues all
     // 2*iters launches without waiting, so the device runs them back to back
@@ -702,8 +772,9 @@ static gr_status run_pagerank(gr_graph *g, const gr_run_opts *o, cudaStream_t s,
   st->iterations = iters;
   st->edges_gathered = (uint64_t)iters * g->H.m_in;
   st->edges_scattered = 0;
-  st->kernel_launches += 1 + (g->pr_hot == 1 ? 3ull : 2ull) * iters;
-  st->kernel_ms[3] = (double)g->pr_kernel;  // which PageRank gather variant ran (0 block .. 3 warp+hot)
+  if (!(g->pr_kernel == 7 && g->pr_loop)) st->kernel_launches += 1 + (g->pr_hot == 1 ? 3ull : 2ull) * iters;
+  st->kernel_ms[3] = (double)g->pr_kernel;  // which PageRank gather variant ran (0 block .. 7 seg)
+  st->kernel_ms[2] = (g->pr_kernel == 7 && g->pr_loop) ? 1.0 : 0.0;  // 1: persistent loop (kernel_ms[0] = whole loop)
   st->bytes_hbm_model = (uint64_t)iters * (4 * g->H.m_in + 12 * g->H.own_n() + 4 * g->H.n);
   g->trace_rows = iters;
   return GR_OK;

@@ -83,6 +83,10 @@ struct gr_graph {
   uint32_t *seg_src = nullptr, *seg_flags = nullptr, *seg_row = nullptr, *seg_off = nullptr;
   uint32_t seg_tiles = 0;
   int seg_var = 0;                 // k_pr_seg variant bits (kernels_pr.cuh)
+  int pr_loop = 0;                 // 1: all supersteps in one cooperative k_pr_seg_loop launch
+  uint32_t *hot_slot = nullptr, *pr_bar = nullptr;
+  uint8_t *hot_split = nullptr;
+  float *hot_buf[2] = {nullptr, nullptr};
   uint64_t seg_items = 0;
 
   // run bookkeeping

@@ -776,6 +776,149 @@ __global__ void k_pr_fixup_long(const __grid_constant__ PrArgs<OffT> a, const ui
   }
 }
 
+// ---------------------------------------------------------------------------
+// Persistent PageRank loop (resident, single GPU; the default with k_pr_seg):
+// ONE cooperative launch runs all supersteps. Per superstep t:
+//   phase 1  every CTA loads the hot table packed after superstep t-1 and
+//            reduces its tiles (seg_tile, as k_pr_seg);
+//   barrier
+//   phase 2  rows split between tiles are finished from the head/carry
+//            records (as k_pr_fixup_short / _long; split hot rows also write
+//            their packed slot), and the other hot sources' new contributions
+//            are packed for superstep t+1 (as k_pr_hot_pack);
+//   barrier.
+// Same tiles, same summation order and same values as the per-superstep
+// launches; what goes away is 3 launches per superstep.
+struct PrLoop {
+  const uint32_t *seg_src, *seg_flags, *seg_row;
+  const uint32_t *hot_ids, *hot_slot;  // packed slot -> vertex, vertex -> slot (0xFFFFFFFF: not hot)
+  const uint8_t *hot_split;            // slot's row is finished by the fix-up phase
+  float *hot_buf[2];                   // packed hot contributions, by superstep parity
+  float *contrib[2];
+  const uint8_t *is_long;
+  const uint32_t *long_c, *long_f;
+  uint32_t n_long, hot_k, num_tiles, iters;
+  uint32_t *bar;                       // [0] arrivals, [1] generation
+};
+
+__device__ __forceinline__ void pr_grid_sync(uint32_t *bar) {
+  __syncthreads();
+  if (threadIdx.x == 0) {
+    volatile uint32_t *gen = bar + 1;
+    const uint32_t g = *gen;
+    __threadfence();
+    if (atomicAdd(bar, 1u) == gridDim.x - 1) {
+      bar[0] = 0;
+      __threadfence();
+      atomicAdd(bar + 1, 1u);
+    } else {
+      while (*gen == g) __nanosleep(20);
+    }
+    __threadfence();
+  }
+  __syncthreads();
+}
+
+template <class OffT>
+__device__ __forceinline__ void pr_apply_fixup(const PrArgs<OffT> &a, const PrLoop &L, float *hot_next, uint32_t lrow,
+                                               float acc) {
+  const float R = a.base + a.d * acc;
+  const uint32_t v = a.own_lo + lrow;
+  if (a.last) {
+    a.rank[lrow] = R;
+  } else {
+    const float c = R * __ldg(a.inv_outdeg + v);
+    a.contrib_out[v] = c;
+    const uint32_t sl = __ldg(L.hot_slot + v);
+    if (sl != 0xFFFFFFFFu) hot_next[sl] = c;
+  }
+}
+
+template <class OffT, int kVar>
+__global__ void __launch_bounds__(1024, 1) k_pr_seg_loop(const __grid_constant__ PrArgs<OffT> a0,
+                                                        const __grid_constant__ PrLoop L) {
+  extern __shared__ __align__(16) float s_hot[];
+  const uint32_t hot_sbase = (uint32_t)__cvta_generic_to_shared(s_hot);
+  const uint32_t lane = threadIdx.x & 31, w = threadIdx.x >> 5, nw = blockDim.x >> 5;
+  float *s_R = s_hot + L.hot_k + 4 + 32 * w;
+  const uint32_t stride = gridDim.x * nw;
+  const uint4 *src4 = reinterpret_cast<const uint4 *>(L.seg_src) + 2 * lane;
+  const uint64_t gtid = blockIdx.x * (uint64_t)blockDim.x + threadIdx.x, gthreads = (uint64_t)gridDim.x * blockDim.x;
+  for (uint32_t t = 0; t < L.iters; t++) {
+    PrArgs<OffT> a = a0;
+    a.contrib_in = L.contrib[t & 1];
+    a.contrib_out = L.contrib[(t + 1) & 1];
+    a.last = (t + 1 == L.iters) ? 1 : 0;
+    const float *hot_cur = L.hot_buf[t & 1];
+    float *hot_next = L.hot_buf[(t + 1) & 1];
+    // ---- phase 1: tiles
+    for (uint32_t k = threadIdx.x * 4; k < L.hot_k; k += blockDim.x * 4)
+      *reinterpret_cast<float4 *>(s_hot + k) = *reinterpret_cast<const float4 *>(hot_cur + k);
+    if (threadIdx.x < 4) s_hot[L.hot_k + threadIdx.x] = 0.f;
+    __syncthreads();
+    uint32_t tile = blockIdx.x * nw + w;
+    if (tile < L.num_tiles) {
+      uint4 s0 = __ldg(src4 + (uint64_t)tile * (kSegTile / 4));
+      uint4 s1 = __ldg(src4 + (uint64_t)tile * (kSegTile / 4) + 1);
+      uint32_t r0 = __ldg(L.seg_row + tile);
+      for (;;) {
+        const uint32_t fw = __ldg(L.seg_flags + (uint64_t)tile * 8 + (lane >> 2));
+        const uint32_t fnext = __ldg(L.seg_flags + (uint64_t)tile * 8 + 8) & 1u;
+        float v[kSegIpt];
+        seg_gather<kVar>(s0, s1, s_hot, hot_sbase, a.contrib_in, v);
+        float pre_inv = 0.f;
+        if (kVar & kSegBuf) {
+          const uint32_t prow = r0 + lane;
+          pre_inv = (!a.last && prow < a.own_n) ? __ldg(a.inv_outdeg + a.own_lo + prow) : 0.f;
+        }
+        const uint32_t b = (fw >> ((lane & 3) * 8)) & 0xFFu;
+        const uint32_t ntile = tile + stride;
+        uint32_t nr0 = 0;
+        if (ntile < L.num_tiles) {
+          s0 = __ldg(src4 + (uint64_t)ntile * (kSegTile / 4));
+          s1 = __ldg(src4 + (uint64_t)ntile * (kSegTile / 4) + 1);
+          nr0 = __ldg(L.seg_row + ntile);
+        }
+        seg_tile<OffT, kVar>(a, tile, r0, b, fnext, pre_inv, v, s_R);
+        if (ntile >= L.num_tiles) break;
+        tile = ntile;
+        r0 = nr0;
+      }
+    }
+    pr_grid_sync(L.bar);
+    // ---- phase 2: rows split between tiles, hot-table pack
+    for (uint64_t c = gtid; c < L.num_tiles; c += gthreads) {
+      const uint32_t row = a.head_row[c];
+      if (row == kNoRow || L.is_long[c]) continue;
+      float acc = a.head_val[c];
+      for (int64_t p = (int64_t)c - 1; p >= 0 && a.carry_row[p] == row; p--) acc += a.carry_val[p];
+      pr_apply_fixup(a, L, hot_next, row, acc);
+    }
+    for (uint64_t i = gtid >> 5; i < L.n_long; i += gthreads >> 5) {
+      const uint32_t c = L.long_c[i], f = L.long_f[i];
+      const uint32_t row = a.head_row[c];
+      float acc = 0.f;
+      for (uint32_t p = f + lane; p < c; p += 32) acc += a.carry_val[p];
+#pragma unroll
+      for (int o = 16; o > 0; o >>= 1) acc += __shfl_xor_sync(0xffffffffu, acc, o);
+      if (lane == 0 && row != kNoRow) pr_apply_fixup(a, L, hot_next, row, a.head_val[c] + acc);
+    }
+    if (!a.last)
+      for (uint64_t k = gtid; k < L.hot_k; k += gthreads)
+        if (!L.hot_split[k]) hot_next[k] = a.contrib_out[L.hot_ids[k]];
+    pr_grid_sync(L.bar);
+  }
+}
+
+// hot_split[k] = 1 when hot slot k's row spans two or more tiles (finished by the fix-up phase)
+static __global__ void k_seg_hot_split(const uint32_t *hot_ids, uint32_t hot_k, const uint32_t *seg_off,
+                                       uint8_t *hot_split) {
+  for (uint32_t k = blockIdx.x * blockDim.x + threadIdx.x; k < hot_k; k += gridDim.x * blockDim.x) {
+    const uint32_t v = hot_ids[k];
+    hot_split[k] = (seg_off[v] / kSegTile) != ((seg_off[v + 1] - 1) / kSegTile) ? 1 : 0;
+  }
+}
+
 // Rows spanning warp tiles: one warp per tile with a head; the preceding
 // tiles' carries of the same row are summed 32 at a time (coalesced, ballot
 // for the run end) in a fixed order.

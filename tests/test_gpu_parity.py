@@ -249,10 +249,18 @@ def test_streamed_frontier_skips_inactive_shards():
         np.testing.assert_array_equal(G.values(), d)
 
 
-@pytest.mark.parametrize("variant", ["block", "warp", "warphot", "range", "rangehot", "pipe", "seg"])
+@pytest.mark.parametrize("variant", ["block", "warp", "warphot", "range", "rangehot", "pipe", "seg", "seg-launches",
+                                     "seg-var0", "seg-var15"])
 def test_pagerank_kernel_variants(variant, monkeypatch):
     """Every PageRank gather variant (CTA / warp merge-path tiles, with or without
-    the shared-memory hot-source table) meets the PageRank bar."""
+    the shared-memory hot-source table; the edge-segmented tiles in the
+    persistent loop or one launch per phase, and its variant bits) meets the
+    PageRank bar."""
+    if variant == "seg-launches":
+        monkeypatch.setenv("GR_PR_LOOP", "0")
+    elif variant.startswith("seg-var"):
+        monkeypatch.setenv("GR_PR_SEG_VAR", variant[7:])
+    variant = variant.split("-")[0]
     monkeypatch.setenv("GR_PR_KERNEL", variant)
     g = grgen.rmat(17, 16, seed=12)  # > 2^20 edges so the hot table engages
     ref, _, _ = oracle.run(g.n, g.src, g.dst, "pagerank", max_iters=30)
