@@ -202,6 +202,8 @@ def main():
     ap.add_argument("--e2e-steps", type=int, default=2)
     ap.add_argument("--scale", type=int, default=26, help="R-MAT scale for --config 5")
     ap.add_argument("--no-cpu", action="store_true")
+    ap.add_argument("--mode", default="auto", choices=["auto", "resident", "streamed"],
+                    help="auto: cfg5 streamed, others resident")
     ap.add_argument("--loop", default="auto", choices=["auto", "host", "device", "persistent"],
                     help="superstep loop for frontier programs (host: profilable by ncu)")
     ap.add_argument("--direction", default="auto", choices=["auto", "push", "pull"],
@@ -267,7 +269,7 @@ def main():
             uid.copy_(torch.frombuffer(bytearray(gr.gr_get_unique_id()), dtype=torch.uint8))
         torch.distributed.broadcast(uid, 0)
         part = dict(world=world, rank=rank, nccl_unique_id=bytes(uid.cpu().numpy().tobytes()))
-    mode = "streamed" if args.config == 5 else "resident"
+    mode = ("streamed" if args.config == 5 else "resident") if args.mode == "auto" else args.mode
     G = gr.GraphReduce(g.n, g.src, g.dst, w, device=local_rank, mode=mode, **part)
     info = G.info()
     print(f"[bench] loaded in {time.perf_counter() - t0:.1f}s total: {info}", file=sys.stderr)

@@ -475,18 +475,45 @@ constexpr int kSegIpt = 8;
 constexpr int kSegHotK = 32768;  // hot sources of the seg kernel (128 KB of shared memory; measured best of 16K-56K)
 constexpr int kSegTile = 32 * kSegIpt;
 
+// Variant bits of k_pr_seg (GR_PR_SEG_VAR; measured in profiles/README.md):
+constexpr int kSegBallot = 1;   // segment starts of the lane scan from one ballot (1 shuffle per step, not 3)
+constexpr int kSegBuf = 2;      // finished rows through a per-warp buffer: coalesced apply, 1/outdeg preloaded
+constexpr int kSegPreFlag = 4;  // head bits loaded one tile ahead
+constexpr int kSegStreamNA = 8;  // item/flag/1-outdeg streams loaded with L1::no_allocate (L1 kept for gathers)
+constexpr int kSegDefaultVar = kSegBallot;  // measured best of the 16 (profiles/README.md)
+
+template <int kVar> __device__ __forceinline__ uint4 seg_ld4(const uint4 *p) {
+  if (kVar & kSegStreamNA) {
+    uint4 v;
+    asm("ld.global.nc.L1::no_allocate.v4.u32 {%0, %1, %2, %3}, [%4];"
+        : "=r"(v.x), "=r"(v.y), "=r"(v.z), "=r"(v.w) : "l"(p));
+    return v;
+  }
+  return __ldg(p);
+}
+template <int kVar> __device__ __forceinline__ uint32_t seg_ld1(const uint32_t *p) {
+  if (kVar & kSegStreamNA) {
+    uint32_t v;
+    asm("ld.global.nc.L1::no_allocate.u32 %0, [%1];" : "=r"(v) : "l"(p));
+    return v;
+  }
+  return __ldg(p);
+}
+template <int kVar> __device__ __forceinline__ float seg_ldf(const float *p) {
+  if (kVar & kSegStreamNA) {
+    float v;
+    asm("ld.global.nc.L1::no_allocate.f32 %0, [%1];" : "=f"(v) : "l"(p));
+    return v;
+  }
+  return __ldg(p);
+}
+
 __device__ __forceinline__ float lds_f32(uint32_t saddr) {
   float v;
   asm("ld.shared.f32 %0, [%1];" : "=f"(v) : "r"(saddr));
   return v;
 }
 
-// Variant bits of k_pr_seg (GR_PR_SEG_VAR; measured in profiles/README.md):
-constexpr int kSegBallot = 1;   // segment starts of the lane scan from one ballot (1 shuffle per step, not 3)
-constexpr int kSegBuf = 2;      // finished rows through a per-warp buffer: coalesced apply, 1/outdeg preloaded
-constexpr int kSegPreFlag = 4;  // head bits loaded one tile ahead
-constexpr int kSegGeneric = 8;  // hot table read through a generic pointer instead of ld.shared
-constexpr int kSegDefaultVar = kSegBallot;  // measured best of the 16 (profiles/README.md)
 
 // contributions of my 8 items: hot sources from the shared table, the rest
 // from global memory (L2-resident)
@@ -496,8 +523,7 @@ __device__ __forceinline__ void seg_gather(const uint4 &s0, const uint4 &s1, con
   const uint32_t src[kSegIpt] = {s0.x, s0.y, s0.z, s0.w, s1.x, s1.y, s1.z, s1.w};
 #pragma unroll
   for (int k = 0; k < kSegIpt; k++) {
-    if (kVar & kSegGeneric) v[k] = (src[k] & kHotTag) ? s_hot[src[k] & ~kHotTag] : __ldg(contrib + src[k]);
-    else v[k] = (src[k] & kHotTag) ? lds_f32(hot_sbase + 4u * (src[k] & ~kHotTag)) : __ldg(contrib + src[k]);
+    v[k] = (src[k] & kHotTag) ? lds_f32(hot_sbase + 4u * (src[k] & ~kHotTag)) : __ldg(contrib + src[k]);
   }
 }
 
@@ -569,7 +595,7 @@ __device__ __forceinline__ void seg_tile(const PrArgs<OffT> &a, uint32_t tile, u
       } else {
         const float R = a.base + a.d * run;
         if (a.last) a.rank[row] = R;
-        else a.contrib_out[a.own_lo + row] = R * __ldg(a.inv_outdeg + a.own_lo + row);
+        else a.contrib_out[a.own_lo + row] = R * seg_ldf<kVar>(a.inv_outdeg + a.own_lo + row);
       }
     }
   }
@@ -611,25 +637,25 @@ __global__ void __launch_bounds__(1024, 1) k_pr_seg(const __grid_constant__ PrAr
   uint32_t tile = blockIdx.x * nw + w;
   if (tile >= num_tiles) return;
   const uint4 *src4 = reinterpret_cast<const uint4 *>(seg_src) + 2 * lane;
-  uint4 s0 = __ldg(src4 + (uint64_t)tile * (kSegTile / 4));
-  uint4 s1 = __ldg(src4 + (uint64_t)tile * (kSegTile / 4) + 1);
-  uint32_t r0 = __ldg(seg_row + tile);
+  uint4 s0 = seg_ld4<kVar>(src4 + (uint64_t)tile * (kSegTile / 4));
+  uint4 s1 = seg_ld4<kVar>(src4 + (uint64_t)tile * (kSegTile / 4) + 1);
+  uint32_t r0 = seg_ld1<kVar>(seg_row + tile);
   uint32_t fw = 0, fnext = 0;
   if (kVar & kSegPreFlag) {
-    fw = __ldg(seg_flags + (uint64_t)tile * 8 + (lane >> 2));
-    fnext = __ldg(seg_flags + (uint64_t)tile * 8 + 8) & 1u;
+    fw = seg_ld1<kVar>(seg_flags + (uint64_t)tile * 8 + (lane >> 2));
+    fnext = seg_ld1<kVar>(seg_flags + (uint64_t)tile * 8 + 8) & 1u;
   }
   for (;;) {
     if (!(kVar & kSegPreFlag)) {  // this tile's head bits, in flight together with the gathers
-      fw = __ldg(seg_flags + (uint64_t)tile * 8 + (lane >> 2));
-      fnext = __ldg(seg_flags + (uint64_t)tile * 8 + 8) & 1u;
+      fw = seg_ld1<kVar>(seg_flags + (uint64_t)tile * 8 + (lane >> 2));
+      fnext = seg_ld1<kVar>(seg_flags + (uint64_t)tile * 8 + 8) & 1u;
     }
     float v[kSegIpt];
     seg_gather<kVar>(s0, s1, s_hot, hot_sbase, a.contrib_in, v);
     float pre_inv = 0.f;
     if (kVar & kSegBuf) {
       const uint32_t prow = r0 + lane;
-      pre_inv = (!a.last && prow < a.own_n) ? __ldg(a.inv_outdeg + a.own_lo + prow) : 0.f;
+      pre_inv = (!a.last && prow < a.own_n) ? seg_ldf<kVar>(a.inv_outdeg + a.own_lo + prow) : 0.f;
     }
     const uint32_t b = (fw >> ((lane & 3) * 8)) & 0xFFu;  // bit k: my item k starts a row
     const uint32_t fn = fnext;
@@ -637,12 +663,12 @@ __global__ void __launch_bounds__(1024, 1) k_pr_seg(const __grid_constant__ PrAr
     const uint32_t ntile = tile + stride;
     uint32_t nr0 = 0;
     if (ntile < num_tiles) {
-      s0 = __ldg(src4 + (uint64_t)ntile * (kSegTile / 4));
-      s1 = __ldg(src4 + (uint64_t)ntile * (kSegTile / 4) + 1);
-      nr0 = __ldg(seg_row + ntile);
+      s0 = seg_ld4<kVar>(src4 + (uint64_t)ntile * (kSegTile / 4));
+      s1 = seg_ld4<kVar>(src4 + (uint64_t)ntile * (kSegTile / 4) + 1);
+      nr0 = seg_ld1<kVar>(seg_row + ntile);
       if (kVar & kSegPreFlag) {
-        fw = __ldg(seg_flags + (uint64_t)ntile * 8 + (lane >> 2));
-        fnext = __ldg(seg_flags + (uint64_t)ntile * 8 + 8) & 1u;
+        fw = seg_ld1<kVar>(seg_flags + (uint64_t)ntile * 8 + (lane >> 2));
+        fnext = seg_ld1<kVar>(seg_flags + (uint64_t)ntile * 8 + 8) & 1u;
       }
     }
     seg_tile<OffT, kVar>(a, tile, r0, b, fn, pre_inv, v, s_R);
@@ -858,26 +884,26 @@ __global__ void __launch_bounds__(1024, 1) k_pr_seg_loop(const __grid_constant__
     __syncthreads();
     uint32_t tile = blockIdx.x * nw + w;
     if (tile < L.num_tiles) {
-      uint4 s0 = __ldg(src4 + (uint64_t)tile * (kSegTile / 4));
-      uint4 s1 = __ldg(src4 + (uint64_t)tile * (kSegTile / 4) + 1);
-      uint32_t r0 = __ldg(L.seg_row + tile);
+      uint4 s0 = seg_ld4<kVar>(src4 + (uint64_t)tile * (kSegTile / 4));
+      uint4 s1 = seg_ld4<kVar>(src4 + (uint64_t)tile * (kSegTile / 4) + 1);
+      uint32_t r0 = seg_ld1<kVar>(L.seg_row + tile);
       for (;;) {
-        const uint32_t fw = __ldg(L.seg_flags + (uint64_t)tile * 8 + (lane >> 2));
-        const uint32_t fnext = __ldg(L.seg_flags + (uint64_t)tile * 8 + 8) & 1u;
+        const uint32_t fw = seg_ld1<kVar>(L.seg_flags + (uint64_t)tile * 8 + (lane >> 2));
+        const uint32_t fnext = seg_ld1<kVar>(L.seg_flags + (uint64_t)tile * 8 + 8) & 1u;
         float v[kSegIpt];
         seg_gather<kVar>(s0, s1, s_hot, hot_sbase, a.contrib_in, v);
         float pre_inv = 0.f;
         if (kVar & kSegBuf) {
           const uint32_t prow = r0 + lane;
-          pre_inv = (!a.last && prow < a.own_n) ? __ldg(a.inv_outdeg + a.own_lo + prow) : 0.f;
+          pre_inv = (!a.last && prow < a.own_n) ? seg_ldf<kVar>(a.inv_outdeg + a.own_lo + prow) : 0.f;
         }
         const uint32_t b = (fw >> ((lane & 3) * 8)) & 0xFFu;
         const uint32_t ntile = tile + stride;
         uint32_t nr0 = 0;
         if (ntile < L.num_tiles) {
-          s0 = __ldg(src4 + (uint64_t)ntile * (kSegTile / 4));
-          s1 = __ldg(src4 + (uint64_t)ntile * (kSegTile / 4) + 1);
-          nr0 = __ldg(L.seg_row + ntile);
+          s0 = seg_ld4<kVar>(src4 + (uint64_t)ntile * (kSegTile / 4));
+          s1 = seg_ld4<kVar>(src4 + (uint64_t)ntile * (kSegTile / 4) + 1);
+          nr0 = seg_ld1<kVar>(L.seg_row + ntile);
         }
         seg_tile<OffT, kVar>(a, tile, r0, b, fnext, pre_inv, v, s_R);
         if (ntile >= L.num_tiles) break;
