@@ -121,8 +121,11 @@ def override_algo(run, args):
     return r
 
 
-def workload_name(cfg, run):
+def workload_name(cfg, run, mode=None, scale=None):
     name = CONFIG_NAMES[cfg]
+    if cfg == 5:
+        name = f"cfg5 shape: PageRank x30 on R-MAT s{scale} ef16, " + (
+            "resident in HBM at 1 GPU" if mode == "resident" else "host-streamed shards (K=2 slots) at 1 GPU")
     if run.get("override"):
         extra = f", tolerance {run['tolerance']:g}" if run["algo"] == "pagerank_delta" else ""
         name += f" [program: {run['algo']}{extra}]"
@@ -233,7 +236,8 @@ def main():
         line = {"impl": "reference", "metric": "GTEPS", "value": val, "unit": "GTEPS", "n_gpus": args.gpus,
                 "steps": args.steps, "warmup": args.warmup, "higher_is_better": True, "scaling": "strong",
                 "vs_baseline": None, "dtype": "f64", "data": "synthetic",
-                "config": {"workload": workload_name(args.config, run), "impl": "single-threaded CPU oracle"},
+                "config": {"workload": workload_name(args.config, run, "streamed", args.scale),
+                           "impl": "single-threaded CPU oracle"},
                 "cpu_baseline": cb, "e2e": {"value": val, "unit": "GTEPS", "h2d_bytes_per_step": 0,
                                             "d2h_bytes_per_step": 0}}
         print(json.dumps(line), flush=True)
@@ -316,7 +320,7 @@ def main():
         if stats["kernel_ms"][2] == 1.0:
             # persistent loop: ONE launch runs all supersteps (tiles, fix-ups, hot-table pack, grid
             # barriers); its event-timed duration is divided per superstep, the unit of the bytes model
-            kname = "k_pr_seg_loop"
+            kname = "k_pr_bseg_loop" if int(stats["kernel_ms"][3]) == 8 else "k_pr_seg_loop"
     else:
         launches_per_step = max(1, stats["iterations"])
         bytes_per_launch = stats["bytes_hbm_model"] / launches_per_step
@@ -329,8 +333,8 @@ def main():
             "frac": round(achieved / peak, 4), "peak_source": peak_src,
             "bytes_per_launch": int(bytes_per_launch), "avg_launch_us": round(avg_launch_s * 1e6, 2),
             "kernel_share_of_step": round(kms / ms, 4) if ms > 0 else None,
-            "per": "superstep (30 per launch)" if kname == "k_pr_seg_loop" else "launch",
-            "traffic": load_traffic(kname)}
+            "per": "superstep (30 per launch)" if kname.endswith("_loop") else "launch",
+            "traffic": load_traffic(f"{kname}@cfg{args.config}" + (f"s{args.scale}" if args.config == 5 else ""))}
     if mode == "streamed":
         h2d_peak = measure_h2d()
         h2d_rate = stats["bytes_h2d"] / (ms_step * 1e-3) / 1e9
@@ -378,7 +382,7 @@ def main():
             "higher_is_better": True, "scaling": "strong", "vs_baseline": None,
             "dtype": "f32" if algo == "pagerank" else ("u64+f32" if algo == "pagerank_delta" else "u32"),
             "data": "synthetic",
-            "config": {"workload": workload_name(args.config, run), "n": n, "m": m, "shards": info["num_shards"],
+            "config": {"workload": workload_name(args.config, run, mode, args.scale), "n": n, "m": m, "shards": info["num_shards"],
                        "mode": mode, "parallelism": f"dst-interval partitions x{world}" if world > 1 else "1 GPU",
                        "l2": "inputs larger than L2 (CSC payload > 126 MB L2); no flush",
                        "iterations": stats["iterations"],

@@ -530,6 +530,117 @@ template <class OffT> static SegKernel<OffT> seg_kernel(int var) {
   return tab[var & 15];
 }
 
+// Source-blocked layout for k_pr_bseg_loop (once per graph):
+// stable radix sort of the CSC edges by source block (CSC order kept inside a
+// block), each block padded to whole tiles, run heads where a row starts or
+// its source block changes, run -> row, first run of every tile.
+template <class OffT> static gr_status pr_bseg_setup(gr_graph *g, uint32_t S) {
+  const HostGraph &H = g->H;
+  cudaStream_t s = g->stream;
+  const uint32_t rows = (uint32_t)H.own_n();
+  const uint64_t m = H.m_in;
+  const OffT *in_off = (const OffT *)g->in_off;
+  const uint32_t B = (uint32_t)((H.n + S - 1) / S);
+  int end_bit = 1;
+  while ((1ull << end_bit) < B) end_bit++;
+  uint32_t *k0 = nullptr, *k1 = nullptr, *v0 = nullptr, *v1 = nullptr, *rowbits = nullptr;
+  uint64_t *bstart = nullptr, *pstart = nullptr;
+  void *tmp = nullptr;
+  size_t need = 0;
+  auto cleanup = [&] {
+    pfree(k0, s); pfree(k1, s); pfree(v0, s); pfree(v1, s); pfree(rowbits, s); pfree(bstart, s); pfree(pstart, s);
+    pfree(tmp, s);
+  };
+  if (pmalloc(&k0, 4 * m, s) != cudaSuccess || pmalloc(&k1, 4 * m, s) != cudaSuccess ||
+      pmalloc(&v0, 4 * m, s) != cudaSuccess || pmalloc(&v1, 4 * m, s) != cudaSuccess ||
+      pmalloc(&rowbits, 4 * (m / 32 + 2), s) != cudaSuccess || pmalloc(&bstart, 8ull * (B + 1), s) != cudaSuccess ||
+      pmalloc(&pstart, 8ull * (B + 1), s) != cudaSuccess) {
+    cleanup();
+    return fail(GR_ENOMEM, "blocked PageRank layout: allocation failed");
+  }
+  k_bseg_key<<<g->num_sms * 16, 256, 0, s>>>(g->in_src, m, S, k0, v0);
+  cub::DoubleBuffer<uint32_t> kk(k0, k1), vv(v0, v1);
+  CK(cub::DeviceRadixSort::SortPairs(nullptr, need, kk, vv, (int64_t)m, 0, end_bit, s));
+  if (pmalloc(&tmp, std::max<size_t>(need, 16), s) != cudaSuccess) {
+    cleanup();
+    return fail(GR_ENOMEM, "blocked PageRank layout: sort temp allocation failed");
+  }
+  CK(cub::DeviceRadixSort::SortPairs(tmp, need, kk, vv, (int64_t)m, 0, end_bit, s));
+  k_bseg_bounds<<<g->num_sms * 16, 256, 0, s>>>(kk.Current(), m, B, bstart);
+  std::vector<uint64_t> hb(B + 1), hp(B + 1);
+  CK(cudaMemcpyAsync(hb.data(), bstart, 8ull * (B + 1), cudaMemcpyDeviceToHost, s));
+  CK(cudaStreamSynchronize(s));
+  std::vector<uint32_t> hbt(B + 1);
+  hp[0] = 0;
+  for (uint32_t b = 0; b < B; b++) {
+    const uint64_t c = hb[b + 1] - hb[b];
+    hp[b + 1] = hp[b] + (c + kSegTile - 1) / kSegTile * kSegTile;
+    hbt[b] = (uint32_t)(hp[b] / kSegTile);
+  }
+  hbt[B] = (uint32_t)(hp[B] / kSegTile);
+  const uint64_t P = hp[B];
+  if (P + kSegTile >= 0xFFFFFFFFull) {
+    cleanup();
+    return fail(GR_EUNSUPPORTED, "blocked PageRank layout: %llu items exceed 32-bit item indices",
+                (unsigned long long)P);
+  }
+  CK(cudaMemcpyAsync(pstart, hp.data(), 8ull * (B + 1), cudaMemcpyHostToDevice, s));
+  gr_status st;
+  if ((st = dev_alloc(g, (void **)&g->b_items, 4 * P + 16)) != GR_OK) { cleanup(); return st; }
+  if ((st = dev_alloc(g, (void **)&g->b_flags, 4 * (P / 32 + 16))) != GR_OK) { cleanup(); return st; }
+  if ((st = dev_alloc(g, (void **)&g->b_blk_tile, 4ull * (B + 1))) != GR_OK) { cleanup(); return st; }
+  if ((st = dev_alloc(g, (void **)&g->b_acc, 4ull * std::max<uint32_t>(rows, 1))) != GR_OK) { cleanup(); return st; }
+  CK(cudaMemcpyAsync(g->b_blk_tile, hbt.data(), 4ull * (B + 1), cudaMemcpyHostToDevice, s));
+  CK(cudaMemsetAsync(g->b_acc, 0, 4ull * rows, s));
+  uint32_t *head = nullptr, *runidx = nullptr;
+  if (pmalloc(&head, 4 * P + 4, s) != cudaSuccess || pmalloc(&runidx, 4 * P + 4, s) != cudaSuccess) {
+    pfree(head, s); pfree(runidx, s);
+    cleanup();
+    return fail(GR_ENOMEM, "blocked PageRank layout: head allocation failed");
+  }
+  k_fill_u32<<<g->num_sms * 8, 256, 0, s>>>(g->b_items, kHotTag | g->hot_k, P);  // padding reads the zero slot
+  CK(cudaMemsetAsync(head, 0, 4 * P + 4, s));
+  CK(cudaMemsetAsync(rowbits, 0, 4 * (m / 32 + 2), s));
+  k_bseg_rowstart<OffT><<<g->num_sms * 8, 256, 0, s>>>(in_off, rows, rowbits);
+  k_bseg_place<<<g->num_sms * 16, 256, 0, s>>>(kk.Current(), vv.Current(), m, bstart, pstart, g->in_src, g->pr_src, S,
+                                               rowbits, g->b_items, head);
+  k_bseg_flags<<<g->num_sms * 8, 256, 0, s>>>(head, P, g->b_flags);
+  pfree(tmp, s);
+  tmp = nullptr;
+  CK(cub::DeviceScan::ExclusiveSum(nullptr, need, head, runidx, (int64_t)P + 1, s));
+  CK(pmalloc(&tmp, std::max<size_t>(need, 16), s));
+  CK(cub::DeviceScan::ExclusiveSum(tmp, need, head, runidx, (int64_t)P + 1, s));
+  uint32_t nruns = 0;
+  CK(cudaMemcpyAsync(&nruns, runidx + P, 4, cudaMemcpyDeviceToHost, s));
+  CK(cudaStreamSynchronize(s));
+  uint32_t *run_off = nullptr;
+  if ((st = dev_alloc(g, (void **)&g->b_run_row, 4ull * (nruns + 64))) != GR_OK) { pfree(head, s); pfree(runidx, s); cleanup(); return st; }
+  CK(pmalloc(&run_off, 4ull * (nruns + 1), s));
+  k_bseg_runs<OffT><<<g->num_sms * 16, 256, 0, s>>>(kk.Current(), vv.Current(), m, bstart, pstart, head, runidx,
+                                                    in_off, rows, run_off, g->b_run_row);
+  const uint32_t Pu = (uint32_t)P;
+  CK(cudaMemcpyAsync(run_off + nruns, &Pu, 4, cudaMemcpyHostToDevice, s));
+  g->b_tiles = (uint32_t)(P / kSegTile);
+  if ((st = dev_alloc(g, (void **)&g->b_tile_run, 4ull * (g->b_tiles + 1))) != GR_OK) { pfree(head, s); pfree(runidx, s); pfree(run_off, s); cleanup(); return st; }
+  uint32_t *d_nlong = nullptr;
+  CK(pmalloc(&d_nlong, 4, s));
+  CK(cudaMemsetAsync(d_nlong, 0, 4, s));
+  k_seg_tiles<<<(g->b_tiles + 255) / 256 + 1, 256, 0, s>>>(run_off, nruns, g->b_tiles, g->b_tile_run, g->w_is_long,
+                                                            g->long_c, g->long_f, d_nlong);
+  CK(cudaGetLastError());
+  CK(cudaMemcpyAsync(&g->n_long, d_nlong, 4, cudaMemcpyDeviceToHost, s));
+  CK(cudaStreamSynchronize(s));
+  pfree(d_nlong, s);
+  pfree(run_off, s);
+  pfree(head, s);
+  pfree(runidx, s);
+  cleanup();
+  g->b_nblk = B;
+  g->b_nruns = nruns;
+  g->b_S = S;
+  return GR_OK;
+}
+
 // Hot-source setup (once per graph): pick the K vertices of largest
 // out-degree (the sources of the most in-edges), tag them in a PageRank copy
 // of the CSC payload, size the persistent grid from the occupancy calculator.
@@ -538,13 +649,21 @@ template <class OffT> static gr_status pr_hot_setup(gr_graph *g) {
   const HostGraph &H = g->H;
   const bool hot_ok = g->mode == GR_MODE_RESIDENT && !g->comm && H.n < 0x80000000ull && H.m_in >= (1u << 20);
   const bool seg_ok = hot_ok && (uint64_t)H.own_n() + H.m_in + 2 * kSegTile < 0xFFFFFFFFull;
-  // kernel variant (GR_PR_KERNEL = block | warp | warphot | range | rangehot | pipe | seg; default seg)
-  g->pr_kernel = seg_ok ? 7 : 3;
+  // source block for the blocked layout: the contributions of one block must stay in L2
+  uint64_t block_mb = 64;  // measured on R-MAT s26: 24 MB 4.81, 40 MB 4.52, 64 MB 4.42 ms per superstep
+  if (const char *bm = getenv("GR_PR_BLOCK_MB")) block_mb = std::max<uint64_t>(1, strtoull(bm, nullptr, 10));
+  uint32_t S = (uint32_t)std::max<uint64_t>(1024, (block_mb << 20) / 4 / 32 * 32);
+  if (const char *bv = getenv("GR_PR_BLOCK_V")) S = (uint32_t)std::max<uint64_t>(32, strtoull(bv, nullptr, 10));  // tests
+  const bool bseg_ok = seg_ok && !g->comm && H.n > S;
+  // kernel variant (GR_PR_KERNEL = block | warp | warphot | range | rangehot | pipe | seg | bseg; default seg,
+  // bseg when the contribution array is larger than one L2 block)
+  g->pr_kernel = bseg_ok ? 8 : seg_ok ? 7 : 3;
   if (const char *k = getenv("GR_PR_KERNEL")) {
     const std::string v(k);
     g->pr_kernel = v == "block" || v == "blockhot" ? 0 : v == "warp" ? 2 : v == "warphot" ? 3 : v == "range" ? 4
-                 : v == "pipe" ? 6 : v == "seg" ? 7 : 5;
+                 : v == "pipe" ? 6 : v == "seg" ? 7 : v == "bseg" ? 8 : 5;
   }
+  if (g->pr_kernel == 8 && !seg_ok) g->pr_kernel = hot_ok ? 3 : 2;
   if ((g->pr_kernel == 3 || g->pr_kernel == 5) && !hot_ok) g->pr_kernel -= 1;
   if (g->pr_kernel == 6 && !hot_ok) g->pr_kernel = 2;
   if (g->pr_kernel == 7 && !seg_ok) g->pr_kernel = hot_ok ? 3 : 2;
@@ -557,9 +676,10 @@ template <class OffT> static gr_status pr_hot_setup(gr_graph *g) {
     g->hot_grid = (uint32_t)(g->num_sms * std::max(bps, 1));
     return GR_OK;
   }
-  if (g->pr_kernel != 3 && g->pr_kernel != 5 && g->pr_kernel != 6 && g->pr_kernel != 7) return GR_OK;
-  // the seg kernel stages nothing in shared memory: its table can be ~3x larger
-  uint64_t K = g->pr_kernel == 7 ? kSegHotK : kHotK;
+  if (g->pr_kernel != 3 && g->pr_kernel != 5 && g->pr_kernel != 6 && g->pr_kernel != 7 && g->pr_kernel != 8)
+    return GR_OK;
+  // the seg kernels stage nothing in shared memory: their table can be ~2x larger
+  uint64_t K = g->pr_kernel >= 7 ? kSegHotK : kHotK;
   if (const char *hk = getenv("GR_PR_HOTK")) K = std::max<uint64_t>(4, std::min<uint64_t>(strtoull(hk, nullptr, 10), 57344));
   K = std::min<uint64_t>(K, H.n);
   uint32_t *d_slot = nullptr;
@@ -571,7 +691,20 @@ template <class OffT> static gr_status pr_hot_setup(gr_graph *g) {
   CK(cudaGetLastError());
   CK(cudaStreamSynchronize(g->stream));
   int bps = 0;
-  if (g->pr_kernel == 7) {
+  if (g->pr_kernel == 8) {
+    if (!g->coop) return fail(GR_EUNSUPPORTED, "blocked PageRank needs cooperative launch");
+    if ((s = pr_bseg_setup<OffT>(g, S)) != GR_OK) return s;
+    g->hot_cta = 1024;
+    g->hot_smem = 4ull * (g->hot_k + 4) + 4ull * 64 * (g->hot_cta / 32);
+    g->b_pol = 1;
+    if (const char *bp = getenv("GR_PR_BLOCK_POLICY")) g->b_pol = atoi(bp) != 0;
+    for (auto kf : {(const void *)k_pr_bseg_loop<OffT, 0>, (const void *)k_pr_bseg_loop<OffT, 1>})
+      CK(cudaFuncSetAttribute(kf, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)g->hot_smem));
+    CK(cudaOccupancyMaxActiveBlocksPerMultiprocessor(&bps, k_pr_bseg_loop<OffT, 1>, g->hot_cta, g->hot_smem));
+    if (bps < 1) return fail(GR_EUNSUPPORTED, "blocked PageRank kernel does not fit on an SM");
+    bps = 1;
+    g->pr_loop = 1;
+  } else if (g->pr_kernel == 7) {
     if ((s = pr_seg_setup<OffT>(g)) != GR_OK) return s;
     g->hot_cta = 1024;
     g->seg_var = kSegDefaultVar;
@@ -696,7 +829,55 @@ static gr_status run_pagerank(gr_graph *g, const gr_run_opts *o, cudaStream_t s,
       g->prof_ev.push_back(e);
     }
   }
-  if (g->pr_kernel == 7 && g->pr_loop) {
+  if (g->pr_kernel == 8) {
+    // source-blocked persistent loop (f3): init, first hot-table pack, ONE cooperative launch
+    if (!g->hot_buf[0]) {
+      for (int i = 0; i < 2; i++) {
+        gr_status s2 = dev_alloc(g, (void **)&g->hot_buf[i], 4ull * (g->hot_k + 4));
+        if (s2 != GR_OK) return s2;
+      }
+      gr_status s2 = dev_alloc(g, (void **)&g->pr_bar, 64);
+      if (s2 != GR_OK) return s2;
+      CK(cudaMemsetAsync(g->pr_bar, 0, 64, s));
+    }
+    PrArgs<OffT> a = pr_args<OffT>(g, 0, iters, d);
+    PrBlk L{};
+    L.items = g->b_items;
+    L.flags = g->b_flags;
+    L.tile_run = g->b_tile_run;
+    L.run_row = g->b_run_row;
+    L.blk_tile = g->b_blk_tile;
+    L.nblk = g->b_nblk;
+    L.nruns = g->b_nruns;
+    L.num_tiles = g->b_tiles;
+    L.iters = iters;
+    L.acc = g->b_acc;
+    L.hot_ids = g->hot_ids;
+    L.hot_buf[0] = g->hot_buf[0];
+    L.hot_buf[1] = g->hot_buf[1];
+    L.contrib[0] = g->contrib[0];
+    L.contrib[1] = g->contrib[1];
+    L.is_long = g->w_is_long;
+    L.long_c = g->long_c;
+    L.long_f = g->long_f;
+    L.n_long = g->n_long;
+    L.hot_k = g->hot_k;
+    L.bar = g->pr_bar;
+    k_pr_init<<<g->num_sms * 4, 256, 0, s>>>((uint32_t)g->H.n, g->inv_outdeg, g->contrib[0]);
+    k_pr_hot_pack<<<(g->hot_k + 255) / 256, 256, 0, s>>>(g->contrib[0], g->hot_ids, g->hot_buf[0], g->hot_k);
+    if (prof) CK(cudaEventRecord(g->prof_ev[0], s));
+    void *args[] = {(void *)&a, (void *)&L};
+    const void *kf = g->b_pol ? (const void *)k_pr_bseg_loop<OffT, 1> : (const void *)k_pr_bseg_loop<OffT, 0>;
+    CK(cudaLaunchCooperativeKernel(kf, dim3(g->hot_grid), dim3(g->hot_cta), args, g->hot_smem, s));
+    if (prof) CK(cudaEventRecord(g->prof_ev[1], s));
+    CK(cudaStreamSynchronize(s));
+    if (prof) {
+      float ms = 0;
+      CK(cudaEventElapsedTime(&ms, g->prof_ev[0], g->prof_ev[1]));
+      st->kernel_ms[0] += ms;
+    }
+    st->kernel_launches += 3;
+  } else if (g->pr_kernel == 7 && g->pr_loop) {
     // persistent loop: init, pack of the first hot table, ONE cooperative launch for all supersteps
     PrArgs<OffT> a = pr_args<OffT>(g, 0, iters, d);
     PrLoop L{};
@@ -772,9 +953,10 @@ static gr_status run_pagerank(gr_graph *g, const gr_run_opts *o, cudaStream_t s,
   st->iterations = iters;
   st->edges_gathered = (uint64_t)iters * g->H.m_in;
   st->edges_scattered = 0;
-  if (!(g->pr_kernel == 7 && g->pr_loop)) st->kernel_launches += 1 + (g->pr_hot == 1 ? 3ull : 2ull) * iters;
-  st->kernel_ms[3] = (double)g->pr_kernel;  // which PageRank gather variant ran (0 block .. 7 seg)
-  st->kernel_ms[2] = (g->pr_kernel == 7 && g->pr_loop) ? 1.0 : 0.0;  // 1: persistent loop (kernel_ms[0] = whole loop)
+  const bool loop = (g->pr_kernel == 7 && g->pr_loop) || g->pr_kernel == 8;
+  if (!loop) st->kernel_launches += 1 + (g->pr_hot == 1 ? 3ull : 2ull) * iters;
+  st->kernel_ms[3] = (double)g->pr_kernel;  // which PageRank gather variant ran (0 block .. 7 seg, 8 blocked seg)
+  st->kernel_ms[2] = loop ? 1.0 : 0.0;      // 1: persistent loop (kernel_ms[0] = whole loop)
   st->bytes_hbm_model = (uint64_t)iters * (4 * g->H.m_in + 12 * g->H.own_n() + 4 * g->H.n);
   g->trace_rows = iters;
   return GR_OK;

@@ -87,6 +87,11 @@ struct gr_graph {
   uint32_t *hot_slot = nullptr, *pr_bar = nullptr;
   uint8_t *hot_split = nullptr;
   float *hot_buf[2] = {nullptr, nullptr};
+  // source-blocked PageRank layout (pr_kernel 8, k_pr_bseg_loop)
+  uint32_t *b_items = nullptr, *b_flags = nullptr, *b_tile_run = nullptr, *b_run_row = nullptr, *b_blk_tile = nullptr;
+  float *b_acc = nullptr;
+  uint32_t b_nblk = 0, b_nruns = 0, b_tiles = 0, b_S = 0;
+  int b_pol = 1;
   uint64_t seg_items = 0;
 
   // run bookkeeping

@@ -936,6 +936,316 @@ __global__ void __launch_bounds__(1024, 1) k_pr_seg_loop(const __grid_constant__
   }
 }
 
+// ---------------------------------------------------------------------------
+// Source-blocked PageRank (§4.2 L210 partition hook,
+// L352): when the contribution array is much larger than L2 (n·4 B ≫ 126 MB,
+// e.g. R-MAT s26+ resident, or cfg5's replicas at G = 8), the sources are cut
+// into B blocks of S vertices whose contributions fit in L2, and the item
+// stream is re-laid out block-major: block b holds the in-edges with a source
+// in block b, in CSC order (by destination). A "run" is the (destination,
+// block) slice of a row; runs play the role rows play in k_pr_seg (one head
+// bit per run start, tiles of 256 items, each block padded to whole tiles).
+// Per superstep the blocks are reduced one after the other, so the random
+// gathers of block b hit an L2-resident 4·S-byte slice (cold gathers carry an
+// L2 evict_last policy, the streamed items evict_first); each finished run
+// adds its partial sum to acc[destination] with one red.global.add — exactly
+// one add per (destination, block) per phase, phases ordered by grid
+// barriers, so the fp32 sum order is fixed — and an apply phase turns acc
+// into ranks / contributions.
+struct PrBlk {
+  const uint32_t *items, *flags, *tile_run;  // concatenated blocks (each padded to whole tiles)
+  const uint32_t *run_row;                   // run -> destination row
+  const uint32_t *blk_tile;                  // [nblk + 1] first tile of each block
+  uint32_t nblk, nruns, num_tiles, iters;
+  float *acc;                                // [n] partial sums (zeroed by the apply phase)
+  const uint32_t *hot_ids;
+  float *hot_buf[2];
+  float *contrib[2];
+  const uint8_t *is_long;
+  const uint32_t *long_c, *long_f;
+  uint32_t n_long, hot_k;
+  uint32_t *bar;
+};
+
+template <int kPol> __device__ __forceinline__ uint4 bseg_ld4(const uint4 *p, uint64_t pol) {
+  if (kPol) {
+    uint4 v;
+    asm("ld.global.nc.L1::no_allocate.L2::cache_hint.v4.u32 {%0, %1, %2, %3}, [%4], %5;"
+        : "=r"(v.x), "=r"(v.y), "=r"(v.z), "=r"(v.w) : "l"(p), "l"(pol));
+    return v;
+  }
+  return __ldg(p);
+}
+template <int kPol> __device__ __forceinline__ float bseg_ldc(const float *p, uint64_t pol) {
+  if (kPol) {
+    float v;
+    asm("ld.global.nc.L2::cache_hint.f32 %0, [%1], %2;" : "=f"(v) : "l"(p), "l"(pol));
+    return v;
+  }
+  return __ldg(p);
+}
+
+// One block tile: like seg_tile, with runs for rows; finished runs (other than
+// the tile's head run) go through the per-warp buffer s_R (64 runs) and are
+// added to acc[run_row] by coalesced red.global.add; rr0/rr1 = run_row of the
+// tile's first 64 runs, loaded with the gathers.
+__device__ __forceinline__ void bseg_tile(const PrBlk &L, uint32_t *head_row, float *head_val, uint32_t *carry_row,
+                                          float *carry_val, uint32_t tile, uint32_t j0, uint32_t b, uint32_t fnext,
+                                          uint32_t rr0, uint32_t rr1, const float (&v)[kSegIpt], float *s_R) {
+  const uint32_t lane = threadIdx.x & 31;
+  uint32_t bn = __shfl_down_sync(0xffffffffu, b, 1) & 1u;
+  if (lane == 31) bn = fnext;
+  const uint32_t ends = (b >> 1) | (bn << 7);
+  float tail = 0.f;
+#pragma unroll
+  for (int k = 0; k < kSegIpt; k++) {
+    if ((b >> k) & 1u) tail = 0.f;
+    tail += v[k];
+  }
+  uint32_t cnt = __popc(b);
+  float x = tail;
+  const uint32_t hl = __ballot_sync(0xffffffffu, b != 0u) & (0xFFFFFFFFu >> (31 - lane));
+  const int seg0 = hl ? 31 - __clz(hl) : 0;
+#pragma unroll
+  for (int o = 1; o < 32; o <<= 1) {
+    const float y = __shfl_up_sync(0xffffffffu, x, o);
+    const uint32_t c = __shfl_up_sync(0xffffffffu, cnt, o);
+    if ((int)lane - o >= seg0) x += y;
+    if (lane >= (uint32_t)o) cnt += c;
+  }
+  float run = __shfl_up_sync(0xffffffffu, x, 1);
+  if (lane == 0) run = 0.f;
+  const uint32_t total_heads = __shfl_sync(0xffffffffu, cnt, 31);
+  const uint32_t h0 = __shfl_sync(0xffffffffu, b, 0) & 1u;
+  uint32_t j = j0 - h0 + (cnt - __popc(b));
+  const bool head_exists = !h0 && (total_heads > 0 || fnext);
+  if (lane == 0 && !head_exists) head_row[tile] = kNoRow;
+#pragma unroll
+  for (int k = 0; k < kSegIpt; k++) {
+    if ((b >> k) & 1u) { run = 0.f; ++j; }
+    run += v[k];
+    if (((ends >> k) & 1u) && j < L.nruns) {
+      const uint32_t idx = j - j0;
+      if (!h0 && idx == 0) {
+        head_row[tile] = j0;
+        head_val[tile] = run;
+      } else if (idx < 64u) {
+        s_R[idx] = run;
+      } else {
+        atomicAdd(L.acc + __ldg(L.run_row + j), run);
+      }
+    }
+  }
+  if (lane == 31) {
+    const bool open = !fnext && j < L.nruns;
+    carry_row[tile] = open ? j : kNoRow;
+    carry_val[tile] = run;
+  }
+  __syncwarp();
+  const int first = h0 ? 0 : 1;
+  const int lastc = (int)(total_heads - h0) - (fnext ? 0 : 1);
+  if ((int)lane >= first && (int)lane <= lastc && j0 + lane < L.nruns) atomicAdd(L.acc + rr0, s_R[lane]);
+  if ((int)lane + 32 >= first && (int)lane + 32 <= lastc && j0 + 32 + lane < L.nruns)
+    atomicAdd(L.acc + rr1, s_R[32 + lane]);
+  __syncwarp();
+}
+
+template <class OffT, int kPol>
+__global__ void __launch_bounds__(1024, 1) k_pr_bseg_loop(const __grid_constant__ PrArgs<OffT> a0,
+                                                         const __grid_constant__ PrBlk L) {
+  extern __shared__ __align__(16) float s_hot[];  // [hot_k + 4] table, then 64 floats per warp
+  const uint32_t hot_sbase = (uint32_t)__cvta_generic_to_shared(s_hot);
+  const uint32_t lane = threadIdx.x & 31, w = threadIdx.x >> 5, nw = blockDim.x >> 5;
+  float *s_R = s_hot + L.hot_k + 4 + 64 * w;
+  const uint32_t gw = blockIdx.x * nw + w, W = gridDim.x * nw;
+  const uint4 *src4 = reinterpret_cast<const uint4 *>(L.items) + 2 * lane;
+  const uint64_t gtid = blockIdx.x * (uint64_t)blockDim.x + threadIdx.x, gthreads = (uint64_t)gridDim.x * blockDim.x;
+  uint64_t pol_keep = 0, pol_stream = 0;
+  if (kPol) {
+    asm("createpolicy.fractional.L2::evict_last.b64 %0, 1.0;" : "=l"(pol_keep));
+    asm("createpolicy.fractional.L2::evict_first.b64 %0, 1.0;" : "=l"(pol_stream));
+  }
+  for (uint32_t t = 0; t < L.iters; t++) {
+    const float *contrib_in = L.contrib[t & 1];
+    float *contrib_out = L.contrib[(t + 1) & 1];
+    const bool last = t + 1 == L.iters;
+    const float *hot_cur = L.hot_buf[t & 1];
+    float *hot_next = L.hot_buf[(t + 1) & 1];
+    for (uint32_t k = threadIdx.x * 4; k < L.hot_k; k += blockDim.x * 4)
+      *reinterpret_cast<float4 *>(s_hot + k) = *reinterpret_cast<const float4 *>(hot_cur + k);
+    if (threadIdx.x < 4) s_hot[L.hot_k + threadIdx.x] = 0.f;
+    __syncthreads();
+    for (uint32_t blk = 0; blk < L.nblk; blk++) {
+      const uint32_t t_lo = L.blk_tile[blk], t_hi = L.blk_tile[blk + 1];
+      // ---- block phase: its tiles (gathers from the L2-resident source slice)
+      uint32_t tile = t_lo + gw;
+      if (tile < t_hi) {
+        uint4 s0 = bseg_ld4<kPol>(src4 + (uint64_t)tile * (kSegTile / 4), pol_stream);
+        uint4 s1 = bseg_ld4<kPol>(src4 + (uint64_t)tile * (kSegTile / 4) + 1, pol_stream);
+        uint32_t j0 = __ldg(L.tile_run + tile);
+        for (;;) {
+          const uint32_t fw = __ldg(L.flags + (uint64_t)tile * 8 + (lane >> 2));
+          const uint32_t fnext = __ldg(L.flags + (uint64_t)tile * 8 + 8) & 1u;
+          const uint32_t rr0 = j0 + lane < L.nruns ? __ldg(L.run_row + j0 + lane) : 0u;
+          const uint32_t rr1 = j0 + 32 + lane < L.nruns ? __ldg(L.run_row + j0 + 32 + lane) : 0u;
+          float v[kSegIpt];
+          {
+            const uint32_t src[kSegIpt] = {s0.x, s0.y, s0.z, s0.w, s1.x, s1.y, s1.z, s1.w};
+#pragma unroll
+            for (int k = 0; k < kSegIpt; k++)
+              v[k] = (src[k] & kHotTag) ? lds_f32(hot_sbase + 4u * (src[k] & ~kHotTag))
+                                        : bseg_ldc<kPol>(contrib_in + src[k], pol_keep);
+          }
+          const uint32_t b = (fw >> ((lane & 3) * 8)) & 0xFFu;
+          const uint32_t ntile = tile + W;
+          uint32_t nj0 = 0;
+          if (ntile < t_hi) {
+            s0 = bseg_ld4<kPol>(src4 + (uint64_t)ntile * (kSegTile / 4), pol_stream);
+            s1 = bseg_ld4<kPol>(src4 + (uint64_t)ntile * (kSegTile / 4) + 1, pol_stream);
+            nj0 = __ldg(L.tile_run + ntile);
+          }
+          bseg_tile(L, a0.head_row, a0.head_val, a0.carry_row, a0.carry_val, tile, j0, b, fnext, rr0, rr1, v, s_R);
+          if (ntile >= t_hi) break;
+          tile = ntile;
+          j0 = nj0;
+        }
+      }
+      pr_grid_sync(L.bar);
+      // ---- runs split between tiles of this block (fixed order)
+      for (uint64_t c = t_lo + gtid; c < t_hi; c += gthreads) {
+        const uint32_t jr = a0.head_row[c];
+        if (jr == kNoRow || L.is_long[c]) continue;
+        float acc = a0.head_val[c];
+        for (int64_t p = (int64_t)c - 1; p >= (int64_t)t_lo && a0.carry_row[p] == jr; p--) acc += a0.carry_val[p];
+        atomicAdd(L.acc + __ldg(L.run_row + jr), acc);
+      }
+      for (uint64_t i = gtid >> 5; i < L.n_long; i += gthreads >> 5) {
+        const uint32_t c = L.long_c[i], f = L.long_f[i];
+        if (c < t_lo || c >= t_hi) continue;
+        const uint32_t jr = a0.head_row[c];
+        float acc = 0.f;
+        for (uint32_t p = f + lane; p < c; p += 32) acc += a0.carry_val[p];
+#pragma unroll
+        for (int o = 16; o > 0; o >>= 1) acc += __shfl_xor_sync(0xffffffffu, acc, o);
+        if (lane == 0 && jr != kNoRow) atomicAdd(L.acc + __ldg(L.run_row + jr), a0.head_val[c] + acc);
+      }
+      pr_grid_sync(L.bar);
+    }
+    // ---- apply: R = (1-d)/n + d * acc, 4 vertices per 128-bit access, 2 accesses in flight per thread
+    {
+      const uint64_t n4 = a0.own_n / 4;
+      float4 *acc4 = reinterpret_cast<float4 *>(L.acc);
+      const float4 *inv4 = reinterpret_cast<const float4 *>(a0.inv_outdeg);
+      float4 *out4 = reinterpret_cast<float4 *>(last ? a0.rank : contrib_out);
+      auto rank4 = [&](float4 x) {
+        return make_float4(a0.base + a0.d * x.x, a0.base + a0.d * x.y, a0.base + a0.d * x.z, a0.base + a0.d * x.w);
+      };
+      for (uint64_t q0 = gtid; q0 < n4; q0 += 2 * gthreads) {
+        float4 x[2], iv[2];
+#pragma unroll
+        for (int u = 0; u < 2; u++) {
+          const uint64_t q = q0 + u * gthreads;
+          if (q < n4) {
+            x[u] = acc4[q];
+            iv[u] = last ? make_float4(1.f, 1.f, 1.f, 1.f) : __ldg(inv4 + q);
+          }
+        }
+#pragma unroll
+        for (int u = 0; u < 2; u++) {
+          const uint64_t q = q0 + u * gthreads;
+          if (q < n4) {
+            const float4 R = rank4(x[u]);
+            acc4[q] = make_float4(0.f, 0.f, 0.f, 0.f);
+            out4[q] = make_float4(R.x * iv[u].x, R.y * iv[u].y, R.z * iv[u].z, R.w * iv[u].w);
+          }
+        }
+      }
+      for (uint64_t v = 4 * n4 + gtid; v < a0.own_n; v += gthreads) {
+        const float R = a0.base + a0.d * L.acc[v];
+        L.acc[v] = 0.f;
+        if (last) a0.rank[v] = R;
+        else contrib_out[v] = R * __ldg(a0.inv_outdeg + v);
+      }
+    }
+    pr_grid_sync(L.bar);
+    if (!last) {
+      for (uint64_t k = gtid; k < L.hot_k; k += gthreads) hot_next[k] = contrib_out[L.hot_ids[k]];
+      pr_grid_sync(L.bar);
+    }
+  }
+}
+
+// --- blocked layout builders (once per graph) ---
+static __global__ void k_bseg_key(const uint32_t *in_src, uint64_t m, uint32_t S, uint32_t *key, uint32_t *val) {
+  for (uint64_t e = blockIdx.x * (uint64_t)blockDim.x + threadIdx.x; e < m; e += (uint64_t)gridDim.x * blockDim.x) {
+    key[e] = in_src[e] / S;
+    val[e] = (uint32_t)e;
+  }
+}
+// first sorted position of every block (bstart[B] = m; empty blocks share the next start)
+static __global__ void k_bseg_bounds(const uint32_t *skey, uint64_t m, uint32_t B, uint64_t *bstart) {
+  for (uint64_t i = blockIdx.x * (uint64_t)blockDim.x + threadIdx.x; i < m; i += (uint64_t)gridDim.x * blockDim.x) {
+    const int64_t k = skey[i];
+    const int64_t kp = i ? (int64_t)skey[i - 1] : -1;
+    if (k != kp)
+      for (int64_t b = kp + 1; b <= k; b++) bstart[b] = i;
+    if (i == m - 1)
+      for (int64_t b = k + 1; b <= (int64_t)B; b++) bstart[b] = m;
+  }
+}
+// row-start bits over edge indices: bit in_off[v] for rows with an in-edge
+template <class OffT>
+__global__ void k_bseg_rowstart(const OffT *in_off, uint32_t rows, uint32_t *bits) {
+  for (uint32_t v = blockIdx.x * blockDim.x + threadIdx.x; v < rows; v += gridDim.x * blockDim.x) {
+    const uint64_t e = in_off[v];
+    if ((uint64_t)in_off[v + 1] > e) atomicOr(bits + (e >> 5), 1u << (e & 31));
+  }
+}
+// place sorted edge i at its padded item position; head = run start
+static __global__ void k_bseg_place(const uint32_t *skey, const uint32_t *sval, uint64_t m, const uint64_t *bstart,
+                                    const uint64_t *pstart, const uint32_t *in_src, const uint32_t *pr_src,
+                                    uint32_t S, const uint32_t *rowbits, uint32_t *items, uint32_t *head) {
+  for (uint64_t i = blockIdx.x * (uint64_t)blockDim.x + threadIdx.x; i < m; i += (uint64_t)gridDim.x * blockDim.x) {
+    const uint32_t b = skey[i], e = sval[i];
+    const uint64_t pos = pstart[b] + (i - bstart[b]);
+    items[pos] = pr_src[e];
+    const bool rs = (rowbits[e >> 5] >> (e & 31)) & 1u;
+    head[pos] = (rs || in_src[e - 1] / S != b) ? 1 : 0;  // e == 0 is always a row start
+  }
+}
+// heads -> packed bits (+ sentinel at P)
+static __global__ void k_bseg_flags(const uint32_t *head, uint64_t P, uint32_t *flags) {
+  for (uint64_t wd = blockIdx.x * (uint64_t)blockDim.x + threadIdx.x; wd * 32 <= P;
+       wd += (uint64_t)gridDim.x * blockDim.x) {
+    uint32_t x = 0;
+    for (int k = 0; k < 32; k++) {
+      const uint64_t i = wd * 32 + k;
+      if (i < P ? head[i] != 0 : i == P) x |= 1u << k;
+    }
+    flags[wd] = x;
+  }
+}
+// runs: run_off[r] = item of the r-th head, run_row[r] = its destination (the edge's row)
+template <class OffT>
+__global__ void k_bseg_runs(const uint32_t *skey, const uint32_t *sval, uint64_t m, const uint64_t *bstart,
+                            const uint64_t *pstart, const uint32_t *head, const uint32_t *runidx, const OffT *in_off,
+                            uint32_t rows, uint32_t *run_off, uint32_t *run_row) {
+  for (uint64_t i = blockIdx.x * (uint64_t)blockDim.x + threadIdx.x; i < m; i += (uint64_t)gridDim.x * blockDim.x) {
+    const uint32_t b = skey[i], e = sval[i];
+    const uint64_t pos = pstart[b] + (i - bstart[b]);
+    if (!head[pos]) continue;
+    uint32_t lo = 0, hi = rows;  // last r with in_off[r] <= e
+    while (hi - lo > 1) {
+      const uint32_t mid = (lo + hi) >> 1;
+      if ((uint64_t)in_off[mid] <= e) lo = mid;
+      else hi = mid;
+    }
+    const uint32_t r = runidx[pos];
+    run_off[r] = (uint32_t)pos;
+    run_row[r] = lo;
+  }
+}
+
 // hot_split[k] = 1 when hot slot k's row spans two or more tiles (finished by the fix-up phase)
 static __global__ void k_seg_hot_split(const uint32_t *hot_ids, uint32_t hot_k, const uint32_t *seg_off,
                                        uint8_t *hot_split) {

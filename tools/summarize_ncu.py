@@ -65,7 +65,7 @@ def full(rep, out, key=None):
         lines.append("")
         rd = to_bytes(r[h.index("dram__bytes_read.sum")], units[h.index("dram__bytes_read.sum")])
         wr = to_bytes(r[h.index("dram__bytes_write.sum")], units[h.index("dram__bytes_write.sum")])
-        if key and key in name:
+        if key and key.split("@")[0] in name:
             traffic.append(rd + wr)
     open(out, "w").write("\n".join(lines) + "\n")
     if key and traffic:
