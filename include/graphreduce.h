@@ -207,6 +207,24 @@ gr_status gr_fetch_vertex_values(gr_graph *g, void *host_dst, uint64_t bytes);
  * FrontierActivate eliminated). *rows = supersteps recorded (<= max_rows). */
 gr_status gr_fetch_frontier_trace(gr_graph *g, uint64_t *host_dst, uint64_t max_rows, uint64_t *rows);
 
+/* ---- run-time GAS programs (§4.1, Fig. 6) ----
+ * Compile a user program at run time and register it. `source` is CUDA C++
+ * that defines `struct <struct_name>` (the library places it inside namespace
+ * gr, where Ctx, kInitAll & co. and the CUDA intrinsics are visible) with the interface
+ * of include/gr/program.cuh: GatherT (4- or 8-byte unsigned), kHasGather,
+ * kUsesWeights, kInit (kInitSource / kInitSourceChanged / kInitAll),
+ * initValue, identity, gatherMap, gatherReduce (associative + commutative),
+ * atomicGather, apply; vertex values are uint32. The library compiles it with
+ * NVRTC for the current device together with its own frontier kernels (the
+ * same gather / apply / FrontierActivate / persistent BSP loop as the built-in
+ * programs) and loads the module; run it with gr_run(algo = GR_CUSTOM,
+ * custom_id = *custom_id) on a resident single-GPU graph (persistent loop).
+ * Ids start at 1000; programs live until process exit.
+ * GR_EINVAL: null argument or empty name; GR_EUNSUPPORTED: libnvrtc /
+ * libcuda not loadable; GR_ECUDA: compile or load error — gr_last_error()
+ * carries the NVRTC log. Thread-safe. */
+gr_status gr_program_compile(const char *source, const char *struct_name, int32_t *custom_id);
+
 gr_status gr_graph_info_get(const gr_graph *g, gr_graph_info *out);
 gr_status gr_shard_info(const gr_graph *g, uint32_t shard, gr_shard_desc *out);
 void gr_graph_free(gr_graph *g); /* NULL-safe */

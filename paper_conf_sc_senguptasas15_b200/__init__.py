@@ -34,7 +34,7 @@ INF = 0xFFFFFFFF
 EXPORTS = [
     "gr_get_unique_id", "gr_graph_load", "gr_graph_load_file", "gr_run", "gr_fetch_vertex_values", "gr_fetch_frontier_trace",
     "gr_graph_info_get", "gr_shard_info", "gr_graph_free", "gr_last_error", "gr_plan_intervals",
-    "gr_host_build", "gr_host_csc", "gr_host_csr", "gr_host_shards", "gr_host_free",
+    "gr_host_build", "gr_host_csc", "gr_host_csr", "gr_host_shards", "gr_host_free", "gr_program_compile",
 ]
 
 
@@ -115,6 +115,7 @@ def lib():
         "gr_fetch_vertex_values": (i32, [vp, vp, u64]),
         "gr_fetch_frontier_trace": (i32, [vp, u64p, u64, u64p]),
         "gr_graph_info_get": (i32, [vp, ctypes.POINTER(gr_graph_info)]),
+        "gr_program_compile": (i32, [ctypes.c_char_p, ctypes.c_char_p, ctypes.POINTER(i32)]),
         "gr_shard_info": (i32, [vp, u32, ctypes.POINTER(gr_shard_desc)]),
         "gr_graph_free": (None, [vp]),
         "gr_last_error": (ctypes.c_char_p, []),
@@ -252,6 +253,14 @@ def gr_run(h, algo, source=0, max_iters=0, damping=0.85, custom_id=0, loop="auto
     st = gr_run_stats()
     _check(lib().gr_run(h, ctypes.byref(o), ctypes.byref(st)))
     return st.as_dict()
+
+
+def gr_program_compile(source: str, struct_name: str) -> int:
+    """Compile a GAS program at run time (NVRTC) and return its custom_id
+    (include/graphreduce.h gr_program_compile)."""
+    cid = ctypes.c_int32(0)
+    _check(lib().gr_program_compile(source.encode(), struct_name.encode(), ctypes.byref(cid)))
+    return int(cid.value)
 
 
 def gr_graph_info_get(h) -> dict:

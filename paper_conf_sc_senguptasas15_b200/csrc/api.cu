@@ -10,6 +10,7 @@
 #include <unistd.h>
 
 #include "engine.h"
+#include "jit.h"
 
 using namespace gr;
 
@@ -167,6 +168,13 @@ gr_status gr_fetch_frontier_trace(gr_graph *g, uint64_t *host_dst, uint64_t max_
   if (!g) return fail(GR_EINVAL, "graph is NULL");
   cudaSetDevice(g->device);
   return fetch_trace(g, host_dst, max_rows, rows);
+}
+
+gr_status gr_program_compile(const char *source, const char *struct_name, int32_t *custom_id) {
+  int id = 0;
+  const gr_status s = gr::jit_compile(source, struct_name, &id);
+  if (s == GR_OK) *custom_id = id;
+  return s;
 }
 
 gr_status gr_graph_info_get(const gr_graph *g, gr_graph_info *o) {

@@ -25,6 +25,7 @@
 #include <vector>
 
 #include "engine.h"
+#include "jit.h"
 #include "kernels_frontier.cuh"
 #include "kernels_pr.cuh"
 
@@ -433,6 +434,97 @@ static gr_status run_frontier(gr_graph *g, const gr_run_opts *o, cudaStream_t s,
   uint64_t sumA = 0, sumC = 0;
   for (uint64_t t = 0; t < g->trace_rows; t++) { sumA += tr[4 * t]; sumC += tr[4 * t + 1]; }
   const uint64_t wb = Prog::kUsesWeights ? 5 : 4;
+  st->bytes_hbm_model = wb * c.tot_gathered + 12 * sumA + 4 * c.tot_scattered + 12 * sumC;
+  return GR_OK;
+}
+
+// Run-time compiled program (csrc/jit.cu): the same setup
+// and persistent BSP loop as run_frontier, with the program's kernels taken
+// from its NVRTC module and its static traits read back at compile time.
+template <class OffT>
+static gr_status run_frontier_jit(gr_graph *g, const gr_run_opts *o, cudaStream_t s, gr_run_stats *st,
+                                  const JitProgram *jp) {
+  const int k = sizeof(OffT) == 8 ? 1 : 0;
+  Part<OffT> P = make_part<OffT>(g);
+  uint64_t launches = 0;
+  if (g->epoch_next > 0xF0000000u) {
+    CK(cudaMemsetAsync(g->stamp, 0, 4ull * std::max<uint64_t>(g->H.own_n(), 1), s));
+    g->epoch_next = 1;
+  }
+  Ctl h{};
+  h.epoch_base = g->epoch_next;
+  h.max_iters = o->max_iters;
+  h.trace_cap = g->trace_cap;
+  h.source = o->source;
+  h.damping = o->damping;
+  h.prof = o->profile ? 1 : 0;
+  h.kstart[0] = h.kstart[1] = ~0ull;
+  prd_setup(h, o, g->H.n);
+  if (g->cbits[0] && o->direction != GR_DIR_PUSH) {
+    uint32_t div = o->pull_div ? o->pull_div : kPullDivDefault;
+    if (const char *e = getenv("GR_PULL_DIV")) div = (uint32_t)strtoul(e, nullptr, 10);
+    h.pull_div = o->direction == GR_DIR_PULL ? 0xFFFFFFFFu : div;
+    CK(cudaMemsetAsync(g->cbits[0], 0, 4 * g->cbits_words, s));
+    CK(cudaMemsetAsync(g->cbits[1], 0, 4 * g->cbits_words, s));
+  }
+  CK(cudaMemcpyAsync(g->ctl, &h, sizeof h, cudaMemcpyHostToDevice, s));
+  gr_status r;
+  uint32_t src = o->source;
+  {
+    void *args[] = {(void *)&P, (void *)&src};
+    if ((r = jit_launch(jp->init_values[k], g->num_sms * 4, 256, args, 0, s, false)) != GR_OK) return r;
+  }
+  {
+    void *acc = g->hub_acc;
+    unsigned long long cnt = g->hub_cap;
+    void *args[] = {(void *)&acc, (void *)&cnt};
+    if ((r = jit_launch(jp->fill, std::min<uint32_t>((g->hub_cap + 255) / 256, 1024) + 1, 256, args, 0, s, false)) !=
+        GR_OK)
+      return r;
+  }
+  CK(cudaMemsetAsync(g->hub_done, 0, 4ull * g->hub_cap, s));
+  launches += 2;
+  if (jp->init == kInitAll && g->n_static_hubs) {
+    CK(cudaMemcpyAsync(g->listH[0], g->static_hubs, 4ull * g->n_static_hubs, cudaMemcpyDeviceToDevice, s));
+    CK(cudaMemcpyAsync(g->chkA_h[0], g->static_chk_h, 4ull * g->n_static_chunks, cudaMemcpyDeviceToDevice, s));
+    CK(cudaMemcpyAsync(g->chkA_c[0], g->static_chk_c, 4ull * g->n_static_chunks, cudaMemcpyDeviceToDevice, s));
+  }
+  {
+    uint32_t nh = (uint32_t)g->n_static_hubs, nc = (uint32_t)g->n_static_chunks;
+    void *args[] = {(void *)&P, (void *)&src, (void *)&nh, (void *)&nc};
+    if ((r = jit_launch(jp->init_frontier[k], 1, kBlock, args, 0, s, false)) != GR_OK) return r;
+  }
+  launches++;
+  int bps = 0;
+  if ((r = jit_occupancy(jp->persistent[k], kBlock, &bps)) != GR_OK) return r;
+  int per_sm = std::min(bps, 4);
+  const uint32_t grid = (uint32_t)g->num_sms * (uint32_t)std::max(1, per_sm);
+  {
+    void *args[] = {(void *)&P};
+    if ((r = jit_launch(jp->persistent[k], grid, kBlock, args, 0, s, true)) != GR_OK) return r;
+  }
+  CK(cudaMemcpyAsync(g->h_ctl, g->ctl, sizeof(Ctl), cudaMemcpyDeviceToHost, s));
+  CK(cudaStreamSynchronize(s));
+  launches += 1;
+  const Ctl &c = *g->h_ctl;
+  if (o->profile) {
+    st->kernel_ms[0] += c.kns[0] * 1e-6;
+    st->kernel_ms[1] += c.kns[1] * 1e-6;
+  }
+  st->iterations = c.iter;
+  st->pull_supersteps = c.tot_pull;
+  st->edges_gathered = c.tot_gathered;
+  st->edges_scattered = c.tot_scattered;
+  st->kernel_launches += launches;
+  g->epoch_next = h.epoch_base + c.iter + 2;
+  g->trace_rows = std::min<uint64_t>(c.iter, g->trace_cap);
+  std::vector<unsigned long long> tr(4 * g->trace_rows);
+  if (g->trace_rows)
+    CK(cudaMemcpyAsync(tr.data(), g->trace, 32 * g->trace_rows, cudaMemcpyDeviceToHost, s));
+  CK(cudaStreamSynchronize(s));
+  uint64_t sumA = 0, sumC = 0;
+  for (uint64_t t = 0; t < g->trace_rows; t++) { sumA += tr[4 * t]; sumC += tr[4 * t + 1]; }
+  const uint64_t wb = jp->uses_weights ? 5 : 4;
   st->bytes_hbm_model = wb * c.tot_gathered + 12 * sumA + 4 * c.tot_scattered + 12 * sumC;
   return GR_OK;
 }
@@ -974,11 +1066,19 @@ gr_status run(gr_graph *g, const gr_run_opts *oin, gr_run_stats *st) {
   if (o.algo == GR_SSSP && !g->H.has_w) return fail(GR_EINVAL, "SSSP needs edge weights");
   if (o.algo < GR_BFS || o.algo > GR_PAGERANK_DELTA) return fail(GR_EINVAL, "unknown algo %d", o.algo);
   if (o.direction < GR_DIR_AUTO || o.direction > GR_DIR_PULL) return fail(GR_EINVAL, "unknown direction %d", o.direction);
+  const JitProgram *jp = nullptr;
   if (o.algo == GR_CUSTOM) {
     bool known = false, uses_w = false;
 #define GR_X(id, T) if (o.custom_id == id) { known = true; uses_w = T::kUsesWeights; }
     GR_CUSTOM_PROGRAMS(GR_X)
 #undef GR_X
+    if (!known && (jp = jit_find(o.custom_id))) {
+      known = true;
+      uses_w = jp->uses_weights;
+      if (g->mode == GR_MODE_STREAMED || g->comm || !g->coop)
+        return fail(GR_EUNSUPPORTED, "run-time program %d: resident single-GPU graphs only (persistent loop)",
+                    o.custom_id);
+    }
     if (!known) return fail(GR_EUNSUPPORTED, "no custom program with id %d is registered", o.custom_id);
     if (uses_w && !g->H.has_w) return fail(GR_EINVAL, "custom program %d needs edge weights", o.custom_id);
     if (o.source >= g->H.n) return fail(GR_EINVAL, "source %u >= num_vertices", o.source);
@@ -1015,6 +1115,7 @@ gr_status run(gr_graph *g, const gr_run_opts *oin, gr_run_stats *st) {
       break;
     case GR_CUSTOM:
       r = GR_EUNSUPPORTED;
+      if (jp) r = g->off64 ? run_frontier_jit<uint64_t>(g, &o, s, st, jp) : run_frontier_jit<uint32_t>(g, &o, s, st, jp);
 #define GR_X(id, T)                                                                                        \
   if (o.custom_id == id)                                                                                   \
     r = g->off64 ? run_frontier<T, uint64_t>(g, &o, s, st, 16 + id) : run_frontier<T, uint32_t>(g, &o, s, st, 16 + id);

@@ -442,7 +442,12 @@ __device__ void close_superstep(const Part<OffT> &P, unsigned long long cond_han
   const bool stop = !c->ext_loop && (empty || (c->max_iters != 0 && t + 1 >= c->max_iters));
   c->stop = stop ? 1u : 0u;
   __threadfence();
+#ifndef GR_JIT  // run-time compiled programs (jit.cpp) run only the persistent loop: no conditional graph node
   if (use_graph) cudaGraphSetConditional((cudaGraphConditionalHandle)cond_handle, stop ? 0u : 1u);
+#else
+  (void)cond_handle;
+  (void)use_graph;
+#endif
 }
 
 

@@ -40,6 +40,21 @@ def test_no_gpu_fails_cleanly():
     assert ei.value.status == gr.GR_ECUDA
 
 
+def test_program_compile_argument_errors():
+    """gr_program_compile rejects bad arguments before doing
+    any work, and without a GPU fails with a status instead of crashing."""
+    import torch
+
+    for name in ("", "1abc", "bad name", "a;b"):
+        with pytest.raises(gr.GrError) as ei:
+            gr.gr_program_compile("struct X {};", name)
+        assert ei.value.status == gr.GR_EINVAL
+    if not torch.cuda.is_available():
+        with pytest.raises(gr.GrError) as ei:
+            gr.gr_program_compile("struct X {};", "X")
+        assert ei.value.status in (gr.GR_ECUDA, gr.GR_EUNSUPPORTED)
+
+
 @pytest.mark.parametrize("P_target", [1 << 26, 5000, 700])
 def test_host_layout_invariants(P_target):
     g = grgen.rmat(12, 16, seed=21)
