@@ -15,9 +15,11 @@ namespace gr {
 // ------------------------------------------------------------------- NCCL
 struct NcclComm : Comm {
   ncclComm_t comm = nullptr;
-  uint64_t *d_small = nullptr;  // world * 8 u64 scratch
+  uint64_t *d_small = nullptr;  // world * 8 u64 scratch (+1 word for the barrier)
   uint64_t *h_small = nullptr;
+  std::vector<void *> opened;   // cudaIpcOpenMemHandle mappings of peer buffers
   ~NcclComm() override {
+    for (void *p : opened) cudaIpcCloseMemHandle(p);
     if (comm) ncclCommDestroy(comm);
     if (d_small) cudaFree(d_small);
     if (h_small) cudaFreeHost(h_small);
@@ -46,6 +48,35 @@ struct NcclComm : Comm {
     for (int q = 0; q < world; q++)
       for (int i = 0; i < k; i++) out[q * k + i] = h_small[q * 8 + i];
     return GR_OK;
+  }
+  gr_status share_buffer(void *local, std::vector<void *> *out, cudaStream_t s) override {
+    static_assert(sizeof(cudaIpcMemHandle_t) == 64, "IPC handle is 8 words");
+    cudaIpcMemHandle_t h;
+    if (cudaIpcGetMemHandle(&h, local) != cudaSuccess) return GR_ECUDA;
+    uint64_t mine[8], all[8 * 64];
+    if (world > 64) return GR_EUNSUPPORTED;
+    std::memcpy(mine, &h, 64);
+    gr_status st = allgather_small(mine, 8, all, s);
+    if (st != GR_OK) return st;
+    out->assign(world, nullptr);
+    (*out)[rank] = local;
+    for (int q = 0; q < world; q++) {
+      if (q == rank) continue;
+      cudaIpcMemHandle_t hq;
+      std::memcpy(&hq, all + 8 * q, 64);
+      void *p = nullptr;
+      if (cudaIpcOpenMemHandle(&p, hq, cudaIpcMemLazyEnablePeerAccess) != cudaSuccess) {
+        cudaGetLastError();
+        return GR_ECUDA;
+      }
+      opened.push_back(p);
+      (*out)[q] = p;
+    }
+    return GR_OK;
+  }
+  gr_status barrier(cudaStream_t s) override {
+    uint64_t *w = d_small + 8ull * world;
+    return ncclAllReduce(w, w, 1, ncclUint64, ncclSum, comm, s) == ncclSuccess ? GR_OK : GR_ENCCL;
   }
 };
 
@@ -122,6 +153,20 @@ struct SimComm : Comm {
     if (!grp->barrier()) return GR_ENCCL;
     return GR_OK;
   }
+  gr_status share_buffer(void *local, std::vector<void *> *out, cudaStream_t s) override {
+    if (cudaStreamSynchronize(s) != cudaSuccess) return fail_all(GR_ECUDA);
+    grp->ptrs[rank] = local;
+    if (!grp->barrier()) return GR_ENCCL;
+    out->resize(world);
+    for (int q = 0; q < world; q++) (*out)[q] = const_cast<void *>(grp->ptrs[q]);
+    if (!grp->barrier()) return GR_ENCCL;  // ptrs is reused by the next exchange
+    return GR_OK;
+  }
+  gr_status barrier(cudaStream_t s) override {
+    // ranks share one device: wait for this rank's work, then for every rank's
+    if (cudaStreamSynchronize(s) != cudaSuccess) return fail_all(GR_ECUDA);
+    return grp->barrier() ? GR_OK : GR_ENCCL;
+  }
 };
 
 gr_status comm_create(int world, int rank, bool sim, const void *id128, int device, Comm **out, std::string *err) {
@@ -169,7 +214,8 @@ gr_status comm_create(int world, int rank, bool sim, const void *id128, int devi
     delete c;
     return GR_ENCCL;
   }
-  if (cudaMalloc(&c->d_small, 64ull * world) != cudaSuccess || cudaMallocHost(&c->h_small, 64ull * world) != cudaSuccess) {
+  if (cudaMalloc(&c->d_small, 64ull * world + 64) != cudaSuccess ||
+      cudaMallocHost(&c->h_small, 64ull * world) != cudaSuccess) {
     delete c;
     *err = "comm scratch allocation failed";
     return GR_ENOMEM;

@@ -29,6 +29,16 @@ struct Comm {
                                const std::vector<uint64_t> &displs, cudaStream_t s) = 0;
   // allgather of k host uint64 per rank (synchronous w.r.t. s): out[r*k + i]
   virtual gr_status allgather_small(const uint64_t *mine, int k, uint64_t *out, cudaStream_t s) = 0;
+  // Map every rank's device buffer `local` into this rank: out[q] is rank q's
+  // buffer (out[rank] = local). NCCL: cudaIpc handles exchanged with
+  // allgather_small and opened with peer access (NVLink); the mappings are
+  // closed when the Comm is destroyed. Simulated: the pointers themselves.
+  // `local` must come from cudaMalloc (IPC-exportable).
+  virtual gr_status share_buffer(void *local, std::vector<void *> *out, cudaStream_t s) = 0;
+  // Stream-ordered barrier: work enqueued on s after it starts only when every
+  // rank's work enqueued before its barrier has completed (so peer stores of
+  // those kernels are visible). NCCL: a one-word allreduce; simulated: host.
+  virtual gr_status barrier(cudaStream_t s) = 0;
 };
 
 // Create the communicator for a loaded partition. world <= 1 returns nullptr.

@@ -230,8 +230,16 @@ gr_status load_device(gr_graph *g) {
   if ((s = dev_alloc(g, (void **)&g->inv_outdeg, 4 * n)) != GR_OK) return s;
   k_inv_outdeg<<<g->num_sms * 4, 256, 0, g->stream>>>((uint32_t)n, g->d_outdeg, g->inv_outdeg);
   CK(cudaGetLastError());
-  for (int i = 0; i < 2; i++)
-    if ((s = dev_alloc(g, (void **)&g->contrib[i], 4 * n)) != GR_OK) return s;
+  for (int i = 0; i < 2; i++) {
+    if (H.owners.size() > 2) {
+      // partitioned: plain cudaMalloc so the replica can be exported to the peers (cudaIpc)
+      CK(cudaMalloc((void **)&g->contrib[i], 4 * std::max<uint64_t>(n, 1)));
+      g->plain_allocs.push_back(g->contrib[i]);
+      g->dev_bytes += 4 * n;
+    } else if ((s = dev_alloc(g, (void **)&g->contrib[i], 4 * n)) != GR_OK) {
+      return s;
+    }
+  }
   if ((s = dev_alloc(g, (void **)&g->rank, 4 * ow)) != GR_OK) return s;
   const uint64_t items = own_n + mi;
   g->pr_tiles = (uint32_t)((items + kPrTile - 1) / kPrTile);
@@ -550,6 +558,11 @@ template <class OffT> static PrArgs<OffT> pr_args(gr_graph *g, uint32_t t, uint3
   a.base = (1.0f - d) / (float)g->H.n;
   a.d = d;
   a.last = (t + 1 == iters) ? 1 : 0;
+  if (g->pr_p2p_on && !a.last) {  // fused exchange: the apply also stores into every peer's replica
+    static_assert(kMaxPeers == 15, "gr_graph::pr_peer size");
+    for (uint32_t q = 0; q < g->pr_npeer; q++) a.peer[q] = g->pr_peer[(t + 1) & 1][q];
+    a.npeer = g->pr_npeer;
+  }
   return a;
 }
 
@@ -739,7 +752,9 @@ template <class OffT> static gr_status pr_bseg_setup(gr_graph *g, uint32_t S) {
 template <class OffT> static gr_status pr_hot_setup(gr_graph *g) {
   g->pr_hot = 0;
   const HostGraph &H = g->H;
-  const bool hot_ok = g->mode == GR_MODE_RESIDENT && !g->comm && H.n < 0x80000000ull && H.m_in >= (1u << 20);
+  uint64_t hot_min = 1u << 20;  // below ~1M edges the plain warp kernel is as fast
+  if (const char *hm = getenv("GR_PR_HOT_MIN_EDGES")) hot_min = strtoull(hm, nullptr, 10);  // tests
+  const bool hot_ok = g->mode == GR_MODE_RESIDENT && H.n < 0x80000000ull && H.m_in >= hot_min && H.m_in > 0;
   const bool seg_ok = hot_ok && (uint64_t)H.own_n() + H.m_in + 2 * kSegTile < 0xFFFFFFFFull;
   // source block for the blocked layout: the contributions of one block must stay in L2
   uint64_t block_mb = 64;  // measured on R-MAT s26: 24 MB 4.81, 40 MB 4.52, 64 MB 4.42 ms per superstep
@@ -809,6 +824,7 @@ template <class OffT> static gr_status pr_hot_setup(gr_graph *g) {
     // persistent loop: one cooperative launch for all supersteps (GR_PR_LOOP=0: one launch per phase)
     g->pr_loop = g->coop ? 1 : 0;
     if (const char *pl = getenv("GR_PR_LOOP")) g->pr_loop = g->coop && atoi(pl) != 0;
+    if (g->comm) g->pr_loop = 0;  // partitioned: one launch per phase, the exchange between supersteps
     if (g->pr_loop) {
       int lbps = 0;
       CK(cudaFuncSetAttribute(seg_loop_kernel<OffT>(g->seg_var), cudaFuncAttributeMaxDynamicSharedMemorySize,
@@ -901,6 +917,19 @@ static void pr_launch_iter(gr_graph *g, cudaStream_t s, uint32_t t, uint32_t ite
   }
   else
     k_pr_fixup<OffT><<<std::max<uint32_t>((tiles + 255) / 256, 1), 256, 0, s>>>(a, tiles);
+}
+
+// Partitioned PageRank (engine_part.cu): the same per-superstep kernels over the
+// rank's owned rows (hot table + edge-segmented tiles when they apply).
+gr_status pr_part_prepare(gr_graph *g) {
+  if (g->pr_hot >= 0) return GR_OK;
+  return g->off64 ? pr_hot_setup<uint64_t>(g) : pr_hot_setup<uint32_t>(g);
+}
+uint32_t pr_part_iter(gr_graph *g, cudaStream_t s, uint32_t t, uint32_t iters, float d) {
+  if (g->off64) pr_launch_iter<uint64_t>(g, s, t, iters, d, nullptr, nullptr);
+  else pr_launch_iter<uint32_t>(g, s, t, iters, d, nullptr, nullptr);
+  const bool warp = g->pr_kernel >= 2;
+  return (g->pr_hot == 1 ? 1u : 0u) + 2u + (warp && g->n_long && g->pr_kernel != 4 && g->pr_kernel != 5 ? 1u : 0u);
 }
 
 template <class OffT>
@@ -1183,6 +1212,7 @@ void destroy(gr_graph *g) {
   delete g->comm;
   g->comm = nullptr;
   for (void *p : g->allocs) cudaFreeAsync(p, g->stream);
+  for (void *p : g->plain_allocs) cudaFree(p);
   cudaStreamSynchronize(g->stream);
   if (g->h_ctl) cudaFreeHost(g->h_ctl);
   if (g->stream) cudaStreamDestroy(g->stream);

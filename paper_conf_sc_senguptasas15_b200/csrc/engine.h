@@ -111,6 +111,13 @@ struct gr_graph {
   bool sim = false;
   uint32_t *X_v = nullptr, *X_val = nullptr;  // exchanged changed set
   float *rank_all = nullptr;                  // PageRank fetch assembly
+  // PageRank fused exchange: every other rank's contribution replica (by parity),
+  // peer-mapped (cudaIpc, NCCL mode) or same-device (simulated ranks)
+  float *pr_peer[2][15] = {};
+  uint32_t pr_npeer = 0;
+  bool pr_p2p = false;          // the mapping exists (set up at load)
+  bool pr_p2p_on = false;       // this run exchanges by peer stores (else NCCL allgatherv)
+  std::vector<void *> plain_allocs;  // cudaMalloc'ed (IPC-exportable) buffers
 };
 
 namespace gr {
@@ -173,6 +180,9 @@ inline void pfree(void *p, cudaStream_t s) {
 gr_status load_device(gr_graph *g);
 gr_status device_build(gr_graph *g, const gr_edges *E, uint64_t shard_edges);
 gr_status select_hot(gr_graph *g, uint64_t K, uint32_t **hot_ids, uint32_t *hot_k, uint32_t **d_slot);
+// partitioned PageRank (engine.cu): kernel/layout selection once per graph, one superstep's launches
+gr_status pr_part_prepare(gr_graph *g);
+uint32_t pr_part_iter(gr_graph *g, cudaStream_t s, uint32_t t, uint32_t iters, float d);
 gr_status run(gr_graph *g, const gr_run_opts *o, gr_run_stats *st);
 gr_status fetch_values(gr_graph *g, void *dst, uint64_t bytes);
 gr_status fetch_trace(gr_graph *g, uint64_t *dst, uint64_t max_rows, uint64_t *rows);

@@ -13,6 +13,8 @@
 #include <cuda_runtime.h>
 
 #include <algorithm>
+#include <cstdlib>
+#include <string>
 #include <vector>
 
 #include "comm.h"
@@ -41,6 +43,29 @@ gr_status part_setup(gr_graph *g) {
   if ((s = dev_alloc(g, (void **)&g->X_v, 4 * n)) != GR_OK) return s;
   if ((s = dev_alloc(g, (void **)&g->X_val, 4 * n)) != GR_OK) return s;
   if ((s = dev_alloc(g, (void **)&g->rank_all, 4 * n)) != GR_OK) return s;
+  // PageRank fused exchange: map every peer's contribution replicas (both
+  // parities). Without a mapping (no peer access) PageRank exchanges with NCCL.
+  Comm *C = g->comm;
+  g->pr_p2p = false;
+  g->pr_npeer = 0;
+  if (C->world - 1 <= 15 && g->contrib[0] && g->contrib[1]) {
+    std::vector<void *> p0, p1;
+    gr_status a = C->share_buffer(g->contrib[0], &p0, g->stream);
+    gr_status b = a == GR_OK ? C->share_buffer(g->contrib[1], &p1, g->stream) : a;
+    if (b == GR_OK) {
+      for (int q = 0; q < C->world; q++) {
+        if (q == C->rank) continue;
+        g->pr_peer[0][g->pr_npeer] = static_cast<float *>(p0[q]);
+        g->pr_peer[1][g->pr_npeer] = static_cast<float *>(p1[q]);
+        g->pr_npeer++;
+      }
+      g->pr_p2p = true;
+    } else if (b == GR_ENCCL) {
+      return fail(b, "PageRank replica mapping: exchange failed");
+    } else {
+      g->pr_npeer = 0;  // every rank reaches the same allgather_small calls; fall back to NCCL
+    }
+  }
   return GR_OK;
 }
 
@@ -152,6 +177,16 @@ gr_status run_frontier_part(gr_graph *g, const gr_run_opts *o, cudaStream_t s, g
   return GR_OK;
 }
 
+// PageRank over owner partitions. Each rank runs the single-GPU superstep
+// kernels (hot-source table + edge-segmented tiles when they apply) over its
+// owned rows, reading the full contribution replica. The exchange of the owned
+// contribution slices is FUSED into the apply (default): every contribution is
+// stored into the local replica and, through the peer mappings, into every
+// other rank's replica for superstep t+1, so the slices travel over NVLink
+// while the rest of the gather runs; a stream-ordered barrier (one-word NCCL
+// allreduce) then orders superstep t+1 after every rank's stores.
+// GR_PR_EXCHANGE=nccl (or no peer mapping): allgatherv of the owned slices
+// after each superstep instead.
 template <class OffT>
 gr_status run_pagerank_part(gr_graph *g, const gr_run_opts *o, cudaStream_t s, gr_run_stats *st) {
   Comm *C = g->comm;
@@ -160,41 +195,34 @@ gr_status run_pagerank_part(gr_graph *g, const gr_run_opts *o, cudaStream_t s, g
   const uint32_t lo = (uint32_t)g->H.own_lo;
   std::vector<uint64_t> cnt, dsp;
   owner_bytes(g, 4, &cnt, &dsp);
+  gr_status ps = pr_part_prepare(g);
+  if (ps != GR_OK) return ps;
+  bool p2p = g->pr_p2p;
+  if (const char *x = getenv("GR_PR_EXCHANGE")) p2p = p2p && std::string(x) != "nccl";
+  g->pr_p2p_on = p2p;
+  uint64_t launches = 1;
   k_pr_init<<<g->num_sms * 4, 256, 0, s>>>((uint32_t)g->H.n, g->inv_outdeg, g->contrib[0]);
+  // every replica is initialised before any rank's first fused store lands in it
+  if (p2p) XCK(C->barrier(s));
   for (uint32_t t = 0; t < iters; t++) {
-    PrArgs<OffT> a{};
-    a.n = (uint32_t)g->H.n;
-    a.own_lo = lo;
-    a.own_n = (uint32_t)g->H.own_n();
-    a.m_in = g->H.m_in;
-    a.in_off = (const OffT *)g->in_off;
-    a.in_src = g->in_src;
-    a.inv_outdeg = g->inv_outdeg;
-    a.contrib_in = g->contrib[t & 1];
-    a.contrib_out = g->contrib[(t + 1) & 1];
-    a.rank = g->rank;
-    a.carry_row = g->carry_row;
-    a.carry_val = g->carry_val;
-    a.head_row = g->head_row;
-    a.head_val = g->head_val;
-    a.tile_row = g->tile_row;
-    a.base = (1.0f - d) / (float)g->H.n;
-    a.d = d;
-    a.last = (t + 1 == iters) ? 1 : 0;
-    k_pr_gather_apply<OffT><<<std::max<uint32_t>(g->pr_tiles, 1), kPrThreads, 0, s>>>(a);
-    k_pr_fixup<OffT><<<std::max<uint32_t>((g->pr_tiles + 255) / 256, 1), 256, 0, s>>>(a, g->pr_tiles);
+    launches += pr_part_iter(g, s, t, iters, d);
     PCK(cudaGetLastError());
-    if (!a.last) {
+    if (t + 1 == iters) break;
+    if (p2p) {
+      XCK(C->barrier(s));
+      C->bytes_in += 4 * (g->H.n - g->H.own_n());
+    } else {
       float *out = g->contrib[(t + 1) & 1];
       XCK(C->allgatherv(out + lo, out, cnt, dsp, s));  // owned slices -> every replica
     }
   }
+  g->pr_p2p_on = false;
   PCK(cudaStreamSynchronize(s));
   st->iterations = iters;
   uint64_t mi = g->H.m_in, tot = 0;
   XCK(global_sum(C, mi, &tot, s));
   st->edges_gathered = (uint64_t)iters * tot;
-  st->kernel_launches += 1 + 2ull * iters;
+  st->kernel_launches += launches;
   st->bytes_nvlink = C->bytes_in;
   st->bytes_hbm_model = (uint64_t)iters * (4 * g->H.m_in + 12 * g->H.own_n() + 4 * g->H.n);
   g->trace_rows = iters;

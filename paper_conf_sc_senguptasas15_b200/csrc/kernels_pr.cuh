@@ -19,6 +19,7 @@
 namespace gr {
 
 constexpr int kPrThreads = 256;
+constexpr int kMaxPeers = 15;  // partitioned PageRank: peers written by the fused exchange
 constexpr int kPrIpt = 8;
 constexpr int kPrTile = kPrThreads * kPrIpt;
 constexpr uint32_t kNoRow = 0xFFFFFFFFu;
@@ -46,14 +47,28 @@ template <class OffT> struct PrArgs {
   const uint32_t *tile_row;  // [num_tiles + 1] merge-path row coordinate of each tile start (precomputed)
   float base, d;             // (1-d)/n, d
   int last;                  // 1: write rank instead of contrib_out
+  // Partitioned runs, fused exchange: the other ranks' contribution
+  // replicas of superstep t+1 (peer-mapped over NVLink, or same-device buffers of
+  // simulated ranks). Every owned contribution the apply writes is stored into
+  // each of them as well, so the allgather of the owned slices is done by the
+  // apply's own stores, row by row, while the gather of other rows continues.
+  float *peer[kMaxPeers];
+  uint32_t npeer;
 };
+
+// contribution of owned vertex v for superstep t+1: the local replica, then every peer's
+template <class OffT>
+__device__ __forceinline__ void pr_store_contrib(const PrArgs<OffT> &a, uint32_t v, float c) {
+  a.contrib_out[v] = c;
+  for (uint32_t q = 0; q < a.npeer; q++) a.peer[q][v] = c;
+}
 
 template <class OffT>
 __device__ __forceinline__ void pr_apply_row(const PrArgs<OffT> &a, uint32_t lrow, float acc) {
   const float R = a.base + a.d * acc;
   const uint32_t v = a.own_lo + lrow;
   if (a.last) a.rank[lrow] = R;
-  else a.contrib_out[v] = R * __ldg(a.inv_outdeg + v);
+  else pr_store_contrib(a, v, R * __ldg(a.inv_outdeg + v));
 }
 
 // Merge-path search over (row ends, edge indices) for diagonal `diag`.
@@ -439,7 +454,7 @@ __global__ void __launch_bounds__(1024, 1) k_pr_warp_pipe(const __grid_constant_
       const float R = a.base + a.d * S.s_tot[pr_pad(k)];
       const uint32_t lrow = i0 + k;
       if (a.last) a.rank[lrow] = R;
-      else a.contrib_out[a.own_lo + lrow] = R * (k < 32 ? inv0 : __ldg(a.inv_outdeg + a.own_lo + lrow));
+      else pr_store_contrib(a, a.own_lo + lrow, R * (k < 32 ? inv0 : __ldg(a.inv_outdeg + a.own_lo + lrow)));
     }
     if (lane == 0) {
       a.head_row[tile] = head ? i0 : kNoRow;
@@ -595,7 +610,7 @@ __device__ __forceinline__ void seg_tile(const PrArgs<OffT> &a, uint32_t tile, u
       } else {
         const float R = a.base + a.d * run;
         if (a.last) a.rank[row] = R;
-        else a.contrib_out[a.own_lo + row] = R * seg_ldf<kVar>(a.inv_outdeg + a.own_lo + row);
+        else pr_store_contrib(a, a.own_lo + row, R * seg_ldf<kVar>(a.inv_outdeg + a.own_lo + row));
       }
     }
   }
@@ -613,7 +628,7 @@ __device__ __forceinline__ void seg_tile(const PrArgs<OffT> &a, uint32_t tile, u
     if ((int)lane >= first && (int)lane <= lastc && myrow < a.own_n) {
       const float R = s_R[lane];
       if (a.last) a.rank[myrow] = R;
-      else a.contrib_out[a.own_lo + myrow] = R * pre_inv;
+      else pr_store_contrib(a, a.own_lo + myrow, R * pre_inv);
     }
     __syncwarp();
   }

@@ -120,3 +120,25 @@ def test_sim_ranks_custom_program():
     for vals, tr in out:
         np.testing.assert_array_equal(vals, ref)
         np.testing.assert_array_equal(tr, rtr)
+
+
+@pytest.mark.timeout(900)
+@pytest.mark.parametrize("G", [2, 4])
+@pytest.mark.parametrize("exchange", ["p2p", "nccl"])
+@pytest.mark.parametrize("hot_min", ["0", "default"])
+def test_sim_ranks_pagerank_exchange(G, exchange, hot_min, monkeypatch):
+    """Partitioned PageRank, both exchanges: the apply's fused stores into every
+    peer replica (p2p; same-device buffers of the simulated ranks stand in for
+    the NVLink peer mappings) and the allgatherv of the owned slices (nccl);
+    with the hot-table edge-segmented tiles (hot_min 0) and the plain warp tiles."""
+    monkeypatch.setenv("GR_PR_EXCHANGE", exchange)
+    if hot_min != "default":
+        monkeypatch.setenv("GR_PR_HOT_MIN_EDGES", hot_min)
+    g = grgen.rmat(14, 16, seed=11)
+    ref, _, _ = oracle.run(g.n, g.src, g.dst, "pagerank", max_iters=30)
+    res = run_sim_ranks(g.n, g.src, g.dst, None, G, "pagerank", max_iters=30)
+    for st, vals, tr, info in res:
+        check_pr(vals, ref, g.n)
+        assert st["iterations"] == 30
+        own = info["own_hi"] - info["own_lo"]
+        assert st["bytes_nvlink"] == 29 * 4 * (g.n - own)  # every other rank's slice, once per exchange
