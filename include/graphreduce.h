@@ -126,7 +126,12 @@ typedef struct gr_run_opts {
 typedef enum gr_direction {
   GR_DIR_AUTO = 0,  /* pull when the changed set is large (|C_t| * pull_div > |V|), else push */
   GR_DIR_PUSH = 1,  /* always expand the out-edges of C_t (stamps + atomics) */
-  GR_DIR_PULL = 2   /* always scan the in-edges of every vertex for a changed source */
+  GR_DIR_PULL = 2,  /* always scan the in-edges of every vertex for a changed source */
+  GR_DIR_FUSED = 3  /* programs declaring kPushFused (SSSP, widest path; gr/program.cuh): apply and
+                       a push FrontierActivate that carries the gather (atomicGather into a per-vertex
+                       accumulator) run as ONE phase per superstep (resident single-rank graphs;
+                       measured slower than AUTO on the road grid, so opt-in); other programs
+                       and modes treat FUSED as AUTO */
 } gr_direction;
 
 typedef struct gr_run_stats {

@@ -28,7 +28,7 @@ FLOAT_ALGOS = ("pagerank", "pagerank_delta")
 MODES = {"auto": 0, "resident": 1, "streamed": 2}
 LOOPS = {"auto": 0, "host": 1, "device": 2, "persistent": 3}
 BUILDS = {"auto": 0, "host": 1, "device": 2}
-DIRECTIONS = {"auto": 0, "push": 1, "pull": 2}
+DIRECTIONS = {"auto": 0, "push": 1, "pull": 2, "fused": 3}
 INF = 0xFFFFFFFF
 
 EXPORTS = [

@@ -58,6 +58,7 @@ struct Ctl {
   uint32_t tot_pull;      // supersteps that activated by pull
   uint32_t dense;         // superstep `iter` gathers densely (previous activation was by pull)
   uint32_t prd_r0;        // ProgPRDelta constants (Ctx)
+  uint32_t push;          // fused push supersteps (gr/program.cuh kPushFused): one phase per superstep
   unsigned long long prd_base, prd_dq;
   double prd_thr;
 };
@@ -83,7 +84,7 @@ __device__ __forceinline__ unsigned long long block_sum_u64(unsigned long long x
 struct View {
   uint32_t stop, t, epoch_base, implicit0, no_hub_c, source, prof;
   uint32_t cntA[2], cntK[2], cntH[2], cntC, cntCH, cntKC;
-  uint32_t pull_div, pull_pending, dirty[2], dense;
+  uint32_t pull_div, pull_pending, dirty[2], dense, push;
   float damping;
   unsigned long long prd_base, prd_dq;
   double prd_thr;
@@ -101,7 +102,7 @@ __device__ __forceinline__ void load_view(const Ctl *c, View &v) {
     const uint32_t h0 = vc->cnt_H[0], h1 = vc->cnt_H[1], ch = vc->cnt_CH;
     const uint32_t pd = vc->pull_div, pp = vc->pull_pending, d0 = vc->dirty[0], d1 = vc->dirty[1], dn = vc->dense;
     v.cntH[0] = h0; v.cntH[1] = h1; v.cntCH = ch;
-    v.pull_div = pd; v.pull_pending = pp; v.dirty[0] = d0; v.dirty[1] = d1; v.dense = dn;
+    v.pull_div = pd; v.pull_pending = pp; v.dirty[0] = d0; v.dirty[1] = d1; v.dense = dn; v.push = vc->push;
     v.prd_base = vc->prd_base; v.prd_dq = vc->prd_dq; v.prd_thr = vc->prd_thr;
     v.cntA[0] = a0; v.cntA[1] = a1; v.cntK[0] = k0; v.cntK[1] = k1;
     v.stop = st; v.t = t; v.epoch_base = eb; v.implicit0 = im; v.no_hub_c = nh;
@@ -151,6 +152,8 @@ template <class OffT> struct Part {
   uint32_t *cbits[2];     // changed-set bitmaps over V for pull activation (by superstep parity)
   uint32_t *hub_act;      // per static hub: some chunk saw a marked source (dense gathers)
   const uint32_t *s_hubs, *s_chk_h, *s_chk_c;  // static in-hub list and its chunks (dense gathers)
+  uint32_t *nxt[2];       // fused push supersteps: per-vertex gather accumulators by parity (GatherT = u32)
+  const uint8_t *out_w;   // activation CSR weights (fused push supersteps of weighted programs)
   uint32_t n_s_hubs, n_s_chunks;
   Ctl *ctl;
   unsigned long long *trace; // [trace_cap][4]

@@ -296,9 +296,47 @@ gr_status load_device(gr_graph *g) {
 }
 
 // -------------------------------------------------------------- frontier run
+// Fused push state (once per graph): the two accumulator arrays and, for
+// weighted programs, the activation CSR's weights. The CSR is the CSC
+// transposed by a stable sort of the CSC sources (device build, or the host
+// layout sorted the same way), so the same stable sort carrying the CSC
+// weights yields them in CSR order.
+static gr_status push_setup(gr_graph *g, bool weights) {
+  const uint64_t n = g->H.n, m = g->H.m_in;
+  cudaStream_t s = g->stream;
+  gr_status st;
+  for (int i = 0; i < 2; i++)
+    if (!g->nxt[i] && (st = dev_alloc(g, (void **)&g->nxt[i], 4 * std::max<uint64_t>(n, 1))) != GR_OK) return st;
+  if (!weights || g->out_w) return GR_OK;
+  if (!g->in_w) return fail(GR_EINVAL, "fused push: the program reads weights but the graph has none");
+  if ((st = dev_alloc(g, (void **)&g->out_w, m + 16)) != GR_OK) return st;
+  CK(cudaMemsetAsync(g->out_w + m, 0, 16, s));
+  uint32_t bits = 1;
+  while ((1ull << bits) < n) bits++;
+  uint32_t *kscratch = nullptr;
+  void *tmp = nullptr;
+  size_t need = 0;
+  CK(pmalloc(&kscratch, 4 * std::max<uint64_t>(m, 1), s));
+  CK(cub::DeviceRadixSort::SortPairs(nullptr, need, g->in_src, kscratch, g->in_w, g->out_w, (int64_t)m, 0,
+                                     (int)bits, s));
+  CK(pmalloc(&tmp, std::max<size_t>(need, 16), s));
+  CK(cub::DeviceRadixSort::SortPairs(tmp, need, g->in_src, kscratch, g->in_w, g->out_w, (int64_t)m, 0, (int)bits,
+                                     s));
+  pfree(tmp, s);
+  pfree(kscratch, s);
+  CK(cudaStreamSynchronize(s));
+  return GR_OK;
+}
+
 template <class Prog, class OffT>
-static void launch_body(gr_graph *g, cudaStream_t s, unsigned long long cond, int use_graph, uint64_t *launches) {
+static void launch_body(gr_graph *g, cudaStream_t s, unsigned long long cond, int use_graph, uint64_t *launches,
+                        bool push) {
   Part<OffT> P = make_part<OffT>(g);
+  if (push) {  // fused push superstep: one kernel
+    k_push_expand<Prog, OffT><<<g->grid_frontier, kBlock, 0, s>>>(P, cond, use_graph);
+    *launches += 1;
+    return;
+  }
   if (Prog::kHasGather) {
     k_gather_apply<Prog, OffT><<<g->grid_frontier, kBlock, 0, s>>>(P);
     k_activate<OffT><<<g->grid_frontier, kBlock, 0, s>>>(P, cond, use_graph);
@@ -314,7 +352,9 @@ static void launch_body(gr_graph *g, cudaStream_t s, unsigned long long cond, in
 }
 
 template <class Prog, class OffT>
-static gr_status get_while_graph(gr_graph *g, int key, cudaGraphExec_t *out, uint64_t *per_iter_launches) {
+static gr_status get_while_graph(gr_graph *g, int key, cudaGraphExec_t *out, uint64_t *per_iter_launches,
+                                 bool push) {
+  if (push) key += 1000;
   auto it = g->while_exec.find(key);
   if (it != g->while_exec.end()) {
     *out = it->second.first;
@@ -337,7 +377,7 @@ static gr_status get_while_graph(gr_graph *g, int key, cudaGraphExec_t *out, uin
   CK(cudaStreamCreateWithFlags(&cs, cudaStreamNonBlocking));
   CK(cudaStreamBeginCaptureToGraph(cs, body, nullptr, nullptr, 0, cudaStreamCaptureModeThreadLocal));
   uint64_t l = 0;
-  launch_body<Prog, OffT>(g, cs, (unsigned long long)h, 1, &l);
+  launch_body<Prog, OffT>(g, cs, (unsigned long long)h, 1, &l, push);
   cudaGraph_t captured = body;
   cudaError_t e = cudaStreamEndCapture(cs, &captured);
   cudaStreamDestroy(cs);
@@ -368,8 +408,27 @@ static gr_status run_frontier(gr_graph *g, const gr_run_opts *o, cudaStream_t s,
   h.prof = o->profile ? 1 : 0;
   h.kstart[0] = h.kstart[1] = ~0ull;
   prd_setup(h, o, g->H.n);
+  // fused push supersteps (gr/program.cuh kPushFused): direction FUSED, resident, one rank.
+  // Not the AUTO choice: on cfg3 (road grid SSSP) one fused phase took 147 us per
+  // superstep against 29 + 28 us for the gather / activate pair (profiles/README.md).
+  bool push = false;
+  if constexpr (PushFused<Prog>::value) {
+    push = Prog::kInit == kInitSourceChanged && !g->comm && g->mode == GR_MODE_RESIDENT &&
+           o->direction == GR_DIR_FUSED;
+    if (const char *e = getenv("GR_PUSH_FUSED")) push = push && atoi(e) != 0;
+    if (push) {
+      gr_status ps = push_setup(g, Prog::kUsesWeights);
+      if (ps != GR_OK) return ps;
+      P = make_part<OffT>(g);
+      const uint32_t id = Prog::identity_host();
+      k_fill<uint32_t><<<g->num_sms * 4, 256, 0, s>>>(g->nxt[0], id, g->H.n);
+      k_fill<uint32_t><<<g->num_sms * 4, 256, 0, s>>>(g->nxt[1], id, g->H.n);
+      launches += 2;
+    }
+  }
+  h.push = push ? 1u : 0u;
   // activation direction (gr_direction); pull needs the bitmaps (resident, one rank)
-  if (g->cbits[0] && o->direction != GR_DIR_PUSH) {
+  if (g->cbits[0] && !push && o->direction != GR_DIR_PUSH) {
     uint32_t div = o->pull_div ? o->pull_div : kPullDivDefault;
     if (const char *e = getenv("GR_PULL_DIV")) div = (uint32_t)strtoul(e, nullptr, 10);
     h.pull_div = o->direction == GR_DIR_PULL ? 0xFFFFFFFFu : div;
@@ -406,7 +465,7 @@ static gr_status run_frontier(gr_graph *g, const gr_run_opts *o, cudaStream_t s,
   } else if (use_graph) {
     cudaGraphExec_t ex;
     uint64_t per = 0;
-    gr_status gs = get_while_graph<Prog, OffT>(g, key, &ex, &per);
+    gr_status gs = get_while_graph<Prog, OffT>(g, key, &ex, &per, push);
     if (gs != GR_OK) return gs;
     CK(cudaGraphLaunch(ex, s));
     CK(cudaMemcpyAsync(g->h_ctl, g->ctl, sizeof(Ctl), cudaMemcpyDeviceToHost, s));
@@ -414,7 +473,7 @@ static gr_status run_frontier(gr_graph *g, const gr_run_opts *o, cudaStream_t s,
     launches += per * std::max<uint32_t>(g->h_ctl->iter, 1);
   } else {
     for (;;) {
-      launch_body<Prog, OffT>(g, s, 0, 0, &launches);
+      launch_body<Prog, OffT>(g, s, 0, 0, &launches, push);
       CK(cudaGetLastError());
       CK(cudaMemcpyAsync(g->h_ctl, g->ctl, sizeof(Ctl), cudaMemcpyDeviceToHost, s));
       CK(cudaStreamSynchronize(s));
@@ -443,6 +502,9 @@ static gr_status run_frontier(gr_graph *g, const gr_run_opts *o, cudaStream_t s,
   for (uint64_t t = 0; t < g->trace_rows; t++) { sumA += tr[4 * t]; sumC += tr[4 * t + 1]; }
   const uint64_t wb = Prog::kUsesWeights ? 5 : 4;
   st->bytes_hbm_model = wb * c.tot_gathered + 12 * sumA + 4 * c.tot_scattered + 12 * sumC;
+  // fused push: no in-edge walk; per A_t vertex acc + value + offsets (16 B), per
+  // pushed edge destination (+ weight), per changed vertex value + offsets (12 B)
+  if (push) st->bytes_hbm_model = 16 * sumA + wb * c.tot_scattered + 12 * sumC;
   return GR_OK;
 }
 
@@ -1094,7 +1156,7 @@ gr_status run(gr_graph *g, const gr_run_opts *oin, gr_run_stats *st) {
     return fail(GR_EINVAL, "source %u >= num_vertices %llu", o.source, (unsigned long long)g->H.n);
   if (o.algo == GR_SSSP && !g->H.has_w) return fail(GR_EINVAL, "SSSP needs edge weights");
   if (o.algo < GR_BFS || o.algo > GR_PAGERANK_DELTA) return fail(GR_EINVAL, "unknown algo %d", o.algo);
-  if (o.direction < GR_DIR_AUTO || o.direction > GR_DIR_PULL) return fail(GR_EINVAL, "unknown direction %d", o.direction);
+  if (o.direction < GR_DIR_AUTO || o.direction > GR_DIR_FUSED) return fail(GR_EINVAL, "unknown direction %d", o.direction);
   const JitProgram *jp = nullptr;
   if (o.algo == GR_CUSTOM) {
     bool known = false, uses_w = false;

@@ -28,6 +28,8 @@ struct gr_graph {
   void *in_off = nullptr, *out_off = nullptr;     // OffT arrays
   uint32_t *in_src = nullptr, *out_dst = nullptr; // resident payloads
   uint8_t *in_w = nullptr;
+  uint8_t *out_w = nullptr;                       // CSR weights (built on first fused push run)
+  uint32_t *nxt[2] = {nullptr, nullptr};          // fused push accumulators (allocated on first use)
   uint32_t *hub_in = nullptr, *hub_out = nullptr, *static_hubs = nullptr;
   uint32_t n_static_hubs = 0;
   // hub chunk lists (kChunk edges per CTA work item)
@@ -130,6 +132,9 @@ template <class OffT> inline Part<OffT> make_part(gr_graph *g) {
   P.in_off = (const OffT *)g->in_off;
   P.in_src = g->in_src;
   P.in_w = g->in_w;
+  P.nxt[0] = g->nxt[0];
+  P.nxt[1] = g->nxt[1];
+  P.out_w = g->out_w;
   P.out_off = (const OffT *)g->out_off;
   P.out_dst = g->out_dst;
   P.hub_in = g->hub_in;

@@ -278,7 +278,7 @@ __device__ void append_hub_C(const Part<OffT> &P, uint32_t v, uint32_t nv) {
 // bit) is issued for the whole batch before any result is consumed, so a lane
 // keeps kBatch independent requests in flight instead of one dependent chain.
 // The first stamper of x appends it (BFS: only if still unvisited).
-template <bool kBfsFilter, class OffT>
+template <bool kBfsFilter, class OffT, bool kByOut = kBfsFilter>
 __device__ __forceinline__ uint32_t activate_batch(const Part<OffT> &P, const bool (&act)[kBatch],
                                                    const uint32_t (&x)[kBatch], uint32_t epoch,
                                                    const uint32_t *hub_bits, WarpQueue &qA, uint32_t slot) {
@@ -287,7 +287,7 @@ __device__ __forceinline__ uint32_t activate_batch(const Part<OffT> &P, const bo
 #pragma unroll
   for (int q = 0; q < kBatch; q++) {
     st[q] = act[q] ? ld_cg(P.stamp + (x[q] - P.own_lo)) : epoch;
-    hb[q] = act[q] && test_bit(hub_bits, kBfsFilter ? x[q] : x[q] - P.own_lo);  // issued with the stamp read
+    hb[q] = act[q] && test_bit(hub_bits, kByOut ? x[q] : x[q] - P.own_lo);  // issued with the stamp read
   }
   bool nw[kBatch];
 #pragma unroll
@@ -305,7 +305,7 @@ __device__ __forceinline__ uint32_t activate_batch(const Part<OffT> &P, const bo
 #pragma unroll
   for (int q = 0; q < kBatch; q++) {
     const bool hub = keep[q] && hb[q];
-    if (hub) append_hub_A<kBfsFilter>(P, x[q], slot);
+    if (hub) append_hub_A<kByOut>(P, x[q], slot);
     qA.push(keep[q] && !hub, x[q], 0, P.listA[slot], nullptr, &P.ctl->cnt_A[slot]);
     cnt += __popc(__ballot_sync(0xffffffffu, nw[q]));
   }
@@ -954,6 +954,200 @@ __global__ void __launch_bounds__(kBlock) k_bfs_expand(const __grid_constant__ P
   finish_superstep(P, cond, use_graph, kPush);
 }
 
+// ------------------------------------------------------ fused push supersteps
+// Programs with kPushFused (gr/program.cuh; SSSP, widest path), resident single
+// GPU: apply and FrontierActivate run as ONE phase per superstep and the gather
+// rides on the activation. For v in A_t: r = acc_t[v] (the atomicGather of the
+// pushes of C_{t-1}), apply(&val[v], r); if v changed, every out-edge (v -> x)
+// does atomicGather(&acc_{t+1}[x], gatherMap(new[v], w)) and stamps x into
+// A_{t+1}. acc is double-buffered by superstep parity and reset when consumed.
+// Values, changed sets and the trace equal the BSP gather over all in-edges
+// (see program.cuh); Sigma_{A_t} indeg is counted from the offsets. BFS's phase
+// fusion (L276) extended to selective monotone gathers: one grid barrier per
+// superstep instead of three, and no in-edge walk.
+template <class Prog, class OffT>
+__device__ __forceinline__ uint32_t push_batch(const Part<OffT> &P, const bool (&act)[kBatch],
+                                               const uint32_t (&x)[kBatch], const uint32_t (&gm)[kBatch],
+                                               uint32_t *accn, uint32_t epoch, WarpQueue &qA, uint32_t slot) {
+#pragma unroll
+  for (int q = 0; q < kBatch; q++)  // fire-and-forget (RED): read only after the barrier
+    if (act[q] && gm[q] != Prog::identity()) Prog::atomicGather(accn + x[q], gm[q]);
+  return activate_batch<false, OffT, true>(P, act, x, epoch, P.hub_out, qA, slot);
+}
+
+// Push the out-edges of up to 32 changed vertices (one per lane: vertex u, new
+// value nv, edges [beg, beg + deg), deg <= kHubDegree), walked 32*kBatch at a time.
+template <class Prog, class OffT>
+__device__ uint32_t expand_warp_push(const Part<OffT> &P, bool valid, uint64_t beg, uint32_t deg, uint32_t u,
+                                     uint32_t nv, const Ctx &cx, uint32_t *accn, uint32_t epoch, WarpQueue &qA,
+                                     uint32_t slot) {
+  const uint32_t lane = lane_id();
+  const uint32_t d = valid ? deg : 0u;
+  const uint32_t incl = warp_incl_scan(d);
+  const uint32_t excl = incl - d;
+  const uint32_t total = __shfl_sync(0xffffffffu, incl, 31);
+  uint32_t nact = 0;
+  for (uint32_t r0 = 0; r0 < total; r0 += 32u * kBatch) {
+    bool act[kBatch];
+    uint32_t x[kBatch], gm[kBatch];
+#pragma unroll
+    for (int q = 0; q < kBatch; q++) {
+      const uint32_t k = r0 + q * 32u + lane;
+      int o = 0;
+#pragma unroll
+      for (int step = 16; step > 0; step >>= 1) {
+        const uint32_t e = __shfl_sync(0xffffffffu, excl, o + step);
+        if (e <= k) o += step;
+      }
+      const uint64_t ob = __shfl_sync(0xffffffffu, beg, o);
+      const uint32_t oe = __shfl_sync(0xffffffffu, excl, o);
+      const uint32_t ov = __shfl_sync(0xffffffffu, nv, o);
+      const uint32_t ou = __shfl_sync(0xffffffffu, u, o);
+      act[q] = k < total;
+      const uint64_t e = ob + (k - oe);
+      x[q] = act[q] ? ldg_nc(P.out_dst + e) : 0u;
+      const uint32_t w = (act[q] && Prog::kUsesWeights) ? (uint32_t)ldg_nc_u8(P.out_w + e) : 0u;
+      gm[q] = act[q] ? Prog::gatherMap(0u, ov, w, ou, cx) : Prog::identity();
+    }
+    nact += push_batch<Prog>(P, act, x, gm, accn, epoch, qA, slot);
+  }
+  return nact;  // warp-uniform
+}
+
+// Block-wide push of one hub chunk (contiguous out-edges of vertex u, new value nv).
+template <class Prog, class OffT>
+__device__ uint32_t expand_block_push(const Part<OffT> &P, uint64_t beg, uint32_t deg, uint32_t u, uint32_t nv,
+                                      const Ctx &cx, uint32_t *accn, uint32_t epoch, WarpQueue &qA, uint32_t slot) {
+  uint32_t nact = 0;
+  for (uint32_t r0 = 0; r0 < deg; r0 += kBlock * kBatch) {
+    bool act[kBatch];
+    uint32_t x[kBatch], gm[kBatch];
+#pragma unroll
+    for (int q = 0; q < kBatch; q++) {
+      const uint32_t k = r0 + q * kBlock + threadIdx.x;
+      act[q] = k < deg;
+      x[q] = act[q] ? ldg_nc(P.out_dst + beg + k) : 0u;
+      const uint32_t w = (act[q] && Prog::kUsesWeights) ? (uint32_t)ldg_nc_u8(P.out_w + beg + k) : 0u;
+      gm[q] = act[q] ? Prog::gatherMap(0u, nv, w, u, cx) : Prog::identity();
+    }
+    nact += push_batch<Prog>(P, act, x, gm, accn, epoch, qA, slot);
+  }
+  return nact;  // per-warp count
+}
+
+template <class Prog, class OffT>
+__device__ __forceinline__ void push_phase(const Part<OffT> &P, const View &V) {
+  Ctl *ctl = P.ctl;
+  const uint32_t t = V.t;
+  const uint32_t slot = t & 1u, ns = slot ^ 1u;
+  const uint32_t epoch = V.epoch_base + t + 1;
+  const uint32_t nA = V.cntA[slot];
+  const uint32_t nK = V.cntK[slot];
+  const uint32_t *LA = P.listA[slot];
+  const uint32_t *LH = P.listH[slot];
+  uint32_t *acc = P.nxt[slot], *accn = P.nxt[ns];
+  const Ctx cx = make_ctx(P, V);
+  prof_begin(ctl, V, 1);
+
+  __shared__ uint32_t sq[kWarpsPerBlock][kQueueCap];
+  __shared__ uint32_t s_h, s_nv;
+  __shared__ bool s_changed;
+  __shared__ uint32_t s_off[kWarpsPerBlock + 1];
+  __shared__ unsigned long long s8[kWarpsPerBlock];
+  const uint32_t warp = threadIdx.x / 32, lane = lane_id();
+  WarpQueue qA{sq[warp], nullptr, 0};
+  unsigned long long my_g = 0, my_s = 0, my_c = 0, my_act = 0;
+
+  const uint32_t gw = blockIdx.x * kWarpsPerBlock + warp, nw = gridDim.x * kWarpsPerBlock;
+  for (uint32_t base = gw * 32u; base < nA; base += nw * 32u) {
+    const uint32_t idx = base + lane;
+    bool changed = false;
+    uint64_t beg = 0;
+    uint32_t deg = 0, v = 0, nv = 0;
+    if (idx < nA) {
+      v = LA[idx];
+      const uint32_t r = acc[v];
+      uint32_t cur = P.val[v];
+      const uint64_t i0 = (uint64_t)P.in_off[v - P.own_lo], i1 = (uint64_t)P.in_off[v - P.own_lo + 1];  // trace
+      acc[v] = Prog::identity();
+      my_g += i1 - i0;
+      if (Prog::apply(&cur, r, cx)) {
+        P.val[v] = cur;
+        nv = cur;
+        changed = true;
+        beg = (uint64_t)P.out_off[v];
+        deg = (uint32_t)((uint64_t)P.out_off[v + 1] - beg);
+        my_s += deg;
+        my_c += 1;
+      }
+    }
+    my_act += expand_warp_push<Prog>(P, changed, beg, deg, v, nv, cx, accn, epoch, qA, ns);
+  }
+  // A_t hubs (out-degree > kHubDegree), one CTA per out-edge chunk: every chunk
+  // applies on a private copy of acc[v] / val[v] (neither changes until all
+  // chunks have read them), pushes its chunk if v changes, and the last chunk
+  // to read commits (value, accumulator reset, trace counts).
+  for (; nK;) {
+    __syncthreads();
+    if (threadIdx.x == 0) s_h = atomicAdd(&ctl->ctr_hub, 1u);
+    __syncthreads();
+    const uint32_t i = s_h;
+    if (i >= nK) break;
+    const uint32_t hp = P.chkA_h[slot][i], ci = P.chkA_c[slot][i];
+    const uint32_t v = LH[hp];
+    const uint64_t beg = (uint64_t)P.out_off[v];
+    const uint64_t deg = (uint64_t)P.out_off[v + 1] - beg;
+    if (threadIdx.x == 0) {
+      const uint32_t r = *(volatile uint32_t *)(acc + v);
+      uint32_t cur = *(volatile uint32_t *)(P.val + v);
+      const bool ch = Prog::apply(&cur, r, cx);
+      s_changed = ch;
+      s_nv = cur;
+      __threadfence();
+      const uint32_t nch = (uint32_t)((deg + kChunk - 1) / kChunk);
+      if (atomicAdd(P.hub_done + hp, 1u) == nch - 1) {
+        P.hub_done[hp] = 0;
+        acc[v] = Prog::identity();
+        if (ch) {
+          P.val[v] = cur;
+          my_c += 1;
+          my_s += deg;
+        }
+        my_g += (uint64_t)P.in_off[v - P.own_lo + 1] - (uint64_t)P.in_off[v - P.own_lo];
+      }
+    }
+    __syncthreads();
+    if (!s_changed) continue;
+    const uint32_t a = expand_block_push<Prog>(P, beg + (uint64_t)ci * kChunk, chunk_len(deg, ci), v, s_nv, cx,
+                                               accn, epoch, qA, ns);
+    if (lane == 0) my_act += a;
+  }
+  qA.block_flush(P.listA[ns], nullptr, &ctl->cnt_A[ns], s_off);
+  my_g = block_sum_u64(my_g, s8);
+  if (threadIdx.x == 0 && my_g) atomicAdd(&ctl->part_g[blockIdx.x % kSlots], my_g);
+  my_s = block_sum_u64(my_s, s8);
+  if (threadIdx.x == 0 && my_s) atomicAdd(&ctl->part_s[blockIdx.x % kSlots], my_s);
+  my_c = block_sum_u64(my_c, s8);
+  if (threadIdx.x == 0 && my_c) atomicAdd(&ctl->part_c[blockIdx.x % kSlots], my_c);
+  my_act = block_sum_u64(lane == 0 ? my_act : 0ull, s8);
+  if (threadIdx.x == 0 && my_act) atomicAdd(&ctl->part_a[blockIdx.x % kSlots], my_act);
+  prof_end(ctl, V, 1);
+}
+
+template <class Prog, class OffT>
+__global__ void __launch_bounds__(kBlock) k_push_expand(const __grid_constant__ Part<OffT> P, unsigned long long cond,
+                                                        int use_graph) {
+  __shared__ View V;
+  load_view(P.ctl, V);
+  if (V.stop) {
+    if (use_graph && blockIdx.x == 0 && threadIdx.x == 0)
+      cudaGraphSetConditional((cudaGraphConditionalHandle)cond, 0u);
+    return;
+  }
+  if constexpr (PushFused<Prog>::value) push_phase<Prog>(P, V);
+  finish_superstep(P, cond, use_graph, kPush);
+}
+
 // Software grid barrier for the persistent loop (cooperative launch guarantees
 // that every CTA is resident). Sense by generation counter.
 __device__ __forceinline__ void grid_sync(Ctl *c) {
@@ -986,6 +1180,14 @@ __global__ void __launch_bounds__(kBlock) k_persistent(const __grid_constant__ P
     load_view(ctl, V);
     if (V.stop) break;
     int pull;
+    if constexpr (PushFused<Prog>::value) {
+      if (V.push) {  // one phase; the last CTA to finish closes the superstep
+        push_phase<Prog>(P, V);
+        finish_superstep(P, 0ull, 0, kPush);
+        grid_sync(ctl);
+        continue;
+      }
+    }
     if (Prog::kHasGather) {
       if (V.dense) gather_phase<Prog, true>(P, V);
       else gather_phase<Prog, false>(P, V);
@@ -1094,7 +1296,20 @@ __global__ void __launch_bounds__(kBlock) k_init_frontier(const __grid_constant_
   WarpQueue qA{sq[warp], nullptr, 0};
   const uint64_t beg = (uint64_t)P.out_off[source];
   const uint32_t deg = (uint32_t)((uint64_t)P.out_off[source + 1] - beg);
-  const uint32_t a = expand_block<false>(P, beg, deg, epoch0, P.hub_in, qA, 0);
+  uint32_t a;
+  if constexpr (PushFused<Prog>::value) {
+    if (ctl->push) {  // fused push supersteps: the source's value is pushed into acc_0
+      Ctx cx{};
+      cx.n = P.n;
+      cx.source = source;
+      cx.outdeg = P.outdeg;
+      a = expand_block_push<Prog>(P, beg, deg, source, P.val[source], cx, P.nxt[0], epoch0, qA, 0);
+    } else {
+      a = expand_block<false>(P, beg, deg, epoch0, P.hub_in, qA, 0);
+    }
+  } else {
+    a = expand_block<false>(P, beg, deg, epoch0, P.hub_in, qA, 0);
+  }
   qA.flush(P.listA[0], nullptr, &ctl->cnt_A[0]);
   if (lane_id() == 0 && a) atomicAdd(&ctl->cnt_act[0], a);
   __syncthreads();

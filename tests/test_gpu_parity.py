@@ -28,7 +28,7 @@ def check_pr(got, ref, n):
     assert abs(got.sum() - ref.sum()) <= 1e-5
 
 
-DIRS = ("auto", "push", "pull")
+DIRS = ("auto", "push", "pull", "fused")
 
 
 def compare(n, src, dst, w, algo, source=0, max_iters=0, loops=("auto", "device", "host"), directions=DIRS,
