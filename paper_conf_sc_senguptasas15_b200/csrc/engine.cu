@@ -296,6 +296,14 @@ gr_status load_device(gr_graph *g) {
 }
 
 // -------------------------------------------------------------- frontier run
+// Tolerance PageRank divisor table: (ceil(2^64 / n_u), n_u); n_u <= 1 keeps m = 0.
+static __global__ void k_prd_div(uint64_t n, const uint32_t *outdeg, ulonglong2 *tab) {
+  for (uint64_t v = blockIdx.x * (uint64_t)blockDim.x + threadIdx.x; v < n; v += (uint64_t)gridDim.x * blockDim.x) {
+    const uint64_t d = outdeg[v];
+    tab[v] = make_ulonglong2(d >= 2 ? (~0ull) / d + 1ull : 0ull, d);
+  }
+}
+
 // Fused push state (once per graph): the two accumulator arrays and, for
 // weighted programs, the activation CSR's weights. The CSR is the CSC
 // transposed by a stable sort of the CSC sources (device build, or the host
@@ -1173,6 +1181,14 @@ gr_status run(gr_graph *g, const gr_run_opts *oin, gr_run_stats *st) {
     if (!known) return fail(GR_EUNSUPPORTED, "no custom program with id %d is registered", o.custom_id);
     if (uses_w && !g->H.has_w) return fail(GR_EINVAL, "custom program %d needs edge weights", o.custom_id);
     if (o.source >= g->H.n) return fail(GR_EINVAL, "source %u >= num_vertices", o.source);
+  }
+  if (o.algo == GR_PAGERANK_DELTA && !g->prd_div) {
+    // exact divisor table (gr/program.cuh ProgPRDelta::gatherMap), once per graph
+    gr_status ds = dev_alloc(g, (void **)&g->prd_div, 16 * std::max<uint64_t>(g->H.n, 1));
+    if (ds != GR_OK) return ds;
+    k_prd_div<<<g->num_sms * 4, 256, 0, g->stream>>>(g->H.n, g->d_outdeg, g->prd_div);
+    CK(cudaGetLastError());
+    CK(cudaStreamSynchronize(g->stream));
   }
   if (g->mode == GR_MODE_STREAMED) return run_streamed(g, &o, st);
   cudaStream_t s = o.stream ? (cudaStream_t)o.stream : g->stream;

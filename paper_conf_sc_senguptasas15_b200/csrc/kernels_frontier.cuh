@@ -43,6 +43,7 @@ template <class OffT> __device__ __forceinline__ Ctx make_ctx(const Part<OffT> &
   cx.prd_dq = V.prd_dq;
   cx.prd_thr = V.prd_thr;
   cx.prd_r0 = 0;
+  cx.prd_div = P.prd_div;
   return cx;
 }
 
