@@ -10,7 +10,7 @@
 extern "C" {
 #endif
 
-enum { OR_BFS = 0, OR_SSSP = 1, OR_PAGERANK = 2, OR_CC = 3, OR_WIDEST = 4, OR_PRDELTA = 5 };
+enum { OR_BFS = 0, OR_SSSP = 1, OR_PAGERANK = 2, OR_CC = 3, OR_WIDEST = 4, OR_PRDELTA = 5, OR_SSSPMSG = 6 };
 #define OR_INF 0xFFFFFFFFu
 
 typedef struct or_graph or_graph;
@@ -33,6 +33,12 @@ void or_graph_free(or_graph *g);
  * q = round(d * 2^20) of the fp32 damping d.
  * OR_WIDEST: single-source widest path (max over paths of the min edge weight),
  * a user GAS program (§4.1) used to check GR_CUSTOM programs.
+ * OR_SSSPMSG: SSSP with mutable edge state (the Scatter phase, §2.1
+ * L66, §4.4): every edge holds a message, initially INF; after the apply
+ * of superstep t and the commit of the new values, every edge (u -> x) with u
+ * changed at t gets S = new[u] + w if that is < val[x] (the committed value),
+ * else INF; the gather takes the min of the messages on the in-edges. The
+ * source is set to 0 and scatters at initialisation.
  * trace_out (nullable): rows of 4 uint64 per superstep t:
  *   |A_t|, |C_t|, sum_{v in A_t} indeg(v) (0 when gather is eliminated),
  *   sum_{u in C_t} outdeg(u) (0 when FrontierActivate is eliminated).

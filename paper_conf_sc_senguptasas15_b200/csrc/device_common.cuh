@@ -153,6 +153,8 @@ template <class OffT> struct Part {
   uint32_t *hub_act;      // per static hub: some chunk saw a marked source (dense gathers)
   const uint32_t *s_hubs, *s_chk_h, *s_chk_c;  // static in-hub list and its chunks (dense gathers)
   const ulonglong2 *prd_div;  // ProgPRDelta divisor table (Ctx::prd_div), or nullptr
+  uint32_t *estate;       // [m_in] edge states in CSC order (programs with kHasScatter)
+  const uint32_t *out_eid;// [m_in] CSC position of every activation-CSR edge (kHasScatter)
   uint32_t *nxt[2];       // fused push supersteps: per-vertex gather accumulators by parity (GatherT = u32)
   const uint8_t *out_w;   // activation CSR weights (fused push supersteps of weighted programs)
   uint32_t n_s_hubs, n_s_chunks;

@@ -309,14 +309,59 @@ static __global__ void k_prd_div(uint64_t n, const uint32_t *outdeg, ulonglong2 
 // transposed by a stable sort of the CSC sources (device build, or the host
 // layout sorted the same way), so the same stable sort carrying the CSC
 // weights yields them in CSR order.
+static gr_status out_w_setup(gr_graph *g);
 static gr_status push_setup(gr_graph *g, bool weights) {
-  const uint64_t n = g->H.n, m = g->H.m_in;
-  cudaStream_t s = g->stream;
+  const uint64_t n = g->H.n;
   gr_status st;
   for (int i = 0; i < 2; i++)
     if (!g->nxt[i] && (st = dev_alloc(g, (void **)&g->nxt[i], 4 * std::max<uint64_t>(n, 1))) != GR_OK) return st;
-  if (!weights || g->out_w) return GR_OK;
-  if (!g->in_w) return fail(GR_EINVAL, "fused push: the program reads weights but the graph has none");
+  return weights ? out_w_setup(g) : GR_OK;
+}
+
+static __global__ void k_iota_u32(uint32_t *p, uint64_t m) {
+  for (uint64_t i = blockIdx.x * (uint64_t)blockDim.x + threadIdx.x; i < m; i += (uint64_t)gridDim.x * blockDim.x)
+    p[i] = (uint32_t)i;
+}
+
+// Mutable edge state (kHasScatter programs, once per graph): the CSC position of
+// every activation-CSR edge — the same stable sort by source carrying the CSC
+// positions — the state array, and the CSR weights when scatter reads them.
+static gr_status scatter_setup(gr_graph *g, bool weights) {
+  const uint64_t n = g->H.n, m = g->H.m_in;
+  cudaStream_t s = g->stream;
+  gr_status st;
+  if (m >= 0xFFFFFFFFull) return fail(GR_EUNSUPPORTED, "edge state: more than 2^32-1 edges");
+  if (!g->estate && (st = dev_alloc(g, (void **)&g->estate, 4 * (m + 4))) != GR_OK) return st;
+  if (!g->out_eid) {
+    if ((st = dev_alloc(g, (void **)&g->out_eid, 4 * (m + 4))) != GR_OK) return st;
+    CK(cudaMemsetAsync(g->out_eid + m, 0, 16, s));
+    uint32_t bits = 1;
+    while ((1ull << bits) < n) bits++;
+    uint32_t *kscratch = nullptr, *iota = nullptr;
+    void *tmp = nullptr;
+    size_t need = 0;
+    CK(pmalloc(&kscratch, 4 * std::max<uint64_t>(m, 1), s));
+    CK(pmalloc(&iota, 4 * std::max<uint64_t>(m, 1), s));
+    k_iota_u32<<<g->num_sms * 8, 256, 0, s>>>(iota, m);
+    CK(cub::DeviceRadixSort::SortPairs(nullptr, need, g->in_src, kscratch, iota, g->out_eid, (int64_t)m, 0,
+                                       (int)bits, s));
+    CK(pmalloc(&tmp, std::max<size_t>(need, 16), s));
+    CK(cub::DeviceRadixSort::SortPairs(tmp, need, g->in_src, kscratch, iota, g->out_eid, (int64_t)m, 0, (int)bits,
+                                       s));
+    pfree(tmp, s);
+    pfree(iota, s);
+    pfree(kscratch, s);
+    CK(cudaStreamSynchronize(s));
+  }
+  return weights ? out_w_setup(g) : GR_OK;
+}
+
+static gr_status out_w_setup(gr_graph *g) {
+  const uint64_t n = g->H.n, m = g->H.m_in;
+  cudaStream_t s = g->stream;
+  gr_status st;
+  if (g->out_w) return GR_OK;
+  if (!g->in_w) return fail(GR_EINVAL, "the program reads edge weights but the graph has none");
   if ((st = dev_alloc(g, (void **)&g->out_w, m + 16)) != GR_OK) return st;
   CK(cudaMemsetAsync(g->out_w + m, 0, 16, s));
   uint32_t bits = 1;
@@ -343,6 +388,13 @@ static void launch_body(gr_graph *g, cudaStream_t s, unsigned long long cond, in
   if (push) {  // fused push superstep: one kernel
     k_push_expand<Prog, OffT><<<g->grid_frontier, kBlock, 0, s>>>(P, cond, use_graph);
     *launches += 1;
+    return;
+  }
+  if constexpr (HasScatter<Prog>::value) {  // gather | commit | scatter + activate
+    k_gather_apply<Prog, OffT><<<g->grid_frontier, kBlock, 0, s>>>(P);
+    k_commit_only<OffT><<<g->grid_frontier, kBlock, 0, s>>>(P);
+    k_scatter_activate<Prog, OffT><<<g->grid_frontier, kBlock, 0, s>>>(P, cond, use_graph);
+    *launches += 3;
     return;
   }
   if (Prog::kHasGather) {
@@ -435,8 +487,17 @@ static gr_status run_frontier(gr_graph *g, const gr_run_opts *o, cudaStream_t s,
     }
   }
   h.push = push ? 1u : 0u;
-  // activation direction (gr_direction); pull needs the bitmaps (resident, one rank)
-  if (g->cbits[0] && !push && o->direction != GR_DIR_PUSH) {
+  constexpr bool kScatter = HasScatter<Prog>::value;
+  if constexpr (kScatter) {  // mutable edge state: layout once per graph, states reset per run
+    gr_status ss = scatter_setup(g, Prog::kUsesWeights);
+    if (ss != GR_OK) return ss;
+    P = make_part<OffT>(g);
+    k_init_edges<Prog, OffT><<<g->num_sms * 8, 256, 0, s>>>(P, g->H.m_in);
+    launches++;
+  }
+  // activation direction (gr_direction); pull needs the bitmaps (resident, one rank);
+  // scatter programs always push (the scatter walks the out-edges of C_t)
+  if (g->cbits[0] && !push && !kScatter && o->direction != GR_DIR_PUSH) {
     uint32_t div = o->pull_div ? o->pull_div : kPullDivDefault;
     if (const char *e = getenv("GR_PULL_DIV")) div = (uint32_t)strtoul(e, nullptr, 10);
     h.pull_div = o->direction == GR_DIR_PULL ? 0xFFFFFFFFu : div;

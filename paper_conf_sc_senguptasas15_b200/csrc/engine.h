@@ -30,7 +30,8 @@ struct gr_graph {
   uint8_t *in_w = nullptr;
   uint8_t *out_w = nullptr;                       // CSR weights (built on first fused push run)
   uint32_t *nxt[2] = {nullptr, nullptr};          // fused push accumulators (allocated on first use)
-  ulonglong2 *prd_div = nullptr;                  // tolerance PageRank divisor table (first GR_PAGERANK_DELTA run)
+  ulonglong2 *prd_div = nullptr;
+  uint32_t *estate = nullptr, *out_eid = nullptr; // mutable edge state (kHasScatter programs; first use)                  // tolerance PageRank divisor table (first GR_PAGERANK_DELTA run)
   uint32_t *hub_in = nullptr, *hub_out = nullptr, *static_hubs = nullptr;
   uint32_t n_static_hubs = 0;
   // hub chunk lists (kChunk edges per CTA work item)
@@ -134,6 +135,8 @@ template <class OffT> inline Part<OffT> make_part(gr_graph *g) {
   P.in_src = g->in_src;
   P.in_w = g->in_w;
   P.prd_div = g->prd_div;
+  P.estate = g->estate;
+  P.out_eid = g->out_eid;
   P.nxt[0] = g->nxt[0];
   P.nxt[1] = g->nxt[1];
   P.out_w = g->out_w;

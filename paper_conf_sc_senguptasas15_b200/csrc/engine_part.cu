@@ -92,6 +92,8 @@ static gr_status global_sum(Comm *c, uint64_t mine, uint64_t *out, cudaStream_t 
 
 template <class Prog, class OffT>
 gr_status run_frontier_part(gr_graph *g, const gr_run_opts *o, cudaStream_t s, gr_run_stats *st) {
+  if constexpr (HasScatter<Prog>::value)
+    return fail(GR_EUNSUPPORTED, "programs with mutable edge state (scatter) run resident on one GPU");
   Comm *C = g->comm;
   Part<OffT> P = make_part<OffT>(g);
   uint64_t launches = 0;

@@ -47,6 +47,15 @@ template <class OffT> __device__ __forceinline__ Ctx make_ctx(const Part<OffT> &
   return cx;
 }
 
+// gatherMap's edge argument: the mutable edge state (kHasScatter programs; an
+// L2-coherent read, the state is rewritten by the previous superstep's
+// scatter), else the weight (or 0)
+template <class Prog, class OffT>
+__device__ __forceinline__ uint32_t edge_w(const Part<OffT> &P, uint64_t e) {
+  if constexpr (HasScatter<Prog>::value) return ld_cg(P.estate + e);
+  else return Prog::kUsesWeights ? (uint32_t)ldg_nc_u8(P.in_w + e) : 0u;
+}
+
 template <class Prog>
 __device__ __forceinline__ typename Prog::GatherT warp_reduce_prog(typename Prog::GatherT x) {
 #pragma unroll
@@ -83,7 +92,7 @@ __device__ typename Prog::GatherT gather_warp(const Part<OffT> &P, bool valid, u
 #pragma unroll
       for (int q = 0; q < 4; q++) {
         u[q] = ldg_nc(P.in_src + b + k + 32 * q);
-        w[q] = Prog::kUsesWeights ? (uint32_t)ldg_nc_u8(P.in_w + b + k + 32 * q) : 0u;
+        w[q] = edge_w<Prog>(P, b + k + 32 * q);
       }
       uint32_t v[4], bw[4];
 #pragma unroll
@@ -99,7 +108,7 @@ __device__ typename Prog::GatherT gather_warp(const Part<OffT> &P, bool valid, u
     }
     for (; k < d; k += 32) {
       const uint32_t u = ldg_nc(P.in_src + b + k);
-      const uint32_t w = Prog::kUsesWeights ? (uint32_t)ldg_nc_u8(P.in_w + b + k) : 0u;
+      const uint32_t w = edge_w<Prog>(P, b + k);
       r = Prog::gatherReduce(r, Prog::gatherMap(dv, P.val[u], w, u, cx));
       if (kDense) hit |= test_bit_cg(bits, u);
     }
@@ -141,7 +150,7 @@ __device__ typename Prog::GatherT gather_warp(const Part<OffT> &P, bool valid, u
       act_q[q] = k < total;
       const uint64_t e = ob + (k - oe);
       su[q] = act_q[q] ? ldg_nc(P.in_src + e) : 0u;
-      sw[q] = (act_q[q] && Prog::kUsesWeights) ? (uint32_t)ldg_nc_u8(P.in_w + e) : 0u;
+      sw[q] = act_q[q] ? edge_w<Prog>(P, e) : 0u;
     }
     uint32_t sv[kBatch], sb[kBatch];
 #pragma unroll
@@ -202,7 +211,7 @@ __device__ typename Prog::GatherT gather_block(const Part<OffT> &P, uint64_t beg
 #pragma unroll
     for (int q = 0; q < 4; q++) {
       u[q] = ldg_nc(P.in_src + beg + k + q * kBlock);
-      w[q] = Prog::kUsesWeights ? (uint32_t)ldg_nc_u8(P.in_w + beg + k + q * kBlock) : 0u;
+      w[q] = edge_w<Prog>(P, beg + k + q * kBlock);
     }
     uint32_t v[4], bw[4];
 #pragma unroll
@@ -218,7 +227,7 @@ __device__ typename Prog::GatherT gather_block(const Part<OffT> &P, uint64_t beg
   }
   for (; k < deg; k += kBlock) {
     const uint32_t u = ldg_nc(P.in_src + beg + k);
-    const uint32_t w = Prog::kUsesWeights ? (uint32_t)ldg_nc_u8(P.in_w + beg + k) : 0u;
+    const uint32_t w = edge_w<Prog>(P, beg + k);
     r = Prog::gatherReduce(r, Prog::gatherMap(dval, P.val[u], w, u, cx));
     if (kDense) hit |= test_bit_cg(bits, u);
   }
@@ -1149,6 +1158,184 @@ __global__ void __launch_bounds__(kBlock) k_push_expand(const __grid_constant__ 
   finish_superstep(P, cond, use_graph, kPush);
 }
 
+// ------------------------------------------------------ scatter (edge state)
+// Programs with kHasScatter (gr/program.cuh): superstep t commits the new
+// values of C_t in its own phase (commit_only_phase), then, after a grid
+// barrier, every out-edge (u -> x) of every u in C_t runs
+// scatter(new[u], val_t[x], w, &state[csc position]) before FrontierActivate
+// (§2.1, §4.4). Each edge has one source, which appears once
+// in C_t, so each state is written by exactly one thread per superstep.
+template <class OffT>
+__device__ __forceinline__ void commit_only_phase(const Part<OffT> &P, const View &V) {
+  const uint32_t nC = V.cntC, nCH = V.cntCH;
+  for (uint32_t i = blockIdx.x * blockDim.x + threadIdx.x; i < nC + nCH; i += gridDim.x * blockDim.x) {
+    const bool h = i >= nC;
+    const uint32_t u = h ? P.CH_v[i - nC] : P.C_v[i];
+    P.val[u] = h ? P.CH_val[i - nC] : P.C_val[i];  // BSP commit of superstep t
+  }
+}
+
+template <class Prog, class OffT>
+__device__ __forceinline__ void scatter_batch(const Part<OffT> &P, const bool (&act)[kBatch],
+                                              const uint32_t (&x)[kBatch], const uint32_t (&w)[kBatch],
+                                              const uint32_t (&eid)[kBatch], const uint32_t (&sv)[kBatch],
+                                              const Ctx &cx) {
+  uint32_t dv[kBatch];
+#pragma unroll
+  for (int q = 0; q < kBatch; q++) dv[q] = act[q] ? ld_cg(P.val + x[q]) : 0u;  // committed values of t
+#pragma unroll
+  for (int q = 0; q < kBatch; q++)
+    if (act[q]) Prog::scatter(sv[q], dv[q], w[q], P.estate + eid[q], cx);
+}
+
+template <class Prog, class OffT>
+__device__ uint32_t expand_warp_scatter(const Part<OffT> &P, bool valid, uint64_t beg, uint32_t deg, uint32_t nv,
+                                        const Ctx &cx, uint32_t epoch, WarpQueue &qA, uint32_t slot) {
+  const uint32_t lane = lane_id();
+  const uint32_t d = valid ? deg : 0u;
+  const uint32_t incl = warp_incl_scan(d);
+  const uint32_t excl = incl - d;
+  const uint32_t total = __shfl_sync(0xffffffffu, incl, 31);
+  uint32_t nact = 0;
+  for (uint32_t r0 = 0; r0 < total; r0 += 32u * kBatch) {
+    bool act[kBatch];
+    uint32_t x[kBatch], w[kBatch], eid[kBatch], sv[kBatch];
+#pragma unroll
+    for (int q = 0; q < kBatch; q++) {
+      const uint32_t k = r0 + q * 32u + lane;
+      int o = 0;
+#pragma unroll
+      for (int step = 16; step > 0; step >>= 1) {
+        const uint32_t e = __shfl_sync(0xffffffffu, excl, o + step);
+        if (e <= k) o += step;
+      }
+      const uint64_t ob = __shfl_sync(0xffffffffu, beg, o);
+      const uint32_t oe = __shfl_sync(0xffffffffu, excl, o);
+      sv[q] = __shfl_sync(0xffffffffu, nv, o);
+      act[q] = k < total;
+      const uint64_t e = ob + (k - oe);
+      x[q] = act[q] ? ldg_nc(P.out_dst + e) : 0u;
+      w[q] = (act[q] && Prog::kUsesWeights) ? (uint32_t)ldg_nc_u8(P.out_w + e) : 0u;
+      eid[q] = act[q] ? ldg_nc(P.out_eid + e) : 0u;
+    }
+    scatter_batch<Prog>(P, act, x, w, eid, sv, cx);
+    nact += activate_batch<false>(P, act, x, epoch, P.hub_in, qA, slot);
+  }
+  return nact;  // warp-uniform
+}
+
+template <class Prog, class OffT>
+__device__ uint32_t expand_block_scatter(const Part<OffT> &P, uint64_t beg, uint32_t deg, uint32_t nv,
+                                         const Ctx &cx, uint32_t epoch, WarpQueue &qA, uint32_t slot) {
+  uint32_t nact = 0;
+  for (uint32_t r0 = 0; r0 < deg; r0 += kBlock * kBatch) {
+    bool act[kBatch];
+    uint32_t x[kBatch], w[kBatch], eid[kBatch], sv[kBatch];
+#pragma unroll
+    for (int q = 0; q < kBatch; q++) {
+      const uint32_t k = r0 + q * kBlock + threadIdx.x;
+      act[q] = k < deg;
+      x[q] = act[q] ? ldg_nc(P.out_dst + beg + k) : 0u;
+      w[q] = (act[q] && Prog::kUsesWeights) ? (uint32_t)ldg_nc_u8(P.out_w + beg + k) : 0u;
+      eid[q] = act[q] ? ldg_nc(P.out_eid + beg + k) : 0u;
+      sv[q] = nv;
+    }
+    scatter_batch<Prog>(P, act, x, w, eid, sv, cx);
+    nact += activate_batch<false>(P, act, x, epoch, P.hub_in, qA, slot);
+  }
+  return nact;  // per-warp count
+}
+
+// scatter + FrontierActivate over C_t (values already committed)
+template <class Prog, class OffT>
+__device__ __forceinline__ void scatter_activate_phase(const Part<OffT> &P, const View &V) {
+  Ctl *ctl = P.ctl;
+  const uint32_t t = V.t;
+  const uint32_t ns = (t + 1) & 1u;
+  const uint32_t epoch = V.epoch_base + t + 1;
+  const uint32_t nC = V.cntC;
+  const uint32_t nKC = V.cntKC;
+  const Ctx cx = make_ctx(P, V);
+  prof_begin(ctl, V, 1);
+
+  __shared__ uint32_t sq[kWarpsPerBlock][kQueueCap];
+  __shared__ uint32_t s_h;
+  __shared__ uint32_t s_off[kWarpsPerBlock + 1];
+  __shared__ unsigned long long s8[kWarpsPerBlock];
+  const uint32_t warp = threadIdx.x / 32, lane = lane_id();
+  WarpQueue qA{sq[warp], nullptr, 0};
+  unsigned long long my_s = 0, my_act = 0;
+
+  const uint32_t gw = blockIdx.x * kWarpsPerBlock + warp, nw = gridDim.x * kWarpsPerBlock;
+  for (uint32_t base = gw * 32u; base < nC; base += nw * 32u) {
+    const uint32_t idx = base + lane;
+    const bool valid = idx < nC;
+    uint64_t beg = 0;
+    uint32_t deg = 0, nv = 0;
+    if (valid) {
+      const uint32_t u = P.C_v[idx];
+      nv = P.C_val[idx];
+      beg = (uint64_t)P.out_off[u];
+      deg = (uint32_t)((uint64_t)P.out_off[u + 1] - beg);
+      my_s += deg;
+    }
+    my_act += expand_warp_scatter<Prog>(P, valid, beg, deg, nv, cx, epoch, qA, ns);
+  }
+  for (; nKC;) {
+    __syncthreads();
+    if (threadIdx.x == 0) s_h = atomicAdd(&ctl->ctr_hub2, 1u);
+    __syncthreads();
+    const uint32_t i = s_h;
+    if (i >= nKC) break;
+    const uint32_t hp = P.chkC_h[i], ci = P.chkC_c[i];
+    const uint32_t u = P.CH_v[hp];
+    const uint64_t beg = (uint64_t)P.out_off[u];
+    const uint64_t deg = (uint64_t)P.out_off[u + 1] - beg;
+    if (threadIdx.x == 0 && ci == 0) my_s += deg;
+    const uint32_t a = expand_block_scatter<Prog>(P, beg + (uint64_t)ci * kChunk, chunk_len(deg, ci), P.CH_val[hp],
+                                                  cx, epoch, qA, ns);
+    if (lane == 0) my_act += a;
+  }
+  qA.block_flush(P.listA[ns], nullptr, &ctl->cnt_A[ns], s_off);
+  my_s = block_sum_u64(my_s, s8);
+  if (threadIdx.x == 0 && my_s) atomicAdd(&ctl->part_s[blockIdx.x % kSlots], my_s);
+  my_act = block_sum_u64(lane == 0 ? my_act : 0ull, s8);
+  if (threadIdx.x == 0 && my_act) atomicAdd(&ctl->part_a[blockIdx.x % kSlots], my_act);
+  prof_end(ctl, V, 1);
+}
+
+template <class OffT>
+__global__ void __launch_bounds__(kBlock) k_commit_only(const __grid_constant__ Part<OffT> P) {
+  __shared__ View V;
+  load_view(P.ctl, V);
+  if (V.stop) return;
+  commit_only_phase(P, V);
+}
+
+template <class Prog, class OffT>
+__global__ void __launch_bounds__(kBlock) k_scatter_activate(const __grid_constant__ Part<OffT> P,
+                                                             unsigned long long cond, int use_graph) {
+  __shared__ View V;
+  load_view(P.ctl, V);
+  if (V.stop) {
+    if (use_graph && blockIdx.x == 0 && threadIdx.x == 0)
+      cudaGraphSetConditional((cudaGraphConditionalHandle)cond, 0u);
+    return;
+  }
+  if constexpr (HasScatter<Prog>::value) scatter_activate_phase<Prog>(P, V);
+  finish_superstep(P, cond, use_graph, kPush);
+}
+
+template <class Prog, class OffT>
+__global__ void k_init_edges(const __grid_constant__ Part<OffT> P, uint64_t m) {
+  if constexpr (HasScatter<Prog>::value) {
+    Ctx cx{};
+    cx.n = P.n;
+    for (uint64_t e = blockIdx.x * (uint64_t)blockDim.x + threadIdx.x; e < m; e += (uint64_t)gridDim.x * blockDim.x)
+      P.estate[e] = Prog::initEdge(P.in_w ? (uint32_t)P.in_w[e] : 0u, cx);
+  }
+}
+
 // Software grid barrier for the persistent loop (cooperative launch guarantees
 // that every CTA is resident). Sense by generation counter.
 __device__ __forceinline__ void grid_sync(Ctl *c) {
@@ -1181,6 +1368,18 @@ __global__ void __launch_bounds__(kBlock) k_persistent(const __grid_constant__ P
     load_view(ctl, V);
     if (V.stop) break;
     int pull;
+    if constexpr (HasScatter<Prog>::value) {  // gather | commit | scatter + activate (push only)
+      gather_phase<Prog, false>(P, V);
+      grid_sync(ctl);
+      load_view(ctl, V);
+      commit_only_phase(P, V);
+      grid_sync(ctl);
+      scatter_activate_phase<Prog>(P, V);
+      grid_sync(ctl);
+      if (blockIdx.x == 0) close_superstep(P, 0ull, 0, kPush);
+      grid_sync(ctl);
+      continue;
+    }
     if constexpr (PushFused<Prog>::value) {
       if (V.push) {  // one phase; the last CTA to finish closes the superstep
         push_phase<Prog>(P, V);
@@ -1298,7 +1497,13 @@ __global__ void __launch_bounds__(kBlock) k_init_frontier(const __grid_constant_
   const uint64_t beg = (uint64_t)P.out_off[source];
   const uint32_t deg = (uint32_t)((uint64_t)P.out_off[source + 1] - beg);
   uint32_t a;
-  if constexpr (PushFused<Prog>::value) {
+  if constexpr (HasScatter<Prog>::value) {  // the source changed at init: it scatters
+    Ctx cx{};
+    cx.n = P.n;
+    cx.source = source;
+    cx.outdeg = P.outdeg;
+    a = expand_block_scatter<Prog>(P, beg, deg, P.val[source], cx, epoch0, qA, 0);
+  } else if constexpr (PushFused<Prog>::value) {
     if (ctl->push) {  // fused push supersteps: the source's value is pushed into acc_0
       Ctx cx{};
       cx.n = P.n;

@@ -275,6 +275,8 @@ static gr_status stream_pagerank(gr_graph *g, const gr_run_opts *o, cudaStream_t
 // ------------------------------------------------------- frontier programs
 template <class Prog, class OffT>
 static gr_status stream_frontier(gr_graph *g, const gr_run_opts *o, cudaStream_t cs, gr_run_stats *st) {
+  if constexpr (HasScatter<Prog>::value)
+    return fail(GR_EUNSUPPORTED, "programs with mutable edge state (scatter) run resident on one GPU");
   Streamer *S = S_(g);
   const HostGraph &H = g->H;
   const uint32_t P = S->P;

@@ -520,3 +520,37 @@ def test_pagerank_delta_rmat_tolerances(tol):
             assert st["iterations"] == rit
         if tol > 0:  # the frontier shrinks (Figs. 16-17): late supersteps gather a fraction of V
             assert rtr[-1, 0] < g.n // 4 and rtr[:, 0].min() < g.n
+
+
+def test_custom_program_edge_messages():
+    """Mutable edge state (the paper's Scatter phase, §2.1, §4.4
+    L253): ProgSSSPMsg (custom id 1) keeps a message on every edge, written by
+    scatter after the commit and read by the gather; bit-exact values and
+    traces against the oracle's OR_SSSPMSG in every loop."""
+    cases = []
+    for seed in (1, 2):
+        g = grgen.rmat(12, 16, seed=seed)
+        cases.append((g.n, g.src, g.dst, grgen.weights(g.m, 1, 64, seed=seed + 7), 0))
+    n, src, dst, w = hub_graph()
+    cases.append((n, src, dst, w, 5))
+    g = grgen.grid_road(80, 80, seed=3)
+    cases.append((g.n, g.src, g.dst, g.w, 0))
+    for (n, src, dst, w, s) in cases:
+        ref, rtr, rit = oracle.run(n, src, dst, "sssp_msg", w=w, source=s)
+        with gr.GraphReduce(n, src, dst, w) as G:
+            for loop in ("auto", "device", "host"):
+                for _ in range(2):  # edge states are reset per run
+                    st = G.run("custom", custom_id=1, source=s, loop=loop)
+                    assert st["iterations"] == rit
+                    np.testing.assert_array_equal(G.values(), ref)
+                    np.testing.assert_array_equal(G.trace(), rtr)
+                    assert st["pull_supersteps"] == 0
+
+
+def test_edge_messages_unsupported_outside_resident():
+    g = grgen.rmat(10, 8, seed=3)
+    w = grgen.weights(g.m, 1, 64, seed=4)
+    with gr.GraphReduce(g.n, g.src, g.dst, w, mode="streamed", shard_edges=2000) as G:
+        with pytest.raises(gr.GrError) as e:
+            G.run("custom", custom_id=1, source=0)
+        assert "scatter" in str(e.value)

@@ -535,3 +535,32 @@ def test_prdelta_rejects_bad_parameters():
     for kw in ({"damping": 0.0}, {"damping": 1.0}, {"tolerance": -1.0}):
         with pytest.raises(ValueError):
             oracle.run(2, src, dst, "pagerank_delta", **kw)
+
+
+# ------------------------------------------------- scatter: SSSP by edge messages
+# OR_SSSPMSG (oracle.h): mutable edge state (§2.1, §4.4).
+# Pinned to the textbook heap Dijkstra (values) and, by the invariance argument
+# of oracle.h (an unsent message could never lower its target), to the frontier
+# trace of the plain SSSP program.
+@pytest.mark.parametrize("seed", range(10))
+def test_sssp_messages_vs_dijkstra(seed):
+    rng = np.random.default_rng(700 + seed)
+    n = int(rng.integers(2, 70))
+    src, dst, w = rand_graph(rng, n, int(rng.integers(0, 4 * n)), wmax=64)
+    s = int(rng.integers(0, n))
+    vals, tr, it = oracle.run(n, src, dst, "sssp_msg", w=w, source=s)
+    np.testing.assert_array_equal(vals, heap_dijkstra(n, src, dst, w, s))
+    v2, tr2, it2 = oracle.run(n, src, dst, "sssp", w=w, source=s)
+    np.testing.assert_array_equal(tr, tr2)
+    assert it == it2
+
+
+def test_sssp_messages_path_and_lattice():
+    # a directed path 0 -> 1 -> ... -> k: prefix sums of the weights, one superstep per hop
+    k = 40
+    src = np.arange(k, dtype=np.uint32)
+    dst = src + 1
+    w = (np.arange(k, dtype=np.uint32) % 7) + 1
+    vals, tr, it = oracle.run(k + 1, src, dst, "sssp_msg", w=w, source=0)
+    np.testing.assert_array_equal(vals, np.concatenate([[0], np.cumsum(w)]).astype(np.uint32))
+    assert it == k and np.all(tr[:, 1] == 1) and tr[-1, 3] == 0  # A_0 = {1}, ..., A_{k-1} = {k}
