@@ -391,6 +391,23 @@ def main():
             "kernel_share_of_step": round(kms / ms, 4) if ms > 0 else None,
             "per": "superstep (30 per launch)" if kname.endswith("_loop") else "launch",
             "traffic": load_traffic(f"{kname}@cfg{args.config}" + (f"s{args.scale}" if args.config == 5 else ""))}
+    if algo == "pagerank" and kname in ("k_pr_seg_loop", "k_pr_seg") and mode == "resident" and world == 1:
+        # diagnostic second roofline (profiles/README.md): the random 4-byte gathers
+        # that leave the SM (sources outside the 32768-entry shared-memory hot table: the top
+        # out-degrees, ties by id — the library's selection rule) against the measured limit of one
+        # L1->L2 request per SM per cycle (tools/gather_paths_bench.cu) at the sampled SM clock
+        od = np.bincount(g.src, minlength=n).astype(np.int64)
+        hot = np.argsort(-od, kind="stable")[:32768]
+        cold = int(m - od[hot].sum())
+        sms = torch.cuda.get_device_properties(local_rank).multi_processor_count
+        mhz = ck.get("sm_mhz") or ck.get("sm_max_mhz") or 1965.0
+        rpeak = sms * mhz * 1e6
+        rate = cold / avg_launch_s
+        roof["gather_requests"] = {"cold_gathers_per_superstep": cold, "achieved_per_s": round(rate / 1e9, 1),
+                                   "peak_per_s": round(rpeak / 1e9, 1), "unit": "G requests/s",
+                                   "frac": round(rate / rpeak, 4),
+                                   "note": "cold gathers estimated from the hot-set rule; peak = 1 request per "
+                                           "SM per cycle (measured, tools/gather_paths_bench.cu) x SMs x clock"}
     if mode == "streamed":
         h2d_peak = measure_h2d()
         h2d_rate = stats["bytes_h2d"] / (ms_step * 1e-3) / 1e9

@@ -326,7 +326,7 @@ static __global__ void k_iota_u32(uint32_t *p, uint64_t m) {
 // Mutable edge state (kHasScatter programs, once per graph): the CSC position of
 // every activation-CSR edge — the same stable sort by source carrying the CSC
 // positions — the state array, and the CSR weights when scatter reads them.
-static gr_status scatter_setup(gr_graph *g, bool weights) {
+gr_status scatter_setup(gr_graph *g, bool weights) {
   const uint64_t n = g->H.n, m = g->H.m_in;
   cudaStream_t s = g->stream;
   gr_status st;

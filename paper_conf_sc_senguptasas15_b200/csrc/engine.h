@@ -192,6 +192,8 @@ gr_status device_build(gr_graph *g, const gr_edges *E, uint64_t shard_edges);
 gr_status select_hot(gr_graph *g, uint64_t K, uint32_t **hot_ids, uint32_t *hot_k, uint32_t **d_slot);
 // partitioned PageRank (engine.cu): kernel/layout selection once per graph, one superstep's launches
 gr_status pr_part_prepare(gr_graph *g);
+// mutable edge state (kHasScatter programs): CSR->CSC position map, state array, CSR weights
+gr_status scatter_setup(gr_graph *g, bool weights);
 uint32_t pr_part_iter(gr_graph *g, cudaStream_t s, uint32_t t, uint32_t iters, float d);
 gr_status run(gr_graph *g, const gr_run_opts *o, gr_run_stats *st);
 gr_status fetch_values(gr_graph *g, void *dst, uint64_t bytes);

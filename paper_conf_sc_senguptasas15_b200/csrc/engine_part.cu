@@ -92,9 +92,12 @@ static gr_status global_sum(Comm *c, uint64_t mine, uint64_t *out, cudaStream_t 
 
 template <class Prog, class OffT>
 gr_status run_frontier_part(gr_graph *g, const gr_run_opts *o, cudaStream_t s, gr_run_stats *st) {
-  if constexpr (HasScatter<Prog>::value)
-    return fail(GR_EUNSUPPORTED, "programs with mutable edge state (scatter) run resident on one GPU");
   Comm *C = g->comm;
+  constexpr bool kScatter = HasScatter<Prog>::value;
+  if constexpr (kScatter) {  // this rank's edges (its CSC and activation CSR) carry the states
+    gr_status ss = scatter_setup(g, Prog::kUsesWeights);
+    if (ss != GR_OK) return ss;
+  }
   Part<OffT> P = make_part<OffT>(g);
   uint64_t launches = 0;
   if (g->epoch_next > 0xF0000000u) {
@@ -113,6 +116,7 @@ gr_status run_frontier_part(gr_graph *g, const gr_run_opts *o, cudaStream_t s, g
   h.kstart[0] = h.kstart[1] = ~0ull;
   PCK(cudaMemcpyAsync(g->ctl, &h, sizeof h, cudaMemcpyHostToDevice, s));
   k_init_values<Prog, OffT><<<g->num_sms * 4, 256, 0, s>>>(P, o->source);
+  if constexpr (kScatter) k_init_edges<Prog, OffT><<<g->num_sms * 8, 256, 0, s>>>(P, g->H.m_in);
   k_fill<typename Prog::GatherT><<<std::min<uint32_t>((g->hub_cap + 255) / 256, 1024), 256, 0, s>>>(
       reinterpret_cast<typename Prog::GatherT *>(g->hub_acc), Prog::identity_host(), g->hub_cap);
   PCK(cudaMemsetAsync(g->hub_done, 0, 4ull * g->hub_cap, s));
@@ -154,7 +158,14 @@ gr_status run_frontier_part(gr_graph *g, const gr_run_opts *o, cudaStream_t s, g
     PCK(cudaMemsetAsync(&g->ctl->cnt_C, 0, sizeof(uint32_t), s));
     if (tot) k_classify<OffT><<<std::min<uint32_t>(grid, (uint32_t)((tot + kBlock - 1) / kBlock)), kBlock, 0, s>>>(
         P, g->X_v, g->X_val, (uint32_t)tot);
-    k_activate<OffT><<<grid, kBlock, 0, s>>>(P, 0ull, 0);
+    if constexpr (kScatter) {
+      // commit every rank's C_t first: scatter reads the committed values of its targets
+      k_commit_only<OffT><<<grid, kBlock, 0, s>>>(P);
+      k_scatter_activate<Prog, OffT><<<grid, kBlock, 0, s>>>(P, 0ull, 0);
+      launches++;
+    } else {
+      k_activate<OffT><<<grid, kBlock, 0, s>>>(P, 0ull, 0);
+    }
     launches += tot ? 3 : 2;
     PCK(cudaGetLastError());
     PCK(cudaMemcpyAsync(g->h_ctl, g->ctl, sizeof(Ctl), cudaMemcpyDeviceToHost, s));

@@ -91,10 +91,14 @@ def test_sim_ranks_hubs_and_configs():
 
 
 @pytest.mark.timeout(600)
-def test_sim_ranks_custom_program():
+@pytest.mark.parametrize("prog", [(0, "widest"), (1, "sssp_msg")])
+def test_sim_ranks_custom_program(prog):
+    """Registered programs over owner partitions; id 1 (SSSP by edge messages)
+    keeps its edge states on the rank that owns the edge's destination."""
+    pid, oname = prog
     g = grgen.rmat(12, 16, seed=3)
     w = grgen.weights(g.m, 1, 64, seed=4)
-    ref, rtr, rit = oracle.run(g.n, g.src, g.dst, "widest", w=w, source=0)
+    ref, rtr, rit = oracle.run(g.n, g.src, g.dst, oname, w=w, source=0)
     import os
     import threading
 
@@ -105,7 +109,7 @@ def test_sim_ranks_custom_program():
         h = None
         try:
             h = gr.gr_graph_load(g.n, g.src, g.dst, w, world=2, rank=r, sim_ranks=2, nccl_unique_id=key)
-            gr.gr_run(h, "custom", custom_id=0, source=0)
+            gr.gr_run(h, "custom", custom_id=pid, source=0)
             out[r] = (gr.gr_fetch_vertex_values(h), gr.gr_fetch_frontier_trace(h))
         except Exception as e:
             errs.append(e)
