@@ -120,7 +120,10 @@ __global__ void k_s_bfs_apply(const __grid_constant__ Part<OffT> P, uint32_t v0,
 }
 
 // FrontierActivate for the changed vertices of one shard (out-edges in a slot).
-template <class OffT>
+// kHasScatter programs first run scatter on every expanded edge (values are
+// committed by k_s_commit; the edge states live in mapped host memory and
+// are updated in place over the host link, P.estate / P.out_eid / P.out_w).
+template <class Prog, class OffT>
 __global__ void __launch_bounds__(kBlock) k_s_activate(const __grid_constant__ Part<OffT> P, uint32_t u0,
                                                        uint32_t u1, const uint64_t *bounds, uint32_t nshards,
                                                        uint8_t *next_flags, const uint32_t *cstamp) {
@@ -128,21 +131,36 @@ __global__ void __launch_bounds__(kBlock) k_s_activate(const __grid_constant__ P
   const uint32_t t = ctl->iter;
   const uint32_t epoch_t = ctl->epoch_base + t, epoch_n = epoch_t + 1;
   const uint32_t warp_lane = lane_id();
+  Ctx cx{};
+  cx.iter = t;
+  cx.n = P.n;
+  cx.source = ctl->source;
+  cx.outdeg = P.outdeg;
   unsigned long long my_s = 0, my_act = 0;
   const uint32_t gw = blockIdx.x * kWarpsPerBlock + threadIdx.x / 32, nw = gridDim.x * kWarpsPerBlock;
   for (uint32_t base = u0 + gw * 32u; base < u1; base += nw * 32u) {
     const uint32_t u = base + warp_lane;
     const bool valid = u < u1 && cstamp[u - P.own_lo] == epoch_t;
     uint64_t beg = 0;
-    uint32_t deg = 0;
+    uint32_t deg = 0, uval = 0;
     if (valid) {
       beg = (uint64_t)P.out_off[u];
       deg = (uint32_t)((uint64_t)P.out_off[u + 1] - beg);
       my_s += deg;
+      if constexpr (HasScatter<Prog>::value) uval = P.val[u];  // committed value of t
     }
     // expand: stamp targets with epoch t+1; first stamper flags the target's shard
     uint32_t big = __ballot_sync(0xffffffffu, valid && deg > 32);
-    auto act_one = [&](bool act, uint32_t x) {
+    auto act_one = [&](bool act, uint32_t x, uint64_t e, uint32_t sv) {
+      if constexpr (HasScatter<Prog>::value) {
+        if (act) {
+          const uint32_t w = Prog::kUsesWeights ? (uint32_t)P.out_w[e] : 0u;
+          Prog::scatter(sv, ld_cg(P.val + x), w, P.estate + P.out_eid[e], cx);
+        }
+      } else {
+        (void)e;
+        (void)sv;
+      }
       bool newly = false;
       if (act) newly = stamp_first(P.stamp + (x - P.own_lo), epoch_n);
       if (newly) next_flags[shard_of(bounds, nshards, x)] = 1;
@@ -153,10 +171,11 @@ __global__ void __launch_bounds__(kBlock) k_s_activate(const __grid_constant__ P
       big &= big - 1;
       const uint64_t b = __shfl_sync(0xffffffffu, beg, L);
       const uint32_t d = __shfl_sync(0xffffffffu, deg, L);
+      const uint32_t sv = __shfl_sync(0xffffffffu, uval, L);
       for (uint32_t r0 = 0; r0 < d; r0 += 32) {
         const uint32_t k = r0 + warp_lane;
         const bool a = k < d;
-        my_act += act_one(a, a ? ldg_nc(P.out_dst + b + k) : 0u);
+        my_act += act_one(a, a ? ldg_nc(P.out_dst + b + k) : 0u, b + k, sv);
       }
     }
     const uint32_t sd = (valid && deg <= 32) ? deg : 0u;
@@ -172,8 +191,9 @@ __global__ void __launch_bounds__(kBlock) k_s_activate(const __grid_constant__ P
       }
       const uint64_t ob = __shfl_sync(0xffffffffu, beg, o);
       const uint32_t oe = __shfl_sync(0xffffffffu, excl, o);
+      const uint32_t sv = __shfl_sync(0xffffffffu, uval, o);
       const bool a = k < total;
-      my_act += act_one(a, a ? ldg_nc(P.out_dst + ob + (k - oe)) : 0u);
+      my_act += act_one(a, a ? ldg_nc(P.out_dst + ob + (k - oe)) : 0u, ob + (k - oe), sv);
     }
   }
   my_s = warp_sum_u64(my_s);
@@ -186,6 +206,24 @@ __global__ void __launch_bounds__(kBlock) k_s_activate(const __grid_constant__ P
 // Close the superstep (one CTA): the same bookkeeping as the resident path.
 template <class OffT> __global__ void k_s_finish(const __grid_constant__ Part<OffT> P) {
   finish_superstep(P, 0ull, 0, kPush);
+}
+
+// kHasScatter programs whose source changes at init: it scatters over its out-edges.
+template <class Prog, class OffT>
+__global__ void k_s_init_scatter(const __grid_constant__ Part<OffT> P, uint32_t source) {
+  if constexpr (HasScatter<Prog>::value) {
+    Ctx cx{};
+    cx.n = P.n;
+    cx.source = source;
+    cx.outdeg = P.outdeg;
+    const uint64_t b = (uint64_t)P.out_off[source], e1 = (uint64_t)P.out_off[source + 1];
+    const uint32_t sv = P.val[source];
+    for (uint64_t e = b + threadIdx.x; e < e1; e += blockDim.x) {
+      const uint32_t x = P.out_dst[e];
+      const uint32_t w = Prog::kUsesWeights ? (uint32_t)P.out_w[e] : 0u;
+      Prog::scatter(sv, P.val[x], w, P.estate + P.out_eid[e], cx);
+    }
+  }
 }
 
 // Stamp a host-computed starting frontier (SSSP: out-neighbours of the source).

@@ -52,7 +52,53 @@ struct Streamer {
   const uint8_t *zc_w = nullptr;
   uint64_t bytes_zc = 0;
   uint32_t zc_phases = 0;
+  // mutable edge state (kHasScatter programs): CSC-ordered states and the CSR -> CSC
+  // position map in mapped pinned host memory, read and written in place over the link
+  uint32_t *h_es = nullptr, *h_eid = nullptr;
+  uint32_t *zc_es = nullptr, *zc_eid = nullptr;
+  uint8_t *zc_ow = nullptr;
 };
+
+// Edge-state layout of a streamed graph (once): the CSR -> CSC position map by a
+// stable bucket pass of the CSC positions over their sources (the host CSR is
+// ordered (src, dst, w), the CSC (dst, src, w): bucketing the CSC by source in
+// order reproduces the CSR order), the state array, the CSR weights mapped.
+static gr_status stream_scatter_setup(gr_graph *g, Streamer *S) {
+  HostGraph &H = g->H;
+  const uint64_t m = H.m_in;
+  if (!S->h_es) {
+    if (H.out_off.size() != H.n + 1) return fail(GR_EUNSUPPORTED, "streamed edge state needs the host CSR offsets");
+    SCK(cudaHostAlloc((void **)&S->h_es, 4 * std::max<uint64_t>(m, 1), cudaHostAllocMapped));
+    SCK(cudaHostAlloc((void **)&S->h_eid, 4 * std::max<uint64_t>(m, 1), cudaHostAllocMapped));
+    g->pinned_bytes += 8 * m;
+    std::vector<uint64_t> pos(H.out_off.begin(), H.out_off.end() - 1);
+    const uint32_t *src = H.in_src.as<uint32_t>();
+    for (uint64_t e = 0; e < m; e++) S->h_eid[pos[src[e]]++] = (uint32_t)e;
+    void *dp = nullptr;
+    SCK(cudaHostGetDevicePointer(&dp, S->h_es, 0));
+    S->zc_es = (uint32_t *)dp;
+    SCK(cudaHostGetDevicePointer(&dp, S->h_eid, 0));
+    S->zc_eid = (uint32_t *)dp;
+    if (H.out_w.p && H.out_w.bytes && !H.out_w.registered) {
+      cudaError_t e = cudaHostRegister(H.out_w.p, H.out_w.bytes, cudaHostRegisterMapped);
+      if (e != cudaSuccess) {
+        cudaGetLastError();
+        return fail(GR_ENOMEM, "cudaHostRegister(out_w): %s", cudaGetErrorString(e));
+      }
+      H.out_w.registered = true;
+      g->pinned_bytes += H.out_w.bytes;
+    }
+    if (H.out_w.p && H.out_w.bytes) {
+      SCK(cudaHostGetDevicePointer(&dp, H.out_w.p, 0));
+      S->zc_ow = (uint8_t *)dp;
+    }
+  }
+  // every Part of this run (make_part) carries the mapped views
+  g->estate = S->zc_es;
+  g->out_eid = S->zc_eid;
+  g->out_w = S->zc_ow;
+  return GR_OK;
+}
 
 // auto mode: read in place when the frontier's edges are < 1/kZcDiv of the
 // edges a whole-shard DMA of the active shards would move
@@ -152,6 +198,11 @@ void stream_destroy(gr_graph *g) {
   }
   if (S->copy_s) cudaStreamDestroy(S->copy_s);
   if (S->h_flags) cudaFreeHost(S->h_flags);
+  if (S->h_es) cudaFreeHost(S->h_es);
+  if (S->h_eid) cudaFreeHost(S->h_eid);
+  if (g->estate == S->zc_es) g->estate = nullptr;
+  if (g->out_eid == S->zc_eid) g->out_eid = nullptr;
+  if (g->out_w == S->zc_ow) g->out_w = nullptr;
   delete S;
   g->streamer = nullptr;
 }
@@ -275,11 +326,15 @@ static gr_status stream_pagerank(gr_graph *g, const gr_run_opts *o, cudaStream_t
 // ------------------------------------------------------- frontier programs
 template <class Prog, class OffT>
 static gr_status stream_frontier(gr_graph *g, const gr_run_opts *o, cudaStream_t cs, gr_run_stats *st) {
-  if constexpr (HasScatter<Prog>::value)
-    return fail(GR_EUNSUPPORTED, "programs with mutable edge state (scatter) run resident on one GPU");
   Streamer *S = S_(g);
   const HostGraph &H = g->H;
   const uint32_t P = S->P;
+  constexpr bool kScatter = HasScatter<Prog>::value;
+  if constexpr (kScatter) {
+    gr_status ss = stream_scatter_setup(g, S);
+    if (ss != GR_OK) return ss;
+    if (Prog::kUsesWeights && !S->zc_ow) return fail(GR_EINVAL, "the program reads edge weights but the graph has none");
+  }
   Part<OffT> P0 = make_part<OffT>(g);
   uint64_t launches = 0;
   if (g->epoch_next > 0xF0000000u) {
@@ -308,6 +363,14 @@ static gr_status stream_frontier(gr_graph *g, const gr_run_opts *o, cudaStream_t
   SCK(cudaMemcpyAsync(g->ctl, &h, sizeof h, cudaMemcpyHostToDevice, cs));
   k_init_values<Prog, OffT><<<g->num_sms * 4, 256, 0, cs>>>(P0, o->source);
   launches++;
+  if constexpr (kScatter) {  // states in host memory, written in place; the source scatters at init
+    k_init_edges<Prog, OffT><<<g->num_sms * 8, 256, 0, cs>>>(P0, H.m_in);
+    launches++;
+    if (Prog::kInit == kInitSourceChanged) {
+      k_s_init_scatter<Prog, OffT><<<1, kBlock, 0, cs>>>(zc_part<OffT>(g, S, false), o->source);
+      launches++;
+    }
+  }
   auto shard_of_host = [&](uint64_t x) {
     return (uint32_t)(std::upper_bound(H.bounds.begin(), H.bounds.end(), x) - H.bounds.begin() - 1);
   };
@@ -391,7 +454,7 @@ static gr_status stream_frontier(gr_graph *g, const gr_run_opts *o, cudaStream_t
     const Part<OffT> Pz_out = zc_part<OffT>(g, S, false);
     if (zc_a && shard_o) {  // in place: one launch over every shard (changed stamps select C_t)
       const uint32_t u0 = (uint32_t)H.bounds[0], u1 = (uint32_t)H.bounds[P];
-      k_s_activate<OffT><<<grid_for(g, u1 - u0), kBlock, 0, cs>>>(Pz_out, u0, u1, S->d_bounds, P, S->d_next,
+      k_s_activate<Prog, OffT><<<grid_for(g, u1 - u0), kBlock, 0, cs>>>(Pz_out, u0, u1, S->d_bounds, P, S->d_next,
                                                                   S->cstamp);
       launches++;
     }
@@ -404,7 +467,7 @@ static gr_status stream_frontier(gr_graph *g, const gr_run_opts *o, cudaStream_t
         if (gs != GR_OK) return gs;
       }
       const Part<OffT> Pk = zc_a ? Pz_out : slot_part<OffT>(g, S, k, false, s);
-      k_s_activate<OffT><<<grid_for(g, u1 - u0), kBlock, 0, cs>>>(Pk, u0, u1, S->d_bounds, P, S->d_next, S->cstamp);
+      k_s_activate<Prog, OffT><<<grid_for(g, u1 - u0), kBlock, 0, cs>>>(Pk, u0, u1, S->d_bounds, P, S->d_next, S->cstamp);
       if (k >= 0) SCK(cudaEventRecord(S->freed[k], cs));
       launches++;
     }

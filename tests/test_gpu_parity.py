@@ -547,10 +547,18 @@ def test_custom_program_edge_messages():
                     assert st["pull_supersteps"] == 0
 
 
-def test_edge_messages_unsupported_outside_resident():
-    g = grgen.rmat(10, 8, seed=3)
-    w = grgen.weights(g.m, 1, 64, seed=4)
-    with gr.GraphReduce(g.n, g.src, g.dst, w, mode="streamed", shard_edges=2000) as G:
-        with pytest.raises(gr.GrError) as e:
-            G.run("custom", custom_id=1, source=0)
-        assert "scatter" in str(e.value)
+@pytest.mark.parametrize("zero_copy", [-1, 0, 1])
+def test_edge_messages_streamed(zero_copy):
+    """Streamed (out-of-core) runs of the scatter program: the edge states live in
+    mapped pinned host memory and are read by the gathers and rewritten by the
+    scatters in place over the host link; shards copied or read in place."""
+    g = grgen.rmat(11, 16, seed=5)
+    w = grgen.weights(g.m, 1, 64, seed=6)
+    ref, rtr, rit = oracle.run(g.n, g.src, g.dst, "sssp_msg", w=w, source=0)
+    with gr.GraphReduce(g.n, g.src, g.dst, w, mode="streamed", shard_edges=3000) as G:
+        assert G.info()["mode"] == gr.MODES["streamed"]
+        for _ in range(2):
+            st = G.run("custom", custom_id=1, source=0, zero_copy=zero_copy)
+            assert st["iterations"] == rit
+            np.testing.assert_array_equal(G.values(), ref)
+            np.testing.assert_array_equal(G.trace(), rtr)
