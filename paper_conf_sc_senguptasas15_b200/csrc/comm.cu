@@ -49,6 +49,15 @@ struct NcclComm : Comm {
       for (int i = 0; i < k; i++) out[q * k + i] = h_small[q * 8 + i];
     return GR_OK;
   }
+  gr_status allgather_dev(const uint64_t *d_mine, int k, uint64_t *out, cudaStream_t s) override {
+    if (k > 8) return GR_EINVAL;
+    if (ncclAllGather(d_mine, d_small, k, ncclUint64, comm, s) != ncclSuccess) return GR_ENCCL;
+    if (cudaMemcpyAsync(h_small, d_small, 8ull * k * world, cudaMemcpyDeviceToHost, s) != cudaSuccess ||
+        cudaStreamSynchronize(s) != cudaSuccess)
+      return GR_ECUDA;
+    for (int i = 0; i < k * world; i++) out[i] = h_small[i];
+    return GR_OK;
+  }
   gr_status share_buffer(void *local, std::vector<void *> *out, cudaStream_t s) override {
     static_assert(sizeof(cudaIpcMemHandle_t) == 64, "IPC handle is 8 words");
     cudaIpcMemHandle_t h;
@@ -152,6 +161,14 @@ struct SimComm : Comm {
       for (int i = 0; i < k; i++) out[q * k + i] = grp->small[q * 8 + i];
     if (!grp->barrier()) return GR_ENCCL;
     return GR_OK;
+  }
+  gr_status allgather_dev(const uint64_t *d_mine, int k, uint64_t *out, cudaStream_t s) override {
+    if (k > 8) return fail_all(GR_EINVAL);
+    uint64_t mine[8];
+    if (cudaMemcpyAsync(mine, d_mine, 8ull * k, cudaMemcpyDeviceToHost, s) != cudaSuccess ||
+        cudaStreamSynchronize(s) != cudaSuccess)
+      return fail_all(GR_ECUDA);
+    return allgather_small(mine, k, out, s);
   }
   gr_status share_buffer(void *local, std::vector<void *> *out, cudaStream_t s) override {
     if (cudaStreamSynchronize(s) != cudaSuccess) return fail_all(GR_ECUDA);

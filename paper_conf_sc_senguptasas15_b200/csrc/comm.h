@@ -29,6 +29,9 @@ struct Comm {
                                const std::vector<uint64_t> &displs, cudaStream_t s) = 0;
   // allgather of k host uint64 per rank (synchronous w.r.t. s): out[r*k + i]
   virtual gr_status allgather_small(const uint64_t *mine, int k, uint64_t *out, cudaStream_t s) = 0;
+  // the same for k <= 8 uint64 already in DEVICE memory (stream-ordered after the
+  // kernel that wrote them; one host synchronisation): out[r*k + i]
+  virtual gr_status allgather_dev(const uint64_t *d_mine, int k, uint64_t *out, cudaStream_t s) = 0;
   // Map every rank's device buffer `local` into this rank: out[q] is rank q's
   // buffer (out[rank] = local). NCCL: cudaIpc handles exchanged with
   // allgather_small and opened with peer access (NVLink); the mappings are

@@ -115,6 +115,7 @@ struct gr_graph {
   bool sim = false;
   uint32_t *X_v = nullptr, *X_val = nullptr;  // exchanged changed set
   float *rank_all = nullptr;                  // PageRank fetch assembly
+  uint64_t *x_cnt = nullptr;                  // per-superstep (|C_t|, |A_t|) for the count exchange
   // PageRank fused exchange: every other rank's contribution replica (by parity),
   // peer-mapped (cudaIpc, NCCL mode) or same-device (simulated ranks)
   float *pr_peer[2][15] = {};

@@ -43,6 +43,7 @@ gr_status part_setup(gr_graph *g) {
   if ((s = dev_alloc(g, (void **)&g->X_v, 4 * n)) != GR_OK) return s;
   if ((s = dev_alloc(g, (void **)&g->X_val, 4 * n)) != GR_OK) return s;
   if ((s = dev_alloc(g, (void **)&g->rank_all, 4 * n)) != GR_OK) return s;
+  if ((s = dev_alloc(g, (void **)&g->x_cnt, 64)) != GR_OK) return s;
   // PageRank fused exchange: map every peer's contribution replicas (both
   // parities). Without a mapping (no peer access) PageRank exchanges with NCCL.
   Comm *C = g->comm;
@@ -90,6 +91,12 @@ static gr_status global_sum(Comm *c, uint64_t mine, uint64_t *out, cudaStream_t 
   return st;
 }
 
+// (|C_t|, |A_t|) of this rank for the count exchange, read where the kernels left them
+static __global__ void k_part_counts(const Ctl *ctl, uint64_t *out) {
+  out[0] = ctl->cnt_C;
+  out[1] = ctl->cnt_act[ctl->iter & 1u];
+}
+
 template <class Prog, class OffT>
 gr_status run_frontier_part(gr_graph *g, const gr_run_opts *o, cudaStream_t s, gr_run_stats *st) {
   Comm *C = g->comm;
@@ -131,26 +138,27 @@ gr_status run_frontier_part(gr_graph *g, const gr_run_opts *o, cudaStream_t s, g
   launches += 3;
   PCK(cudaGetLastError());
   PCK(cudaMemsetAsync(&g->ctl->stop, 0, sizeof(uint32_t), s));  // the host decides termination
-  PCK(cudaMemcpyAsync(g->h_ctl, g->ctl, sizeof(Ctl), cudaMemcpyDeviceToHost, s));
-  PCK(cudaStreamSynchronize(s));
-  uint64_t active = 0;
-  XCK(global_sum(C, g->h_ctl->cnt_act[0], &active, s));
   uint32_t t = 0;
-  std::vector<uint64_t> cnt(C->world), dsp(C->world), all(C->world);
+  std::vector<uint64_t> cnt(C->world), dsp(C->world), all(2 * C->world);
   const uint32_t grid = g->grid_frontier;
-  while (active > 0 && (o->max_iters == 0 || t < o->max_iters)) {
+  // One host synchronisation per superstep: after the gather, every rank's
+  // (|C_t|, |A_t|) pair is allgathered straight from device memory; it sizes
+  // the exchange of C_t and decides termination (no active vertex on any rank:
+  // the gather of an empty frontier changed nothing and the run ends at t).
+  while (o->max_iters == 0 || t < o->max_iters) {
     k_gather_apply<Prog, OffT><<<grid, kBlock, 0, s>>>(P);
-    PCK(cudaMemcpyAsync(g->h_ctl, g->ctl, sizeof(Ctl), cudaMemcpyDeviceToHost, s));
-    PCK(cudaStreamSynchronize(s));
-    // exchange the changed set C_t (vertex, new value)
-    const uint64_t mine = g->h_ctl->cnt_C;
-    XCK(C->allgather_small(&mine, 1, all.data(), s));
-    uint64_t tot = 0;
+    k_part_counts<<<1, 1, 0, s>>>(g->ctl, g->x_cnt);
+    launches += 2;
+    XCK(C->allgather_dev(g->x_cnt, 2, all.data(), s));
+    uint64_t tot = 0, active = 0;
     for (int q = 0; q < C->world; q++) {
-      cnt[q] = 4 * all[q];
+      cnt[q] = 4 * all[2 * q];
       dsp[q] = 4 * tot;
-      tot += all[q];
+      tot += all[2 * q];
+      active += all[2 * q + 1];
     }
+    if (active == 0) break;
+    // exchange the changed set C_t (vertex, new value)
     if (tot) {
       XCK(C->allgatherv(g->C_v, g->X_v, cnt, dsp, s));
       XCK(C->allgatherv(g->C_val, g->X_val, cnt, dsp, s));
@@ -166,13 +174,12 @@ gr_status run_frontier_part(gr_graph *g, const gr_run_opts *o, cudaStream_t s, g
     } else {
       k_activate<OffT><<<grid, kBlock, 0, s>>>(P, 0ull, 0);
     }
-    launches += tot ? 3 : 2;
+    launches += tot ? 2 : 1;
     PCK(cudaGetLastError());
-    PCK(cudaMemcpyAsync(g->h_ctl, g->ctl, sizeof(Ctl), cudaMemcpyDeviceToHost, s));
-    PCK(cudaStreamSynchronize(s));
-    t = g->h_ctl->iter;
-    XCK(global_sum(C, g->h_ctl->cnt_act[t & 1u], &active, s));
+    t++;
   }
+  PCK(cudaMemcpyAsync(g->h_ctl, g->ctl, sizeof(Ctl), cudaMemcpyDeviceToHost, s));
+  PCK(cudaStreamSynchronize(s));
   const Ctl &c = *g->h_ctl;
   uint64_t v[2] = {c.tot_gathered, c.tot_scattered}, av[64];
   XCK(C->allgather_small(v, 2, av, s));
