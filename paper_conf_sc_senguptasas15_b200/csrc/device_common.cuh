@@ -155,6 +155,16 @@ template <class OffT> struct Part {
   const ulonglong2 *prd_div;  // ProgPRDelta divisor table (Ctx::prd_div), or nullptr
   uint32_t *estate;       // [m_in] edge states in CSC order (programs with kHasScatter)
   const uint32_t *out_eid;// [m_in] CSC position of every activation-CSR edge (kHasScatter)
+  // dense (pull) supersteps of kDstFreeGather programs: edge-segmented tiles over the
+  // CSC (kernels_frontier.cuh dense_seg_phase); ds_tiles == 0: not built
+  const uint32_t *ds_src;  // [tiles * 256] CSC sources, kDsNoSrc for an empty row's item and the padding
+  const uint8_t *ds_w;     // [tiles * 256] weights per item (weighted graphs)
+  const uint32_t *ds_flags;// head bit of the first item of every row (+ a sentinel)
+  const uint32_t *ds_row;  // [tiles] row of each tile's first item
+  const uint32_t *ds_split;// rows with items in more than one tile
+  void *ds_acc;            // [own_n] GatherT slots (8 B) of the split rows, identity between uses
+  uint32_t *ds_act;        // [own_n / 32 + 1] active bits of the split rows
+  uint32_t ds_tiles, ds_nsplit;
   uint32_t *nxt[2];       // fused push supersteps: per-vertex gather accumulators by parity (GatherT = u32)
   const uint8_t *out_w;   // activation CSR weights (fused push supersteps of weighted programs)
   uint32_t n_s_hubs, n_s_chunks;

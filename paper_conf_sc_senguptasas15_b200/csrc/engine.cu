@@ -296,6 +296,94 @@ gr_status load_device(gr_graph *g) {
 }
 
 // -------------------------------------------------------------- frontier run
+// Dense edge-segmented layout (kernels_frontier.cuh dense_seg_phase), once per
+// graph: the PageRank seg layout over the CSC without hot tags (items =
+// max(indeg, 1) per row, kDsNoSrc for an empty row's item and the padding),
+// the weights per item, each tile's first row, and the rows spanning tiles.
+template <class OffT>
+static __global__ void k_ds_fill_w(const OffT *in_off, uint32_t rows, uint64_t m, const uint8_t *w,
+                                   const uint32_t *seg_off, uint8_t *ds_w) {
+  for (uint64_t e = blockIdx.x * (uint64_t)blockDim.x + threadIdx.x; e < m; e += (uint64_t)gridDim.x * blockDim.x) {
+    uint32_t lo = 0, hi = rows;
+    while (hi - lo > 1) {
+      const uint32_t mid = (lo + hi) >> 1;
+      if ((uint64_t)in_off[mid] <= e) lo = mid;
+      else hi = mid;
+    }
+    ds_w[seg_off[lo] + (e - (uint64_t)in_off[lo])] = w[e];
+  }
+}
+static __global__ void k_ds_tiles(const uint32_t *seg_off, uint32_t rows, uint32_t tiles, uint32_t *ds_row) {
+  for (uint32_t c = blockIdx.x * blockDim.x + threadIdx.x; c < tiles; c += gridDim.x * blockDim.x) {
+    const uint64_t i0 = (uint64_t)c * kDsTile;
+    uint32_t lo = 0, hi = rows;  // last r with seg_off[r] <= i0
+    while (hi - lo > 1) {
+      const uint32_t mid = (lo + hi) >> 1;
+      if (seg_off[mid] <= i0) lo = mid;
+      else hi = mid;
+    }
+    ds_row[c] = lo;
+  }
+}
+static __global__ void k_ds_split(const uint32_t *seg_off, uint32_t rows, uint32_t *split, uint32_t *nsplit) {
+  for (uint32_t r = blockIdx.x * blockDim.x + threadIdx.x; r < rows; r += gridDim.x * blockDim.x)
+    if (seg_off[r] / kDsTile != (seg_off[r + 1] - 1) / kDsTile) split[atomicAdd(nsplit, 1u)] = r;
+}
+template <class OffT> static gr_status ds_setup(gr_graph *g) {
+  g->ds_tried = true;
+  const HostGraph &H = g->H;
+  cudaStream_t s = g->stream;
+  const uint32_t rows = (uint32_t)H.own_n();
+  const uint64_t m = H.m_in;
+  if ((uint64_t)rows + m + 2 * kDsTile >= 0xFFFFFFFFull || rows == 0) return GR_OK;  // stays on the vertex path
+  const OffT *in_off = (const OffT *)g->in_off;
+  uint32_t *seg_off = nullptr, *degp = nullptr, *d_n = nullptr;
+  void *tmp = nullptr;
+  size_t need = 0;
+  CK(pmalloc(&seg_off, 4ull * (rows + 1), s));
+  CK(pmalloc(&degp, 4ull * rows, s));
+  k_seg_deg<OffT><<<g->num_sms * 8, 256, 0, s>>>(in_off, rows, degp);
+  CK(cub::DeviceScan::InclusiveSum(nullptr, need, degp, seg_off + 1, (int64_t)rows, s));
+  CK(pmalloc(&tmp, std::max<size_t>(need, 16), s));
+  CK(cub::DeviceScan::InclusiveSum(tmp, need, degp, seg_off + 1, (int64_t)rows, s));
+  CK(cudaMemsetAsync(seg_off, 0, 4, s));
+  uint32_t items = 0;
+  CK(cudaMemcpyAsync(&items, seg_off + rows, 4, cudaMemcpyDeviceToHost, s));
+  CK(cudaStreamSynchronize(s));
+  const uint32_t tiles = (items + kDsTile - 1) / kDsTile;
+  const uint64_t padded = (uint64_t)tiles * kDsTile;
+  gr_status st;
+  if ((st = dev_alloc(g, (void **)&g->ds_src, 4 * padded + 16)) != GR_OK) return st;
+  if ((st = dev_alloc(g, (void **)&g->ds_flags, 4ull * (tiles + 2) * 8)) != GR_OK) return st;
+  if ((st = dev_alloc(g, (void **)&g->ds_row, 4ull * (tiles + 1))) != GR_OK) return st;
+  if ((st = dev_alloc(g, (void **)&g->ds_split, 4ull * rows)) != GR_OK) return st;
+  if ((st = dev_alloc(g, (void **)&g->ds_acc, 8ull * rows)) != GR_OK) return st;
+  if ((st = dev_alloc(g, (void **)&g->ds_act, 4ull * (rows / 32 + 2))) != GR_OK) return st;
+  CK(cudaMemsetAsync(g->ds_flags, 0, 4ull * (tiles + 2) * 8, s));
+  k_seg_fill<OffT><<<g->num_sms * 16, 256, 0, s>>>(in_off, rows, m, g->in_src, seg_off, g->ds_src);
+  k_seg_rows<OffT><<<g->num_sms * 8, 256, 0, s>>>(in_off, rows, seg_off, g->ds_src, g->ds_flags, kDsNoSrc, padded);
+  if (g->in_w) {
+    if ((st = dev_alloc(g, (void **)&g->ds_w, padded + 16)) != GR_OK) return st;
+    CK(cudaMemsetAsync(g->ds_w, 0, padded + 16, s));
+    k_ds_fill_w<OffT><<<g->num_sms * 16, 256, 0, s>>>(in_off, rows, m, g->in_w, seg_off, g->ds_w);
+  }
+  k_ds_tiles<<<(tiles + 255) / 256, 256, 0, s>>>(seg_off, rows, tiles, g->ds_row);
+  CK(pmalloc(&d_n, 4, s));
+  CK(cudaMemsetAsync(d_n, 0, 4, s));
+  k_ds_split<<<g->num_sms * 8, 256, 0, s>>>(seg_off, rows, g->ds_split, d_n);
+  CK(cudaGetLastError());
+  uint32_t nsplit = 0;
+  CK(cudaMemcpyAsync(&nsplit, d_n, 4, cudaMemcpyDeviceToHost, s));
+  CK(cudaStreamSynchronize(s));
+  pfree(seg_off, s);
+  pfree(degp, s);
+  pfree(tmp, s);
+  pfree(d_n, s);
+  g->ds_tiles = tiles;
+  g->ds_nsplit = nsplit;
+  return GR_OK;
+}
+
 // Tolerance PageRank divisor table: (ceil(2^64 / n_u), n_u); n_u <= 1 keeps m = 0.
 static __global__ void k_prd_div(uint64_t n, const uint32_t *outdeg, ulonglong2 *tab) {
   for (uint64_t v = blockIdx.x * (uint64_t)blockDim.x + threadIdx.x; v < n; v += (uint64_t)gridDim.x * blockDim.x) {
@@ -497,7 +585,32 @@ static gr_status run_frontier(gr_graph *g, const gr_run_opts *o, cudaStream_t s,
   }
   // activation direction (gr_direction); pull needs the bitmaps (resident, one rank);
   // scatter programs always push (the scatter walks the out-edges of C_t)
-  if (g->cbits[0] && !push && !kScatter && o->direction != GR_DIR_PUSH) {
+  const bool may_pull = g->cbits[0] && !push && !kScatter && o->direction != GR_DIR_PUSH;
+  bool dseg = false;
+  if constexpr (DstFree<Prog>::value) {
+    // dense supersteps on edge-segmented tiles: the default for 64-bit gathers
+    // (measured: f2 on cfg2 91 -> 57 ms), opt-in for 32-bit ones (cfg4 CC was
+    // slower, R-MAT SSSP faster: profiles/README.md); GR_DENSE_SEG=0/1 forces
+    const char *e = getenv("GR_DENSE_SEG");
+    const bool want = e ? atoi(e) != 0 : sizeof(typename Prog::GatherT) == 8;
+    const bool ploop = (o->loop == GR_LOOP_AUTO || o->loop == GR_LOOP_PERSISTENT) && g->coop;
+    if (may_pull && want && ploop && !g->ds_tried) {
+      gr_status ds = ds_setup<OffT>(g);
+      if (ds != GR_OK) return ds;
+    }
+    const bool on = may_pull && want && ploop && g->ds_tiles;
+    dseg = on;
+    if (on) {
+      using G = typename Prog::GatherT;
+      k_fill<G><<<g->num_sms * 4, 256, 0, s>>>(reinterpret_cast<G *>(g->ds_acc), Prog::identity_host(),
+                                              g->H.own_n());
+      CK(cudaMemsetAsync(g->ds_act, 0, 4ull * (g->H.own_n() / 32 + 2), s));
+      launches++;
+    }
+    P = make_part<OffT>(g);
+    if (!on) P.ds_tiles = 0;
+  }
+  if (may_pull) {
     uint32_t div = o->pull_div ? o->pull_div : kPullDivDefault;
     if (const char *e = getenv("GR_PULL_DIV")) div = (uint32_t)strtoul(e, nullptr, 10);
     h.pull_div = o->direction == GR_DIR_PULL ? 0xFFFFFFFFu : div;
@@ -522,12 +635,13 @@ static gr_status run_frontier(gr_graph *g, const gr_run_opts *o, cudaStream_t s,
   const bool use_graph = !persistent && (o->loop == GR_LOOP_DEVICE || o->loop == GR_LOOP_AUTO);
   if (persistent) {
     int bps = 0;
-    CK(cudaOccupancyMaxActiveBlocksPerMultiprocessor(&bps, k_persistent<Prog, OffT>, kBlock, 0));
+    const void *kf = dseg ? (const void *)k_persistent_ds<Prog, OffT> : (const void *)k_persistent<Prog, OffT>;
+    CK(cudaOccupancyMaxActiveBlocksPerMultiprocessor(&bps, kf, kBlock, 0));
     int per_sm = std::min(bps, 4);
     if (const char *e = getenv("GR_PERSIST_CTAS_PER_SM")) per_sm = std::min(bps, atoi(e));
     const uint32_t grid = (uint32_t)g->num_sms * (uint32_t)std::max(1, per_sm);
     void *args[] = {(void *)&P};
-    CK(cudaLaunchCooperativeKernel((const void *)k_persistent<Prog, OffT>, dim3(grid), dim3(kBlock), args, 0, s));
+    CK(cudaLaunchCooperativeKernel(kf, dim3(grid), dim3(kBlock), args, 0, s));
     CK(cudaMemcpyAsync(g->h_ctl, g->ctl, sizeof(Ctl), cudaMemcpyDeviceToHost, s));
     CK(cudaStreamSynchronize(s));
     launches += 1;

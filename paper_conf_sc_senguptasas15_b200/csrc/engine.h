@@ -31,7 +31,13 @@ struct gr_graph {
   uint8_t *out_w = nullptr;                       // CSR weights (built on first fused push run)
   uint32_t *nxt[2] = {nullptr, nullptr};          // fused push accumulators (allocated on first use)
   ulonglong2 *prd_div = nullptr;
-  uint32_t *estate = nullptr, *out_eid = nullptr; // mutable edge state (kHasScatter programs; first use)                  // tolerance PageRank divisor table (first GR_PAGERANK_DELTA run)
+  uint32_t *estate = nullptr, *out_eid = nullptr; // mutable edge state (kHasScatter programs; first use)
+  // dense edge-segmented gather layout (kDstFreeGather programs; built on the first run that may pull)
+  uint32_t *ds_src = nullptr, *ds_flags = nullptr, *ds_row = nullptr, *ds_split = nullptr, *ds_act = nullptr;
+  uint8_t *ds_w = nullptr;
+  void *ds_acc = nullptr;
+  uint32_t ds_tiles = 0, ds_nsplit = 0;
+  bool ds_tried = false;                  // tolerance PageRank divisor table (first GR_PAGERANK_DELTA run)
   uint32_t *hub_in = nullptr, *hub_out = nullptr, *static_hubs = nullptr;
   uint32_t n_static_hubs = 0;
   // hub chunk lists (kChunk edges per CTA work item)
@@ -138,6 +144,15 @@ template <class OffT> inline Part<OffT> make_part(gr_graph *g) {
   P.prd_div = g->prd_div;
   P.estate = g->estate;
   P.out_eid = g->out_eid;
+  P.ds_src = g->ds_src;
+  P.ds_w = g->ds_w;
+  P.ds_flags = g->ds_flags;
+  P.ds_row = g->ds_row;
+  P.ds_split = g->ds_split;
+  P.ds_acc = g->ds_acc;
+  P.ds_act = g->ds_act;
+  P.ds_tiles = g->ds_tiles;
+  P.ds_nsplit = g->ds_nsplit;
   P.nxt[0] = g->nxt[0];
   P.nxt[1] = g->nxt[1];
   P.out_w = g->out_w;

@@ -1336,6 +1336,207 @@ __global__ void k_init_edges(const __grid_constant__ Part<OffT> P, uint64_t m) {
   }
 }
 
+// ------------------------------------------------ dense edge-segmented gather
+// Dense (pull) supersteps of kDstFreeGather programs (gr/program.cuh): instead
+// of 32 vertices per warp with a shuffle owner search per edge, the CSC is laid
+// out as 256-item tiles (one item per in-edge, one empty item per row without
+// in-edges, a head bit at each row's first item; the PageRank seg layout
+// without hot tags). A warp walks whole tiles: lane L loads items 8L..8L+7 with
+// two 128-bit loads, maps them (gatherMap of the source's value; the changed
+// bit of the source marks the row active), reduces them in registers and joins
+// rows split between lanes with one segmented shuffle scan. Rows that lie in
+// one tile apply at once; rows spanning tiles (listed once per graph) combine
+// their pieces with atomicGather / atomicOr and apply after a grid barrier
+// (dense_split_phase). gatherReduce is associative and commutative (R9), and
+// exact for every program with this trait (integer min / max / sum), so the
+// result does not depend on the piece order.
+constexpr uint32_t kDsIpt = 8;
+constexpr uint32_t kDsTile = 32 * kDsIpt;
+constexpr uint32_t kDsNoSrc = 0xFFFFFFFFu;
+
+template <class Prog, class OffT>
+__device__ __forceinline__ void ds_apply_row(const Part<OffT> &P, uint32_t lv, typename Prog::GatherT acc,
+                                             const Ctx &cx, WarpQueue &qC, bool p, unsigned long long &my_g,
+                                             unsigned long long &my_c, unsigned long long &my_a, bool no_hub_c) {
+  // every lane calls (qC.push is warp-collective); p: this lane applies row lv
+  bool changed = false, hubo = false;
+  uint32_t v = 0, nv = 0;
+  if (p) {
+    v = P.own_lo + lv;
+    const uint32_t cur = P.val[v];
+    my_g += (uint64_t)P.in_off[lv + 1] - (uint64_t)P.in_off[lv];
+    my_a += 1;
+    nv = cur;
+    changed = Prog::apply(&nv, acc, cx);
+    if (changed) {
+      my_c += 1;
+      hubo = !no_hub_c && test_bit(P.hub_out, v);
+      if (hubo) append_hub_C(P, v, nv);
+    }
+  }
+  qC.push(changed && !hubo, v, nv, P.C_v, P.C_val, &P.ctl->cnt_C);
+}
+
+template <class Prog, class OffT>
+__device__ __forceinline__ void dense_seg_phase(const Part<OffT> &P, const View &V) {
+  using G = typename Prog::GatherT;
+  Ctl *ctl = P.ctl;
+  const uint32_t slot = V.t & 1u;
+  const uint32_t *bits = P.cbits[slot ^ 1u];  // C_{t-1}
+  const Ctx cx = make_ctx(P, V);
+  const bool no_hub_c = V.no_hub_c != 0;
+  prof_begin(ctl, V, 0);
+  __shared__ unsigned long long s8[kWarpsPerBlock];
+  const uint32_t warp = threadIdx.x / 32, lane = lane_id();
+  __shared__ uint32_t sq[kWarpsPerBlock][2][kQueueCap];
+  __shared__ uint32_t s_off[kWarpsPerBlock + 1];
+  WarpQueue qC{sq[warp][0], sq[warp][1], 0};
+  unsigned long long my_g = 0, my_c = 0, my_a = 0;
+  G *acc_g = reinterpret_cast<G *>(P.ds_acc);
+  const uint32_t gw = blockIdx.x * kWarpsPerBlock + warp, nw = gridDim.x * kWarpsPerBlock;
+  for (uint32_t tile = gw; tile < P.ds_tiles; tile += nw) {
+    const uint4 *s4 = reinterpret_cast<const uint4 *>(P.ds_src + (uint64_t)tile * kDsTile) + 2 * lane;
+    const uint4 s0 = __ldg(s4), s1 = __ldg(s4 + 1);
+    const uint32_t fw = __ldg(P.ds_flags + (uint64_t)tile * 8 + (lane >> 2));
+    const uint32_t fnext = __ldg(P.ds_flags + (uint64_t)tile * 8 + 8) & 1u;
+    const uint32_t r0 = __ldg(P.ds_row + tile);
+    const uint32_t src[kDsIpt] = {s0.x, s0.y, s0.z, s0.w, s1.x, s1.y, s1.z, s1.w};
+    uint32_t w8[kDsIpt];
+    if (Prog::kUsesWeights) {
+      const uint2 wv = __ldg(reinterpret_cast<const uint2 *>(P.ds_w + (uint64_t)tile * kDsTile) + lane);
+#pragma unroll
+      for (int k = 0; k < 4; k++) { w8[k] = (wv.x >> (8 * k)) & 0xFFu; w8[k + 4] = (wv.y >> (8 * k)) & 0xFFu; }
+    }
+    uint32_t sv[kDsIpt];
+    bool sa[kDsIpt];
+#pragma unroll
+    for (int k = 0; k < kDsIpt; k++) {  // all loads of the 8 items in flight together
+      const bool ok = src[k] != kDsNoSrc;
+      sv[k] = ok ? __ldg(P.val + src[k]) : 0u;
+      sa[k] = ok && test_bit(bits, src[k]);
+    }
+    G g[kDsIpt];
+#pragma unroll
+    for (int k = 0; k < kDsIpt; k++)
+      g[k] = src[k] != kDsNoSrc ? Prog::gatherMap(0u, sv[k], Prog::kUsesWeights ? w8[k] : 0u, src[k], cx)
+                                : Prog::identity();
+    const uint32_t b = (fw >> ((lane & 3) * 8)) & 0xFFu;  // bit k: my item k starts a row
+    uint32_t bn = __shfl_down_sync(0xffffffffu, b, 1) & 1u;
+    if (lane == 31) bn = fnext;
+    const uint32_t ends = (b >> 1) | (bn << 7);  // bit k: my item k ends a row
+    // lane tail (after my last head) and its active flag
+    G tail = Prog::identity();
+    bool tact = false;
+#pragma unroll
+    for (int k = 0; k < kDsIpt; k++) {
+      if ((b >> k) & 1u) { tail = Prog::identity(); tact = false; }
+      tail = Prog::gatherReduce(tail, g[k]);
+      tact = tact || sa[k];
+    }
+    // segmented inclusive scan of the tails over lanes (segments start at lanes with a head)
+    uint32_t cnt = __popc(b);
+    G x = tail;
+    uint32_t xa = tact ? 1u : 0u;
+    const uint32_t hl = __ballot_sync(0xffffffffu, b != 0u) & (0xFFFFFFFFu >> (31 - lane));
+    const int seg0 = hl ? 31 - __clz(hl) : 0;
+#pragma unroll
+    for (int o = 1; o < 32; o <<= 1) {
+      const G y = __shfl_up_sync(0xffffffffu, x, o);
+      const uint32_t ya = __shfl_up_sync(0xffffffffu, xa, o);
+      const uint32_t c = __shfl_up_sync(0xffffffffu, cnt, o);
+      if ((int)lane - o >= seg0) { x = Prog::gatherReduce(x, y); xa |= ya; }
+      if (lane >= (uint32_t)o) cnt += c;
+    }
+    G run = __shfl_up_sync(0xffffffffu, x, 1);
+    uint32_t ract = __shfl_up_sync(0xffffffffu, xa, 1);
+    if (lane == 0) { run = Prog::identity(); ract = 0u; }
+    const uint32_t h0 = __shfl_sync(0xffffffffu, b, 0) & 1u;
+    uint32_t row = r0 - h0 + (cnt - __popc(b));  // row of the item before my first head
+    // walk my items: complete rows apply (collectively, one row per lane per step),
+    // pieces of rows spanning tiles go to the split accumulators
+    uint32_t done_rows = 0;  // bit k: my item k completes a row that started in this tile
+    G done_val[kDsIpt];
+    bool done_act[kDsIpt];
+#pragma unroll
+    for (int k = 0; k < kDsIpt; k++) {
+      if ((b >> k) & 1u) { run = Prog::identity(); ract = 0u; ++row; }
+      run = Prog::gatherReduce(run, g[k]);
+      ract |= sa[k] ? 1u : 0u;
+      done_val[k] = run;
+      done_act[k] = ract != 0u;
+      if (((ends >> k) & 1u) && row < P.own_n) {
+        if (!h0 && row == r0) {  // began in an earlier tile: a piece
+          Prog::atomicGather(acc_g + row, run);
+          if (ract) atomicOr(P.ds_act + (row >> 5), 1u << (row & 31));
+        } else {
+          done_rows |= 1u << k;
+        }
+      }
+    }
+    if (lane == 31 && !fnext && row < P.own_n) {  // the last row continues in the next tile: a piece
+      Prog::atomicGather(acc_g + row, run);
+      if (ract) atomicOr(P.ds_act + (row >> 5), 1u << (row & 31));
+    }
+    // apply the complete active rows (row counter replayed; warp-collective per item slot)
+    uint32_t rr = r0 - h0 + (cnt - __popc(b));
+#pragma unroll
+    for (int k = 0; k < kDsIpt; k++) {
+      if ((b >> k) & 1u) ++rr;
+      const bool p = ((done_rows >> k) & 1u) && done_act[k];
+      if (__any_sync(0xffffffffu, p))
+        ds_apply_row<Prog>(P, rr, done_val[k], cx, qC, p, my_g, my_c, my_a, no_hub_c);
+    }
+  }
+  qC.block_flush(P.C_v, P.C_val, &ctl->cnt_C, s_off);
+  my_g = block_sum_u64(my_g, s8);
+  if (threadIdx.x == 0 && my_g) atomicAdd(&ctl->part_g[blockIdx.x % kSlots], my_g);
+  my_c = block_sum_u64(my_c, s8);
+  if (threadIdx.x == 0 && my_c) atomicAdd(&ctl->part_c[blockIdx.x % kSlots], my_c);
+  my_a = block_sum_u64(my_a, s8);
+  if (threadIdx.x == 0 && my_a) atomicAdd(&ctl->cnt_act[slot], (uint32_t)my_a);
+  prof_end(ctl, V, 0);
+}
+
+// the rows spanning tiles (after a grid barrier): combined pieces apply, slots reset
+template <class Prog, class OffT>
+__device__ __forceinline__ void dense_split_phase(const Part<OffT> &P, const View &V) {
+  using G = typename Prog::GatherT;
+  Ctl *ctl = P.ctl;
+  const uint32_t slot = V.t & 1u;
+  const Ctx cx = make_ctx(P, V);
+  const bool no_hub_c = V.no_hub_c != 0;
+  __shared__ uint32_t sq[kWarpsPerBlock][2][kQueueCap];
+  __shared__ uint32_t s_off[kWarpsPerBlock + 1];
+  __shared__ unsigned long long s8[kWarpsPerBlock];
+  const uint32_t warp = threadIdx.x / 32;
+  WarpQueue qC{sq[warp][0], sq[warp][1], 0};
+  unsigned long long my_g = 0, my_c = 0, my_a = 0;
+  G *acc_g = reinterpret_cast<G *>(P.ds_acc);
+  const uint32_t gw = blockIdx.x * kWarpsPerBlock + warp, nw = gridDim.x * kWarpsPerBlock;
+  for (uint32_t base = gw * 32u; base < P.ds_nsplit; base += nw * 32u) {
+    const uint32_t i = base + lane_id();
+    bool p = false;
+    uint32_t r = 0;
+    G acc = Prog::identity();
+    if (i < P.ds_nsplit) {
+      r = P.ds_split[i];
+      acc = acc_g[r];
+      acc_g[r] = Prog::identity();
+      const uint32_t m = 1u << (r & 31);
+      p = (ld_cg(P.ds_act + (r >> 5)) & m) != 0u;
+      if (p) atomicAnd(P.ds_act + (r >> 5), ~m);
+    }
+    ds_apply_row<Prog>(P, r, acc, cx, qC, p, my_g, my_c, my_a, no_hub_c);
+  }
+  qC.block_flush(P.C_v, P.C_val, &ctl->cnt_C, s_off);
+  my_g = block_sum_u64(my_g, s8);
+  if (threadIdx.x == 0 && my_g) atomicAdd(&ctl->part_g[blockIdx.x % kSlots], my_g);
+  my_c = block_sum_u64(my_c, s8);
+  if (threadIdx.x == 0 && my_c) atomicAdd(&ctl->part_c[blockIdx.x % kSlots], my_c);
+  my_a = block_sum_u64(my_a, s8);
+  if (threadIdx.x == 0 && my_a) atomicAdd(&ctl->cnt_act[slot], (uint32_t)my_a);
+}
+
 // Software grid barrier for the persistent loop (cooperative launch guarantees
 // that every CTA is resident). Sense by generation counter.
 __device__ __forceinline__ void grid_sync(Ctl *c) {
@@ -1360,8 +1561,8 @@ __device__ __forceinline__ void grid_sync(Ctl *c) {
 // separated by grid barriers instead of kernel boundaries, and CTA 0 closes
 // each superstep while the others wait — no launch or host round trip per
 // superstep (the latency floor of high-diameter graphs, cfg3).
-template <class Prog, class OffT>
-__global__ void __launch_bounds__(kBlock) k_persistent(const __grid_constant__ Part<OffT> P) {
+template <class Prog, class OffT, bool kDS>
+__device__ __forceinline__ void persistent_body(const Part<OffT> &P) {
   Ctl *ctl = P.ctl;
   __shared__ View V;
   for (;;) {
@@ -1389,8 +1590,17 @@ __global__ void __launch_bounds__(kBlock) k_persistent(const __grid_constant__ P
       }
     }
     if (Prog::kHasGather) {
-      if (V.dense) gather_phase<Prog, true>(P, V);
-      else gather_phase<Prog, false>(P, V);
+      if (V.dense) {
+        if constexpr (kDS && DstFree<Prog>::value) {  // edge-segmented tiles, then the split rows
+          dense_seg_phase<Prog>(P, V);
+          grid_sync(ctl);
+          dense_split_phase<Prog>(P, V);
+        } else {
+          gather_phase<Prog, true>(P, V);
+        }
+      } else {
+        gather_phase<Prog, false>(P, V);
+      }
       grid_sync(ctl);
       load_view(ctl, V);
       clear_dirty(P, V, cbits_words(P));
@@ -1413,6 +1623,21 @@ __global__ void __launch_bounds__(kBlock) k_persistent(const __grid_constant__ P
     grid_sync(ctl);
   }
 }
+
+template <class Prog, class OffT>
+__global__ void __launch_bounds__(kBlock) k_persistent(const __grid_constant__ Part<OffT> P) {
+  persistent_body<Prog, OffT, false>(P);
+}
+
+#ifndef GR_JIT
+// the loop with dense supersteps on edge-segmented tiles (a kernel of its own:
+// the tile code's registers would otherwise lower the occupancy of every phase)
+template <class Prog, class OffT>
+__global__ void __launch_bounds__(kBlock, 3) k_persistent_ds(const __grid_constant__ Part<OffT> P) {
+  persistent_body<Prog, OffT, DstFree<Prog>::value>(P);
+}
+#endif
+
 
 // Partitioned runs: split the exchanged changed set (every rank's C_t) into
 // the local non-hub list and the local changed-hub chunks (hub-ness depends on
