@@ -562,3 +562,20 @@ def test_edge_messages_streamed(zero_copy):
             assert st["iterations"] == rit
             np.testing.assert_array_equal(G.values(), ref)
             np.testing.assert_array_equal(G.trace(), rtr)
+
+
+@pytest.mark.parametrize("force", ["1", "0"])
+@pytest.mark.parametrize("algo", ["sssp", "cc", "pagerank_delta"])
+def test_dense_tile_gather_forced(algo, force, monkeypatch):
+    """Dense (pull) supersteps on edge-segmented tiles (GR_DENSE_SEG=1, the
+    default only for 64-bit gathers) and on the vertex path (GR_DENSE_SEG=0):
+    identical values and traces, including hubs whose rows span many tiles."""
+    monkeypatch.setenv("GR_DENSE_SEG", force)
+    g = grgen.rmat(13, 16, seed=21)
+    src, dst = g.src, g.dst
+    if algo == "cc":
+        src, dst = np.concatenate([g.src, g.dst]), np.concatenate([g.dst, g.src])
+    w = grgen.weights(len(src), 1, 64, seed=22)
+    compare(g.n, src, dst, w, algo, loops=("auto",), directions=("pull", "auto"))
+    n, s2, d2, w2 = hub_graph()
+    compare(n, s2, d2, w2, algo, loops=("auto",), directions=("pull",))
