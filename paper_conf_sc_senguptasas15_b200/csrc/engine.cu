@@ -329,27 +329,52 @@ static __global__ void k_ds_split(const uint32_t *seg_off, uint32_t rows, uint32
   for (uint32_t r = blockIdx.x * blockDim.x + threadIdx.x; r < rows; r += gridDim.x * blockDim.x)
     if (seg_off[r] / kDsTile != (seg_off[r + 1] - 1) / kDsTile) split[atomicAdd(nsplit, 1u)] = r;
 }
+// share of the in-edges that sit in rows longer than one tile (the rows the
+// vertex path serves least well: warp-cooperative / hub chunks), once per graph
+template <class OffT> static gr_status ds_long_fraction(gr_graph *g) {
+  const uint32_t rows = (uint32_t)g->H.own_n();
+  std::vector<OffT> hoff(rows + 1);
+  CK(cudaMemcpyAsync(hoff.data(), g->in_off, sizeof(OffT) * (rows + 1), cudaMemcpyDeviceToHost, g->stream));
+  CK(cudaStreamSynchronize(g->stream));
+  uint64_t lng = 0;
+  for (uint32_t r = 0; r < rows; r++) {
+    const uint64_t d = (uint64_t)hoff[r + 1] - (uint64_t)hoff[r];
+    if (d > kDsTile) lng += d;
+  }
+  g->ds_long_frac = g->H.m_in ? (double)lng / (double)g->H.m_in : 0.0;
+  return GR_OK;
+}
+
 template <class OffT> static gr_status ds_setup(gr_graph *g) {
   g->ds_tried = true;
   const HostGraph &H = g->H;
   cudaStream_t s = g->stream;
   const uint32_t rows = (uint32_t)H.own_n();
   const uint64_t m = H.m_in;
-  if ((uint64_t)rows + m + 2 * kDsTile >= 0xFFFFFFFFull || rows == 0) return GR_OK;  // stays on the vertex path
+  if (rows == 0) return GR_OK;
   const OffT *in_off = (const OffT *)g->in_off;
-  uint32_t *seg_off = nullptr, *degp = nullptr, *d_n = nullptr;
-  void *tmp = nullptr;
-  size_t need = 0;
-  CK(pmalloc(&seg_off, 4ull * (rows + 1), s));
-  CK(pmalloc(&degp, 4ull * rows, s));
-  k_seg_deg<OffT><<<g->num_sms * 8, 256, 0, s>>>(in_off, rows, degp);
-  CK(cub::DeviceScan::InclusiveSum(nullptr, need, degp, seg_off + 1, (int64_t)rows, s));
-  CK(pmalloc(&tmp, std::max<size_t>(need, 16), s));
-  CK(cub::DeviceScan::InclusiveSum(tmp, need, degp, seg_off + 1, (int64_t)rows, s));
-  CK(cudaMemsetAsync(seg_off, 0, 4, s));
-  uint32_t items = 0;
-  CK(cudaMemcpyAsync(&items, seg_off + rows, 4, cudaMemcpyDeviceToHost, s));
+  // Row placement (host, once per graph): items = max(indeg, 1) per row; a row
+  // of at most one tile that would cross a tile boundary starts at the next
+  // tile instead (the gap is padding, absorbed by the previous row as identity
+  // items), so only rows longer than a tile are split between tiles.
+  std::vector<OffT> hoff(rows + 1);
+  CK(cudaMemcpyAsync(hoff.data(), in_off, sizeof(OffT) * (rows + 1), cudaMemcpyDeviceToHost, s));
   CK(cudaStreamSynchronize(s));
+  std::vector<uint32_t> pos(rows + 1);
+  uint64_t p = 0;
+  for (uint32_t r = 0; r < rows; r++) {
+    const uint64_t d = (uint64_t)hoff[r + 1] - (uint64_t)hoff[r];
+    const uint64_t L = d ? d : 1;
+    if (L <= kDsTile && (p % kDsTile) + L > kDsTile) p = (p + kDsTile - 1) / kDsTile * kDsTile;
+    if (p + L + 2 * kDsTile >= 0xFFFFFFFFull) return GR_OK;  // stays on the vertex path
+    pos[r] = (uint32_t)p;
+    p += L;
+  }
+  pos[rows] = (uint32_t)p;
+  const uint32_t items = (uint32_t)p;
+  uint32_t *seg_off = nullptr, *d_n = nullptr;
+  CK(pmalloc(&seg_off, 4ull * (rows + 1), s));
+  CK(cudaMemcpyAsync(seg_off, pos.data(), 4ull * (rows + 1), cudaMemcpyHostToDevice, s));
   const uint32_t tiles = (items + kDsTile - 1) / kDsTile;
   const uint64_t padded = (uint64_t)tiles * kDsTile;
   gr_status st;
@@ -360,6 +385,7 @@ template <class OffT> static gr_status ds_setup(gr_graph *g) {
   if ((st = dev_alloc(g, (void **)&g->ds_acc, 8ull * rows)) != GR_OK) return st;
   if ((st = dev_alloc(g, (void **)&g->ds_act, 4ull * (rows / 32 + 2))) != GR_OK) return st;
   CK(cudaMemsetAsync(g->ds_flags, 0, 4ull * (tiles + 2) * 8, s));
+  k_fill_u32<<<g->num_sms * 8, 256, 0, s>>>(g->ds_src, kDsNoSrc, padded);  // padding between rows
   k_seg_fill<OffT><<<g->num_sms * 16, 256, 0, s>>>(in_off, rows, m, g->in_src, seg_off, g->ds_src);
   k_seg_rows<OffT><<<g->num_sms * 8, 256, 0, s>>>(in_off, rows, seg_off, g->ds_src, g->ds_flags, kDsNoSrc, padded);
   if (g->in_w) {
@@ -376,8 +402,6 @@ template <class OffT> static gr_status ds_setup(gr_graph *g) {
   CK(cudaMemcpyAsync(&nsplit, d_n, 4, cudaMemcpyDeviceToHost, s));
   CK(cudaStreamSynchronize(s));
   pfree(seg_off, s);
-  pfree(degp, s);
-  pfree(tmp, s);
   pfree(d_n, s);
   g->ds_tiles = tiles;
   g->ds_nsplit = nsplit;
@@ -589,11 +613,26 @@ static gr_status run_frontier(gr_graph *g, const gr_run_opts *o, cudaStream_t s,
   bool dseg = false;
   if constexpr (DstFree<Prog>::value) {
     // dense supersteps on edge-segmented tiles: the default for 64-bit gathers
-    // (measured: f2 on cfg2 91 -> 57 ms), opt-in for 32-bit ones (cfg4 CC was
-    // slower, R-MAT SSSP faster: profiles/README.md); GR_DENSE_SEG=0/1 forces
+    // and for graphs with >= 25 % of their in-edges in rows longer than a tile
+    // (measured on R-MAT: tolerance PageRank 89.8 -> 56.8 ms, CC 4.9 -> 2.8 ms,
+    // SSSP 0.89 -> 0.67 ms; the web graph of cfg4 (12 %) stays on the vertex
+    // path: 12.3 vs 13.2 ms; profiles/README.md); GR_DENSE_SEG=0/1 forces
     const char *e = getenv("GR_DENSE_SEG");
-    const bool want = e ? atoi(e) != 0 : sizeof(typename Prog::GatherT) == 8;
     const bool ploop = (o->loop == GR_LOOP_AUTO || o->loop == GR_LOOP_PERSISTENT) && g->coop;
+    bool want = false;
+    if (e) {
+      want = atoi(e) != 0;
+    } else if (may_pull && ploop) {
+      if (sizeof(typename Prog::GatherT) == 8) {
+        want = true;
+      } else {
+        if (g->ds_long_frac < 0) {
+          gr_status lf = ds_long_fraction<OffT>(g);
+          if (lf != GR_OK) return lf;
+        }
+        want = g->ds_long_frac >= 0.25;
+      }
+    }
     if (may_pull && want && ploop && !g->ds_tried) {
       gr_status ds = ds_setup<OffT>(g);
       if (ds != GR_OK) return ds;

@@ -37,7 +37,8 @@ struct gr_graph {
   uint8_t *ds_w = nullptr;
   void *ds_acc = nullptr;
   uint32_t ds_tiles = 0, ds_nsplit = 0;
-  bool ds_tried = false;                  // tolerance PageRank divisor table (first GR_PAGERANK_DELTA run)
+  bool ds_tried = false;
+  double ds_long_frac = -1.0;  // share of in-edges in rows longer than one tile (< 0: not computed)                  // tolerance PageRank divisor table (first GR_PAGERANK_DELTA run)
   uint32_t *hub_in = nullptr, *hub_out = nullptr, *static_hubs = nullptr;
   uint32_t n_static_hubs = 0;
   // hub chunk lists (kChunk edges per CTA work item)

@@ -1477,14 +1477,34 @@ __device__ __forceinline__ void dense_seg_phase(const Part<OffT> &P, const View 
       Prog::atomicGather(acc_g + row, run);
       if (ract) atomicOr(P.ds_act + (row >> 5), 1u << (row & 31));
     }
-    // apply the complete active rows (row counter replayed; warp-collective per item slot)
+    // apply the complete active rows, each lane its own: the loads of all of them
+    // first (one round trip), then the applies, then one warp-queue push per item slot
     uint32_t rr = r0 - h0 + (cnt - __popc(b));
+    uint32_t cur[kDsIpt], dg[kDsIpt], vv[kDsIpt];
 #pragma unroll
     for (int k = 0; k < kDsIpt; k++) {
       if ((b >> k) & 1u) ++rr;
+      vv[k] = P.own_lo + rr;
       const bool p = ((done_rows >> k) & 1u) && done_act[k];
-      if (__any_sync(0xffffffffu, p))
-        ds_apply_row<Prog>(P, rr, done_val[k], cx, qC, p, my_g, my_c, my_a, no_hub_c);
+      cur[k] = p ? P.val[vv[k]] : 0u;
+      dg[k] = p ? (uint32_t)((uint64_t)P.in_off[rr + 1] - (uint64_t)P.in_off[rr]) : 0u;
+    }
+    uint32_t chg = 0;
+#pragma unroll
+    for (int k = 0; k < kDsIpt; k++) {
+      if (((done_rows >> k) & 1u) && done_act[k]) {
+        my_g += dg[k];
+        my_a += 1;
+        if (Prog::apply(&cur[k], done_val[k], cx)) {
+          my_c += 1;
+          if (!no_hub_c && test_bit(P.hub_out, vv[k])) append_hub_C(P, vv[k], cur[k]);
+          else chg |= 1u << k;
+        }
+      }
+    }
+    if (__any_sync(0xffffffffu, chg != 0u)) {
+#pragma unroll
+      for (int k = 0; k < kDsIpt; k++) qC.push((chg >> k) & 1u, vv[k], cur[k], P.C_v, P.C_val, &ctl->cnt_C);
     }
   }
   qC.block_flush(P.C_v, P.C_val, &ctl->cnt_C, s_off);
