@@ -58,29 +58,49 @@ struct NcclComm : Comm {
     for (int i = 0; i < k * world; i++) out[i] = h_small[i];
     return GR_OK;
   }
+  // Every rank makes the same sequence of allgathers whatever happens locally, and
+  // the result is agreed: GR_OK on all ranks or GR_EUNSUPPORTED on all ranks (a
+  // rank without peer access must not leave the others waiting in a collective).
   gr_status share_buffer(void *local, std::vector<void *> *out, cudaStream_t s) override {
     static_assert(sizeof(cudaIpcMemHandle_t) == 64, "IPC handle is 8 words");
-    cudaIpcMemHandle_t h;
-    if (cudaIpcGetMemHandle(&h, local) != cudaSuccess) return GR_ECUDA;
-    uint64_t mine[8], all[8 * 64];
     if (world > 64) return GR_EUNSUPPORTED;
-    std::memcpy(mine, &h, 64);
-    gr_status st = allgather_small(mine, 8, all, s);
+    cudaIpcMemHandle_t h;
+    std::memset(&h, 0, sizeof h);
+    uint64_t ok = cudaIpcGetMemHandle(&h, local) == cudaSuccess ? 1 : 0;
+    if (!ok) cudaGetLastError();
+    uint64_t oks[64], mine[8], all[8 * 64];
+    gr_status st = allgather_small(&ok, 1, oks, s);
     if (st != GR_OK) return st;
+    for (int q = 0; q < world; q++)
+      if (!oks[q]) return GR_EUNSUPPORTED;
+    std::memcpy(mine, &h, 64);
+    if ((st = allgather_small(mine, 8, all, s)) != GR_OK) return st;
     out->assign(world, nullptr);
     (*out)[rank] = local;
-    for (int q = 0; q < world; q++) {
+    std::vector<void *> mine_opened;
+    ok = 1;
+    for (int q = 0; q < world && ok; q++) {
       if (q == rank) continue;
       cudaIpcMemHandle_t hq;
       std::memcpy(&hq, all + 8 * q, 64);
       void *p = nullptr;
       if (cudaIpcOpenMemHandle(&p, hq, cudaIpcMemLazyEnablePeerAccess) != cudaSuccess) {
         cudaGetLastError();
-        return GR_ECUDA;
+        ok = 0;
+        break;
       }
-      opened.push_back(p);
+      mine_opened.push_back(p);
       (*out)[q] = p;
     }
+    if ((st = allgather_small(&ok, 1, oks, s)) != GR_OK) return st;
+    bool all_ok = true;
+    for (int q = 0; q < world; q++) all_ok = all_ok && oks[q];
+    if (!all_ok) {
+      for (void *p : mine_opened) cudaIpcCloseMemHandle(p);
+      out->clear();
+      return GR_EUNSUPPORTED;
+    }
+    opened.insert(opened.end(), mine_opened.begin(), mine_opened.end());
     return GR_OK;
   }
   gr_status barrier(cudaStream_t s) override {

@@ -36,7 +36,9 @@ struct Comm {
   // buffer (out[rank] = local). NCCL: cudaIpc handles exchanged with
   // allgather_small and opened with peer access (NVLink); the mappings are
   // closed when the Comm is destroyed. Simulated: the pointers themselves.
-  // `local` must come from cudaMalloc (IPC-exportable).
+  // `local` must come from cudaMalloc (IPC-exportable). Collective: every rank
+  // gets the same answer (GR_OK everywhere, or GR_EUNSUPPORTED everywhere when
+  // some rank cannot export or map a peer buffer; the caller then falls back).
   virtual gr_status share_buffer(void *local, std::vector<void *> *out, cudaStream_t s) = 0;
   // Stream-ordered barrier: work enqueued on s after it starts only when every
   // rank's work enqueued before its barrier has completed (so peer stores of

@@ -51,6 +51,7 @@ gr_status part_setup(gr_graph *g) {
   g->pr_npeer = 0;
   if (C->world - 1 <= 15 && g->contrib[0] && g->contrib[1]) {
     std::vector<void *> p0, p1;
+    // both calls are collective and agree on every rank (comm.h)
     gr_status a = C->share_buffer(g->contrib[0], &p0, g->stream);
     gr_status b = a == GR_OK ? C->share_buffer(g->contrib[1], &p1, g->stream) : a;
     if (b == GR_OK) {
@@ -61,10 +62,10 @@ gr_status part_setup(gr_graph *g) {
         g->pr_npeer++;
       }
       g->pr_p2p = true;
-    } else if (b == GR_ENCCL) {
-      return fail(b, "PageRank replica mapping: exchange failed");
+    } else if (b == GR_EUNSUPPORTED) {
+      g->pr_npeer = 0;  // no peer mapping on some rank: every rank exchanges with NCCL
     } else {
-      g->pr_npeer = 0;  // every rank reaches the same allgather_small calls; fall back to NCCL
+      return fail(b, "PageRank replica mapping: exchange failed");
     }
   }
   return GR_OK;
