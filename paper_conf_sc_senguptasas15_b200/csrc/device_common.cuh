@@ -165,6 +165,11 @@ template <class OffT> struct Part {
   void *ds_acc;            // [own_n] GatherT slots (8 B) of the split rows, identity between uses
   uint32_t *ds_act;        // [own_n / 32 + 1] active bits of the split rows
   uint32_t ds_tiles, ds_nsplit;
+  // partitioned frontier programs, exchange fused into the gather: every rank's
+  // changed-set buffers of this superstep's parity (own included), written at
+  // xp_off (= own_lo) + list position as the gather appends (WarpQueue mirrors)
+  uint32_t *xp_v[16], *xp_val[16];
+  uint32_t n_xp, xp_off;
   uint32_t *nxt[2];       // fused push supersteps: per-vertex gather accumulators by parity (GatherT = u32)
   const uint8_t *out_w;   // activation CSR weights (fused push supersteps of weighted programs)
   uint32_t n_s_hubs, n_s_chunks;
@@ -239,6 +244,17 @@ struct WarpQueue {
   uint32_t *s_a;   // [kQueueCap] shared
   uint32_t *s_b;   // [kQueueCap] shared or nullptr (pair lists)
   uint32_t n;      // warp-uniform fill level
+  // optional mirrors (partitioned frontier exchange fused into the gather): every
+  // flushed entry at list position p is also stored at mir_off + p of each mirror
+  uint32_t *const *mir_a = nullptr;
+  uint32_t *const *mir_b = nullptr;
+  uint32_t n_mir = 0, mir_off = 0;
+  __device__ __forceinline__ void mirror(uint32_t pos, uint32_t a, uint32_t b) const {
+    for (uint32_t q = 0; q < n_mir; q++) {
+      mir_a[q][mir_off + pos] = a;
+      mir_b[q][mir_off + pos] = b;
+    }
+  }
   __device__ void flush(uint32_t *g_a, uint32_t *g_b, uint32_t *g_cnt) {
     __syncwarp();
     if (n == 0) return;
@@ -248,6 +264,7 @@ struct WarpQueue {
     for (uint32_t i = lane_id(); i < n; i += 32) {
       g_a[base + i] = s_a[i];
       if (g_b) g_b[base + i] = s_b[i];
+      if (n_mir) mirror(base + i, s_a[i], s_b[i]);
     }
     __syncwarp();
     n = 0;
@@ -268,6 +285,7 @@ struct WarpQueue {
     for (uint32_t i = threadIdx.x & 31; i < n; i += 32) {
       g_a[base + i] = s_a[i];
       if (g_b) g_b[base + i] = s_b[i];
+      if (n_mir) mirror(base + i, s_a[i], s_b[i]);
     }
     __syncwarp();
     n = 0;

@@ -123,6 +123,10 @@ struct gr_graph {
   uint32_t *X_v = nullptr, *X_val = nullptr;  // exchanged changed set
   float *rank_all = nullptr;                  // PageRank fetch assembly
   uint64_t *x_cnt = nullptr;                  // per-superstep (|C_t|, |A_t|) for the count exchange
+  // fused frontier exchange: own buffers by parity and every rank's (peer-mapped)
+  uint32_t *fx_own_v[2] = {}, *fx_own_val[2] = {};
+  uint32_t *fx_v[2][16] = {}, *fx_val[2][16] = {};
+  bool fx_ok = false;
   // PageRank fused exchange: every other rank's contribution replica (by parity),
   // peer-mapped (cudaIpc, NCCL mode) or same-device (simulated ranks)
   float *pr_peer[2][15] = {};

@@ -44,6 +44,37 @@ gr_status part_setup(gr_graph *g) {
   if ((s = dev_alloc(g, (void **)&g->X_val, 4 * n)) != GR_OK) return s;
   if ((s = dev_alloc(g, (void **)&g->rank_all, 4 * n)) != GR_OK) return s;
   if ((s = dev_alloc(g, (void **)&g->x_cnt, 64)) != GR_OK) return s;
+  // frontier exchange buffers by parity (cudaMalloc: exported to the peers), n entries
+  // each: rank q's C_t lands at [own_lo_q, own_lo_q + |C_t^q|)
+  g->fx_ok = false;
+  if (g->comm->world <= 16) {
+    bool ok = true;
+    for (int b = 0; b < 2 && ok; b++)
+      for (uint32_t **arr : {&g->fx_own_v[b], &g->fx_own_val[b]}) {
+        if (cudaMalloc((void **)arr, 4 * std::max<uint64_t>(n, 1)) != cudaSuccess) {
+          cudaGetLastError();
+          return fail(GR_ENOMEM, "frontier exchange buffers");
+        }
+        g->plain_allocs.push_back(*arr);
+        g->dev_bytes += 4 * n;
+      }
+    for (int b = 0; b < 2 && ok; b++) {
+      std::vector<void *> pv, pval;
+      gr_status a = g->comm->share_buffer(g->fx_own_v[b], &pv, g->stream);
+      gr_status c = a == GR_OK ? g->comm->share_buffer(g->fx_own_val[b], &pval, g->stream) : a;
+      if (c == GR_OK) {
+        for (int q = 0; q < g->comm->world; q++) {
+          g->fx_v[b][q] = static_cast<uint32_t *>(pv[q]);
+          g->fx_val[b][q] = static_cast<uint32_t *>(pval[q]);
+        }
+      } else if (c == GR_EUNSUPPORTED) {
+        ok = false;  // agreed by every rank: the allgatherv exchange stays
+      } else {
+        return fail(c, "frontier exchange buffer mapping failed");
+      }
+    }
+    g->fx_ok = ok;
+  }
   // PageRank fused exchange: map every peer's contribution replicas (both
   // parities). Without a mapping (no peer access) PageRank exchanges with NCCL.
   Comm *C = g->comm;
@@ -146,8 +177,25 @@ gr_status run_frontier_part(gr_graph *g, const gr_run_opts *o, cudaStream_t s, g
   // (|C_t|, |A_t|) pair is allgathered straight from device memory; it sizes
   // the exchange of C_t and decides termination (no active vertex on any rank:
   // the gather of an empty frontier changed nothing and the run ends at t).
+  // Fused exchange (default when every rank mapped every peer's exchange buffers):
+  // the gather's C_t appends also land in each rank's buffer of this parity at
+  // own_lo + position, so after the count exchange every rank already holds
+  // all of C_t — no allgatherv. Parity double buffering: a rank may start the
+  // gather of t+1 while a peer still classifies t.
+  bool fx = g->fx_ok;
+  if (const char *e = getenv("GR_FRONTIER_EXCHANGE")) fx = fx && std::string(e) != "nccl";
   while (o->max_iters == 0 || t < o->max_iters) {
+    const uint32_t par = t & 1u;
+    if (fx) {
+      for (int q = 0; q < C->world; q++) {
+        P.xp_v[q] = g->fx_v[par][q];
+        P.xp_val[q] = g->fx_val[par][q];
+      }
+      P.n_xp = (uint32_t)C->world;
+      P.xp_off = (uint32_t)g->H.own_lo;
+    }
     k_gather_apply<Prog, OffT><<<grid, kBlock, 0, s>>>(P);
+    P.n_xp = 0;
     k_part_counts<<<1, 1, 0, s>>>(g->ctl, g->x_cnt);
     launches += 2;
     XCK(C->allgather_dev(g->x_cnt, 2, all.data(), s));
@@ -160,13 +208,27 @@ gr_status run_frontier_part(gr_graph *g, const gr_run_opts *o, cudaStream_t s, g
     }
     if (active == 0) break;
     // exchange the changed set C_t (vertex, new value)
-    if (tot) {
+    XRanges R{};
+    const uint32_t *xv = g->X_v, *xval = g->X_val;
+    if (fx) {
+      uint32_t acc = 0;
+      for (int q = 0; q < C->world; q++) {
+        R.off[q] = (uint32_t)g->H.owners[q];
+        R.pre[q] = acc;
+        acc += (uint32_t)all[2 * q];
+        if (q != C->rank) C->bytes_in += 8 * all[2 * q];
+      }
+      R.pre[C->world] = acc;
+      R.nr = (uint32_t)C->world;
+      xv = g->fx_v[par][C->rank];
+      xval = g->fx_val[par][C->rank];
+    } else if (tot) {
       XCK(C->allgatherv(g->C_v, g->X_v, cnt, dsp, s));
       XCK(C->allgatherv(g->C_val, g->X_val, cnt, dsp, s));
     }
     PCK(cudaMemsetAsync(&g->ctl->cnt_C, 0, sizeof(uint32_t), s));
     if (tot) k_classify<OffT><<<std::min<uint32_t>(grid, (uint32_t)((tot + kBlock - 1) / kBlock)), kBlock, 0, s>>>(
-        P, g->X_v, g->X_val, (uint32_t)tot);
+        P, xv, xval, (uint32_t)tot, R);
     if constexpr (kScatter) {
       // commit every rank's C_t first: scatter reads the committed values of its targets
       k_commit_only<OffT><<<grid, kBlock, 0, s>>>(P);

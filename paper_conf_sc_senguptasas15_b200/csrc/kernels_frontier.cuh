@@ -674,6 +674,12 @@ __device__ __forceinline__ void gather_phase(const Part<OffT> &P, const View &V)
   __shared__ unsigned long long s8[kWarpsPerBlock];
   const uint32_t warp = threadIdx.x / 32, lane = lane_id();
   WarpQueue qC{sq[warp][0], sq[warp][1], 0};
+  if (P.n_xp) {  // partitioned, fused exchange: C_t also lands in every rank's exchange buffer
+    qC.mir_a = P.xp_v;
+    qC.mir_b = P.xp_val;
+    qC.n_mir = P.n_xp;
+    qC.mir_off = P.xp_off;
+  }
   unsigned long long my_g = 0, my_c = 0, my_a = 0;
 
   // Phase 1: non-hub active vertices, 32 per warp, static grid stride
@@ -760,6 +766,7 @@ __device__ __forceinline__ void gather_phase(const Part<OffT> &P, const View &V)
             const uint32_t pos = atomicAdd(&ctl->cnt_C, 1u);
             P.C_v[pos] = v;
             P.C_val[pos] = nv;
+            if (P.n_xp) qC.mirror(pos, v, nv);
           }
         }
       }
@@ -1659,12 +1666,19 @@ __global__ void __launch_bounds__(kBlock, 3) k_persistent_ds(const __grid_consta
 #endif
 
 
+// Regions of the exchange buffer holding each rank's C_t (fused exchange): rank q's
+// entries at [off[q], off[q] + pre[q+1] - pre[q]); nr == 0: one contiguous list
+struct XRanges {
+  uint32_t off[16], pre[17];
+  uint32_t nr;
+};
+
 // Partitioned runs: split the exchanged changed set (every rank's C_t) into
 // the local non-hub list and the local changed-hub chunks (hub-ness depends on
 // this rank's activation CSR).
 template <class OffT>
 __global__ void __launch_bounds__(kBlock) k_classify(const __grid_constant__ Part<OffT> P, const uint32_t *X_v,
-                                                     const uint32_t *X_val, uint32_t nX) {
+                                                     const uint32_t *X_val, uint32_t nX, const XRanges R) {
   __shared__ uint32_t sq[kWarpsPerBlock][2][kQueueCap];
   __shared__ uint32_t s_off[kWarpsPerBlock + 1];
   const uint32_t warp = threadIdx.x / 32, lane = lane_id();
@@ -1673,7 +1687,13 @@ __global__ void __launch_bounds__(kBlock) k_classify(const __grid_constant__ Par
   for (uint32_t base = gw * 32u; base < nX; base += nw * 32u) {
     const uint32_t i = base + lane;
     const bool valid = i < nX;
-    const uint32_t u = valid ? X_v[i] : 0u, val = valid ? X_val[i] : 0u;
+    uint32_t at = i;  // fused exchange: entry i of the concatenation of the rank regions
+    if (valid && R.nr) {
+      uint32_t q = 0;
+      while (q + 1 < R.nr && R.pre[q + 1] <= i) q++;
+      at = R.off[q] + (i - R.pre[q]);
+    }
+    const uint32_t u = valid ? X_v[at] : 0u, val = valid ? X_val[at] : 0u;
     const bool hub = valid && test_bit(P.hub_out, u);
     if (hub) append_hub_C(P, u, val);
     qC.push(valid && !hub, u, val, P.C_v, P.C_val, &P.ctl->cnt_C);

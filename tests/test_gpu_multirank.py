@@ -48,9 +48,15 @@ def run_sim_ranks(n, src, dst, w, G, algo, source=0, max_iters=0):
 
 
 @pytest.mark.timeout(900)
+@pytest.mark.parametrize("exchange", ["fused", "nccl"])
 @pytest.mark.parametrize("G", [2, 3])
 @pytest.mark.parametrize("algo", ["bfs", "sssp", "cc", "pagerank", "pagerank_delta"])
-def test_sim_ranks_equal_oracle(G, algo):
+def test_sim_ranks_equal_oracle(G, algo, exchange, monkeypatch):
+    """fused: the changed set is stored into every rank's exchange buffer by the
+    gather's own appends (peer mappings; same-device buffers for simulated ranks);
+    nccl: the allgatherv of the changed set after the gather."""
+    if exchange == "nccl":
+        monkeypatch.setenv("GR_FRONTIER_EXCHANGE", "nccl")
     g = grgen.rmat(13, 16, seed=8)
     src, dst = g.src, g.dst
     if algo == "cc":
