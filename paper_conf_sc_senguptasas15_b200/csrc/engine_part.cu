@@ -194,7 +194,8 @@ gr_status run_frontier_part(gr_graph *g, const gr_run_opts *o, cudaStream_t s, g
       P.n_xp = (uint32_t)C->world;
       P.xp_off = (uint32_t)g->H.own_lo;
     }
-    k_gather_apply<Prog, OffT><<<grid, kBlock, 0, s>>>(P);
+    if (fx) k_gather_apply_x<Prog, OffT><<<grid, kBlock, 0, s>>>(P);
+    else k_gather_apply<Prog, OffT><<<grid, kBlock, 0, s>>>(P);
     P.n_xp = 0;
     k_part_counts<<<1, 1, 0, s>>>(g->ctl, g->x_cnt);
     launches += 2;

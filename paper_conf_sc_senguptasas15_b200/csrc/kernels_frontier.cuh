@@ -647,7 +647,7 @@ __global__ void __launch_bounds__(kBlock) k_pull(const __grid_constant__ Part<Of
 // superstep activated by pull): A_t is not materialised — every owned vertex
 // is gathered and is active iff one of its in-edge sources is marked in the
 // changed bitmap of t-1; only active vertices apply and count in the trace.
-template <class Prog, bool kDense, class OffT>
+template <class Prog, bool kDense, class OffT, bool kMirror = false>
 __device__ __forceinline__ void gather_phase(const Part<OffT> &P, const View &V) {
   using G = typename Prog::GatherT;
   Ctl *ctl = P.ctl;
@@ -674,7 +674,7 @@ __device__ __forceinline__ void gather_phase(const Part<OffT> &P, const View &V)
   __shared__ unsigned long long s8[kWarpsPerBlock];
   const uint32_t warp = threadIdx.x / 32, lane = lane_id();
   WarpQueue qC{sq[warp][0], sq[warp][1], 0};
-  if (P.n_xp) {  // partitioned, fused exchange: C_t also lands in every rank's exchange buffer
+  if constexpr (kMirror) {  // partitioned, fused exchange: C_t also lands in every rank's exchange buffer
     qC.mir_a = P.xp_v;
     qC.mir_b = P.xp_val;
     qC.n_mir = P.n_xp;
@@ -766,7 +766,7 @@ __device__ __forceinline__ void gather_phase(const Part<OffT> &P, const View &V)
             const uint32_t pos = atomicAdd(&ctl->cnt_C, 1u);
             P.C_v[pos] = v;
             P.C_val[pos] = nv;
-            if (P.n_xp) qC.mirror(pos, v, nv);
+            if constexpr (kMirror) qC.mirror(pos, v, nv);
           }
         }
       }
@@ -791,6 +791,17 @@ __global__ void __launch_bounds__(kBlock) k_gather_apply(const __grid_constant__
   if (V.dense) gather_phase<Prog, true>(P, V);
   else gather_phase<Prog, false>(P, V);
 }
+
+#ifndef GR_JIT
+// partitioned runs with the exchange fused into the gather (sparse supersteps only)
+template <class Prog, class OffT>
+__global__ void __launch_bounds__(kBlock) k_gather_apply_x(const __grid_constant__ Part<OffT> P) {
+  __shared__ View V;
+  load_view(P.ctl, V);
+  if (V.stop) return;
+  gather_phase<Prog, false, OffT, true>(P, V);
+}
+#endif
 
 // Commit C_t and FrontierActivate (the other phase of superstep t).
 template <class OffT>
