@@ -342,20 +342,30 @@ def main():
     torch.cuda.synchronize()
     clocks = ClockSampler(local_rank)
     clocks.start()
-    e0, e1 = torch.cuda.Event(enable_timing=True), torch.cuda.Event(enable_timing=True)
+    # graph payload (CSC ids [+ weights] + offsets) vs the 126 MB L2: a graph that fits is run
+    # cold — L2 flushed (256 MB written) before every timed step, outside the step's events
+    payload = 4 * g.m + (g.m if w is not None else 0) + 8 * (g.n + 1)
+    flush = payload < 2 * 126 * 2**20 and mode == "resident"
+    scratch = torch.empty(256 * 2**20, dtype=torch.uint8, device="cuda") if flush else None
+    evs = [(torch.cuda.Event(enable_timing=True), torch.cuda.Event(enable_timing=True)) for _ in range(args.steps)]
     kms, launches, stats = 0.0, 0, None
     phase_ms = [0.0, 0.0]
-    e0.record(stream)
-    for _ in range(args.steps):
+    for e0, e1 in evs:
+        if flush:
+            scratch.fill_(1)
+        e0.record(stream)
         stats = G.run(algo, stream=sp, profile=True, **kw)
+        e1.record(stream)
         kms += stats["kernel_ms"][0] if algo != "bfs" else stats["kernel_ms"][1]
         phase_ms[0] += stats["kernel_ms"][0]
         phase_ms[1] += stats["kernel_ms"][1]
         launches += stats["kernel_launches"]
-    e1.record(stream)
     torch.cuda.synchronize()
     ck = clocks.stop()
-    ms = e0.elapsed_time(e1)
+    ms = sum(e0.elapsed_time(e1) for e0, e1 in evs)
+    l2_note = (f"graph payload {payload / 2**20:.0f} MB < 2x L2: L2 flushed (256 MB write) before every timed step, "
+               "outside the step's CUDA events" if flush else
+               f"inputs larger than L2 (graph payload {payload / 2**20:.0f} MB > 2x 126 MB L2); no flush")
     if world > 1:
         t = torch.tensor([ms], device="cuda")
         torch.distributed.all_reduce(t, op=torch.distributed.ReduceOp.MAX)
@@ -461,7 +471,7 @@ def main():
             "data": "synthetic",
             "config": {"workload": workload_name(args.config, run, mode, args.scale), "n": n, "m": m, "shards": info["num_shards"],
                        "mode": mode, "parallelism": f"dst-interval partitions x{world}" if world > 1 else "1 GPU",
-                       "l2": "inputs larger than L2 (CSC payload > 126 MB L2); no flush",
+                       "l2": l2_note,
                        "iterations": stats["iterations"],
                        **({} if algo == "pagerank" else {"direction": args.direction,
                                                           "pull_supersteps": stats["pull_supersteps"]})},
