@@ -61,6 +61,7 @@ struct Ctl {
   uint32_t push;          // fused push supersteps (gr/program.cuh kPushFused): one phase per superstep
   unsigned long long prd_base, prd_dq;
   double prd_thr;
+  unsigned long long tot_A, tot_C;  // sum |A_t|, sum |C_t| over the run (bytes model; no trace read-back)
 };
 
 constexpr int kSlots = 64;

@@ -656,7 +656,8 @@ static gr_status run_frontier(gr_graph *g, const gr_run_opts *o, cudaStream_t s,
     CK(cudaMemsetAsync(g->cbits[0], 0, 4 * g->cbits_words, s));
     CK(cudaMemsetAsync(g->cbits[1], 0, 4 * g->cbits_words, s));
   }
-  CK(cudaMemcpyAsync(g->ctl, &h, sizeof h, cudaMemcpyHostToDevice, s));
+  *g->h_ctl = h;  // pinned staging: an async copy, not a pageable one (the last run synchronised)
+  CK(cudaMemcpyAsync(g->ctl, g->h_ctl, sizeof h, cudaMemcpyHostToDevice, s));
   k_init_values<Prog, OffT><<<g->num_sms * 4, 256, 0, s>>>(P, o->source);
   k_fill<typename Prog::GatherT><<<std::min<uint32_t>((g->hub_cap + 255) / 256, 1024), 256, 0, s>>>(
       reinterpret_cast<typename Prog::GatherT *>(g->hub_acc), Prog::identity_host(), g->hub_cap);
@@ -716,12 +717,7 @@ static gr_status run_frontier(gr_graph *g, const gr_run_opts *o, cudaStream_t s,
   g->trace_rows = std::min<uint64_t>(c.iter, g->trace_cap);
   // algorithmic bytes: 4 B/in-edge (+1 weight), 12 B per active vertex,
   // 4 B per activated out-edge, 8 B per changed vertex (value commit + offsets)
-  std::vector<unsigned long long> tr(4 * g->trace_rows);
-  if (g->trace_rows)
-    CK(cudaMemcpyAsync(tr.data(), g->trace, 32 * g->trace_rows, cudaMemcpyDeviceToHost, s));
-  CK(cudaStreamSynchronize(s));
-  uint64_t sumA = 0, sumC = 0;
-  for (uint64_t t = 0; t < g->trace_rows; t++) { sumA += tr[4 * t]; sumC += tr[4 * t + 1]; }
+  const uint64_t sumA = c.tot_A, sumC = c.tot_C;  // accumulated by close_superstep
   const uint64_t wb = Prog::kUsesWeights ? 5 : 4;
   st->bytes_hbm_model = wb * c.tot_gathered + 12 * sumA + 4 * c.tot_scattered + 12 * sumC;
   // fused push: no in-edge walk; per A_t vertex acc + value + offsets (16 B), per
@@ -759,7 +755,8 @@ static gr_status run_frontier_jit(gr_graph *g, const gr_run_opts *o, cudaStream_
     CK(cudaMemsetAsync(g->cbits[0], 0, 4 * g->cbits_words, s));
     CK(cudaMemsetAsync(g->cbits[1], 0, 4 * g->cbits_words, s));
   }
-  CK(cudaMemcpyAsync(g->ctl, &h, sizeof h, cudaMemcpyHostToDevice, s));
+  *g->h_ctl = h;  // pinned staging: an async copy, not a pageable one (the last run synchronised)
+  CK(cudaMemcpyAsync(g->ctl, g->h_ctl, sizeof h, cudaMemcpyHostToDevice, s));
   gr_status r;
   uint32_t src = o->source;
   {
@@ -810,12 +807,7 @@ static gr_status run_frontier_jit(gr_graph *g, const gr_run_opts *o, cudaStream_
   st->kernel_launches += launches;
   g->epoch_next = h.epoch_base + c.iter + 2;
   g->trace_rows = std::min<uint64_t>(c.iter, g->trace_cap);
-  std::vector<unsigned long long> tr(4 * g->trace_rows);
-  if (g->trace_rows)
-    CK(cudaMemcpyAsync(tr.data(), g->trace, 32 * g->trace_rows, cudaMemcpyDeviceToHost, s));
-  CK(cudaStreamSynchronize(s));
-  uint64_t sumA = 0, sumC = 0;
-  for (uint64_t t = 0; t < g->trace_rows; t++) { sumA += tr[4 * t]; sumC += tr[4 * t + 1]; }
+  const uint64_t sumA = c.tot_A, sumC = c.tot_C;  // accumulated by close_superstep
   const uint64_t wb = jp->uses_weights ? 5 : 4;
   st->bytes_hbm_model = wb * c.tot_gathered + 12 * sumA + 4 * c.tot_scattered + 12 * sumC;
   return GR_OK;

@@ -422,6 +422,8 @@ __device__ void close_superstep(const Part<OffT> &P, unsigned long long cond_han
     }
   }
   const unsigned long long scat = c->scattered;
+  c->tot_A = c->tot_A + c->cnt_act[slot];
+  c->tot_C = c->tot_C + c->changed;
   c->tot_gathered = c->tot_gathered + c->gathered;
   c->tot_scattered = c->tot_scattered + c->scattered;
   c->changed = 0;

@@ -53,6 +53,12 @@ def compare(n, src, dst, w, algo, source=0, max_iters=0, loops=("auto", "device"
                 np.testing.assert_array_equal(tr, rtr, err_msg=f"{loop} {d}")
                 assert st["edges_gathered"] == int(rtr[:, 2].sum())
                 assert st["edges_scattered"] == int(rtr[:, 3].sum())
+                if resident1:  # bytes model from the device's running sums of |A_t|, |C_t|
+                    wb = 5 if algo == "sssp" else 4
+                    sa, sc = int(rtr[:, 0].sum()), int(rtr[:, 1].sum())
+                    sg, ss = int(rtr[:, 2].sum()), int(rtr[:, 3].sum())
+                    assert st["bytes_hbm_model"] in (wb * sg + 12 * sa + 4 * ss + 12 * sc,
+                                                     16 * sa + wb * ss + 12 * sc), (loop, d)
                 if d == "push" or not resident1:
                     assert st["pull_supersteps"] == 0
                 elif d == "pull" and rtr[:, 1].sum() > 0:
