@@ -653,16 +653,12 @@ static gr_status run_frontier(gr_graph *g, const gr_run_opts *o, cudaStream_t s,
     uint32_t div = o->pull_div ? o->pull_div : kPullDivDefault;
     if (const char *e = getenv("GR_PULL_DIV")) div = (uint32_t)strtoul(e, nullptr, 10);
     h.pull_div = o->direction == GR_DIR_PULL ? 0xFFFFFFFFu : div;
-    CK(cudaMemsetAsync(g->cbits[0], 0, 4 * g->cbits_words, s));
-    CK(cudaMemsetAsync(g->cbits[1], 0, 4 * g->cbits_words, s));
   }
   *g->h_ctl = h;  // pinned staging: an async copy, not a pageable one (the last run synchronised)
   CK(cudaMemcpyAsync(g->ctl, g->h_ctl, sizeof h, cudaMemcpyHostToDevice, s));
-  k_init_values<Prog, OffT><<<g->num_sms * 4, 256, 0, s>>>(P, o->source);
-  k_fill<typename Prog::GatherT><<<std::min<uint32_t>((g->hub_cap + 255) / 256, 1024), 256, 0, s>>>(
-      reinterpret_cast<typename Prog::GatherT *>(g->hub_acc), Prog::identity_host(), g->hub_cap);
-  CK(cudaMemsetAsync(g->hub_done, 0, 4ull * g->hub_cap, s));
-  launches += 2;
+  // values, hub accumulators / done counters and (pull) both changed bitmaps in one launch
+  k_init_run<Prog, OffT><<<g->num_sms * 4, 256, 0, s>>>(P, o->source, g->hub_cap, g->cbits_words, may_pull ? 1 : 0);
+  launches += 1;
   if (Prog::kInit == kInitAll && g->n_static_hubs) {
     CK(cudaMemcpyAsync(g->listH[0], g->static_hubs, 4ull * g->n_static_hubs, cudaMemcpyDeviceToDevice, s));
     CK(cudaMemcpyAsync(g->chkA_h[0], g->static_chk_h, 4ull * g->n_static_chunks, cudaMemcpyDeviceToDevice, s));

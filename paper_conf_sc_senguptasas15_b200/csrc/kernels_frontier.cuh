@@ -1725,6 +1725,31 @@ __global__ void k_init_values(const __grid_constant__ Part<OffT> P, uint32_t sou
     P.val[v] = Prog::initValue((uint32_t)v, cx);
 }
 
+// All per-run resets of a resident frontier run in one launch (small graphs are
+// bound by the launches before the persistent loop): initial values, the hub
+// accumulators (identity) and done counters, and (pull) both changed bitmaps.
+template <class Prog, class OffT>
+__global__ void k_init_run(const __grid_constant__ Part<OffT> P, uint32_t source, uint64_t hub_cap,
+                           uint64_t cbits_words, int zero_cbits) {
+  using G = typename Prog::GatherT;
+  Ctx cx{};
+  cx.n = P.n;
+  cx.source = source;
+  cx.prd_r0 = P.ctl->prd_r0;
+  const uint64_t i0 = blockIdx.x * (uint64_t)blockDim.x + threadIdx.x, st = (uint64_t)gridDim.x * blockDim.x;
+  for (uint64_t v = i0; v < P.n; v += st) P.val[v] = Prog::initValue((uint32_t)v, cx);
+  G *ha = reinterpret_cast<G *>(P.hub_acc);
+  for (uint64_t i = i0; i < hub_cap; i += st) {
+    ha[i] = Prog::identity();
+    P.hub_done[i] = 0u;
+  }
+  if (zero_cbits)
+    for (uint64_t i = i0; i < cbits_words; i += st) {
+      P.cbits[0][i] = 0u;
+      P.cbits[1][i] = 0u;
+    }
+}
+
 template <class T> __global__ void k_fill(T *p, T value, uint64_t count) {
   for (uint64_t i = blockIdx.x * (uint64_t)blockDim.x + threadIdx.x; i < count; i += (uint64_t)gridDim.x * blockDim.x)
     p[i] = value;
