@@ -785,7 +785,7 @@ static gr_status run_frontier_jit(gr_graph *g, const gr_run_opts *o, cudaStream_
   launches++;
   int bps = 0;
   if ((r = jit_occupancy(jp->persistent[k], kBlock, &bps)) != GR_OK) return r;
-  int per_sm = std::min(bps, 4);
+  int per_sm = std::min(bps, g->H.own_n() < (uint64_t)g->num_sms * 4 * kBlock ? 2 : 4);  // as run_frontier
   const uint32_t grid = (uint32_t)g->num_sms * (uint32_t)std::max(1, per_sm);
   {
     void *args[] = {(void *)&P};
