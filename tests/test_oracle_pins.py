@@ -564,3 +564,66 @@ def test_sssp_messages_path_and_lattice():
     vals, tr, it = oracle.run(k + 1, src, dst, "sssp_msg", w=w, source=0)
     np.testing.assert_array_equal(vals, np.concatenate([[0], np.cumsum(w)]).astype(np.uint32))
     assert it == k and np.all(tr[:, 1] == 1) and tr[-1, 3] == 0  # A_0 = {1}, ..., A_{k-1} = {k}
+
+
+# ------------------- tolerance-driven PageRank: exact brute force of the rule
+# DESIGN.md §2 / reading R17-R18 (Figs. 16-17): the
+# specification restated with Python's unbounded integers and Fractions (no
+# 64/128-bit arithmetic, no ldexp), as a set-based BSP superstep. The oracle's
+# values AND its whole frontier trace — so prd_apply's change rule
+# |R_new - R_old| > tolerance/n — must equal it exactly.
+def _prd_brute(n, src, dst, tau, max_iters, d=0.85):
+    from fractions import Fraction
+    import math
+
+    ins = collections.defaultdict(list)
+    outs = collections.defaultdict(list)
+    for a, b in zip(src.tolist(), dst.tolist()):
+        ins[b].append(a)
+        outs[a].append(b)
+    f32 = lambda x: float(np.float32(x))  # round to nearest fp32
+    q = math.floor(f32(d) * 2**20 + 0.5)  # round(d * 2^20) of the fp32 damping
+    base = ((2**20 - q) * 2**42) // n  # fixed-point (1 - d)/n
+    thr = f32(tau) / n
+
+    def fix(r):  # floor(R * 2^62), exact
+        return math.floor(Fraction(r) * 2**62)
+
+    def to_f32(rfix):  # fp32(double(R_fix) * 2^-62): nearest double, then nearest fp32
+        return f32(float(rfix) * 2.0**-62)
+
+    val = {v: to_f32(2**62 // n) for v in range(n)}
+    A, rows, t = set(range(n)), [], 0
+    while A and t < max_iters:
+        new, gathered = {}, 0
+        for v in A:
+            S = sum(fix(val[u]) // len(outs[u]) for u in ins[v])
+            gathered += len(ins[v])
+            new[v] = to_f32(base + (S * q) // 2**20)
+        C = {v for v in A if abs(new[v] - val[v]) > thr}
+        for v in C:
+            val[v] = new[v]
+        rows.append((len(A), len(C), gathered, sum(len(outs[u]) for u in C)))
+        A = {x for u in C for x in outs[u]}
+        t += 1
+    return np.array([val[v] for v in range(n)], np.float32), np.array(rows, np.uint64).reshape(-1, 4), t
+
+
+@pytest.mark.parametrize("tau", [0.0, 1e-6, 1e-3])
+@pytest.mark.parametrize("seed", range(8))
+def test_prdelta_values_and_trace_vs_exact_bruteforce(seed, tau):
+    rng = np.random.default_rng(900 + seed)
+    n = int(rng.integers(2, 48))
+    src, dst, _ = rand_graph(rng, n, int(rng.integers(0, 4 * n)))
+    if seed % 2:  # a hub with many in- and out-edges: large sums, many distinct n_u
+        hub = rng.integers(0, n, 3 * n).astype(np.uint32)
+        src = np.concatenate([src, hub, np.zeros(n, np.uint32)])
+        dst = np.concatenate([dst, np.zeros(3 * n, np.uint32), np.arange(n, dtype=np.uint32)])
+    mi = 60
+    vals, tr, it = oracle.run(n, src, dst, "pagerank_delta", max_iters=mi, tolerance=tau)
+    bv, btr, bit = _prd_brute(n, src, dst, tau, mi)
+    assert it == bit
+    np.testing.assert_array_equal(tr, btr)
+    np.testing.assert_array_equal(vals.view(np.uint32), bv.view(np.uint32))
+    if tau == 1e-3:  # the rule really skips: some superstep leaves an active vertex unchanged
+        assert it < mi and np.any(tr[:, 1] < tr[:, 0]) or len(src) == 0
