@@ -108,6 +108,20 @@ def grid_road(W: int, H: int, p: float = 0.58, wmax: int = 64, seed: int = 3) ->
     return Graph(n=W * H, src=src, dst=dst, w=w, name=f"grid{W}x{H}_s{seed}")
 
 
+def heat_grid(W: int, H: int, p: float = 0.58, wmax: int = 60, seed: int = 6) -> Graph:
+    """Heat-simulation input (§2.1): the road-like lattice with symmetric
+    conductances w in [1, wmax] plus one self-loop per vertex whose weight makes every
+    vertex's out-weights satisfy sum (w + 1) = 256 (the heat a vertex keeps). Needs
+    4 * (wmax + 1) <= 255."""
+    assert 4 * (wmax + 1) <= 255
+    g = grid_road(W, H, p=p, wmax=wmax, seed=seed)
+    out = np.bincount(g.src, weights=g.w.astype(np.float64) + 1.0, minlength=g.n).astype(np.int64)
+    self_w = (255 - out).astype(np.uint32)
+    v = np.arange(g.n, dtype=np.uint32)
+    return Graph(n=g.n, src=np.concatenate([g.src, v]), dst=np.concatenate([g.dst, v]),
+                 w=np.concatenate([g.w, self_w]), name=f"heat{W}x{H}_s{seed}")
+
+
 WEB_DEFAULTS = dict(xmin=2.8, zexp=2.5, dmax=1 << 20, p_local=0.75, geo_p=1.0 / 64,
                     local_cap=4096, rank_exp=0.8)
 

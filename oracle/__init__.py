@@ -22,7 +22,8 @@ _SO = os.path.join(_HERE, "liboracle.so")
 _SRC = os.path.join(_HERE, "oracle.c")
 _lib = None
 
-ALGOS = {"bfs": 0, "sssp": 1, "pagerank": 2, "cc": 3, "widest": 4, "pagerank_delta": 5, "sssp_msg": 6}
+ALGOS = {"bfs": 0, "sssp": 1, "pagerank": 2, "cc": 3, "widest": 4, "pagerank_delta": 5, "sssp_msg": 6, "heat": 7}
+HEAT_H0 = 0x40000000
 INF = 0xFFFFFFFF
 
 

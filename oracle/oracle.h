@@ -10,7 +10,8 @@
 extern "C" {
 #endif
 
-enum { OR_BFS = 0, OR_SSSP = 1, OR_PAGERANK = 2, OR_CC = 3, OR_WIDEST = 4, OR_PRDELTA = 5, OR_SSSPMSG = 6 };
+enum { OR_BFS = 0, OR_SSSP = 1, OR_PAGERANK = 2, OR_CC = 3, OR_WIDEST = 4, OR_PRDELTA = 5, OR_SSSPMSG = 6, OR_HEAT = 7 };
+#define OR_HEAT_H0 0x40000000u /* OR_HEAT: heat at the source at initialisation */
 #define OR_INF 0xFFFFFFFFu
 
 typedef struct or_graph or_graph;
@@ -39,6 +40,15 @@ void or_graph_free(or_graph *g);
  * changed at t gets S = new[u] + w if that is < val[x] (the committed value),
  * else INF; the gather takes the min of the messages on the in-edges. The
  * source is set to 0 and scatters at initialisation.
+ * OR_HEAT: heat diffusion with mutable edge state (§2.1 "Heat
+ * Simulation"; Scatter L66): temperatures are uint32 heat units, the source
+ * starts at OR_HEAT_H0 and everything else at 0; every edge holds the heat
+ * its source sends along it, initially 0. The source counts as changed at
+ * initialisation and scatters. Superstep t: T_new[x] = sum of the states of
+ * x's in-edges (changed iff it differs); after the commit every edge
+ * (u -> x) with u changed gets floor(T[u] * (w + 1) / 256). With
+ * sum_x (w(u->x) + 1) = 256 for every u (a self-loop carries the heat u
+ * keeps) this is the explicit heat step T' = W^T T in fixed point.
  * trace_out (nullable): rows of 4 uint64 per superstep t:
  *   |A_t|, |C_t|, sum_{v in A_t} indeg(v) (0 when gather is eliminated),
  *   sum_{u in C_t} outdeg(u) (0 when FrontierActivate is eliminated).

@@ -627,3 +627,71 @@ def test_prdelta_values_and_trace_vs_exact_bruteforce(seed, tau):
     np.testing.assert_array_equal(vals.view(np.uint32), bv.view(np.uint32))
     if tau == 1e-3:  # the rule really skips: some superstep leaves an active vertex unchanged
         assert it < mi and np.any(tr[:, 1] < tr[:, 0]) or len(src) == 0
+
+
+# --------------------------- heat diffusion with mutable edge state (OR_HEAT)
+# PAPER.md §2.1 L68 ("Heat Simulation"), Scatter L66. Pinned to (a) the plain
+# definition — the full fixed-point heat step T_{k+1}[x] = sum_{(u->x)}
+# floor(T_k[u] (w+1) / 256) applied to EVERY vertex, no frontier, no edge
+# state — so the frontier + scatter + edge-state machinery must reproduce it
+# exactly; (b) the fp64 matrix power (W^T)^k T_0 within the floor-loss bound
+# k*m in L1 (W^T has unit column sums, so it does not expand L1 errors);
+# (c) heat conservation up to that loss.
+def _heat_full(n, src, dst, w, s, iters):
+    T = [0] * n
+    T[s] = oracle.HEAT_H0
+    seq = [list(T)]
+    for _ in range(iters):
+        N = [0] * n
+        for a, b, c in zip(src.tolist(), dst.tolist(), w.tolist()):
+            N[b] += T[a] * (c + 1) // 256
+        T = N
+        seq.append(list(T))
+    return seq
+
+
+def _heat_graph(rng, W, H):
+    import grgen
+
+    g = grgen.heat_grid(W, H, seed=int(rng.integers(1, 1000)))
+    return g.n, g.src, g.dst, g.w
+
+
+@pytest.mark.parametrize("seed", range(6))
+def test_heat_vs_full_iteration_and_matrix_power(seed):
+    rng = np.random.default_rng(1000 + seed)
+    W, H = int(rng.integers(2, 9)), int(rng.integers(2, 9))
+    n, src, dst, w = _heat_graph(rng, W, H)
+    s = int(rng.integers(0, n))
+    mi = int(rng.integers(1, 40))
+    vals, tr, it = oracle.run(n, src, dst, "heat", w=w, source=s, max_iters=mi)
+    seq = _heat_full(n, src, dst, w, s, it + 1)
+    np.testing.assert_array_equal(vals, np.array(seq[it], np.uint32))
+    if it < mi:  # the frontier emptied: a fixed point of the full step
+        assert seq[it + 1] == seq[it]
+    # (b) fp64 matrix power, (c) conservation
+    Wm = np.zeros((n, n))
+    np.add.at(Wm, (src, dst), (w.astype(np.float64) + 1) / 256)
+    np.testing.assert_allclose(Wm.sum(1), 1.0)  # every vertex keeps or sends all its heat
+    T0 = np.zeros(n)
+    T0[s] = oracle.HEAT_H0
+    exact = np.linalg.matrix_power(Wm.T, it) @ T0
+    err = np.abs(vals.astype(np.float64) - exact).sum()
+    assert err <= it * len(src) + 1e-3, (err, it * len(src))  # + fp64 rounding of the power
+    assert oracle.HEAT_H0 - it * len(src) <= int(vals.astype(np.int64).sum()) <= oracle.HEAT_H0
+    assert tr[0, 0] == len(set(dst[src == s].tolist()))  # A_0 = out-neighbours of the source
+
+
+def test_heat_two_vertices_closed_form():
+    # 0 <-> 1 with conductance w: each keeps (255 - (w+1) + 1)/256 and sends (w+1)/256
+    w1 = 63  # (w+1)/256 = 1/4
+    src = np.array([0, 1, 0, 1], np.uint32)
+    dst = np.array([1, 0, 0, 1], np.uint32)
+    w = np.array([w1, w1, 255 - (w1 + 1), 255 - (w1 + 1)], np.uint32)
+    vals, tr, it = oracle.run(2, src, dst, "heat", w=w, source=0, max_iters=1)
+    H0 = oracle.HEAT_H0
+    np.testing.assert_array_equal(vals, [H0 * 3 // 4, H0 // 4])
+    # T_k = H0/2 (1 +- (1/2)^k) exactly while the shares divide evenly
+    vals, tr, it = oracle.run(2, src, dst, "heat", w=w, source=0, max_iters=10)
+    np.testing.assert_array_equal(vals, [H0 // 2 + (H0 >> 11), H0 // 2 - (H0 >> 11)])
+    assert it == 10 and np.all(tr[:, 1] == 2)
