@@ -13,6 +13,7 @@ from __future__ import annotations
 import argparse
 import json
 import os
+import platform
 import subprocess
 import sys
 import threading
@@ -198,35 +199,56 @@ def metric_edges(cfg_run, stats, m):
     return stats["edges_scattered"] + stats["edges_gathered"]  # BFS/SSSP: edges traversed
 
 
+def cpu_model():
+    try:
+        for line in open("/proc/cpuinfo"):
+            if line.startswith("model name"):
+                return line.split(":", 1)[1].strip()
+    except OSError:
+        pass
+    return platform.processor() or "unknown"
+
+
 def cpu_oracle_sample(g, w, run, budget_s=20.0):
-    """Time the oracle as it stands on a bounded sample of the workload."""
+    """Time the oracle as it stands on a bounded sample of the workload, pinned to one
+    core (the calling thread's affinity = {first allowed core}, as `taskset -c`)."""
     import oracle
 
     og = oracle.OracleGraph(g.n, g.src, g.dst, w)
+    old_aff = os.sched_getaffinity(0)
+    core = min(old_aff)
+    os.sched_setaffinity(0, {core})
     try:
-        if run["algo"] == "pagerank":
-            iters = 2
-            t = time.perf_counter()
-            og.run("pagerank", max_iters=iters)
-            dt = time.perf_counter() - t
-            return dict(value=iters * g.m / dt / 1e9, unit="GTEPS", cores=1, kind="oracle",
-                        sample=f"PageRank {iters} of 30 supersteps on the full graph (m={g.m}); "
-                               f"oracle CSC build not timed; {dt:.2f} s")
-        reps, t = 0, time.perf_counter()
-        while True:  # small runs (cfg1: ms) are repeated until the sample spans >= 1 s
-            if run["algo"] == "pagerank_delta":  # bounded sample: the first 3 supersteps
-                vals, tr, it = og.run("pagerank_delta", max_iters=3, tolerance=run["tolerance"])
-            else:
-                vals, tr, it = og.run(run["algo"], source=run.get("source", 0))
-            reps += 1
-            dt = time.perf_counter() - t
-            if dt >= 1.0:
-                break
-        edges = int(tr[:, 2].sum() + tr[:, 3].sum()) if run["algo"] != "cc" else g.m
-        return dict(value=reps * edges / dt / 1e9, unit="GTEPS", cores=1, kind="oracle",
-                    sample=f"{reps} x full {run['algo']} run ({it} supersteps); {dt:.2f} s")
+        res = _cpu_oracle_sample(og, g, run)
+        res.update(pinned_core=core, cpu_model=cpu_model(), host_cores=os.cpu_count())
+        return res
     finally:
+        os.sched_setaffinity(0, old_aff)
         og.close()
+
+
+def _cpu_oracle_sample(og, g, run):
+    if run["algo"] == "pagerank":
+        iters = 2
+        t = time.perf_counter()
+        og.run("pagerank", max_iters=iters)
+        dt = time.perf_counter() - t
+        return dict(value=iters * g.m / dt / 1e9, unit="GTEPS", cores=1, kind="oracle",
+                    sample=f"PageRank {iters} of 30 supersteps on the full graph (m={g.m}); "
+                           f"oracle CSC build not timed; {dt:.2f} s")
+    reps, t = 0, time.perf_counter()
+    while True:  # small runs (cfg1: ms) are repeated until the sample spans >= 1 s
+        if run["algo"] == "pagerank_delta":  # bounded sample: the first 3 supersteps
+            vals, tr, it = og.run("pagerank_delta", max_iters=3, tolerance=run["tolerance"])
+        else:
+            vals, tr, it = og.run(run["algo"], source=run.get("source", 0))
+        reps += 1
+        dt = time.perf_counter() - t
+        if dt >= 1.0:
+            break
+    edges = int(tr[:, 2].sum() + tr[:, 3].sum()) if run["algo"] != "cc" else g.m
+    return dict(value=reps * edges / dt / 1e9, unit="GTEPS", cores=1, kind="oracle",
+                sample=f"{reps} x full {run['algo']} run ({it} supersteps); {dt:.2f} s")
 
 
 def measure_h2d():
@@ -327,14 +349,19 @@ def main():
               loop=args.loop, direction=args.direction)
     if algo == "pagerank_delta":
         kw["tolerance"] = run["tolerance"]
-    part = {}
-    if world > 1:
-        # NCCL bootstrap: rank 0 creates the unique id, the torch process group broadcasts it
+    def bootstrap():
+        # NCCL bootstrap: rank 0 creates a unique id, the torch process group broadcasts it. An id
+        # bootstraps ONE communicator (its root listener is gone after the first init), so every
+        # gr_graph_load of a multi-rank graph takes a fresh one.
+        if world <= 1:
+            return {}
         uid = torch.zeros(128, dtype=torch.uint8, device="cuda")
         if rank == 0:
             uid.copy_(torch.frombuffer(bytearray(gr.gr_get_unique_id()), dtype=torch.uint8))
         torch.distributed.broadcast(uid, 0)
-        part = dict(world=world, rank=rank, nccl_unique_id=bytes(uid.cpu().numpy().tobytes()))
+        return dict(world=world, rank=rank, nccl_unique_id=bytes(uid.cpu().numpy().tobytes()))
+
+    part = bootstrap()
     mode = ("streamed" if args.config == 5 else "resident") if args.mode == "auto" else args.mode
     G = gr.GraphReduce(g.n, g.src, g.dst, w, device=local_rank, mode=mode, **part)
     info = G.info()
@@ -444,6 +471,7 @@ def main():
     for i in range(args.e2e_steps + (1 if args.e2e_steps > 0 else 0)):
         # step 0 is an untimed warm-up of the e2e path (the device pool grows to hold a
         # second graph next to the benchmark's; later loads reuse it, as a user's do)
+        part = bootstrap()  # a fresh NCCL id per multi-rank load (untimed)
         t0 = time.perf_counter()
         H = gr.gr_graph_load(n, src_p, dst_p, w_p, device=local_rank, mode=mode, **part)
         gr.gr_run(H, algo, **kw)

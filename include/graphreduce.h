@@ -57,7 +57,8 @@ typedef enum gr_algo {
   GR_CC = 3,       /* Fig. 6: min-label propagation; input must be symmetric (L290) */
   GR_CUSTOM = 4,   /* program compiled into the library: GR_CUSTOM_PROGRAMS in gr/program.cuh
                       (0: widest path; 1: SSSP by edge messages — mutable edge state written by
-                      the Scatter phase, every mode) */
+                      the Scatter phase, every mode; 2: heat diffusion, §2.1 L68 — the
+                      heat flow stored on the edges, fixed-point explicit step, every mode) */
   GR_PAGERANK_DELTA = 5 /* tolerance-driven PageRank (Figs. 16-17): a vertex
                            stays active while |dR| > tolerance/n; exact fixed-point gather, so the
                            frontier is reproducible (gr/program.cuh ProgPRDelta); fp32 rank values */

@@ -154,6 +154,7 @@ template <class OffT> struct Part {
   uint32_t *hub_act;      // per static hub: some chunk saw a marked source (dense gathers)
   const uint32_t *s_hubs, *s_chk_h, *s_chk_c;  // static in-hub list and its chunks (dense gathers)
   const ulonglong2 *prd_div;  // ProgPRDelta divisor table (Ctx::prd_div), or nullptr
+  uint32_t gate;          // dense supersteps of Selective<> programs read only the changed sources' values
   uint32_t *estate;       // [m_in] edge states in CSC order (programs with kHasScatter)
   const uint32_t *out_eid;// [m_in] CSC position of every activation-CSR edge (kHasScatter)
   // dense (pull) supersteps of kDstFreeGather programs: edge-segmented tiles over the

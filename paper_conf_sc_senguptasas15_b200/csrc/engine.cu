@@ -563,6 +563,17 @@ static gr_status get_while_graph(gr_graph *g, int key, cudaGraphExec_t *out, uin
   return GR_OK;
 }
 
+// CTAs per SM of the persistent frontier loop (built-in and run-time programs
+// alike): 4; 2 when the owned range has fewer vertices than 4 CTAs per SM have
+// threads (cheaper grid barriers: cfg1 BFS 0.392 -> 0.372 ms; SSSP / CC there
+// unchanged; cfg3 / cfg4 need 4: 858 vs 783 ms, 20.0 vs 12.3 ms at 2);
+// GR_PERSIST_CTAS_PER_SM overrides; never more than the occupancy bps allows.
+static uint32_t persistent_grid(const gr_graph *g, int bps) {
+  int per_sm = std::min(bps, g->H.own_n() < (uint64_t)g->num_sms * 4 * kBlock ? 2 : 4);
+  if (const char *e = getenv("GR_PERSIST_CTAS_PER_SM")) per_sm = std::min(bps, atoi(e));
+  return (uint32_t)g->num_sms * (uint32_t)std::max(1, per_sm);
+}
+
 template <class Prog, class OffT>
 static gr_status run_frontier(gr_graph *g, const gr_run_opts *o, cudaStream_t s, gr_run_stats *st, int key) {
   Part<OffT> P = make_part<OffT>(g);
@@ -673,12 +684,7 @@ static gr_status run_frontier(gr_graph *g, const gr_run_opts *o, cudaStream_t s,
     int bps = 0;
     const void *kf = dseg ? (const void *)k_persistent_ds<Prog, OffT> : (const void *)k_persistent<Prog, OffT>;
     CK(cudaOccupancyMaxActiveBlocksPerMultiprocessor(&bps, kf, kBlock, 0));
-    // 4 CTAs per SM; 2 when the owned range has fewer vertices than 4 CTAs per SM have
-    // threads (cheaper grid barriers: cfg1 BFS 0.392 -> 0.372 ms; SSSP / CC there
-    // unchanged; cfg3 / cfg4 need 4: 858 vs 783 ms, 20.0 vs 12.3 ms at 2)
-    int per_sm = std::min(bps, g->H.own_n() < (uint64_t)g->num_sms * 4 * kBlock ? 2 : 4);
-    if (const char *e = getenv("GR_PERSIST_CTAS_PER_SM")) per_sm = std::min(bps, atoi(e));
-    const uint32_t grid = (uint32_t)g->num_sms * (uint32_t)std::max(1, per_sm);
+    const uint32_t grid = persistent_grid(g, bps);
     void *args[] = {(void *)&P};
     CK(cudaLaunchCooperativeKernel(kf, dim3(grid), dim3(kBlock), args, 0, s));
     CK(cudaMemcpyAsync(g->h_ctl, g->ctl, sizeof(Ctl), cudaMemcpyDeviceToHost, s));
@@ -747,7 +753,18 @@ static gr_status run_frontier_jit(gr_graph *g, const gr_run_opts *o, cudaStream_
   h.prof = o->profile ? 1 : 0;
   h.kstart[0] = h.kstart[1] = ~0ull;
   prd_setup(h, o, g->H.n);
-  if (g->cbits[0] && o->direction != GR_DIR_PUSH) {
+  if (jp->scatter) {  // mutable edge state: layout once per graph, states reset per run
+    gr_status ss = scatter_setup(g, jp->uses_weights);
+    if (ss != GR_OK) return ss;
+    P = make_part<OffT>(g);
+    uint64_t m_in = g->H.m_in;
+    void *args[] = {(void *)&P, (void *)&m_in};
+    gr_status r0 = jit_launch(jp->init_edges[k], g->num_sms * 8, 256, args, 0, s, false);
+    if (r0 != GR_OK) return r0;
+    launches++;
+  }
+  // scatter programs always push (the scatter walks the out-edges of C_t)
+  if (g->cbits[0] && o->direction != GR_DIR_PUSH && !jp->scatter) {
     uint32_t div = o->pull_div ? o->pull_div : kPullDivDefault;
     if (const char *e = getenv("GR_PULL_DIV")) div = (uint32_t)strtoul(e, nullptr, 10);
     h.pull_div = o->direction == GR_DIR_PULL ? 0xFFFFFFFFu : div;
@@ -785,8 +802,7 @@ static gr_status run_frontier_jit(gr_graph *g, const gr_run_opts *o, cudaStream_
   launches++;
   int bps = 0;
   if ((r = jit_occupancy(jp->persistent[k], kBlock, &bps)) != GR_OK) return r;
-  int per_sm = std::min(bps, g->H.own_n() < (uint64_t)g->num_sms * 4 * kBlock ? 2 : 4);  // as run_frontier
-  const uint32_t grid = (uint32_t)g->num_sms * (uint32_t)std::max(1, per_sm);
+  const uint32_t grid = persistent_grid(g, bps);
   {
     void *args[] = {(void *)&P};
     if ((r = jit_launch(jp->persistent[k], grid, kBlock, args, 0, s, true)) != GR_OK) return r;
@@ -1295,6 +1311,12 @@ static gr_status run_pagerank(gr_graph *g, const gr_run_opts *o, cudaStream_t s,
     L.num_tiles = g->seg_tiles;
     L.iters = iters;
     L.bar = g->pr_bar;
+    // GR_PR_PHASES=1: per-superstep split of the loop (tiles vs fix-ups + pack + barriers),
+    // stamped with %globaltimer by CTA 0 after each grid barrier, printed on stderr
+    static const bool phases = getenv("GR_PR_PHASES") && atoi(getenv("GR_PR_PHASES")) != 0;
+    unsigned long long *d_ts = nullptr;
+    if (phases) CK(cudaMallocAsync((void **)&d_ts, 8ull * (2 * iters + 1), s));
+    L.ts = d_ts;
     k_pr_init<<<g->num_sms * 4, 256, 0, s>>>((uint32_t)g->H.n, g->inv_outdeg, g->contrib[0]);
     k_pr_hot_pack<<<(g->hot_k + 255) / 256, 256, 0, s>>>(g->contrib[0], g->hot_ids, g->hot_buf[0], g->hot_k);
     if (prof) CK(cudaEventRecord(g->prof_ev[0], s));
@@ -1303,6 +1325,18 @@ static gr_status run_pagerank(gr_graph *g, const gr_run_opts *o, cudaStream_t s,
                                    dim3(g->hot_cta), args, g->hot_smem, s));
     if (prof) CK(cudaEventRecord(g->prof_ev[1], s));
     CK(cudaStreamSynchronize(s));
+    if (phases) {
+      std::vector<unsigned long long> ts(2 * iters + 1);
+      CK(cudaMemcpy(ts.data(), d_ts, 8 * ts.size(), cudaMemcpyDeviceToHost));
+      CK(cudaFreeAsync(d_ts, s));
+      double p1 = 0, p2 = 0;
+      for (uint32_t t = 0; t < iters; t++) {
+        p1 += (double)(ts[1 + 2 * t] - ts[2 * t]);
+        p2 += (double)(ts[2 + 2 * t] - ts[1 + 2 * t]);
+      }
+      fprintf(stderr, "[gr] k_pr_seg_loop phases per superstep: tiles %.2f us, fix-ups + pack + barriers %.2f us "
+              "(%u supersteps)\n", p1 / iters / 1e3, p2 / iters / 1e3, iters);
+    }
     if (prof) {
       float ms = 0;
       CK(cudaEventElapsedTime(&ms, g->prof_ev[0], g->prof_ev[1]));
@@ -1379,9 +1413,17 @@ gr_status run(gr_graph *g, const gr_run_opts *oin, gr_run_stats *st) {
     if (!known && (jp = jit_find(o.custom_id))) {
       known = true;
       uses_w = jp->uses_weights;
-      if (g->mode == GR_MODE_STREAMED || g->comm || !g->coop)
-        return fail(GR_EUNSUPPORTED, "run-time program %d: resident single-GPU graphs only (persistent loop)",
-                    o.custom_id);
+      if (jp->device != g->device)
+        return fail(GR_EINVAL, "run-time program %d was compiled on device %d; the graph lives on device %d "
+                    "(compile it with that device current)", o.custom_id, jp->device, g->device);
+      // resident single-GPU graphs run the program's persistent BSP loop; streamed and
+      // partitioned graphs run their drivers with the program's kernel table (prog_desc.h)
+      if (g->mode != GR_MODE_STREAMED && !g->comm) {
+        if (!g->coop) return fail(GR_EUNSUPPORTED, "run-time program %d needs cooperative launch", o.custom_id);
+        if (o.loop != GR_LOOP_AUTO && o.loop != GR_LOOP_PERSISTENT)
+          return fail(GR_EUNSUPPORTED, "run-time program %d: resident graphs run the persistent loop only "
+                      "(loop = auto or persistent)", o.custom_id);
+      }
     }
     if (!known) return fail(GR_EUNSUPPORTED, "no custom program with id %d is registered", o.custom_id);
     if (uses_w && !g->H.has_w) return fail(GR_EINVAL, "custom program %d needs edge weights", o.custom_id);

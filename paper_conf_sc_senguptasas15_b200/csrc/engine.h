@@ -2,6 +2,7 @@
 #pragma once
 #include <cmath>
 #include <cstring>
+#include <cstdlib>
 #include <cuda_runtime.h>
 
 #include <map>
@@ -147,6 +148,10 @@ template <class OffT> inline Part<OffT> make_part(gr_graph *g) {
   P.in_src = g->in_src;
   P.in_w = g->in_w;
   P.prd_div = g->prd_div;
+  {
+    static const int gate = getenv("GR_GATE") ? atoi(getenv("GR_GATE")) : 1;
+    P.gate = (uint32_t)gate;
+  }
   P.estate = g->estate;
   P.out_eid = g->out_eid;
   P.ds_src = g->ds_src;

@@ -21,6 +21,7 @@
 #include "engine.h"
 #include "kernels_frontier.cuh"
 #include "kernels_pr.cuh"
+#include "prog_desc.h"
 
 namespace gr {
 
@@ -129,12 +130,21 @@ static __global__ void k_part_counts(const Ctl *ctl, uint64_t *out) {
   out[1] = ctl->cnt_act[ctl->iter & 1u];
 }
 
-template <class Prog, class OffT>
-gr_status run_frontier_part(gr_graph *g, const gr_run_opts *o, cudaStream_t s, gr_run_stats *st) {
+// D: the program's traits and kernels (prog_desc.h) — built-in or run-time compiled
+template <class OffT>
+gr_status run_frontier_part(gr_graph *g, const gr_run_opts *o, cudaStream_t s, gr_run_stats *st,
+                            const ProgDesc &D) {
+  constexpr int K = sizeof(OffT) == 8 ? 1 : 0;
+#define KL(fn, grid, block, ...)                                   \
+  do {                                                             \
+    void *a_[] = {__VA_ARGS__};                                    \
+    gr_status r_ = klaunch(D, fn, (grid), (block), a_, s);         \
+    if (r_ != GR_OK) return r_;                                    \
+  } while (0)
   Comm *C = g->comm;
-  constexpr bool kScatter = HasScatter<Prog>::value;
-  if constexpr (kScatter) {  // this rank's edges (its CSC and activation CSR) carry the states
-    gr_status ss = scatter_setup(g, Prog::kUsesWeights);
+  const bool kScatter = D.scatter;
+  if (kScatter) {  // this rank's edges (its CSC and activation CSR) carry the states
+    gr_status ss = scatter_setup(g, D.uses_weights);
     if (ss != GR_OK) return ss;
   }
   Part<OffT> P = make_part<OffT>(g);
@@ -154,19 +164,29 @@ gr_status run_frontier_part(gr_graph *g, const gr_run_opts *o, cudaStream_t s, g
   prd_setup(h, o, g->H.n);
   h.kstart[0] = h.kstart[1] = ~0ull;
   PCK(cudaMemcpyAsync(g->ctl, &h, sizeof h, cudaMemcpyHostToDevice, s));
-  k_init_values<Prog, OffT><<<g->num_sms * 4, 256, 0, s>>>(P, o->source);
-  if constexpr (kScatter) k_init_edges<Prog, OffT><<<g->num_sms * 8, 256, 0, s>>>(P, g->H.m_in);
-  k_fill<typename Prog::GatherT><<<std::min<uint32_t>((g->hub_cap + 255) / 256, 1024), 256, 0, s>>>(
-      reinterpret_cast<typename Prog::GatherT *>(g->hub_acc), Prog::identity_host(), g->hub_cap);
+  uint32_t src0 = o->source;
+  KL(D.init_values[K], g->num_sms * 4, 256, &P, &src0);
+  if (kScatter) {
+    uint64_t m_in = g->H.m_in;
+    KL(D.init_edges[K], g->num_sms * 8, 256, &P, &m_in);
+  }
+  {
+    void *acc = g->hub_acc;
+    unsigned long long cnt = g->hub_cap;
+    KL(D.fill, std::min<uint32_t>((g->hub_cap + 255) / 256, 1024) + 1, 256, &acc, &cnt);
+  }
   PCK(cudaMemsetAsync(g->hub_done, 0, 4ull * g->hub_cap, s));
-  if (Prog::kInit == kInitAll && g->n_static_hubs) {
+  if (D.init == kInitAll && g->n_static_hubs) {
     PCK(cudaMemcpyAsync(g->listH[0], g->static_hubs, 4ull * g->n_static_hubs, cudaMemcpyDeviceToDevice, s));
     PCK(cudaMemcpyAsync(g->chkA_h[0], g->static_chk_h, 4ull * g->n_static_chunks, cudaMemcpyDeviceToDevice, s));
     PCK(cudaMemcpyAsync(g->chkA_c[0], g->static_chk_c, 4ull * g->n_static_chunks, cudaMemcpyDeviceToDevice, s));
   }
   // BFS runs unfused here (apply, exchange, activate), so its A lists are built
   // by the generic activation (hub chunks by in-degree).
-  k_init_frontier<Prog, OffT><<<1, kBlock, 0, s>>>(P, o->source, g->n_static_hubs, g->n_static_chunks);
+  {
+    uint32_t nh = (uint32_t)g->n_static_hubs, nc = (uint32_t)g->n_static_chunks;
+    KL(D.init_frontier[K], 1, kBlock, &P, &src0, &nh, &nc);
+  }
   launches += 3;
   PCK(cudaGetLastError());
   PCK(cudaMemsetAsync(&g->ctl->stop, 0, sizeof(uint32_t), s));  // the host decides termination
@@ -194,8 +214,7 @@ gr_status run_frontier_part(gr_graph *g, const gr_run_opts *o, cudaStream_t s, g
       P.n_xp = (uint32_t)C->world;
       P.xp_off = (uint32_t)g->H.own_lo;
     }
-    if (fx) k_gather_apply_x<Prog, OffT><<<grid, kBlock, 0, s>>>(P);
-    else k_gather_apply<Prog, OffT><<<grid, kBlock, 0, s>>>(P);
+    KL(fx ? D.gather_apply_x[K] : D.gather_apply[K], grid, kBlock, &P);
     P.n_xp = 0;
     k_part_counts<<<1, 1, 0, s>>>(g->ctl, g->x_cnt);
     launches += 2;
@@ -230,10 +249,12 @@ gr_status run_frontier_part(gr_graph *g, const gr_run_opts *o, cudaStream_t s, g
     PCK(cudaMemsetAsync(&g->ctl->cnt_C, 0, sizeof(uint32_t), s));
     if (tot) k_classify<OffT><<<std::min<uint32_t>(grid, (uint32_t)((tot + kBlock - 1) / kBlock)), kBlock, 0, s>>>(
         P, xv, xval, (uint32_t)tot, R);
-    if constexpr (kScatter) {
+    if (kScatter) {
       // commit every rank's C_t first: scatter reads the committed values of its targets
       k_commit_only<OffT><<<grid, kBlock, 0, s>>>(P);
-      k_scatter_activate<Prog, OffT><<<grid, kBlock, 0, s>>>(P, 0ull, 0);
+      unsigned long long cond = 0;
+      int ug = 0;
+      KL(D.scatter_activate[K], grid, kBlock, &P, &cond, &ug);
       launches++;
     } else {
       k_activate<OffT><<<grid, kBlock, 0, s>>>(P, 0ull, 0);
@@ -257,8 +278,9 @@ gr_status run_frontier_part(gr_graph *g, const gr_run_opts *o, cudaStream_t s, g
   st->bytes_nvlink = C->bytes_in;
   g->epoch_next = h.epoch_base + t + 2;
   g->trace_rows = std::min<uint64_t>(t, g->trace_cap);
-  st->bytes_hbm_model = (Prog::kUsesWeights ? 5 : 4) * c.tot_gathered + 4 * c.tot_scattered;
+  st->bytes_hbm_model = (D.uses_weights ? 5 : 4) * c.tot_gathered + 4 * c.tot_scattered;
   return GR_OK;
+#undef KL
 }
 
 // PageRank over owner partitions. Each rank runs the single-GPU superstep
@@ -372,27 +394,12 @@ gr_status part_fetch_trace(gr_graph *g, uint64_t *dst, uint64_t max_rows, uint64
 }
 
 gr_status run_part(gr_graph *g, const gr_run_opts *o, cudaStream_t s, gr_run_stats *st) {
-  switch (o->algo) {
-    case GR_BFS:
-      return g->off64 ? run_frontier_part<ProgBFS, uint64_t>(g, o, s, st) : run_frontier_part<ProgBFS, uint32_t>(g, o, s, st);
-    case GR_SSSP:
-      return g->off64 ? run_frontier_part<ProgSSSP, uint64_t>(g, o, s, st)
-                      : run_frontier_part<ProgSSSP, uint32_t>(g, o, s, st);
-    case GR_CC:
-      return g->off64 ? run_frontier_part<ProgCC, uint64_t>(g, o, s, st) : run_frontier_part<ProgCC, uint32_t>(g, o, s, st);
-    case GR_PAGERANK_DELTA:
-      return g->off64 ? run_frontier_part<ProgPRDelta, uint64_t>(g, o, s, st)
-                      : run_frontier_part<ProgPRDelta, uint32_t>(g, o, s, st);
-    case GR_CUSTOM:
-#define GR_X(id, T)                                                                                         \
-  if (o->custom_id == id)                                                                                   \
-    return g->off64 ? run_frontier_part<T, uint64_t>(g, o, s, st) : run_frontier_part<T, uint32_t>(g, o, s, st);
-      GR_CUSTOM_PROGRAMS(GR_X)
-#undef GR_X
-      return fail(GR_EUNSUPPORTED, "no custom program %d", o->custom_id);
-    default:
-      return g->off64 ? run_pagerank_part<uint64_t>(g, o, s, st) : run_pagerank_part<uint32_t>(g, o, s, st);
-  }
+  if (o->algo == GR_PAGERANK)
+    return g->off64 ? run_pagerank_part<uint64_t>(g, o, s, st) : run_pagerank_part<uint32_t>(g, o, s, st);
+  ProgDesc D;
+  gr_status r = prog_desc(o->algo, o->custom_id, &D);
+  if (r != GR_OK) return r;
+  return g->off64 ? run_frontier_part<uint64_t>(g, o, s, st, D) : run_frontier_part<uint32_t>(g, o, s, st, D);
 }
 
 }  // namespace gr

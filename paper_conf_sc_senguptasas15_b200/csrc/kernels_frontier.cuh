@@ -76,6 +76,9 @@ __device__ typename Prog::GatherT gather_warp(const Part<OffT> &P, bool valid, u
   const uint32_t lane = lane_id();
   G acc = Prog::identity();
   act = false;
+  // dense supersteps of selective programs may read val[u] only for changed sources
+  // (Selective<>; P.gate, GR_GATE)
+  const bool kGate = kDense && Selective<Prog>::value && P.gate;
   // warp-cooperative: one vertex of degree in (32, kHubDegree] at a time
   uint32_t big = __ballot_sync(0xffffffffu, valid && deg > 32);
   while (big) {
@@ -97,20 +100,27 @@ __device__ typename Prog::GatherT gather_warp(const Part<OffT> &P, bool valid, u
       uint32_t v[4], bw[4];
 #pragma unroll
       for (int q = 0; q < 4; q++) {
-        v[q] = P.val[u[q]];
+        if (!kGate) v[q] = P.val[u[q]];
         if (kDense) bw[q] = ld_cg(bits + (u[q] >> 5));
+      }
+      bool h[4];
+#pragma unroll
+      for (int q = 0; q < 4; q++) {
+        h[q] = kDense && ((bw[q] >> (u[q] & 31)) & 1u);
+        if (kGate) v[q] = h[q] ? P.val[u[q]] : 0u;
       }
 #pragma unroll
       for (int q = 0; q < 4; q++) {
-        r = Prog::gatherReduce(r, Prog::gatherMap(dv, v[q], w[q], u[q], cx));
-        if (kDense) hit |= (bw[q] >> (u[q] & 31)) & 1u;
+        if (!kGate || h[q]) r = Prog::gatherReduce(r, Prog::gatherMap(dv, v[q], w[q], u[q], cx));
+        hit |= h[q];
       }
     }
     for (; k < d; k += 32) {
       const uint32_t u = ldg_nc(P.in_src + b + k);
       const uint32_t w = edge_w<Prog>(P, b + k);
-      r = Prog::gatherReduce(r, Prog::gatherMap(dv, P.val[u], w, u, cx));
-      if (kDense) hit |= test_bit_cg(bits, u);
+      const bool h = kDense && test_bit_cg(bits, u);
+      if (!kGate || h) r = Prog::gatherReduce(r, Prog::gatherMap(dv, P.val[u], w, u, cx));
+      hit |= h;
     }
     r = warp_reduce_prog<Prog>(r);
     const bool any = kDense ? (__any_sync(0xffffffffu, hit) != 0) : false;
@@ -155,8 +165,15 @@ __device__ typename Prog::GatherT gather_warp(const Part<OffT> &P, bool valid, u
     uint32_t sv[kBatch], sb[kBatch];
 #pragma unroll
     for (int q = 0; q < kBatch; q++) {
-      sv[q] = act_q[q] ? P.val[su[q]] : 0u;
+      if (!kGate) sv[q] = act_q[q] ? P.val[su[q]] : 0u;
       if (kDense) sb[q] = act_q[q] ? ld_cg(bits + (su[q] >> 5)) : 0u;
+    }
+    if (kGate) {  // only the changed sources' values: unmarked items map to identity()
+#pragma unroll
+      for (int q = 0; q < kBatch; q++) {
+        act_q[q] = act_q[q] && ((sb[q] >> (su[q] & 31)) & 1u);
+        sv[q] = act_q[q] ? P.val[su[q]] : 0u;
+      }
     }
 #pragma unroll
     for (int q = 0; q < kBatch; q++) {
@@ -203,6 +220,7 @@ __device__ typename Prog::GatherT gather_block(const Part<OffT> &P, uint64_t beg
                                                typename Prog::GatherT *sblk, const Ctx &cx, const uint32_t *bits,
                                                bool *act) {
   using G = typename Prog::GatherT;
+  const bool kGate = kDense && Selective<Prog>::value && P.gate;  // see gather_warp
   G r = Prog::identity();
   bool hit = false;
   uint32_t k = threadIdx.x;
@@ -216,20 +234,27 @@ __device__ typename Prog::GatherT gather_block(const Part<OffT> &P, uint64_t beg
     uint32_t v[4], bw[4];
 #pragma unroll
     for (int q = 0; q < 4; q++) {
-      v[q] = P.val[u[q]];
+      if (!kGate) v[q] = P.val[u[q]];
       if (kDense) bw[q] = ld_cg(bits + (u[q] >> 5));
+    }
+    bool h[4];
+#pragma unroll
+    for (int q = 0; q < 4; q++) {
+      h[q] = kDense && ((bw[q] >> (u[q] & 31)) & 1u);
+      if (kGate) v[q] = h[q] ? P.val[u[q]] : 0u;
     }
 #pragma unroll
     for (int q = 0; q < 4; q++) {
-      r = Prog::gatherReduce(r, Prog::gatherMap(dval, v[q], w[q], u[q], cx));
-      if (kDense) hit |= (bw[q] >> (u[q] & 31)) & 1u;
+      if (!kGate || h[q]) r = Prog::gatherReduce(r, Prog::gatherMap(dval, v[q], w[q], u[q], cx));
+      hit |= h[q];
     }
   }
   for (; k < deg; k += kBlock) {
     const uint32_t u = ldg_nc(P.in_src + beg + k);
     const uint32_t w = edge_w<Prog>(P, beg + k);
-    r = Prog::gatherReduce(r, Prog::gatherMap(dval, P.val[u], w, u, cx));
-    if (kDense) hit |= test_bit_cg(bits, u);
+    const bool h = kDense && test_bit_cg(bits, u);
+    if (!kGate || h) r = Prog::gatherReduce(r, Prog::gatherMap(dval, P.val[u], w, u, cx));
+    hit |= h;
   }
   if (kDense) {
     const int any = __syncthreads_or(hit ? 1 : 0);
@@ -794,7 +819,6 @@ __global__ void __launch_bounds__(kBlock) k_gather_apply(const __grid_constant__
   else gather_phase<Prog, false>(P, V);
 }
 
-#ifndef GR_JIT
 // partitioned runs with the exchange fused into the gather (sparse supersteps only)
 template <class Prog, class OffT>
 __global__ void __launch_bounds__(kBlock) k_gather_apply_x(const __grid_constant__ Part<OffT> P) {
@@ -803,7 +827,6 @@ __global__ void __launch_bounds__(kBlock) k_gather_apply_x(const __grid_constant
   if (V.stop) return;
   gather_phase<Prog, false, OffT, true>(P, V);
 }
-#endif
 
 // Commit C_t and FrontierActivate (the other phase of superstep t).
 template <class OffT>
@@ -1338,8 +1361,10 @@ __global__ void __launch_bounds__(kBlock) k_scatter_activate(const __grid_consta
   __shared__ View V;
   load_view(P.ctl, V);
   if (V.stop) {
+#ifndef GR_JIT  // run-time programs never run inside a conditional graph node
     if (use_graph && blockIdx.x == 0 && threadIdx.x == 0)
       cudaGraphSetConditional((cudaGraphConditionalHandle)cond, 0u);
+#endif
     return;
   }
   if constexpr (HasScatter<Prog>::value) scatter_activate_phase<Prog>(P, V);
@@ -1429,17 +1454,23 @@ __device__ __forceinline__ void dense_seg_phase(const Part<OffT> &P, const View 
     }
     uint32_t sv[kDsIpt];
     bool sa[kDsIpt];
+    const bool kGate = Selective<Prog>::value && P.gate;  // read only the changed sources' values (gather_warp)
 #pragma unroll
     for (int k = 0; k < kDsIpt; k++) {  // all loads of the 8 items in flight together
       const bool ok = src[k] != kDsNoSrc;
-      sv[k] = ok ? __ldg(P.val + src[k]) : 0u;
+      if (!kGate) sv[k] = ok ? __ldg(P.val + src[k]) : 0u;
       sa[k] = ok && test_bit(bits, src[k]);
+    }
+    if (kGate) {
+#pragma unroll
+      for (int k = 0; k < kDsIpt; k++) sv[k] = sa[k] ? __ldg(P.val + src[k]) : 0u;
     }
     G g[kDsIpt];
 #pragma unroll
     for (int k = 0; k < kDsIpt; k++)
-      g[k] = src[k] != kDsNoSrc ? Prog::gatherMap(0u, sv[k], Prog::kUsesWeights ? w8[k] : 0u, src[k], cx)
-                                : Prog::identity();
+      g[k] = (kGate ? sa[k] : src[k] != kDsNoSrc)
+                 ? Prog::gatherMap(0u, sv[k], Prog::kUsesWeights ? w8[k] : 0u, src[k], cx)
+                 : Prog::identity();
     const uint32_t b = (fw >> ((lane & 3) * 8)) & 0xFFu;  // bit k: my item k starts a row
     uint32_t bn = __shfl_down_sync(0xffffffffu, b, 1) & 1u;
     if (lane == 31) bn = fnext;
@@ -1753,6 +1784,14 @@ __global__ void k_init_run(const __grid_constant__ Part<OffT> P, uint32_t source
 template <class T> __global__ void k_fill(T *p, T value, uint64_t count) {
   for (uint64_t i = blockIdx.x * (uint64_t)blockDim.x + threadIdx.x; i < count; i += (uint64_t)gridDim.x * blockDim.x)
     p[i] = value;
+}
+
+// identity() into a gather accumulator array of the program's GatherT (hub slots)
+template <class Prog> __global__ void k_prog_fill(void *p, unsigned long long count) {
+  typename Prog::GatherT *a = reinterpret_cast<typename Prog::GatherT *>(p);
+  for (unsigned long long i = blockIdx.x * (unsigned long long)blockDim.x + threadIdx.x; i < count;
+       i += (unsigned long long)gridDim.x * blockDim.x)
+    a[i] = Prog::identity();
 }
 
 static __global__ void k_fill_u32(uint32_t *p, uint32_t value, uint64_t count) {

@@ -840,6 +840,7 @@ struct PrLoop {
   const uint32_t *long_c, *long_f;
   uint32_t n_long, hot_k, num_tiles, iters;
   uint32_t *bar;                       // [0] arrivals, [1] generation
+  unsigned long long *ts;              // GR_PR_PHASES=1: %globaltimer at the loop start and after each barrier
 };
 
 __device__ __forceinline__ void pr_grid_sync(uint32_t *bar) {
@@ -885,6 +886,8 @@ __global__ void __launch_bounds__(1024, 1) k_pr_seg_loop(const __grid_constant__
   const uint32_t stride = gridDim.x * nw;
   const uint4 *src4 = reinterpret_cast<const uint4 *>(L.seg_src) + 2 * lane;
   const uint64_t gtid = blockIdx.x * (uint64_t)blockDim.x + threadIdx.x, gthreads = (uint64_t)gridDim.x * blockDim.x;
+  const bool stamp = L.ts && blockIdx.x == 0 && threadIdx.x == 0;
+  if (stamp) L.ts[0] = gtimer();
   for (uint32_t t = 0; t < L.iters; t++) {
     PrArgs<OffT> a = a0;
     a.contrib_in = L.contrib[t & 1];
@@ -927,6 +930,7 @@ __global__ void __launch_bounds__(1024, 1) k_pr_seg_loop(const __grid_constant__
       }
     }
     pr_grid_sync(L.bar);
+    if (stamp) L.ts[1 + 2 * t] = gtimer();
     // ---- phase 2: rows split between tiles, hot-table pack
     for (uint64_t c = gtid; c < L.num_tiles; c += gthreads) {
       const uint32_t row = a.head_row[c];
@@ -948,6 +952,7 @@ __global__ void __launch_bounds__(1024, 1) k_pr_seg_loop(const __grid_constant__
       for (uint64_t k = gtid; k < L.hot_k; k += gthreads)
         if (!L.hot_split[k]) hot_next[k] = a.contrib_out[L.hot_ids[k]];
     pr_grid_sync(L.bar);
+    if (stamp) L.ts[2 + 2 * t] = gtimer();
   }
 }
 

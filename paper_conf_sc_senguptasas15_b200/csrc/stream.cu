@@ -21,6 +21,7 @@
 #include "engine.h"
 #include "kernels_pr.cuh"
 #include "kernels_stream.cuh"
+#include "prog_desc.h"
 
 namespace gr {
 
@@ -324,16 +325,25 @@ static gr_status stream_pagerank(gr_graph *g, const gr_run_opts *o, cudaStream_t
 }
 
 // ------------------------------------------------------- frontier programs
-template <class Prog, class OffT>
-static gr_status stream_frontier(gr_graph *g, const gr_run_opts *o, cudaStream_t cs, gr_run_stats *st) {
+// D: the program's traits and kernels (prog_desc.h) — built-in or run-time compiled
+template <class OffT>
+static gr_status stream_frontier(gr_graph *g, const gr_run_opts *o, cudaStream_t cs, gr_run_stats *st,
+                                 const ProgDesc &D) {
+  constexpr int K = sizeof(OffT) == 8 ? 1 : 0;
+#define KL(fn, grid, block, ...)                                   \
+  do {                                                             \
+    void *a_[] = {__VA_ARGS__};                                    \
+    gr_status r_ = klaunch(D, fn[K], (grid), (block), a_, cs);     \
+    if (r_ != GR_OK) return r_;                                    \
+  } while (0)
   Streamer *S = S_(g);
   const HostGraph &H = g->H;
   const uint32_t P = S->P;
-  constexpr bool kScatter = HasScatter<Prog>::value;
-  if constexpr (kScatter) {
+  const bool kScatter = D.scatter;
+  if (kScatter) {
     gr_status ss = stream_scatter_setup(g, S);
     if (ss != GR_OK) return ss;
-    if (Prog::kUsesWeights && !S->zc_ow) return fail(GR_EINVAL, "the program reads edge weights but the graph has none");
+    if (D.uses_weights && !S->zc_ow) return fail(GR_EINVAL, "the program reads edge weights but the graph has none");
   }
   Part<OffT> P0 = make_part<OffT>(g);
   uint64_t launches = 0;
@@ -351,7 +361,7 @@ static gr_status stream_frontier(gr_graph *g, const gr_run_opts *o, cudaStream_t
   prd_setup(h, o, H.n);
   std::vector<uint8_t> act(P, 0);
   std::vector<uint32_t> a0;
-  if (Prog::kInit == kInitSourceChanged) {
+  if (D.init == kInitSourceChanged) {
     // A_0 = out-neighbours of the source, read straight from the pinned host CSR
     for (uint64_t e = H.out_off[o->source]; e < H.out_off[o->source + 1]; e++)
       a0.push_back(H.out_dst.as<uint32_t>()[e]);
@@ -361,20 +371,23 @@ static gr_status stream_frontier(gr_graph *g, const gr_run_opts *o, cudaStream_t
     h.stop = a0.empty() ? 1u : 0u;
   }
   SCK(cudaMemcpyAsync(g->ctl, &h, sizeof h, cudaMemcpyHostToDevice, cs));
-  k_init_values<Prog, OffT><<<g->num_sms * 4, 256, 0, cs>>>(P0, o->source);
+  uint32_t src0 = o->source;
+  KL(D.init_values, g->num_sms * 4, 256, &P0, &src0);
   launches++;
-  if constexpr (kScatter) {  // states in host memory, written in place; the source scatters at init
-    k_init_edges<Prog, OffT><<<g->num_sms * 8, 256, 0, cs>>>(P0, H.m_in);
+  if (kScatter) {  // states in host memory, written in place; the source scatters at init
+    uint64_t m_in = H.m_in;
+    KL(D.init_edges, g->num_sms * 8, 256, &P0, &m_in);
     launches++;
-    if (Prog::kInit == kInitSourceChanged) {
-      k_s_init_scatter<Prog, OffT><<<1, kBlock, 0, cs>>>(zc_part<OffT>(g, S, false), o->source);
+    if (D.init == kInitSourceChanged) {
+      Part<OffT> Pz = zc_part<OffT>(g, S, false);
+      KL(D.s_init_scatter, 1, kBlock, &Pz, &src0);
       launches++;
     }
   }
   auto shard_of_host = [&](uint64_t x) {
     return (uint32_t)(std::upper_bound(H.bounds.begin(), H.bounds.end(), x) - H.bounds.begin() - 1);
   };
-  if (Prog::kInit == kInitSourceChanged) {
+  if (D.init == kInitSourceChanged) {
     if (!a0.empty()) {
       SCK(cudaMemcpyAsync(S->d_list, a0.data(), 4 * a0.size(), cudaMemcpyHostToDevice, cs));
       k_s_stamp_list<OffT><<<std::max<uint32_t>(1, (uint32_t)std::min<size_t>(1024, (a0.size() + 255) / 256)), 256, 0,
@@ -383,9 +396,10 @@ static gr_status stream_frontier(gr_graph *g, const gr_run_opts *o, cudaStream_t
     }
     for (uint32_t x : a0) act[shard_of_host(x)] = 1;
   } else {
-    k_init_frontier<Prog, OffT><<<1, kBlock, 0, cs>>>(P0, o->source, 0u, 0u);
+    uint32_t z0 = 0, z1 = 0;
+    KL(D.init_frontier, 1, kBlock, &P0, &src0, &z0, &z1);
     launches++;
-    if (Prog::kInit == kInitAll) std::fill(act.begin(), act.end(), 1);
+    if (D.init == kInitAll) std::fill(act.begin(), act.end(), 1);
     else act[shard_of_host(o->source)] = 1;
   }
   SCK(cudaGetLastError());
@@ -394,7 +408,7 @@ static gr_status stream_frontier(gr_graph *g, const gr_run_opts *o, cudaStream_t
   uint8_t *h_changed = S->h_flags, *h_next = S->h_flags + P;
   const double avg_in = H.own_n() ? (double)H.m_in / (double)H.own_n() : 0.0;
   const double avg_out = H.n ? (double)H.m_in / (double)H.n : 0.0;
-  const uint64_t wb = Prog::kUsesWeights ? 5 : 4;
+  const uint64_t wb = D.uses_weights ? 5 : 4;
   // ablation knob (Fig. 15): GR_STREAM_NO_SKIP=1 moves and scans every shard every superstep
   const bool no_skip = getenv("GR_STREAM_NO_SKIP") && getenv("GR_STREAM_NO_SKIP")[0] == '1';
   if (no_skip) std::fill(act.begin(), act.end(), 1);
@@ -403,7 +417,7 @@ static gr_status stream_frontier(gr_graph *g, const gr_run_opts *o, cudaStream_t
     SCK(cudaMemsetAsync(S->d_changed, 0, P, cs));
     // gather phase: whole-shard DMA, or in place when A_t's in-edges are few (f1)
     bool zc_g = false;
-    if (Prog::kHasGather) {
+    if (D.has_gather) {
       uint64_t shard_e = 0;
       for (uint32_t s = 0; s < P; s++)
         if (act[s] || no_skip) shard_e += S->in_b[s + 1] - S->in_b[s];
@@ -412,32 +426,33 @@ static gr_status stream_frontier(gr_graph *g, const gr_run_opts *o, cudaStream_t
       zc_g = want_zc(o, (uint64_t)(nA * avg_in), shard_e);
       if (zc_g) S->zc_phases++;
     }
-    const Part<OffT> Pz_in = zc_part<OffT>(g, S, true);
+    Part<OffT> Pz_in = zc_part<OffT>(g, S, true);
     if (zc_g) {  // in place: one launch over every shard (stamps select A_t)
-      const uint32_t v0 = (uint32_t)H.own_lo, v1 = (uint32_t)H.own_hi;
-      k_s_gather_apply<Prog, OffT><<<grid_for(g, v1 - v0), kBlock, 0, cs>>>(Pz_in, v0, v1, kAllShards, S->d_changed,
-                                                                            S->cstamp, S->d_bounds, P);
+      uint32_t v0 = (uint32_t)H.own_lo, v1 = (uint32_t)H.own_hi, all = kAllShards, np = P;
+      KL(D.s_gather_apply, grid_for(g, v1 - v0), kBlock, &Pz_in, &v0, &v1, &all, &S->d_changed, &S->cstamp,
+         &S->d_bounds, &np);
       launches++;
     }
     for (uint32_t s = 0; s < P && !zc_g; s++) {
       if (!act[s] && !no_skip) continue;  // frontier skipping: no copy, no launch
-      const uint32_t v0 = (uint32_t)H.bounds[s], v1 = (uint32_t)H.bounds[s + 1];
-      if (Prog::kHasGather) {
+      uint32_t v0 = (uint32_t)H.bounds[s], v1 = (uint32_t)H.bounds[s + 1];
+      if (D.has_gather) {
         int k = -1;
         if (!zc_g) {
-          gr_status gs = stage(g, S, cs, true, s, Prog::kUsesWeights, &k);
+          gr_status gs = stage(g, S, cs, true, s, D.uses_weights, &k);
           if (gs != GR_OK) return gs;
         }
-        const Part<OffT> Pk = zc_g ? Pz_in : slot_part<OffT>(g, S, k, true, s);
-        k_s_gather_apply<Prog, OffT><<<grid_for(g, (v1 - v0)), kBlock, 0, cs>>>(Pk, v0, v1, s, S->d_changed,
-                                                                                   S->cstamp, S->d_bounds, P);
+        Part<OffT> Pk = zc_g ? Pz_in : slot_part<OffT>(g, S, k, true, s);
+        uint32_t sh = s, np = P;
+        KL(D.s_gather_apply, grid_for(g, v1 - v0), kBlock, &Pk, &v0, &v1, &sh, &S->d_changed, &S->cstamp,
+           &S->d_bounds, &np);
         if (k >= 0) SCK(cudaEventRecord(S->freed[k], cs));
       } else {
         k_s_bfs_apply<OffT><<<grid_for(g, v1 - v0), kBlock, 0, cs>>>(P0, v0, v1, s, S->d_changed, S->cstamp);
       }
       launches++;
     }
-    if (Prog::kHasGather) {
+    if (D.has_gather) {
       k_s_commit<OffT><<<g->num_sms * 2, 256, 0, cs>>>(P0);
       launches++;
     }
@@ -451,23 +466,22 @@ static gr_status stream_frontier(gr_graph *g, const gr_run_opts *o, cudaStream_t
       if (h_changed[s] || no_skip) shard_o += S->out_b[s + 1] - S->out_b[s];
     const bool zc_a = want_zc(o, (uint64_t)((double)g->h_ctl->changed * avg_out), shard_o);
     if (zc_a && shard_o) S->zc_phases++;
-    const Part<OffT> Pz_out = zc_part<OffT>(g, S, false);
+    Part<OffT> Pz_out = zc_part<OffT>(g, S, false);
     if (zc_a && shard_o) {  // in place: one launch over every shard (changed stamps select C_t)
-      const uint32_t u0 = (uint32_t)H.bounds[0], u1 = (uint32_t)H.bounds[P];
-      k_s_activate<Prog, OffT><<<grid_for(g, u1 - u0), kBlock, 0, cs>>>(Pz_out, u0, u1, S->d_bounds, P, S->d_next,
-                                                                  S->cstamp);
+      uint32_t u0 = (uint32_t)H.bounds[0], u1 = (uint32_t)H.bounds[P], np = P;
+      KL(D.s_activate, grid_for(g, u1 - u0), kBlock, &Pz_out, &u0, &u1, &S->d_bounds, &np, &S->d_next, &S->cstamp);
       launches++;
     }
     for (uint32_t s = 0; s < P && !zc_a; s++) {
       if (!h_changed[s] && !no_skip) continue;
-      const uint32_t u0 = (uint32_t)H.bounds[s], u1 = (uint32_t)H.bounds[s + 1];
+      uint32_t u0 = (uint32_t)H.bounds[s], u1 = (uint32_t)H.bounds[s + 1], np = P;
       int k = -1;
       if (!zc_a) {
         gr_status gs = stage(g, S, cs, false, s, false, &k);
         if (gs != GR_OK) return gs;
       }
-      const Part<OffT> Pk = zc_a ? Pz_out : slot_part<OffT>(g, S, k, false, s);
-      k_s_activate<Prog, OffT><<<grid_for(g, u1 - u0), kBlock, 0, cs>>>(Pk, u0, u1, S->d_bounds, P, S->d_next, S->cstamp);
+      Part<OffT> Pk = zc_a ? Pz_out : slot_part<OffT>(g, S, k, false, s);
+      KL(D.s_activate, grid_for(g, u1 - u0), kBlock, &Pk, &u0, &u1, &S->d_bounds, &np, &S->d_next, &S->cstamp);
       if (k >= 0) SCK(cudaEventRecord(S->freed[k], cs));
       launches++;
     }
@@ -489,8 +503,9 @@ static gr_status stream_frontier(gr_graph *g, const gr_run_opts *o, cudaStream_t
   st->kernel_launches += launches;
   g->epoch_next = h.epoch_base + c.iter + 2;
   g->trace_rows = std::min<uint64_t>(c.iter, g->trace_cap);
-  st->bytes_hbm_model = (Prog::kUsesWeights ? 5 : 4) * c.tot_gathered + 4 * c.tot_scattered;
+  st->bytes_hbm_model = (D.uses_weights ? 5 : 4) * c.tot_gathered + 4 * c.tot_scattered;
   return GR_OK;
+#undef KL
 }
 
 gr_status run_streamed(gr_graph *g, const gr_run_opts *o, gr_run_stats *st) {
@@ -502,31 +517,12 @@ gr_status run_streamed(gr_graph *g, const gr_run_opts *o, gr_run_stats *st) {
   S->zc_phases = 0;
   SCK(cudaEventRecord(g->ev_start, cs));
   gr_status r;
-  switch (o->algo) {
-    case GR_BFS:
-      r = g->off64 ? stream_frontier<ProgBFS, uint64_t>(g, o, cs, st) : stream_frontier<ProgBFS, uint32_t>(g, o, cs, st);
-      break;
-    case GR_SSSP:
-      r = g->off64 ? stream_frontier<ProgSSSP, uint64_t>(g, o, cs, st)
-                   : stream_frontier<ProgSSSP, uint32_t>(g, o, cs, st);
-      break;
-    case GR_CC:
-      r = g->off64 ? stream_frontier<ProgCC, uint64_t>(g, o, cs, st) : stream_frontier<ProgCC, uint32_t>(g, o, cs, st);
-      break;
-    case GR_PAGERANK_DELTA:
-      r = g->off64 ? stream_frontier<ProgPRDelta, uint64_t>(g, o, cs, st)
-                   : stream_frontier<ProgPRDelta, uint32_t>(g, o, cs, st);
-      break;
-    case GR_CUSTOM:
-      r = GR_EUNSUPPORTED;
-#define GR_X(id, T)                                                                                           \
-  if (o->custom_id == id)                                                                                     \
-    r = g->off64 ? stream_frontier<T, uint64_t>(g, o, cs, st) : stream_frontier<T, uint32_t>(g, o, cs, st);
-      GR_CUSTOM_PROGRAMS(GR_X)
-#undef GR_X
-      break;
-    default:
-      r = g->off64 ? stream_pagerank<uint64_t>(g, o, cs, st) : stream_pagerank<uint32_t>(g, o, cs, st);
+  if (o->algo == GR_PAGERANK) {
+    r = g->off64 ? stream_pagerank<uint64_t>(g, o, cs, st) : stream_pagerank<uint32_t>(g, o, cs, st);
+  } else {
+    ProgDesc D;
+    if ((r = prog_desc(o->algo, o->custom_id, &D)) != GR_OK) return r;
+    r = g->off64 ? stream_frontier<uint64_t>(g, o, cs, st, D) : stream_frontier<uint32_t>(g, o, cs, st, D);
   }
   if (r != GR_OK) return r;
   SCK(cudaEventRecord(g->ev_stop, cs));

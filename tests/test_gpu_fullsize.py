@@ -88,3 +88,42 @@ def test_cfg4_cc_full():
         np.testing.assert_array_equal(G.values("cc"), ref)
         np.testing.assert_array_equal(G.trace(), rtr)
         assert st["iterations"] == rit
+
+
+# ---- cfg5 shape (BASELINE.json configs[4]: R-MAT ef16, seed 5, host-streamed
+# shards at 1 GPU) in the configuration bench.py --config 5 runs: streamed
+# mode, K = 2 device slots, zero_copy auto, default shard size (2^26 in+out
+# edges per shard) — at scale 22, the largest the oracle finishes in a test
+# (§3.2, §4.3). A second shard size cuts the
+# same graph into ~32 shards so slots are reused many times per superstep.
+@pytest.fixture(scope="module")
+def cfg5_s22():
+    g = grgen.rmat(22, 16, seed=5)
+    og = oracle.OracleGraph(g.n, g.src, g.dst)
+    pr, _, _ = og.run("pagerank", max_iters=30, damping=0.85)
+    bfs, btr, bit = og.run("bfs", source=0)
+    og.close()
+    return g, pr, (bfs, btr, bit)
+
+
+@pytest.mark.parametrize("shard_edges", [0, 1 << 22])
+def test_cfg5_shape_streamed_pagerank_and_bfs(cfg5_s22, shard_edges):
+    g, pr, (bfs, btr, bit) = cfg5_s22
+    with gr.GraphReduce(g.n, g.src, g.dst, mode="streamed", shard_edges=shard_edges) as G:
+        info = G.info()
+        assert info["mode"] == gr.MODES["streamed"]
+        assert info["num_shards"] >= (2 if shard_edges == 0 else 16)
+        st = G.run("pagerank", max_iters=30, damping=0.85)
+        assert st["iterations"] == 30
+        assert st["bytes_h2d"] >= 30 * 4 * g.m  # every shard's sources cross the link every superstep
+        got = G.values("pagerank").astype(np.float64)
+        err = np.abs(got - pr)
+        assert err.max() <= 1e-6, err.max()
+        assert err.sum() <= 1e-5, err.sum()
+        big = pr >= 1.0 / g.n
+        assert (err[big] / pr[big]).max() <= 1e-4
+        assert abs(got.sum() - pr.sum()) <= 1e-5
+        st = G.run("bfs", source=0)
+        np.testing.assert_array_equal(G.values("bfs"), bfs)
+        np.testing.assert_array_equal(G.trace(), btr)
+        assert st["iterations"] == bit

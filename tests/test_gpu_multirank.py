@@ -15,7 +15,7 @@ pytestmark = pytest.mark.gpu
 
 
 # ------------------------------------------------- partitioned (simulated ranks)
-def run_sim_ranks(n, src, dst, w, G, algo, source=0, max_iters=0):
+def run_sim_ranks(n, src, dst, w, G, algo, source=0, max_iters=0, custom_id=0):
     """G owner partitions on ONE device, one host thread each, exchanging through
     device copies (the same protocol NCCL runs across GPUs)."""
     import os
@@ -28,7 +28,7 @@ def run_sim_ranks(n, src, dst, w, G, algo, source=0, max_iters=0):
         h = None
         try:
             h = gr.gr_graph_load(n, src, dst, w, world=G, rank=r, sim_ranks=G, nccl_unique_id=key)
-            st = gr.gr_run(h, algo, source=source, max_iters=max_iters)
+            st = gr.gr_run(h, algo, source=source, max_iters=max_iters, custom_id=custom_id)
             vals = gr.gr_fetch_vertex_values(h, dtype=np.float32 if algo in gr.FLOAT_ALGOS else np.uint32)
             tr = gr.gr_fetch_frontier_trace(h)
             out[r] = (st, vals, tr, gr.gr_graph_info_get(h))

@@ -465,7 +465,7 @@ def test_runtime_program_equals_oracle(prog):
 
 
 def test_runtime_program_errors():
-    """Compile errors carry the NVRTC log; unsupported modes are refused."""
+    """Compile errors carry the NVRTC log; a program reading weights needs them."""
     with pytest.raises(gr.GrError) as ei:
         gr.gr_program_compile("struct Broken { this is not C++ };", "Broken")
     assert ei.value.status == gr.GR_ECUDA and "NVRTC" in str(ei.value)
@@ -475,11 +475,6 @@ def test_runtime_program_errors():
         with pytest.raises(gr.GrError) as ei:
             G.run("custom", custom_id=cid)
         assert ei.value.status == gr.GR_EINVAL
-    w = grgen.weights(g.m, 1, 64, seed=3)
-    with gr.GraphReduce(g.n, g.src, g.dst, w, mode="streamed", shard_edges=2000) as G:
-        with pytest.raises(gr.GrError) as ei:
-            G.run("custom", custom_id=cid)
-        assert ei.value.status == gr.GR_EUNSUPPORTED
 
 
 @pytest.mark.parametrize("fmt", ["coo", "csr"])
