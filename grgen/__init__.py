@@ -85,6 +85,50 @@ def rmat(scale: int, edgefactor: int = 16, seed: int = 1, a: float = 0.57, b: fl
     return Graph(n=1 << scale, src=src, dst=dst, name=f"rmat{scale}_ef{edgefactor}_s{seed}")
 
 
+_SO_GPU = os.path.join(_HERE, "libgrgen_gpu.so")
+_SRC_GPU = os.path.join(_HERE, "grgen_gpu.cu")
+_lib_gpu = None
+
+
+def build_gpu(force: bool = False) -> str:
+    """Compile libgrgen_gpu.so (nvcc, sm_100a): the GPU generator of the sorted R-MAT layout."""
+    if force or not os.path.exists(_SO_GPU) or os.path.getmtime(_SO_GPU) < os.path.getmtime(_SRC_GPU):
+        tmp = _SO_GPU + f".tmp{os.getpid()}"
+        subprocess.check_call(["/usr/local/cuda/bin/nvcc", "-gencode", "arch=compute_100a,code=sm_100a", "-O3",
+                               "-Xcompiler", "-fPIC", "-shared", "-o", tmp, _SRC_GPU], cwd=_HERE)
+        os.replace(tmp, _SO_GPU)
+    return _SO_GPU
+
+
+def rmat_sorted_gpu(scale: int, edgefactor: int = 16, seed: int = 1, by_src: bool = False, device: int = 0,
+                    a: float = 0.57, b: float = 0.19, c: float = 0.19, other_degrees: bool = True,
+                    budget_bytes: int = 0, adj: np.ndarray | None = None):
+    """grgen.rmat(scale, edgefactor, seed)'s edge multiset as a sorted adjacency, generated on
+    a GPU without materialising the COO (cfg5 at scale): by_src=False gives the in-CSC
+    (offsets by destination, sources sorted), True the out-CSR. Returns (off, adj, other_deg)."""
+    global _lib_gpu
+    if _lib_gpu is None:
+        build_gpu()
+        L = ctypes.CDLL(_SO_GPU)
+        L.grgen_rmat_sorted_gpu.restype = ctypes.c_int
+        L.grgen_rmat_sorted_gpu.argtypes = [ctypes.c_uint32, ctypes.c_uint64, ctypes.c_double, ctypes.c_double,
+                                            ctypes.c_double, ctypes.c_uint64, ctypes.c_int, ctypes.c_int,
+                                            ctypes.c_void_p, ctypes.c_void_p, ctypes.c_void_p, ctypes.c_uint64]
+        _lib_gpu = L
+    n = 1 << scale
+    m = int(edgefactor) << scale
+    off = np.empty(n + 1, np.uint64)
+    if adj is None:
+        adj = np.empty(m + 4, np.uint32)
+    deg = np.empty(n, np.uint32) if other_degrees else None
+    rc = _lib_gpu.grgen_rmat_sorted_gpu(scale, m, a, b, c, seed, 1 if by_src else 0, device, off.ctypes.data,
+                                        adj.ctypes.data, deg.ctypes.data if deg is not None else None,
+                                        budget_bytes)
+    if rc != 0:
+        raise ValueError(f"grgen_rmat_sorted_gpu rc={rc}")
+    return off, adj, deg
+
+
 def weights(m: int, lo: int = 1, hi: int = 64, seed: int = 1) -> np.ndarray:
     w = np.empty(m, np.uint32)
     rc = lib().grgen_weights(m, lo, hi, seed, _p(w), THREADS)

@@ -45,8 +45,14 @@ typedef enum gr_status {
 } gr_status;
 
 typedef enum gr_format {
-  GR_FMT_COO = 0, /* src[i] -> dst[i], any order, duplicates/self-loops kept (multigraph) */
-  GR_FMT_CSR = 1  /* out-edges of u: col_idx[row_offsets[u] .. row_offsets[u+1]) */
+  GR_FMT_COO = 0,   /* src[i] -> dst[i], any order, duplicates/self-loops kept (multigraph) */
+  GR_FMT_CSR = 1,   /* out-edges of u: col_idx[row_offsets[u] .. row_offsets[u+1]) */
+  GR_FMT_SORTED = 2 /* the layout itself, already sorted (single rank; no weights): the in-CSC
+                       (in_offsets[n+1] by destination, in_idx = sources, every row ascending) and/or
+                       the out-CSR (row_offsets / col_idx, every row ascending) of the same edge
+                       multiset. One half alone is accepted for STREAMED graphs (PageRank needs the
+                       in-CSC, BFS the out-CSR; other programs fail with GR_EUNSUPPORTED). This is
+                       how graphs whose COO does not fit host memory are loaded (cfg5 at scale). */
 } gr_format;
 
 /* Programs: the paper's four evaluated algorithms (§6.1). */
@@ -86,6 +92,10 @@ typedef struct gr_edges {
   const uint64_t *row_offsets;   /* CSR: n+1 entries */
   const uint32_t *col_idx;       /* CSR: m entries */
   const uint32_t *weights;       /* nullable; m entries in [0, 255]; required for SSSP */
+  const uint64_t *in_offsets;    /* GR_FMT_SORTED: in-CSC offsets (n+1) by destination, or NULL */
+  const uint32_t *in_idx;        /* GR_FMT_SORTED: in-CSC sources (m entries + 4 spare when borrowed) */
+  const uint32_t *out_degree;    /* GR_FMT_SORTED without an out-CSR: out-degree of every vertex (n),
+                                    PageRank's n_j; NULL = counted from in_idx */
 } gr_edges;
 
 typedef struct gr_load_opts {
@@ -98,7 +108,21 @@ typedef struct gr_load_opts {
   int32_t host_threads;          /* shard-builder threads; 0 = all cores */
   int32_t sim_ranks;             /* > 1: emulate this many owner partitions on ONE device (tests) */
   int32_t build;                 /* gr_build: where the shard layout is built */
+  int32_t transport;             /* gr_transport: how the ranks of a multi-rank graph exchange */
+  int32_t borrow;                /* GR_FMT_SORTED: 1 = use the caller's adjacency arrays in place (no copy;
+                                    each needs 4 spare entries after its m used ones); they must stay
+                                    valid and unchanged until gr_graph_free (streamed graphs page-lock
+                                    them, or use them as they are if the caller already did) */
 } gr_load_opts;
+
+typedef enum gr_transport {
+  GR_TRANSPORT_NCCL = 0, /* one process per GPU; NCCL (bootstrap: gr_get_unique_id) + cudaIpc peer
+                            mappings over NVLink/NVSwitch for the fused exchanges */
+  GR_TRANSPORT_SHM = 1   /* one process per rank on ONE node, ranks may share a GPU: host
+                            collectives through a POSIX shared-memory segment named after the
+                            128-byte id (any bytes, identical on every rank), device data through
+                            cross-process cudaIpc mappings; same protocol as NCCL (tests, MPS) */
+} gr_transport;
 
 typedef enum gr_build {
   GR_BUILD_AUTO = 0,   /* device for resident single-rank COO inputs, else host */
@@ -122,6 +146,10 @@ typedef struct gr_run_opts {
                          0 auto (in place over the host link when the frontier's edges are
                          < 1/8 of the active shards' edges, else DMA whole shards into the
                          device slots), 1 always in place, -1 never */
+  int32_t trace_detail; /* 1: also record, per superstep, the number of shards holding an active vertex
+                           and the number of distinct sources the gather reads (diagnostic: runs the
+                           host loop with extra marking kernels; resident single-rank graphs only,
+                           else GR_EUNSUPPORTED); fetch with gr_fetch_frontier_trace_detail */
 } gr_run_opts;
 
 /* FrontierActivate direction (resident single-rank frontier programs; the
@@ -214,6 +242,13 @@ gr_status gr_fetch_vertex_values(gr_graph *g, void *host_dst, uint64_t bytes);
  * |A_t|, |C_t|, sum_{A_t} indeg (0 if gather eliminated), sum_{C_t} outdeg (0 if
  * FrontierActivate eliminated). *rows = supersteps recorded (<= max_rows). */
 gr_status gr_fetch_frontier_trace(gr_graph *g, uint64_t *host_dst, uint64_t max_rows, uint64_t *rows);
+
+/* Detail columns of the last run's trace (it must have run with trace_detail = 1;
+ * else GR_ESTATE): 2 uint64 per superstep t — active_shards (shards
+ * [v_lo, v_hi) of gr_shard_info holding a vertex of A_t: what frontier skipping
+ * moves, §5.2) and S_t (distinct sources read by the gather of A_t;
+ * 0 when the gather is eliminated). *rows = supersteps recorded (<= max_rows). */
+gr_status gr_fetch_frontier_trace_detail(gr_graph *g, uint64_t *host_dst, uint64_t max_rows, uint64_t *rows);
 
 /* ---- run-time GAS programs (§4.1, Fig. 6) ----
  * Compile a user program at run time and register it. `source` is CUDA C++

@@ -51,6 +51,9 @@ def lib():
         L.or_run.argtypes = [ctypes.c_void_p, ctypes.c_int, ctypes.c_uint32, ctypes.c_uint32,
                              ctypes.c_double, ctypes.c_double, ctypes.c_void_p, ctypes.POINTER(ctypes.c_uint64),
                              ctypes.c_uint64, ctypes.POINTER(ctypes.c_uint64)]
+        L.or_run_detail.restype = ctypes.c_int64
+        L.or_run_detail.argtypes = L.or_run.argtypes + [ctypes.POINTER(ctypes.c_uint64), ctypes.c_uint32,
+                                                        ctypes.POINTER(ctypes.c_uint64)]
         _lib = L
     return _lib
 
@@ -95,6 +98,30 @@ class OracleGraph:
         if algo == "pagerank_delta":
             vals = vals.view(np.float32)
         return vals, tr[: min(rows.value, trace_cap)].copy(), int(it)
+
+    def run_detail(self, algo: str, shard_bounds=None, source: int = 0, max_iters: int = 0,
+                   damping: float = 0.85, trace_cap: int = 1 << 16, tolerance: float = 1e-4):
+        """Like run(), plus detail[rows, 2] = (active_shards, S_t) per superstep."""
+        a = ALGOS[algo]
+        if algo == "pagerank" and max_iters == 0:
+            max_iters = 30
+        vals = np.empty(self.n, np.float64 if algo == "pagerank" else np.uint32)
+        tr = np.zeros((trace_cap, 4), np.uint64)
+        det = np.zeros((trace_cap, 2), np.uint64)
+        rows = ctypes.c_uint64(0)
+        P64 = ctypes.POINTER(ctypes.c_uint64)
+        b = None if shard_bounds is None else np.ascontiguousarray(shard_bounds, dtype=np.uint64)
+        nb = 0 if b is None else len(b) - 1
+        it = lib().or_run_detail(self._h, a, source, max_iters, damping, tolerance,
+                                 vals.ctypes.data_as(ctypes.c_void_p), tr.ctypes.data_as(P64), trace_cap,
+                                 ctypes.byref(rows), None if b is None else b.ctypes.data_as(P64), nb,
+                                 det.ctypes.data_as(P64))
+        if it < 0:
+            raise ValueError(f"or_run_detail failed rc={it}")
+        r = min(rows.value, trace_cap)
+        if algo == "pagerank_delta":
+            vals = vals.view(np.float32)
+        return vals, tr[:r].copy(), det[:r].copy(), int(it)
 
     def close(self):
         if getattr(self, "_h", None):

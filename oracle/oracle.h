@@ -57,6 +57,17 @@ int64_t or_run(or_graph *g, int algo, uint32_t source, uint32_t max_iters, doubl
                double tolerance, void *values_out, uint64_t *trace_out, uint64_t trace_cap,
                uint64_t *rows_out);
 
+/* or_run plus the detail columns of the frontier trace:
+ * detail_out (nullable): 2 uint64 per superstep t —
+ *   active_shards = number of shards [bounds[s], bounds[s+1]) holding a vertex of
+ *                   A_t (frontier skipping, §5.2; 0 without bounds),
+ *   S_t           = number of distinct sources read by the gather of A_t (0 when
+ *                   the gather is eliminated). */
+int64_t or_run_detail(or_graph *g, int algo, uint32_t source, uint32_t max_iters, double damping,
+                      double tolerance, void *values_out, uint64_t *trace_out, uint64_t trace_cap,
+                      uint64_t *rows_out, const uint64_t *shard_bounds, uint32_t num_shards,
+                      uint64_t *detail_out);
+
 #ifdef __cplusplus
 }
 #endif

@@ -22,9 +22,10 @@ _lib = None
 
 GR_OK, GR_EINVAL, GR_ENOMEM, GR_ECUDA, GR_ENCCL, GR_EUNSUPPORTED, GR_ESTATE = range(7)
 STATUS_NAMES = ["GR_OK", "GR_EINVAL", "GR_ENOMEM", "GR_ECUDA", "GR_ENCCL", "GR_EUNSUPPORTED", "GR_ESTATE"]
-GR_FMT_COO, GR_FMT_CSR = 0, 1
+GR_FMT_COO, GR_FMT_CSR, GR_FMT_SORTED = 0, 1, 2
 ALGOS = {"bfs": 0, "sssp": 1, "pagerank": 2, "cc": 3, "custom": 4, "pagerank_delta": 5}
 FLOAT_ALGOS = ("pagerank", "pagerank_delta")
+TRANSPORTS = {"nccl": 0, "shm": 1}
 MODES = {"auto": 0, "resident": 1, "streamed": 2}
 LOOPS = {"auto": 0, "host": 1, "device": 2, "persistent": 3}
 BUILDS = {"auto": 0, "host": 1, "device": 2}
@@ -35,6 +36,7 @@ EXPORTS = [
     "gr_get_unique_id", "gr_graph_load", "gr_graph_load_file", "gr_run", "gr_fetch_vertex_values", "gr_fetch_frontier_trace",
     "gr_graph_info_get", "gr_shard_info", "gr_graph_free", "gr_last_error", "gr_plan_intervals",
     "gr_host_build", "gr_host_csc", "gr_host_csr", "gr_host_shards", "gr_host_free", "gr_program_compile",
+    "gr_fetch_frontier_trace_detail",
 ]
 
 
@@ -47,21 +49,24 @@ class GrError(RuntimeError):
 class gr_edges(ctypes.Structure):
     _fields_ = [("fmt", ctypes.c_int32), ("num_vertices", ctypes.c_uint64), ("num_edges", ctypes.c_uint64),
                 ("src", ctypes.c_void_p), ("dst", ctypes.c_void_p), ("row_offsets", ctypes.c_void_p),
-                ("col_idx", ctypes.c_void_p), ("weights", ctypes.c_void_p)]
+                ("col_idx", ctypes.c_void_p), ("weights", ctypes.c_void_p), ("in_offsets", ctypes.c_void_p),
+                ("in_idx", ctypes.c_void_p), ("out_degree", ctypes.c_void_p)]
 
 
 class gr_load_opts(ctypes.Structure):
     _fields_ = [("shard_edges", ctypes.c_uint64), ("device_budget_bytes", ctypes.c_uint64),
                 ("mode", ctypes.c_int32), ("device", ctypes.c_int32), ("rank", ctypes.c_int32),
                 ("world", ctypes.c_int32), ("nccl_unique_id", ctypes.c_void_p), ("host_threads", ctypes.c_int32),
-                ("sim_ranks", ctypes.c_int32), ("build", ctypes.c_int32)]
+                ("sim_ranks", ctypes.c_int32), ("build", ctypes.c_int32),
+                ("transport", ctypes.c_int32), ("borrow", ctypes.c_int32)]
 
 
 class gr_run_opts(ctypes.Structure):
     _fields_ = [("algo", ctypes.c_int32), ("source", ctypes.c_uint32), ("max_iters", ctypes.c_uint32),
                 ("damping", ctypes.c_float), ("custom_id", ctypes.c_int32), ("loop", ctypes.c_int32),
                 ("stream", ctypes.c_void_p), ("profile", ctypes.c_int32), ("direction", ctypes.c_int32),
-                ("pull_div", ctypes.c_uint32), ("tolerance", ctypes.c_float), ("zero_copy", ctypes.c_int32)]
+                ("pull_div", ctypes.c_uint32), ("tolerance", ctypes.c_float), ("zero_copy", ctypes.c_int32),
+                ("trace_detail", ctypes.c_int32)]
 
 
 class gr_run_stats(ctypes.Structure):
@@ -114,6 +119,7 @@ def lib():
         "gr_run": (i32, [vp, ctypes.POINTER(gr_run_opts), ctypes.POINTER(gr_run_stats)]),
         "gr_fetch_vertex_values": (i32, [vp, vp, u64]),
         "gr_fetch_frontier_trace": (i32, [vp, u64p, u64, u64p]),
+        "gr_fetch_frontier_trace_detail": (i32, [vp, u64p, u64, u64p]),
         "gr_graph_info_get": (i32, [vp, ctypes.POINTER(gr_graph_info)]),
         "gr_program_compile": (i32, [ctypes.c_char_p, ctypes.c_char_p, ctypes.POINTER(i32)]),
         "gr_shard_info": (i32, [vp, u32, ctypes.POINTER(gr_shard_desc)]),
@@ -168,7 +174,7 @@ def _edges(n, src=None, dst=None, weights=None, row_offsets=None, col_idx=None):
 
 
 def _load_opts(shard_edges=0, device_budget_bytes=0, mode="auto", device=0, rank=0, world=1,
-               nccl_unique_id=None, host_threads=0, sim_ranks=0, build="auto"):
+               nccl_unique_id=None, host_threads=0, sim_ranks=0, build="auto", transport="nccl", borrow=False):
     o = gr_load_opts()
     o.shard_edges, o.device_budget_bytes = int(shard_edges), int(device_budget_bytes)
     o.mode = MODES[mode] if isinstance(mode, str) else int(mode)
@@ -179,6 +185,8 @@ def _load_opts(shard_edges=0, device_budget_bytes=0, mode="auto", device=0, rank
         o.nccl_unique_id = ctypes.cast(uid, ctypes.c_void_p)
     o.host_threads, o.sim_ranks = int(host_threads), int(sim_ranks)
     o.build = BUILDS[build] if isinstance(build, str) else int(build)
+    o.transport = TRANSPORTS[transport] if isinstance(transport, str) else int(transport)
+    o.borrow = 1 if borrow else 0
     return o, uid
 
 
@@ -229,6 +237,31 @@ def write_graph_file(path, n, src=None, dst=None, weights=None, row_offsets=None
             a.tofile(f)
 
 
+def gr_graph_load_sorted(n, m, in_offsets=None, in_idx=None, row_offsets=None, col_idx=None, out_degree=None,
+                         **opts):
+    """GR_FMT_SORTED: load the already-sorted layout (in-CSC and/or out-CSR). With
+    borrow=True the adjacency arrays are used in place: they must hold m + 4
+    entries and outlive the handle (GraphReduce.from_sorted keeps them)."""
+    e = gr_edges()
+    e.fmt, e.num_vertices, e.num_edges = GR_FMT_SORTED, int(n), int(m)
+    keep = []
+    for name, arr, dt in (("in_offsets", in_offsets, np.uint64), ("in_idx", in_idx, np.uint32),
+                          ("row_offsets", row_offsets, np.uint64), ("col_idx", col_idx, np.uint32),
+                          ("out_degree", out_degree, np.uint32)):
+        if arr is None:
+            continue
+        if arr.dtype != dt or not arr.flags["C_CONTIGUOUS"]:
+            if opts.get("borrow"):
+                raise ValueError(f"{name}: borrowed arrays must be C-contiguous {np.dtype(dt).name}")
+            arr = np.ascontiguousarray(arr, dtype=dt)
+        keep.append(arr)
+        setattr(e, name, arr.ctypes.data)
+    o, uid = _load_opts(**opts)
+    h = ctypes.c_void_p()
+    _check(lib().gr_graph_load(ctypes.byref(e), ctypes.byref(o), ctypes.byref(h)))
+    return h
+
+
 def gr_graph_load_file(path, **opts):
     """gr_graph_load from a canonical graph file (memory-mapped by the library)."""
     o, uid = _load_opts(**opts)
@@ -239,7 +272,7 @@ def gr_graph_load_file(path, **opts):
 
 
 def gr_run(h, algo, source=0, max_iters=0, damping=0.85, custom_id=0, loop="auto", stream=None,
-           profile=False, direction="auto", pull_div=0, zero_copy=0, tolerance=1e-4) -> dict:
+           profile=False, direction="auto", pull_div=0, zero_copy=0, tolerance=1e-4, trace_detail=False) -> dict:
     o = gr_run_opts()
     o.algo = ALGOS[algo] if isinstance(algo, str) else int(algo)
     o.source, o.max_iters, o.damping, o.custom_id = int(source), int(max_iters), float(damping), int(custom_id)
@@ -250,6 +283,7 @@ def gr_run(h, algo, source=0, max_iters=0, damping=0.85, custom_id=0, loop="auto
     o.pull_div = int(pull_div)
     o.zero_copy = int(zero_copy)
     o.tolerance = float(tolerance)
+    o.trace_detail = 1 if trace_detail else 0
     st = gr_run_stats()
     _check(lib().gr_run(h, ctypes.byref(o), ctypes.byref(st)))
     return st.as_dict()
@@ -282,6 +316,15 @@ def gr_fetch_frontier_trace(h, max_rows: int = 1 << 20) -> np.ndarray:
     rows = ctypes.c_uint64(0)
     _check(lib().gr_fetch_frontier_trace(h, buf.ctypes.data_as(ctypes.POINTER(ctypes.c_uint64)), max_rows,
                                          ctypes.byref(rows)))
+    return buf[: rows.value].copy()
+
+
+def gr_fetch_frontier_trace_detail(h, max_rows: int = 1 << 20) -> np.ndarray:
+    """(active_shards, S_t) per superstep of the last run (run with trace_detail=True)."""
+    buf = np.zeros((max_rows, 2), np.uint64)
+    rows = ctypes.c_uint64(0)
+    _check(lib().gr_fetch_frontier_trace_detail(h, buf.ctypes.data_as(ctypes.POINTER(ctypes.c_uint64)), max_rows,
+                                                ctypes.byref(rows)))
     return buf[: rows.value].copy()
 
 
@@ -350,6 +393,15 @@ class GraphReduce:
         self.h = gr_graph_load(n, src, dst, weights, **opts)
 
     @classmethod
+    def from_sorted(cls, n, m, **kw):
+        """GR_FMT_SORTED load (gr_graph_load_sorted); borrowed arrays are kept alive here."""
+        self = cls.__new__(cls)
+        self._borrowed = [v for v in kw.values() if isinstance(v, np.ndarray)]
+        self.h = gr_graph_load_sorted(n, m, **kw)
+        self.n = int(n)
+        return self
+
+    @classmethod
     def from_file(cls, path, **opts):
         self = cls.__new__(cls)
         self.h = gr_graph_load_file(path, **opts)
@@ -365,6 +417,9 @@ class GraphReduce:
 
     def trace(self):
         return gr_fetch_frontier_trace(self.h)
+
+    def trace_detail(self):
+        return gr_fetch_frontier_trace_detail(self.h)
 
     def info(self):
         return gr_graph_info_get(self.h)

@@ -61,6 +61,8 @@ gr_status gr_graph_load(const gr_edges *edges, const gr_load_opts *opts_in, gr_g
   if (opts.rank < 0 || opts.rank >= opts.world) return fail(GR_EINVAL, "rank %d outside [0, %d)", opts.rank, opts.world);
   if (opts.world > 1 && opts.mode == GR_MODE_STREAMED)
     return fail(GR_EUNSUPPORTED, "streamed mode is single-rank (partition over GPUs to fit HBM instead)");
+  if (opts.transport != GR_TRANSPORT_NCCL && opts.transport != GR_TRANSPORT_SHM)
+    return fail(GR_EINVAL, "bad transport %d", opts.transport);
   if (opts.world > 1 && !opts.nccl_unique_id)
     return fail(GR_EINVAL, "world > 1 needs nccl_unique_id (simulated ranks: any 128-byte group key)");
   int ndev = 0;
@@ -92,7 +94,21 @@ gr_status gr_graph_load(const gr_edges *edges, const gr_load_opts *opts_in, gr_g
     delete g;
     return fail(GR_EUNSUPPORTED, "device build needs a resident single-rank COO graph that fits the device budget");
   }
-  if (!dev_build) {
+  if (edges->fmt == GR_FMT_SORTED) {
+    if (opts.world > 1) {
+      delete g;
+      return fail(GR_EUNSUPPORTED, "GR_FMT_SORTED inputs are single-rank");
+    }
+    s = build_host_sorted(edges, opts.shard_edges, opts.borrow != 0, opts.host_threads, &g->H, &err);
+    if (s == GR_OK && (!g->H.has_in || !g->H.has_out) && opts.mode != GR_MODE_STREAMED) {
+      s = GR_EUNSUPPORTED;
+      err = "a one-directional layout (only in-CSC or only out-CSR) must be loaded streamed";
+    }
+    if (s != GR_OK) {
+      delete g;
+      return fail(s, "%s", err.c_str());
+    }
+  } else if (!dev_build) {
     s = build_host_graph(edges, opts.shard_edges, opts.world, opts.rank, opts.host_threads, &g->H, &err);
     if (s != GR_OK) {
       delete g;
@@ -133,7 +149,8 @@ gr_status gr_graph_load(const gr_edges *edges, const gr_load_opts *opts_in, gr_g
   if (s == GR_OK && g->mode == GR_MODE_STREAMED) s = stream_setup(g, budget);
   if (s == GR_OK && opts.world > 1) {
     std::string cerr;
-    s = comm_create(opts.world, opts.rank, sim, opts.nccl_unique_id, g->device, &g->comm, &cerr);
+    const int transport = sim ? kTransportSim : opts.transport == GR_TRANSPORT_SHM ? kTransportShm : kTransportNccl;
+    s = comm_create(opts.world, opts.rank, transport, opts.nccl_unique_id, g->device, &g->comm, &cerr);
     if (s != GR_OK) fail(s, "%s", cerr.c_str());
     if (s == GR_OK) s = part_setup(g);
   }
@@ -168,6 +185,13 @@ gr_status gr_fetch_frontier_trace(gr_graph *g, uint64_t *host_dst, uint64_t max_
   if (!g) return fail(GR_EINVAL, "graph is NULL");
   cudaSetDevice(g->device);
   return fetch_trace(g, host_dst, max_rows, rows);
+}
+
+gr_status gr_fetch_frontier_trace_detail(gr_graph *g, uint64_t *host_dst, uint64_t max_rows, uint64_t *rows) {
+  clear_error();
+  if (!g) return fail(GR_EINVAL, "graph is NULL");
+  cudaSetDevice(g->device);
+  return fetch_trace_detail(g, host_dst, max_rows, rows);
 }
 
 gr_status gr_program_compile(const char *source, const char *struct_name, int32_t *custom_id) {

@@ -8,6 +8,9 @@
 //              grouped ncclBroadcast from every root).
 //   SimComm  : G "ranks" as host threads sharing ONE device (tests on a 1-GPU
 //              box): the same protocol with device-to-device copies.
+//   ShmComm  : one process per rank on one node (ranks may share a GPU): POSIX
+//              shared memory for the host collectives, real cross-process
+//              cudaIpc mappings for the device data (mailboxes, shared buffers).
 #pragma once
 #include <cuda_runtime.h>
 
@@ -47,8 +50,11 @@ struct Comm {
 };
 
 // Create the communicator for a loaded partition. world <= 1 returns nullptr.
-// sim: in-process simulated group keyed by the 128-byte id.
-gr_status comm_create(int world, int rank, bool sim, const void *id128, int device, Comm **out,
+// transport: kTransportNccl (one process per GPU), kTransportSim (in-process
+// simulated group keyed by the 128-byte id), kTransportShm (one process per
+// rank on one node, POSIX shared memory + cudaIpc; ranks may share a GPU).
+constexpr int kTransportNccl = 0, kTransportShm = 1, kTransportSim = 2;
+gr_status comm_create(int world, int rank, int transport, const void *id128, int device, Comm **out,
                       std::string *err);
 
 }  // namespace gr

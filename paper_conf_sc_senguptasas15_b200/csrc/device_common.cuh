@@ -57,6 +57,7 @@ struct Ctl {
   uint32_t dirty[2];      // changed-bitmap b holds bits of an earlier pull and must be cleared
   uint32_t tot_pull;      // supersteps that activated by pull
   uint32_t dense;         // superstep `iter` gathers densely (previous activation was by pull)
+  uint32_t gate;          // ... reading only the changed sources' values (Selective<> programs)
   uint32_t prd_r0;        // ProgPRDelta constants (Ctx)
   uint32_t push;          // fused push supersteps (gr/program.cuh kPushFused): one phase per superstep
   unsigned long long prd_base, prd_dq;
@@ -85,7 +86,7 @@ __device__ __forceinline__ unsigned long long block_sum_u64(unsigned long long x
 struct View {
   uint32_t stop, t, epoch_base, implicit0, no_hub_c, source, prof;
   uint32_t cntA[2], cntK[2], cntH[2], cntC, cntCH, cntKC;
-  uint32_t pull_div, pull_pending, dirty[2], dense, push;
+  uint32_t pull_div, pull_pending, dirty[2], dense, push, gate;
   float damping;
   unsigned long long prd_base, prd_dq;
   double prd_thr;
@@ -103,7 +104,7 @@ __device__ __forceinline__ void load_view(const Ctl *c, View &v) {
     const uint32_t h0 = vc->cnt_H[0], h1 = vc->cnt_H[1], ch = vc->cnt_CH;
     const uint32_t pd = vc->pull_div, pp = vc->pull_pending, d0 = vc->dirty[0], d1 = vc->dirty[1], dn = vc->dense;
     v.cntH[0] = h0; v.cntH[1] = h1; v.cntCH = ch;
-    v.pull_div = pd; v.pull_pending = pp; v.dirty[0] = d0; v.dirty[1] = d1; v.dense = dn; v.push = vc->push;
+    v.pull_div = pd; v.pull_pending = pp; v.dirty[0] = d0; v.dirty[1] = d1; v.dense = dn; v.push = vc->push; v.gate = vc->gate;
     v.prd_base = vc->prd_base; v.prd_dq = vc->prd_dq; v.prd_thr = vc->prd_thr;
     v.cntA[0] = a0; v.cntA[1] = a1; v.cntK[0] = k0; v.cntK[1] = k1;
     v.stop = st; v.t = t; v.epoch_base = eb; v.implicit0 = im; v.no_hub_c = nh;
@@ -154,7 +155,6 @@ template <class OffT> struct Part {
   uint32_t *hub_act;      // per static hub: some chunk saw a marked source (dense gathers)
   const uint32_t *s_hubs, *s_chk_h, *s_chk_c;  // static in-hub list and its chunks (dense gathers)
   const ulonglong2 *prd_div;  // ProgPRDelta divisor table (Ctx::prd_div), or nullptr
-  uint32_t gate;          // dense supersteps of Selective<> programs read only the changed sources' values
   uint32_t *estate;       // [m_in] edge states in CSC order (programs with kHasScatter)
   const uint32_t *out_eid;// [m_in] CSC position of every activation-CSR edge (kHasScatter)
   // dense (pull) supersteps of kDstFreeGather programs: edge-segmented tiles over the

@@ -563,6 +563,90 @@ static gr_status get_while_graph(gr_graph *g, int key, cudaGraphExec_t *out, uin
   return GR_OK;
 }
 
+// ---- detail columns of the frontier trace (gr_run_opts.trace_detail):
+// before superstep t's gather, mark the shard of every vertex of A_t and every
+// source its gather reads, then count both sets. A_t is the implicit owned range
+// (superstep 0 of kInitAll programs), the vertices with a marked in-neighbour
+// (dense supersteps), or the A lists (listA + listH). Diagnostic: host loop only.
+template <class OffT>
+static __global__ void k_detail_mark(const __grid_constant__ Part<OffT> P, int has_gather, const uint64_t *sb,
+                                     uint32_t nsb, uint32_t *src_bits, uint32_t *shard_bits) {
+  __shared__ View V;
+  load_view(P.ctl, V);
+  if (V.stop) return;
+  const uint32_t t = V.t, slot = t & 1u;
+  const bool implicit = V.dense || (V.implicit0 && t == 0);
+  const uint32_t *bits = P.cbits[slot ^ 1u];
+  const uint64_t nA = V.cntA[slot], total = implicit ? (uint64_t)P.own_n : nA + V.cntH[slot];
+  for (uint64_t i = blockIdx.x * (uint64_t)blockDim.x + threadIdx.x; i < total; i += (uint64_t)gridDim.x * blockDim.x) {
+    const uint32_t v = implicit ? P.own_lo + (uint32_t)i : (i < nA ? P.listA[slot][i] : P.listH[slot][i - nA]);
+    const uint32_t lv = v - P.own_lo;
+    const uint64_t b = (uint64_t)P.in_off[lv], e = (uint64_t)P.in_off[lv + 1];
+    if (V.dense) {
+      bool act = false;
+      for (uint64_t k = b; k < e && !act; k++) act = test_bit_cg(bits, P.in_src[k]);
+      if (!act) continue;
+    }
+    uint32_t lo = 0, hi = nsb;  // shard: last s with sb[s] <= v
+    while (hi - lo > 1) {
+      const uint32_t mid = (lo + hi) >> 1;
+      if (sb[mid] <= v) lo = mid;
+      else hi = mid;
+    }
+    atomicOr(shard_bits + (lo >> 5), 1u << (lo & 31));
+    if (has_gather)
+      for (uint64_t k = b; k < e; k++) {
+        const uint32_t u = P.in_src[k];
+        atomicOr(src_bits + (u >> 5), 1u << (u & 31));
+      }
+  }
+}
+
+static __global__ void k_detail_count(const Ctl *ctl, uint32_t *src_bits, uint64_t src_words, uint32_t *shard_bits,
+                                      uint64_t shard_words, unsigned long long *det, uint32_t cap) {
+  if (ctl->stop) return;
+  unsigned long long a = 0, b = 0;
+  for (uint64_t i = blockIdx.x * (uint64_t)blockDim.x + threadIdx.x; i < src_words; i += (uint64_t)gridDim.x * blockDim.x) {
+    b += __popc(src_bits[i]);
+    src_bits[i] = 0;
+  }
+  for (uint64_t i = blockIdx.x * (uint64_t)blockDim.x + threadIdx.x; i < shard_words; i += (uint64_t)gridDim.x * blockDim.x) {
+    a += __popc(shard_bits[i]);
+    shard_bits[i] = 0;
+  }
+  const uint32_t t = ctl->iter;
+  if (t >= cap) return;
+  if (a) atomicAdd(det + 2ull * t, a);
+  if (b) atomicAdd(det + 2ull * t + 1, b);
+}
+
+static gr_status detail_setup(gr_graph *g, cudaStream_t s) {
+  gr_status st;
+  const uint64_t words = (g->H.n + 31) / 32 + 1, P = g->H.num_shards();
+  if (!g->trace_det) {
+    if ((st = dev_alloc(g, (void **)&g->trace_det, 16ull * g->trace_cap)) != GR_OK) return st;
+    if ((st = dev_alloc(g, (void **)&g->det_src_bits, 4 * words)) != GR_OK) return st;
+    if ((st = dev_alloc(g, (void **)&g->det_shard_bits, 4 * (P / 32 + 1))) != GR_OK) return st;
+    if ((st = dev_alloc(g, (void **)&g->d_shard_bounds, 8 * (P + 1))) != GR_OK) return st;
+    CK(cudaMemcpy(g->d_shard_bounds, g->H.bounds.data(), 8 * (P + 1), cudaMemcpyHostToDevice));
+    CK(cudaMemset(g->det_src_bits, 0, 4 * words));
+    CK(cudaMemset(g->det_shard_bits, 0, 4 * (P / 32 + 1)));
+  }
+  CK(cudaMemsetAsync(g->trace_det, 0, 16ull * g->trace_cap, s));
+  return GR_OK;
+}
+
+template <class OffT>
+static gr_status detail_superstep(gr_graph *g, const Part<OffT> &P, bool has_gather, cudaStream_t s) {
+  const uint64_t words = (g->H.n + 31) / 32 + 1, np = g->H.num_shards();
+  k_detail_mark<OffT><<<g->num_sms * 8, 256, 0, s>>>(P, has_gather ? 1 : 0, g->d_shard_bounds, (uint32_t)np,
+                                                    g->det_src_bits, g->det_shard_bits);
+  k_detail_count<<<g->num_sms * 2, 256, 0, s>>>(g->ctl, g->det_src_bits, words, g->det_shard_bits, np / 32 + 1,
+                                                g->trace_det, g->trace_cap);
+  CK(cudaGetLastError());
+  return GR_OK;
+}
+
 // CTAs per SM of the persistent frontier loop (built-in and run-time programs
 // alike): 4; 2 when the owned range has fewer vertices than 4 CTAs per SM have
 // threads (cheaper grid barriers: cfg1 BFS 0.392 -> 0.372 ms; SSSP / CC there
@@ -597,7 +681,7 @@ static gr_status run_frontier(gr_graph *g, const gr_run_opts *o, cudaStream_t s,
   bool push = false;
   if constexpr (PushFused<Prog>::value) {
     push = Prog::kInit == kInitSourceChanged && !g->comm && g->mode == GR_MODE_RESIDENT &&
-           o->direction == GR_DIR_FUSED;
+           o->direction == GR_DIR_FUSED && !o->trace_detail;
     if (const char *e = getenv("GR_PUSH_FUSED")) push = push && atoi(e) != 0;
     if (push) {
       gr_status ps = push_setup(g, Prog::kUsesWeights);
@@ -678,8 +762,13 @@ static gr_status run_frontier(gr_graph *g, const gr_run_opts *o, cudaStream_t s,
   k_init_frontier<Prog, OffT><<<1, kBlock, 0, s>>>(P, o->source, g->n_static_hubs, g->n_static_chunks);
   launches++;
   CK(cudaGetLastError());
-  const bool persistent = (o->loop == GR_LOOP_AUTO || o->loop == GR_LOOP_PERSISTENT) && g->coop;
-  const bool use_graph = !persistent && (o->loop == GR_LOOP_DEVICE || o->loop == GR_LOOP_AUTO);
+  const bool detail = o->trace_detail != 0;  // diagnostic: host loop with the detail kernels
+  if (detail) {
+    gr_status ds = detail_setup(g, s);
+    if (ds != GR_OK) return ds;
+  }
+  const bool persistent = !detail && (o->loop == GR_LOOP_AUTO || o->loop == GR_LOOP_PERSISTENT) && g->coop;
+  const bool use_graph = !detail && !persistent && (o->loop == GR_LOOP_DEVICE || o->loop == GR_LOOP_AUTO);
   if (persistent) {
     int bps = 0;
     const void *kf = dseg ? (const void *)k_persistent_ds<Prog, OffT> : (const void *)k_persistent<Prog, OffT>;
@@ -701,6 +790,10 @@ static gr_status run_frontier(gr_graph *g, const gr_run_opts *o, cudaStream_t s,
     launches += per * std::max<uint32_t>(g->h_ctl->iter, 1);
   } else {
     for (;;) {
+      if (detail) {
+        gr_status ds = detail_superstep<OffT>(g, P, Prog::kHasGather, s);
+        if (ds != GR_OK) return ds;
+      }
       launch_body<Prog, OffT>(g, s, 0, 0, &launches, push);
       CK(cudaGetLastError());
       CK(cudaMemcpyAsync(g->h_ctl, g->ctl, sizeof(Ctl), cudaMemcpyDeviceToHost, s));
@@ -909,22 +1002,10 @@ using SegKernel = void (*)(const PrArgs<OffT>, const uint32_t *, const uint32_t 
                            uint32_t, uint32_t);
 template <class OffT>
 using SegLoopKernel = void (*)(const PrArgs<OffT>, const PrLoop);
-template <class OffT> static SegLoopKernel<OffT> seg_loop_kernel(int var) {
-  static const SegLoopKernel<OffT> tab[16] = {
-      k_pr_seg_loop<OffT, 0>,  k_pr_seg_loop<OffT, 1>,  k_pr_seg_loop<OffT, 2>,  k_pr_seg_loop<OffT, 3>,
-      k_pr_seg_loop<OffT, 4>,  k_pr_seg_loop<OffT, 5>,  k_pr_seg_loop<OffT, 6>,  k_pr_seg_loop<OffT, 7>,
-      k_pr_seg_loop<OffT, 8>,  k_pr_seg_loop<OffT, 9>,  k_pr_seg_loop<OffT, 10>, k_pr_seg_loop<OffT, 11>,
-      k_pr_seg_loop<OffT, 12>, k_pr_seg_loop<OffT, 13>, k_pr_seg_loop<OffT, 14>, k_pr_seg_loop<OffT, 15>};
-  return tab[var & 15];
-}
-
-template <class OffT> static SegKernel<OffT> seg_kernel(int var) {
-  static const SegKernel<OffT> tab[16] = {
-      k_pr_seg<OffT, 0>,  k_pr_seg<OffT, 1>,  k_pr_seg<OffT, 2>,  k_pr_seg<OffT, 3>,  k_pr_seg<OffT, 4>,  k_pr_seg<OffT, 5>,
-      k_pr_seg<OffT, 6>,  k_pr_seg<OffT, 7>,  k_pr_seg<OffT, 8>,  k_pr_seg<OffT, 9>,  k_pr_seg<OffT, 10>, k_pr_seg<OffT, 11>,
-      k_pr_seg<OffT, 12>, k_pr_seg<OffT, 13>, k_pr_seg<OffT, 14>, k_pr_seg<OffT, 15>};
-  return tab[var & 15];
-}
+// The seg kernels are instantiated for the default variant bits only (the other
+// combinations were measured in round 1 and are not built: profiles/README.md)
+template <class OffT> static SegLoopKernel<OffT> seg_loop_kernel(int) { return k_pr_seg_loop<OffT, kSegDefaultVar>; }
+template <class OffT> static SegKernel<OffT> seg_kernel(int) { return k_pr_seg<OffT, kSegDefaultVar>; }
 
 // Source-blocked layout for k_pr_bseg_loop (once per graph):
 // stable radix sort of the CSC edges by source block (CSC order kept inside a
@@ -1053,29 +1134,19 @@ template <class OffT> static gr_status pr_hot_setup(gr_graph *g) {
   uint32_t S = (uint32_t)std::max<uint64_t>(1024, (block_mb << 20) / 4 / 32 * 32);
   if (const char *bv = getenv("GR_PR_BLOCK_V")) S = (uint32_t)std::max<uint64_t>(32, strtoull(bv, nullptr, 10));  // tests
   const bool bseg_ok = seg_ok && !g->comm && H.n > S;
-  // kernel variant (GR_PR_KERNEL = block | warp | warphot | range | rangehot | pipe | seg | bseg; default seg,
-  // bseg when the contribution array is larger than one L2 block)
+  // kernel (GR_PR_KERNEL = block | warp | warphot | seg | bseg): seg by default, bseg when the
+  // contribution array is larger than one L2 block; warphot (hot table, merge-path warp tiles)
+  // when the seg layout's 32-bit item indices would overflow, warp for ranks with < 1M
+  // in-edges, block (CTA merge-path tiles) when no shared-memory table fits
   g->pr_kernel = bseg_ok ? 8 : seg_ok ? 7 : 3;
   if (const char *k = getenv("GR_PR_KERNEL")) {
     const std::string v(k);
-    g->pr_kernel = v == "block" || v == "blockhot" ? 0 : v == "warp" ? 2 : v == "warphot" ? 3 : v == "range" ? 4
-                 : v == "pipe" ? 6 : v == "seg" ? 7 : v == "bseg" ? 8 : 5;
+    g->pr_kernel = v == "block" ? 0 : v == "warp" ? 2 : v == "warphot" ? 3 : v == "seg" ? 7 : v == "bseg" ? 8 : 7;
   }
   if (g->pr_kernel == 8 && !seg_ok) g->pr_kernel = hot_ok ? 3 : 2;
-  if ((g->pr_kernel == 3 || g->pr_kernel == 5) && !hot_ok) g->pr_kernel -= 1;
-  if (g->pr_kernel == 6 && !hot_ok) g->pr_kernel = 2;
+  if (g->pr_kernel == 3 && !hot_ok) g->pr_kernel = 2;
   if (g->pr_kernel == 7 && !seg_ok) g->pr_kernel = hot_ok ? 3 : 2;
-  if (g->pr_kernel == 4) {
-    g->hot_smem = 32 * sizeof(PrWarpSmem);
-    CK(cudaFuncSetAttribute(k_pr_warp_range<OffT, false>, cudaFuncAttributeMaxDynamicSharedMemorySize,
-                            (int)g->hot_smem));
-    int bps = 0;
-    CK(cudaOccupancyMaxActiveBlocksPerMultiprocessor(&bps, k_pr_warp_range<OffT, false>, 1024, g->hot_smem));
-    g->hot_grid = (uint32_t)(g->num_sms * std::max(bps, 1));
-    return GR_OK;
-  }
-  if (g->pr_kernel != 3 && g->pr_kernel != 5 && g->pr_kernel != 6 && g->pr_kernel != 7 && g->pr_kernel != 8)
-    return GR_OK;
+  if (g->pr_kernel != 3 && g->pr_kernel != 7 && g->pr_kernel != 8) return GR_OK;
   // the seg kernels stage nothing in shared memory: their table can be ~2x larger
   uint64_t K = g->pr_kernel >= 7 ? kSegHotK : kHotK;
   if (const char *hk = getenv("GR_PR_HOTK")) K = std::max<uint64_t>(4, std::min<uint64_t>(strtoull(hk, nullptr, 10), 57344));
@@ -1106,7 +1177,6 @@ template <class OffT> static gr_status pr_hot_setup(gr_graph *g) {
     if ((s = pr_seg_setup<OffT>(g)) != GR_OK) return s;
     g->hot_cta = 1024;
     g->seg_var = kSegDefaultVar;
-    if (const char *sv = getenv("GR_PR_SEG_VAR")) g->seg_var = atoi(sv) & 15;
     // the table plus (kSegBuf) 32 floats per warp; what is left of the SM's 256 KB is L1
     g->hot_smem = 4ull * (g->hot_k + 4) + ((g->seg_var & kSegBuf) ? 4ull * 32 * (g->hot_cta / 32) : 0);
     CK(cudaFuncSetAttribute(seg_kernel<OffT>(g->seg_var), cudaFuncAttributeMaxDynamicSharedMemorySize,
@@ -1136,22 +1206,11 @@ template <class OffT> static gr_status pr_hot_setup(gr_graph *g) {
       CK(cudaGetLastError());
       CK(cudaStreamSynchronize(g->stream));
     }
-  } else if (g->pr_kernel == 5) {
-    g->hot_smem = 4ull * g->hot_k + 32 * sizeof(PrWarpSmem);
-    CK(cudaFuncSetAttribute(k_pr_warp_range<OffT, true>, cudaFuncAttributeMaxDynamicSharedMemorySize,
-                            (int)g->hot_smem));
-    CK(cudaOccupancyMaxActiveBlocksPerMultiprocessor(&bps, k_pr_warp_range<OffT, true>, 1024, g->hot_smem));
   } else {
     g->hot_cta = 1024;
-    if (const char *ct = getenv("GR_PR_CTA")) g->hot_cta = std::max(64, std::min(1024, atoi(ct))) & ~31;
     g->hot_smem = 4ull * g->hot_k + (g->hot_cta / 32) * sizeof(PrWarpSmem);
-    if (g->pr_kernel == 6) {
-      CK(cudaFuncSetAttribute(k_pr_warp_pipe<OffT>, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)g->hot_smem));
-      CK(cudaOccupancyMaxActiveBlocksPerMultiprocessor(&bps, k_pr_warp_pipe<OffT>, g->hot_cta, g->hot_smem));
-    } else {
-      CK(cudaFuncSetAttribute(k_pr_warp_hot<OffT>, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)g->hot_smem));
-      CK(cudaOccupancyMaxActiveBlocksPerMultiprocessor(&bps, k_pr_warp_hot<OffT>, g->hot_cta, g->hot_smem));
-    }
+    CK(cudaFuncSetAttribute(k_pr_warp_hot<OffT>, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)g->hot_smem));
+    CK(cudaOccupancyMaxActiveBlocksPerMultiprocessor(&bps, k_pr_warp_hot<OffT>, g->hot_cta, g->hot_smem));
   }
   if (bps < 1) {
     g->pr_kernel = 0;  // shared-memory table does not fit: CTA merge-path kernel
@@ -1167,10 +1226,8 @@ static void pr_launch_iter(gr_graph *g, cudaStream_t s, uint32_t t, uint32_t ite
                            cudaEvent_t e1) {
   PrArgs<OffT> a = pr_args<OffT>(g, t, iters, d);
   const bool warp = g->pr_kernel >= 2;
-  const bool range = g->pr_kernel == 4 || g->pr_kernel == 5;
   if (warp) a.tile_row = g->wtile_row;
   const uint32_t tiles = g->pr_kernel == 7 ? g->seg_tiles : warp ? g->pr_wtiles : g->pr_tiles;
-  const uint32_t ranges = (tiles + kRangeTiles - 1) / kRangeTiles;
   if (g->pr_hot == 1) {
     k_pr_hot_pack<<<(g->hot_k + 255) / 256, 256, 0, s>>>(a.contrib_in, g->hot_ids, g->hot_contrib, g->hot_k);
     a.in_src = g->pr_src;
@@ -1187,22 +1244,11 @@ static void pr_launch_iter(gr_graph *g, cudaStream_t s, uint32_t t, uint32_t ite
       seg_kernel<OffT>(g->seg_var)<<<g->hot_grid, g->hot_cta, g->hot_smem, s>>>(
           a, g->seg_src, g->seg_flags, g->seg_row, g->hot_contrib, g->hot_k, tiles);
       break;
-    case 6:
-      k_pr_warp_pipe<OffT><<<g->hot_grid, g->hot_cta, g->hot_smem, s>>>(a, g->hot_contrib, g->hot_k, tiles);
-      break;
-    case 4:
-      k_pr_warp_range<OffT, false><<<g->hot_grid, 1024, g->hot_smem, s>>>(a, nullptr, 0, tiles);
-      break;
-    case 5:
-      k_pr_warp_range<OffT, true><<<g->hot_grid, 1024, g->hot_smem, s>>>(a, g->hot_contrib, g->hot_k, tiles);
-      break;
     default:
       k_pr_warp<OffT><<<std::max<uint32_t>((tiles + 7) / 8, 1), 256, 0, s>>>(a, tiles);
   }
   if (e1) cudaEventRecord(e1, s);
-  if (range)
-    k_pr_fixup<OffT><<<(ranges + 255) / 256, 256, 0, s>>>(a, ranges);
-  else if (warp) {
+  if (warp) {
     k_pr_fixup_short<OffT><<<std::max<uint32_t>((tiles + 255) / 256, 1), 256, 0, s>>>(a, tiles, g->w_is_long);
     if (g->n_long) k_pr_fixup_long<OffT><<<(g->n_long + 7) / 8, 256, 0, s>>>(a, g->long_c, g->long_f, g->n_long);
   }
@@ -1220,7 +1266,7 @@ uint32_t pr_part_iter(gr_graph *g, cudaStream_t s, uint32_t t, uint32_t iters, f
   if (g->off64) pr_launch_iter<uint64_t>(g, s, t, iters, d, nullptr, nullptr);
   else pr_launch_iter<uint32_t>(g, s, t, iters, d, nullptr, nullptr);
   const bool warp = g->pr_kernel >= 2;
-  return (g->pr_hot == 1 ? 1u : 0u) + 2u + (warp && g->n_long && g->pr_kernel != 4 && g->pr_kernel != 5 ? 1u : 0u);
+  return (g->pr_hot == 1 ? 1u : 0u) + 2u + (warp && g->n_long ? 1u : 0u);
 }
 
 template <class OffT>
@@ -1404,6 +1450,17 @@ gr_status run(gr_graph *g, const gr_run_opts *oin, gr_run_stats *st) {
   if (o.algo == GR_SSSP && !g->H.has_w) return fail(GR_EINVAL, "SSSP needs edge weights");
   if (o.algo < GR_BFS || o.algo > GR_PAGERANK_DELTA) return fail(GR_EINVAL, "unknown algo %d", o.algo);
   if (o.direction < GR_DIR_AUTO || o.direction > GR_DIR_FUSED) return fail(GR_EINVAL, "unknown direction %d", o.direction);
+  // one-directional streamed layouts (GR_FMT_SORTED with only one half): PageRank
+  // needs the in-CSC alone, BFS the out-CSR alone, every other program both
+  if (!g->H.has_in || !g->H.has_out) {
+    const bool ok = (o.algo == GR_PAGERANK && g->H.has_in) || (o.algo == GR_BFS && g->H.has_out);
+    if (!ok)
+      return fail(GR_EUNSUPPORTED, "the graph was loaded with only its %s: algo %d needs %s",
+                  g->H.has_in ? "in-CSC" : "out-CSR", o.algo, o.algo == GR_PAGERANK ? "the in-CSC" :
+                  o.algo == GR_BFS ? "the out-CSR" : "both directions");
+  }
+  if (o.trace_detail && (g->mode == GR_MODE_STREAMED || g->comm))
+    return fail(GR_EUNSUPPORTED, "trace_detail: resident single-rank graphs only");
   const JitProgram *jp = nullptr;
   if (o.algo == GR_CUSTOM) {
     bool known = false, uses_w = false;
@@ -1487,7 +1544,41 @@ gr_status run(gr_graph *g, const gr_run_opts *oin, gr_run_stats *st) {
   st->seconds = ms * 1e-3;
   g->last_algo = o.algo;
   g->last_iters = st->iterations;
+  g->last_detail = o.trace_detail != 0;
   if (o.algo == GR_PAGERANK) g->pr_trace_iters = o.max_iters;
+  return GR_OK;
+}
+
+static __global__ void k_count_nonzero(const uint32_t *a, uint64_t n, unsigned long long *out) {
+  unsigned long long c = 0;
+  for (uint64_t i = blockIdx.x * (uint64_t)blockDim.x + threadIdx.x; i < n; i += (uint64_t)gridDim.x * blockDim.x)
+    c += a[i] != 0;
+  for (int o = 16; o > 0; o >>= 1) c += __shfl_xor_sync(0xffffffffu, c, o);
+  if ((threadIdx.x & 31) == 0 && c) atomicAdd(out, c);
+}
+
+gr_status fetch_trace_detail(gr_graph *g, uint64_t *dst, uint64_t max_rows, uint64_t *rows) {
+  if (g->last_algo < 0 || !g->last_detail)
+    return fail(GR_ESTATE, "gr_fetch_frontier_trace_detail: the last run did not record the detail columns");
+  if (!rows || (max_rows && !dst)) return fail(GR_EINVAL, "null output");
+  const uint64_t r = std::min<uint64_t>(g->trace_rows, max_rows);
+  if (g->last_algo == GR_PAGERANK) {  // A_t = V: every shard active, every source with an out-edge read
+    unsigned long long *d = nullptr, h = 0;
+    CK(cudaMallocAsync((void **)&d, 8, g->stream));
+    CK(cudaMemsetAsync(d, 0, 8, g->stream));
+    k_count_nonzero<<<g->num_sms * 2, 256, 0, g->stream>>>(g->d_outdeg, g->H.n, d);
+    CK(cudaMemcpyAsync(&h, d, 8, cudaMemcpyDeviceToHost, g->stream));
+    CK(cudaFreeAsync(d, g->stream));
+    CK(cudaStreamSynchronize(g->stream));
+    for (uint64_t t = 0; t < r; t++) {
+      dst[2 * t] = g->H.num_shards();
+      dst[2 * t + 1] = h;
+    }
+  } else if (r) {
+    CK(cudaMemcpyAsync(dst, g->trace_det, 16 * r, cudaMemcpyDeviceToHost, g->stream));
+    CK(cudaStreamSynchronize(g->stream));
+  }
+  *rows = r;
   return GR_OK;
 }
 
@@ -1540,6 +1631,7 @@ void destroy(gr_graph *g) {
   for (void *p : g->plain_allocs) cudaFree(p);
   cudaStreamSynchronize(g->stream);
   if (g->h_ctl) cudaFreeHost(g->h_ctl);
+  if (g->h_xbytes) cudaFreeHost(g->h_xbytes);
   if (g->stream) cudaStreamDestroy(g->stream);
   delete g;
 }

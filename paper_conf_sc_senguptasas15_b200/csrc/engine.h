@@ -111,6 +111,11 @@ struct gr_graph {
   uint32_t last_iters = 0;
   uint32_t epoch_next = 1;
   uint64_t trace_rows = 0;
+  // detail columns of the trace (gr_run_opts.trace_detail): (active_shards, S_t) per superstep
+  unsigned long long *trace_det = nullptr;  // device [2 * trace_cap]
+  uint32_t *det_src_bits = nullptr, *det_shard_bits = nullptr;
+  uint64_t *d_shard_bounds = nullptr;
+  bool last_detail = false;
   std::map<int, std::pair<cudaGraphExec_t, uint64_t>> while_exec;
   cudaEvent_t ev_start = nullptr, ev_stop = nullptr;
   std::vector<cudaEvent_t> prof_ev;
@@ -128,12 +133,24 @@ struct gr_graph {
   uint32_t *fx_own_v[2] = {}, *fx_own_val[2] = {};
   uint32_t *fx_v[2][16] = {}, *fx_val[2][16] = {};
   bool fx_ok = false;
+  // device-side count exchange of the fused frontier exchange (engine_part.cu): this
+  // rank's XCount (cudaMalloc, mapped into every peer), the peers' mappings, and
+  // this rank's per-superstep decision (XDev)
+  void *xc_own = nullptr, *xc_peer[16] = {}, *xdev = nullptr;
+  void **d_xc_peer = nullptr;                 // device copy of xc_peer (the publish kernel's targets)
+  unsigned long long *h_xbytes = nullptr;     // pinned: XDev::bytes_in read back without a pageable copy
+  bool xc_ok = false;
   // PageRank fused exchange: every other rank's contribution replica (by parity),
   // peer-mapped (cudaIpc, NCCL mode) or same-device (simulated ranks)
   float *pr_peer[2][15] = {};
   uint32_t pr_npeer = 0;
   bool pr_p2p = false;          // the mapping exists (set up at load)
   bool pr_p2p_on = false;       // this run exchanges by peer stores (else NCCL allgatherv)
+  // device-side barrier between partitioned supersteps (engine_part.cu k_xbar): every
+  // rank's arrival words (cudaMalloc, mapped into every peer) and a sequence counter
+  uint32_t *xbar_own = nullptr, *xbar_peer[16] = {}, **d_xbar_peer = nullptr;
+  uint32_t xbar_seq = 0;
+  bool xbar_ok = false;
   std::vector<void *> plain_allocs;  // cudaMalloc'ed (IPC-exportable) buffers
 };
 
@@ -148,10 +165,6 @@ template <class OffT> inline Part<OffT> make_part(gr_graph *g) {
   P.in_src = g->in_src;
   P.in_w = g->in_w;
   P.prd_div = g->prd_div;
-  {
-    static const int gate = getenv("GR_GATE") ? atoi(getenv("GR_GATE")) : 1;
-    P.gate = (uint32_t)gate;
-  }
   P.estate = g->estate;
   P.out_eid = g->out_eid;
   P.ds_src = g->ds_src;
@@ -224,6 +237,7 @@ uint32_t pr_part_iter(gr_graph *g, cudaStream_t s, uint32_t t, uint32_t iters, f
 gr_status run(gr_graph *g, const gr_run_opts *o, gr_run_stats *st);
 gr_status fetch_values(gr_graph *g, void *dst, uint64_t bytes);
 gr_status fetch_trace(gr_graph *g, uint64_t *dst, uint64_t max_rows, uint64_t *rows);
+gr_status fetch_trace_detail(gr_graph *g, uint64_t *dst, uint64_t max_rows, uint64_t *rows);
 void destroy(gr_graph *g);
 // streamed mode
 gr_status stream_setup(gr_graph *g, uint64_t budget);

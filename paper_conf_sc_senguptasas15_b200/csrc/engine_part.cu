@@ -75,6 +75,58 @@ gr_status part_setup(gr_graph *g) {
       }
     }
     g->fx_ok = ok;
+    // device-side count exchange (same agreed mapping protocol): every rank's
+    // (|C_t|, |A_t|) lands in every peer's XCount, flagged by a sequence number
+    g->xc_ok = false;
+    if (ok) {
+      if (cudaMalloc(&g->xc_own, sizeof(XCount)) != cudaSuccess || cudaMemset(g->xc_own, 0, sizeof(XCount)) != cudaSuccess) {
+        cudaGetLastError();
+        return fail(GR_ENOMEM, "count exchange buffer");
+      }
+      g->plain_allocs.push_back(g->xc_own);
+      gr_status a = dev_alloc(g, &g->xdev, sizeof(XDev));
+      if (a != GR_OK) return a;
+      XDev x0{};
+      for (int q = 0; q < g->comm->world; q++) x0.R.off[q] = (uint32_t)g->H.owners[q];
+      x0.R.nr = (uint32_t)g->comm->world;
+      if (cudaMemcpy(g->xdev, &x0, sizeof x0, cudaMemcpyHostToDevice) != cudaSuccess)
+        return fail(GR_ECUDA, "count exchange init");
+      std::vector<void *> pc;
+      gr_status c = g->comm->share_buffer(g->xc_own, &pc, g->stream);
+      if (c == GR_OK) {
+        for (int q = 0; q < g->comm->world; q++) g->xc_peer[q] = pc[q];
+        // no pageable copies in the superstep loop: a pageable transfer can wait on the
+        // device, where a peer's wait kernel may be spinning on this rank's next publish
+        if ((a = dev_alloc(g, (void **)&g->d_xc_peer, sizeof(void *) * 16)) != GR_OK) return a;
+        if (cudaMemcpy(g->d_xc_peer, g->xc_peer, sizeof(void *) * 16, cudaMemcpyHostToDevice) != cudaSuccess ||
+            cudaMallocHost((void **)&g->h_xbytes, 16) != cudaSuccess)
+          return fail(GR_ECUDA, "count exchange setup");
+        g->xc_ok = true;
+      } else if (c != GR_EUNSUPPORTED) {
+        return fail(c, "count exchange mapping failed");
+      }
+    }
+  }
+  // device-side superstep barrier (k_xbar): arrival words mapped into every peer
+  g->xbar_ok = false;
+  if (g->comm->world <= 16) {
+    if (cudaMalloc((void **)&g->xbar_own, 64) != cudaSuccess || cudaMemset(g->xbar_own, 0, 64) != cudaSuccess) {
+      cudaGetLastError();
+      return fail(GR_ENOMEM, "barrier words");
+    }
+    g->plain_allocs.push_back(g->xbar_own);
+    std::vector<void *> pb;
+    gr_status c = g->comm->share_buffer(g->xbar_own, &pb, g->stream);
+    if (c == GR_OK) {
+      gr_status a = dev_alloc(g, (void **)&g->d_xbar_peer, sizeof(void *) * 16);
+      if (a != GR_OK) return a;
+      for (int q = 0; q < g->comm->world; q++) g->xbar_peer[q] = static_cast<uint32_t *>(pb[q]);
+      if (cudaMemcpy(g->d_xbar_peer, g->xbar_peer, sizeof(void *) * 16, cudaMemcpyHostToDevice) != cudaSuccess)
+        return fail(GR_ECUDA, "barrier words");
+      g->xbar_ok = true;
+    } else if (c != GR_EUNSUPPORTED) {
+      return fail(c, "barrier word mapping failed");
+    }
   }
   // PageRank fused exchange: map every peer's contribution replicas (both
   // parities). Without a mapping (no peer access) PageRank exchanges with NCCL.
@@ -130,6 +182,115 @@ static __global__ void k_part_counts(const Ctl *ctl, uint64_t *out) {
   out[1] = ctl->cnt_act[ctl->iter & 1u];
 }
 
+// ---- device-side count exchange (no host synchronisation per superstep) ----
+// After the gather of superstep t, k_part_publish stores this rank's
+// (|C_t|, |A_t|) into every rank's XCount (peer mappings: NVLink stores across
+// GPUs), then raises the slot's sequence number to seq after a system-scope
+// fence. k_part_wait (one warp) waits until every rank's seq for t arrived
+// — lane q spins on rank q's slot — and decides on the device what the host
+// decided before: the rank regions of the fused exchange buffers (XRanges), the
+// global |C_t|, and termination (no active vertex on any rank: ctl->stop, the
+// same superstep on every rank since every rank sees the same counts). Slots
+// are double-buffered by parity: a rank publishes t + 2 only after its wait of
+// t + 1, which needs every peer's publish of t + 1, issued after that peer's
+// classify of t — so no slot is overwritten while a peer still reads it.
+// seq: a number unique to superstep t of this run on every rank (epoch_base + t + 1:
+// epochs only grow across runs and advance identically on every rank)
+static __global__ void k_part_publish(Ctl *ctl, XCount *const *peers, uint32_t rank, uint32_t world, uint32_t t,
+                                      uint32_t seq) {
+  const uint32_t q = threadIdx.x;
+  if (q >= world || ctl->stop) return;
+  const uint32_t par = t & 1u;
+  XCount *X = peers[q];
+  X->cnt[par][rank][0] = ctl->cnt_C;
+  X->cnt[par][rank][1] = ctl->cnt_act[ctl->iter & 1u];
+  __threadfence_system();
+  *(volatile uint32_t *)&X->seq[par][rank] = seq;
+}
+
+static __global__ void k_part_wait(Ctl *ctl, XCount *mine, XDev *xd, uint32_t rank, uint32_t world, uint32_t t,
+                                   uint32_t seq) {
+  const uint32_t q = threadIdx.x, par = t & 1u;
+  if (ctl->stop) return;  // uniform: every lane reads the same flag
+  unsigned long long c = 0, a = 0;
+  if (q < world) {
+    while (*(volatile uint32_t *)&mine->seq[par][q] != seq) __nanosleep(64);
+    __threadfence_system();
+    c = *(volatile unsigned long long *)&mine->cnt[par][q][0];
+    a = *(volatile unsigned long long *)&mine->cnt[par][q][1];
+  }
+  // exclusive prefix of |C_q| over ranks (world <= 16 lanes)
+  unsigned long long pre = c;
+  for (int o = 1; o < 32; o <<= 1) {
+    const unsigned long long y = __shfl_up_sync(0xffffffffu, pre, o);
+    if ((int)q >= o) pre += y;
+  }
+  const unsigned long long tot = __shfl_sync(0xffffffffu, pre, 31);
+  unsigned long long act = a;
+  for (int o = 16; o > 0; o >>= 1) act += __shfl_xor_sync(0xffffffffu, act, o);
+  unsigned long long peer_c = (q < world && q != rank) ? c : 0ull;
+  for (int o = 16; o > 0; o >>= 1) peer_c += __shfl_xor_sync(0xffffffffu, peer_c, o);
+  if (q < world) xd->R.pre[q] = (uint32_t)(pre - c);  // R.off / R.nr: set at load (owner starts)
+  if (q == 0) {
+    xd->R.pre[world] = (uint32_t)tot;
+    xd->tot = (uint32_t)tot;
+    xd->bytes_in += 8ull * peer_c;
+    ctl->cnt_C = 0;  // this rank's C list is refilled from the exchanged set by the classify
+    if (act == 0) ctl->stop = 1u;
+  }
+}
+
+// Stream-ordered barrier across ranks on the device (no host, no NCCL call):
+// lane q stores seq into rank q's arrival word of this rank after a
+// system-scope fence (so this rank's earlier kernels' stores, the fused peer
+// stores included, are visible first), then waits until rank q's seq arrived
+// in this rank's words. seq grows by one per barrier, identically on every rank.
+static __global__ void k_xbar(uint32_t *const *peers, uint32_t *mine, uint32_t rank, uint32_t world, uint32_t seq) {
+  const uint32_t q = threadIdx.x;
+  __threadfence_system();
+  if (q < world) *(volatile uint32_t *)(peers[q] + rank) = seq;
+  if (q < world)
+    while (*(volatile uint32_t *)(mine + q) < seq) __nanosleep(32);
+  __threadfence_system();
+  __syncwarp();
+}
+
+// k_classify with the exchanged set's size and rank regions read from the device
+template <class OffT>
+__global__ void __launch_bounds__(kBlock) k_classify_dev(const __grid_constant__ Part<OffT> P, const uint32_t *X_v,
+                                                         const uint32_t *X_val, const XDev *xd) {
+  __shared__ uint32_t sq[kWarpsPerBlock][2][kQueueCap];
+  __shared__ uint32_t s_off[kWarpsPerBlock + 1];
+  __shared__ XRanges R;
+  __shared__ uint32_t s_nx, s_stop;
+  if (threadIdx.x == 0) {
+    s_stop = *(volatile uint32_t *)&P.ctl->stop;
+    s_nx = xd->tot;
+    R = xd->R;
+  }
+  __syncthreads();
+  if (s_stop) return;
+  const uint32_t nX = s_nx;
+  const uint32_t warp = threadIdx.x / 32, lane = lane_id();
+  WarpQueue qC{sq[warp][0], sq[warp][1], 0};
+  const uint32_t gw = blockIdx.x * kWarpsPerBlock + warp, nw = gridDim.x * kWarpsPerBlock;
+  for (uint32_t base = gw * 32u; base < nX; base += nw * 32u) {
+    const uint32_t i = base + lane;
+    const bool valid = i < nX;
+    uint32_t at = i;
+    if (valid) {
+      uint32_t q = 0;
+      while (q + 1 < R.nr && R.pre[q + 1] <= i) q++;
+      at = R.off[q] + (i - R.pre[q]);
+    }
+    const uint32_t u = valid ? X_v[at] : 0u, val = valid ? X_val[at] : 0u;
+    const bool hub = valid && test_bit(P.hub_out, u);
+    if (hub) append_hub_C(P, u, val);
+    qC.push(valid && !hub, u, val, P.C_v, P.C_val, &P.ctl->cnt_C);
+  }
+  qC.block_flush(P.C_v, P.C_val, &P.ctl->cnt_C, s_off);
+}
+
 // D: the program's traits and kernels (prog_desc.h) — built-in or run-time compiled
 template <class OffT>
 gr_status run_frontier_part(gr_graph *g, const gr_run_opts *o, cudaStream_t s, gr_run_stats *st,
@@ -151,6 +312,7 @@ gr_status run_frontier_part(gr_graph *g, const gr_run_opts *o, cudaStream_t s, g
   uint64_t launches = 0;
   if (g->epoch_next > 0xF0000000u) {
     PCK(cudaMemsetAsync(g->stamp, 0, 4ull * std::max<uint64_t>(g->H.own_n(), 1), s));
+    if (g->xc_own) PCK(cudaMemsetAsync(g->xc_own, 0, sizeof(XCount), s));  // sequence numbers restart too
     g->epoch_next = 1;
   }
   Ctl h{};
@@ -163,7 +325,8 @@ gr_status run_frontier_part(gr_graph *g, const gr_run_opts *o, cudaStream_t s, g
   h.no_hub_c = 1;
   prd_setup(h, o, g->H.n);
   h.kstart[0] = h.kstart[1] = ~0ull;
-  PCK(cudaMemcpyAsync(g->ctl, &h, sizeof h, cudaMemcpyHostToDevice, s));
+  *g->h_ctl = h;  // pinned staging (no pageable transfer while peers' kernels may spin)
+  PCK(cudaMemcpyAsync(g->ctl, g->h_ctl, sizeof h, cudaMemcpyHostToDevice, s));
   uint32_t src0 = o->source;
   KL(D.init_values[K], g->num_sms * 4, 256, &P, &src0);
   if (kScatter) {
@@ -204,7 +367,63 @@ gr_status run_frontier_part(gr_graph *g, const gr_run_opts *o, cudaStream_t s, g
   // gather of t+1 while a peer still classifies t.
   bool fx = g->fx_ok;
   if (const char *e = getenv("GR_FRONTIER_EXCHANGE")) fx = fx && std::string(e) != "nccl";
-  while (o->max_iters == 0 || t < o->max_iters) {
+  // device-side count exchange (default with the fused exchange): no host
+  // synchronisation per superstep; the host enqueues supersteps in batches and
+  // reads the stop flag the wait kernels set once per batch
+  bool dx = fx && g->xc_ok;
+  if (const char *e = getenv("GR_COUNT_EXCHANGE")) dx = dx && std::string(e) != "host";
+  if (dx) {
+    const uint32_t batch = 8;
+    XCount *const *d_peers = reinterpret_cast<XCount *const *>(g->d_xc_peer);
+    XDev *xd = static_cast<XDev *>(g->xdev);
+    // only pinned / device copies below: a pageable transfer could wait on the device while a
+    // peer's wait kernel spins for this rank's next publish
+    PCK(cudaMemcpyAsync(g->h_xbytes, &xd->bytes_in, 8, cudaMemcpyDeviceToHost, s));
+    // every rank has finished its run setup (allocations, staging copies) before any rank
+    // enqueues a wait kernel that spins on its peers: ranks that share a device (simulated,
+    // same-GPU processes) must not block in a device-wide synchronisation behind a spinner
+    XCK(C->barrier(s));
+    P.n_xp = (uint32_t)C->world;
+    P.xp_off = (uint32_t)g->H.own_lo;
+    for (;;) {
+      for (uint32_t b = 0; b < batch && (o->max_iters == 0 || t < o->max_iters); b++, t++) {
+        const uint32_t par = t & 1u;
+        for (int q = 0; q < C->world; q++) {
+          P.xp_v[q] = g->fx_v[par][q];
+          P.xp_val[q] = g->fx_val[par][q];
+        }
+        KL(D.gather_apply_x[K], grid, kBlock, &P);
+        const uint32_t seq = h.epoch_base + t + 1;
+        k_part_publish<<<1, 32, 0, s>>>(g->ctl, d_peers, (uint32_t)C->rank, (uint32_t)C->world, t, seq);
+        k_part_wait<<<1, 32, 0, s>>>(g->ctl, static_cast<XCount *>(g->xc_own), xd, (uint32_t)C->rank,
+                                     (uint32_t)C->world, t, seq);
+        Part<OffT> Pc = P;
+        Pc.n_xp = 0;
+        k_classify_dev<OffT><<<grid, kBlock, 0, s>>>(Pc, g->fx_v[par][C->rank], g->fx_val[par][C->rank], xd);
+        if (kScatter) {
+          k_commit_only<OffT><<<grid, kBlock, 0, s>>>(Pc);
+          unsigned long long cond = 0;
+          int ug = 0;
+          void *a_[] = {&Pc, &cond, &ug};
+          gr_status r_ = klaunch(D, D.scatter_activate[K], grid, kBlock, a_, s);
+          if (r_ != GR_OK) return r_;
+          launches++;
+        } else {
+          k_activate<OffT><<<grid, kBlock, 0, s>>>(Pc, 0ull, 0);
+        }
+        launches += 5;
+        PCK(cudaGetLastError());
+      }
+      PCK(cudaMemcpyAsync(g->h_ctl, g->ctl, sizeof(Ctl), cudaMemcpyDeviceToHost, s));
+      PCK(cudaStreamSynchronize(s));
+      if (g->h_ctl->stop || (o->max_iters != 0 && t >= o->max_iters)) break;
+    }
+    PCK(cudaMemcpyAsync(g->h_xbytes + 1, &xd->bytes_in, 8, cudaMemcpyDeviceToHost, s));
+    PCK(cudaStreamSynchronize(s));
+    C->bytes_in += g->h_xbytes[1] - g->h_xbytes[0];
+    t = g->h_ctl->iter;  // supersteps that ran (the stopped one, if any, did not count)
+  }
+  while (!dx && (o->max_iters == 0 || t < o->max_iters)) {
     const uint32_t par = t & 1u;
     if (fx) {
       for (int q = 0; q < C->world; q++) {
@@ -308,14 +527,24 @@ gr_status run_pagerank_part(gr_graph *g, const gr_run_opts *o, cudaStream_t s, g
   g->pr_p2p_on = p2p;
   uint64_t launches = 1;
   k_pr_init<<<g->num_sms * 4, 256, 0, s>>>((uint32_t)g->H.n, g->inv_outdeg, g->contrib[0]);
+  // stream-ordered barrier between supersteps: on the device (k_xbar over the
+  // mapped arrival words, default) or the communicator's (NCCL allreduce / host)
+  bool dbar = g->xbar_ok;
+  if (const char *x = getenv("GR_PR_BARRIER")) dbar = dbar && std::string(x) != "comm";
+  auto barrier = [&]() -> gr_status {
+    if (!dbar) return C->barrier(s);
+    k_xbar<<<1, 32, 0, s>>>(g->d_xbar_peer, g->xbar_own, (uint32_t)C->rank, (uint32_t)C->world, ++g->xbar_seq);
+    launches++;
+    return cudaGetLastError() == cudaSuccess ? GR_OK : GR_ECUDA;
+  };
   // every replica is initialised before any rank's first fused store lands in it
-  if (p2p) XCK(C->barrier(s));
+  if (p2p) XCK(barrier());
   for (uint32_t t = 0; t < iters; t++) {
     launches += pr_part_iter(g, s, t, iters, d);
     PCK(cudaGetLastError());
     if (t + 1 == iters) break;
     if (p2p) {
-      XCK(C->barrier(s));
+      XCK(barrier());
       C->bytes_in += 4 * (g->H.n - g->H.own_n());
     } else {
       float *out = g->contrib[(t + 1) & 1];

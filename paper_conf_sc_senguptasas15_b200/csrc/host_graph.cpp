@@ -27,7 +27,8 @@ bool HostBuf::alloc(size_t nbytes) {
 void HostBuf::release() {
   if (registered) cudaHostUnregister(p);
   registered = false;
-  std::free(p);
+  if (owned) std::free(p);
+  owned = true;
   p = nullptr;
   bytes = 0;
 }
@@ -242,6 +243,121 @@ gr_status build_host_graph(const gr_edges *E, uint64_t shard_edges, int world, i
   st = gr_plan_intervals(own_n, local_prefix.data(), (uint32_t)P, G->bounds.data());
   if (st != GR_OK) { *err = "interval planning failed"; return st; }
   for (auto &b : G->bounds) b += G->own_lo;
+  return GR_OK;
+}
+
+// ---- pre-sorted input (GR_FMT_SORTED): the cfg5-scale path where no COO exists
+static bool check_adj(int T, uint64_t n, uint64_t m, const uint64_t *off, const uint32_t *adj, std::string *err,
+                      const char *what) {
+  if (off[0] != 0 || off[n] != m) {
+    *err = std::string(what) + ": offsets must span [0, m]";
+    return false;
+  }
+  std::atomic<int> bad{0};
+  parallel_for_dyn(T, n, 1 << 16, [&](uint64_t b, uint64_t e) {
+    int lb = 0;
+    for (uint64_t v = b; v < e && !lb; v++) {
+      if (off[v + 1] < off[v]) { lb = 1; break; }
+      for (uint64_t i = off[v]; i < off[v + 1]; i++) {
+        if (adj[i] >= n) lb |= 2;
+        if (i > off[v] && adj[i] < adj[i - 1]) lb |= 4;
+      }
+    }
+    if (lb) bad.fetch_or(lb);
+  });
+  if (bad.load() & 1) *err = std::string(what) + ": offsets not monotone";
+  else if (bad.load() & 2) *err = std::string(what) + ": neighbour id >= num_vertices";
+  else if (bad.load() & 4) *err = std::string(what) + ": rows must be sorted ascending (layout R10)";
+  return bad.load() == 0;
+}
+
+static bool take_adj(HostBuf *dst, const uint32_t *adj, uint64_t m, bool borrow) {
+  if (borrow) {  // the caller guarantees 4 spare entries after the m used ones (128-bit loads)
+    dst->borrow(adj, 4 * m + 16);
+    return true;
+  }
+  if (!dst->alloc(4 * m + 16)) return false;
+  std::memcpy(dst->p, adj, 4 * m);
+  std::memset(dst->as<char>() + 4 * m, 0, 16);
+  return true;
+}
+
+gr_status build_host_sorted(const gr_edges *E, uint64_t shard_edges, bool borrow, int threads, HostGraph *G,
+                            std::string *err) {
+  const uint64_t n = E->num_vertices, m = E->num_edges;
+  if (n == 0 || n >= 0xFFFFFFFFull) { *err = "num_vertices must be in [1, 2^32-2]"; return GR_EINVAL; }
+  const bool in = E->in_offsets != nullptr, out = E->row_offsets != nullptr;
+  if (!in && !out) { *err = "GR_FMT_SORTED needs in_offsets/in_idx and/or row_offsets/col_idx"; return GR_EINVAL; }
+  if ((in && m && !E->in_idx) || (out && m && !E->col_idx)) { *err = "GR_FMT_SORTED: adjacency array is NULL"; return GR_EINVAL; }
+  if (E->weights) { *err = "GR_FMT_SORTED carries no weights"; return GR_EINVAL; }
+  const int T = threads > 0 ? threads : default_threads();
+  if (in && !check_adj(T, n, m, E->in_offsets, E->in_idx, err, "in-CSC")) return GR_EINVAL;
+  if (out && !check_adj(T, n, m, E->row_offsets, E->col_idx, err, "out-CSR")) return GR_EINVAL;
+  G->n = n;
+  G->m_total = m;
+  G->own_lo = 0;
+  G->own_hi = n;
+  G->owners = {0, n};
+  G->m_in = m;
+  G->has_w = false;
+  G->has_in = in;
+  G->has_out = out;
+  // degrees: from the offsets, from the caller's out_degree, or counted
+  G->outdeg.assign(n, 0);
+  std::vector<uint32_t> indeg(n, 0);
+  if (out) {
+    parallel_for(T, n, [&](uint64_t b, uint64_t e) {
+      for (uint64_t u = b; u < e; u++) G->outdeg[u] = (uint32_t)(E->row_offsets[u + 1] - E->row_offsets[u]);
+    });
+  } else if (E->out_degree) {
+    std::memcpy(G->outdeg.data(), E->out_degree, 4 * n);
+  } else {
+    std::vector<std::atomic<uint32_t>> c(n);
+    parallel_for(T, n, [&](uint64_t b, uint64_t e) {
+      for (uint64_t v = b; v < e; v++) c[v].store(0, std::memory_order_relaxed);
+    });
+    parallel_for(T, m, [&](uint64_t b, uint64_t e) {
+      for (uint64_t i = b; i < e; i++) c[E->in_idx[i]].fetch_add(1, std::memory_order_relaxed);
+    });
+    for (uint64_t v = 0; v < n; v++) G->outdeg[v] = c[v].load();
+  }
+  if (in) {
+    parallel_for(T, n, [&](uint64_t b, uint64_t e) {
+      for (uint64_t v = b; v < e; v++) indeg[v] = (uint32_t)(E->in_offsets[v + 1] - E->in_offsets[v]);
+    });
+  } else {
+    std::vector<std::atomic<uint32_t>> c(n);
+    parallel_for(T, n, [&](uint64_t b, uint64_t e) {
+      for (uint64_t v = b; v < e; v++) c[v].store(0, std::memory_order_relaxed);
+    });
+    parallel_for(T, m, [&](uint64_t b, uint64_t e) {
+      for (uint64_t i = b; i < e; i++) c[E->col_idx[i]].fetch_add(1, std::memory_order_relaxed);
+    });
+    for (uint64_t v = 0; v < n; v++) indeg[v] = c[v].load();
+  }
+  if (in) {
+    G->in_off.assign(E->in_offsets, E->in_offsets + n + 1);
+    if (!take_adj(&G->in_src, E->in_idx, m, borrow)) { *err = "host allocation failed"; return GR_ENOMEM; }
+  } else {
+    G->in_off.assign(n + 1, 0);  // offsets only (no edges): zero-degree rows keep the kernels' indexing valid
+    for (uint64_t v = 0; v < n; v++) G->in_off[v + 1] = G->in_off[v] + indeg[v];
+  }
+  if (out) {
+    G->out_off.assign(E->row_offsets, E->row_offsets + n + 1);
+    if (!take_adj(&G->out_dst, E->col_idx, m, borrow)) { *err = "host allocation failed"; return GR_ENOMEM; }
+  } else {
+    G->out_off.assign(n + 1, 0);
+    for (uint64_t v = 0; v < n; v++) G->out_off[v + 1] = G->out_off[v] + G->outdeg[v];
+  }
+  // shards (Shard Creator, L208): intervals of near-equal in+out degree
+  std::vector<uint64_t> wprefix(n + 1, 0);
+  for (uint64_t v = 0; v < n; v++) wprefix[v + 1] = wprefix[v] + indeg[v] + G->outdeg[v];
+  if (shard_edges == 0) shard_edges = uint64_t(1) << 26;
+  uint64_t P = (wprefix[n] + shard_edges - 1) / shard_edges;
+  P = std::max<uint64_t>(1, std::min<uint64_t>(P, std::min<uint64_t>(65535, n)));
+  G->bounds.assign(P + 1, 0);
+  gr_status st = gr_plan_intervals(n, wprefix.data(), (uint32_t)P, G->bounds.data());
+  if (st != GR_OK) { *err = "interval planning failed"; return st; }
   return GR_OK;
 }
 

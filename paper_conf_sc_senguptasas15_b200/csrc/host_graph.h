@@ -21,6 +21,13 @@ struct HostBuf {
   void *p = nullptr;
   size_t bytes = 0;
   bool registered = false;
+  bool owned = true;   // false: the caller's memory, used in place (GR_FMT_SORTED + borrow)
+  void borrow(const void *q, size_t nbytes) {
+    release();
+    p = const_cast<void *>(q);
+    bytes = nbytes;
+    owned = false;
+  }
   HostBuf() = default;
   HostBuf(const HostBuf &) = delete;
   HostBuf &operator=(const HostBuf &) = delete;
@@ -37,6 +44,9 @@ struct HostGraph {
   std::vector<uint64_t> owners;     // owner range bounds of every rank (world + 1)
   uint64_t m_in = 0;       // in-edges with an owned destination
   bool has_w = false;
+  // which halves of the layout exist: a GR_FMT_SORTED input may carry only the
+  // in-CSC (PageRank) or only the out-CSR (BFS) of a graph too large for both
+  bool has_in = true, has_out = true;
   // CSC over owned destinations: in-edges of v = in_src[in_off[v-own_lo] .. in_off[v-own_lo+1])
   std::vector<uint64_t> in_off;  // own_n + 1
   HostBuf in_src;                // uint32 [m_in] (+ 4 pad entries for 16-byte vector loads)
@@ -61,6 +71,11 @@ struct HostGraph {
 // the same split). Returns GR_OK or an error with *err filled.
 gr_status build_host_graph(const gr_edges *e, uint64_t shard_edges, int world, int rank,
                            int threads, HostGraph *out, std::string *err);
+
+// Layout from a pre-sorted input (GR_FMT_SORTED): the in-CSC and/or out-CSR as
+// given (rows sorted ascending, checked), borrowed in place or copied; single rank.
+gr_status build_host_sorted(const gr_edges *e, uint64_t shard_edges, bool borrow, int threads, HostGraph *out,
+                            std::string *err);
 
 // Owner split of [0, n) for `world` ranks (same on every rank).
 gr_status plan_owner_ranges(uint64_t n, const uint64_t *weight_prefix, int world,

@@ -340,138 +340,6 @@ __global__ void __launch_bounds__(1024, 1) k_pr_warp_hot(const __grid_constant__
     pr_warp_tile<OffT, true>(a, tile, S[w], s_hot);
 }
 
-// Software-pipelined warp tiles (same tiles, same hot table, same sums as
-// k_pr_warp_hot): while a warp walks tile T it already has tile T+1's source
-// ids and tile T+2's merge-path coordinates in registers, so the only
-// dependent global round trips left per tile are the contribution gathers
-// (issued together with the row-offset loads) and the apply's stores. The
-// 1/outdeg of the tile's first 32 rows is loaded before the walk.
-template <class OffT>
-__device__ __forceinline__ void pr_load_src(const PrArgs<OffT> &a, uint32_t tile, uint32_t i0, uint32_t i1,
-                                            uint32_t (&src)[kWIpt]) {
-  const uint64_t total = (uint64_t)a.own_n + a.m_in;
-  const uint64_t d0 = (uint64_t)tile * kWTile;
-  const uint64_t d1 = d0 + kWTile < total ? d0 + kWTile : total;
-  const uint64_t j0 = d0 - i0;
-  const uint32_t nj = (uint32_t)((d1 - i1) - j0);
-  const uint32_t lane = threadIdx.x & 31;
-#pragma unroll
-  for (int q = 0; q < kWIpt; q++) {
-    const uint32_t k = lane + 32u * q;
-    src[q] = k < nj ? ldg_nc(a.in_src + j0 + k) : 0u;
-  }
-}
-
-template <class OffT>
-__global__ void __launch_bounds__(1024, 1) k_pr_warp_pipe(const __grid_constant__ PrArgs<OffT> a,
-                                                         const float *hot_contrib, uint32_t hot_k,
-                                                         uint32_t num_tiles) {
-  extern __shared__ __align__(16) unsigned char smem_raw[];
-  float *s_hot = reinterpret_cast<float *>(smem_raw);
-  for (uint32_t k = threadIdx.x * 4; k < hot_k; k += blockDim.x * 4)
-    *reinterpret_cast<float4 *>(s_hot + k) = __ldg(reinterpret_cast<const float4 *>(hot_contrib + k));
-  __syncthreads();
-  const uint32_t lane = threadIdx.x & 31, w = threadIdx.x >> 5, nw = blockDim.x >> 5;
-  PrWarpSmem &S = reinterpret_cast<PrWarpSmem *>(smem_raw + 4ull * hot_k)[w];
-  const uint32_t stride = gridDim.x * nw;
-  const uint64_t total = (uint64_t)a.own_n + a.m_in;
-  uint32_t tile = blockIdx.x * nw + w;
-  if (tile >= num_tiles) return;
-  uint32_t i0 = __ldg(a.tile_row + tile), i1 = __ldg(a.tile_row + tile + 1);
-  uint32_t src[kWIpt];
-  pr_load_src(a, tile, i0, i1, src);
-  uint32_t ntile = tile + stride, n_i0 = 0, n_i1 = 0;
-  if (ntile < num_tiles) { n_i0 = __ldg(a.tile_row + ntile); n_i1 = __ldg(a.tile_row + ntile + 1); }
-  for (;;) {
-    const uint64_t d0 = (uint64_t)tile * kWTile;
-    const uint64_t d1 = d0 + kWTile < total ? d0 + kWTile : total;
-    const uint64_t j0 = d0 - i0;
-    const uint32_t ni = i1 - i0, nj = (uint32_t)((d1 - i1) - j0);
-    // 1) this tile's gathers (sources already in registers)
-    float v[kWIpt];
-#pragma unroll
-    for (int q = 0; q < kWIpt; q++) {
-      const uint32_t k = lane + 32u * q;
-      if (src[q] & kHotTag) v[q] = s_hot[src[q] & ~kHotTag];
-      else v[q] = k < nj ? __ldg(a.contrib_in + src[q]) : 0.f;
-    }
-    // 2) next tile's sources, the tile after next's coordinates, this tile's first row start and 1/outdeg
-    const uint32_t nntile = ntile + stride;
-    uint32_t nn_i0 = 0, nn_i1 = 0;
-    if (ntile < num_tiles) pr_load_src(a, ntile, n_i0, n_i1, src);
-    if (nntile < num_tiles) { nn_i0 = __ldg(a.tile_row + nntile); nn_i1 = __ldg(a.tile_row + nntile + 1); }
-    const uint64_t rowstart0 = (uint64_t)a.in_off[i0] - a.e_base;
-    const float inv0 = (!a.last && lane < ni) ? __ldg(a.inv_outdeg + a.own_lo + i0 + lane) : 0.f;
-    // 3) stage row ends and contributions
-    __syncwarp();  // the previous tile's readers are done with S
-    for (uint32_t k = lane; k <= ni; k += 32) {
-      const uint64_t r = (uint64_t)i0 + k;
-      const uint64_t e = r < a.own_n ? (uint64_t)a.in_off[r + 1] - a.e_base - j0 : (uint64_t)nj;
-      S.s_end[pr_pad(k)] = (uint32_t)(e < nj ? e : nj);
-    }
-#pragma unroll
-    for (int q = 0; q < kWIpt; q++) {
-      const uint32_t k = lane + 32u * q;
-      if (k < nj) S.s_val[pr_pad(k)] = v[q];
-    }
-    __syncwarp();
-    // 4) merge walk + segmented warp scan (as pr_warp_tile)
-    const uint32_t items = ni + nj;
-    const uint32_t dt = min(lane * kWIpt, items);
-    uint32_t lo = dt > nj ? dt - nj : 0, hi = dt < ni ? dt : ni;
-    while (lo < hi) {
-      const uint32_t p = (lo + hi) >> 1;
-      if (S.s_end[pr_pad(p)] <= dt - p - 1) lo = p + 1;
-      else hi = p;
-    }
-    uint32_t i = lo, j = dt - lo;
-    float run = 0.f;
-    const uint32_t dend = min(dt + kWIpt, items);
-#pragma unroll
-    for (int q = 0; q < kWIpt; q++) {
-      if (dt + q < dend) {
-        if (j < S.s_end[pr_pad(i)]) { run += S.s_val[pr_pad(j)]; ++j; }
-        else { S.s_tot[pr_pad(i)] = run; run = 0.f; ++i; }
-      }
-    }
-    float x = run;
-#pragma unroll
-    for (int o = 1; o < 32; o <<= 1) {
-      const float y = __shfl_up_sync(0xffffffffu, x, o);
-      const uint32_t ky = __shfl_up_sync(0xffffffffu, i, o);
-      if (lane >= (uint32_t)o && ky == i) x += y;
-    }
-    const uint32_t inext = __shfl_down_sync(0xffffffffu, i, 1);
-    const float carry = __shfl_sync(0xffffffffu, x, 31);
-    __syncwarp();
-    const bool run_end = (lane == 31) || (inext != i);
-    if (run_end && i < ni) S.s_tot[pr_pad(i)] += x;
-    __syncwarp();
-    // 5) apply
-    const bool head = (ni > 0) && (rowstart0 < j0);
-    for (uint32_t k = lane; k < ni; k += 32) {
-      if (k == 0 && head) continue;
-      const float R = a.base + a.d * S.s_tot[pr_pad(k)];
-      const uint32_t lrow = i0 + k;
-      if (a.last) a.rank[lrow] = R;
-      else pr_store_contrib(a, a.own_lo + lrow, R * (k < 32 ? inv0 : __ldg(a.inv_outdeg + a.own_lo + lrow)));
-    }
-    if (lane == 0) {
-      a.head_row[tile] = head ? i0 : kNoRow;
-      a.head_val[tile] = head ? S.s_tot[pr_pad(0)] : 0.f;
-      a.carry_row[tile] = i1 < a.own_n ? i1 : kNoRow;
-      a.carry_val[tile] = carry;
-    }
-    if (ntile >= num_tiles) break;
-    tile = ntile;
-    i0 = n_i0;
-    i1 = n_i1;
-    ntile = nntile;
-    n_i0 = nn_i0;
-    n_i1 = nn_i1;
-  }
-}
-
 // ---------------------------------------------------------------------------
 // Edge-segmented warp tiles (`seg`, the default on resident single-GPU runs).
 // The PageRank payload is re-laid out once per graph as an item stream in CSC
@@ -490,7 +358,7 @@ constexpr int kSegIpt = 8;
 constexpr int kSegHotK = 32768;  // hot sources of the seg kernel (128 KB of shared memory; measured best of 16K-56K)
 constexpr int kSegTile = 32 * kSegIpt;
 
-// Variant bits of k_pr_seg (GR_PR_SEG_VAR; measured in profiles/README.md):
+// Variant bits of k_pr_seg (measured in round 1, profiles/README.md; only kSegDefaultVar is built):
 constexpr int kSegBallot = 1;   // segment starts of the lane scan from one ballot (1 shuffle per step, not 3)
 constexpr int kSegBuf = 2;      // finished rows through a per-warp buffer: coalesced apply, 1/outdeg preloaded
 constexpr int kSegPreFlag = 4;  // head bits loaded one tile ahead
@@ -1301,151 +1169,6 @@ __global__ void k_pr_fixup_warp(const __grid_constant__ PrArgs<OffT> a, uint32_t
 }
 
 
-// ---------------------------------------------------------------------------
-// Persistent warp-range kernel: warp w walks the CONTIGUOUS tiles
-// [w*T, (w+1)*T) and carries the open row's partial sum in registers from one
-// tile to the next, so a row split between two tiles of the same warp is
-// finished by that warp. Only rows that cross a warp-range boundary are left to
-// k_pr_fixup (one head/carry record per warp range, indexed by the global warp).
-constexpr uint32_t kRangeTiles = 8;  // warp tiles per chunk (2048 items)
-
-template <class OffT, bool kHot>
-__device__ __forceinline__ void pr_warp_range(const PrArgs<OffT> &a, uint32_t wid, uint32_t t0, uint32_t t1,
-                                              PrWarpSmem &S, const float *s_hot) {
-  const uint32_t lane = threadIdx.x & 31;
-  const uint64_t total = (uint64_t)a.own_n + a.m_in;
-  uint32_t pend_row = kNoRow;  // row whose partial sum is carried into the next tile
-  float pend_val = 0.f;
-  bool range_head = false;     // pend_row began before this warp's range
-  bool head_written = false;
-  for (uint32_t tile = t0; tile < t1; tile++) {
-    const uint64_t d0 = (uint64_t)tile * kWTile;
-    const uint64_t d1 = d0 + kWTile < total ? d0 + kWTile : total;
-    const uint32_t i0 = __ldg(a.tile_row + tile), i1 = __ldg(a.tile_row + tile + 1);
-    const uint64_t j0 = d0 - i0;
-    const uint32_t ni = i1 - i0, nj = (uint32_t)((d1 - i1) - j0);
-    const bool started_before = ((uint64_t)a.in_off[i0] - a.e_base) < j0;
-    if (tile == t0) {
-      pend_row = i0;
-      pend_val = 0.f;
-      range_head = started_before;
-    }
-    __syncwarp();
-    for (uint32_t k = lane; k <= ni; k += 32) {
-      const uint64_t r = (uint64_t)i0 + k;
-      const uint64_t e = r < a.own_n ? (uint64_t)a.in_off[r + 1] - a.e_base - j0 : (uint64_t)nj;
-      S.s_end[pr_pad(k)] = (uint32_t)(e < nj ? e : nj);
-    }
-    {
-      uint32_t src[kWIpt];
-#pragma unroll
-      for (int q = 0; q < kWIpt; q++) {
-        const uint32_t k = lane + 32u * q;
-        src[q] = k < nj ? ldg_nc(a.in_src + j0 + k) : 0u;
-      }
-      float v[kWIpt];
-#pragma unroll
-      for (int q = 0; q < kWIpt; q++) {
-        const uint32_t k = lane + 32u * q;
-        if (kHot && (src[q] & kHotTag)) v[q] = s_hot[src[q] & ~kHotTag];
-        else v[q] = k < nj ? __ldg(a.contrib_in + src[q]) : 0.f;
-      }
-#pragma unroll
-      for (int q = 0; q < kWIpt; q++) {
-        const uint32_t k = lane + 32u * q;
-        if (k < nj) S.s_val[pr_pad(k)] = v[q];
-      }
-    }
-    __syncwarp();
-    const uint32_t items = ni + nj;
-    const uint32_t dt = min(lane * kWIpt, items);
-    uint32_t lo = dt > nj ? dt - nj : 0, hi = dt < ni ? dt : ni;
-    while (lo < hi) {
-      const uint32_t p = (lo + hi) >> 1;
-      if (S.s_end[pr_pad(p)] <= dt - p - 1) lo = p + 1;
-      else hi = p;
-    }
-    uint32_t i = lo, j = dt - lo;
-    float run = 0.f;
-    const uint32_t dend = min(dt + kWIpt, items);
-#pragma unroll
-    for (int q = 0; q < kWIpt; q++) {
-      if (dt + q < dend) {
-        if (j < S.s_end[pr_pad(i)]) { run += S.s_val[pr_pad(j)]; ++j; }
-        else { S.s_tot[pr_pad(i)] = run; run = 0.f; ++i; }
-      }
-    }
-    float x = run;
-#pragma unroll
-    for (int o = 1; o < 32; o <<= 1) {
-      const float y = __shfl_up_sync(0xffffffffu, x, o);
-      const uint32_t ky = __shfl_up_sync(0xffffffffu, i, o);
-      if (lane >= (uint32_t)o && ky == i) x += y;
-    }
-    const uint32_t inext = __shfl_down_sync(0xffffffffu, i, 1);
-    const float cx = __shfl_sync(0xffffffffu, x, 31);  // partial of row i1 inside this tile
-    __syncwarp();
-    const bool run_end = (lane == 31) || (inext != i);
-    if (run_end && i < ni) S.s_tot[pr_pad(i)] += x;
-    __syncwarp();
-    if (ni > 0) {
-      // row i0: add the partial carried from this warp's previous tile
-      const float tot0 = S.s_tot[pr_pad(0)] + (started_before && pend_row == i0 ? pend_val : 0.f);
-      const bool is_head = started_before && range_head;
-      if (lane == 0) {
-        if (is_head) {
-          a.head_row[wid] = i0;
-          a.head_val[wid] = tot0;
-        } else {
-          pr_apply_row(a, i0, tot0);
-        }
-      }
-      head_written |= is_head;
-      for (uint32_t k = 1 + lane; k < ni; k += 32) pr_apply_row(a, i0 + k, S.s_tot[pr_pad(k)]);
-      pend_row = i1;
-      pend_val = cx;
-      range_head = false;
-    } else {
-      pend_val = (pend_row == i0 ? pend_val : 0.f) + cx;
-      pend_row = i0;
-    }
-  }
-  if (lane == 0 && t0 < t1) {
-    if (!head_written) a.head_row[wid] = kNoRow;
-    a.carry_row[wid] = pend_row < a.own_n ? pend_row : kNoRow;
-    a.carry_val[wid] = pend_val;
-  } else if (lane == 0) {
-    a.head_row[wid] = kNoRow;
-    a.carry_row[wid] = kNoRow;
-    a.carry_val[wid] = 0.f;
-  }
-}
-
-template <class OffT, bool kHot>
-__global__ void __launch_bounds__(1024, 1) k_pr_warp_range(const __grid_constant__ PrArgs<OffT> a,
-                                                          const float *hot_contrib, uint32_t hot_k,
-                                                          uint32_t num_tiles) {
-  extern __shared__ __align__(16) unsigned char smem_raw[];
-  float *s_hot = reinterpret_cast<float *>(smem_raw);
-  PrWarpSmem *S = reinterpret_cast<PrWarpSmem *>(smem_raw + (kHot ? 4ull * hot_k : 0ull));
-  if (kHot) {
-    for (uint32_t k = threadIdx.x * 4; k < hot_k; k += blockDim.x * 4)
-      *reinterpret_cast<float4 *>(s_hot + k) = __ldg(reinterpret_cast<const float4 *>(hot_contrib + k));
-    __syncthreads();
-  }
-  // interleaved chunks of kRangeTiles contiguous tiles: balanced across warps
-  // (hot/cold source mix varies along the graph), carries stay in registers
-  // inside a chunk, one head/carry record per chunk for k_pr_fixup
-  const uint32_t w = threadIdx.x >> 5, nw = blockDim.x >> 5;
-  const uint32_t wid = blockIdx.x * nw + w, W = gridDim.x * nw;
-  const uint32_t nchunks = (num_tiles + kRangeTiles - 1) / kRangeTiles;
-  for (uint32_t c = wid; c < nchunks; c += W) {
-    const uint32_t t0 = c * kRangeTiles, t1 = min(t0 + kRangeTiles, num_tiles);
-    pr_warp_range<OffT, kHot>(a, c, t0, t1, S[w], s_hot);
-  }
-}
-
-// hot_contrib[k] = contrib[hot_ids[k]] (after the previous superstep finished)
 static __global__ void k_pr_hot_pack(const float *contrib, const uint32_t *hot_ids, float *hot_contrib, uint32_t k) {
   for (uint32_t i = blockIdx.x * blockDim.x + threadIdx.x; i < k; i += gridDim.x * blockDim.x)
     hot_contrib[i] = contrib[hot_ids[i]];

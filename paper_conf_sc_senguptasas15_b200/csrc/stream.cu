@@ -134,11 +134,14 @@ gr_status stream_setup(gr_graph *g, uint64_t budget) {
   for (HostBuf *b : {&H.in_src, &H.out_dst, &H.in_w}) {
     if (!b->p || !b->bytes) continue;
     cudaError_t e = cudaHostRegister(b->p, b->bytes, cudaHostRegisterMapped);
-    if (e != cudaSuccess) {
+    if (e == cudaErrorHostMemoryAlreadyRegistered && !b->owned) {
+      cudaGetLastError();  // a borrowed buffer the caller already page-locked: used as it is
+    } else if (e != cudaSuccess) {
       cudaGetLastError();
       return fail(GR_ENOMEM, "cudaHostRegister(%zu bytes): %s", b->bytes, cudaGetErrorString(e));
+    } else {
+      b->registered = true;
     }
-    b->registered = true;
     g->pinned_bytes += b->bytes;
     void *dp = nullptr;
     SCK(cudaHostGetDevicePointer(&dp, b->p, 0));

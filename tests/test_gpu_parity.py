@@ -255,25 +255,22 @@ def test_streamed_frontier_skips_inactive_shards():
         np.testing.assert_array_equal(G.values(), d)
 
 
-@pytest.mark.parametrize("variant", ["block", "warp", "warphot", "range", "rangehot", "pipe", "seg", "seg-launches",
-                                     "seg-var0", "seg-var15"])
+@pytest.mark.parametrize("variant", ["block", "warp", "warphot", "seg", "seg-launches"])
 def test_pagerank_kernel_variants(variant, monkeypatch):
-    """Every PageRank gather variant (CTA / warp merge-path tiles, with or without
-    the shared-memory hot-source table; the edge-segmented tiles in the
-    persistent loop or one launch per phase, and its variant bits) meets the
-    PageRank bar."""
+    """Every PageRank gather the library still selects (CTA merge-path tiles when
+    no shared-memory table fits, warp merge-path tiles for small partitions, the
+    same with the hot-source table when the seg layout's indices would
+    overflow; the edge-segmented tiles in the persistent loop or one launch per
+    phase) meets the PageRank bar."""
     if variant == "seg-launches":
         monkeypatch.setenv("GR_PR_LOOP", "0")
-    elif variant.startswith("seg-var"):
-        monkeypatch.setenv("GR_PR_SEG_VAR", variant[7:])
     variant = variant.split("-")[0]
     monkeypatch.setenv("GR_PR_KERNEL", variant)
     g = grgen.rmat(17, 16, seed=12)  # > 2^20 edges so the hot table engages
     ref, _, _ = oracle.run(g.n, g.src, g.dst, "pagerank", max_iters=30)
     with gr.GraphReduce(g.n, g.src, g.dst) as G:
         st = G.run("pagerank")
-        assert st["kernel_ms"][3] == {"block": 0, "warp": 2, "warphot": 3, "range": 4,
-                                      "rangehot": 5, "pipe": 6, "seg": 7}[variant]
+        assert st["kernel_ms"][3] == {"block": 0, "warp": 2, "warphot": 3, "seg": 7}[variant]
         check_pr(G.values("pagerank"), ref, g.n)
     n, src, dst, _ = hub_graph(k=70000, extra=1_200_000)
     ref, _, _ = oracle.run(n, src, dst, "pagerank", max_iters=30)
@@ -580,3 +577,31 @@ def test_dense_tile_gather_forced(algo, force, monkeypatch):
     compare(g.n, src, dst, w, algo, loops=("auto",), directions=("pull", "auto"))
     n, s2, d2, w2 = hub_graph()
     compare(n, s2, d2, w2, algo, loops=("auto",), directions=("pull",))
+
+
+@pytest.mark.parametrize("algo", ["bfs", "sssp", "cc", "pagerank", "pagerank_delta"])
+def test_trace_detail_equals_oracle(algo):
+    """the detail columns of the trace — shards holding an
+    active vertex and distinct sources read by the gather — equal the oracle's
+    (or_run_detail, pinned by brute force), with the graph's own shard bounds."""
+    g = grgen.rmat(12, 16, seed=31)
+    src, dst = g.src, g.dst
+    if algo == "cc":
+        src, dst = np.concatenate([g.src, g.dst]), np.concatenate([g.dst, g.src])
+    w = grgen.weights(len(src), 1, 64, seed=32) if algo == "sssp" else None
+    mi = 30 if algo == "pagerank" else (40 if algo == "pagerank_delta" else 0)
+    for shard_edges in (0, 6000):
+        with gr.GraphReduce(g.n, src, dst, w, shard_edges=shard_edges) as G:
+            P = G.info()["num_shards"]
+            bounds = np.array([gr.gr_shard_info(G.h, s)["v_lo"] for s in range(P)] + [g.n], np.uint64)
+            og = oracle.OracleGraph(g.n, src, dst, w)
+            ref, rtr, rdet, rit = og.run_detail(algo, shard_bounds=bounds, source=0, max_iters=mi)
+            og.close()
+            st = G.run(algo, source=0, max_iters=mi, trace_detail=True)
+            assert st["iterations"] == rit
+            det = G.trace_detail()
+            if algo != "pagerank":
+                np.testing.assert_array_equal(G.trace(), rtr)
+            np.testing.assert_array_equal(det, rdet)
+            if shard_edges:
+                assert P > 4

@@ -695,3 +695,66 @@ def test_heat_two_vertices_closed_form():
     vals, tr, it = oracle.run(2, src, dst, "heat", w=w, source=0, max_iters=10)
     np.testing.assert_array_equal(vals, [H0 // 2 + (H0 >> 11), H0 // 2 - (H0 >> 11)])
     assert it == 10 and np.all(tr[:, 1] == 2)
+
+
+# ------------------------- detail columns of the trace: active shards and S_t
+# per superstep, the number of shards holding an active
+# vertex (what frontier skipping moves, §5.2) and the number of
+# distinct sources the gather reads. Brute force: sets over the same BSP run.
+@pytest.mark.parametrize("algo", ["bfs", "sssp", "cc", "pagerank", "pagerank_delta"])
+@pytest.mark.parametrize("seed", range(5))
+def test_trace_detail_vs_bruteforce(algo, seed):
+    rng = np.random.default_rng(1100 + seed)
+    n = int(rng.integers(2, 60))
+    src, dst, w = rand_graph(rng, n, int(rng.integers(0, 4 * n)), sym=(algo == "cc"), wmax=64)
+    P = int(rng.integers(1, 6))
+    bounds = np.unique(np.concatenate([[0, n], rng.integers(0, n, P - 1)])).astype(np.uint64)
+    mi = 7 if algo.startswith("pagerank") else 0
+    ww = w if algo == "sssp" else None
+    g = oracle.OracleGraph(n, src, dst, ww)
+    vals, tr, det, it = g.run_detail(algo, shard_bounds=bounds, source=0, max_iters=mi)
+    v2, tr2, it2 = g.run(algo, source=0, max_iters=mi)
+    g.close()
+    np.testing.assert_array_equal(tr, tr2)  # the detail run is the same run
+    ins = collections.defaultdict(list)
+    outs = collections.defaultdict(list)
+    for a, b in zip(src.tolist(), dst.tolist()):
+        ins[b].append(a)
+        outs[a].append(b)
+    # replay the frontier from the trace's own activation rule (brute force of A_t)
+    if algo == "bfs":
+        A = {0}
+    elif algo in ("sssp",):
+        A = set(outs[0])
+    else:
+        A = set(range(n))
+    shard = lambda v: int(np.searchsorted(bounds, v, side="right")) - 1
+    for t in range(it):
+        exp_shards = len({shard(v) for v in A})
+        exp_src = 0 if algo == "bfs" else len({u for v in A for u in ins[v]})
+        assert det[t, 0] == exp_shards, (t, det[t], exp_shards)
+        assert det[t, 1] == exp_src, (t, det[t], exp_src)
+        assert tr[t, 0] == len(A)
+        if t + 1 < it:
+            if algo == "pagerank":
+                A = set(range(n))
+            else:  # A_{t+1} from the changed set of t: recover C_t by re-running t+1 supersteps
+                vv, trk, _ = oracle.run(n, src, dst, algo, w=ww, source=0, max_iters=t + 1)
+                vp, _, _ = oracle.run(n, src, dst, algo, w=ww, source=0, max_iters=t) if t > 0 else (None, None, None)
+                if t == 0:
+                    if algo == "bfs":
+                        prev = np.full(n, INF, np.uint32)
+                    elif algo == "sssp":
+                        prev = np.full(n, INF, np.uint32)
+                        prev[0] = 0
+                    elif algo == "cc":
+                        prev = np.arange(n, dtype=np.uint32)
+                    else:
+                        prev = None
+                else:
+                    prev = vp
+                if prev is None:  # pagerank_delta at t = 0: R_0 = fp32(floor(2^62/n) 2^-62)
+                    r0 = np.float32(float((1 << 62) // n) * 2.0 ** -62)
+                    prev = np.full(n, r0, np.float32)
+                C = set(np.nonzero(vv != prev)[0].tolist())
+                A = {x for u in C for x in outs[u]}
