@@ -109,8 +109,13 @@ struct NcclComm : Comm {
     return GR_OK;
   }
   gr_status barrier(cudaStream_t s) override {
+    if (!comm) return GR_ENCCL;
     uint64_t *w = d_small + 8ull * world;
     return ncclAllReduce(w, w, 1, ncclUint64, ncclSum, comm, s) == ncclSuccess ? GR_OK : GR_ENCCL;
+  }
+  void abort_group() override {
+    if (comm) ncclCommAbort(comm);
+    comm = nullptr;
   }
 };
 
@@ -209,6 +214,8 @@ struct SimComm : Comm {
     if (cudaStreamSynchronize(s) != cudaSuccess) return fail_all(GR_ECUDA);
     return grp->barrier() ? GR_OK : GR_ENCCL;
   }
+  void abort_group() override { grp->poison(); }
+  bool own_context() const override { return false; }  // threads of one process share a context
 };
 
 // ------------------------------------------------- process-shared memory
@@ -378,6 +385,7 @@ struct ShmComm : Comm {
     if (cudaStreamSynchronize(s) != cudaSuccess) return fail_all(GR_ECUDA);
     return host_barrier() ? GR_OK : GR_ENCCL;
   }
+  void abort_group() override { h->poisoned.store(1); }
 };
 
 static gr_status shm_create(int world, int rank, const void *id128, ShmComm **out, std::string *err) {

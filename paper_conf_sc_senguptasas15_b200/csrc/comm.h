@@ -47,6 +47,15 @@ struct Comm {
   // rank's work enqueued before its barrier has completed (so peer stores of
   // those kernels are visible). NCCL: a one-word allreduce; simulated: host.
   virtual gr_status barrier(cudaStream_t s) = 0;
+  // A rank that fails between collectives: make the peers' pending and next
+  // collectives fail instead of waiting for it (NCCL: ncclCommAbort; shared
+  // memory and simulated groups: the group is poisoned). The graph must be freed.
+  virtual void abort_group() = 0;
+  // Whether every rank runs in a CUDA context of its own (a process per rank). Kernels
+  // that spin on a peer's stores (the device-side count exchange and barrier) need it:
+  // streams of ONE context may share a hardware queue, so a spinning kernel could sit
+  // in front of the very kernel it waits for (simulated ranks use the host paths).
+  virtual bool own_context() const { return true; }
 };
 
 // Create the communicator for a loaded partition. world <= 1 returns nullptr.

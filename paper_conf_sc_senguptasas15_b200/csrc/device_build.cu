@@ -227,6 +227,52 @@ static gr_status scan_offsets(gr_graph *g, const uint32_t *deg, uint64_t n, OffT
   return GR_OK;
 }
 
+// destination of every CSC position: the v with in_off[v] <= e < in_off[v+1]
+template <class OffT>
+static __global__ void k_csc_dst(const OffT *in_off, uint64_t n, uint64_t m, uint32_t *dst) {
+  for (uint64_t e = blockIdx.x * (uint64_t)blockDim.x + threadIdx.x; e < m; e += (uint64_t)gridDim.x * blockDim.x) {
+    uint64_t lo = 0, hi = n;  // last v with in_off[v] <= e
+    while (hi - lo > 1) {
+      const uint64_t mid = (lo + hi) >> 1;
+      if ((uint64_t)in_off[mid] <= e) lo = mid;
+      else hi = mid;
+    }
+    dst[e] = (uint32_t)lo;
+  }
+}
+
+// CSR (activation) = transpose of the CSC: a stable sort of the CSC's sources
+// (32-bit keys, `bits` wide) carrying the destinations. The CSC is ordered by
+// (dst, src, w), so each CSR segment comes out ordered by dst — the host
+// builder's layout exactly (tests/test_gpu_parity.py).
+template <class OffT> static gr_status build_csr(gr_graph *g) {
+  const uint64_t n = g->H.n, m = g->H.m_in;
+  cudaStream_t s = g->stream;
+  uint32_t *d_dst = nullptr, *kscratch = nullptr;
+  void *tmp = nullptr;
+  size_t need = 0;
+  DCK(pmalloc(&d_dst, 4 * std::max<uint64_t>(m, 1), s));
+  DCK(pmalloc(&kscratch, 4 * std::max<uint64_t>(m, 1), s));
+  k_csc_dst<OffT><<<g->num_sms * 8, 256, 0, s>>>((const OffT *)g->in_off, n, m, d_dst);
+  DCK(cub::DeviceRadixSort::SortPairs(nullptr, need, g->in_src, kscratch, d_dst, g->out_dst, (int64_t)m, 0,
+                                      (int)g->csr_bits, s));
+  DCK(pmalloc(&tmp, std::max<size_t>(need, 16), s));
+  DCK(cub::DeviceRadixSort::SortPairs(tmp, need, g->in_src, kscratch, d_dst, g->out_dst, (int64_t)m, 0,
+                                      (int)g->csr_bits, s));
+  pfree(tmp, s);
+  pfree(kscratch, s);
+  pfree(d_dst, s);
+  DCK(cudaStreamSynchronize(s));
+  g->csr_pending = false;
+  tmark("device build: CSR sort (first run that activates)");
+  return GR_OK;
+}
+
+gr_status ensure_csr(gr_graph *g) {
+  if (!g->csr_pending) return GR_OK;
+  return g->off64 ? build_csr<uint64_t>(g) : build_csr<uint32_t>(g);
+}
+
 template <class OffT>
 static gr_status build_typed(gr_graph *g, const uint32_t *d_src, uint32_t *d_dst, const uint32_t *d_w,
                              uint64_t n, uint64_t m, uint32_t *d_indeg, uint32_t *d_outdeg, cudaStream_t s) {
@@ -244,25 +290,13 @@ static gr_status build_typed(gr_graph *g, const uint32_t *d_src, uint32_t *d_dst
   if ((st = sort_edges(g, d_dst, d_src, d_w, m, bits, g->in_src, d_w ? g->in_w : nullptr, d_dst, s)) != GR_OK)
     return st;
   tmark("device build: CSC sort");
-  // CSR (activation) = transpose of the CSC: a stable sort of the CSC's sources
-  // (32-bit keys, `bits` wide) carrying the destinations. The CSC is ordered by
-  // (dst, src, w), so each CSR segment comes out ordered by dst.
+  // The activation CSR's payload (out_dst) is built on the first run that needs
+  // it (ensure_csr): PageRank eliminates FrontierActivate (L274) and never does,
+  // so a load followed by PageRank skips one of the two sorts.
   if ((st = dev_alloc(g, (void **)&g->out_dst, 4 * (m + 4))) != GR_OK) return st;
   DCK(cudaMemsetAsync(g->out_dst + m, 0, 16, s));
-  {
-    uint32_t *kscratch = nullptr;
-    void *tmp = nullptr;
-    size_t need = 0;
-    DCK(pmalloc(&kscratch, 4 * std::max<uint64_t>(m, 1), s));
-    DCK(cub::DeviceRadixSort::SortPairs(nullptr, need, g->in_src, kscratch, d_dst, g->out_dst, (int64_t)m, 0,
-                                        (int)bits, s));
-    DCK(pmalloc(&tmp, std::max<size_t>(need, 16), s));
-    DCK(cub::DeviceRadixSort::SortPairs(tmp, need, g->in_src, kscratch, d_dst, g->out_dst, (int64_t)m, 0,
-                                        (int)bits, s));
-    pfree(tmp, s);
-    pfree(kscratch, s);
-  }
-  tmark("device build: CSR sort");
+  g->csr_pending = true;
+  g->csr_bits = bits;
   // offsets
   if ((st = dev_alloc(g, &g->in_off, sizeof(OffT) * (n + 1))) != GR_OK) return st;
   if ((st = dev_alloc(g, &g->out_off, sizeof(OffT) * (n + 1))) != GR_OK) return st;

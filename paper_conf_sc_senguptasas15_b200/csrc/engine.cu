@@ -1004,7 +1004,9 @@ template <class OffT>
 using SegLoopKernel = void (*)(const PrArgs<OffT>, const PrLoop);
 // The seg kernels are instantiated for the default variant bits only (the other
 // combinations were measured in round 1 and are not built: profiles/README.md)
-template <class OffT> static SegLoopKernel<OffT> seg_loop_kernel(int) { return k_pr_seg_loop<OffT, kSegDefaultVar>; }
+template <class OffT> static SegLoopKernel<OffT> seg_loop_kernel(int, bool phases = false) {
+  return phases ? k_pr_seg_loop<OffT, kSegDefaultVar, true> : k_pr_seg_loop<OffT, kSegDefaultVar, false>;
+}
 template <class OffT> static SegKernel<OffT> seg_kernel(int) { return k_pr_seg<OffT, kSegDefaultVar>; }
 
 // Source-blocked layout for k_pr_bseg_loop (once per graph):
@@ -1367,7 +1369,10 @@ static gr_status run_pagerank(gr_graph *g, const gr_run_opts *o, cudaStream_t s,
     k_pr_hot_pack<<<(g->hot_k + 255) / 256, 256, 0, s>>>(g->contrib[0], g->hot_ids, g->hot_buf[0], g->hot_k);
     if (prof) CK(cudaEventRecord(g->prof_ev[0], s));
     void *args[] = {(void *)&a, (void *)&L};
-    CK(cudaLaunchCooperativeKernel((const void *)seg_loop_kernel<OffT>(g->seg_var), dim3(g->hot_grid),
+    if (phases)
+      CK(cudaFuncSetAttribute(seg_loop_kernel<OffT>(g->seg_var, true), cudaFuncAttributeMaxDynamicSharedMemorySize,
+                              (int)g->hot_smem));
+    CK(cudaLaunchCooperativeKernel((const void *)seg_loop_kernel<OffT>(g->seg_var, phases), dim3(g->hot_grid),
                                    dim3(g->hot_cta), args, g->hot_smem, s));
     if (prof) CK(cudaEventRecord(g->prof_ev[1], s));
     CK(cudaStreamSynchronize(s));
@@ -1493,6 +1498,10 @@ gr_status run(gr_graph *g, const gr_run_opts *oin, gr_run_stats *st) {
     k_prd_div<<<g->num_sms * 4, 256, 0, g->stream>>>(g->H.n, g->d_outdeg, g->prd_div);
     CK(cudaGetLastError());
     CK(cudaStreamSynchronize(g->stream));
+  }
+  if (o.algo != GR_PAGERANK) {  // every program but PageRank activates along the out-edges
+    gr_status cs = ensure_csr(g);
+    if (cs != GR_OK) return cs;
   }
   if (g->mode == GR_MODE_STREAMED) return run_streamed(g, &o, st);
   cudaStream_t s = o.stream ? (cudaStream_t)o.stream : g->stream;

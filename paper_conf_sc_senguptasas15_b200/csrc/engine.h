@@ -53,6 +53,8 @@ struct gr_graph {
   uint32_t *static_chk_h = nullptr, *static_chk_c = nullptr;
   uint32_t n_static_chunks = 0, hub_cap = 0;
   bool dev_built = false;        // layout built on the GPU (device_build.cu)
+  bool csr_pending = false;      // device build: out_dst not sorted yet (ensure_csr on first need)
+  uint32_t csr_bits = 32;
   uint64_t dev_hubs_in = 0, dev_chunks_in = 0, dev_hubs_out = 0, dev_chunks_out = 0;
 
   // frontier-program state
@@ -228,6 +230,7 @@ inline void pfree(void *p, cudaStream_t s) {
 }
 gr_status load_device(gr_graph *g);
 gr_status device_build(gr_graph *g, const gr_edges *E, uint64_t shard_edges);
+gr_status ensure_csr(gr_graph *g);  // device-built graphs: the activation CSR payload, built lazily
 gr_status select_hot(gr_graph *g, uint64_t K, uint32_t **hot_ids, uint32_t *hot_k, uint32_t **d_slot);
 // partitioned PageRank (engine.cu): kernel/layout selection once per graph, one superstep's launches
 gr_status pr_part_prepare(gr_graph *g);

@@ -99,7 +99,7 @@ gr_status part_setup(gr_graph *g) {
         // device, where a peer's wait kernel may be spinning on this rank's next publish
         if ((a = dev_alloc(g, (void **)&g->d_xc_peer, sizeof(void *) * 16)) != GR_OK) return a;
         if (cudaMemcpy(g->d_xc_peer, g->xc_peer, sizeof(void *) * 16, cudaMemcpyHostToDevice) != cudaSuccess ||
-            cudaMallocHost((void **)&g->h_xbytes, 16) != cudaSuccess)
+            cudaMallocHost((void **)&g->h_xbytes, 32) != cudaSuccess)
           return fail(GR_ECUDA, "count exchange setup");
         g->xc_ok = true;
       } else if (c != GR_EUNSUPPORTED) {
@@ -208,13 +208,23 @@ static __global__ void k_part_publish(Ctl *ctl, XCount *const *peers, uint32_t r
   *(volatile uint32_t *)&X->seq[par][rank] = seq;
 }
 
+constexpr unsigned long long kSpinLimitNs = 60ull * 1000000000ull;  // 60 s without a peer's count
 static __global__ void k_part_wait(Ctl *ctl, XCount *mine, XDev *xd, uint32_t rank, uint32_t world, uint32_t t,
                                    uint32_t seq) {
   const uint32_t q = threadIdx.x, par = t & 1u;
   if (ctl->stop) return;  // uniform: every lane reads the same flag
   unsigned long long c = 0, a = 0;
   if (q < world) {
-    while (*(volatile uint32_t *)&mine->seq[par][q] != seq) __nanosleep(64);
+    // a peer that never publishes (it failed, or its process died) must not hang this
+    // GPU: after kSpinLimitNs the run stops with XDev::timeout set (the host reports it)
+    const unsigned long long t0 = gtimer();
+    while (*(volatile uint32_t *)&mine->seq[par][q] != seq) {
+      __nanosleep(64);
+      if (gtimer() - t0 > kSpinLimitNs) {
+        atomicExch(&xd->timeout, ((unsigned long long)q << 32) | seq);
+        break;
+      }
+    }
     __threadfence_system();
     c = *(volatile unsigned long long *)&mine->cnt[par][q][0];
     a = *(volatile unsigned long long *)&mine->cnt[par][q][1];
@@ -236,7 +246,7 @@ static __global__ void k_part_wait(Ctl *ctl, XCount *mine, XDev *xd, uint32_t ra
     xd->tot = (uint32_t)tot;
     xd->bytes_in += 8ull * peer_c;
     ctl->cnt_C = 0;  // this rank's C list is refilled from the exchanged set by the classify
-    if (act == 0) ctl->stop = 1u;
+    if (act == 0 || xd->timeout) ctl->stop = 1u;
   }
 }
 
@@ -249,8 +259,10 @@ static __global__ void k_xbar(uint32_t *const *peers, uint32_t *mine, uint32_t r
   const uint32_t q = threadIdx.x;
   __threadfence_system();
   if (q < world) *(volatile uint32_t *)(peers[q] + rank) = seq;
-  if (q < world)
-    while (*(volatile uint32_t *)(mine + q) < seq) __nanosleep(32);
+  if (q < world) {
+    const unsigned long long t0 = gtimer();
+    while (*(volatile uint32_t *)(mine + q) < seq && gtimer() - t0 < kSpinLimitNs) __nanosleep(32);
+  }
   __threadfence_system();
   __syncwarp();
 }
@@ -370,7 +382,7 @@ gr_status run_frontier_part(gr_graph *g, const gr_run_opts *o, cudaStream_t s, g
   // device-side count exchange (default with the fused exchange): no host
   // synchronisation per superstep; the host enqueues supersteps in batches and
   // reads the stop flag the wait kernels set once per batch
-  bool dx = fx && g->xc_ok;
+  bool dx = fx && g->xc_ok && C->own_context();
   if (const char *e = getenv("GR_COUNT_EXCHANGE")) dx = dx && std::string(e) != "host";
   if (dx) {
     const uint32_t batch = 8;
@@ -419,8 +431,16 @@ gr_status run_frontier_part(gr_graph *g, const gr_run_opts *o, cudaStream_t s, g
       if (g->h_ctl->stop || (o->max_iters != 0 && t >= o->max_iters)) break;
     }
     PCK(cudaMemcpyAsync(g->h_xbytes + 1, &xd->bytes_in, 8, cudaMemcpyDeviceToHost, s));
+    PCK(cudaMemcpyAsync(g->h_xbytes + 2, &xd->timeout, 8, cudaMemcpyDeviceToHost, s));
     PCK(cudaStreamSynchronize(s));
     C->bytes_in += g->h_xbytes[1] - g->h_xbytes[0];
+    if (g->h_xbytes[2]) {
+      const unsigned long long tv = g->h_xbytes[2];
+      PCK(cudaMemsetAsync(&xd->timeout, 0, 8, s));
+      return fail(GR_ENCCL, "count exchange: rank %d waited %llu s for rank %u's counts of superstep seq %u "
+                  "(peer failed or stalled)", C->rank, kSpinLimitNs / 1000000000ull, (unsigned)(tv >> 32),
+                  (unsigned)tv);
+    }
     t = g->h_ctl->iter;  // supersteps that ran (the stopped one, if any, did not count)
   }
   while (!dx && (o->max_iters == 0 || t < o->max_iters)) {
@@ -529,7 +549,7 @@ gr_status run_pagerank_part(gr_graph *g, const gr_run_opts *o, cudaStream_t s, g
   k_pr_init<<<g->num_sms * 4, 256, 0, s>>>((uint32_t)g->H.n, g->inv_outdeg, g->contrib[0]);
   // stream-ordered barrier between supersteps: on the device (k_xbar over the
   // mapped arrival words, default) or the communicator's (NCCL allreduce / host)
-  bool dbar = g->xbar_ok;
+  bool dbar = g->xbar_ok && C->own_context();
   if (const char *x = getenv("GR_PR_BARRIER")) dbar = dbar && std::string(x) != "comm";
   auto barrier = [&]() -> gr_status {
     if (!dbar) return C->barrier(s);
@@ -599,10 +619,21 @@ gr_status part_fetch_trace(gr_graph *g, uint64_t *dst, uint64_t max_rows, uint64
   }
   std::vector<uint64_t> cnt(C->world, 32 * r), dsp(C->world);
   for (int q = 0; q < C->world; q++) dsp[q] = 32 * r * q;
+  // local steps first, then one agreed flag: a rank that failed here must not leave the
+  // others waiting in the allgatherv (every rank takes the same collective sequence)
   char *base = nullptr;
-  PCK(cudaMalloc((void **)&base, 32 * std::max<uint64_t>(r, 1) * C->world));
-  PCK(cudaStreamSynchronize(g->stream));  // the trace of the last run is complete
-  PCK(cudaMemcpyAsync(base + 32 * r * C->rank, g->trace, 32 * r, cudaMemcpyDeviceToDevice, g->stream));
+  uint64_t ok = cudaMalloc((void **)&base, 32 * std::max<uint64_t>(r, 1) * C->world) == cudaSuccess &&
+                cudaStreamSynchronize(g->stream) == cudaSuccess &&  // the trace of the last run is complete
+                cudaMemcpyAsync(base + 32 * r * C->rank, g->trace, 32 * r, cudaMemcpyDeviceToDevice,
+                                g->stream) == cudaSuccess;
+  if (!ok) cudaGetLastError();
+  std::vector<uint64_t> oks(C->world);
+  XCK(C->allgather_small(&ok, 1, oks.data(), g->stream));
+  for (int q = 0; q < C->world; q++)
+    if (!oks[q]) {
+      if (base) cudaFree(base);
+      return fail(GR_ECUDA, "trace exchange: rank %d failed locally", q);
+    }
   gr_status xs = C->allgatherv(base + 32 * r * C->rank, base, cnt, dsp, g->stream);
   std::vector<uint64_t> all(4 * r * C->world);
   cudaError_t ce = cudaStreamSynchronize(g->stream);
@@ -623,12 +654,19 @@ gr_status part_fetch_trace(gr_graph *g, uint64_t *dst, uint64_t max_rows, uint64
 }
 
 gr_status run_part(gr_graph *g, const gr_run_opts *o, cudaStream_t s, gr_run_stats *st) {
-  if (o->algo == GR_PAGERANK)
-    return g->off64 ? run_pagerank_part<uint64_t>(g, o, s, st) : run_pagerank_part<uint32_t>(g, o, s, st);
-  ProgDesc D;
-  gr_status r = prog_desc(o->algo, o->custom_id, &D);
-  if (r != GR_OK) return r;
-  return g->off64 ? run_frontier_part<uint64_t>(g, o, s, st, D) : run_frontier_part<uint32_t>(g, o, s, st, D);
+  gr_status r;
+  if (o->algo == GR_PAGERANK) {
+    r = g->off64 ? run_pagerank_part<uint64_t>(g, o, s, st) : run_pagerank_part<uint32_t>(g, o, s, st);
+  } else {
+    ProgDesc D;
+    r = prog_desc(o->algo, o->custom_id, &D);
+    if (r == GR_OK)
+      r = g->off64 ? run_frontier_part<uint64_t>(g, o, s, st, D) : run_frontier_part<uint32_t>(g, o, s, st, D);
+  }
+  // a rank that fails mid-run (a launch error, a local allocation) aborts the group, so
+  // its peers return errors from their next collective instead of waiting forever
+  if (r != GR_OK) g->comm->abort_group();
+  return r;
 }
 
 }  // namespace gr

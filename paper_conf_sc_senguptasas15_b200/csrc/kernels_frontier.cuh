@@ -1751,6 +1751,7 @@ struct XDev {
   XRanges R;
   uint32_t tot;                 // global |C_t|
   unsigned long long bytes_in;  // changed-set bytes received from peers (stats)
+  unsigned long long timeout;   // (rank << 32 | seq) of a count that never arrived (0: none)
 };
 
 // Partitioned runs: split the exchanged changed set (every rank's C_t) into

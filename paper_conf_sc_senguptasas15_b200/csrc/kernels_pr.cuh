@@ -744,7 +744,7 @@ __device__ __forceinline__ void pr_apply_fixup(const PrArgs<OffT> &a, const PrLo
   }
 }
 
-template <class OffT, int kVar>
+template <class OffT, int kVar, bool kPhases = false>
 __global__ void __launch_bounds__(1024, 1) k_pr_seg_loop(const __grid_constant__ PrArgs<OffT> a0,
                                                         const __grid_constant__ PrLoop L) {
   extern __shared__ __align__(16) float s_hot[];
@@ -754,8 +754,8 @@ __global__ void __launch_bounds__(1024, 1) k_pr_seg_loop(const __grid_constant__
   const uint32_t stride = gridDim.x * nw;
   const uint4 *src4 = reinterpret_cast<const uint4 *>(L.seg_src) + 2 * lane;
   const uint64_t gtid = blockIdx.x * (uint64_t)blockDim.x + threadIdx.x, gthreads = (uint64_t)gridDim.x * blockDim.x;
-  const bool stamp = L.ts && blockIdx.x == 0 && threadIdx.x == 0;
-  if (stamp) L.ts[0] = gtimer();
+  // kPhases (GR_PR_PHASES=1, a separate instantiation): CTA 0 stamps %globaltimer
+  if (kPhases && blockIdx.x == 0 && threadIdx.x == 0) L.ts[0] = gtimer();
   for (uint32_t t = 0; t < L.iters; t++) {
     PrArgs<OffT> a = a0;
     a.contrib_in = L.contrib[t & 1];
@@ -798,7 +798,7 @@ __global__ void __launch_bounds__(1024, 1) k_pr_seg_loop(const __grid_constant__
       }
     }
     pr_grid_sync(L.bar);
-    if (stamp) L.ts[1 + 2 * t] = gtimer();
+    if (kPhases && blockIdx.x == 0 && threadIdx.x == 0) L.ts[1 + 2 * t] = gtimer();
     // ---- phase 2: rows split between tiles, hot-table pack
     for (uint64_t c = gtid; c < L.num_tiles; c += gthreads) {
       const uint32_t row = a.head_row[c];
@@ -820,7 +820,7 @@ __global__ void __launch_bounds__(1024, 1) k_pr_seg_loop(const __grid_constant__
       for (uint64_t k = gtid; k < L.hot_k; k += gthreads)
         if (!L.hot_split[k]) hot_next[k] = a.contrib_out[L.hot_ids[k]];
     pr_grid_sync(L.bar);
-    if (stamp) L.ts[2 + 2 * t] = gtimer();
+    if (kPhases && blockIdx.x == 0 && threadIdx.x == 0) L.ts[2 + 2 * t] = gtimer();
   }
 }
 

@@ -66,7 +66,7 @@ CASES = {
 
 
 @pytest.mark.timeout(900)
-@pytest.mark.parametrize("exchange", ["fused", "allgatherv"])
+@pytest.mark.parametrize("exchange", ["fused", "fused-hostcounts", "allgatherv"])
 @pytest.mark.parametrize("algo", list(CASES))
 def test_two_processes_equal_oracle(tmp_path, algo, exchange):
     g, kind = CASES[algo]()
@@ -75,7 +75,11 @@ def test_two_processes_equal_oracle(tmp_path, algo, exchange):
         src, dst = np.concatenate([g.src, g.dst]), np.concatenate([g.dst, g.src])
     if kind == "w":
         w = grgen.weights(g.m, 1, 64, seed=9)
-    env = {"GR_FRONTIER_EXCHANGE": "nccl", "GR_PR_EXCHANGE": "nccl"} if exchange == "allgatherv" else {}
+    # fused: changed sets stored into the peers by the gather, counts exchanged and the
+    # PageRank supersteps separated on the device (k_part_publish / k_part_wait / k_xbar);
+    # fused-hostcounts: the counts allgathered through the host, the communicator's barrier
+    env = {"GR_FRONTIER_EXCHANGE": "nccl", "GR_PR_EXCHANGE": "nccl"} if exchange == "allgatherv" else \
+        {"GR_COUNT_EXCHANGE": "host", "GR_PR_BARRIER": "comm"} if exchange == "fused-hostcounts" else {}
     mi = 30 if algo == "pagerank" else 0
     ref, rtr, rit = oracle.run(g.n, src, dst, algo, w=w, source=0, max_iters=mi)
     res = run_ranks(tmp_path, g.n, src, dst, w, algo, source=0, max_iters=mi, env=env)
@@ -95,7 +99,7 @@ def test_two_processes_equal_oracle(tmp_path, algo, exchange):
                     ref_ = ref
                 np.testing.assert_array_equal(vals, ref_)
                 np.testing.assert_array_equal(r["tr"][k], rtr)
-        if exchange == "fused" and algo != "pagerank":
+        if exchange.startswith("fused") and algo != "pagerank":
             assert r["st"][0]["bytes_nvlink"] > 0  # the peers' changed sets arrived
     assert owned == g.n
 
