@@ -568,6 +568,9 @@ static gr_status get_while_graph(gr_graph *g, int key, cudaGraphExec_t *out, uin
 // source its gather reads, then count both sets. A_t is the implicit owned range
 // (superstep 0 of kInitAll programs), the vertices with a marked in-neighbour
 // (dense supersteps), or the A lists (listA + listH). Diagnostic: host loop only.
+// BFS (no gather, apply-only): its A lists hold only the unvisited
+// activated vertices, so A_t is recovered from the depths instead — v ∈ A_t iff
+// an in-neighbour has depth t-1 (C_{t-1}: the vertices reached at t-1), A_0 = {source}.
 template <class OffT>
 static __global__ void k_detail_mark(const __grid_constant__ Part<OffT> P, int has_gather, const uint64_t *sb,
                                      uint32_t nsb, uint32_t *src_bits, uint32_t *shard_bits) {
@@ -575,14 +578,19 @@ static __global__ void k_detail_mark(const __grid_constant__ Part<OffT> P, int h
   load_view(P.ctl, V);
   if (V.stop) return;
   const uint32_t t = V.t, slot = t & 1u;
-  const bool implicit = V.dense || (V.implicit0 && t == 0);
+  const bool bfs = !has_gather;
+  const bool implicit = bfs || V.dense || (V.implicit0 && t == 0);
   const uint32_t *bits = P.cbits[slot ^ 1u];
   const uint64_t nA = V.cntA[slot], total = implicit ? (uint64_t)P.own_n : nA + V.cntH[slot];
   for (uint64_t i = blockIdx.x * (uint64_t)blockDim.x + threadIdx.x; i < total; i += (uint64_t)gridDim.x * blockDim.x) {
     const uint32_t v = implicit ? P.own_lo + (uint32_t)i : (i < nA ? P.listA[slot][i] : P.listH[slot][i - nA]);
     const uint32_t lv = v - P.own_lo;
     const uint64_t b = (uint64_t)P.in_off[lv], e = (uint64_t)P.in_off[lv + 1];
-    if (V.dense) {
+    if (bfs) {
+      bool act = t == 0 ? v == V.source : false;
+      for (uint64_t k = b; k < e && !act && t > 0; k++) act = ld_cg(P.val + P.in_src[k]) == t - 1;
+      if (!act) continue;
+    } else if (V.dense) {
       bool act = false;
       for (uint64_t k = b; k < e && !act; k++) act = test_bit_cg(bits, P.in_src[k]);
       if (!act) continue;

@@ -133,9 +133,25 @@ gr_status stream_setup(gr_graph *g, uint64_t budget) {
   // page-lock the host payloads for DMA
   for (HostBuf *b : {&H.in_src, &H.out_dst, &H.in_w}) {
     if (!b->p || !b->bytes) continue;
+    if (!b->owned) {  // a borrowed buffer the caller already page-locked (cudaHostAlloc / torch pinned): as is
+      cudaPointerAttributes pa{};
+      if (cudaPointerGetAttributes(&pa, b->p) == cudaSuccess && pa.type == cudaMemoryTypeHost) {
+        g->pinned_bytes += b->bytes;
+        void *dp = pa.devicePointer;
+        if (!dp && cudaHostGetDevicePointer(&dp, b->p, 0) != cudaSuccess) {
+          cudaGetLastError();
+          return fail(GR_EUNSUPPORTED, "borrowed pinned buffer is not mapped into the device address space");
+        }
+        if (b == &H.in_src) S->zc_in = (const uint32_t *)dp;
+        else if (b == &H.out_dst) S->zc_out = (const uint32_t *)dp;
+        else S->zc_w = (const uint8_t *)dp;
+        continue;
+      }
+      cudaGetLastError();
+    }
     cudaError_t e = cudaHostRegister(b->p, b->bytes, cudaHostRegisterMapped);
     if (e == cudaErrorHostMemoryAlreadyRegistered && !b->owned) {
-      cudaGetLastError();  // a borrowed buffer the caller already page-locked: used as it is
+      cudaGetLastError();  // registered by the caller in the meantime: used as it is
     } else if (e != cudaSuccess) {
       cudaGetLastError();
       return fail(GR_ENOMEM, "cudaHostRegister(%zu bytes): %s", b->bytes, cudaGetErrorString(e));
