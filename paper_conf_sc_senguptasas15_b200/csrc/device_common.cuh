@@ -143,8 +143,6 @@ template <class OffT> struct Part {
   uint32_t *val;          // [n] vertex values (replica of superstep t-1; BSP read side)
   uint32_t *stamp;        // [own_n] activation epoch per owned vertex (dedup)
   uint32_t *listA[2];     // non-hub A lists (owned ids, global)
-  uint32_t *listAb[2], *listAd[2];  // carry (gather programs, 32-bit offsets): each entry's CSC begin and in-degree
-  uint32_t carry;         // 1: the A-list producers write listAb / listAd and the sparse gathers read them
   uint32_t *listH[2];     // hub A lists
   uint32_t *C_v, *C_val;  // changed list (non-hub)
   uint32_t *CH_v, *CH_val;// changed list (activation hubs)
@@ -248,10 +246,6 @@ struct WarpQueue {
   uint32_t *s_a;   // [kQueueCap] shared
   uint32_t *s_b;   // [kQueueCap] shared or nullptr (pair lists)
   uint32_t n;      // warp-uniform fill level
-  // A lists that carry each entry's CSC range (Part::carry): s_b / s_c hold (beg, deg),
-  // flushed to ab / ad at the entry's list position (nullptr: not carried)
-  uint32_t *s_c = nullptr;
-  uint32_t *ab = nullptr, *ad = nullptr;
   // optional mirrors (partitioned frontier exchange fused into the gather): every
   // flushed entry at list position p is also stored at mir_off + p of each mirror
   uint32_t *const *mir_a = nullptr;
@@ -272,7 +266,6 @@ struct WarpQueue {
     for (uint32_t i = lane_id(); i < n; i += 32) {
       g_a[base + i] = s_a[i];
       if (g_b) g_b[base + i] = s_b[i];
-      if (ab) { ab[base + i] = s_b[i]; ad[base + i] = s_c[i]; }
       if (n_mir) mirror(base + i, s_a[i], s_b[i]);
     }
     __syncwarp();
@@ -294,25 +287,10 @@ struct WarpQueue {
     for (uint32_t i = threadIdx.x & 31; i < n; i += 32) {
       g_a[base + i] = s_a[i];
       if (g_b) g_b[base + i] = s_b[i];
-      if (ab) { ab[base + i] = s_b[i]; ad[base + i] = s_c[i]; }
       if (n_mir) mirror(base + i, s_a[i], s_b[i]);
     }
     __syncwarp();
     n = 0;
-  }
-  // push of an A-list entry with its CSC range (stored only when the queue carries)
-  __device__ void push_a(bool p, uint32_t a, uint32_t beg, uint32_t deg, uint32_t *g_a, uint32_t *g_cnt) {
-    uint32_t mask = __ballot_sync(0xffffffffu, p);
-    if (mask == 0) return;
-    uint32_t k = __popc(mask);
-    if (n + k > (uint32_t)kQueueCap) flush(g_a, nullptr, g_cnt);
-    if (p) {
-      uint32_t pos = n + __popc(mask & lanemask_lt());
-      s_a[pos] = a;
-      if (ab) { s_b[pos] = beg; s_c[pos] = deg; }
-    }
-    n += k;
-    __syncwarp();
   }
   __device__ void push(bool p, uint32_t a, uint32_t b, uint32_t *g_a, uint32_t *g_b, uint32_t *g_cnt) {
     uint32_t mask = __ballot_sync(0xffffffffu, p);

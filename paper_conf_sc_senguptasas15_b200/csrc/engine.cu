@@ -214,8 +214,6 @@ gr_status load_device(gr_graph *g) {
   for (int i = 0; i < 2; i++) {
     if ((s = dev_alloc(g, (void **)&g->listA[i], 4 * ow)) != GR_OK) return s;
     if ((s = dev_alloc(g, (void **)&g->listH[i], 4 * ow)) != GR_OK) return s;
-    if ((s = dev_alloc(g, (void **)&g->listAb[i], 4 * ow)) != GR_OK) return s;
-    if ((s = dev_alloc(g, (void **)&g->listAd[i], 4 * ow)) != GR_OK) return s;
   }
   // changed lists: owned vertices only, except in partitioned runs where the
   // exchanged changed set of every rank is classified into them

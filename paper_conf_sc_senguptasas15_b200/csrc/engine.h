@@ -60,7 +60,6 @@ struct gr_graph {
   // frontier-program state
   uint32_t *val = nullptr, *stamp = nullptr;
   uint32_t *listA[2] = {nullptr, nullptr}, *listH[2] = {nullptr, nullptr};
-  uint32_t *listAb[2] = {nullptr, nullptr}, *listAd[2] = {nullptr, nullptr};  // carried CSC ranges
   uint32_t *C_v = nullptr, *C_val = nullptr, *CH_v = nullptr, *CH_val = nullptr;
   gr::Ctl *ctl = nullptr;
   gr::Ctl *h_ctl = nullptr;      // pinned mirror
@@ -189,13 +188,6 @@ template <class OffT> inline Part<OffT> make_part(gr_graph *g) {
   P.val = g->val;
   P.stamp = g->stamp;
   for (int i = 0; i < 2; i++) { P.listA[i] = g->listA[i]; P.listH[i] = g->listH[i]; }
-  for (int i = 0; i < 2; i++) { P.listAb[i] = g->listAb[i]; P.listAd[i] = g->listAd[i]; }
-  {
-    // A lists carry each entry's CSC range (one dependent load less in the sparse gathers)
-    // when the offsets are 32-bit; GR_CARRY=0 turns it off (A/B)
-    static const int carry_env = getenv("GR_CARRY") ? atoi(getenv("GR_CARRY")) : 1;
-    P.carry = (g->listAb[0] && !g->off64 && carry_env) ? 1u : 0u;
-  }
   P.C_v = g->C_v; P.C_val = g->C_val; P.CH_v = g->CH_v; P.CH_val = g->CH_val;
   for (int i = 0; i < 2; i++) { P.chkA_h[i] = g->chkA_h[i]; P.chkA_c[i] = g->chkA_c[i]; }
   P.chkC_h = g->chkC_h; P.chkC_c = g->chkC_c;

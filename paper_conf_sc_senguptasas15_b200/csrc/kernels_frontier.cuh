@@ -324,18 +324,10 @@ __device__ __forceinline__ uint32_t activate_batch(const Part<OffT> &P, const bo
                                                    const uint32_t *hub_bits, WarpQueue &qA, uint32_t slot) {
   uint32_t st[kBatch];
   bool hb[kBatch];
-  // carried A lists (gather programs): each entry's CSC range, loaded with the stamp read
-  // (no extra hop here) so the next superstep's gather skips its offsets load
-  const bool carry = !kByOut && qA.s_c != nullptr && P.carry;
-  qA.ab = carry ? P.listAb[slot] : nullptr;
-  qA.ad = carry ? P.listAd[slot] : nullptr;
-  uint32_t ob[kBatch], oe[kBatch];
 #pragma unroll
   for (int q = 0; q < kBatch; q++) {
     st[q] = act[q] ? ld_cg(P.stamp + (x[q] - P.own_lo)) : epoch;
     hb[q] = act[q] && test_bit(hub_bits, kByOut ? x[q] : x[q] - P.own_lo);  // issued with the stamp read
-    ob[q] = (carry && act[q]) ? (uint32_t)P.in_off[x[q] - P.own_lo] : 0u;
-    oe[q] = (carry && act[q]) ? (uint32_t)P.in_off[x[q] - P.own_lo + 1] : 0u;
   }
   bool nw[kBatch];
 #pragma unroll
@@ -354,7 +346,7 @@ __device__ __forceinline__ uint32_t activate_batch(const Part<OffT> &P, const bo
   for (int q = 0; q < kBatch; q++) {
     const bool hub = keep[q] && hb[q];
     if (hub) append_hub_A<kByOut>(P, x[q], slot);
-    qA.push_a(keep[q] && !hub, x[q], ob[q], oe[q] - ob[q], P.listA[slot], &P.ctl->cnt_A[slot]);
+    qA.push(keep[q] && !hub, x[q], 0, P.listA[slot], nullptr, &P.ctl->cnt_A[slot]);
     cnt += __popc(__ballot_sync(0xffffffffu, nw[q]));
   }
   return cnt;
@@ -729,18 +721,11 @@ __device__ __forceinline__ void gather_phase(const Part<OffT> &P, const View &V)
 
   // Phase 1: non-hub active vertices, 32 per warp, static grid stride
   const uint32_t gw = blockIdx.x * kWarpsPerBlock + warp, nw = gridDim.x * kWarpsPerBlock;
-  // carried A lists (activate_batch): the entry's CSC range comes with it, loaded in
-  // the same round trip as the entry (the fused push supersteps do not carry)
-  const bool carried = Prog::kHasGather && !implicit && P.carry && !V.push;
   for (uint32_t base = gw * 32u; base < nA; base += nw * 32u) {
     const uint32_t idx = base + lane;
     bool valid = idx < nA;
-    uint32_t v = 0, cb = 0, cd = 0;
+    uint32_t v = 0;
     if (valid) v = implicit ? P.own_lo + idx : LA[idx];
-    if (valid && carried) {
-      cb = P.listAb[slot][idx];
-      cd = P.listAd[slot][idx];
-    }
     const uint32_t lv = v - P.own_lo;
     if (valid && implicit && test_bit(P.hub_in, lv)) valid = false;  // served by the hub chunks
     uint64_t beg = 0;
@@ -748,13 +733,8 @@ __device__ __forceinline__ void gather_phase(const Part<OffT> &P, const View &V)
     bool hubv = false;
     if (valid) {
       if (Prog::kHasGather) {
-        if (carried) {
-          beg = cb;
-          deg = cd;
-        } else {
-          beg = (uint64_t)P.in_off[lv];
-          deg = (uint32_t)((uint64_t)P.in_off[lv + 1] - beg);
-        }
+        beg = (uint64_t)P.in_off[lv];
+        deg = (uint32_t)((uint64_t)P.in_off[lv + 1] - beg);
       }
       cur = P.val[v];
       hubv = !no_hub_c && test_bit(P.hub_out, v);  // issued with the offsets, used after apply
@@ -887,9 +867,7 @@ __device__ __forceinline__ void activate_phase(const Part<OffT> &P, const View &
   __shared__ uint32_t s_off[kWarpsPerBlock + 1];
   __shared__ unsigned long long s8[kWarpsPerBlock];
   const uint32_t warp = threadIdx.x / 32, lane = lane_id();
-  __shared__ uint32_t sqc[kWarpsPerBlock][2][kQueueCap];  // carried CSC ranges of the A entries
-  WarpQueue qA{sq[warp], sqc[warp][0], 0};
-  qA.s_c = sqc[warp][1];
+  WarpQueue qA{sq[warp], nullptr, 0};
   unsigned long long my_s = 0, my_act = 0;
 
   const uint32_t gw = blockIdx.x * kWarpsPerBlock + warp, nw = gridDim.x * kWarpsPerBlock;
@@ -1351,9 +1329,7 @@ __device__ __forceinline__ void scatter_activate_phase(const Part<OffT> &P, cons
   __shared__ uint32_t s_off[kWarpsPerBlock + 1];
   __shared__ unsigned long long s8[kWarpsPerBlock];
   const uint32_t warp = threadIdx.x / 32, lane = lane_id();
-  __shared__ uint32_t sqc[kWarpsPerBlock][2][kQueueCap];  // carried CSC ranges of the A entries
-  WarpQueue qA{sq[warp], sqc[warp][0], 0};
-  qA.s_c = sqc[warp][1];
+  WarpQueue qA{sq[warp], nullptr, 0};
   unsigned long long my_s = 0, my_act = 0;
 
   const uint32_t gw = blockIdx.x * kWarpsPerBlock + warp, nw = gridDim.x * kWarpsPerBlock;
@@ -1899,15 +1875,7 @@ __global__ void __launch_bounds__(kBlock) k_init_frontier(const __grid_constant_
         const bool hub = test_bit(Prog::kHasGather ? P.hub_in : P.hub_out,
                                   Prog::kHasGather ? source - P.own_lo : source);
         if (hub) append_hub_A<!Prog::kHasGather>(P, source, 0);
-        else {
-          P.listA[0][0] = source;
-          if (P.carry && Prog::kHasGather) {  // the carried CSC range of the entry (gather programs)
-            const uint32_t b = (uint32_t)P.in_off[source - P.own_lo];
-            P.listAb[0][0] = b;
-            P.listAd[0][0] = (uint32_t)P.in_off[source - P.own_lo + 1] - b;
-          }
-          ctl->cnt_A[0] = 1;
-        }
+        else { P.listA[0][0] = source; ctl->cnt_A[0] = 1; }
         ctl->cnt_act[0] = 1;
       }
       ctl->stop = owned ? 0u : 1u;
@@ -1917,9 +1885,7 @@ __global__ void __launch_bounds__(kBlock) k_init_frontier(const __grid_constant_
   // kInitSourceChanged: the source is "changed" at initialisation; A_0 = out-neighbours.
   __shared__ uint32_t sq[kWarpsPerBlock][kQueueCap];
   const uint32_t warp = threadIdx.x / 32;
-  __shared__ uint32_t sqc[kWarpsPerBlock][2][kQueueCap];  // carried CSC ranges of the A entries
-  WarpQueue qA{sq[warp], sqc[warp][0], 0};
-  qA.s_c = sqc[warp][1];
+  WarpQueue qA{sq[warp], nullptr, 0};
   const uint64_t beg = (uint64_t)P.out_off[source];
   const uint32_t deg = (uint32_t)((uint64_t)P.out_off[source + 1] - beg);
   uint32_t a;
