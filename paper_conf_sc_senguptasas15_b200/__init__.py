@@ -362,6 +362,26 @@ class HostLayout:
             L.gr_host_free(h)
         self.__dict__.update(info)
 
+    @classmethod
+    def from_sorted(cls, n, m, in_offsets, in_idx, row_offsets, col_idx, **opts):
+        """gr_host_build of a GR_FMT_SORTED input (both halves), copied out like __init__."""
+        self = cls.__new__(cls)
+        e = gr_edges()
+        e.fmt, e.num_vertices, e.num_edges = GR_FMT_SORTED, int(n), int(m)
+        keep = [np.ascontiguousarray(in_offsets, dtype=np.uint64), np.ascontiguousarray(in_idx, dtype=np.uint32),
+                np.ascontiguousarray(row_offsets, dtype=np.uint64), np.ascontiguousarray(col_idx, dtype=np.uint32)]
+        e.in_offsets, e.in_idx, e.row_offsets, e.col_idx = (a.ctypes.data for a in keep)
+        o, uid = _load_opts(**opts)
+        h = ctypes.c_void_p()
+        L = lib()
+        _check(L.gr_host_build(ctypes.byref(e), ctypes.byref(o), ctypes.byref(h)))
+        try:
+            info = self._copy(L, h, int(n), False)
+        finally:
+            L.gr_host_free(h)
+        self.__dict__.update(info)
+        return self
+
     @staticmethod
     def _copy(L, h, n, has_w):
         u64p, u32p, u8p = (ctypes.POINTER(ctypes.c_uint64), ctypes.POINTER(ctypes.c_uint32),

@@ -303,10 +303,13 @@ gr_status gr_host_build(const gr_edges *edges, const gr_load_opts *opts_in, gr_h
   *out = nullptr;
   gr_load_opts opts{};
   if (opts_in) opts = *opts_in;
+  if (!edges) return fail(GR_EINVAL, "edges is NULL");
   auto *h = new gr_host_graph();
   std::string err;
-  gr_status s = build_host_graph(edges, opts.shard_edges, opts.world > 0 ? opts.world : 1, opts.rank,
-                                 opts.host_threads, &h->H, &err);
+  gr_status s = edges->fmt == GR_FMT_SORTED
+                    ? build_host_sorted(edges, opts.shard_edges, opts.borrow != 0, opts.host_threads, &h->H, &err)
+                    : build_host_graph(edges, opts.shard_edges, opts.world > 0 ? opts.world : 1, opts.rank,
+                                       opts.host_threads, &h->H, &err);
   if (s != GR_OK) {
     delete h;
     return fail(s, "%s", err.c_str());

@@ -196,3 +196,50 @@ def test_graph_file_validation(tmp_path):
             with pytest.raises(gr.GrError) as ei:
                 gr.gr_graph_load_file(p)
             assert ei.value.status == gr.GR_ECUDA
+
+
+def _sorted_halves(g):
+    n = g.n
+    oi = np.lexsort((g.src, g.dst))
+    in_off = np.zeros(n + 1, np.uint64)
+    in_off[1:] = np.cumsum(np.bincount(g.dst, minlength=n))
+    oo = np.lexsort((g.dst, g.src))
+    out_off = np.zeros(n + 1, np.uint64)
+    out_off[1:] = np.cumsum(np.bincount(g.src, minlength=n))
+    return in_off, g.src[oi], out_off, g.dst[oo]
+
+
+@pytest.mark.parametrize("shard_edges", [0, 3000])
+def test_sorted_input_layout_equals_coo_layout(shard_edges):
+    """GR_FMT_SORTED (the cfg5-at-scale input: an already-sorted in-CSC + out-CSR)
+    gives the host builder's layout of the same edge multiset exactly."""
+    g = grgen.rmat(12, 16, seed=23)
+    a = gr.HostLayout(g.n, g.src, g.dst, shard_edges=shard_edges)
+    b = gr.HostLayout.from_sorted(g.n, g.m, *_sorted_halves(g), shard_edges=shard_edges)
+    for k in ("bounds", "in_off", "in_src", "out_off", "out_dst"):
+        np.testing.assert_array_equal(getattr(a, k), getattr(b, k), err_msg=k)
+
+
+def test_sorted_input_is_validated():
+    g = grgen.rmat(8, 8, seed=24)
+    in_off, in_src, out_off, out_dst = _sorted_halves(g)
+    bad = in_src.copy()
+    bad[5] = g.n  # id out of range
+    with pytest.raises(gr.GrError) as ei:
+        gr.HostLayout.from_sorted(g.n, g.m, in_off, bad, out_off, out_dst)
+    assert ei.value.status == gr.GR_EINVAL
+    # a row whose first two sources differ, swapped into descending order
+    starts = in_off[:-1].astype(np.int64)
+    two = (np.diff(in_off.astype(np.int64)) >= 2)
+    cand = [int(b) for b in starts[two] if in_src[b] != in_src[b + 1]]
+    b0 = cand[0]
+    uns = in_src.copy()
+    uns[b0], uns[b0 + 1] = in_src[b0 + 1], in_src[b0]
+    with pytest.raises(gr.GrError) as ei:
+        gr.HostLayout.from_sorted(g.n, g.m, in_off, uns, out_off, out_dst)
+    assert ei.value.status == gr.GR_EINVAL
+    short = out_off.copy()
+    short[-1] -= 1  # does not span [0, m]
+    with pytest.raises(gr.GrError) as ei:
+        gr.HostLayout.from_sorted(g.n, g.m, in_off, in_src, short, out_dst)
+    assert ei.value.status == gr.GR_EINVAL
