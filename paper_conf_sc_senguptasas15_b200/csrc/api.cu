@@ -116,16 +116,12 @@ gr_status gr_graph_load(const gr_edges *edges, const gr_load_opts *opts_in, gr_g
     }
   }
   cudaDeviceGetAttribute(&g->num_sms, cudaDevAttrMultiProcessorCount, g->device);
-  if (cudaStreamCreateWithFlags(&g->stream, cudaStreamNonBlocking) != cudaSuccess ||
-      cudaEventCreate(&g->ev_start) != cudaSuccess || cudaEventCreate(&g->ev_stop) != cudaSuccess ||
-      cudaMallocHost((void **)&g->h_ctl, sizeof(Ctl)) != cudaSuccess) {
+  // stream, events and the pinned control block: reused from graphs freed earlier on
+  // this device (creating them, the pinned allocation above all, costs milliseconds of
+  // every load: the e2e path)
+  if (!acquire_handles(g)) {
     destroy(g);
     return fail(GR_ECUDA, "stream/event/pinned setup failed");
-  }
-  for (int i = 0; i < 2; i++) {
-    cudaEvent_t e;
-    cudaEventCreate(&e);
-    g->prof_ev.push_back(e);
   }
   tmark("load: host build / setup");
   if (dev_build) {

@@ -21,6 +21,7 @@
 #include <cstdio>
 #include <cstring>
 #include <map>
+#include <mutex>
 #include <string>
 #include <vector>
 
@@ -1632,24 +1633,74 @@ gr_status fetch_trace(gr_graph *g, uint64_t *dst, uint64_t max_rows, uint64_t *r
   return GR_OK;
 }
 
+// Per-device cache of the per-graph handles (stream, 4 events, pinned Ctl block):
+// a reload takes them back instead of creating them (e2e load path).
+namespace {
+struct Handles {
+  cudaStream_t stream;
+  cudaEvent_t ev[4];
+  Ctl *h_ctl;
+};
+std::mutex g_handles_mu;
+std::vector<Handles> g_handles[64];
+}  // namespace
+
+bool acquire_handles(gr_graph *g) {
+  {
+    std::lock_guard<std::mutex> lk(g_handles_mu);
+    if (g->device >= 0 && g->device < 64 && !g_handles[g->device].empty()) {
+      const Handles h = g_handles[g->device].back();
+      g_handles[g->device].pop_back();
+      g->stream = h.stream;
+      g->ev_start = h.ev[0];
+      g->ev_stop = h.ev[1];
+      g->prof_ev = {h.ev[2], h.ev[3]};
+      g->h_ctl = h.h_ctl;
+      return true;
+    }
+  }
+  if (cudaStreamCreateWithFlags(&g->stream, cudaStreamNonBlocking) != cudaSuccess ||
+      cudaEventCreate(&g->ev_start) != cudaSuccess || cudaEventCreate(&g->ev_stop) != cudaSuccess ||
+      cudaMallocHost((void **)&g->h_ctl, sizeof(Ctl)) != cudaSuccess)
+    return false;
+  for (int i = 0; i < 2; i++) {
+    cudaEvent_t e;
+    if (cudaEventCreate(&e) != cudaSuccess) return false;
+    g->prof_ev.push_back(e);
+  }
+  return true;
+}
+
+static void release_handles(gr_graph *g) {
+  if (g->stream && g->ev_start && g->ev_stop && g->h_ctl && g->prof_ev.size() >= 2 && g->device >= 0 &&
+      g->device < 64) {
+    Handles h{g->stream, {g->ev_start, g->ev_stop, g->prof_ev[0], g->prof_ev[1]}, g->h_ctl};
+    for (size_t i = 2; i < g->prof_ev.size(); i++) cudaEventDestroy(g->prof_ev[i]);
+    std::lock_guard<std::mutex> lk(g_handles_mu);
+    g_handles[g->device].push_back(h);
+    return;
+  }
+  for (auto e : g->prof_ev) cudaEventDestroy(e);
+  if (g->ev_start) cudaEventDestroy(g->ev_start);
+  if (g->ev_stop) cudaEventDestroy(g->ev_stop);
+  if (g->h_ctl) cudaFreeHost(g->h_ctl);
+  if (g->stream) cudaStreamDestroy(g->stream);
+}
+
 void destroy(gr_graph *g) {
   if (!g) return;
   cudaSetDevice(g->device);
   cudaDeviceSynchronize();
   for (auto &kv : g->while_exec) cudaGraphExecDestroy(kv.second.first);
   if (g->pr_exec) cudaGraphExecDestroy(g->pr_exec);
-  for (auto e : g->prof_ev) cudaEventDestroy(e);
-  if (g->ev_start) cudaEventDestroy(g->ev_start);
-  if (g->ev_stop) cudaEventDestroy(g->ev_stop);
   stream_destroy(g);
   delete g->comm;
   g->comm = nullptr;
   for (void *p : g->allocs) cudaFreeAsync(p, g->stream);
   for (void *p : g->plain_allocs) cudaFree(p);
   cudaStreamSynchronize(g->stream);
-  if (g->h_ctl) cudaFreeHost(g->h_ctl);
   if (g->h_xbytes) cudaFreeHost(g->h_xbytes);
-  if (g->stream) cudaStreamDestroy(g->stream);
+  release_handles(g);  // stream, events, pinned Ctl back to the device's cache
   delete g;
 }
 

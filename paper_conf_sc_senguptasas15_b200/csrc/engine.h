@@ -242,6 +242,7 @@ gr_status fetch_values(gr_graph *g, void *dst, uint64_t bytes);
 gr_status fetch_trace(gr_graph *g, uint64_t *dst, uint64_t max_rows, uint64_t *rows);
 gr_status fetch_trace_detail(gr_graph *g, uint64_t *dst, uint64_t max_rows, uint64_t *rows);
 void destroy(gr_graph *g);
+bool acquire_handles(gr_graph *g);  // stream, events, pinned Ctl (cached per device)
 // streamed mode
 gr_status stream_setup(gr_graph *g, uint64_t budget);
 gr_status run_streamed(gr_graph *g, const gr_run_opts *o, gr_run_stats *st);
