@@ -65,7 +65,7 @@ int main() {
   ap.type = CU_MEM_ALLOCATION_TYPE_PINNED;
   ap.location.type = CU_MEM_LOCATION_TYPE_DEVICE;
   ap.location.id = 0;
-  ap.requestedHandleTypes = mp.handleTypes;
+  ap.requestedHandleTypes = (CUmemAllocationHandleType)mp.handleTypes;
   CUmemGenericAllocationHandle ph;
   CU(cuMemCreate(&ph, size, &ap, 0));
   CU(cuMulticastBindMem(mch, 0, ph, 0, size, 0));
