@@ -331,7 +331,7 @@ def bench_sorted(args):
     print(f"[bench] loaded in {load_s:.1f}s: {info}", file=sys.stderr)
     stream = torch.cuda.current_stream()
     sp = stream.cuda_stream
-    rkw = dict(source=0, max_iters=30 if algo == "pagerank" else 0)
+    rkw = dict(source=0, max_iters=30 if algo == "pagerank" else 0, zero_copy=args.zero_copy)
     for _ in range(max(1, args.warmup)):
         G.run(algo, stream=sp, **rkw)
     torch.cuda.synchronize()
@@ -373,6 +373,8 @@ def bench_sorted(args):
                                f"{'in-CSC' if algo == 'pagerank' else 'out-CSR'} only, borrowed in place",
                    "n": n, "m": m, "scale": scale, "requested_scale": args.scale, "shards": info["num_shards"],
                    "mode": "streamed", "parallelism": "1 GPU", "iterations": stats["iterations"],
+                   "zero_copy": {"policy": args.zero_copy, "phases_in_place": stats["zero_copy_phases"],
+                                 "bytes_in_place": stats["bytes_h2d_zero_copy"]},
                    "l2": "inputs far larger than L2 (streamed from host memory); no flush",
                    "host_ram": {"available_bytes": avail, "needed_bytes": sorted_host_bytes(scale),
                                 "rule": "4 B/edge adjacency + 44 B/vertex (DESIGN.md §11)"},
@@ -415,6 +417,8 @@ def main():
                     help="run another program on the config's graph (e.g. --config 5 --algo bfs, "
                          "--config 2 --algo pagerank_delta)")
     ap.add_argument("--tolerance", type=float, default=1e-4, help="pagerank_delta: |dR| threshold x n")
+    ap.add_argument("--zero-copy", type=int, default=0, choices=[-1, 0, 1],
+                    help="streamed runs: 0 auto (in place when the frontier is thin), 1 always in place, -1 never")
     ap.add_argument("--other-configs", type=int, default=1,
                     help="default cfg2 run: also measure configs 1, 3, 4 and the cfg5 shape (s26, streamed) in "
                          "subprocesses and summarise them under other_configs (0: off)")

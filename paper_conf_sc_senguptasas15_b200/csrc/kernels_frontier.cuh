@@ -1494,12 +1494,14 @@ __device__ __forceinline__ void dense_seg_phase(const Part<OffT> &P, const View 
 #pragma unroll
     for (int k = 0; k < kDsIpt; k++) {  // all loads of the 8 items in flight together
       const bool ok = src[k] != kDsNoSrc;
-      if (!kGate) sv[k] = ok ? __ldg(P.val + src[k]) : 0u;
-      sa[k] = ok && test_bit(bits, src[k]);
+      // values and changed bits were written earlier in this (persistent) launch: coherent
+      // loads, not the read-only .nc path (valid only for data read-only during the kernel)
+      if (!kGate) sv[k] = ok ? P.val[src[k]] : 0u;
+      sa[k] = ok && test_bit_cg(bits, src[k]);
     }
     if (kGate) {
 #pragma unroll
-      for (int k = 0; k < kDsIpt; k++) sv[k] = sa[k] ? __ldg(P.val + src[k]) : 0u;
+      for (int k = 0; k < kDsIpt; k++) sv[k] = sa[k] ? P.val[src[k]] : 0u;
     }
     G g[kDsIpt];
 #pragma unroll

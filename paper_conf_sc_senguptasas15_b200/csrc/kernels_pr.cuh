@@ -391,6 +391,17 @@ template <int kVar> __device__ __forceinline__ float seg_ldf(const float *p) {
   return __ldg(p);
 }
 
+// The contributions of superstep t-1 were written by other CTAs earlier in the same
+// (persistent) launch: an ordinary weak load, ordered after those writes by the grid
+// barrier's fences — NOT ld.global.nc (the read-only path is defined only for data that
+// stays unchanged for the whole kernel). Measured: same rate as __ldg
+// (tools/gather_paths_bench.cu: ld.global and LDG.CONSTANT both 1.00 per SM per cycle).
+__device__ __forceinline__ float ld_weak_f32(const float *p) {
+  float v;
+  asm("ld.global.f32 %0, [%1];" : "=f"(v) : "l"(p));
+  return v;
+}
+
 __device__ __forceinline__ float lds_f32(uint32_t saddr) {
   float v;
   asm("ld.shared.f32 %0, [%1];" : "=f"(v) : "r"(saddr));
@@ -406,7 +417,7 @@ __device__ __forceinline__ void seg_gather(const uint4 &s0, const uint4 &s1, con
   const uint32_t src[kSegIpt] = {s0.x, s0.y, s0.z, s0.w, s1.x, s1.y, s1.z, s1.w};
 #pragma unroll
   for (int k = 0; k < kSegIpt; k++) {
-    v[k] = (src[k] & kHotTag) ? lds_f32(hot_sbase + 4u * (src[k] & ~kHotTag)) : __ldg(contrib + src[k]);
+    v[k] = (src[k] & kHotTag) ? lds_f32(hot_sbase + 4u * (src[k] & ~kHotTag)) : ld_weak_f32(contrib + src[k]);
   }
 }
 
@@ -867,10 +878,10 @@ template <int kPol> __device__ __forceinline__ uint4 bseg_ld4(const uint4 *p, ui
 template <int kPol> __device__ __forceinline__ float bseg_ldc(const float *p, uint64_t pol) {
   if (kPol) {
     float v;
-    asm("ld.global.nc.L2::cache_hint.f32 %0, [%1], %2;" : "=f"(v) : "l"(p), "l"(pol));
+    asm("ld.global.L2::cache_hint.f32 %0, [%1], %2;" : "=f"(v) : "l"(p), "l"(pol));  // written in-launch: not .nc
     return v;
   }
-  return __ldg(p);
+  return ld_weak_f32(p);
 }
 
 // One block tile: like seg_tile, with runs for rows; finished runs (other than
