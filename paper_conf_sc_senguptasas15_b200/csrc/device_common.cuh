@@ -113,6 +113,32 @@ __device__ __forceinline__ void load_view(const Ctl *c, View &v) {
   __syncthreads();
 }
 
+// Software grid barrier of the persistent loops (cooperative launch: every CTA
+// is resident). The arrival counter only grows within a launch (zeroed before
+// it): barrier k of the launch is passed once it reaches k * gridDim.x, so no
+// reset and no separate generation word are needed. The arrival is an acq_rel
+// atomic (publishes this CTA's writes: MEMBAR.ALL.GPU, and invalidates L1 on
+// return), the wait an ld.acquire spin — no fence.sc. Measured 1.2-1.5 us per
+// barrier at 148-592 CTAs against 2.3-3.0 us for a fenced count-and-generation
+// barrier (profiles/microbench_r02_grid_sync.txt). `target` is thread 0's
+// running k * gridDim.x (start at 0).
+__device__ __forceinline__ void grid_barrier(uint32_t *count, uint32_t &target) {
+  __syncthreads();
+  if (threadIdx.x == 0) {
+    target += gridDim.x;
+    uint32_t old;
+    asm volatile("atom.add.acq_rel.gpu.global.u32 %0, [%1], 1;" : "=r"(old) : "l"(count) : "memory");
+    if (old != target - 1) {
+      for (;;) {
+        uint32_t now;
+        asm volatile("ld.acquire.gpu.global.u32 %0, [%1];" : "=r"(now) : "l"(count) : "memory");
+        if ((int32_t)(now - target) >= 0) break;
+      }
+    }
+  }
+  __syncthreads();
+}
+
 __device__ __forceinline__ unsigned long long gtimer() {
   unsigned long long t;
   asm volatile("mov.u64 %0, %%globaltimer;" : "=l"(t));
@@ -167,6 +193,14 @@ template <class OffT> struct Part {
   void *ds_acc;            // [own_n] GatherT slots (8 B) of the split rows, identity between uses
   uint32_t *ds_act;        // [own_n / 32 + 1] active bits of the split rows
   uint32_t ds_tiles, ds_nsplit;
+  // vertex records (low-degree graphs, kernels_frontier.cuh kRecDeg): one 32-byte
+  // record per vertex holding its first kRecDeg neighbours, their weights, the
+  // degree and the CSR/CSC offset, so a lane reads its whole adjacency of degree
+  // <= kRecDeg with one sector instead of offsets + sources + weights.
+  // rec_in[2 lv]: {src[4]}, rec_in[2 lv + 1]: {w[4] as bytes, deg, beg lo, beg hi} (owned rows);
+  // rec_out[2 u]: {dst[4]}, rec_out[2 u + 1]: {0, deg, beg lo, beg hi} (activation CSR). nullptr: off
+  const uint4 *rec_in;
+  const uint4 *rec_out;
   // partitioned frontier programs, exchange fused into the gather: every rank's
   // changed-set buffers of this superstep's parity (own included), written at
   // xp_off (= own_lo) + list position as the gather appends (WarpQueue mirrors)
@@ -200,6 +234,12 @@ __device__ __forceinline__ uint8_t ldg_nc_u8(const uint8_t *p) {
   uint16_t v;
   asm volatile("ld.global.nc.L1::no_allocate.u8 %0, [%1];" : "=h"(v) : "l"(p));
   return (uint8_t)v;
+}
+
+__device__ __forceinline__ uint4 ldg_nc_v4(const uint4 *p) {
+  uint4 v;
+  asm("ld.global.nc.v4.u32 {%0, %1, %2, %3}, [%4];" : "=r"(v.x), "=r"(v.y), "=r"(v.z), "=r"(v.w) : "l"(p));
+  return v;
 }
 
 // L2-coherent read (bypasses L1, so stamps written by other SMs are seen)

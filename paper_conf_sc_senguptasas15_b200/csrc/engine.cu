@@ -346,6 +346,59 @@ template <class OffT> static gr_status ds_long_fraction(gr_graph *g) {
   return GR_OK;
 }
 
+// Vertex records (Part::rec_in / rec_out, kernels_frontier.cuh kRecDeg), once per
+// resident single-rank graph whose vertices nearly all have degree <= kRecDeg in
+// both directions (road networks, meshes: cfg3): a lane then reads a vertex's
+// whole adjacency with one 32-byte sector — one dependent load and two
+// requests less per gathered or expanded vertex. GR_REC=0/1 forces.
+template <class OffT>
+static __global__ void k_rec_count(const OffT *off, uint32_t rows, unsigned long long *n_small) {
+  unsigned long long c = 0;
+  for (uint32_t r = blockIdx.x * blockDim.x + threadIdx.x; r < rows; r += gridDim.x * blockDim.x)
+    c += (uint64_t)off[r + 1] - (uint64_t)off[r] <= kRecDeg;
+  for (int o = 16; o > 0; o >>= 1) c += __shfl_xor_sync(0xffffffffu, c, o);
+  if ((threadIdx.x & 31) == 0 && c) atomicAdd(n_small, c);
+}
+template <class OffT>
+static __global__ void k_rec_fill(const OffT *off, const uint32_t *adj, const uint8_t *w, uint32_t rows, uint4 *rec) {
+  for (uint32_t r = blockIdx.x * blockDim.x + threadIdx.x; r < rows; r += gridDim.x * blockDim.x) {
+    const uint64_t b = (uint64_t)off[r], d = (uint64_t)off[r + 1] - b;
+    uint32_t a[kRecDeg] = {0, 0, 0, 0}, w4 = 0;
+    for (uint32_t q = 0; q < kRecDeg && q < d; q++) {
+      a[q] = adj[b + q];
+      if (w) w4 |= (uint32_t)w[b + q] << (8 * q);
+    }
+    rec[2ull * r] = make_uint4(a[0], a[1], a[2], a[3]);
+    rec[2ull * r + 1] = make_uint4(w4, (uint32_t)d, (uint32_t)b, (uint32_t)(b >> 32));
+  }
+}
+template <class OffT> static gr_status rec_setup(gr_graph *g) {
+  g->rec_tried = true;
+  const uint32_t rows = (uint32_t)g->H.own_n(), n = (uint32_t)g->H.n;
+  const char *e = getenv("GR_REC");
+  if ((e && atoi(e) == 0) || !rows || !g->in_src || !g->out_dst) return GR_OK;
+  cudaStream_t s = g->stream;
+  unsigned long long *cnt = nullptr, h[2] = {0, 0};
+  CK(cudaMallocAsync(&cnt, sizeof h, s));
+  CK(cudaMemsetAsync(cnt, 0, sizeof h, s));
+  k_rec_count<OffT><<<g->num_sms * 8, 256, 0, s>>>((const OffT *)g->in_off, rows, cnt);
+  k_rec_count<OffT><<<g->num_sms * 8, 256, 0, s>>>((const OffT *)g->out_off, n, cnt + 1);
+  CK(cudaMemcpyAsync(h, cnt, sizeof h, cudaMemcpyDeviceToHost, s));
+  CK(cudaFreeAsync(cnt, s));
+  CK(cudaStreamSynchronize(s));
+  if (!(e || (h[0] >= 0.9 * rows && h[1] >= 0.9 * n))) return GR_OK;
+  uint4 *ri = nullptr, *ro = nullptr;
+  if (dev_alloc(g, (void **)&ri, 32ull * rows) != GR_OK || dev_alloc(g, (void **)&ro, 32ull * n) != GR_OK)
+    return GR_OK;  // records are an accelerator: run without them
+  k_rec_fill<OffT><<<g->num_sms * 8, 256, 0, s>>>((const OffT *)g->in_off, g->in_src, g->in_w, rows, ri);
+  k_rec_fill<OffT><<<g->num_sms * 8, 256, 0, s>>>((const OffT *)g->out_off, g->out_dst, nullptr, n, ro);
+  CK(cudaGetLastError());
+  g->rec_in = ri;
+  const char *eo = getenv("GR_REC_OUT");  // A/B: records for the gather only
+  g->rec_out = (eo && atoi(eo) == 0) ? nullptr : ro;
+  return GR_OK;
+}
+
 template <class OffT> static gr_status ds_setup(gr_graph *g) {
   g->ds_tried = true;
   const HostGraph &H = g->H;
@@ -1332,7 +1385,7 @@ static gr_status run_pagerank(gr_graph *g, const gr_run_opts *o, cudaStream_t s,
     L.n_long = g->n_long;
     L.hot_k = g->hot_k;
     L.bar = g->pr_bar;
-    k_pr_init<<<g->num_sms * 4, 256, 0, s>>>((uint32_t)g->H.n, g->inv_outdeg, g->contrib[0]);
+    k_pr_init<<<g->num_sms * 4, 256, 0, s>>>((uint32_t)g->H.n, g->inv_outdeg, g->contrib[0], g->pr_bar);
     k_pr_hot_pack<<<(g->hot_k + 255) / 256, 256, 0, s>>>(g->contrib[0], g->hot_ids, g->hot_buf[0], g->hot_k);
     if (prof) CK(cudaEventRecord(g->prof_ev[0], s));
     void *args[] = {(void *)&a, (void *)&L};
@@ -1374,7 +1427,7 @@ static gr_status run_pagerank(gr_graph *g, const gr_run_opts *o, cudaStream_t s,
     unsigned long long *d_ts = nullptr;
     if (phases) CK(cudaMallocAsync((void **)&d_ts, 8ull * (2 * iters + 1), s));
     L.ts = d_ts;
-    k_pr_init<<<g->num_sms * 4, 256, 0, s>>>((uint32_t)g->H.n, g->inv_outdeg, g->contrib[0]);
+    k_pr_init<<<g->num_sms * 4, 256, 0, s>>>((uint32_t)g->H.n, g->inv_outdeg, g->contrib[0], g->pr_bar);
     k_pr_hot_pack<<<(g->hot_k + 255) / 256, 256, 0, s>>>(g->contrib[0], g->hot_ids, g->hot_buf[0], g->hot_k);
     if (prof) CK(cudaEventRecord(g->prof_ev[0], s));
     void *args[] = {(void *)&a, (void *)&L};
@@ -1511,6 +1564,10 @@ gr_status run(gr_graph *g, const gr_run_opts *oin, gr_run_stats *st) {
   if (o.algo != GR_PAGERANK) {  // every program but PageRank activates along the out-edges
     gr_status cs = ensure_csr(g);
     if (cs != GR_OK) return cs;
+  }
+  if (o.algo != GR_PAGERANK && o.algo != GR_BFS && g->mode == GR_MODE_RESIDENT && !g->comm && !g->rec_tried) {
+    gr_status rs = g->off64 ? rec_setup<uint64_t>(g) : rec_setup<uint32_t>(g);
+    if (rs != GR_OK) return rs;
   }
   if (g->mode == GR_MODE_STREAMED) return run_streamed(g, &o, st);
   cudaStream_t s = o.stream ? (cudaStream_t)o.stream : g->stream;

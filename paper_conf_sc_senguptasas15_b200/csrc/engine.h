@@ -39,6 +39,8 @@ struct gr_graph {
   void *ds_acc = nullptr;
   uint32_t ds_tiles = 0, ds_nsplit = 0;
   bool ds_tried = false;
+  uint4 *rec_in = nullptr, *rec_out = nullptr;  // vertex records (low-degree graphs; first gather-program run)
+  bool rec_tried = false;
   double ds_long_frac = -1.0;  // share of in-edges in rows longer than one tile (< 0: not computed)                  // tolerance PageRank divisor table (first GR_PAGERANK_DELTA run)
   uint32_t *hub_in = nullptr, *hub_out = nullptr, *static_hubs = nullptr;
   uint32_t n_static_hubs = 0;
@@ -178,6 +180,8 @@ template <class OffT> inline Part<OffT> make_part(gr_graph *g) {
   P.ds_act = g->ds_act;
   P.ds_tiles = g->ds_tiles;
   P.ds_nsplit = g->ds_nsplit;
+  P.rec_in = g->rec_in;
+  P.rec_out = g->rec_out;
   P.nxt[0] = g->nxt[0];
   P.nxt[1] = g->nxt[1];
   P.out_w = g->out_w;

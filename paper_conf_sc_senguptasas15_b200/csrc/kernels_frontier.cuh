@@ -26,6 +26,8 @@
 namespace gr {
 
 constexpr int kBatch = 4;  // edges in flight per lane per memory phase
+constexpr uint32_t kRecDeg = 4;  // neighbours held in a vertex record (Part::rec_in / rec_out)
+static_assert(kRecDeg == (uint32_t)kBatch, "a record's neighbours form one activation batch");
 #ifdef GR_NO_GATE  // A/B build: dense supersteps read every source's value
 constexpr bool kGateSelective = false;
 #else
@@ -76,7 +78,8 @@ __device__ __forceinline__ typename Prog::GatherT warp_reduce_prog(typename Prog
 template <class Prog, bool kDense, bool kGateT = false, class OffT>
 __device__ typename Prog::GatherT gather_warp(const Part<OffT> &P, bool valid, uint64_t beg, uint32_t deg,
                                               uint32_t dval, typename Prog::GatherT *sred, const Ctx &cx,
-                                              const uint32_t *bits, bool &act) {
+                                              const uint32_t *bits, bool &act, bool direct = false,
+                                              uint4 rs = uint4{}, uint32_t w4 = 0) {
   using G = typename Prog::GatherT;
   const uint32_t lane = lane_id();
   G acc = Prog::identity();
@@ -84,6 +87,35 @@ __device__ typename Prog::GatherT gather_warp(const Part<OffT> &P, bool valid, u
   // dense supersteps of selective programs may read val[u] only for changed sources
   // (Selective<>; chosen per superstep by close_superstep: Ctl::gate)
   constexpr bool kGate = kDense && kGateT && kGateSelective && Selective<Prog>::value;
+  // vertex records: a lane whose vertex has degree <= kRecDeg holds its sources
+  // (rs) and weights (w4) already and gathers alone, all loads in one phase
+  if (direct) {
+    const uint32_t us[kRecDeg] = {rs.x, rs.y, rs.z, rs.w};
+    uint32_t ew[kRecDeg], vv[kRecDeg], bw[kRecDeg];
+    bool a[kRecDeg], h[kRecDeg];
+#pragma unroll
+    for (uint32_t q = 0; q < kRecDeg; q++) {
+      a[q] = q < deg;
+      if constexpr (HasScatter<Prog>::value) ew[q] = a[q] ? ld_cg(P.estate + beg + q) : 0u;
+      else ew[q] = Prog::kUsesWeights ? (w4 >> (8 * q)) & 0xFFu : 0u;
+      if (!kGate) vv[q] = a[q] ? P.val[us[q]] : 0u;
+      bw[q] = (kDense && a[q]) ? ld_cg(bits + (us[q] >> 5)) : 0u;
+    }
+    G r = Prog::identity();
+    bool hh = false;
+#pragma unroll
+    for (uint32_t q = 0; q < kRecDeg; q++) {
+      h[q] = kDense && a[q] && ((bw[q] >> (us[q] & 31)) & 1u);
+      if (kGate) vv[q] = h[q] ? P.val[us[q]] : 0u;
+    }
+#pragma unroll
+    for (uint32_t q = 0; q < kRecDeg; q++) {
+      if (a[q] && (!kGate || h[q])) r = Prog::gatherReduce(r, Prog::gatherMap(dval, vv[q], ew[q], us[q], cx));
+      hh |= h[q];
+    }
+    acc = r;
+    act = hh;
+  }
   // warp-cooperative: one vertex of degree in (32, kHubDegree] at a time
   uint32_t big = __ballot_sync(0xffffffffu, valid && deg > 32);
   while (big) {
@@ -137,7 +169,7 @@ __device__ typename Prog::GatherT gather_warp(const Part<OffT> &P, bool valid, u
   // fine-grained: pack the edges of all lanes with degree <= 32, 32 per round;
   // kBatch rounds' loads (sources + weights, then source values) are issued
   // together before their segmented reductions
-  const uint32_t sd = (valid && deg <= 32) ? deg : 0u;
+  const uint32_t sd = (valid && !direct && deg <= 32) ? deg : 0u;
   const uint32_t incl = warp_incl_scan(sd);
   const uint32_t excl = incl - sd;
   const uint32_t total = __shfl_sync(0xffffffffu, incl, 31);
@@ -186,11 +218,8 @@ __device__ typename Prog::GatherT gather_warp(const Part<OffT> &P, bool valid, u
       const int o = own[q];
       if (kDense) {
         const bool h = act_q[q] && ((sb[q] >> (su[q] & 31)) & 1u);
-        // owners of hits: OR of (1 << owner) over the warp
-        uint32_t m = h ? (1u << o) : 0u;
-#pragma unroll
-        for (int dd = 16; dd > 0; dd >>= 1) m |= __shfl_xor_sync(0xffffffffu, m, dd);
-        hitmask |= m;
+        // owners of hits: OR of (1 << owner) over the warp (one REDUX)
+        hitmask |= __reduce_or_sync(0xffffffffu, h ? (1u << o) : 0u);
       }
       G x = act_q[q] ? Prog::gatherMap(dv[q], sv[q], sw[q], su[q], cx) : Prog::identity();
       // segmented inclusive scan keyed by owner lane (owners are non-decreasing)
@@ -432,30 +461,37 @@ __device__ void close_superstep(const Part<OffT> &P, unsigned long long cond_han
   if (threadIdx.x != 0) return;
   unsigned long long sg = 0, sc = 0, ss = 0, sa = 0;
   for (int w = 0; w < kWarpsPerBlock; w++) { sg += s_red[0][w]; sc += s_red[1][w]; ss += s_red[2][w]; sa += s_red[3][w]; }
-  const uint32_t t = c->iter, slot = t & 1u, ns = slot ^ 1u;
-  c->gathered = c->gathered + sg;
-  c->changed = c->changed + sc;
-  c->scattered = c->scattered + ss;
-  c->cnt_act[ns] = c->cnt_act[ns] + (uint32_t)sa;
-  if (t < c->trace_cap) {
+  // every field read at once (independent loads: one L2 round trip, not one per
+  // field — this runs on the critical path of every superstep), then every write
+  const uint32_t t = c->iter, act0 = c->cnt_act[0], act1 = c->cnt_act[1], trace_cap = c->trace_cap;
+  const uint32_t slot = t & 1u, ns = slot ^ 1u;
+  const uint32_t act_ns = slot ? act0 : act1, act_s = slot ? act1 : act0;
+  const unsigned long long prof = c->prof, gath0 = c->gathered, chg0 = c->changed, scat0 = c->scattered;
+  const unsigned long long totA = c->tot_A, totC = c->tot_C, totG = c->tot_gathered, totS = c->tot_scattered;
+  const uint32_t ext_loop = c->ext_loop, max_iters = c->max_iters, tot_pull = c->tot_pull;
+  const unsigned long long gath = gath0 + sg, chg = chg0 + sc, scat = scat0 + ss;
+  const uint32_t act_next = act_ns + (uint32_t)sa;
+  c->cnt_act[ns] = act_next;
+  if (t < trace_cap) {
     volatile unsigned long long *row = P.trace + 4ull * t;
-    row[0] = c->cnt_act[slot];
-    row[1] = c->changed;
-    row[2] = c->gathered;
-    row[3] = c->scattered;
+    row[0] = act_s;
+    row[1] = chg;
+    row[2] = gath;
+    row[3] = scat;
   }
-  if (c->prof) {
+  if (prof) {
+    unsigned long long ks[2], ke[2], kn[2];
+    for (int k = 0; k < 2; k++) { ks[k] = c->kstart[k]; ke[k] = c->kend[k]; kn[k] = c->kns[k]; }
     for (int k = 0; k < 2; k++) {
-      if (c->kend[k] > c->kstart[k]) c->kns[k] = c->kns[k] + (c->kend[k] - c->kstart[k]);
+      if (ke[k] > ks[k]) c->kns[k] = kn[k] + (ke[k] - ks[k]);
       c->kstart[k] = ~0ull;
       c->kend[k] = 0;
     }
   }
-  const unsigned long long scat = c->scattered, chg = c->changed;
-  c->tot_A = c->tot_A + c->cnt_act[slot];
-  c->tot_C = c->tot_C + c->changed;
-  c->tot_gathered = c->tot_gathered + c->gathered;
-  c->tot_scattered = c->tot_scattered + c->scattered;
+  c->tot_A = totA + act_s;
+  c->tot_C = totC + chg;
+  c->tot_gathered = totG + gath;
+  c->tot_scattered = totS + scat;
   c->changed = 0;
   c->gathered = 0;
   c->scattered = 0;
@@ -473,7 +509,7 @@ __device__ void close_superstep(const Part<OffT> &P, unsigned long long cond_han
   c->dirty[ns] = 0;
   if (pulled) {
     c->dirty[slot] = 1;
-    c->tot_pull = c->tot_pull + 1;
+    c->tot_pull = tot_pull + 1;
   }
   c->pull_pending = 0;
   // kPullDense: A_{t+1} is found by the dense gather of t+1; it is empty iff
@@ -485,8 +521,8 @@ __device__ void close_superstep(const Part<OffT> &P, unsigned long long cond_han
   // 2.72 -> 2.42 ms; the web graph's all-changed supersteps 12.2 -> 12.8 ms ungated)
   c->gate = (pulled == kPullDense && 2ull * chg < (unsigned long long)P.own_n) ? 1u : 0u;
   c->iter = t + 1;
-  const bool empty = (pulled == kPullDense) ? (scat == 0) : (c->cnt_act[ns] == 0);
-  const bool stop = !c->ext_loop && (empty || (c->max_iters != 0 && t + 1 >= c->max_iters));
+  const bool empty = (pulled == kPullDense) ? (scat == 0) : (act_next == 0);
+  const bool stop = !ext_loop && (empty || (max_iters != 0 && t + 1 >= max_iters));
   c->stop = stop ? 1u : 0u;
   __threadfence();
 #ifndef GR_JIT  // run-time compiled programs (jit.cpp) run only the persistent loop: no conditional graph node
@@ -729,18 +765,29 @@ __device__ __forceinline__ void gather_phase(const Part<OffT> &P, const View &V)
     const uint32_t lv = v - P.own_lo;
     if (valid && implicit && test_bit(P.hub_in, lv)) valid = false;  // served by the hub chunks
     uint64_t beg = 0;
-    uint32_t deg = 0, cur = 0;
+    uint32_t deg = 0, cur = 0, w4 = 0;
+    uint4 rs{};
     bool hubv = false;
     if (valid) {
       if (Prog::kHasGather) {
-        beg = (uint64_t)P.in_off[lv];
-        deg = (uint32_t)((uint64_t)P.in_off[lv + 1] - beg);
+        if (P.rec_in) {  // vertex record: sources, weights, degree and offset in one sector
+          rs = ldg_nc_v4(P.rec_in + 2ull * lv);
+          const uint4 r1 = ldg_nc_v4(P.rec_in + 2ull * lv + 1);
+          w4 = r1.x;
+          deg = r1.y;
+          beg = (uint64_t)r1.z | ((uint64_t)r1.w << 32);
+        } else {
+          beg = (uint64_t)P.in_off[lv];
+          deg = (uint32_t)((uint64_t)P.in_off[lv + 1] - beg);
+        }
       }
       cur = P.val[v];
       hubv = !no_hub_c && test_bit(P.hub_out, v);  // issued with the offsets, used after apply
     }
     bool hit = false;
-    const G acc = Prog::kHasGather ? gather_warp<Prog, kDense, kGate>(P, valid, beg, deg, cur, sred[warp], cx, bits, hit)
+    const bool direct = P.rec_in != nullptr && valid && deg <= kRecDeg;
+    const G acc = Prog::kHasGather ? gather_warp<Prog, kDense, kGate>(P, valid, beg, deg, cur, sred[warp], cx, bits, hit,
+                                                                       direct, rs, w4)
                                    : Prog::identity();
     const bool active = valid && (!kDense || hit);
     bool changed = false;
@@ -876,14 +923,30 @@ __device__ __forceinline__ void activate_phase(const Part<OffT> &P, const View &
     const bool valid = idx < nC;
     uint64_t beg = 0;
     uint32_t deg = 0;
+    uint4 rd{};
     if (valid) {
       const uint32_t u = P.C_v[idx];
       P.val[u] = P.C_val[idx];  // BSP commit of superstep t
-      beg = (uint64_t)P.out_off[u];
-      deg = (uint32_t)((uint64_t)P.out_off[u + 1] - beg);
+      if (P.rec_out) {  // vertex record: targets, degree and offset in one sector
+        rd = ldg_nc_v4(P.rec_out + 2ull * u);
+        const uint4 r1 = ldg_nc_v4(P.rec_out + 2ull * u + 1);
+        deg = r1.y;
+        beg = (uint64_t)r1.z | ((uint64_t)r1.w << 32);
+      } else {
+        beg = (uint64_t)P.out_off[u];
+        deg = (uint32_t)((uint64_t)P.out_off[u + 1] - beg);
+      }
       my_s += deg;
     }
-    my_act += expand_warp<false>(P, valid, beg, deg, epoch, P.hub_in, qA, ns);
+    const bool direct = P.rec_out != nullptr && valid && deg <= kRecDeg;
+    if (__any_sync(0xffffffffu, direct)) {  // record lanes: their targets are one activation batch
+      const uint32_t x[kBatch] = {rd.x, rd.y, rd.z, rd.w};
+      bool a[kBatch];
+#pragma unroll
+      for (uint32_t q = 0; q < kRecDeg; q++) a[q] = direct && q < deg;
+      my_act += activate_batch<false>(P, a, x, epoch, P.hub_in, qA, ns);
+    }
+    my_act += expand_warp<false>(P, valid && !direct, beg, deg, epoch, P.hub_in, qA, ns);
   }
   // changed hubs: out-edge chunks, dynamic over CTAs
   for (; nKC;) {
@@ -1646,25 +1709,9 @@ __device__ __forceinline__ void dense_split_phase(const Part<OffT> &P, const Vie
   if (threadIdx.x == 0 && my_a) atomicAdd(&ctl->cnt_act[slot], (uint32_t)my_a);
 }
 
-// Software grid barrier for the persistent loop (cooperative launch guarantees
-// that every CTA is resident). Sense by generation counter.
-__device__ __forceinline__ void grid_sync(Ctl *c) {
-  __syncthreads();
-  if (threadIdx.x == 0) {
-    volatile uint32_t *gen = &c->bar_gen;
-    const uint32_t g = *gen;
-    __threadfence();
-    if (atomicAdd(&c->bar_count, 1u) == gridDim.x - 1) {
-      c->bar_count = 0;
-      __threadfence();
-      atomicAdd(&c->bar_gen, 1u);
-    } else {
-      while (*gen == g) __nanosleep(32);
-    }
-    __threadfence();
-  }
-  __syncthreads();
-}
+// Grid barrier of the persistent loop: the monotone arrival counter in the
+// control block (zeroed with the rest of it before every run).
+__device__ __forceinline__ void grid_sync(Ctl *c, uint32_t &bar) { grid_barrier(&c->bar_count, bar); }
 
 // Persistent device-side BSP loop (one cooperative launch per run): phases are
 // separated by grid barriers instead of kernel boundaries, and CTA 0 closes
@@ -1674,27 +1721,28 @@ template <class Prog, class OffT, bool kDS>
 __device__ __forceinline__ void persistent_body(const Part<OffT> &P) {
   Ctl *ctl = P.ctl;
   __shared__ View V;
+  uint32_t bar = 0;  // grid barrier target (thread 0)
   for (;;) {
     load_view(ctl, V);
     if (V.stop) break;
     int pull;
     if constexpr (HasScatter<Prog>::value) {  // gather | commit | scatter + activate (push only)
       gather_phase<Prog, false>(P, V);
-      grid_sync(ctl);
+      grid_sync(ctl, bar);
       load_view(ctl, V);
       commit_only_phase(P, V);
-      grid_sync(ctl);
+      grid_sync(ctl, bar);
       scatter_activate_phase<Prog>(P, V);
-      grid_sync(ctl);
+      grid_sync(ctl, bar);
       if (blockIdx.x == 0) close_superstep(P, 0ull, 0, kPush);
-      grid_sync(ctl);
+      grid_sync(ctl, bar);
       continue;
     }
     if constexpr (PushFused<Prog>::value) {
       if (V.push) {  // one phase; the last CTA to finish closes the superstep
         push_phase<Prog>(P, V);
         finish_superstep(P, 0ull, 0, kPush);
-        grid_sync(ctl);
+        grid_sync(ctl, bar);
         continue;
       }
     }
@@ -1703,7 +1751,7 @@ __device__ __forceinline__ void persistent_body(const Part<OffT> &P) {
         if constexpr (kDS && DstFree<Prog>::value) {  // edge-segmented tiles, then the split rows
           if (kGateSelective && Selective<Prog>::value && V.gate) dense_seg_phase<Prog, true>(P, V);
           else dense_seg_phase<Prog, false>(P, V);
-          grid_sync(ctl);
+          grid_sync(ctl, bar);
           dense_split_phase<Prog>(P, V);
         } else {
           dense_gather_phase<Prog>(P, V);
@@ -1711,7 +1759,7 @@ __device__ __forceinline__ void persistent_body(const Part<OffT> &P) {
       } else {
         gather_phase<Prog, false>(P, V);
       }
-      grid_sync(ctl);
+      grid_sync(ctl, bar);
       load_view(ctl, V);
       clear_dirty(P, V, cbits_words(P));
       pull = pull_mode(V, P.own_n, frontier_gather(V)) ? kPullDense : kPush;
@@ -1722,20 +1770,24 @@ __device__ __forceinline__ void persistent_body(const Part<OffT> &P) {
       pull = pull_mode(V, P.own_n, frontier_bfs(V)) ? kPullScan : kPush;
       if (pull) {
         bfs_apply_phase(P, V);
-        grid_sync(ctl);
+        grid_sync(ctl, bar);
         pull_phase<true>(P, V);
       } else {
         bfs_phase(P, V);
       }
     }
-    grid_sync(ctl);
+    grid_sync(ctl, bar);
     if (blockIdx.x == 0) close_superstep(P, 0ull, 0, pull);
-    grid_sync(ctl);
+    grid_sync(ctl, bar);
   }
 }
 
+// 32-bit gathers are compiled for 4 resident CTAs per SM (64 registers): the
+// dense CC superstep is occupancy-bound (cfg4: 12.4 ms at 64 registers, 14.6 ms
+// when ptxas picked 80 for the same code)
+template <class Prog> struct PersistMinCtas { static constexpr int value = sizeof(typename Prog::GatherT) == 4 ? 4 : 3; };
 template <class Prog, class OffT>
-__global__ void __launch_bounds__(kBlock) k_persistent(const __grid_constant__ Part<OffT> P) {
+__global__ void __launch_bounds__(kBlock, PersistMinCtas<Prog>::value) k_persistent(const __grid_constant__ Part<OffT> P) {
   persistent_body<Prog, OffT, false>(P);
 }
 

@@ -722,23 +722,9 @@ struct PrLoop {
   unsigned long long *ts;              // GR_PR_PHASES=1: %globaltimer at the loop start and after each barrier
 };
 
-__device__ __forceinline__ void pr_grid_sync(uint32_t *bar) {
-  __syncthreads();
-  if (threadIdx.x == 0) {
-    volatile uint32_t *gen = bar + 1;
-    const uint32_t g = *gen;
-    __threadfence();
-    if (atomicAdd(bar, 1u) == gridDim.x - 1) {
-      bar[0] = 0;
-      __threadfence();
-      atomicAdd(bar + 1, 1u);
-    } else {
-      while (*gen == g) __nanosleep(20);
-    }
-    __threadfence();
-  }
-  __syncthreads();
-}
+// grid barrier of the persistent PageRank loops: bar[0] is the monotone arrival
+// counter (zeroed before every launch), `tgt` thread 0's running target
+__device__ __forceinline__ void pr_grid_sync(uint32_t *bar, uint32_t &tgt) { grid_barrier(bar, tgt); }
 
 template <class OffT>
 __device__ __forceinline__ void pr_apply_fixup(const PrArgs<OffT> &a, const PrLoop &L, float *hot_next, uint32_t lrow,
@@ -766,6 +752,7 @@ __global__ void __launch_bounds__(1024, 1) k_pr_seg_loop(const __grid_constant__
   const uint4 *src4 = reinterpret_cast<const uint4 *>(L.seg_src) + 2 * lane;
   const uint64_t gtid = blockIdx.x * (uint64_t)blockDim.x + threadIdx.x, gthreads = (uint64_t)gridDim.x * blockDim.x;
   // kPhases (GR_PR_PHASES=1, a separate instantiation): CTA 0 stamps %globaltimer
+  uint32_t bar_tgt = 0;  // grid barrier target (thread 0)
   if (kPhases && blockIdx.x == 0 && threadIdx.x == 0) L.ts[0] = gtimer();
   for (uint32_t t = 0; t < L.iters; t++) {
     PrArgs<OffT> a = a0;
@@ -808,7 +795,7 @@ __global__ void __launch_bounds__(1024, 1) k_pr_seg_loop(const __grid_constant__
         r0 = nr0;
       }
     }
-    pr_grid_sync(L.bar);
+    pr_grid_sync(L.bar, bar_tgt);
     if (kPhases && blockIdx.x == 0 && threadIdx.x == 0) L.ts[1 + 2 * t] = gtimer();
     // ---- phase 2: rows split between tiles, hot-table pack
     for (uint64_t c = gtid; c < L.num_tiles; c += gthreads) {
@@ -830,7 +817,7 @@ __global__ void __launch_bounds__(1024, 1) k_pr_seg_loop(const __grid_constant__
     if (!a.last)
       for (uint64_t k = gtid; k < L.hot_k; k += gthreads)
         if (!L.hot_split[k]) hot_next[k] = a.contrib_out[L.hot_ids[k]];
-    pr_grid_sync(L.bar);
+    pr_grid_sync(L.bar, bar_tgt);
     if (kPhases && blockIdx.x == 0 && threadIdx.x == 0) L.ts[2 + 2 * t] = gtimer();
   }
 }
@@ -964,6 +951,7 @@ __global__ void __launch_bounds__(1024, 1) k_pr_bseg_loop(const __grid_constant_
     asm("createpolicy.fractional.L2::evict_last.b64 %0, 1.0;" : "=l"(pol_keep));
     asm("createpolicy.fractional.L2::evict_first.b64 %0, 1.0;" : "=l"(pol_stream));
   }
+  uint32_t bar_tgt = 0;  // grid barrier target (thread 0)
   for (uint32_t t = 0; t < L.iters; t++) {
     const float *contrib_in = L.contrib[t & 1];
     float *contrib_out = L.contrib[(t + 1) & 1];
@@ -1009,7 +997,7 @@ __global__ void __launch_bounds__(1024, 1) k_pr_bseg_loop(const __grid_constant_
           j0 = nj0;
         }
       }
-      pr_grid_sync(L.bar);
+      pr_grid_sync(L.bar, bar_tgt);
       // ---- runs split between tiles of this block (fixed order)
       for (uint64_t c = t_lo + gtid; c < t_hi; c += gthreads) {
         const uint32_t jr = a0.head_row[c];
@@ -1028,7 +1016,7 @@ __global__ void __launch_bounds__(1024, 1) k_pr_bseg_loop(const __grid_constant_
         for (int o = 16; o > 0; o >>= 1) acc += __shfl_xor_sync(0xffffffffu, acc, o);
         if (lane == 0 && jr != kNoRow) atomicAdd(L.acc + __ldg(L.run_row + jr), a0.head_val[c] + acc);
       }
-      pr_grid_sync(L.bar);
+      pr_grid_sync(L.bar, bar_tgt);
     }
     // ---- apply: R = (1-d)/n + d * acc, 4 vertices per 128-bit access, 2 accesses in flight per thread
     {
@@ -1066,10 +1054,10 @@ __global__ void __launch_bounds__(1024, 1) k_pr_bseg_loop(const __grid_constant_
         else contrib_out[v] = R * __ldg(a0.inv_outdeg + v);
       }
     }
-    pr_grid_sync(L.bar);
+    pr_grid_sync(L.bar, bar_tgt);
     if (!last) {
       for (uint64_t k = gtid; k < L.hot_k; k += gthreads) hot_next[k] = contrib_out[L.hot_ids[k]];
-      pr_grid_sync(L.bar);
+      pr_grid_sync(L.bar, bar_tgt);
     }
   }
 }
@@ -1220,7 +1208,9 @@ __global__ void k_pr_tiles(const OffT *in_off, uint64_t e_base, uint32_t rows, u
 }
 
 // contrib_0[u] = R_0(u) / outdeg(u) with R_0 = 1/n (reading R3); dangling -> 0 (R2).
-static __global__ void k_pr_init(uint32_t n, const float *inv_outdeg, float *contrib) {
+// (+ zeroes the grid-barrier counter of the persistent loop that follows, if any)
+static __global__ void k_pr_init(uint32_t n, const float *inv_outdeg, float *contrib, uint32_t *bar = nullptr) {
+  if (bar && blockIdx.x == 0 && threadIdx.x == 0) bar[0] = 0;
   const float r0 = 1.0f / (float)n;
   for (uint64_t v = blockIdx.x * (uint64_t)blockDim.x + threadIdx.x; v < n; v += (uint64_t)gridDim.x * blockDim.x)
     contrib[v] = r0 * inv_outdeg[v];

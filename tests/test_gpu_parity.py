@@ -579,6 +579,58 @@ def test_dense_tile_gather_forced(algo, force, monkeypatch):
     compare(n, s2, d2, w2, algo, loops=("auto",), directions=("pull",))
 
 
+def _oracle_run(n, src, dst, w, algo, source, max_iters=0):
+    if algo == "widest":
+        return oracle.run(n, src, dst, "widest", w=w, source=source)
+    if algo == "heat":
+        return oracle.run(n, src, dst, "heat", w=w, source=source, max_iters=max_iters)
+    og = oracle.OracleGraph(n, src, dst, w)
+    try:
+        return og.run(algo, source=source, max_iters=max_iters)
+    finally:
+        og.close()
+
+
+@pytest.mark.parametrize("force", ["1", "0"])
+@pytest.mark.parametrize("algo", ["sssp", "cc", "widest", "heat"])
+def test_vertex_records_forced(algo, force, monkeypatch):
+    """Vertex records (GR_REC=1: one 32-byte record per vertex with its first
+    kRecDeg = 4 neighbours, weights, degree and offset; the default for graphs
+    whose vertices nearly all have degree <= 4, e.g. the cfg3 road grid) against
+    the CSR/CSC path (GR_REC=0): identical values and traces in every loop and
+    direction. The R-MAT graph mixes record lanes (degree <= 4) with packed,
+    warp-cooperative and hub lanes in one warp; the road grid is all records;
+    heat diffusion reads its edge states through the record's offset."""
+    monkeypatch.setenv("GR_REC", force)
+    cases = []
+    road = grgen.grid_road(70, 61, seed=44)
+    cases.append((road.n, road.src, road.dst, road.w))
+    if algo != "heat":
+        g = grgen.rmat(12, 8, seed=45)
+        src, dst = g.src, g.dst
+        if algo == "cc":
+            src, dst = np.concatenate([g.src, g.dst]), np.concatenate([g.dst, g.src])
+        cases.append((g.n, src, dst, grgen.weights(len(src), 1, 64, seed=46)))
+        cases.append(hub_graph())
+    else:
+        h = grgen.heat_grid(40, 33, seed=47)
+        cases = [(h.n, h.src, h.dst, h.w)]
+    for n, src, dst, w in cases:
+        mi = 60 if algo == "heat" else 0
+        ref, rtr, rit = _oracle_run(n, src, dst, w, algo, 3, mi)
+        with gr.GraphReduce(n, src, dst, w) as G:
+            for loop in ("auto", "device", "host"):
+                for d in (("push", "pull", "auto") if algo in ("sssp", "cc") else ("auto",)):
+                    if algo in ("widest", "heat"):
+                        cid = 0 if algo == "widest" else 2
+                        st = G.run("custom", custom_id=cid, source=3, loop=loop, direction=d, max_iters=mi)
+                    else:
+                        st = G.run(algo, source=3, loop=loop, direction=d)
+                    assert st["iterations"] == rit, (loop, d)
+                    np.testing.assert_array_equal(G.values(), ref, err_msg=f"{loop} {d}")
+                    np.testing.assert_array_equal(G.trace(), rtr, err_msg=f"{loop} {d}")
+
+
 @pytest.mark.parametrize("algo", ["bfs", "sssp", "cc", "pagerank", "pagerank_delta"])
 def test_trace_detail_equals_oracle(algo):
     """the detail columns of the trace — shards holding an

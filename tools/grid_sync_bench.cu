@@ -55,9 +55,70 @@ __device__ __forceinline__ void grid_sync2(Bar *b, unsigned *grp_cnt) {
   __syncthreads();
 }
 
+__device__ __forceinline__ unsigned ld_acq(const unsigned *p) {
+  unsigned v;
+  asm volatile("ld.acquire.gpu.global.u32 %0, [%1];" : "=r"(v) : "l"(p) : "memory");
+  return v;
+}
+__device__ __forceinline__ unsigned atom_add_acqrel(unsigned *p, unsigned x) {
+  unsigned v;
+  asm volatile("atom.add.acq_rel.gpu.global.u32 %0, [%1], %2;" : "=r"(v) : "l"(p), "r"(x) : "memory");
+  return v;
+}
+__device__ __forceinline__ void st_rel(unsigned *p, unsigned x) {
+  asm volatile("st.release.gpu.global.u32 [%0], %1;" ::"l"(p), "r"(x) : "memory");
+}
+__device__ __forceinline__ void st_relaxed(unsigned *p, unsigned x) {
+  asm volatile("st.relaxed.gpu.global.u32 [%0], %1;" ::"l"(p), "r"(x) : "memory");
+}
+// release/acquire: the arrival atom is acq_rel (publishes this CTA's writes,
+// sees the others' on the last arrival), the release is a st.release of the new
+// generation, waiters spin with ld.acquire; no fence.sc
+__device__ __forceinline__ void grid_sync3(Bar *b) {
+  __syncthreads();
+  if (threadIdx.x == 0) {
+    const unsigned g = ld_acq(&b->gen);
+    if (atom_add_acqrel(&b->count, 1u) == gridDim.x - 1) {
+      st_relaxed(&b->count, 0);
+      st_rel(&b->gen, g + 1);
+    } else {
+      while (ld_acq(&b->gen) == g) {}
+    }
+  }
+  __syncthreads();
+}
+// same, with __nanosleep(32) in the spin
+__device__ __forceinline__ void grid_sync4(Bar *b) {
+  __syncthreads();
+  if (threadIdx.x == 0) {
+    const unsigned g = ld_acq(&b->gen);
+    if (atom_add_acqrel(&b->count, 1u) == gridDim.x - 1) {
+      st_relaxed(&b->count, 0);
+      st_rel(&b->gen, g + 1);
+    } else {
+      while (ld_acq(&b->gen) == g) __nanosleep(32);
+    }
+  }
+  __syncthreads();
+}
+// counter that never resets: arrival k of barrier i returns i*grid + k; waiters
+// spin until the counter reaches (i+1)*grid (no separate generation word)
+__device__ __forceinline__ void grid_sync5(Bar *b, unsigned i) {
+  __syncthreads();
+  if (threadIdx.x == 0) {
+    const unsigned target = (i + 1) * gridDim.x;
+    if (atom_add_acqrel(&b->count, 1u) != target - 1)
+      while (ld_acq(&b->count) < target) {}
+  }
+  __syncthreads();
+}
+
 __global__ void k_sync(Bar *b, unsigned *grp, int iters, int hier) {
   for (int i = 0; i < iters; i++) {
-    if (hier) grid_sync2(b, grp);
+    if (hier == 1) grid_sync2(b, grp);
+    else if (hier == 2) grid_sync3(b);
+    else if (hier == 3) grid_sync4(b);
+    else if (hier == 4) grid_sync5(b, (unsigned)i);
     else grid_sync(b);
   }
 }
@@ -101,19 +162,21 @@ int main() {
   unsigned *grp;
   cudaMalloc(&b, sizeof(Bar));
   cudaMalloc(&grp, 4096);
-  for (int hier = 0; hier < 2; hier++)
+  const char *names[] = {"", "(hier16)", "(acq_rel)", "(acq_rel+sleep)", "(monotone count)"};
+  for (int hier = 0; hier < 5; hier++)
     for (int grid : {148, 296, 592, 1184}) {
       cudaMemset(b, 0, sizeof(Bar));
       cudaMemset(grp, 0, 4096);
       int iters = 2000;
       void *args[] = {&b, &grp, &iters, &hier};
       cudaLaunchCooperativeKernel((void *)k_sync, grid, 256, args, 0, s);
+      cudaMemsetAsync(b, 0, sizeof(Bar), s);
       cudaEventRecord(a, s);
       cudaLaunchCooperativeKernel((void *)k_sync, grid, 256, args, 0, s);
       cudaEventRecord(z, s);
       cudaError_t e = cudaEventSynchronize(z);
       cudaEventElapsedTime(&ms, a, z);
-      printf("grid_sync%s grid=%d: %.2f us/barrier (%s)\n", hier ? "(hier16)" : "", grid, ms * 1000 / iters,
+      printf("grid_sync%s grid=%d: %.2f us/barrier (%s)\n", names[hier], grid, ms * 1000 / iters,
              cudaGetErrorString(e));
     }
   return 0;
