@@ -201,6 +201,7 @@ template <class OffT> struct Part {
   // rec_out[2 u]: {dst[4]}, rec_out[2 u + 1]: {0, deg, beg lo, beg hi} (activation CSR). nullptr: off
   const uint4 *rec_in;
   const uint4 *rec_out;
+  uint32_t stamp_direct;  // FrontierActivate issues the first-stamper atomic without the filter read
   // partitioned frontier programs, exchange fused into the gather: every rank's
   // changed-set buffers of this superstep's parity (own included), written at
   // xp_off (= own_lo) + list position as the gather appends (WarpQueue mirrors)

@@ -387,15 +387,21 @@ template <class OffT> static gr_status rec_setup(gr_graph *g) {
   CK(cudaFreeAsync(cnt, s));
   CK(cudaStreamSynchronize(s));
   if (!(e || (h[0] >= 0.9 * rows && h[1] >= 0.9 * n))) return GR_OK;
+  // activation records: measured no gain on cfg3 (the 32-byte out-records double the
+  // L2 footprint of the wavefront: gather 214 -> 250 ms, activation 320 -> 297 ms);
+  // GR_REC_OUT=1 builds and uses them
+  const char *eo = getenv("GR_REC_OUT");
+  const bool out = eo && atoi(eo) != 0;
   uint4 *ri = nullptr, *ro = nullptr;
-  if (dev_alloc(g, (void **)&ri, 32ull * rows) != GR_OK || dev_alloc(g, (void **)&ro, 32ull * n) != GR_OK)
+  if (dev_alloc(g, (void **)&ri, 32ull * rows) != GR_OK || (out && dev_alloc(g, (void **)&ro, 32ull * n) != GR_OK))
     return GR_OK;  // records are an accelerator: run without them
   k_rec_fill<OffT><<<g->num_sms * 8, 256, 0, s>>>((const OffT *)g->in_off, g->in_src, g->in_w, rows, ri);
-  k_rec_fill<OffT><<<g->num_sms * 8, 256, 0, s>>>((const OffT *)g->out_off, g->out_dst, nullptr, n, ro);
+  if (out) k_rec_fill<OffT><<<g->num_sms * 8, 256, 0, s>>>((const OffT *)g->out_off, g->out_dst, nullptr, n, ro);
   CK(cudaGetLastError());
   g->rec_in = ri;
-  const char *eo = getenv("GR_REC_OUT");  // A/B: records for the gather only
-  g->rec_out = (eo && atoi(eo) == 0) ? nullptr : ro;
+  g->rec_out = ro;
+  const char *sd = getenv("GR_STAMP_DIRECT");
+  g->stamp_direct = sd ? atoi(sd) != 0 : true;
   return GR_OK;
 }
 
@@ -1066,7 +1072,9 @@ template <class OffT>
 using SegLoopKernel = void (*)(const PrArgs<OffT>, const PrLoop);
 // The seg kernels are instantiated for the default variant bits only (the other
 // combinations were measured in round 1 and are not built: profiles/README.md)
-template <class OffT> static SegLoopKernel<OffT> seg_loop_kernel(int, bool phases = false) {
+template <class OffT> static SegLoopKernel<OffT> seg_loop_kernel(int, bool phases = false, bool tma = false) {
+  if (tma)
+    return phases ? k_pr_seg_loop<OffT, kSegDefaultVar, true, true> : k_pr_seg_loop<OffT, kSegDefaultVar, false, true>;
   return phases ? k_pr_seg_loop<OffT, kSegDefaultVar, true> : k_pr_seg_loop<OffT, kSegDefaultVar, false>;
 }
 template <class OffT> static SegKernel<OffT> seg_kernel(int) { return k_pr_seg<OffT, kSegDefaultVar>; }
@@ -1251,11 +1259,27 @@ template <class OffT> static gr_status pr_hot_setup(gr_graph *g) {
     if (const char *pl = getenv("GR_PR_LOOP")) g->pr_loop = g->coop && atoi(pl) != 0;
     if (g->comm) g->pr_loop = 0;  // partitioned: one launch per phase, the exchange between supersteps
     if (g->pr_loop) {
+      // the item and head-bit streams by TMA bulk copies into two staging buffers per
+      // warp (GR_PR_TMA=0: 128-bit loads through L1)
+      // measured slower (tiles phase 314 vs 173 us per superstep on cfg2, profiles/README.md):
+      // opt-in with GR_PR_TMA=1
+      g->pr_tma = false;
+      if (const char *e = getenv("GR_PR_TMA")) g->pr_tma = atoi(e) != 0;
+      g->tma_off = (uint32_t)((g->hot_smem + 127) / 128 * 128);
+      g->loop_smem = g->pr_tma ? g->tma_off + (g->hot_cta / 32) * (2 * kTmaBufBytes + 16) : g->hot_smem;
       int lbps = 0;
-      CK(cudaFuncSetAttribute(seg_loop_kernel<OffT>(g->seg_var), cudaFuncAttributeMaxDynamicSharedMemorySize,
-                              (int)g->hot_smem));
-      CK(cudaOccupancyMaxActiveBlocksPerMultiprocessor(&lbps, seg_loop_kernel<OffT>(g->seg_var), g->hot_cta,
-                                                       g->hot_smem));
+      CK(cudaFuncSetAttribute(seg_loop_kernel<OffT>(g->seg_var, false, g->pr_tma),
+                              cudaFuncAttributeMaxDynamicSharedMemorySize, (int)g->loop_smem));
+      CK(cudaOccupancyMaxActiveBlocksPerMultiprocessor(&lbps, seg_loop_kernel<OffT>(g->seg_var, false, g->pr_tma),
+                                                       g->hot_cta, g->loop_smem));
+      if (lbps < 1 && g->pr_tma) {  // does not fit next to the table: the load path
+        g->pr_tma = false;
+        g->loop_smem = g->hot_smem;
+        CK(cudaFuncSetAttribute(seg_loop_kernel<OffT>(g->seg_var), cudaFuncAttributeMaxDynamicSharedMemorySize,
+                                (int)g->loop_smem));
+        CK(cudaOccupancyMaxActiveBlocksPerMultiprocessor(&lbps, seg_loop_kernel<OffT>(g->seg_var), g->hot_cta,
+                                                         g->loop_smem));
+      }
       if (lbps < 1) g->pr_loop = 0;
     }
     if (g->pr_loop) {
@@ -1421,6 +1445,7 @@ static gr_status run_pagerank(gr_graph *g, const gr_run_opts *o, cudaStream_t s,
     L.num_tiles = g->seg_tiles;
     L.iters = iters;
     L.bar = g->pr_bar;
+    L.tma_off = g->tma_off;
     // GR_PR_PHASES=1: per-superstep split of the loop (tiles vs fix-ups + pack + barriers),
     // stamped with %globaltimer by CTA 0 after each grid barrier, printed on stderr
     static const bool phases = getenv("GR_PR_PHASES") && atoi(getenv("GR_PR_PHASES")) != 0;
@@ -1432,10 +1457,10 @@ static gr_status run_pagerank(gr_graph *g, const gr_run_opts *o, cudaStream_t s,
     if (prof) CK(cudaEventRecord(g->prof_ev[0], s));
     void *args[] = {(void *)&a, (void *)&L};
     if (phases)
-      CK(cudaFuncSetAttribute(seg_loop_kernel<OffT>(g->seg_var, true), cudaFuncAttributeMaxDynamicSharedMemorySize,
-                              (int)g->hot_smem));
-    CK(cudaLaunchCooperativeKernel((const void *)seg_loop_kernel<OffT>(g->seg_var, phases), dim3(g->hot_grid),
-                                   dim3(g->hot_cta), args, g->hot_smem, s));
+      CK(cudaFuncSetAttribute(seg_loop_kernel<OffT>(g->seg_var, true, g->pr_tma),
+                              cudaFuncAttributeMaxDynamicSharedMemorySize, (int)g->loop_smem));
+    CK(cudaLaunchCooperativeKernel((const void *)seg_loop_kernel<OffT>(g->seg_var, phases, g->pr_tma),
+                                   dim3(g->hot_grid), dim3(g->hot_cta), args, g->loop_smem, s));
     if (prof) CK(cudaEventRecord(g->prof_ev[1], s));
     CK(cudaStreamSynchronize(s));
     if (phases) {

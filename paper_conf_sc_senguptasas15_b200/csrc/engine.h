@@ -41,6 +41,7 @@ struct gr_graph {
   bool ds_tried = false;
   uint4 *rec_in = nullptr, *rec_out = nullptr;  // vertex records (low-degree graphs; first gather-program run)
   bool rec_tried = false;
+  bool stamp_direct = false;  // low-degree graph: activation atomics without the filter read (GR_STAMP_DIRECT)
   double ds_long_frac = -1.0;  // share of in-edges in rows longer than one tile (< 0: not computed)                  // tolerance PageRank divisor table (first GR_PAGERANK_DELTA run)
   uint32_t *hub_in = nullptr, *hub_out = nullptr, *static_hubs = nullptr;
   uint32_t n_static_hubs = 0;
@@ -95,6 +96,9 @@ struct gr_graph {
   float *hot_contrib = nullptr;
   uint32_t hot_k = 0, hot_grid = 0;
   size_t hot_smem = 0;
+  size_t loop_smem = 0;     // k_pr_seg_loop: hot_smem + (pr_tma) the per-warp TMA staging buffers
+  uint32_t tma_off = 0;     // byte offset of that staging in the loop's dynamic shared memory
+  bool pr_tma = false;      // item / head-bit streams by TMA bulk copies (GR_PR_TMA)
   // edge-segmented PageRank layout (pr_kernel 7, kernels_pr.cuh k_pr_seg)
   uint32_t *seg_src = nullptr, *seg_flags = nullptr, *seg_row = nullptr, *seg_off = nullptr;
   uint32_t seg_tiles = 0;
@@ -182,6 +186,7 @@ template <class OffT> inline Part<OffT> make_part(gr_graph *g) {
   P.ds_nsplit = g->ds_nsplit;
   P.rec_in = g->rec_in;
   P.rec_out = g->rec_out;
+  P.stamp_direct = g->stamp_direct ? 1u : 0u;
   P.nxt[0] = g->nxt[0];
   P.nxt[1] = g->nxt[1];
   P.out_w = g->out_w;

@@ -347,7 +347,10 @@ __device__ void append_hub_C(const Part<OffT> &P, uint32_t v, uint32_t nv) {
 // bit) is issued for the whole batch before any result is consumed, so a lane
 // keeps kBatch independent requests in flight instead of one dependent chain.
 // The first stamper of x appends it (BFS: only if still unvisited).
-template <bool kBfsFilter, class OffT, bool kByOut = kBfsFilter>
+// kPreRead = false (vertex-record lanes: a target of a degree-<=4 source has few
+// in-neighbours, so the filter rarely saves an atomic): the atomic is issued at
+// once, one dependent L2 round trip less.
+template <bool kBfsFilter, class OffT, bool kByOut = kBfsFilter, bool kPreRead = true>
 __device__ __forceinline__ uint32_t activate_batch(const Part<OffT> &P, const bool (&act)[kBatch],
                                                    const uint32_t (&x)[kBatch], uint32_t epoch,
                                                    const uint32_t *hub_bits, WarpQueue &qA, uint32_t slot) {
@@ -355,7 +358,7 @@ __device__ __forceinline__ uint32_t activate_batch(const Part<OffT> &P, const bo
   bool hb[kBatch];
 #pragma unroll
   for (int q = 0; q < kBatch; q++) {
-    st[q] = act[q] ? ld_cg(P.stamp + (x[q] - P.own_lo)) : epoch;
+    st[q] = (act[q] && kPreRead) ? ld_cg(P.stamp + (x[q] - P.own_lo)) : (act[q] ? ~epoch : epoch);
     hb[q] = act[q] && test_bit(hub_bits, kByOut ? x[q] : x[q] - P.own_lo);  // issued with the stamp read
   }
   bool nw[kBatch];
@@ -385,7 +388,7 @@ __device__ __forceinline__ uint32_t activate_batch(const Part<OffT> &P, const bo
 // kHubDegree): their edge ranges are concatenated and walked 32*kBatch edges at
 // a time; each element finds its source lane by a shuffle binary search over
 // the warp's exclusive degree prefix.
-template <bool kBfsFilter, class OffT>
+template <bool kBfsFilter, class OffT, bool kPreRead = true>
 __device__ uint32_t expand_warp(const Part<OffT> &P, bool valid, uint64_t beg, uint32_t deg, uint32_t epoch,
                                 const uint32_t *hub_bits, WarpQueue &qA, uint32_t slot) {
   const uint32_t lane = lane_id();
@@ -411,7 +414,7 @@ __device__ uint32_t expand_warp(const Part<OffT> &P, bool valid, uint64_t beg, u
       act[q] = k < total;
       x[q] = act[q] ? ldg_nc(P.out_dst + ob + (k - oe)) : 0u;
     }
-    nact += activate_batch<kBfsFilter>(P, act, x, epoch, hub_bits, qA, slot);
+    nact += activate_batch<kBfsFilter, OffT, kBfsFilter, kPreRead>(P, act, x, epoch, hub_bits, qA, slot);
   }
   return nact;  // warp-uniform
 }
@@ -944,9 +947,12 @@ __device__ __forceinline__ void activate_phase(const Part<OffT> &P, const View &
       bool a[kBatch];
 #pragma unroll
       for (uint32_t q = 0; q < kRecDeg; q++) a[q] = direct && q < deg;
-      my_act += activate_batch<false>(P, a, x, epoch, P.hub_in, qA, ns);
+      my_act += activate_batch<false, OffT, false, false>(P, a, x, epoch, P.hub_in, qA, ns);
     }
-    my_act += expand_warp<false>(P, valid && !direct, beg, deg, epoch, P.hub_in, qA, ns);
+    // low-degree graphs (Part::stamp_direct): few in-neighbours per target, so the
+    // first-stamper filter read rarely saves an atomic — issue the atomic at once
+    if (P.stamp_direct) my_act += expand_warp<false, OffT, false>(P, valid && !direct, beg, deg, epoch, P.hub_in, qA, ns);
+    else my_act += expand_warp<false>(P, valid && !direct, beg, deg, epoch, P.hub_in, qA, ns);
   }
   // changed hubs: out-edge chunks, dynamic over CTAs
   for (; nKC;) {
@@ -1785,7 +1791,12 @@ __device__ __forceinline__ void persistent_body(const Part<OffT> &P) {
 // 32-bit gathers are compiled for 4 resident CTAs per SM (64 registers): the
 // dense CC superstep is occupancy-bound (cfg4: 12.4 ms at 64 registers, 14.6 ms
 // when ptxas picked 80 for the same code)
-template <class Prog> struct PersistMinCtas { static constexpr int value = sizeof(typename Prog::GatherT) == 4 ? 4 : 3; };
+#ifndef GR_PERSIST_CTAS32  // A/B builds: resident CTAs per SM the 32-bit-gather loops are compiled for
+#define GR_PERSIST_CTAS32 4
+#endif
+template <class Prog> struct PersistMinCtas {
+  static constexpr int value = sizeof(typename Prog::GatherT) == 4 ? GR_PERSIST_CTAS32 : 3;
+};
 template <class Prog, class OffT>
 __global__ void __launch_bounds__(kBlock, PersistMinCtas<Prog>::value) k_persistent(const __grid_constant__ Part<OffT> P) {
   persistent_body<Prog, OffT, false>(P);

@@ -408,6 +408,50 @@ __device__ __forceinline__ float lds_f32(uint32_t saddr) {
   return v;
 }
 
+// TMA bulk copies (cp.async.bulk, non-tensor) into shared memory, completed on
+// an mbarrier: the copy engine fetches the item / head-bit streams, so they
+// take no slots of the SM's L1->L2 request port (the PageRank floor,
+// profiles/pr_floor_r02.md) and no registers while in flight.
+__device__ __forceinline__ void mbar_init(uint32_t mbar, uint32_t count) {
+  asm volatile("mbarrier.init.shared::cta.b64 [%0], %1;" ::"r"(mbar), "r"(count) : "memory");
+}
+__device__ __forceinline__ void mbar_expect_tx(uint32_t mbar, uint32_t bytes) {
+  asm volatile("mbarrier.arrive.expect_tx.shared::cta.b64 _, [%0], %1;" ::"r"(mbar), "r"(bytes) : "memory");
+}
+__device__ __forceinline__ void mbar_wait(uint32_t mbar, uint32_t parity) {
+  asm volatile(
+      "{\n\t.reg .pred P1;\n"
+      "LAB_WAIT:\n\t"
+      "mbarrier.try_wait.parity.shared::cta.b64 P1, [%0], %1;\n\t"
+      "@P1 bra DONE;\n\t"
+      "bra LAB_WAIT;\n"
+      "DONE:\n\t}" ::"r"(mbar), "r"(parity) : "memory");
+}
+__device__ __forceinline__ void tma_bulk_g2s(uint32_t dst, const void *src, uint32_t bytes, uint32_t mbar) {
+  asm volatile("cp.async.bulk.shared::cluster.global.mbarrier::complete_tx::bytes [%0], [%1], %2, [%3];"
+               ::"r"(dst), "l"(src), "r"(bytes), "r"(mbar) : "memory");
+}
+// the generic-proxy reads of a staging buffer are ordered before the next bulk
+// copy (async proxy) that overwrites it
+__device__ __forceinline__ void fence_proxy_async_smem() {
+  asm volatile("fence.proxy.async.shared::cta;" ::: "memory");
+}
+__device__ __forceinline__ uint4 lds_v4(uint32_t saddr) {
+  uint4 v;
+  asm volatile("ld.shared.v4.u32 {%0, %1, %2, %3}, [%4];" : "=r"(v.x), "=r"(v.y), "=r"(v.z), "=r"(v.w) : "r"(saddr));
+  return v;
+}
+__device__ __forceinline__ uint32_t lds_u32(uint32_t saddr) {
+  uint32_t v;
+  asm volatile("ld.shared.u32 %0, [%1];" : "=r"(v) : "r"(saddr));
+  return v;
+}
+// per-warp staging of one tile: 256 items (1 KB) + its 8 head-bit words and the
+// next tile's first word (copied as 48 bytes: bulk sizes are multiples of 16)
+constexpr uint32_t kTmaItemBytes = kSegTile * 4;
+constexpr uint32_t kTmaFlagBytes = 48;
+constexpr uint32_t kTmaBufBytes = kTmaItemBytes + 64;
+
 
 // contributions of my 8 items: hot sources from the shared table, the rest
 // from global memory (L2-resident)
@@ -711,6 +755,7 @@ __global__ void k_pr_fixup_long(const __grid_constant__ PrArgs<OffT> a, const ui
 // launches; what goes away is 3 launches per superstep.
 struct PrLoop {
   const uint32_t *seg_src, *seg_flags, *seg_row;
+  uint32_t tma_off;  // kTma: byte offset of the per-warp staging buffers in dynamic shared memory
   const uint32_t *hot_ids, *hot_slot;  // packed slot -> vertex, vertex -> slot (0xFFFFFFFF: not hot)
   const uint8_t *hot_split;            // slot's row is finished by the fix-up phase
   float *hot_buf[2];                   // packed hot contributions, by superstep parity
@@ -741,7 +786,7 @@ __device__ __forceinline__ void pr_apply_fixup(const PrArgs<OffT> &a, const PrLo
   }
 }
 
-template <class OffT, int kVar, bool kPhases = false>
+template <class OffT, int kVar, bool kPhases = false, bool kTma = false>
 __global__ void __launch_bounds__(1024, 1) k_pr_seg_loop(const __grid_constant__ PrArgs<OffT> a0,
                                                         const __grid_constant__ PrLoop L) {
   extern __shared__ __align__(16) float s_hot[];
@@ -751,6 +796,26 @@ __global__ void __launch_bounds__(1024, 1) k_pr_seg_loop(const __grid_constant__
   const uint32_t stride = gridDim.x * nw;
   const uint4 *src4 = reinterpret_cast<const uint4 *>(L.seg_src) + 2 * lane;
   const uint64_t gtid = blockIdx.x * (uint64_t)blockDim.x + threadIdx.x, gthreads = (uint64_t)gridDim.x * blockDim.x;
+  // kTma: two staging buffers per warp (tile i in buffer i & 1), each with its mbarrier;
+  // `tph` holds the parity of the next completion of each buffer
+  const uint32_t st0 = hot_sbase + L.tma_off + 2u * w * kTmaBufBytes;
+  const uint32_t mb0 = hot_sbase + L.tma_off + 2u * nw * kTmaBufBytes + 16u * w;
+  uint32_t tph = 0;
+  if (kTma) {
+    if (lane == 0) {
+      mbar_init(mb0, 1);
+      mbar_init(mb0 + 8, 1);
+      asm volatile("fence.mbarrier_init.release.cluster;" ::: "memory");
+    }
+    __syncwarp();
+  }
+  auto tma_issue = [&](uint32_t tl, uint32_t j) {  // lane 0: tile tl into buffer j
+    const uint32_t dst = st0 + j * kTmaBufBytes, mb = mb0 + 8u * j;
+    fence_proxy_async_smem();
+    mbar_expect_tx(mb, kTmaItemBytes + kTmaFlagBytes);
+    tma_bulk_g2s(dst, L.seg_src + (uint64_t)tl * kSegTile, kTmaItemBytes, mb);
+    tma_bulk_g2s(dst + kTmaItemBytes, L.seg_flags + (uint64_t)tl * 8, kTmaFlagBytes, mb);
+  };
   // kPhases (GR_PR_PHASES=1, a separate instantiation): CTA 0 stamps %globaltimer
   uint32_t bar_tgt = 0;  // grid barrier target (thread 0)
   if (kPhases && blockIdx.x == 0 && threadIdx.x == 0) L.ts[0] = gtimer();
@@ -767,7 +832,37 @@ __global__ void __launch_bounds__(1024, 1) k_pr_seg_loop(const __grid_constant__
     if (threadIdx.x < 4) s_hot[L.hot_k + threadIdx.x] = 0.f;
     __syncthreads();
     uint32_t tile = blockIdx.x * nw + w;
-    if (tile < L.num_tiles) {
+    if (kTma && tile < L.num_tiles) {
+      if (lane == 0) tma_issue(tile, 0);
+      uint32_t r0 = seg_ld1<kVar>(L.seg_row + tile);
+      for (uint32_t j = 0;; j ^= 1u) {
+        const uint32_t buf = st0 + j * kTmaBufBytes;
+        mbar_wait(mb0 + 8u * j, (tph >> j) & 1u);
+        tph ^= 1u << j;
+        const uint4 s0 = lds_v4(buf + 32u * lane), s1 = lds_v4(buf + 32u * lane + 16u);
+        const uint32_t fw = lds_u32(buf + kTmaItemBytes + 4u * (lane >> 2));
+        const uint32_t fnext = lds_u32(buf + kTmaItemBytes + 32u) & 1u;
+        float v[kSegIpt];
+        seg_gather<kVar>(s0, s1, s_hot, hot_sbase, a.contrib_in, v);
+        float pre_inv = 0.f;
+        if (kVar & kSegBuf) {
+          const uint32_t prow = r0 + lane;
+          pre_inv = (!a.last && prow < a.own_n) ? seg_ldf<kVar>(a.inv_outdeg + a.own_lo + prow) : 0.f;
+        }
+        const uint32_t b = (fw >> ((lane & 3) * 8)) & 0xFFu;
+        const uint32_t ntile = tile + stride;
+        uint32_t nr0 = 0;
+        if (ntile < L.num_tiles) {
+          __syncwarp();  // every lane has read the other buffer's previous tile
+          if (lane == 0) tma_issue(ntile, j ^ 1u);
+          nr0 = seg_ld1<kVar>(L.seg_row + ntile);
+        }
+        seg_tile<OffT, kVar>(a, tile, r0, b, fnext, pre_inv, v, s_R);
+        if (ntile >= L.num_tiles) break;
+        tile = ntile;
+        r0 = nr0;
+      }
+    } else if (!kTma && tile < L.num_tiles) {
       uint4 s0 = seg_ld4<kVar>(src4 + (uint64_t)tile * (kSegTile / 4));
       uint4 s1 = seg_ld4<kVar>(src4 + (uint64_t)tile * (kSegTile / 4) + 1);
       uint32_t r0 = seg_ld1<kVar>(L.seg_row + tile);

@@ -279,6 +279,28 @@ def test_pagerank_kernel_variants(variant, monkeypatch):
         check_pr(G.values("pagerank"), ref, n)
 
 
+def test_pagerank_tma_stream(monkeypatch):
+    """The persistent PageRank loop with its item / head-bit streams moved by TMA
+    bulk copies into per-warp staging (GR_PR_TMA=1, cp.async.bulk + mbarrier)
+    sums in exactly the order of the load path (GR_PR_TMA=0): bit-identical
+    ranks, both within the PageRank bar of the oracle. Graphs with hub rows
+    spanning many tiles and with more tiles than warps (several tiles per warp,
+    both staging buffers reused across supersteps)."""
+    for g in (grgen.rmat(17, 16, seed=12), grgen.rmat(16, 24, seed=13)):
+        ref, _, _ = oracle.run(g.n, g.src, g.dst, "pagerank", max_iters=30)
+        got = {}
+        for tma in ("1", "0"):
+            monkeypatch.setenv("GR_PR_TMA", tma)
+            with gr.GraphReduce(g.n, g.src, g.dst) as G:
+                st = G.run("pagerank")
+                assert st["kernel_ms"][3] == 7
+                got[tma] = G.values("pagerank").copy()
+                G.run("pagerank")  # a second run reuses the mbarriers' phases from zero
+                np.testing.assert_array_equal(G.values("pagerank").view(np.uint32), got[tma].view(np.uint32))
+            check_pr(got[tma], ref, g.n)
+        np.testing.assert_array_equal(got["1"].view(np.uint32), got["0"].view(np.uint32))
+
+
 @pytest.mark.parametrize("block_v,policy", [(10000, "1"), (10000, "0"), (40000, "1"), (1 << 16, "1")])
 def test_pagerank_source_blocked(block_v, policy, monkeypatch):
     """the source-blocked layout (sources cut into blocks whose
@@ -591,17 +613,18 @@ def _oracle_run(n, src, dst, w, algo, source, max_iters=0):
         og.close()
 
 
-@pytest.mark.parametrize("force", ["1", "0"])
+@pytest.mark.parametrize("force", ["1", "1out", "0"])
 @pytest.mark.parametrize("algo", ["sssp", "cc", "widest", "heat"])
 def test_vertex_records_forced(algo, force, monkeypatch):
     """Vertex records (GR_REC=1: one 32-byte record per vertex with its first
     kRecDeg = 4 neighbours, weights, degree and offset; the default for graphs
     whose vertices nearly all have degree <= 4, e.g. the cfg3 road grid) against
-    the CSR/CSC path (GR_REC=0): identical values and traces in every loop and
-    direction. The R-MAT graph mixes record lanes (degree <= 4) with packed,
+    the CSR/CSC path (GR_REC=0), with and without the activation records
+    (GR_REC_OUT): identical values and traces in every loop and direction. The R-MAT graph mixes record lanes (degree <= 4) with packed,
     warp-cooperative and hub lanes in one warp; the road grid is all records;
     heat diffusion reads its edge states through the record's offset."""
-    monkeypatch.setenv("GR_REC", force)
+    monkeypatch.setenv("GR_REC", force[0])
+    monkeypatch.setenv("GR_REC_OUT", "1" if force == "1out" else "0")  # activation records too
     cases = []
     road = grgen.grid_road(70, 61, seed=44)
     cases.append((road.n, road.src, road.dst, road.w))
