@@ -372,6 +372,17 @@ static __global__ void k_rec_fill(const OffT *off, const uint32_t *adj, const ui
     rec[2ull * r + 1] = make_uint4(w4, (uint32_t)d, (uint32_t)b, (uint32_t)(b >> 32));
   }
 }
+// the activation CSR equals the CSC (same offsets, same sorted adjacency): the
+// graph is symmetric and a vertex's in-record lists its out-neighbours too
+template <class OffT>
+static __global__ void k_same_adj(const OffT *a_off, const OffT *b_off, uint32_t rows, const uint32_t *a,
+                                  const uint32_t *b, uint64_t m, unsigned long long *diff) {
+  unsigned long long c = 0;
+  const uint64_t tid = blockIdx.x * (uint64_t)blockDim.x + threadIdx.x, nt = (uint64_t)gridDim.x * blockDim.x;
+  for (uint64_t r = tid; r <= rows; r += nt) c += (uint64_t)a_off[r] != (uint64_t)b_off[r];
+  for (uint64_t e = tid; e < m; e += nt) c += a[e] != b[e];
+  if (c) atomicAdd(diff, c);
+}
 template <class OffT> static gr_status rec_setup(gr_graph *g) {
   g->rec_tried = true;
   const uint32_t rows = (uint32_t)g->H.own_n(), n = (uint32_t)g->H.n;
@@ -400,6 +411,23 @@ template <class OffT> static gr_status rec_setup(gr_graph *g) {
   CK(cudaGetLastError());
   g->rec_in = ri;
   g->rec_out = ro;
+  // symmetric graphs (road networks, meshes, symmetrized inputs) may let the
+  // activation read the in-record of the changed vertex (no second record array);
+  // measured slower on cfg3 (537 -> 583 ms: the per-lane record batches leave
+  // lanes idle where the CSR expansion packs 32 edges per round), so opt-in:
+  // GR_REC_SYM=1
+  const char *esym = getenv("GR_REC_SYM");
+  if (!out && esym && atoi(esym) != 0 && rows == n && g->out_off) {
+    unsigned long long *d = nullptr, hd = 1;
+    CK(cudaMallocAsync(&d, sizeof hd, s));
+    CK(cudaMemsetAsync(d, 0, sizeof hd, s));
+    k_same_adj<OffT><<<g->num_sms * 8, 256, 0, s>>>((const OffT *)g->in_off, (const OffT *)g->out_off, rows,
+                                                    g->in_src, g->out_dst, g->H.m_in, d);
+    CK(cudaMemcpyAsync(&hd, d, sizeof hd, cudaMemcpyDeviceToHost, s));
+    CK(cudaFreeAsync(d, s));
+    CK(cudaStreamSynchronize(s));
+    if (hd == 0) g->rec_out = ri;
+  }
   const char *sd = getenv("GR_STAMP_DIRECT");
   g->stamp_direct = sd ? atoi(sd) != 0 : true;
   return GR_OK;

@@ -613,18 +613,21 @@ def _oracle_run(n, src, dst, w, algo, source, max_iters=0):
         og.close()
 
 
-@pytest.mark.parametrize("force", ["1", "1out", "0"])
+@pytest.mark.parametrize("force", ["1", "1out", "1nosym", "0"])
 @pytest.mark.parametrize("algo", ["sssp", "cc", "widest", "heat"])
 def test_vertex_records_forced(algo, force, monkeypatch):
     """Vertex records (GR_REC=1: one 32-byte record per vertex with its first
     kRecDeg = 4 neighbours, weights, degree and offset; the default for graphs
     whose vertices nearly all have degree <= 4, e.g. the cfg3 road grid) against
     the CSR/CSC path (GR_REC=0), with and without the activation records
-    (GR_REC_OUT): identical values and traces in every loop and direction. The R-MAT graph mixes record lanes (degree <= 4) with packed,
+    (GR_REC_OUT), and with the in-records serving the activation of symmetric
+    graphs (the road grid, the hub graph; GR_REC_SYM): identical values and
+    traces in every loop and direction. The R-MAT graph mixes record lanes (degree <= 4) with packed,
     warp-cooperative and hub lanes in one warp; the road grid is all records;
     heat diffusion reads its edge states through the record's offset."""
     monkeypatch.setenv("GR_REC", force[0])
     monkeypatch.setenv("GR_REC_OUT", "1" if force == "1out" else "0")  # activation records too
+    monkeypatch.setenv("GR_REC_SYM", "0" if force == "1nosym" else "1")  # symmetric graphs: in-records activate
     cases = []
     road = grgen.grid_road(70, 61, seed=44)
     cases.append((road.n, road.src, road.dst, road.w))
