@@ -99,7 +99,7 @@ __device__ typename Prog::GatherT gather_warp(const Part<OffT> &P, bool valid, u
       if constexpr (HasScatter<Prog>::value) ew[q] = a[q] ? ld_cg(P.estate + beg + q) : 0u;
       else ew[q] = Prog::kUsesWeights ? (w4 >> (8 * q)) & 0xFFu : 0u;
       if (!kGate) vv[q] = a[q] ? P.val[us[q]] : 0u;
-      bw[q] = (kDense && a[q]) ? ld_cg(bits + (us[q] >> 5)) : 0u;
+      bw[q] = (kDense && a[q]) ? ld_bits(bits, us[q]) : 0u;
     }
     G r = Prog::identity();
     bool hh = false;
@@ -138,7 +138,7 @@ __device__ typename Prog::GatherT gather_warp(const Part<OffT> &P, bool valid, u
 #pragma unroll
       for (int q = 0; q < 4; q++) {
         if (!kGate) v[q] = P.val[u[q]];
-        if (kDense) bw[q] = ld_cg(bits + (u[q] >> 5));
+        if (kDense) bw[q] = ld_bits(bits, u[q]);
       }
       bool h[4];
 #pragma unroll
@@ -155,7 +155,7 @@ __device__ typename Prog::GatherT gather_warp(const Part<OffT> &P, bool valid, u
     for (; k < d; k += 32) {
       const uint32_t u = ldg_nc(P.in_src + b + k);
       const uint32_t w = edge_w<Prog>(P, b + k);
-      const bool h = kDense && test_bit_cg(bits, u);
+      const bool h = kDense && test_bit_w(bits, u);
       if (!kGate || h) r = Prog::gatherReduce(r, Prog::gatherMap(dv, P.val[u], w, u, cx));
       hit |= h;
     }
@@ -203,7 +203,7 @@ __device__ typename Prog::GatherT gather_warp(const Part<OffT> &P, bool valid, u
 #pragma unroll
     for (int q = 0; q < kBatch; q++) {
       if (!kGate) sv[q] = act_q[q] ? P.val[su[q]] : 0u;
-      if (kDense) sb[q] = act_q[q] ? ld_cg(bits + (su[q] >> 5)) : 0u;
+      if (kDense) sb[q] = act_q[q] ? ld_bits(bits, su[q]) : 0u;
     }
     if (kGate) {  // only the changed sources' values: unmarked items map to identity()
 #pragma unroll
@@ -269,7 +269,7 @@ __device__ typename Prog::GatherT gather_block(const Part<OffT> &P, uint64_t beg
 #pragma unroll
     for (int q = 0; q < 4; q++) {
       if (!kGate) v[q] = P.val[u[q]];
-      if (kDense) bw[q] = ld_cg(bits + (u[q] >> 5));
+      if (kDense) bw[q] = ld_bits(bits, u[q]);
     }
     bool h[4];
 #pragma unroll
@@ -286,7 +286,7 @@ __device__ typename Prog::GatherT gather_block(const Part<OffT> &P, uint64_t beg
   for (; k < deg; k += kBlock) {
     const uint32_t u = ldg_nc(P.in_src + beg + k);
     const uint32_t w = edge_w<Prog>(P, beg + k);
-    const bool h = kDense && test_bit_cg(bits, u);
+    const bool h = kDense && test_bit_w(bits, u);
     if (!kGate || h) r = Prog::gatherReduce(r, Prog::gatherMap(dval, P.val[u], w, u, cx));
     hit |= h;
   }
@@ -669,14 +669,14 @@ __device__ __forceinline__ void pull_phase(const Part<OffT> &P, const View &V) {
     for (uint32_t q = 0; q < kProbe; q++) src[q] = (q < deg) ? ldg_nc(P.in_src + beg + q) : 0u;
     bool found = false;
 #pragma unroll
-    for (uint32_t q = 0; q < kProbe; q++) found |= (q < deg) && test_bit_cg(bits, src[q]);
+    for (uint32_t q = 0; q < kProbe; q++) found |= (q < deg) && test_bit_w(bits, src[q]);
     // moderate degrees: each lane continues its own scan, kProbe loads in flight
     for (uint64_t k = beg + kProbe; !found && deg <= kPullLane && k < end; k += kProbe) {
       uint32_t u[kProbe];
 #pragma unroll
       for (uint32_t q = 0; q < kProbe; q++) u[q] = (k + q < end) ? ldg_nc(P.in_src + k + q) : 0u;
 #pragma unroll
-      for (uint32_t q = 0; q < kProbe; q++) found |= (k + q < end) && test_bit_cg(bits, u[q]);
+      for (uint32_t q = 0; q < kProbe; q++) found |= (k + q < end) && test_bit_w(bits, u[q]);
     }
     // large degrees: the whole warp scans one vertex at a time
     uint32_t pend = __ballot_sync(0xffffffffu, !found && deg > kPullLane);
@@ -687,7 +687,7 @@ __device__ __forceinline__ void pull_phase(const Part<OffT> &P, const View &V) {
       const uint64_t b = __shfl_sync(0xffffffffu, beg, l) + kProbe, e = __shfl_sync(0xffffffffu, end, l);
       for (uint64_t k = b; k < e; k += 32) {
         const uint64_t kk = k + lane;
-        const bool hit = kk < e && test_bit_cg(bits, ldg_nc(P.in_src + kk));
+        const bool hit = kk < e && test_bit_w(bits, ldg_nc(P.in_src + kk));
         if (__ballot_sync(0xffffffffu, hit)) {
           fm |= 1u << l;
           break;
@@ -1566,7 +1566,7 @@ __device__ __forceinline__ void dense_seg_phase(const Part<OffT> &P, const View 
       // values and changed bits were written earlier in this (persistent) launch: coherent
       // loads, not the read-only .nc path (valid only for data read-only during the kernel)
       if (!kGate) sv[k] = ok ? P.val[src[k]] : 0u;
-      sa[k] = ok && test_bit_cg(bits, src[k]);
+      sa[k] = ok && test_bit_w(bits, src[k]);
     }
     if (kGate) {
 #pragma unroll
