@@ -15,8 +15,8 @@
 //   k_bfs_expand    : BFS phase fusion (L276): apply (depth = t) + activate in
 //                     one pass over A_t; gather eliminated (L274).
 // Load balancing (CTA load balancing from the active list, L270, L352): a warp
-// takes 32 list entries; lanes with degree > 32 are processed warp-
-// cooperatively one at a time, lanes with degree <= 32 are packed 32 edges per
+// takes 32 list entries; lanes with degree > kPackDeg are processed warp-
+// cooperatively one at a time, lanes with degree <= kPackDeg are packed 32 edges per
 // round (owner found by a shuffle binary search); vertices with degree >
 // kHubDegree live in a separate hub list processed one CTA per vertex.
 #pragma once
@@ -26,6 +26,15 @@
 namespace gr {
 
 constexpr int kBatch = 4;  // edges in flight per lane per memory phase
+#ifndef GR_PACK_DEG  // A/B builds
+#define GR_PACK_DEG 128
+#endif
+// gather lanes whose vertex has at most kPackDeg in-edges have their edges packed
+// 32 per round across the warp; larger ones (up to kHubDegree) are walked by the
+// whole warp one vertex at a time (128 edges per step). 128 rather than 32: the
+// web graph's rows of 33-128 in-edges (14 % of cfg4's edges, ~1.4 per 32-vertex
+// group) each cost a whole warp step with most lanes idle.
+constexpr uint32_t kPackDeg = GR_PACK_DEG;
 constexpr uint32_t kRecDeg = 4;  // neighbours held in a vertex record (Part::rec_in / rec_out)
 static_assert(kRecDeg == (uint32_t)kBatch, "a record's neighbours form one activation batch");
 #ifdef GR_NO_GATE  // A/B build: dense supersteps read every source's value
@@ -117,7 +126,7 @@ __device__ typename Prog::GatherT gather_warp(const Part<OffT> &P, bool valid, u
     act = hh;
   }
   // warp-cooperative: one vertex of degree in (32, kHubDegree] at a time
-  uint32_t big = __ballot_sync(0xffffffffu, valid && deg > 32);
+  uint32_t big = __ballot_sync(0xffffffffu, valid && deg > kPackDeg);
   while (big) {
     const int L = __ffs(big) - 1;
     big &= big - 1;
@@ -166,10 +175,10 @@ __device__ typename Prog::GatherT gather_warp(const Part<OffT> &P, bool valid, u
       act = any;
     }
   }
-  // fine-grained: pack the edges of all lanes with degree <= 32, 32 per round;
+  // fine-grained: pack the edges of all lanes with degree <= kPackDeg, 32 per round;
   // kBatch rounds' loads (sources + weights, then source values) are issued
   // together before their segmented reductions
-  const uint32_t sd = (valid && !direct && deg <= 32) ? deg : 0u;
+  const uint32_t sd = (valid && !direct && deg <= kPackDeg) ? deg : 0u;
   const uint32_t incl = warp_incl_scan(sd);
   const uint32_t excl = incl - sd;
   const uint32_t total = __shfl_sync(0xffffffffu, incl, 31);
