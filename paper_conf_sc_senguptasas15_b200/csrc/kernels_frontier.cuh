@@ -96,6 +96,15 @@ __device__ typename Prog::GatherT gather_warp(const Part<OffT> &P, bool valid, u
   // dense supersteps of selective programs may read val[u] only for changed sources
   // (Selective<>; chosen per superstep by close_superstep: Ctl::gate)
   constexpr bool kGate = kDense && kGateT && kGateSelective && Selective<Prog>::value;
+#ifndef GR_NO_PREFETCH
+  // the packed rounds below walk the rows of up to kPackDeg in-edges 32 edges at a
+  // time; prefetching each row's first and last line into L1 now turns the source
+  // loads of all but the first rounds into L1 hits (one dependent L2 trip less each)
+  if (valid && !direct && deg > 0 && deg <= kPackDeg) {
+    asm volatile("prefetch.global.L1 [%0];" ::"l"(P.in_src + beg));
+    if (deg > 8) asm volatile("prefetch.global.L1 [%0];" ::"l"(P.in_src + beg + deg - 1));
+  }
+#endif
   // vertex records: a lane whose vertex has degree <= kRecDeg holds its sources
   // (rs) and weights (w4) already and gathers alone, all loads in one phase
   if (direct) {
