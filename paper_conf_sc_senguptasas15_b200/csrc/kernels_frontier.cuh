@@ -35,6 +35,24 @@ constexpr int kBatch = 4;  // edges in flight per lane per memory phase
 // web graph's rows of 33-128 in-edges (14 % of cfg4's edges, ~1.4 per 32-vertex
 // group) each cost a whole warp step with most lanes idle.
 constexpr uint32_t kPackDeg = GR_PACK_DEG;
+// One shared-memory scratch for the staging arrays of every phase of a kernel: the
+// phases of the persistent loop are separated by grid barriers (which begin and end
+// with __syncthreads), so their per-warp queues and reduction slots are never live
+// together. Declared once at namespace scope, it costs the kernel the largest
+// phase's footprint (10.3 KB) instead of the sum over its inlined phases (up to 38 KB
+// for SSSP), leaving that much more of the SM's 256 KB to L1 — which the random
+// gathers hit (GR_NO_SMEM_UNION: per-phase arrays, for A/B).
+constexpr uint32_t kSqBytes1 = kWarpsPerBlock * kQueueCap * 4;      // one queue array per warp
+constexpr uint32_t kSqBytes2 = 2 * kSqBytes1;                         // two (pair lists)
+constexpr uint32_t kPhaseSmemBytes = kSqBytes2 + kWarpsPerBlock * 32 * 8 + kWarpsPerBlock * 8;
+__shared__ __align__(16) unsigned char g_phase_smem[kPhaseSmemBytes];
+#ifdef GR_NO_SMEM_UNION
+#define GR_SQ1(name) __shared__ uint32_t name[kWarpsPerBlock][kQueueCap]
+#define GR_SQ2(name) __shared__ uint32_t name[kWarpsPerBlock][2][kQueueCap]
+#else
+#define GR_SQ1(name) auto &name = *reinterpret_cast<uint32_t(*)[kWarpsPerBlock][kQueueCap]>(g_phase_smem)
+#define GR_SQ2(name) auto &name = *reinterpret_cast<uint32_t(*)[kWarpsPerBlock][2][kQueueCap]>(g_phase_smem)
+#endif
 constexpr uint32_t kRecDeg = 4;  // neighbours held in a vertex record (Part::rec_in / rec_out)
 static_assert(kRecDeg == (uint32_t)kBatch, "a record's neighbours form one activation batch");
 #ifdef GR_NO_GATE  // A/B build: dense supersteps read every source's value
@@ -665,7 +683,7 @@ __device__ __forceinline__ void pull_phase(const Part<OffT> &P, const View &V) {
   const uint32_t t = V.t, ns = (t + 1) & 1u;
   const uint32_t *bits = P.cbits[t & 1u];
   prof_begin(ctl, V, 1);
-  __shared__ uint32_t sq[kWarpsPerBlock][kQueueCap];
+  GR_SQ1(sq);
   __shared__ uint32_t s_off[kWarpsPerBlock + 1];
   __shared__ unsigned long long s8[kWarpsPerBlock];
   const uint32_t warp = threadIdx.x / 32, lane = lane_id();
@@ -759,9 +777,16 @@ __device__ __forceinline__ void gather_phase(const Part<OffT> &P, const View &V)
   const bool no_hub_c = V.no_hub_c != 0;
   prof_begin(ctl, V, 0);
 
-  __shared__ uint32_t sq[kWarpsPerBlock][2][kQueueCap];
+#ifdef GR_NO_SMEM_UNION
+  GR_SQ2(sq);
   __shared__ G sred[kWarpsPerBlock][32];
   __shared__ G sblk[kWarpsPerBlock];
+#else
+  static_assert(sizeof(G) <= 8, "gather results up to 8 bytes");
+  GR_SQ2(sq);
+  auto &sred = *reinterpret_cast<G(*)[kWarpsPerBlock][32]>(g_phase_smem + kSqBytes2);
+  auto &sblk = *reinterpret_cast<G(*)[kWarpsPerBlock]>(g_phase_smem + kSqBytes2 + kWarpsPerBlock * 32 * 8);
+#endif
   __shared__ uint32_t s_h;
   __shared__ bool s_act;
   __shared__ uint32_t s_off[kWarpsPerBlock + 1];
@@ -930,7 +955,7 @@ __device__ __forceinline__ void activate_phase(const Part<OffT> &P, const View &
   const uint32_t nKC = V.cntKC;
   prof_begin(ctl, V, 1);
 
-  __shared__ uint32_t sq[kWarpsPerBlock][kQueueCap];
+  GR_SQ1(sq);
   __shared__ uint32_t s_h;
   __shared__ uint32_t s_off[kWarpsPerBlock + 1];
   __shared__ unsigned long long s8[kWarpsPerBlock];
@@ -1032,7 +1057,7 @@ __device__ __forceinline__ void bfs_phase(const Part<OffT> &P, const View &V) {
   const uint32_t *LH = P.listH[slot];
   prof_begin(ctl, V, 1);
 
-  __shared__ uint32_t sq[kWarpsPerBlock][kQueueCap];
+  GR_SQ1(sq);
   __shared__ uint32_t s_h;
   __shared__ bool s_changed;
   __shared__ uint32_t s_off[kWarpsPerBlock + 1];
@@ -1212,7 +1237,7 @@ __device__ __forceinline__ void push_phase(const Part<OffT> &P, const View &V) {
   const Ctx cx = make_ctx(P, V);
   prof_begin(ctl, V, 1);
 
-  __shared__ uint32_t sq[kWarpsPerBlock][kQueueCap];
+  GR_SQ1(sq);
   __shared__ uint32_t s_h, s_nv;
   __shared__ bool s_changed;
   __shared__ uint32_t s_off[kWarpsPerBlock + 1];
@@ -1411,7 +1436,7 @@ __device__ __forceinline__ void scatter_activate_phase(const Part<OffT> &P, cons
   const Ctx cx = make_ctx(P, V);
   prof_begin(ctl, V, 1);
 
-  __shared__ uint32_t sq[kWarpsPerBlock][kQueueCap];
+  GR_SQ1(sq);
   __shared__ uint32_t s_h;
   __shared__ uint32_t s_off[kWarpsPerBlock + 1];
   __shared__ unsigned long long s8[kWarpsPerBlock];
@@ -1538,8 +1563,13 @@ struct DsSmem {
   uint32_t s_off[kWarpsPerBlock + 1];
 };
 __device__ __forceinline__ DsSmem &ds_smem() {
+#ifdef GR_NO_SMEM_UNION
   __shared__ DsSmem s;
   return s;
+#else
+  static_assert(sizeof(DsSmem) <= kPhaseSmemBytes, "dense-tile scratch fits the phase scratch");
+  return *reinterpret_cast<DsSmem *>(g_phase_smem);
+#endif
 }
 
 template <class Prog, bool kGateT, class OffT>
@@ -1701,7 +1731,7 @@ __device__ __forceinline__ void dense_split_phase(const Part<OffT> &P, const Vie
   const uint32_t slot = V.t & 1u;
   const Ctx cx = make_ctx(P, V);
   const bool no_hub_c = V.no_hub_c != 0;
-  __shared__ uint32_t sq[kWarpsPerBlock][2][kQueueCap];
+  GR_SQ2(sq);
   __shared__ uint32_t s_off[kWarpsPerBlock + 1];
   __shared__ unsigned long long s8[kWarpsPerBlock];
   const uint32_t warp = threadIdx.x / 32;
@@ -1856,7 +1886,7 @@ struct XDev {
 template <class OffT>
 __global__ void __launch_bounds__(kBlock) k_classify(const __grid_constant__ Part<OffT> P, const uint32_t *X_v,
                                                      const uint32_t *X_val, uint32_t nX, const XRanges R) {
-  __shared__ uint32_t sq[kWarpsPerBlock][2][kQueueCap];
+  GR_SQ2(sq);
   __shared__ uint32_t s_off[kWarpsPerBlock + 1];
   const uint32_t warp = threadIdx.x / 32, lane = lane_id();
   WarpQueue qC{sq[warp][0], sq[warp][1], 0};
