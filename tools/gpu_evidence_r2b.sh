@@ -1,7 +1,7 @@
 #!/bin/bash
 # round-2 (second session) evidence: every config line, reference arm, f-rows, ncu launch list +
 # --set full of the PageRank loop and of a dense CC gather superstep, PR phase split
-T=${1:-ev4}
+T=${1:-ev5}
 mkdir -p gpurun_out
 timeout 900 python -m pytest tests -m gpu -q > gpurun_out/${T}_tests.log 2>&1; echo "tests rc=$?" >> gpurun_out/${T}_tests.log
 timeout 120 python __graft_entry__.py > gpurun_out/${T}_smoke.log 2>&1; echo "smoke rc=$?" >> gpurun_out/${T}_smoke.log
