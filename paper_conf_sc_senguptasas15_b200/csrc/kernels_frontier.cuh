@@ -90,6 +90,14 @@ __device__ __forceinline__ uint32_t edge_w(const Part<OffT> &P, uint64_t e) {
   else return Prog::kUsesWeights ? (uint32_t)ldg_nc_u8(P.in_w + e) : 0u;
 }
 
+// CSC / CSR position of packed item k owned by lane o, from o's (row start - packed
+// offset): one shuffle (two for 64-bit offsets) instead of the start and the offset
+template <class OffT>
+__device__ __forceinline__ uint64_t packed_pos(uint64_t bx, int o, uint32_t k) {
+  if constexpr (sizeof(OffT) == 4) return (uint32_t)(__shfl_sync(0xffffffffu, (uint32_t)bx, o) + k);
+  else return __shfl_sync(0xffffffffu, bx, o) + k;
+}
+
 template <class Prog>
 __device__ __forceinline__ typename Prog::GatherT warp_reduce_prog(typename Prog::GatherT x) {
 #pragma unroll
@@ -211,6 +219,7 @@ __device__ typename Prog::GatherT gather_warp(const Part<OffT> &P, bool valid, u
   const uint32_t total = __shfl_sync(0xffffffffu, incl, 31);
   if (total == 0) return acc;
   sred[lane] = Prog::identity();
+  const uint64_t bx = beg - excl;  // CSC position of packed item k of this lane's row: bx + k
   uint32_t hitmask = 0;  // kDense: owner lanes with a marked source (warp-uniform)
   __syncwarp();
   for (uint32_t rb = 0; rb < total; rb += 32u * kBatch) {
@@ -227,11 +236,9 @@ __device__ typename Prog::GatherT gather_warp(const Part<OffT> &P, bool valid, u
         if (e <= k) o += step;
       }
       own[q] = o;
-      const uint64_t ob = __shfl_sync(0xffffffffu, beg, o);
-      const uint32_t oe = __shfl_sync(0xffffffffu, excl, o);
-      dv[q] = __shfl_sync(0xffffffffu, dval, o);
+      const uint64_t e = packed_pos<OffT>(bx, o, k);
+      dv[q] = DstFree<Prog>::value ? 0u : __shfl_sync(0xffffffffu, dval, o);  // gatherMap ignores it otherwise
       act_q[q] = k < total;
-      const uint64_t e = ob + (k - oe);
       su[q] = act_q[q] ? ldg_nc(P.in_src + e) : 0u;
       sw[q] = act_q[q] ? edge_w<Prog>(P, e) : 0u;
     }
@@ -432,6 +439,7 @@ __device__ uint32_t expand_warp(const Part<OffT> &P, bool valid, uint64_t beg, u
   const uint32_t incl = warp_incl_scan(d);
   const uint32_t excl = incl - d;
   const uint32_t total = __shfl_sync(0xffffffffu, incl, 31);
+  const uint64_t bx = beg - excl;  // CSR position of packed item k of this lane's row: bx + k
   uint32_t nact = 0;
   for (uint32_t r0 = 0; r0 < total; r0 += 32u * kBatch) {
     bool act[kBatch];
@@ -445,10 +453,9 @@ __device__ uint32_t expand_warp(const Part<OffT> &P, bool valid, uint64_t beg, u
         const uint32_t e = __shfl_sync(0xffffffffu, excl, o + step);
         if (e <= k) o += step;
       }
-      const uint64_t ob = __shfl_sync(0xffffffffu, beg, o);
-      const uint32_t oe = __shfl_sync(0xffffffffu, excl, o);
+      const uint64_t pos = packed_pos<OffT>(bx, o, k);  // a shuffle: every lane, outside the condition
       act[q] = k < total;
-      x[q] = act[q] ? ldg_nc(P.out_dst + ob + (k - oe)) : 0u;
+      x[q] = act[q] ? ldg_nc(P.out_dst + pos) : 0u;
     }
     nact += activate_batch<kBfsFilter, OffT, kBfsFilter, kPreRead>(P, act, x, epoch, hub_bits, qA, slot);
   }
